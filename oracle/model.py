@@ -1,0 +1,471 @@
+"""EATSS tile-selection model, brute force -- TEST INFRASTRUCTURE ONLY.
+
+Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline leg may import it.
+The product enumerator (csrc/model.cpp) is written independently and shares no
+code with this file.
+
+This is the *model oracle*: the non-linear integer formulation of PAPER.md §IV
+(lines 86-181) written out rule by rule under "reading R" (the
+same reading as SURVEY.md §8(c-2)), and maximised by evaluating EVERY point of
+the tile domain -- no pruning, no search heuristics -- instead of Z3's iterative
+"OBJ_{n+1} > OBJ_n" loop.  Both reach the exact maximum; Z3
+returns an arbitrary optimum, we add a deterministic tie-break (rule 13).
+
+Rules (PAPER.md citation for each):
+  1  dedupe references per nest; compound R/W counts once
+  2  cache-line groups -> nrefs ("references accessing distinct cache lines")
+  3  cnt(l) = #groups whose stride-1 (last) subscript uses l    ("H_i ... stride-1")
+  4  l_s1 = parallel loop stride-1 in most groups, ties innermost
+  5  L1_set = refs stride-1 in l_s1, SH_set = the rest           (Eq. 1)
+  6  V(f) = prod of T over iterators used by f
+  7  B_size = prod of T over up to the first three parallel loops
+  8  H(l) = cnt(l) * (WAF if l == l_s1); 0 for serial loops in >=3-D nests;
+     0 for parallel loops in 2-D nests
+  9  OBJ = B_size + sum H(l)*T_l, summed over nests              (Eq. 2; multi-nest sum Q15)
+ 10  domain: multiples of WAF in [WAF, min(T_P_B, N)]
+ 11  REG_SM = B_size * nrefs * FP_factor <= R_P_S
+ 12  M_SH <= SPLIT*L1_SH, M_L1 <= (1-SPLIT)*L1_SH, M_L2 <= L2, element units
+     (P:167); SPLIT=1 swaps the L1 bound for L2/#SM; SPLIT=0 puts
+     everything in the combined L1; B200 mode clamps M_SH to the opt-in
+     shared memory per block (reading Q18).
+ 13  tie-break: max OBJ, then min sum of T on objective-free positions,
+     then max T_{l_s1}, then lexicographically smallest T (reading Q16).
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass, field
+from typing import Dict, List, Optional, Sequence, Tuple
+
+import numpy as np
+
+# --------------------------------------------------------------- descriptors
+
+
+@dataclass(frozen=True)
+class Ref:
+    array: str
+    # one entry per array dimension: (sorted tuple of iterator names, constant offset)
+    subs: Tuple[Tuple[Tuple[str, ...], int], ...]
+    write: bool = False
+
+    def key(self):
+        return (self.array, self.subs)
+
+    def iters(self):
+        s = set()
+        for its, _ in self.subs:
+            s.update(its)
+        return frozenset(s)
+
+    def last_iters(self):
+        return frozenset(self.subs[-1][0])
+
+
+@dataclass
+class Loop:
+    name: str
+    extent: int
+    parallel: bool
+
+
+@dataclass
+class Nest:
+    loops: List[Loop]
+    refs: List[Ref]
+
+
+@dataclass
+class Program:
+    name: str
+    nests: List[Nest]
+    dtype_bytes: int = 4  # 4 = fp32, 8 = fp64
+
+    @property
+    def L(self) -> int:
+        return max(len(n.loops) for n in self.nests)
+
+
+def ref(array: str, *subs, write: bool = False) -> Ref:
+    """ref('A', 'i', 'k') or ref('A', ('i', 1), 'j') -> A[i+1][j]."""
+    out = []
+    for s in subs:
+        if isinstance(s, tuple):
+            name, off = s
+        else:
+            name, off = s, 0
+        its = tuple(sorted(name.split("+"))) if name else tuple()
+        out.append((its, int(off)))
+    return Ref(array, tuple(out), write)
+
+
+# ------------------------------------------------------------- GPU params
+
+
+@dataclass
+class Gpu:
+    T_P_B: int
+    T_P_W: int
+    R_P_S: int
+    R_P_B: int
+    R_P_T: int
+    L1_SH: int  # bytes
+    L2: int  # bytes
+    n_SM: int
+    max_smem_per_block: int  # bytes
+
+
+# GA100 as printed in Table I + SM count from Table III.
+# KB/MB read as KiB/MiB (reading Q2, pinned by the worked example).
+GA100 = Gpu(T_P_B=1024, T_P_W=32, R_P_S=65536, R_P_B=65536, R_P_T=255,
+            L1_SH=192 * 1024, L2=40 * 1024 * 1024, n_SM=108, max_smem_per_block=48 * 1024)
+
+# B200 nominal values: L1+SMEM 256 KiB per SM, L2 126 MiB,
+# 148 SMs, 227 KiB opt-in shared memory per block.
+B200 = Gpu(T_P_B=1024, T_P_W=32, R_P_S=65536, R_P_B=65536, R_P_T=255,
+           L1_SH=256 * 1024, L2=126 * 1024 * 1024, n_SM=148, max_smem_per_block=232448)
+
+
+@dataclass
+class Opts:
+    split_pct: int = 50
+    waf: int = 16
+    mode: int = 1  # 0 = paper mode, 1 = B200 mode (SMEM clamp)
+
+
+# ------------------------------------------------------------- derivation
+
+
+@dataclass
+class Derived:
+    loops: List[Loop]
+    refs: List[Ref]  # deduped
+    nrefs: int
+    cnt: Dict[str, int]
+    ls1: str
+    l1_refs: List[Ref]
+    sh_refs: List[Ref]
+    l1_fp: List[frozenset]  # footprints (iterator sets)
+    sh_fp: List[frozenset]
+    all_fp: List[frozenset]
+    bset: List[str]
+    H: Dict[str, int]
+
+
+def derive(nest: Nest, waf: int) -> Derived:
+    loops = nest.loops
+    depth = len(loops)
+    # rule 1: dedupe
+    seen, refs = set(), []
+    for r in nest.refs:
+        if r.key() not in seen:
+            seen.add(r.key())
+            refs.append(r)
+    # rule 2: cache-line groups
+    groups = set()
+    for r in refs:
+        groups.add((r.array, r.subs[:-1], r.last_iters()))
+    nrefs = len(groups)
+    # rule 3: counts over groups
+    cnt = {l.name: sum(1 for g in groups if l.name in g[2]) for l in loops}
+    # rule 4: CMA loop
+    cands = [(cnt[l.name], d, l.name) for d, l in enumerate(loops) if l.parallel and cnt[l.name] > 0]
+    if not cands:
+        cands = [(cnt[l.name], d, l.name) for d, l in enumerate(loops)]
+    ls1 = max(cands)[2]
+    # rule 5: sets
+    l1_refs = [r for r in refs if ls1 in r.last_iters()]
+    sh_refs = [r for r in refs if ls1 not in r.last_iters()]
+
+    def fps(rs):
+        out = []
+        for r in rs:
+            f = (r.array, r.iters())
+            if f not in out:
+                out.append(f)
+        return out
+
+    l1_fp = fps(l1_refs)
+    sh_fp = [f for f in fps(sh_refs) if f not in l1_fp]
+    all_fp = l1_fp + sh_fp
+    # rule 7: B-set
+    par = [l.name for l in loops if l.parallel]
+    bset = ([ls1] if ls1 in par else []) + [p for p in par if p != ls1]
+    bset = bset[:3]
+    # rule 8: weights
+    H = {}
+    for l in loops:
+        h = cnt[l.name] * (waf if l.name == ls1 else 1)
+        if depth >= 3 and not l.parallel:
+            h = 0
+        if depth == 2 and l.parallel:
+            h = 0
+        H[l.name] = h
+    return Derived(loops, refs, nrefs, cnt, ls1, l1_refs, sh_refs,
+                   [f[1] for f in l1_fp], [f[1] for f in sh_fp], [f[1] for f in all_fp], bset, H)
+
+
+def table2(nest: Nest, waf: int = 16):
+    """Per-reference Table II row: (ref, memory, cma, T-reuse loops, S-reuse loops)."""
+    d = derive(nest, waf)
+    rows = []
+    for r in d.refs:
+        mem = "L1" if r in d.l1_refs else "SH"
+        cma = d.ls1 in r.last_iters()
+        t_reuse = [l.name for l in d.loops if l.name not in r.iters()]
+        s_reuse = [l.name for l in d.loops if l.name in r.last_iters()]
+        rows.append((r, mem, cma, t_reuse, s_reuse))
+    return rows
+
+
+# ------------------------------------------------------------- capacities
+
+
+def caps(gpu: Gpu, opts: Opts, e: int):
+    """Element-unit capacities (rule 12). Returns dict with possibly-None entries."""
+    pct = opts.split_pct
+    c = {}
+    if pct == 0:
+        c["all_l1"] = (gpu.L1_SH) // e  # L1 u SH footprints share the whole L1
+        c["l1"] = None
+        c["sh"] = None
+    elif pct == 100:
+        c["all_l1"] = None
+        c["l1"] = gpu.L2 // (gpu.n_SM * e)
+        c["sh"] = gpu.L1_SH // e
+    else:
+        c["all_l1"] = None
+        c["l1"] = ((100 - pct) * gpu.L1_SH) // (100 * e)
+        c["sh"] = (pct * gpu.L1_SH) // (100 * e)
+    c["l2"] = gpu.L2 // e
+    if opts.mode == 1:
+        clamp = gpu.max_smem_per_block // e
+        c["sh"] = clamp if c["sh"] is None else min(c["sh"], clamp)
+        if pct == 0:
+            c["sh"] = None  # SH set lives in L1 when no shared memory is carved out
+    return c
+
+
+def domain(extent: int, gpu: Gpu, waf: int) -> List[int]:
+    hi = min(gpu.T_P_B, extent)
+    d = list(range(waf, hi + 1, waf))
+    if not d:
+        d = [extent]  # reading Q13
+    return d
+
+
+# ------------------------------------------------------------- evaluation
+
+
+@dataclass
+class Result:
+    tiles: Optional[Tuple[int, ...]]
+    obj: int
+    n_feasible: int
+    n_ties: int
+    ties: List[Tuple[int, ...]] = field(default_factory=list)
+
+
+def _prod(T, names, pos):
+    v = np.ones_like(T[0])
+    for n in names:
+        v = v * T[pos[n]]
+    return v
+
+
+def evaluate(prog: Program, gpu: Gpu, opts: Opts, T: Sequence[np.ndarray]):
+    """Vectorised rules 6-12 over arrays of tile values T[p] (one array per position).
+
+    Returns (feasible bool array, OBJ int64 array)."""
+    e = prog.dtype_bytes
+    fpf = 1 if e == 4 else 2
+    c = caps(gpu, opts, e)
+    feas = np.ones(T[0].shape, dtype=bool)
+    obj = np.zeros(T[0].shape, dtype=np.int64)
+    for nest in prog.nests:
+        d = derive(nest, opts.waf)
+        pos = {l.name: p for p, l in enumerate(nest.loops)}
+        Bn = _prod(T, d.bset, pos)
+        # rule 11
+        feas &= Bn * d.nrefs * fpf <= gpu.R_P_S
+        # rule 12
+        ml1 = sum((_prod(T, f, pos) for f in d.l1_fp), np.zeros_like(Bn))
+        msh = sum((_prod(T, f, pos) for f in d.sh_fp), np.zeros_like(Bn))
+        mall = ml1 + msh
+        if c["all_l1"] is not None:
+            feas &= mall <= c["all_l1"]
+        if c["l1"] is not None:
+            feas &= ml1 <= c["l1"]
+        if c["sh"] is not None:
+            feas &= msh <= c["sh"]
+        feas &= mall <= c["l2"]
+        # rules 8-9
+        obj = obj + Bn
+        for l in nest.loops:
+            if d.H[l.name]:
+                obj = obj + d.H[l.name] * T[pos[l.name]]
+    return feas, obj
+
+
+def objective_free_positions(prog: Program, waf: int) -> List[int]:
+    free = []
+    for p in range(prog.L):
+        ok = True
+        for nest in prog.nests:
+            if p >= len(nest.loops):
+                continue
+            d = derive(nest, waf)
+            name = nest.loops[p].name
+            if d.H[name] != 0 or name in d.bset:
+                ok = False
+        if ok:
+            free.append(p)
+    return free
+
+
+def extents(prog: Program) -> List[int]:
+    L = prog.L
+    ex = [0] * L
+    for nest in prog.nests:
+        for p, l in enumerate(nest.loops):
+            ex[p] = max(ex[p], l.extent)
+    return ex
+
+
+def select_tiles(prog: Program, gpu: Gpu, opts: Opts, keep_ties: bool = True) -> Result:
+    """Exhaustive maximisation of OBJ over the whole domain (no pruning)."""
+    L = prog.L
+    doms = [np.array(domain(n, gpu, opts.waf), dtype=np.int64) for n in extents(prog)]
+    free = objective_free_positions(prog, opts.waf)
+    ls1_pos = [l.name for l in prog.nests[0].loops].index(derive(prog.nests[0], opts.waf).ls1)
+    best_key, best, ties, n_feas = None, None, [], 0
+    # iterate the first position in Python, the rest as one numpy meshgrid block
+    rest = np.meshgrid(*doms[1:], indexing="ij") if L > 1 else []
+    rest = [r.ravel() for r in rest]
+    for t0 in doms[0]:
+        T = [np.full(rest[0].shape if rest else (1,), t0, dtype=np.int64)] + rest
+        feas, obj = evaluate(prog, gpu, opts, T)
+        n_feas += int(feas.sum())
+        if not feas.any():
+            continue
+        idx = np.nonzero(feas)[0]
+        o = obj[idx]
+        omax = int(o.max())
+        if best is not None and omax < best:
+            continue
+        sel = idx[o == omax]
+        cand = [tuple(int(T[p][k]) for p in range(L)) for k in sel]
+        if best is None or omax > best:
+            best, ties = omax, cand
+        else:
+            ties.extend(cand)
+
+    if best is None:
+        return Result(None, 0, 0, 0, [])
+
+    def key(t):
+        return (sum(t[p] for p in free), -t[ls1_pos], t)
+
+    ties.sort(key=key)
+    return Result(ties[0], best, n_feas, len(ties), ties if keep_ties else [])
+
+
+# ------------------------------------------------------------- builtins
+
+
+def P(name: str, nests: List[Nest], dtype_bytes: int = 4) -> Program:
+    return Program(name, nests, dtype_bytes)
+
+
+def matmul_paper(n: int = 1024, dtype_bytes: int = 8) -> Program:
+    """Fig. 4 matmul Out[i][j] += In[i][k] * Ker[k][j]."""
+    return P("matmul", [Nest(
+        [Loop("i", n, True), Loop("j", n, True), Loop("k", n, False)],
+        [ref("Out", "i", "j", write=True), ref("Out", "i", "j"), ref("In", "i", "k"), ref("Ker", "k", "j")],
+    )], dtype_bytes)
+
+
+def gemm(ni=4000, nj=4000, nk=4000, dtype_bytes=4) -> Program:
+    return P("gemm", [Nest(
+        [Loop("i", ni, True), Loop("j", nj, True), Loop("k", nk, False)],
+        [ref("C", "i", "j", write=True), ref("C", "i", "j"), ref("A", "i", "k"), ref("B", "k", "j")],
+    )], dtype_bytes)
+
+
+def two_mm(ni=4000, nj=4000, nk=4000, nl=4000, dtype_bytes=4) -> Program:
+    n1 = Nest([Loop("i", ni, True), Loop("j", nj, True), Loop("k", nk, False)],
+              [ref("tmp", "i", "j", write=True), ref("A", "i", "k"), ref("B", "k", "j")])
+    n2 = Nest([Loop("i", ni, True), Loop("j", nl, True), Loop("k", nj, False)],
+              [ref("D", "i", "j", write=True), ref("tmp", "i", "k"), ref("C", "k", "j")])
+    return P("2mm", [n1, n2], dtype_bytes)
+
+
+def three_mm(ni=4000, nj=4000, nk=4000, nl=4000, nm=4000, dtype_bytes=4) -> Program:
+    n1 = Nest([Loop("i", ni, True), Loop("j", nj, True), Loop("k", nk, False)],
+              [ref("E", "i", "j", write=True), ref("A", "i", "k"), ref("B", "k", "j")])
+    n2 = Nest([Loop("i", nj, True), Loop("j", nl, True), Loop("k", nm, False)],
+              [ref("F", "i", "j", write=True), ref("C", "i", "k"), ref("D", "k", "j")])
+    n3 = Nest([Loop("i", ni, True), Loop("j", nl, True), Loop("k", nj, False)],
+              [ref("G", "i", "j", write=True), ref("E", "i", "k"), ref("F", "k", "j")])
+    return P("3mm", [n1, n2, n3], dtype_bytes)
+
+
+def syrk(ni=4000, nj=4000, dtype_bytes=4) -> Program:
+    return P("syrk", [Nest(
+        [Loop("i", ni, True), Loop("j", ni, True), Loop("k", nj, False)],
+        [ref("C", "i", "j", write=True), ref("A", "i", "k"), ref("A", "j", "k")],
+    )], dtype_bytes)
+
+
+def jacobi2d(n=4000, dtype_bytes=4) -> Program:
+    """jacobi-2d-imper: compute nest + copy nest; time loop excluded (Q14)."""
+    m = n - 2  # interior extent
+    c = Nest([Loop("i", m, True), Loop("j", m, True)],
+             [ref("B", "i", "j", write=True), ref("A", "i", "j"), ref("A", "i", ("j", -1)),
+              ref("A", "i", ("j", 1)), ref("A", ("i", 1), "j"), ref("A", ("i", -1), "j")])
+    cp = Nest([Loop("i", m, True), Loop("j", m, True)],
+              [ref("A", "i", "j", write=True), ref("B", "i", "j")])
+    return P("jacobi-2d", [c, cp], dtype_bytes)
+
+
+def heat3d(n=120, dtype_bytes=4) -> Program:
+    """heat-3d: one sweep nest (B = f(A)); the A = f(B) nest is identical in shape."""
+    m = n - 2
+    loops = [Loop("i", m, True), Loop("j", m, True), Loop("k", m, True)]
+
+    def sweep(dst, src):
+        return Nest(list(loops), [
+            ref(dst, "i", "j", "k", write=True),
+            ref(src, ("i", 1), "j", "k"), ref(src, "i", "j", "k"), ref(src, ("i", -1), "j", "k"),
+            ref(src, "i", ("j", 1), "k"), ref(src, "i", ("j", -1), "k"),
+            ref(src, "i", "j", ("k", 1)), ref(src, "i", "j", ("k", -1)),
+        ])
+
+    return P("heat-3d", [sweep("B", "A"), sweep("A", "B")], dtype_bytes)
+
+
+def ccsd_t_d1(d=48, dtype_bytes=4) -> Program:
+    names = ["h3", "h2", "h1", "p6", "p5", "p4", "h7"]
+    loops = [Loop(nm, d, nm != "h7") for nm in names]
+    return P("ccsd_t_d1", [Nest(loops, [
+        ref("t3", "h3", "h2", "h1", "p6", "p5", "p4", write=True),
+        ref("t2", "h7", "p4", "p5", "h1"),
+        ref("v2", "h3", "h2", "p6", "h7"),
+    ])], dtype_bytes)
+
+
+def fdtd2d(nx=1000, ny=1000, dtype_bytes=8) -> Program:
+    """PolyBench fdtd-2d nests (for the nrefs = 4 pin)."""
+    n1 = Nest([Loop("i", nx - 1, True), Loop("j", ny, True)],
+              [ref("ey", "i", "j", write=True), ref("hz", "i", "j"), ref("hz", ("i", -1), "j")])
+    n2 = Nest([Loop("i", nx, True), Loop("j", ny - 1, True)],
+              [ref("ex", "i", "j", write=True), ref("hz", "i", "j"), ref("hz", "i", ("j", -1))])
+    n3 = Nest([Loop("i", nx - 1, True), Loop("j", ny - 1, True)],
+              [ref("hz", "i", "j", write=True), ref("ex", "i", ("j", 1)), ref("ex", "i", "j"),
+               ref("ey", ("i", 1), "j"), ref("ey", "i", "j")])
+    return P("fdtd-2d", [n1, n2, n3], dtype_bytes)
+
+
+BUILTINS = {
+    "gemm": gemm, "2mm": two_mm, "3mm": three_mm, "syrk": syrk,
+    "jacobi-2d": jacobi2d, "heat-3d": heat3d, "ccsd_t_d1": ccsd_t_d1,
+}

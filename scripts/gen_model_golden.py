@@ -1,0 +1,70 @@
+#!/usr/bin/env python
+"""Write tests/golden/model_golden.json by calling ONLY oracle/model.py (brute force).
+
+The C++ enumerator in libeatss.so is checked against this file bit-exactly
+(tiles, OBJ, #ties, #feasible).  Re-run after any change of reading.
+"""
+import json
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+from oracle import model as M  # noqa: E402
+
+CASES = []
+
+
+def add(kernel, dims, dtype_bytes, gpu, split, waf, mode):
+    CASES.append(dict(kernel=kernel, dims=list(dims), dtype_bytes=dtype_bytes, gpu=gpu,
+                      split_pct=split, waf=waf, mode=mode))
+
+
+# the paper-mode pin first
+add("gemm", (1024, 1024, 1024), 8, "GA100", 50, 16, 0)
+for split in (0, 25, 50, 75, 100):
+    add("gemm", (4000, 4000, 4000), 4, "B200", split, 16, 1)
+add("gemm", (4000, 4000, 4000), 8, "B200", 50, 16, 1)
+add("gemm", (256, 256, 256), 4, "B200", 50, 16, 1)
+add("gemm", (4000, 4000, 4000), 4, "B200", 50, 32, 1)
+add("gemm", (4000, 4000, 4000), 4, "B200", 50, 8, 1)
+add("gemm", (1000, 3000, 200), 4, "B200", 50, 16, 1)
+add("2mm", (4000, 4000, 4000, 4000), 4, "B200", 50, 16, 1)
+add("2mm", (4000, 4000, 4000, 4000), 4, "B200", 100, 16, 1)
+add("3mm", (4000, 4000, 4000, 4000, 4000), 4, "B200", 50, 16, 1)
+add("3mm", (4000, 4000, 4000, 4000, 4000), 4, "B200", 0, 16, 1)
+add("syrk", (4000, 4000), 4, "B200", 50, 16, 1)
+add("syrk", (4000, 4000), 4, "B200", 100, 8, 1)
+add("jacobi-2d", (4000,), 4, "B200", 50, 16, 1)
+add("jacobi-2d", (4000,), 4, "B200", 0, 32, 1)
+for waf in (4, 8, 16, 32):
+    add("heat-3d", (120,), 4, "B200", 50, waf, 1)
+for waf in (4, 8, 16, 32):
+    for split in (0, 50, 100):
+        add("heat-3d", (120,), 8, "GA100", split, waf, 0)
+add("ccsd_t_d1", (48,), 4, "B200", 50, 4, 1)
+add("ccsd_t_d1", (48,), 4, "B200", 50, 8, 1)
+add("ccsd_t_d1", (16,), 4, "B200", 50, 4, 1)
+
+
+def main():
+    out = []
+    for c in CASES:
+        prog = M.BUILTINS[c["kernel"]](*c["dims"], dtype_bytes=c["dtype_bytes"])
+        gpu = M.GA100 if c["gpu"] == "GA100" else M.B200
+        r = M.select_tiles(prog, gpu, M.Opts(c["split_pct"], c["waf"], c["mode"]), keep_ties=False)
+        c = dict(c, tiles=list(r.tiles) if r.tiles else None, obj=r.obj, n_ties=r.n_ties,
+                 n_feasible=r.n_feasible)
+        print(c)
+        out.append(c)
+    path = os.path.join(ROOT, "tests", "golden", "model_golden.json")
+    with open(path, "w") as f:
+        json.dump({"generator": "scripts/gen_model_golden.py (oracle/model.py brute force only)",
+                   "gpus": {"GA100": M.GA100.__dict__, "B200": M.B200.__dict__},
+                   "cases": out}, f, indent=1)
+    print("wrote", path)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,148 @@
+"""Pins for the model oracle (oracle/model.py) against the paper and an independent solver.
+
+* tests/golden/worked_example.json -- the paper's worked example.
+* tests/golden/paper_facts.json    -- l_s1, Table II, no.references, heat-3d 9/12.
+* Z3 (the paper's own solver), driven iteratively exactly as the paper
+  describes, on formulations typed from the paper's printed constraints.
+* A small space whose optimum is worked out by hand in the docstring.
+"""
+import json
+import os
+
+import pytest
+
+from oracle import model as M
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def _load(name):
+    with open(os.path.join(GOLD, name)) as f:
+        return json.load(f)
+
+
+def test_worked_example_unique_optimum():
+    g = _load("worked_example.json")
+    gpu = M.Gpu(T_P_B=g["gpu"]["T_P_B"], T_P_W=32, R_P_S=g["gpu"]["R_P_S"], R_P_B=65536, R_P_T=255,
+                L1_SH=g["gpu"]["L1_SH_bytes"], L2=g["gpu"]["L2_bytes"], n_SM=g["gpu"]["n_SM"],
+                max_smem_per_block=48 * 1024)
+    prog = M.matmul_paper(n=1024, dtype_bytes=8)
+    d = M.derive(prog.nests[0], g["waf"])
+    assert d.H == g["H"]
+    assert d.nrefs == g["no_references"]
+    r = M.select_tiles(prog, gpu, M.Opts(g["split_pct"], g["waf"], mode=0))
+    assert r.tiles == tuple(g["tiles"])
+    assert r.n_ties == 1  # unique: no tie-break involved
+    Ti, Tj, Tk = g["tiles"]
+    assert r.obj == Ti * Tj + 2 * 16 * Tj
+
+
+def test_paper_facts_matmul():
+    f = _load("paper_facts.json")
+    nest = M.matmul_paper().nests[0]
+    assert M.derive(nest, 16).ls1 == f["matmul_ls1"]["value"]
+    rows = {r.array: (mem, cma, t, s) for r, mem, cma, t, s in M.table2(nest)}
+    for arr, want in f["matmul_table2"]["rows"].items():
+        mem, cma, t, s = rows[arr]
+        assert mem == want["memory"] and cma == want["cma"] and s == want["S"]
+        if "T" in want:
+            assert t == want["T"]
+    assert M.derive(nest, 16).nrefs == f["nrefs"]["matmul"]
+    assert max(M.derive(n, 16).nrefs for n in M.fdtd2d().nests) == f["nrefs"]["fdtd-2d"]
+
+
+def test_heat3d_feasible_configurations_on_ga100():
+    f = _load("paper_facts.json")["heat3d_feasible_configs"]
+    for n in (120, 200):
+        feas = {}
+        for wf in (0.125, 0.25, 0.5, 1.0):
+            for split in (0, 50, 100):
+                r = M.select_tiles(M.heat3d(n, 8), M.GA100, M.Opts(split, int(wf * 32), 0), keep_ties=False)
+                feas[(wf, split)] = r.tiles is not None
+        assert sum(feas.values()) == f["value"]
+        assert not any(v for (wf, _), v in feas.items() if wf == f["infeasible_warp_frac"])
+
+
+def test_hand_checked_small_space():
+    """gemm 64^3 fp32, B200, split 50%, WAF 16 -> domain {16,32,48,64}^3.
+
+    Caps (elements): L1 = SH = 50% * 262144 B / 4 = 32768; REG: Ti*Tj*3 <= 65536.
+    The largest footprints are Ti*Tj + Tk*Tj = 8192 and Ti*Tk = 4096, and
+    Ti*Tj*3 = 12288, so all 64 points are feasible.  OBJ = Ti*Tj + 2*16*Tj is
+    maximal at Ti = Tj = 64 (4096 + 2048 = 6144) for every Tk: 4 ties, broken by
+    the smallest objective-free Tk -> (64, 64, 16).
+    """
+    r = M.select_tiles(M.gemm(64, 64, 64), M.B200, M.Opts(50, 16, 1))
+    assert r.n_feasible == 64
+    assert r.obj == 6144 and r.n_ties == 4
+    assert r.tiles == (64, 64, 16)
+
+
+def test_infeasible_spaces():
+    assert M.select_tiles(M.heat3d(120), M.B200, M.Opts(50, 32, 1)).tiles is None
+    for waf in (8, 16):
+        assert M.select_tiles(M.ccsd_t_d1(48), M.B200, M.Opts(50, waf, 1)).tiles is None
+
+
+def _z3_iterative(build):
+    """The paper's procedure: solve, add OBJ > OBJ_n, repeat until UNSAT."""
+    z3 = pytest.importorskip("z3")
+    s = z3.Solver()
+    T, obj = build(z3, s)
+    best, model, calls = None, None, 0
+    while True:
+        calls += 1
+        if s.check() != z3.sat:
+            break
+        m = s.model()
+        best = m.eval(obj).as_long()
+        model = tuple(m.eval(t).as_long() for t in T)
+        s.add(obj > best)
+    return best, model, calls
+
+
+def test_z3_on_the_printed_worked_example_formulation():
+    # Constraints exactly as printed at P:117-121 (+ bounds/alignment of P:123-125).
+    def build(z3, s):
+        Ti, Tj, Tk = z3.Ints("Ti Tj Tk")
+        for t in (Ti, Tj, Tk):
+            s.add(t >= 16, t <= 1024, t % 16 == 0)
+        m_l1 = 50 * 192 * 1024 // (100 * 8)
+        m_sh = 50 * 192 * 1024 // (100 * 8)
+        s.add(Ti * Tj * 3 * 2 <= 65536, Ti * Tj + Tk * Tj <= m_l1, Ti * Tk <= m_sh)
+        return (Ti, Tj, Tk), Ti * Tj + 2 * 16 * Tj
+
+    best, model, _ = _z3_iterative(build)
+    assert (best, model) == (18432, (16, 384, 16))
+    r = M.select_tiles(M.matmul_paper(1024, 8), M.GA100, M.Opts(50, 16, 0))
+    assert r.obj == best and model in r.ties
+
+
+@pytest.mark.parametrize("split", [25, 50, 75])
+def test_z3_gemm_b200_objective_matches_enumeration(split):
+    e = 4
+    l1 = (100 - split) * 256 * 1024 // (100 * e)
+    sh = min(split * 256 * 1024 // (100 * e), 232448 // e)
+
+    def build(z3, s):
+        Ti, Tj, Tk = z3.Ints("Ti Tj Tk")
+        for t in (Ti, Tj, Tk):
+            s.add(t >= 16, t <= 1024, t % 16 == 0)
+        s.add(Ti * Tj * 3 <= 65536, Ti * Tj + Tk * Tj <= l1, Ti * Tk <= sh)
+        s.add(Ti * Tj + Tk * Tj + Ti * Tk <= 126 * 1024 * 1024 // e)
+        return (Ti, Tj, Tk), Ti * Tj + 2 * 16 * Tj
+
+    best, model, _ = _z3_iterative(build)
+    r = M.select_tiles(M.gemm(), M.B200, M.Opts(split, 16, 1))
+    assert r.obj == best and model in r.ties
+
+
+def test_model_golden_regenerates():
+    """tests/golden/model_golden.json was written by scripts/gen_model_golden.py (oracle only)."""
+    g = _load("model_golden.json")
+    for case in g["cases"][:6]:
+        prog = M.BUILTINS[case["kernel"]](*case["dims"], dtype_bytes=case["dtype_bytes"])
+        gpu = M.GA100 if case["gpu"] == "GA100" else M.B200
+        r = M.select_tiles(prog, gpu, M.Opts(case["split_pct"], case["waf"], case["mode"]))
+        assert (list(r.tiles) if r.tiles else None) == case["tiles"]
+        assert r.obj == case["obj"] and r.n_ties == case["n_ties"] and r.n_feasible == case["n_feasible"]
