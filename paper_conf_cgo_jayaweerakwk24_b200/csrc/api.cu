@@ -1,0 +1,577 @@
+// api.cu -- the C ABI of libeatss.so (include/eatss.h): descriptors, GPU
+// parameters, launch plans and execution.  The tile model lives in model.cpp,
+// the kernels in contract.cu / stencil.cu / ccsd.cu, energy in energy.cpp.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "contract.cuh"
+#include "desc.hpp"
+
+namespace eatss {
+
+static thread_local std::string g_err;
+void set_error(const std::string &m) { g_err = m; }
+eatss_status fail(eatss_status s, const std::string &m) {
+    g_err = m;
+    return s;
+}
+static eatss_status cuda_fail(cudaError_t e, const char *where) {
+    return fail(EATSS_E_CUDA, std::string(where) + ": " + cudaGetErrorName(e) + " (" +
+                                  cudaGetErrorString(e) + ")");
+}
+
+// stencil.cu / ccsd.cu entry points
+cudaError_t launch_jacobi2d_sweep(void *dst, const void *src, const void *bsrc, int64_t n, int64_t Ti,
+                                  int64_t Tj, bool f64, int carveout, int32_t *counts, cudaStream_t s);
+cudaError_t launch_interior_copy2d(void *dst, const void *src, int64_t n, bool f64, cudaStream_t s);
+cudaError_t launch_heat3d_sweep(void *dst, const void *src, int64_t n, int64_t Ti, int64_t Tj,
+                                int64_t Tk, bool f64, int carveout, int32_t *counts, cudaStream_t s);
+void stencil_plan_dims(bool heat, int64_t n, const int64_t *t, bool f64, int64_t *gx, int64_t *gy,
+                       int *bx, int *by, int *vec);
+cudaError_t launch_ccsd_d1(float *t3, const float *t2, const float *v2, const int64_t *dims,
+                           const int64_t *tiles, int64_t h3_begin, int64_t h3_count, int carveout,
+                           int32_t *counts, cudaStream_t s);
+void ccsd_plan_dims(const int64_t *dims, const int64_t *tiles, int64_t *gx, int64_t *gy, int *bx,
+                    int *by, int *rm, int *rn, int *passes, int *smem);
+
+// ------------------------------------------------------------------ builtin nests
+// Loop positions are bits: the model only needs which loops a subscript uses.
+static Sub S(uint32_t iters, int off = 0) {
+    Sub s;
+    s.iters = iters;
+    s.off = off;
+    return s;
+}
+static Ref R(int array, std::vector<Sub> subs, bool write = false) {
+    Ref r;
+    r.array = array;
+    r.subs = std::move(subs);
+    r.write = write;
+    return r;
+}
+static Nest N3(int64_t e0, int64_t e1, int64_t e2, bool p2, std::vector<Ref> refs) {
+    Nest n;
+    n.loops = {{e0, true}, {e1, true}, {e2, p2}};
+    n.refs = std::move(refs);
+    return n;
+}
+
+enum : uint32_t { I = 1u, J = 2u, K = 4u };
+
+// gemm-like nest Out[i][j] (+)= In[i][k] * Ker[k][j]   (Fig. 4)
+static Nest mm_nest(int64_t ni, int64_t nj, int64_t nk, int out, int in, int ker, bool out_read) {
+    std::vector<Ref> refs{R(out, {S(I), S(J)}, true)};
+    if (out_read) refs.push_back(R(out, {S(I), S(J)}));
+    refs.push_back(R(in, {S(I), S(K)}));
+    refs.push_back(R(ker, {S(K), S(J)}));
+    return N3(ni, nj, nk, false, refs);
+}
+
+static eatss_status build(eatss_kernel_desc *d) {
+    const auto &x = d->dims;
+    switch (d->kind) {
+        case EATSS_GEMM:  // C A B
+            d->nests = {mm_nest(x[0], x[1], x[2], 0, 1, 2, true)};
+            d->buffer_elems = {x[0] * x[1], x[0] * x[2], x[2] * x[1]};
+            break;
+        case EATSS_2MM:  // tmp A B C D ; dims ni nj nk nl
+            d->nests = {mm_nest(x[0], x[1], x[2], 0, 1, 2, false), mm_nest(x[0], x[3], x[1], 4, 0, 3, true)};
+            d->buffer_elems = {x[0] * x[1], x[0] * x[2], x[2] * x[1], x[1] * x[3], x[0] * x[3]};
+            break;
+        case EATSS_3MM:  // E A B F C D G ; dims ni nj nk nl nm
+            d->nests = {mm_nest(x[0], x[1], x[2], 0, 1, 2, false), mm_nest(x[1], x[3], x[4], 3, 4, 5, false),
+                        mm_nest(x[0], x[3], x[1], 6, 0, 3, false)};
+            d->buffer_elems = {x[0] * x[1], x[0] * x[2], x[2] * x[1], x[1] * x[3],
+                               x[1] * x[4], x[4] * x[3], x[0] * x[3]};
+            break;
+        case EATSS_SYRK: {  // C A ; dims ni nj
+            d->nests = {N3(x[0], x[0], x[1], false,
+                           {R(0, {S(I), S(J)}, true), R(0, {S(I), S(J)}), R(1, {S(I), S(K)}), R(1, {S(J), S(K)})})};
+            d->buffer_elems = {x[0] * x[0], x[0] * x[1]};
+            break;
+        }
+        case EATSS_JACOBI2D: {  // A B ; dims n ; interior extent n-2, time loop excluded
+            const int64_t m = x[0] - 2;
+            Nest c, cp;
+            c.loops = {{m, true}, {m, true}};
+            c.refs = {R(1, {S(I), S(J)}, true), R(0, {S(I), S(J)}), R(0, {S(I), S(J, -1)}),
+                      R(0, {S(I), S(J, 1)}), R(0, {S(I, 1), S(J)}), R(0, {S(I, -1), S(J)})};
+            cp.loops = c.loops;
+            cp.refs = {R(0, {S(I), S(J)}, true), R(1, {S(I), S(J)})};
+            d->nests = {c, cp};
+            d->buffer_elems = {x[0] * x[0], x[0] * x[0]};
+            break;
+        }
+        case EATSS_HEAT3D: {  // A B ; dims n
+            const int64_t m = x[0] - 2;
+            auto sweep = [&](int dst, int src) {
+                Nest n;
+                n.loops = {{m, true}, {m, true}, {m, true}};
+                n.refs = {R(dst, {S(I), S(J), S(K)}, true),
+                          R(src, {S(I, 1), S(J), S(K)}), R(src, {S(I), S(J), S(K)}), R(src, {S(I, -1), S(J), S(K)}),
+                          R(src, {S(I), S(J, 1), S(K)}), R(src, {S(I), S(J, -1), S(K)}),
+                          R(src, {S(I), S(J), S(K, 1)}), R(src, {S(I), S(J), S(K, -1)})};
+                return n;
+            };
+            d->nests = {sweep(1, 0), sweep(0, 1)};
+            d->buffer_elems = {x[0] * x[0] * x[0], x[0] * x[0] * x[0]};
+            break;
+        }
+        case EATSS_CCSD_T_D1: {  // t3 t2 v2 ; loops h3 h2 h1 p6 p5 p4 h7
+            Nest n;
+            for (int p = 0; p < 7; p++) n.loops.push_back({x[p], p != 6});
+            const uint32_t h3 = 1, h2 = 2, h1 = 4, p6 = 8, p5 = 16, p4 = 32, h7 = 64;
+            n.refs = {R(0, {S(h3), S(h2), S(h1), S(p6), S(p5), S(p4)}, true),
+                      R(0, {S(h3), S(h2), S(h1), S(p6), S(p5), S(p4)}),
+                      R(1, {S(h7), S(p4), S(p5), S(h1)}), R(2, {S(h3), S(h2), S(p6), S(h7)})};
+            d->nests = {n};
+            d->buffer_elems = {x[0] * x[1] * x[2] * x[3] * x[4] * x[5], x[6] * x[5] * x[4] * x[2],
+                               x[0] * x[1] * x[3] * x[6]};
+            break;
+        }
+        default:
+            return fail(EATSS_E_INVALID, "eatss_desc_builtin: unknown builtin");
+    }
+    d->num_buffers = (int)d->buffer_elems.size();
+    return EATSS_OK;
+}
+
+static const int kDimsPerBuiltin[] = {3, 4, 5, 2, 1, 1, 7};
+
+// ------------------------------------------------------------------ execution helpers
+static int smem_limit_bytes() {
+    int dev = 0, v = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return 232448;
+    if (cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev) != cudaSuccess) return 232448;
+    return v;
+}
+
+// The gemm-family nests of a program as executor arguments.
+static std::vector<ContractNest> contraction_nests(const eatss_kernel_desc *d, void *const *b) {
+    const auto &x = d->dims;
+    const bool f64 = d->dtype == EATSS_F64;
+    auto mk = [&](int64_t M, int64_t Nn, int64_t Kk, const void *A, int64_t lda, const void *B, int64_t ldb,
+                  bool tB, void *C, int64_t ldc, double al, double be, bool z) {
+        ContractNest n;
+        n.M = M; n.N = Nn; n.K = Kk; n.A = A; n.lda = lda; n.B = B; n.ldb = ldb; n.transB = tB;
+        n.C = C; n.ldc = ldc; n.alpha = al; n.beta = be; n.init_zero = z; n.f64 = f64;
+        return n;
+    };
+    std::vector<ContractNest> v;
+    switch (d->kind) {
+        case EATSS_GEMM:
+            v.push_back(mk(x[0], x[1], x[2], b[1], x[2], b[2], x[1], false, b[0], x[1], d->alpha, d->beta, false));
+            break;
+        case EATSS_2MM:
+            v.push_back(mk(x[0], x[1], x[2], b[1], x[2], b[2], x[1], false, b[0], x[1], d->alpha, 0.0, true));
+            v.push_back(mk(x[0], x[3], x[1], b[0], x[1], b[3], x[3], false, b[4], x[3], 1.0, d->beta, false));
+            break;
+        case EATSS_3MM:
+            v.push_back(mk(x[0], x[1], x[2], b[1], x[2], b[2], x[1], false, b[0], x[1], 1.0, 0.0, true));
+            v.push_back(mk(x[1], x[3], x[4], b[4], x[4], b[5], x[3], false, b[3], x[3], 1.0, 0.0, true));
+            v.push_back(mk(x[0], x[3], x[1], b[0], x[1], b[3], x[3], false, b[6], x[3], 1.0, 0.0, true));
+            break;
+        case EATSS_SYRK:
+            v.push_back(mk(x[0], x[0], x[1], b[1], x[1], b[1], x[1], true, b[0], x[0], d->alpha, d->beta, false));
+            break;
+        default:
+            break;
+    }
+    return v;
+}
+
+static bool is_contraction(eatss_builtin k) {
+    return k == EATSS_GEMM || k == EATSS_2MM || k == EATSS_3MM || k == EATSS_SYRK;
+}
+
+static eatss_status check_tiles(const eatss_kernel_desc *d, const int64_t *tiles) {
+    if (!tiles) return fail(EATSS_E_INVALID, "tiles is null");
+    const int L = eatss_desc_num_loops(d);
+    for (int p = 0; p < L; p++)
+        if (tiles[p] <= 0) return fail(EATSS_E_INVALID, "tile entries must be >= 1");
+    return EATSS_OK;
+}
+
+static eatss_status check_bufs(const eatss_kernel_desc *d, void *const *b) {
+    if (!b) return fail(EATSS_E_INVALID, "buffers is null");
+    for (int i = 0; i < d->num_buffers; i++)
+        if (!b[i] && d->buffer_elems[i] > 0) return fail(EATSS_E_INVALID, "buffer pointer is null");
+    return EATSS_OK;
+}
+
+// Issue the stencil time loop on stream s (no graph).
+static cudaError_t stencil_issue(const eatss_kernel_desc *d, const int64_t *t, void *const *b, cudaStream_t s) {
+    const bool f64 = d->dtype == EATSS_F64;
+    const int64_t n = d->dims[0];
+    const int cv = d->exec.split_pct;
+    cudaError_t e = cudaSuccess;
+    if (n < 3) return cudaSuccess;
+    if (d->kind == EATSS_JACOBI2D) {
+        void *A = b[0], *B = b[1];
+        for (int64_t step = 0; step < d->tsteps && e == cudaSuccess; step++) {
+            if (step % 2 == 0) e = launch_jacobi2d_sweep(B, A, A, n, t[0], t[1], f64, cv, nullptr, s);
+            else e = launch_jacobi2d_sweep(A, B, A, n, t[0], t[1], f64, cv, nullptr, s);
+        }
+        if (e == cudaSuccess && d->tsteps > 0) {
+            // the literal copy nest of the last step (both interiors end equal to X_T)
+            if (d->tsteps % 2 == 1) e = launch_interior_copy2d(A, B, n, f64, s);
+            else e = launch_interior_copy2d(B, A, n, f64, s);
+        }
+    } else {
+        void *A = b[0], *B = b[1];
+        for (int64_t step = 0; step < d->tsteps && e == cudaSuccess; step++) {
+            e = launch_heat3d_sweep(B, A, n, t[0], t[1], t[2], f64, cv, nullptr, s);
+            if (e == cudaSuccess) e = launch_heat3d_sweep(A, B, n, t[0], t[1], t[2], f64, cv, nullptr, s);
+        }
+    }
+    return e;
+}
+
+static eatss_status stencil_run(eatss_kernel_desc *d, const int64_t *t, void *const *b, cudaStream_t s) {
+    if (!d->exec.use_graph || d->tsteps <= 1) {
+        cudaError_t e = stencil_issue(d, t, b, s);
+        return e == cudaSuccess ? EATSS_OK : cuda_fail(e, "eatss_run(stencil)");
+    }
+    GraphKey key;
+    key.tiles.assign(t, t + eatss_desc_num_loops(d));
+    for (int i = 0; i < d->num_buffers; i++) key.bufs.push_back((uintptr_t)b[i]);
+    key.stream = 0;  // graphs are stream-independent; launched on the caller's stream
+    cudaGraphExec_t exec = nullptr;
+    {
+        std::lock_guard<std::mutex> lk(d->graph_mu);
+        auto it = d->graphs.find(key);
+        if (it != d->graphs.end()) exec = (cudaGraphExec_t)it->second;
+    }
+    if (!exec) {
+        // set function attributes outside capture by issuing nothing: attributes are
+        // set inside the launchers, which is legal during thread-local capture.
+        cudaStream_t cs;
+        cudaError_t e = cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaStreamCreate");
+        e = cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal);
+        if (e != cudaSuccess) {
+            cudaStreamDestroy(cs);
+            return cuda_fail(e, "cudaStreamBeginCapture");
+        }
+        cudaError_t ei = stencil_issue(d, t, b, cs);
+        cudaGraph_t g = nullptr;
+        e = cudaStreamEndCapture(cs, &g);
+        cudaStreamDestroy(cs);
+        if (ei != cudaSuccess) {
+            if (g) cudaGraphDestroy(g);
+            return cuda_fail(ei, "stencil capture");
+        }
+        if (e != cudaSuccess) return cuda_fail(e, "cudaStreamEndCapture");
+        e = cudaGraphInstantiate(&exec, g, 0);
+        cudaGraphDestroy(g);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaGraphInstantiate");
+        std::lock_guard<std::mutex> lk(d->graph_mu);
+        d->graphs[key] = exec;
+    }
+    cudaError_t e = cudaGraphLaunch(exec, s);
+    return e == cudaSuccess ? EATSS_OK : cuda_fail(e, "cudaGraphLaunch");
+}
+
+}  // namespace eatss
+
+using namespace eatss;
+
+eatss_kernel_desc::~eatss_kernel_desc() {
+    for (auto &kv : graphs) cudaGraphExecDestroy((cudaGraphExec_t)kv.second);
+}
+
+extern "C" {
+
+const char *eatss_last_error(void) { return g_err.c_str(); }
+int eatss_abi_version(void) { return EATSS_ABI_VERSION; }
+
+eatss_status eatss_desc_builtin(eatss_builtin k, const int64_t *dims, int ndims, eatss_dtype dt,
+                                int64_t tsteps, eatss_kernel_desc **out) {
+    if (!out) return fail(EATSS_E_INVALID, "eatss_desc_builtin: out is null");
+    *out = nullptr;
+    if ((int)k < 0 || (int)k > (int)EATSS_CCSD_T_D1) return fail(EATSS_E_INVALID, "eatss_desc_builtin: bad builtin");
+    if (dt != EATSS_F32 && dt != EATSS_F64) return fail(EATSS_E_INVALID, "eatss_desc_builtin: bad dtype");
+    if (!dims) return fail(EATSS_E_INVALID, "eatss_desc_builtin: dims is null");
+    const int want = kDimsPerBuiltin[k];
+    std::vector<int64_t> dv;
+    if (k == EATSS_CCSD_T_D1 && ndims == 1) dv.assign(7, dims[0]);
+    else if (ndims == want) dv.assign(dims, dims + ndims);
+    else return fail(EATSS_E_INVALID, "eatss_desc_builtin: wrong number of dims");
+    for (int64_t v : dv)
+        if (v <= 0) return fail(EATSS_E_INVALID, "eatss_desc_builtin: dims must be >= 1");
+    if ((k == EATSS_JACOBI2D || k == EATSS_HEAT3D) && (dv[0] < 3 || tsteps < 0))
+        return fail(EATSS_E_INVALID, "eatss_desc_builtin: stencils need n >= 3 and tsteps >= 0");
+    if (k == EATSS_CCSD_T_D1 && dt != EATSS_F32)
+        return fail(EATSS_E_UNSUPPORTED, "eatss_desc_builtin: ccsd_t_d1 is fp32 only in this build");
+    auto *d = new (std::nothrow) eatss_kernel_desc();
+    if (!d) return fail(EATSS_E_NOMEM, "eatss_desc_builtin: out of memory");
+    d->kind = k;
+    d->dtype = dt;
+    d->dims = dv;
+    d->tsteps = tsteps;
+    eatss_status st = build(d);
+    if (st != EATSS_OK) {
+        delete d;
+        return st;
+    }
+    *out = d;
+    return EATSS_OK;
+}
+
+void eatss_desc_destroy(eatss_kernel_desc *d) { delete d; }
+
+int eatss_desc_num_loops(const eatss_kernel_desc *d) {
+    if (!d) return -1;
+    size_t L = 0;
+    for (const Nest &n : d->nests) L = std::max(L, n.loops.size());
+    return (int)L;
+}
+int eatss_desc_num_nests(const eatss_kernel_desc *d) { return d ? (int)d->nests.size() : -1; }
+int eatss_desc_num_buffers(const eatss_kernel_desc *d) { return d ? d->num_buffers : -1; }
+int64_t eatss_desc_buffer_elems(const eatss_kernel_desc *d, int i) {
+    if (!d || i < 0 || i >= d->num_buffers) return -1;
+    return d->buffer_elems[i];
+}
+
+double eatss_desc_flops(const eatss_kernel_desc *d) {
+    if (!d) return 0;
+    const auto &x = d->dims;
+    auto D = [](int64_t v) { return (double)v; };
+    switch (d->kind) {
+        case EATSS_GEMM: return 2 * D(x[0]) * D(x[1]) * D(x[2]);
+        case EATSS_2MM: return 2 * D(x[0]) * D(x[1]) * D(x[2]) + 2 * D(x[0]) * D(x[3]) * D(x[1]);
+        case EATSS_3MM:
+            return 2 * (D(x[0]) * D(x[1]) * D(x[2]) + D(x[1]) * D(x[3]) * D(x[4]) + D(x[0]) * D(x[3]) * D(x[1]));
+        case EATSS_SYRK: return 2 * D(x[0]) * D(x[0]) * D(x[1]);
+        case EATSS_JACOBI2D: return 5 * D(x[0] - 2) * D(x[0] - 2) * D(d->tsteps);
+        case EATSS_HEAT3D: return 15 * D(x[0] - 2) * D(x[0] - 2) * D(x[0] - 2) * 2 * D(d->tsteps);
+        case EATSS_CCSD_T_D1: return 2 * D(x[0]) * D(x[1]) * D(x[2]) * D(x[3]) * D(x[4]) * D(x[5]) * D(x[6]);
+    }
+    return 0;
+}
+
+double eatss_desc_bytes(const eatss_kernel_desc *d) {
+    if (!d) return 0;
+    const double e = dtype_bytes(d->dtype);
+    const auto &x = d->dims;
+    auto D = [](int64_t v) { return (double)v; };
+    switch (d->kind) {
+        case EATSS_GEMM: return e * (D(x[0]) * D(x[2]) + D(x[2]) * D(x[1]) + 2 * D(x[0]) * D(x[1]));
+        case EATSS_2MM:  // A B read, tmp written; tmp C read, D read+written
+            return e * (D(x[0]) * D(x[2]) + D(x[2]) * D(x[1]) + D(x[0]) * D(x[1]) + D(x[0]) * D(x[1]) +
+                        D(x[1]) * D(x[3]) + 2 * D(x[0]) * D(x[3]));
+        case EATSS_3MM: {
+            double s = 0;
+            for (int i = 0; i < 7; i++) s += D(d->buffer_elems[i]);
+            return e * (s + D(d->buffer_elems[0]) + D(d->buffer_elems[3]));  // E, F re-read by G
+        }
+        case EATSS_SYRK: return e * (D(x[0]) * D(x[1]) + 2 * D(x[0]) * D(x[0]));
+        case EATSS_JACOBI2D:  // per sweep (no time tiling): read src + write dst; + final copy
+            return e * 2 * D(x[0]) * D(x[0]) * (D(d->tsteps) + (d->tsteps > 0 ? 1 : 0));
+        case EATSS_HEAT3D: return e * 2 * D(x[0]) * D(x[0]) * D(x[0]) * 2 * D(d->tsteps);
+        case EATSS_CCSD_T_D1:
+            return e * (2 * D(d->buffer_elems[0]) + D(d->buffer_elems[1]) + D(d->buffer_elems[2]));
+    }
+    return 0;
+}
+
+eatss_status eatss_desc_set_scalars(eatss_kernel_desc *d, double alpha, double beta) {
+    if (!d) return fail(EATSS_E_INVALID, "eatss_desc_set_scalars: null descriptor");
+    d->alpha = alpha;
+    d->beta = beta;
+    return EATSS_OK;
+}
+
+eatss_status eatss_desc_set_exec(eatss_kernel_desc *d, const eatss_exec_opts *o) {
+    if (!d || !o) return fail(EATSS_E_INVALID, "eatss_desc_set_exec: null argument");
+    if (o->split_pct < 0 || o->split_pct > 100) return fail(EATSS_E_INVALID, "split_pct must be 0..100");
+    if (o->engine < 0 || o->engine > 2) return fail(EATSS_E_INVALID, "bad engine");
+    d->exec = *o;
+    return EATSS_OK;
+}
+
+eatss_status eatss_gpu_params_b200(eatss_gpu_params *o) {
+    if (!o) return fail(EATSS_E_INVALID, "null");
+    *o = {1024, 32, 255, 65536, 65536, 256 * 1024, 126LL * 1024 * 1024, 148, 232448};
+    return EATSS_OK;
+}
+
+eatss_status eatss_gpu_params_ga100(eatss_gpu_params *o) {
+    if (!o) return fail(EATSS_E_INVALID, "null");
+    // Table I: KB/MB read as KiB/MiB (reading Q2); SMs from Table III
+    *o = {1024, 32, 255, 65536, 65536, 192 * 1024, 40LL * 1024 * 1024, 108, 48 * 1024};
+    return EATSS_OK;
+}
+
+eatss_status eatss_gpu_params_query(int device, eatss_gpu_params *o) {
+    if (!o) return fail(EATSS_E_INVALID, "null");
+    int v[8];
+    cudaDeviceAttr a[8] = {cudaDevAttrMaxThreadsPerBlock, cudaDevAttrWarpSize, cudaDevAttrMaxRegistersPerMultiprocessor,
+                           cudaDevAttrMaxRegistersPerBlock, cudaDevAttrL2CacheSize, cudaDevAttrMultiProcessorCount,
+                           cudaDevAttrMaxSharedMemoryPerBlockOptin, cudaDevAttrMaxSharedMemoryPerMultiprocessor};
+    for (int i = 0; i < 8; i++) {
+        cudaError_t e = cudaDeviceGetAttribute(&v[i], a[i], device);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaDeviceGetAttribute");
+    }
+    o->threads_per_block = v[0];
+    o->threads_per_warp = v[1];
+    o->regs_per_thread = 255;
+    o->regs_per_sm = v[2];
+    o->regs_per_block = v[3];
+    // combined L1 + shared memory per SM is not queryable: datasheet 256 KiB on sm_100
+    o->l1_shared_bytes = 256 * 1024;
+    o->l2_bytes = v[4];
+    o->num_sms = v[5];
+    o->max_smem_per_block = v[6];
+    return EATSS_OK;
+}
+
+eatss_status eatss_plan(const eatss_kernel_desc *d, const int64_t *tiles, eatss_launch_plan *plans,
+                        int max_plans, int *n_plans) {
+    if (!d || !plans || !n_plans) return fail(EATSS_E_INVALID, "eatss_plan: null argument");
+    eatss_status st = check_tiles(d, tiles);
+    if (st != EATSS_OK) return st;
+    const int nn = (int)d->nests.size();
+    if (max_plans < nn) return fail(EATSS_E_INVALID, "eatss_plan: max_plans < number of nests");
+    const int L = eatss_desc_num_loops(d);
+    const bool f64 = d->dtype == EATSS_F64;
+    *n_plans = 0;
+    if (is_contraction(d->kind)) {
+        // alignment-dependent choices assume 256-byte aligned buffers (cudaMalloc / torch)
+        std::vector<char> fake(16);
+        void *b[EATSS_MAX_BUFFERS];
+        for (int i = 0; i < EATSS_MAX_BUFFERS; i++) b[i] = (void *)(uintptr_t)(256 * (i + 1));
+        auto cn = contraction_nests(d, b);
+        for (int i = 0; i < (int)cn.size(); i++) {
+            ContractPlan p = plan_contraction(cn[i], tiles, 232448);
+            eatss_launch_plan &o = plans[i];
+            std::memset(&o, 0, sizeof(o));
+            o.nest = i; o.engine = 1;
+            o.grid_x = p.grid_x; o.grid_y = p.grid_y; o.grid_z = 1;
+            o.block_x = p.bx; o.block_y = p.by; o.rm = p.rm; o.rn = p.rn; o.vec = p.vec;
+            o.passes = p.passes_i * p.passes_j; o.smem_bytes = p.smem_bytes;
+            o.a_in_smem = p.a_smem; o.b_in_smem = p.b_smem; o.carveout_pct = d->exec.split_pct;
+            o.simt_x = std::min(32, p.bx);
+            o.tile[0] = p.Ti; o.tile[1] = p.Tj; o.tile[2] = p.Tk;
+        }
+        *n_plans = (int)cn.size();
+    } else if (d->kind == EATSS_JACOBI2D || d->kind == EATSS_HEAT3D) {
+        for (int i = 0; i < nn; i++) {
+            eatss_launch_plan &o = plans[i];
+            std::memset(&o, 0, sizeof(o));
+            o.nest = i; o.engine = 1;
+            int64_t t[3];
+            for (int p = 0; p < L; p++) t[p] = std::min(tiles[p], d->dims[0]);
+            stencil_plan_dims(d->kind == EATSS_HEAT3D, d->dims[0], t, f64, &o.grid_x, &o.grid_y, &o.block_x,
+                              &o.block_y, &o.vec);
+            o.grid_z = 1; o.rm = 1; o.rn = o.vec; o.passes = 1; o.carveout_pct = d->exec.split_pct;
+            o.simt_x = std::min(32, o.block_x);
+            for (int p = 0; p < L; p++) o.tile[p] = t[p];
+        }
+        *n_plans = nn;
+    } else {
+        eatss_launch_plan &o = plans[0];
+        std::memset(&o, 0, sizeof(o));
+        o.engine = 1;
+        ccsd_plan_dims(d->dims.data(), tiles, &o.grid_x, &o.grid_y, &o.block_x, &o.block_y, &o.rm, &o.rn,
+                       &o.passes, &o.smem_bytes);
+        o.grid_z = 1; o.vec = 1; o.a_in_smem = 1; o.b_in_smem = 1; o.carveout_pct = d->exec.split_pct;
+        o.simt_x = std::min(32, o.block_x);
+        for (int p = 0; p < 7; p++) o.tile[p] = std::min(tiles[p], d->dims[p]);
+        *n_plans = 1;
+    }
+    return EATSS_OK;
+}
+
+static eatss_status run_impl(const eatss_kernel_desc *cd, int only_nest, const int64_t *tiles,
+                             void *const *buffers, void *stream) {
+    auto *d = const_cast<eatss_kernel_desc *>(cd);
+    if (!d) return fail(EATSS_E_INVALID, "eatss_run: null descriptor");
+    eatss_status st = check_tiles(d, tiles);
+    if (st != EATSS_OK) return st;
+    st = check_bufs(d, buffers);
+    if (st != EATSS_OK) return st;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0)
+        return fail(EATSS_E_CUDA, "eatss_run: no CUDA device (there is no CPU fallback)");
+    cudaStream_t s = (cudaStream_t)stream;
+    if (is_contraction(d->kind)) {
+        auto cn = contraction_nests(d, buffers);
+        const int sl = smem_limit_bytes();
+        for (int i = 0; i < (int)cn.size(); i++) {
+            if (only_nest >= 0 && i != only_nest) continue;
+            ContractPlan p = plan_contraction(cn[i], tiles, sl);
+            cudaError_t e = launch_contraction(cn[i], p, d->exec.split_pct, nullptr, s);
+            if (e != cudaSuccess) return cuda_fail(e, "eatss_run(contraction)");
+        }
+        return EATSS_OK;
+    }
+    if (d->kind == EATSS_JACOBI2D || d->kind == EATSS_HEAT3D) {
+        if (only_nest >= 0) return fail(EATSS_E_UNSUPPORTED, "eatss_run_nest: stencils run whole time loops");
+        return stencil_run(d, tiles, buffers, s);
+    }
+    cudaError_t e = launch_ccsd_d1((float *)buffers[0], (const float *)buffers[1], (const float *)buffers[2],
+                                   d->dims.data(), tiles, 0, d->dims[0], d->exec.split_pct, nullptr, s);
+    return e == cudaSuccess ? EATSS_OK : cuda_fail(e, "eatss_run(ccsd_t_d1)");
+}
+
+eatss_status eatss_run(const eatss_kernel_desc *d, const int64_t *tiles, void *const *buffers, void *stream) {
+    return run_impl(d, -1, tiles, buffers, stream);
+}
+
+eatss_status eatss_run_nest(const eatss_kernel_desc *d, int nest, const int64_t *tiles, void *const *buffers,
+                            void *stream) {
+    if (!d || nest < 0 || nest >= (int)d->nests.size()) return fail(EATSS_E_INVALID, "eatss_run_nest: bad nest");
+    return run_impl(d, nest, tiles, buffers, stream);
+}
+
+eatss_status eatss_coverage(const eatss_kernel_desc *d, int nest, const int64_t *tiles, int32_t *counts,
+                            void *stream) {
+    if (!d || !counts || nest < 0 || nest >= (int)d->nests.size())
+        return fail(EATSS_E_INVALID, "eatss_coverage: bad argument");
+    eatss_status st = check_tiles(d, tiles);
+    if (st != EATSS_OK) return st;
+    cudaStream_t s = (cudaStream_t)stream;
+    const bool f64 = d->dtype == EATSS_F64;
+    if (is_contraction(d->kind)) {
+        // operand pointers are never dereferenced in coverage mode; use aligned dummies
+        void *b[EATSS_MAX_BUFFERS];
+        for (int i = 0; i < EATSS_MAX_BUFFERS; i++) b[i] = (void *)(uintptr_t)(256 * (i + 1));
+        auto cn = contraction_nests(d, b);
+        ContractPlan p = plan_contraction(cn[nest], tiles, smem_limit_bytes());
+        p.a_smem = false;  // no operand traffic in coverage mode
+        p.b_smem = false;
+        p.smem_bytes = 0;
+        cudaError_t e = launch_contraction(cn[nest], p, d->exec.split_pct, counts, s);
+        return e == cudaSuccess ? EATSS_OK : cuda_fail(e, "eatss_coverage");
+    }
+    const int64_t n = d->dims[0];
+    cudaError_t e;
+    if (d->kind == EATSS_JACOBI2D)
+        e = launch_jacobi2d_sweep(nullptr, nullptr, nullptr, n, tiles[0], tiles[1], f64, d->exec.split_pct, counts, s);
+    else if (d->kind == EATSS_HEAT3D)
+        e = launch_heat3d_sweep(nullptr, nullptr, n, tiles[0], tiles[1], tiles[2], f64, d->exec.split_pct, counts, s);
+    else
+        e = launch_ccsd_d1(nullptr, nullptr, nullptr, d->dims.data(), tiles, 0, d->dims[0], d->exec.split_pct,
+                           counts, s);
+    return e == cudaSuccess ? EATSS_OK : cuda_fail(e, "eatss_coverage");
+}
+
+int64_t eatss_launches_per_run(const eatss_kernel_desc *d, const int64_t *tiles) {
+    (void)tiles;
+    if (!d) return -1;
+    switch (d->kind) {
+        case EATSS_GEMM: case EATSS_SYRK: case EATSS_CCSD_T_D1: return 1;
+        case EATSS_2MM: return 2;
+        case EATSS_3MM: return 3;
+        case EATSS_JACOBI2D: return d->tsteps + (d->tsteps > 0 ? 1 : 0);
+        case EATSS_HEAT3D: return 2 * d->tsteps;
+    }
+    return -1;
+}
+
+}  // extern "C"

@@ -1,0 +1,43 @@
+// contract.cuh -- internal interface of the tiled contraction executors.
+#pragma once
+#include <cstdint>
+
+#include <cuda_runtime.h>
+
+namespace eatss {
+
+// One gemm-like nest of the gemm family (gemm, 2mm, 3mm, syrk):
+//   C(i,j) = [init_zero ? 0 : beta*C(i,j)] + alpha * sum_k A(i,k) * B(k,j)
+//   A(i,k) = A[i*lda + k];  B(k,j) = transB ? B[j*ldb + k] : B[k*ldb + j];  C(i,j) = C[i*ldc + j]
+struct ContractNest {
+    int64_t M = 0, N = 0, K = 0;
+    const void *A = nullptr;
+    int64_t lda = 0;
+    const void *B = nullptr;
+    int64_t ldb = 0;
+    bool transB = false;
+    void *C = nullptr;
+    int64_t ldc = 0;
+    double alpha = 1.0, beta = 1.0;
+    bool init_zero = false;
+    bool f64 = false;
+};
+
+struct ContractPlan {
+    int64_t Ti = 0, Tj = 0, Tk = 0;  // clipped tile
+    int rm = 1, rn = 1, vec = 1;
+    int bx = 1, by = 1;
+    int passes_i = 1, passes_j = 1;
+    bool stream = false;  // accumulators not resident: RMW of C per k-tile through L1
+    bool a_smem = true, b_smem = false;
+    int nbuf = 1;
+    int tkp = 0, tjp = 0;  // shared-memory pitches (elements)
+    int smem_bytes = 0;
+    int64_t grid_x = 1, grid_y = 1;
+};
+
+ContractPlan plan_contraction(const ContractNest &n, const int64_t *tiles, int smem_limit);
+cudaError_t launch_contraction(const ContractNest &n, const ContractPlan &p, int carveout_pct,
+                               int32_t *coverage_counts, cudaStream_t s);
+
+}  // namespace eatss

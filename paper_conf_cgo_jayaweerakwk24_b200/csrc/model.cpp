@@ -1,0 +1,326 @@
+// model.cpp -- the EATSS non-linear integer tile model (§IV),
+// re-evaluated for B200 limits and maximised by exhaustive enumeration with
+// monotone pruning instead of Z3's iterative search.
+//
+// Reading R rule by rule; each function cites the passage:
+//   derive_nest   rules 1-8   (Table II)
+//   capacities    rule 12
+//   enumerate     rules 9-13  (Eq. 2, tie-break Q16)
+// Every constraint left-hand side is a sum of products of tile sizes, hence
+// monotone non-decreasing in every T_p: with unassigned positions set to their
+// smallest domain value, a violated constraint stays violated for every larger
+// value, so the DFS stops the loop at that depth (exact, no approximation).
+#include <algorithm>
+#include <chrono>
+#include <cstring>
+#include <set>
+#include <tuple>
+
+#include "desc.hpp"
+
+namespace eatss {
+
+static int popcount32(uint32_t x) { return __builtin_popcount(x); }
+
+// Rules 1-8 for one nest.
+NestModel derive_nest(const Nest &n, int waf) {
+    const int depth = (int)n.loops.size();
+    NestModel m;
+    // rule 1 -- dedupe: (array, subscripts) identical => one reference
+    std::vector<const Ref *> refs;
+    auto same = [](const Ref &a, const Ref &b) {
+        if (a.array != b.array || a.subs.size() != b.subs.size()) return false;
+        for (size_t i = 0; i < a.subs.size(); i++)
+            if (a.subs[i].iters != b.subs[i].iters || a.subs[i].off != b.subs[i].off) return false;
+        return true;
+    };
+    for (const Ref &r : n.refs) {
+        bool dup = false;
+        for (const Ref *q : refs) dup = dup || same(*q, r);
+        if (!dup) refs.push_back(&r);
+    }
+    // rule 2 -- cache-line groups: (array, all-but-last subscripts with offsets,
+    // iterator set of the last subscript) ("distinct cache lines")
+    std::set<std::vector<int64_t>> groups;
+    for (const Ref *r : refs) {
+        std::vector<int64_t> key{r->array};
+        for (size_t i = 0; i + 1 < r->subs.size(); i++) {
+            key.push_back(r->subs[i].iters);
+            key.push_back(r->subs[i].off);
+        }
+        key.push_back(-1);
+        key.push_back(r->subs.back().iters);
+        groups.insert(key);
+    }
+    m.nrefs = (int)groups.size();
+    // rule 3 -- cnt(l): groups whose stride-1 subscript uses loop l
+    m.cnt.assign(depth, 0);
+    for (const auto &g : groups) {
+        uint32_t last = (uint32_t)g.back();
+        for (int p = 0; p < depth; p++)
+            if (last & (1u << p)) m.cnt[p]++;
+    }
+    // rule 4 -- l_s1: parallel loop with the largest count, ties -> innermost
+    int best = -1;
+    for (int p = 0; p < depth; p++) {
+        if (!n.loops[p].parallel || m.cnt[p] == 0) continue;
+        if (best < 0 || m.cnt[p] > m.cnt[best] || (m.cnt[p] == m.cnt[best] && p > best)) best = p;
+    }
+    if (best < 0) {
+        for (int p = 0; p < depth; p++)
+            if (best < 0 || m.cnt[p] > m.cnt[best] || (m.cnt[p] == m.cnt[best] && p > best)) best = p;
+    }
+    m.ls1 = best;
+    // rule 5 -- L1_set / SH_set (Eq. 1); footprints deduped per (array, iterators)
+    std::vector<std::pair<int, uint32_t>> l1, sh;
+    auto all_iters = [](const Ref *r) {
+        uint32_t s = 0;
+        for (const Sub &x : r->subs) s |= x.iters;
+        return s;
+    };
+    for (const Ref *r : refs) {
+        std::pair<int, uint32_t> f{r->array, all_iters(r)};
+        bool in_l1 = (r->subs.back().iters >> m.ls1) & 1u;
+        auto &dst = in_l1 ? l1 : sh;
+        if (std::find(dst.begin(), dst.end(), f) == dst.end()) dst.push_back(f);
+    }
+    for (auto &f : l1) m.l1_fp.push_back(f.second);
+    for (auto &f : sh)
+        if (std::find(l1.begin(), l1.end(), f) == l1.end()) m.sh_fp.push_back(f.second);
+    // rule 7 -- B-set: l_s1 (if parallel) then the outermost other parallel loops, <= 3
+    int nb = 0;
+    if (n.loops[m.ls1].parallel) {
+        m.bset |= 1u << m.ls1;
+        nb++;
+    }
+    for (int p = 0; p < depth && nb < 3; p++) {
+        if (p == m.ls1 || !n.loops[p].parallel) continue;
+        m.bset |= 1u << p;
+        nb++;
+    }
+    // rule 8 -- H weights
+    m.H.assign(depth, 0);
+    for (int p = 0; p < depth; p++) {
+        int64_t h = (int64_t)m.cnt[p] * (p == m.ls1 ? waf : 1);
+        if (depth >= 3 && !n.loops[p].parallel) h = 0;
+        if (depth == 2 && n.loops[p].parallel) h = 0;
+        m.H[p] = h;
+    }
+    return m;
+}
+
+std::vector<int64_t> program_extents(const eatss_kernel_desc &d) {
+    size_t L = 0;
+    for (const Nest &n : d.nests) L = std::max(L, n.loops.size());
+    std::vector<int64_t> ex(L, 0);
+    for (const Nest &n : d.nests)
+        for (size_t p = 0; p < n.loops.size(); p++) ex[p] = std::max(ex[p], n.loops[p].extent);
+    return ex;
+}
+
+namespace {
+
+struct Caps {
+    int64_t all_l1 = -1, l1 = -1, sh = -1, l2 = -1;  // -1 = no such constraint
+};
+
+// rule 12: capacities in element units, integer floors
+Caps capacities(const eatss_gpu_params &g, const eatss_model_opts &o, int e) {
+    Caps c;
+    const int64_t pct = o.split_pct;
+    if (pct == 0) {
+        c.all_l1 = g.l1_shared_bytes / e;
+    } else if (pct == 100) {
+        c.l1 = g.l2_bytes / (g.num_sms * e);  // L2 per SM replaces L1
+        c.sh = g.l1_shared_bytes / e;
+    } else {
+        c.l1 = ((100 - pct) * g.l1_shared_bytes) / (100 * e);
+        c.sh = (pct * g.l1_shared_bytes) / (100 * e);
+    }
+    c.l2 = g.l2_bytes / e;
+    if (o.mode == 1 && pct != 0) {
+        int64_t clamp = g.max_smem_per_block / e;
+        c.sh = std::min(c.sh, clamp);
+    }
+    return c;
+}
+
+struct NestEval {
+    const Nest *nest;
+    NestModel m;
+};
+
+struct Search {
+    int L = 0;
+    std::vector<std::vector<int64_t>> dom;
+    std::vector<NestEval> nests;
+    Caps caps;
+    int64_t regs = 0;
+    int fpf = 1;
+    uint32_t free_mask = 0;
+    int ls1_pos = 0;
+    // result
+    std::vector<int64_t> T, best;
+    int64_t best_obj = -1, best_free = 0, n_feasible = 0, n_ties = 0;
+    bool found = false;
+
+    static int64_t prod(const std::vector<int64_t> &T, uint32_t mask) {
+        int64_t v = 1;
+        for (int p = 0; mask; p++, mask >>= 1)
+            if (mask & 1u) v *= T[p];
+        return v;
+    }
+
+    bool feasible(const std::vector<int64_t> &T) const {
+        for (const NestEval &ne : nests) {
+            const NestModel &m = ne.m;
+            const int64_t B = prod(T, m.bset);
+            if (B * m.nrefs * fpf > regs) return false;  // rule 11
+            int64_t ml1 = 0, msh = 0;
+            for (uint32_t f : m.l1_fp) ml1 += prod(T, f);
+            for (uint32_t f : m.sh_fp) msh += prod(T, f);
+            if (caps.all_l1 >= 0 && ml1 + msh > caps.all_l1) return false;
+            if (caps.l1 >= 0 && ml1 > caps.l1) return false;
+            if (caps.sh >= 0 && msh > caps.sh) return false;
+            if (ml1 + msh > caps.l2) return false;
+        }
+        return true;
+    }
+
+    int64_t objective(const std::vector<int64_t> &T) const {  // Eq. 2, summed over nests
+        int64_t obj = 0;
+        for (const NestEval &ne : nests) {
+            obj += prod(T, ne.m.bset);
+            for (size_t p = 0; p < ne.m.H.size(); p++) obj += ne.m.H[p] * T[p];
+        }
+        return obj;
+    }
+
+    // rule 13: is candidate T better than the incumbent (both with OBJ == best_obj)?
+    bool better_tie(const std::vector<int64_t> &T, int64_t fsum) const {
+        if (fsum != best_free) return fsum < best_free;
+        if (T[ls1_pos] != best[ls1_pos]) return T[ls1_pos] > best[ls1_pos];
+        return T < best;  // lexicographically smallest
+    }
+
+    void leaf() {
+        n_feasible++;
+        const int64_t obj = objective(T);
+        int64_t fsum = 0;
+        for (int p = 0; p < L; p++)
+            if ((free_mask >> p) & 1u) fsum += T[p];
+        if (!found || obj > best_obj) {
+            found = true;
+            best_obj = obj;
+            best = T;
+            best_free = fsum;
+            n_ties = 1;
+        } else if (obj == best_obj) {
+            n_ties++;
+            if (better_tie(T, fsum)) {
+                best = T;
+                best_free = fsum;
+            }
+        }
+    }
+
+    void dfs(int p) {
+        if (p == L) {
+            leaf();
+            return;
+        }
+        for (int64_t v : dom[p]) {
+            T[p] = v;
+            // positions > p sit at their minimum; monotone constraints => break
+            if (!feasible(T)) break;
+            dfs(p + 1);
+        }
+        T[p] = dom[p].front();
+    }
+};
+
+}  // namespace
+}  // namespace eatss
+
+using namespace eatss;
+
+extern "C" eatss_status eatss_select_tiles(const eatss_kernel_desc *d, const eatss_gpu_params *g,
+                                           const eatss_model_opts *o, int64_t *tiles,
+                                           eatss_model_report *rep) {
+    if (!d || !g || !o || !tiles) return fail(EATSS_E_INVALID, "eatss_select_tiles: null argument");
+    if (o->split_pct < 0 || o->split_pct > 100)
+        return fail(EATSS_E_INVALID, "eatss_select_tiles: split_pct must be in 0..100");
+    if (o->warp_align <= 0 || o->warp_align > 1024)
+        return fail(EATSS_E_INVALID, "eatss_select_tiles: warp_align must be in 1..1024");
+    if (g->num_sms <= 0 || g->l1_shared_bytes <= 0 || g->l2_bytes <= 0 || g->regs_per_sm <= 0 ||
+        g->threads_per_block <= 0)
+        return fail(EATSS_E_INVALID, "eatss_select_tiles: bad gpu params");
+    auto t0 = std::chrono::steady_clock::now();
+    Search s;
+    const std::vector<int64_t> ext = program_extents(*d);
+    s.L = (int)ext.size();
+    const int e = dtype_bytes(d->dtype);
+    s.fpf = (e == 8) ? 2 : 1;  // FP_factor
+    s.regs = g->regs_per_sm;
+    s.caps = capacities(*g, *o, e);
+    // rule 10 -- domain: multiples of WAF in [WAF, min(T_P_B, N)]; N < WAF -> {N}
+    for (int p = 0; p < s.L; p++) {
+        std::vector<int64_t> dm;
+        const int64_t hi = std::min<int64_t>(g->threads_per_block, ext[p]);
+        for (int64_t v = o->warp_align; v <= hi; v += o->warp_align) dm.push_back(v);
+        if (dm.empty()) dm.push_back(ext[p]);
+        s.dom.push_back(dm);
+    }
+    for (const Nest &n : d->nests) s.nests.push_back({&n, derive_nest(n, o->warp_align)});
+    // objective-free positions: H == 0 and outside the B-set in every nest
+    for (int p = 0; p < s.L; p++) {
+        bool fr = true;
+        for (const NestEval &ne : s.nests) {
+            if (p >= (int)ne.nest->loops.size()) continue;
+            if (ne.m.H[p] != 0 || ((ne.m.bset >> p) & 1u)) fr = false;
+        }
+        if (fr) s.free_mask |= 1u << p;
+    }
+    s.ls1_pos = s.nests[0].m.ls1;
+    s.T.resize(s.L);
+    for (int p = 0; p < s.L; p++) s.T[p] = s.dom[p].front();
+    s.dfs(0);
+    double secs = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+    if (rep) {
+        std::memset(rep, 0, sizeof(*rep));
+        rep->ls1_loop = s.ls1_pos;
+        for (const NestEval &ne : s.nests) rep->nrefs = std::max(rep->nrefs, ne.m.nrefs);
+        rep->n_feasible = s.n_feasible;
+        rep->n_ties = s.n_ties;
+        rep->solve_seconds = secs;
+        if (s.found) {
+            rep->obj = s.best_obj;
+            for (const NestEval &ne : s.nests) {
+                int64_t ml1 = 0, msh = 0;
+                for (uint32_t f : ne.m.l1_fp) ml1 += Search::prod(s.best, f);
+                for (uint32_t f : ne.m.sh_fp) msh += Search::prod(s.best, f);
+                const int64_t B = Search::prod(s.best, ne.m.bset);
+                rep->m_l1 = std::max(rep->m_l1, ml1);
+                rep->m_sh = std::max(rep->m_sh, msh);
+                rep->b_size = std::max(rep->b_size, B);
+                rep->reg_sm = std::max(rep->reg_sm, B * ne.m.nrefs * s.fpf);
+            }
+        }
+    }
+    if (!s.found)
+        return fail(EATSS_E_INFEASIBLE, "eatss_select_tiles: no tile vector satisfies the constraints");
+    for (int p = 0; p < s.L; p++) tiles[p] = s.best[p];
+    return EATSS_OK;
+}
+
+extern "C" eatss_status eatss_desc_model_info(const eatss_kernel_desc *d, int nest, int waf,
+                                              int32_t *ls1, int32_t *nrefs, int64_t *H) {
+    if (!d || nest < 0 || nest >= (int)d->nests.size() || waf <= 0)
+        return fail(EATSS_E_INVALID, "eatss_desc_model_info: bad nest or waf");
+    NestModel m = derive_nest(d->nests[nest], waf);
+    if (ls1) *ls1 = m.ls1;
+    if (nrefs) *nrefs = m.nrefs;
+    if (H)
+        for (size_t p = 0; p < m.H.size(); p++) H[p] = m.H[p];
+    return EATSS_OK;
+}

@@ -1,0 +1,254 @@
+// stencil.cu -- tiled stencil executors for jacobi-2d and heat-3d (sm_100a, CUDA cores).
+//
+// Only the space dimensions are tiled, the time loop is not ("PPCG does not
+// exploit inter-step data reuse (time tiling), and only the space dimensions are
+// tiled").  A tile (Ti, Tj[, Tk]) is one CTA (ti -> blockIdx.y, tj -> blockIdx.x,
+// P:74-75); tiles are aligned to multiples of T in absolute coordinates, clipped
+// to the interior 1..n-2 (reading Q25).  Both arrays are L1_set references
+// (stride-1 in l_s1 = the last dimension), read through L1 with
+// 16-byte vector loads along the contiguous dimension; each CTA streams its tile
+// once per sweep, so HBM traffic is one read of the source and one write of the
+// destination per sweep (8 B/point fp32) -- the kernel is HBM-bound.
+//
+// jacobi-2d (PolyBench 3.2, two nests per step: B = f(A); A = B) is executed as
+// a ping-pong X_{t+1} = f(X_t) over the two buffers plus ONE final copy nest:
+// the copy nest only moves B's interior into A, so after step t both interiors
+// hold X_t and A's boundary is the only boundary ever read.  A sweep that reads B
+// therefore takes its boundary cells from A (`bsrc`), which makes every X_t
+// bit-identical to the literal two-nest program while halving the traffic.
+// heat-3d (PolyBench 4.x) is already a ping-pong (B = f(A); A = f(B)).
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+namespace eatss {
+
+__device__ __forceinline__ int64_t smin64(int64_t a, int64_t b) { return a < b ? a : b; }
+__device__ __forceinline__ int64_t smax64(int64_t a, int64_t b) { return a > b ? a : b; }
+
+// ------------------------------------------------------------------ jacobi-2d
+// dst interior = 0.2 * (s[i][j] + s[i][j-1] + s[i][1+j] + s[1+i][j] + s[i-1][j]),
+// where s = src on the interior and s = bsrc on the boundary.
+template <typename T, int V, bool COVER>
+__global__ void __launch_bounds__(256) jacobi2d_sweep(T *__restrict__ dst, const T *__restrict__ src,
+                                                      const T *__restrict__ bsrc, int64_t n, int Ti,
+                                                      int Tj, int32_t *counts) {
+    const int64_t ti0 = (int64_t)blockIdx.y * Ti, tj0 = (int64_t)blockIdx.x * Tj;
+    const int64_t ilo = smax64(ti0, 1), ihi = smin64(ti0 + Ti, n - 1);  // [ilo, ihi)
+    const int64_t jlo = smax64(tj0, 1), jhi = smin64(tj0 + Tj, n - 1);
+    if (ilo >= ihi || jlo >= jhi) return;
+    const T c02 = T(0.2);
+    // groups of V consecutive columns, aligned in absolute coordinates
+    const int64_t g0 = tj0 / V, g1 = (jhi - 1) / V + 1;
+    auto S = [&](int64_t i, int64_t j) -> T {
+        const bool b = (i == 0) | (i == n - 1) | (j == 0) | (j == n - 1);
+        return b ? bsrc[i * n + j] : src[i * n + j];
+    };
+    for (int64_t i = ilo + threadIdx.y; i < ihi; i += blockDim.y) {
+        for (int64_t g = g0 + threadIdx.x; g < g1; g += blockDim.x) {
+            const int64_t j = g * V;
+            if constexpr (COVER) {
+                for (int q = 0; q < V; q++)
+                    if (j + q >= jlo && j + q < jhi) atomicAdd(counts + i * n + j + q, 1);
+                continue;
+            }
+            if constexpr (V == 4) {
+                const bool fast = (j >= jlo) && (j + 3 < jhi) && (j - 1 >= 1) && (j + 4 <= n - 2) &&
+                                  (i - 1 >= 1) && (i + 1 <= n - 2);
+                if (fast) {
+                    const float4 c = *reinterpret_cast<const float4 *>(src + i * n + j);
+                    const float4 u = *reinterpret_cast<const float4 *>(src + (i - 1) * n + j);
+                    const float4 d = *reinterpret_cast<const float4 *>(src + (i + 1) * n + j);
+                    const float l = src[i * n + j - 1], r = src[i * n + j + 4];
+                    float4 o;
+                    o.x = c02 * ((((c.x + l) + c.y) + d.x) + u.x);
+                    o.y = c02 * ((((c.y + c.x) + c.z) + d.y) + u.y);
+                    o.z = c02 * ((((c.z + c.y) + c.w) + d.z) + u.z);
+                    o.w = c02 * ((((c.w + c.z) + r) + d.w) + u.w);
+                    *reinterpret_cast<float4 *>(dst + i * n + j) = o;
+                    continue;
+                }
+            }
+            for (int q = 0; q < V; q++) {
+                const int64_t jj = j + q;
+                if (jj < jlo || jj >= jhi) continue;
+                dst[i * n + jj] =
+                    c02 * ((((S(i, jj) + S(i, jj - 1)) + S(i, jj + 1)) + S(i + 1, jj)) + S(i - 1, jj));
+            }
+        }
+    }
+}
+
+// copy nest: dst interior = src interior
+template <typename T>
+__global__ void __launch_bounds__(256) interior_copy2d(T *__restrict__ dst, const T *__restrict__ src,
+                                                       int64_t n) {
+    const int64_t m = n - 2;
+    const int64_t total = m * m;
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total;
+         e += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t i = 1 + e / m, j = 1 + e % m;
+        dst[i * n + j] = src[i * n + j];
+    }
+}
+
+// ------------------------------------------------------------------ heat-3d
+// dst = 0.125*(s[i+1]-2s+s[i-1]) + 0.125*(s[j+1]-2s+s[j-1]) + 0.125*(s[k+1]-2s+s[k-1]) + s
+template <typename T, int V, bool COVER>
+__global__ void __launch_bounds__(256) heat3d_sweep(T *__restrict__ dst, const T *__restrict__ src,
+                                                    int64_t n, int Ti, int Tj, int Tk, int nbj,
+                                                    int32_t *counts) {
+    // blockIdx.x -> k-tile, blockIdx.y -> (i-tile, j-tile)
+    const int64_t tk0 = (int64_t)blockIdx.x * Tk;
+    const int64_t ti0 = (int64_t)(blockIdx.y / nbj) * Ti, tj0 = (int64_t)(blockIdx.y % nbj) * Tj;
+    const int64_t ilo = smax64(ti0, 1), ihi = smin64(ti0 + Ti, n - 1);
+    const int64_t jlo = smax64(tj0, 1), jhi = smin64(tj0 + Tj, n - 1);
+    const int64_t klo = smax64(tk0, 1), khi = smin64(tk0 + Tk, n - 1);
+    if (ilo >= ihi || jlo >= jhi || klo >= khi) return;
+    const int64_t g0 = tk0 / V, g1 = (khi - 1) / V + 1;
+    const int64_t ng = g1 - g0, nj = jhi - jlo, ni = ihi - ilo;
+    const int64_t total = ni * nj * ng;
+    const T c = T(0.125), two = T(2.0);
+    const int64_t nn = n * n;
+    for (int64_t e = threadIdx.x; e < total; e += blockDim.x) {
+        const int64_t g = g0 + e % ng;
+        const int64_t r = e / ng;
+        const int64_t j = jlo + r % nj, i = ilo + r / nj;
+        const int64_t k = g * V;
+        const int64_t base = i * nn + j * n;
+        if constexpr (COVER) {
+            for (int q = 0; q < V; q++)
+                if (k + q >= klo && k + q < khi) atomicAdd(counts + base + k + q, 1);
+            continue;
+        }
+        if constexpr (V == 4) {
+            if (k >= klo && k + 3 < khi && k >= 1 && k + 4 <= n - 1) {
+                const float4 x = *reinterpret_cast<const float4 *>(src + base + k);
+                const float4 ip = *reinterpret_cast<const float4 *>(src + base + nn + k);
+                const float4 im = *reinterpret_cast<const float4 *>(src + base - nn + k);
+                const float4 jp = *reinterpret_cast<const float4 *>(src + base + n + k);
+                const float4 jm = *reinterpret_cast<const float4 *>(src + base - n + k);
+                const float km1 = src[base + k - 1], kp4 = src[base + k + 4];
+                float4 o;
+#define HEAT_PT(X, IP, IM, JP, JM, KP, KM) \
+    (c * (IP - two * X + IM) + c * (JP - two * X + JM) + c * (KP - two * X + KM) + X)
+                o.x = HEAT_PT(x.x, ip.x, im.x, jp.x, jm.x, x.y, km1);
+                o.y = HEAT_PT(x.y, ip.y, im.y, jp.y, jm.y, x.z, x.x);
+                o.z = HEAT_PT(x.z, ip.z, im.z, jp.z, jm.z, x.w, x.y);
+                o.w = HEAT_PT(x.w, ip.w, im.w, jp.w, jm.w, kp4, x.z);
+                *reinterpret_cast<float4 *>(dst + base + k) = o;
+                continue;
+            }
+        }
+        for (int q = 0; q < V; q++) {
+            const int64_t kk = k + q;
+            if (kk < klo || kk >= khi) continue;
+            const int64_t o = base + kk;
+            const T x = src[o];
+            dst[o] = HEAT_PT(x, src[o + nn], src[o - nn], src[o + n], src[o - n], src[o + 1], src[o - 1]);
+        }
+#undef HEAT_PT
+    }
+}
+
+// ------------------------------------------------------------------ launchers
+static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+struct StencilPlan {
+    int64_t gx, gy;
+    int bx, by;
+    int vec;
+};
+
+StencilPlan plan_jacobi2d(int64_t n, int64_t Ti, int64_t Tj, bool f64) {
+    StencilPlan p;
+    p.vec = (!f64 && n % 4 == 0) ? 4 : 1;
+    p.gx = cdiv(n - 1, Tj);
+    p.gy = cdiv(n - 1, Ti);
+    const int64_t groups = cdiv(Tj, p.vec) + 1;
+    p.bx = (int)std::min<int64_t>(groups, 256);
+    p.bx = ((p.bx + 31) / 32) * 32;
+    if (p.bx > 256) p.bx = 256;
+    p.by = (int)std::max<int64_t>(1, std::min<int64_t>(Ti, 256 / p.bx));
+    return p;
+}
+
+StencilPlan plan_heat3d(int64_t n, int64_t Ti, int64_t Tj, int64_t Tk, bool f64) {
+    StencilPlan p;
+    p.vec = (!f64 && n % 4 == 0) ? 4 : 1;
+    p.gx = cdiv(n - 1, Tk);
+    const int64_t nbi = cdiv(n - 1, Ti), nbj = cdiv(n - 1, Tj);
+    p.gy = nbi * nbj;
+    const int64_t pts = Ti * Tj * (cdiv(Tk, p.vec) + 1);
+    p.bx = (int)std::min<int64_t>(256, ((pts + 31) / 32) * 32);
+    p.by = 1;
+    return p;
+}
+
+cudaError_t launch_jacobi2d_sweep(void *dst, const void *src, const void *bsrc, int64_t n, int64_t Ti,
+                                  int64_t Tj, bool f64, int carveout, int32_t *counts, cudaStream_t s) {
+    StencilPlan p = plan_jacobi2d(n, Ti, Tj, f64);
+    dim3 grid((unsigned)p.gx, (unsigned)p.gy), block(p.bx, p.by);
+    if (p.gy > 65535) return cudaErrorInvalidConfiguration;
+#define JL(T, V, C)                                                                               \
+    do {                                                                                          \
+        cudaFuncSetAttribute(jacobi2d_sweep<T, V, C>, cudaFuncAttributePreferredSharedMemoryCarveout, \
+                             carveout);                                                           \
+        jacobi2d_sweep<T, V, C><<<grid, block, 0, s>>>((T *)dst, (const T *)src, (const T *)bsrc, n, \
+                                                       (int)Ti, (int)Tj, counts);                 \
+    } while (0)
+    if (counts) {
+        if (f64) JL(double, 1, true);
+        else if (p.vec == 4) JL(float, 4, true);
+        else JL(float, 1, true);
+    } else {
+        if (f64) JL(double, 1, false);
+        else if (p.vec == 4) JL(float, 4, false);
+        else JL(float, 1, false);
+    }
+#undef JL
+    return cudaGetLastError();
+}
+
+cudaError_t launch_interior_copy2d(void *dst, const void *src, int64_t n, bool f64, cudaStream_t s) {
+    const int64_t m = n - 2;
+    if (m <= 0) return cudaSuccess;
+    const int64_t blocks = std::min<int64_t>(cdiv(m * m, 256), 148 * 16);
+    if (f64) interior_copy2d<double><<<(unsigned)blocks, 256, 0, s>>>((double *)dst, (const double *)src, n);
+    else interior_copy2d<float><<<(unsigned)blocks, 256, 0, s>>>((float *)dst, (const float *)src, n);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_heat3d_sweep(void *dst, const void *src, int64_t n, int64_t Ti, int64_t Tj,
+                                int64_t Tk, bool f64, int carveout, int32_t *counts, cudaStream_t s) {
+    StencilPlan p = plan_heat3d(n, Ti, Tj, Tk, f64);
+    if (p.gy > 65535) return cudaErrorInvalidConfiguration;
+    const int nbj = (int)cdiv(n - 1, Tj);
+    dim3 grid((unsigned)p.gx, (unsigned)p.gy), block(p.bx, 1);
+#define HL(T, V, C)                                                                              \
+    do {                                                                                         \
+        cudaFuncSetAttribute(heat3d_sweep<T, V, C>, cudaFuncAttributePreferredSharedMemoryCarveout, \
+                             carveout);                                                          \
+        heat3d_sweep<T, V, C><<<grid, block, 0, s>>>((T *)dst, (const T *)src, n, (int)Ti, (int)Tj, \
+                                                     (int)Tk, nbj, counts);                      \
+    } while (0)
+    if (counts) {
+        if (f64) HL(double, 1, true);
+        else if (p.vec == 4) HL(float, 4, true);
+        else HL(float, 1, true);
+    } else {
+        if (f64) HL(double, 1, false);
+        else if (p.vec == 4) HL(float, 4, false);
+        else HL(float, 1, false);
+    }
+#undef HL
+    return cudaGetLastError();
+}
+
+void stencil_plan_dims(bool heat, int64_t n, const int64_t *t, bool f64, int64_t *gx, int64_t *gy,
+                       int *bx, int *by, int *vec) {
+    StencilPlan p = heat ? plan_heat3d(n, t[0], t[1], t[2], f64) : plan_jacobi2d(n, t[0], t[1], f64);
+    *gx = p.gx; *gy = p.gy; *bx = p.bx; *by = p.by; *vec = p.vec;
+}
+
+}  // namespace eatss

@@ -1,0 +1,173 @@
+"""CPU-only tests of libeatss.so: ABI surface, the C++ tile model against the
+brute-force oracle, error paths and launch-plan invariants.  No compute calls."""
+import json
+import os
+import re
+import subprocess
+
+import numpy as np
+import pytest
+
+import paper_conf_cgo_jayaweerakwk24_b200 as E
+from paper_conf_cgo_jayaweerakwk24_b200 import _abi
+from oracle import model as M
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def header_symbols():
+    src = open(os.path.join(ROOT, "include", "eatss.h")).read()
+    return sorted(set(re.findall(r"\b(eatss_[a-z0-9_]+)\s*\(", src)))
+
+
+def test_library_exports_every_declared_symbol():
+    out = subprocess.run(["nm", "-D", "--defined-only", E.lib_path], capture_output=True, text=True).stdout
+    exported = set(re.findall(r" T (eatss_\w+)", out))
+    declared = header_symbols()
+    assert declared and set(declared) <= exported, set(declared) - exported
+    # the ctypes table covers exactly the header
+    assert sorted(n for n, _, _ in _abi.DECLS) == declared
+
+
+def test_abi_version():
+    assert E.abi_version() == 1
+
+
+def _gpu(name):
+    return E.gpu_params_ga100() if name == "GA100" else E.gpu_params_b200()
+
+
+def test_gpu_param_tables_match_oracle():
+    for name, ref in (("GA100", M.GA100), ("B200", M.B200)):
+        g = _gpu(name)
+        assert g.threads_per_block == ref.T_P_B and g.regs_per_sm == ref.R_P_S
+        assert g.l1_shared_bytes == ref.L1_SH and g.l2_bytes == ref.L2 and g.num_sms == ref.n_SM
+        assert g.max_smem_per_block == ref.max_smem_per_block
+
+
+GOLD = json.load(open(os.path.join(ROOT, "tests", "golden", "model_golden.json")))
+
+
+@pytest.mark.parametrize("case", GOLD["cases"], ids=lambda c: f"{c['kernel']}-{c['gpu']}-{c['split_pct']}-{c['waf']}-{c['dtype_bytes']}")
+def test_cpp_model_bit_exact_vs_bruteforce_golden(case):
+    dtype = "f64" if case["dtype_bytes"] == 8 else "f32"
+    d = E.desc_builtin(case["kernel"], case["dims"], dtype, tsteps=1 if case["kernel"] in ("jacobi-2d", "heat-3d") else 0)
+    g = _gpu(case["gpu"])
+    if case["tiles"] is None:
+        with pytest.raises(E.EatssError) as ei:
+            E.select_tiles(d, g, case["split_pct"], case["waf"], case["mode"])
+        assert ei.value.status == _abi.EATSS_E_INFEASIBLE
+        return
+    tiles, rep = E.select_tiles(d, g, case["split_pct"], case["waf"], case["mode"])
+    assert list(tiles) == case["tiles"]
+    assert rep.obj == case["obj"]
+    assert rep.n_ties == case["n_ties"]
+    assert rep.n_feasible == case["n_feasible"]
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_cpp_model_matches_bruteforce_on_random_small_programs(seed):
+    """Random extents / splits / WAF on small spaces: C++ DFS vs unpruned numpy brute force."""
+    g = np.random.default_rng(seed)
+    kind = ["gemm", "2mm", "3mm", "syrk", "jacobi-2d", "heat-3d"][seed % 6]
+    waf = int(g.choice([4, 8, 16]))
+    split = int(g.choice([0, 25, 50, 67, 100]))
+    mode = int(g.integers(0, 2))
+    gpu_name = ["GA100", "B200"][int(g.integers(0, 2))]
+    db = int(g.choice([4, 8]))
+    if kind == "gemm":
+        dims = tuple(int(x) for x in g.integers(20, 300, 3))
+    elif kind == "2mm":
+        dims = tuple(int(x) for x in g.integers(20, 200, 4))
+    elif kind == "3mm":
+        dims = tuple(int(x) for x in g.integers(20, 150, 5))
+    elif kind == "syrk":
+        dims = tuple(int(x) for x in g.integers(20, 300, 2))
+    elif kind == "jacobi-2d":
+        dims = (int(g.integers(30, 900)),)
+    else:
+        dims = (int(g.integers(10, 90)),)
+    prog = M.BUILTINS[kind](*dims, dtype_bytes=db)
+    ref = M.select_tiles(prog, M.GA100 if gpu_name == "GA100" else M.B200, M.Opts(split, waf, mode))
+    d = E.desc_builtin(kind, dims, "f64" if db == 8 else "f32", tsteps=1 if kind in ("jacobi-2d", "heat-3d") else 0)
+    try:
+        tiles, rep = E.select_tiles(d, _gpu(gpu_name), split, waf, mode)
+    except E.EatssError as e:
+        assert e.status == _abi.EATSS_E_INFEASIBLE and ref.tiles is None
+        return
+    assert tiles == ref.tiles
+    assert (rep.obj, rep.n_ties, rep.n_feasible) == (ref.obj, ref.n_ties, ref.n_feasible)
+
+
+def test_model_info_matches_paper_example():
+    d = E.desc_builtin("gemm", (1024, 1024, 1024), "f64")
+    ls1, nrefs, H = d.model_info(0, 16)
+    assert ls1 == 1 and nrefs == 3 and H == [0, 32, 0]
+
+
+def test_error_paths():
+    with pytest.raises(E.EatssError) as e:
+        E.desc_builtin("gemm", (4000, 4000))
+    assert e.value.status == _abi.EATSS_E_INVALID
+    with pytest.raises(E.EatssError):
+        E.desc_builtin("gemm", (4000, 0, 4000))
+    with pytest.raises(E.EatssError):
+        E.desc_builtin("jacobi-2d", (2,), tsteps=1)
+    d = E.desc_builtin("gemm", (64, 64, 64))
+    with pytest.raises(E.EatssError) as e:
+        E.select_tiles(d, E.gpu_params_b200(), split_pct=101)
+    assert e.value.status == _abi.EATSS_E_INVALID
+    with pytest.raises(E.EatssError) as e:
+        E.plan(d, (16, 0, 16))
+    assert e.value.status == _abi.EATSS_E_INVALID
+    lib = E._lib
+    assert lib.eatss_select_tiles(None, None, None, None, None) == _abi.EATSS_E_INVALID
+    assert lib.eatss_run(None, None, None, None) == _abi.EATSS_E_INVALID
+    with pytest.raises(ValueError):
+        E.run(d, (16, 16, 16), [1, 2])  # wrong number of buffers
+
+
+def test_run_without_gpu_fails_loudly():
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    d = E.desc_builtin("gemm", (64, 64, 64))
+    with pytest.raises(E.EatssError) as e:
+        E.run(d, (16, 16, 16), [256, 512, 768], stream=0)
+    assert e.value.status == _abi.EATSS_E_CUDA
+
+
+def test_flops_and_bytes_accounting():
+    d = E.desc_builtin("gemm", (4000, 4000, 4000))
+    assert d.flops == 2 * 4000 ** 3
+    assert d.bytes == 4 * 4 * 4000 ** 2  # A, B read; C read + written
+    assert E.desc_builtin("ccsd_t_d1", (48,)).flops == 2 * 48 ** 7
+    assert E.desc_builtin("jacobi-2d", (4000,), tsteps=500).flops == 5 * 3998 ** 2 * 500
+    assert E.desc_builtin("heat-3d", (120,), tsteps=500).flops == 15 * 118 ** 3 * 1000
+    assert E.launches_per_run(E.desc_builtin("jacobi-2d", (64,), tsteps=7), (16, 16)) == 8
+
+
+@pytest.mark.parametrize("tiles", [(16, 1024, 16), (32, 32, 32), (4, 4, 4), (1024, 1024, 1024), (24, 768, 48), (7, 13, 5)])
+def test_contraction_plan_invariants(tiles):
+    M_, N_, K_ = 4000, 4000, 4000
+    d = E.desc_builtin("gemm", (M_, N_, K_))
+    (p,) = E.plan(d, tiles)
+    Ti, Tj, Tk = (min(t, n) for t, n in zip(tiles, (M_, N_, K_)))
+    assert (p.tile[0], p.tile[1], p.tile[2]) == (Ti, Tj, Tk)
+    assert p.grid_x == -(-N_ // Tj) and p.grid_y == -(-M_ // Ti)       # Fig. 4: tj -> x, ti -> y
+    assert 1 <= p.block_x * p.block_y <= 1024                         # tile != block (Q1)
+    # a pass covers (by*rm) x (bx*rn) outputs; passes cover the tile
+    cover_i = p.block_y * p.rm
+    cover_j = p.block_x * p.rn
+    assert p.passes >= 1
+    assert p.passes == (-(-Ti // cover_i)) * (-(-Tj // cover_j))
+    assert p.smem_bytes <= 232448
+    if p.a_in_smem:
+        assert p.smem_bytes >= Ti * Tk * 4
+
+
+def test_eatss_pick_is_register_resident():
+    d = E.desc_builtin("gemm", (4000, 4000, 4000))
+    tiles, _ = E.select_tiles(d, E.gpu_params_b200(), 50, 16)
+    (p,) = E.plan(d, tiles)
+    assert tiles == (16, 1024, 16) and p.passes == 1 and p.a_in_smem and p.vec == 4
