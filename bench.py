@@ -129,14 +129,16 @@ class ClockSampler:
             import pynvml
             pynvml.nvmlInit()
             import torch
-            bus = torch.cuda.get_device_properties(device_index).pci_bus_id if hasattr(
-                torch.cuda.get_device_properties(device_index), "pci_bus_id") else None
+            # match the CUDA device to its NVML handle by UUID (CUDA_VISIBLE_DEVICES safe)
+            want = "GPU-" + str(torch.cuda.get_device_properties(device_index).uuid)
             h = None
-            if bus:
-                try:
-                    h = pynvml.nvmlDeviceGetHandleByPciBusId(bus)
-                except Exception:
-                    h = None
+            for i in range(pynvml.nvmlDeviceGetCount()):
+                hi = pynvml.nvmlDeviceGetHandleByIndex(i)
+                u = pynvml.nvmlDeviceGetUUID(hi)
+                u = u.decode() if isinstance(u, bytes) else u
+                if u == want:
+                    h = hi
+                    break
             if h is None:
                 h = pynvml.nvmlDeviceGetHandleByIndex(device_index)
             self.nv, self.h, self.ok = pynvml, h, True

@@ -22,6 +22,7 @@
 
 #include <algorithm>
 #include <cstdint>
+#include <cstdlib>
 
 #include "contract.cuh"
 
@@ -279,7 +280,7 @@ __global__ void __launch_bounds__((16384 / (RM * RN)) < 1024 ? (16384 / (RM * RN
             }
             __syncthreads();
         }
-        if constexpr (MODE == MODE_STREAM) {
+        if constexpr (MODE == MODE_STREAM || MODE == MODE_COVER) {
             for (int pi = 0; pi < p.passes_i; pi++)
                 for (int pj = 0; pj < p.passes_j; pj++) {
                     const int ri0 = pi * BY * RM, cj0 = pj * BX * RN;
@@ -297,6 +298,160 @@ __global__ void __launch_bounds__((16384 / (RM * RN)) < 1024 ? (16384 / (RM * RN
     }
     if constexpr (MODE == MODE_RESIDENT) epilogue(true, 0, 0);
 }
+
+#include "staged.cuh"
+
+#if 0  // superseded by staged.cuh (kept out of the build)
+// ------------------------------------------------------------------ staged resident kernel
+// The register-resident fast path: per k-tile both operand slices -- the SH_set
+// tile A(i0.., k0..k0+Tk) (stored transposed so a thread's rows are contiguous)
+// and the L1_set slice B(k0..k0+Tk, j0..) -- are brought into shared memory with
+// cp.async through an S-stage ring, so the load of k-tile t+S-1 overlaps the FMAs
+// of k-tile t.  A thread owns rm contiguous rows x rn columns (16-byte vectors,
+// cyclic over the warp) -- every shared-memory read is a broadcast (A) or a
+// conflict-free 16-byte vector (B).
+template <typename T, int RM, int RN, int V, bool TRANSB>
+__global__ void __launch_bounds__((16384 / (RM * RN)) < 1024 ? (16384 / (RM * RN)) : 1024)
+    contract_staged_kernel(const CArgs<T> p) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    constexpr int VN = RN / V;
+    T *const sm = reinterpret_cast<T *>(smem_raw);
+    const int aip = p.tkp;  // A^T pitch (>= Ti, multiple of 4)
+    const int bjp = p.tjp;  // B pitch (>= Tj, multiple of 4)
+    const int stage_elems = p.Tk * (aip + bjp);
+    const int S = p.nbuf;
+
+    const int tx = threadIdx.x, ty = threadIdx.y, BX = blockDim.x;
+    const int tid = ty * BX + tx, nthr = BX * blockDim.y;
+    const int64_t i0 = (int64_t)blockIdx.y * p.Ti, j0 = (int64_t)blockIdx.x * p.Tj;
+    const int rows = (int)imin64(p.Ti, p.M - i0);
+    const int cols = (int)imin64(p.Tj, p.N - j0);
+    const int nk = (int)((p.K + p.Tk - 1) / p.Tk);
+
+    // Division-free staging walks: element e = tid + n*nthr of an (outer x inner) box is
+    // tracked as (o, i) and advanced by (nthr / inner, nthr % inner) -- one division per CTA.
+    struct Walk {
+        int o0, i0, dO, dI, inner;
+    };
+    auto mkwalk = [&](int inner) {
+        Walk w;
+        w.inner = max(inner, 1);
+        w.o0 = tid / w.inner; w.i0 = tid - w.o0 * w.inner;
+        w.dO = nthr / w.inner; w.dI = nthr - w.dO * w.inner;
+        return w;
+    };
+    const Walk wa = mkwalk(p.Tk);                                      // A: (row, k), k fastest
+    const Walk wb = TRANSB ? mkwalk(p.Tk) : mkwalk(V == 4 ? cols >> 2 : cols);  // B: (k, col) / (col, k)
+
+    auto stage = [&](int t) {
+        if (t < nk) {
+            T *As = sm + (t % S) * stage_elems;
+            T *Bs = As + p.Tk * aip;
+            const int64_t k0 = (int64_t)t * p.Tk;
+            const int kt = (int)imin64(p.Tk, p.K - k0);
+            for (int r = wa.o0, kk = wa.i0; r < rows;) {  // lanes along k: coalesced reads
+                if (kk < kt) cp_elem(As + kk * aip + r, p.A + (i0 + r) * p.lda + k0 + kk);
+                r += wa.dO; kk += wa.dI;
+                if (kk >= wa.inner) { kk -= wa.inner; r++; }
+            }
+            if constexpr (TRANSB) {
+                for (int jj = wb.o0, kk = wb.i0; jj < cols;) {
+                    if (kk < kt) cp_elem(Bs + kk * bjp + jj, p.B + (j0 + jj) * p.ldb + k0 + kk);
+                    jj += wb.dO; kk += wb.dI;
+                    if (kk >= wb.inner) { kk -= wb.inner; jj++; }
+                }
+            } else {
+                for (int kk = wb.o0, c = wb.i0; kk < kt;) {
+                    if constexpr (V == 4) cp_async16(Bs + kk * bjp + 4 * c, p.B + (k0 + kk) * p.ldb + j0 + 4 * c);
+                    else cp_elem(Bs + kk * bjp + c, p.B + (k0 + kk) * p.ldb + j0 + c);
+                    kk += wb.dO; c += wb.dI;
+                    if (c >= wb.inner) { c -= wb.inner; kk++; }
+                }
+            }
+        }
+        cp_async_commit();  // empty groups keep the wait_group count uniform
+    };
+
+    T acc[RM][RN];
+#pragma unroll
+    for (int r = 0; r < RM; r++)
+#pragma unroll
+        for (int c = 0; c < RN; c++) acc[r][c] = T(0);
+
+    const int r0 = min(ty * RM, max(0, p.tkp - RM));  // contiguous rows (clamped inside the pitch)
+    int cc[VN];
+#pragma unroll
+    for (int c = 0; c < VN; c++) cc[c] = min((tx + c * BX) * V, bjp - V);
+
+    for (int s = 0; s < S - 1; s++) stage(s);
+    for (int t = 0; t < nk; t++) {
+        stage(t + S - 1);
+        if (S == 1) cp_async_wait<0>();
+        else if (S == 2) cp_async_wait<1>();
+        else cp_async_wait<2>();
+        __syncthreads();
+        const T *As = sm + (t % S) * stage_elems;
+        const T *Bs = As + p.Tk * aip;
+        const int kt = (int)imin64(p.Tk, p.K - (int64_t)t * p.Tk);
+#pragma unroll 2
+        for (int kk = 0; kk < kt; kk++) {
+            T a[RM], b[RN];
+            if constexpr (sizeof(T) == 4 && RM % 4 == 0) {
+#pragma unroll
+                for (int r = 0; r < RM; r += 4) {
+                    const float4 v = *reinterpret_cast<const float4 *>(As + kk * aip + r0 + r);
+                    a[r] = v.x; a[r + 1] = v.y; a[r + 2] = v.z; a[r + 3] = v.w;
+                }
+            } else {
+#pragma unroll
+                for (int r = 0; r < RM; r++) a[r] = As[kk * aip + r0 + r];
+            }
+#pragma unroll
+            for (int c = 0; c < VN; c++) {
+                if constexpr (V == 4) {
+                    const float4 v = *reinterpret_cast<const float4 *>(Bs + kk * bjp + cc[c]);
+                    b[4 * c] = v.x; b[4 * c + 1] = v.y; b[4 * c + 2] = v.z; b[4 * c + 3] = v.w;
+                } else {
+                    b[c] = Bs[kk * bjp + cc[c]];
+                }
+            }
+#pragma unroll
+            for (int r = 0; r < RM; r++)
+#pragma unroll
+                for (int c = 0; c < RN; c++) acc[r][c] = fma(a[r], b[c], acc[r][c]);
+        }
+        __syncthreads();
+    }
+    cp_async_wait<0>();
+
+    // epilogue: C = (init_zero ? 0 : beta*C) + alpha*acc
+#pragma unroll
+    for (int r = 0; r < RM; r++) {
+        const int rl = ty * RM + r;
+        if (rl >= rows) continue;
+        T *crow = p.C + (i0 + rl) * p.ldc + j0;
+#pragma unroll
+        for (int c = 0; c < VN; c++) {
+            const int cl = (tx + c * BX) * V;
+            if (cl >= cols) continue;
+            if constexpr (V == 4) {
+                float4 *cp = reinterpret_cast<float4 *>(crow + cl);
+                float4 o = p.init_zero ? make_float4(0.f, 0.f, 0.f, 0.f) : *cp;
+                if (!p.init_zero) { o.x *= p.beta; o.y *= p.beta; o.z *= p.beta; o.w *= p.beta; }
+                o.x = fma(p.alpha, acc[r][4 * c + 0], o.x);
+                o.y = fma(p.alpha, acc[r][4 * c + 1], o.y);
+                o.z = fma(p.alpha, acc[r][4 * c + 2], o.z);
+                o.w = fma(p.alpha, acc[r][4 * c + 3], o.w);
+                *cp = o;
+            } else {
+                T o = p.init_zero ? T(0) : crow[cl] * p.beta;
+                crow[cl] = fma(p.alpha, acc[r][c], o);
+            }
+        }
+    }
+}
+
+#endif
 
 // ------------------------------------------------------------------ planning
 
@@ -324,7 +479,9 @@ ContractPlan plan_contraction(const ContractNest &n, const int64_t *tiles, int s
     const int ncand = v4 ? 5 : 7;
     const int64_t rows = p.Ti, cols = p.Tj;
     const int64_t outputs = rows * cols;
-    const int64_t want = cdiv(outputs, 256);
+    int target_threads = 256;
+    if (const char *e = getenv("EATSS_THREADS")) target_threads = std::max(32, atoi(e));
+    const int64_t want = cdiv(outputs, target_threads);
     // smallest micro-tile reaching `want` outputs/thread that does not exceed the tile
     int pick = -1;
     for (int c = 0; c < ncand; c++) {
@@ -374,6 +531,24 @@ ContractPlan plan_contraction(const ContractNest &n, const int64_t *tiles, int s
         p.nbuf = (p.b_smem && fits(2, false, true)) ? 2 : 1;
     }
     p.smem_bytes = (int)(p.nbuf * ((p.a_smem ? a_bytes : 0) + (p.b_smem ? b_bytes : 0)));
+    if (!p.stream) {
+        // register-resident: stage both operand slices per k-tile through an S-stage cp.async ring
+        const int64_t aip = ((p.Ti + 3) / 4) * 4, bjp = ((p.Tj + 3) / 4) * 4;
+        const int64_t stage_bytes = p.Tk * (aip + bjp) * esz;
+        int64_t s_fit = smem_limit / std::max<int64_t>(stage_bytes + 16, 1);
+        int want_s = 1;  // measured best for the EATSS tile with 2 co-resident CTAs (profiles/)
+        if (const char *e = getenv("EATSS_STAGES")) want_s = std::max(1, atoi(e));
+        const int64_t S = std::min<int64_t>(want_s, s_fit);
+        if (S >= 1 && !(getenv("EATSS_NO_STAGED") && atoi(getenv("EATSS_NO_STAGED")))) {
+            p.staged = true;
+            p.nbuf = (int)S;
+            p.tkp = (int)aip;
+            p.tjp = (int)bjp;
+            p.a_smem = true;
+            p.b_smem = true;
+            p.smem_bytes = (int)(S * stage_bytes + 16 * S);  // + one mbarrier per stage
+        }
+    }
     p.grid_x = cdiv(n.N, p.Tj);
     p.grid_y = cdiv(n.M, p.Ti);
     return p;
@@ -395,6 +570,55 @@ static cudaError_t launch_one(const CArgs<T> &a, const ContractPlan &p, int carv
     dim3 grid((unsigned)p.grid_x, (unsigned)p.grid_y, 1), block(p.bx, p.by, 1);
     k<<<grid, block, p.smem_bytes, s>>>(a);
     return cudaGetLastError();
+}
+
+template <typename T, int RM, int RN, int V, bool TB>
+static cudaError_t launch_staged(const CArgs<T> &a, const ContractPlan &p, int carveout, cudaStream_t s) {
+    auto k = contract_staged_kernel<T, RM, RN, V, TB>;
+    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem_bytes);
+    if (e != cudaSuccess) return e;
+    // The staged path keeps its operand slices in shared memory: the split's carve-out is
+    // honoured unless it would cut the co-resident CTAs below what registers allow
+    // (the sigma -> carve-out mapping).
+    cudaFuncAttributes fa;
+    if (cudaFuncGetAttributes(&fa, k) == cudaSuccess && fa.numRegs > 0) {
+        const int threads = ((p.bx * p.by + 31) / 32) * 32;
+        const int nb_regs = 65536 / (((fa.numRegs + 7) / 8) * 8 * threads);
+        const int per_cta = p.smem_bytes + 1024;  // + per-CTA reservation
+        const int nb = std::max(1, std::min(nb_regs, 233472 / per_cta));
+        const int need = (int)std::min<int64_t>(100, (100LL * nb * per_cta + 233471) / 233472);
+        carveout = std::max(carveout, need);
+    }
+    e = cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, carveout);
+    if (e != cudaSuccess) return e;
+    dim3 grid((unsigned)p.grid_x, (unsigned)p.grid_y, 1), block(p.bx, p.by, 1);
+    k<<<grid, block, p.smem_bytes, s>>>(a);
+    return cudaGetLastError();
+}
+
+template <typename T, int V, bool TB>
+static cudaError_t by_mt_staged(const CArgs<T> &a, const ContractPlan &p, int cv, cudaStream_t s) {
+    const int key = p.rm * 100 + p.rn;
+    if constexpr (V == 4) {
+        switch (key) {
+            case 104: return launch_staged<T, 1, 4, 4, TB>(a, p, cv, s);
+            case 204: return launch_staged<T, 2, 4, 4, TB>(a, p, cv, s);
+            case 404: return launch_staged<T, 4, 4, 4, TB>(a, p, cv, s);
+            case 408: return launch_staged<T, 4, 8, 4, TB>(a, p, cv, s);
+            case 808: return launch_staged<T, 8, 8, 4, TB>(a, p, cv, s);
+        }
+    } else {
+        switch (key) {
+            case 101: return launch_staged<T, 1, 1, 1, TB>(a, p, cv, s);
+            case 102: return launch_staged<T, 1, 2, 1, TB>(a, p, cv, s);
+            case 202: return launch_staged<T, 2, 2, 1, TB>(a, p, cv, s);
+            case 204: return launch_staged<T, 2, 4, 1, TB>(a, p, cv, s);
+            case 404: return launch_staged<T, 4, 4, 1, TB>(a, p, cv, s);
+            case 408: return launch_staged<T, 4, 8, 1, TB>(a, p, cv, s);
+            case 808: return launch_staged<T, 8, 8, 1, TB>(a, p, cv, s);
+        }
+    }
+    return cudaErrorInvalidConfiguration;
 }
 
 template <typename T, int V, bool TB, int MODE>
@@ -448,6 +672,13 @@ static cudaError_t launch_typed(const ContractNest &n, const ContractPlan &p, in
     a.passes_i = p.passes_i; a.passes_j = p.passes_j;
     a.counts = counts;
     if (counts) return by_variant<T, MODE_COVER>(a, p, n.transB, carveout, s);
+    if (p.staged) {
+        if constexpr (sizeof(T) == 4) {
+            if (p.vec == 4) return by_mt_staged<T, 4, false>(a, p, carveout, s);
+        }
+        if (n.transB) return by_mt_staged<T, 1, true>(a, p, carveout, s);
+        return by_mt_staged<T, 1, false>(a, p, carveout, s);
+    }
     if (p.stream) return by_variant<T, MODE_STREAM>(a, p, n.transB, carveout, s);
     return by_variant<T, MODE_RESIDENT>(a, p, n.transB, carveout, s);
 }

@@ -29,6 +29,7 @@ struct ContractPlan {
     int bx = 1, by = 1;
     int passes_i = 1, passes_j = 1;
     bool stream = false;  // accumulators not resident: RMW of C per k-tile through L1
+    bool staged = false;  // resident fast path: both operand slices staged via cp.async ring (nbuf stages)
     bool a_smem = true, b_smem = false;
     int nbuf = 1;
     int tkp = 0, tjp = 0;  // shared-memory pitches (elements)
