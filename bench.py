@@ -322,7 +322,9 @@ def main():
                        "source": "NVML total-energy counter over the timed region, summed over ranks"},
             "roofline": {"bound": "alu", "achieved": achieved, "peak": fp32_peak, "unit": "TFLOP/s",
                          "frac": achieved / fp32_peak, "traffic": traffic,
-                         "kernel": "contract_kernel<float,8,8,4,false,RESIDENT>",
+                         "kernel": (f"contract_staged_kernel<float,{p0.rm},{p0.rn},{p0.vec},false>"
+                                    if (p0.b_in_smem and p0.passes == 1) else
+                                    f"contract_kernel<float,{p0.rm},{p0.rn},{p0.vec},false>"),
                          "peak_source": f"148 SMs x 128 FP32 lanes x 2 flop x {sm_max:.0f} MHz (sm max clock)",
                          "frac_at_observed_clock": (achieved / (SM_COUNT * FP32_LANES * 2 * clocks["sm_mhz"] * 1e-6))
                          if clocks.get("sm_mhz") else None},
