@@ -505,7 +505,12 @@ static eatss_status run_impl(const eatss_kernel_desc *cd, int only_nest, const i
         for (int i = 0; i < (int)cn.size(); i++) {
             if (only_nest >= 0 && i != only_nest) continue;
             ContractPlan p = plan_contraction(cn[i], tiles, sl);
-            cudaError_t e = launch_contraction(cn[i], p, d->exec.split_pct, nullptr, s);
+            int tsm = 0, tcols = 0;
+            const bool tc = d->exec.engine == EATSS_ENGINE_TENSOR && tc_plan(cn[i], p, &tsm, &tcols);
+            if (d->exec.engine == EATSS_ENGINE_TENSOR && !tc)
+                return fail(EATSS_E_UNSUPPORTED, "eatss_run: tensor engine not applicable to this tile/operand layout");
+            cudaError_t e = tc ? launch_tc_contraction(cn[i], p, d->exec.split_pct, s)
+                               : launch_contraction(cn[i], p, d->exec.split_pct, nullptr, s);
             if (e != cudaSuccess) return cuda_fail(e, "eatss_run(contraction)");
         }
         return EATSS_OK;

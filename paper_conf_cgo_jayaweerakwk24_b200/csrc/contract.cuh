@@ -38,6 +38,9 @@ struct ContractPlan {
 };
 
 ContractPlan plan_contraction(const ContractNest &n, const int64_t *tiles, int smem_limit);
+// tensor-core (tcgen05, 3xTF32) executor: applicability / launch (tc_gemm.cu)
+bool tc_plan(const ContractNest &n, const ContractPlan &p, int *smem_bytes, int *tmem_cols);
+cudaError_t launch_tc_contraction(const ContractNest &n, const ContractPlan &p, int carveout, cudaStream_t s);
 cudaError_t launch_contraction(const ContractNest &n, const ContractPlan &p, int carveout_pct,
                                int32_t *coverage_counts, cudaStream_t s);
 

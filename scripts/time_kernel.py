@@ -21,11 +21,12 @@ def main():
     ap.add_argument("--tsteps", type=int, default=0)
     ap.add_argument("--iters", type=int, default=20)
     ap.add_argument("--split", type=int, default=50)
+    ap.add_argument("--engine", type=int, default=0)
     a = ap.parse_args()
     dims = [int(x) for x in a.dims.split(",")]
     tiles = [int(x) for x in a.tiles.split(",")]
     d = E.desc_builtin(a.kind, dims, tsteps=a.tsteps)
-    d.set_exec(split_pct=a.split)
+    d.set_exec(split_pct=a.split, engine=a.engine)
     bufs = [torch.rand(d.buffer_elems(i), device="cuda") * 2 - 1 for i in range(d.num_buffers)]
     if a.kind == "ccsd_t_d1":
         bufs[0].zero_()
