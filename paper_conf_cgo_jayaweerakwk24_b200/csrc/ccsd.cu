@@ -17,6 +17,7 @@
 
 #include <algorithm>
 #include <cstdint>
+#include <cstdlib>
 
 namespace eatss {
 
@@ -193,8 +194,105 @@ __global__ void __launch_bounds__(RM * RN >= 32 ? 512 : 1024) ccsd_d1_kernel(con
     }
 }
 
+#include "ccsd_fast.cuh"
+
 // ------------------------------------------------------------------ planning / launch
 static inline int64_t cdiv6(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+struct CcsdFastPlan {
+    bool ok = false;
+    int rm, rn, vec, bx, by, rtp, ctp, S, smem, kst, t3s_off;
+};
+
+static CcsdFastPlan plan_ccsd_fast(const int64_t *dims, const int *T, int Rt, int Ct) {
+    CcsdFastPlan f;
+    f.vec = (dims[5] % 4 == 0 && T[5] % 4 == 0) ? 4 : 1;
+    struct MT { int rm, rn; };
+    const MT c4[] = {{1, 4}, {2, 4}, {4, 4}, {4, 8}, {8, 8}};
+    const MT c1[] = {{1, 1}, {1, 2}, {2, 2}, {2, 4}, {4, 4}, {4, 8}, {8, 8}};
+    const MT *cand = f.vec == 4 ? c4 : c1;
+    const int nc = f.vec == 4 ? 5 : 7;
+    const int64_t want = cdiv6((int64_t)Rt * Ct, 512);
+    int pick = 0;
+    for (int c = 0; c < nc; c++) {
+        if (c > 0 && (cand[c].rm > Rt || cand[c].rn > ((Ct + f.vec - 1) / f.vec) * f.vec)) continue;
+        pick = c;
+        if (cand[c].rm * cand[c].rn >= want) break;
+    }
+    f.rm = cand[pick].rm;
+    f.rn = cand[pick].rn;
+    const int maxt = f.rm * f.rn >= 32 ? 512 : 1024;
+    const int64_t by = cdiv6(Rt, f.rm), bx = cdiv6(Ct, f.rn);
+    if (by * bx > maxt) return f;
+    f.by = (int)by;
+    f.bx = (int)bx;
+    f.rtp = ((Rt + 3) / 4) * 4 + (f.rm < 4 ? 0 : 0);
+    f.ctp = ((Ct + 3) / 4) * 4;
+    f.S = 3;
+    int group = std::max(1, (16 + T[6] - 1) / T[6]);
+    if (const char *e = getenv("EATSS_CCSD_GROUP")) group = std::max(1, atoi(e));
+    const bool want_prefetch = !(getenv("EATSS_CCSD_NOPREFETCH") && atoi(getenv("EATSS_CCSD_NOPREFETCH")));
+    auto layout = [&](int kst, bool pre, int64_t *bytes, int *t3s_off) {
+        const int64_t ring = (int64_t)f.S * kst * (f.rtp + f.ctp);
+        const int64_t tab = ((ring + 1) & ~1LL);
+        const int64_t t3s = ((tab + (int64_t)Rt * 4 + (int64_t)Ct * 3 + 3) & ~3LL);
+        *t3s_off = pre ? (int)t3s : -1;
+        *bytes = (pre ? t3s + (int64_t)Rt * Ct : t3s) * 4;
+    };
+    f.t3s_off = -1;
+    for (int g = group; g >= 1 && want_prefetch; g--) {
+        const int kst = (int)std::min<int64_t>((int64_t)T[6] * g, dims[6]);
+        int64_t bytes;
+        int off;
+        layout(kst, true, &bytes, &off);
+        if (bytes <= 227 * 1024) {
+            f.kst = kst;
+            f.t3s_off = off;
+            f.smem = (int)bytes;
+            f.ok = true;
+            return f;
+        }
+    }
+    f.kst = (int)std::min<int64_t>((int64_t)T[6] * group, dims[6]);
+    int64_t bytes;
+    int off;
+    layout(f.kst, false, &bytes, &off);
+    if (bytes > 227 * 1024) return f;
+    f.smem = (int)bytes;
+    f.ok = true;
+    return f;
+}
+
+template <int RM, int RN, int V>
+static cudaError_t ccsd_fast_launch(const CcsdFastArgs &a, const CcsdFastPlan &f, int64_t gx, int64_t gy,
+                                    int carveout, cudaStream_t s) {
+    auto k = ccsd_fast_kernel<RM, RN, V>;
+    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, f.smem);
+    if (e != cudaSuccess) return e;
+    cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, std::max(carveout, 50));
+    k<<<dim3((unsigned)gx, (unsigned)gy), dim3(f.bx, f.by), f.smem, s>>>(a);
+    return cudaGetLastError();
+}
+
+static cudaError_t ccsd_fast_dispatch(const CcsdFastArgs &a, const CcsdFastPlan &f, int64_t gx, int64_t gy,
+                                      int cv, cudaStream_t s) {
+    const int key = f.vec * 10000 + f.rm * 100 + f.rn;
+    switch (key) {
+        case 40104: return ccsd_fast_launch<1, 4, 4>(a, f, gx, gy, cv, s);
+        case 40204: return ccsd_fast_launch<2, 4, 4>(a, f, gx, gy, cv, s);
+        case 40404: return ccsd_fast_launch<4, 4, 4>(a, f, gx, gy, cv, s);
+        case 40408: return ccsd_fast_launch<4, 8, 4>(a, f, gx, gy, cv, s);
+        case 40808: return ccsd_fast_launch<8, 8, 4>(a, f, gx, gy, cv, s);
+        case 10101: return ccsd_fast_launch<1, 1, 1>(a, f, gx, gy, cv, s);
+        case 10102: return ccsd_fast_launch<1, 2, 1>(a, f, gx, gy, cv, s);
+        case 10202: return ccsd_fast_launch<2, 2, 1>(a, f, gx, gy, cv, s);
+        case 10204: return ccsd_fast_launch<2, 4, 1>(a, f, gx, gy, cv, s);
+        case 10404: return ccsd_fast_launch<4, 4, 1>(a, f, gx, gy, cv, s);
+        case 10408: return ccsd_fast_launch<4, 8, 1>(a, f, gx, gy, cv, s);
+        case 10808: return ccsd_fast_launch<8, 8, 1>(a, f, gx, gy, cv, s);
+    }
+    return cudaErrorInvalidConfiguration;
+}
 
 struct CcsdPlan {
     int T[7];
@@ -274,6 +372,22 @@ cudaError_t launch_ccsd_d1(float *t3, const float *t2, const float *v2, const in
     d2[0] = h3_count;
     CcsdPlan p = plan_ccsd(d2, tiles);
     if (p.gy > 65535 || p.gx > 2147483647LL) return cudaErrorInvalidConfiguration;
+    if (!counts && !(getenv("EATSS_CCSD_SLOW") && atoi(getenv("EATSS_CCSD_SLOW")))) {
+        CcsdFastPlan f = plan_ccsd_fast(d2, p.T, p.Rt, p.Ct);
+        if (f.ok) {
+            CcsdFastArgs a;
+            a.t3 = t3; a.t2 = t2; a.v2 = v2;
+            a.H3 = h3_begin + h3_count; a.H2 = dims[1]; a.H1 = dims[2]; a.P6 = dims[3]; a.P5 = dims[4];
+            a.P4 = dims[5]; a.H7 = dims[6];
+            for (int i = 0; i < 7; i++) a.T[i] = p.T[i];
+            a.nt_h1 = (int)cdiv6(dims[2], p.T[2]); a.nt_p5 = (int)cdiv6(dims[4], p.T[4]);
+            a.nt_p4 = (int)cdiv6(dims[5], p.T[5]); a.nt_h2 = (int)cdiv6(dims[1], p.T[1]);
+            a.nt_p6 = (int)cdiv6(dims[3], p.T[3]);
+            a.Rt = p.Rt; a.Ct = p.Ct; a.rtp = f.rtp; a.ctp = f.ctp; a.S = f.S; a.kst = f.kst; a.t3s_off = f.t3s_off;
+            a.h3_off = h3_begin;
+            return ccsd_fast_dispatch(a, f, p.gx, p.gy, carveout, s);
+        }
+    }
     if (p.smem > 227 * 1024) return cudaErrorInvalidConfiguration;
     CcsdArgs a;
     a.t3 = t3; a.t2 = t2; a.v2 = v2;
