@@ -1,0 +1,90 @@
+#!/usr/bin/env python
+"""Summarise a sweep JSONL (harness/sweep.py): performance- vs energy-optimal tiles.
+
+    python harness/report.py run.jsonl [--json out.json]
+
+Reports (P:225 energy = P_avg * t; P:231-234 PPW = FLOP/s / W = FLOP/J):
+  * the performance-optimal variant (max TFLOP/s) and the energy-optimal one (min J/run
+    == max GFLOP/s/W) among variants that passed the exactness check;
+  * whether they differ and by how much PPW differs, against the anchor-estimated noise
+    (spread of the repeated default / EATSS anchors);
+  * where the EATSS pick and the default 32^3 tile rank, and the share of variants that
+    beat the default (the paper: 15% for gemm on GA100).
+"""
+import argparse
+import json
+import statistics
+
+import numpy as np
+
+
+def load(path):
+    meta, var, anc = None, [], {"anchor_default": [], "anchor_eatss": []}
+    for line in open(path):
+        r = json.loads(line)
+        k = r.get("kind")
+        if k == "meta":
+            meta = meta or r
+        elif k == "variant":
+            var.append(r)
+        elif k in anc:
+            anc[k].append(r)
+    return meta, var, anc
+
+
+def summarise(path):
+    meta, var, anc = load(path)
+    ok = [r for r in var if r.get("status") == 0 and r.get("exact", True) and (r.get("joules") or 0) > 0]
+    bad = [r for r in var if not r.get("exact", True)]
+    out = {"file": path, "variants": len(var), "measured_ok": len(ok), "inexact": len(bad),
+           "eatss_tile": meta.get("eatss_tile") if meta else None, "nvml_update_ms": meta.get("nvml_update_ms") if meta else None}
+    if not ok:
+        return out
+    perf = max(ok, key=lambda r: r["tflops"])
+    energy = min(ok, key=lambda r: r["joules"])
+    ppw = sorted(ok, key=lambda r: -r["gflops_per_watt"])
+    out["perf_optimal"] = {k: perf[k] for k in ("tile", "tflops", "joules", "watts", "gflops_per_watt", "ms")}
+    out["energy_optimal"] = {k: energy[k] for k in ("tile", "tflops", "joules", "watts", "gflops_per_watt", "ms")}
+    out["energy_optimal_differs"] = perf["tile"] != energy["tile"]
+    out["ppw_gain_energy_vs_perf_optimal"] = energy["gflops_per_watt"] / perf["gflops_per_watt"]
+    for name, key in (("default", "anchor_default"), ("eatss", "anchor_eatss")):
+        a = [r for r in anc[key] if r.get("status") == 0 and (r.get("joules") or 0) > 0]
+        if a:
+            p = [r["gflops_per_watt"] for r in a]
+            t = [r["tflops"] for r in a]
+            out[f"anchor_{name}"] = {"tile": a[0]["tile"], "n": len(a), "ppw_median": statistics.median(p),
+                                     "ppw_rel_spread": (max(p) - min(p)) / statistics.median(p),
+                                     "tflops_median": statistics.median(t),
+                                     "tflops_rel_spread": (max(t) - min(t)) / statistics.median(t)}
+    noise = max([out.get(f"anchor_{n}", {}).get("ppw_rel_spread", 0) for n in ("default", "eatss")] or [0])
+    out["ppw_noise_rel"] = noise
+    out["finding_energy_beats_perf_on_ppw"] = bool(out["energy_optimal_differs"] and
+                                                   out["ppw_gain_energy_vs_perf_optimal"] - 1 > noise)
+    tiles_by_ppw = [tuple(r["tile"]) for r in ppw]
+    tiles_by_perf = [tuple(r["tile"]) for r in sorted(ok, key=lambda r: -r["tflops"])]
+    for name, key in (("eatss", "eatss_tile"),):
+        t = tuple(meta.get(key) or ())
+        if t in tiles_by_ppw:
+            out[f"{name}_rank_ppw"] = tiles_by_ppw.index(t) + 1
+            out[f"{name}_rank_perf"] = tiles_by_perf.index(t) + 1
+    d = out.get("anchor_default")
+    if d:
+        out["share_beating_default_perf"] = float(np.mean([r["tflops"] > d["tflops_median"] for r in ok]))
+        out["share_beating_default_ppw"] = float(np.mean([r["gflops_per_watt"] > d["ppw_median"] for r in ok]))
+    out["top5_ppw"] = [{"tile": r["tile"], "gflops_per_watt": r["gflops_per_watt"], "tflops": r["tflops"],
+                        "watts": r["watts"]} for r in ppw[:5]]
+    out["top5_perf"] = [{"tile": r["tile"], "gflops_per_watt": r["gflops_per_watt"], "tflops": r["tflops"],
+                         "watts": r["watts"]} for r in sorted(ok, key=lambda r: -r["tflops"])[:5]]
+    return out
+
+
+if __name__ == "__main__":
+    ap = argparse.ArgumentParser()
+    ap.add_argument("path")
+    ap.add_argument("--json", default="")
+    a = ap.parse_args()
+    s = summarise(a.path)
+    txt = json.dumps(s, indent=1)
+    print(txt)
+    if a.json:
+        open(a.json, "w").write(txt)

@@ -156,21 +156,69 @@ extern "C" eatss_status eatss_sweep(const eatss_kernel_desc *d, const int64_t *v
         cudaEventSynchronize(ev1);
         float ms1 = 0;
         cudaEventElapsedTime(&ms1, ev0, ev1);
-        const int64_t runs = std::max<int64_t>(1, (int64_t)std::ceil(min_window_s * 1e3 / std::max(ms1, 1e-3f)));
+        // The NVML energy counter updates in steps (~100 ms on B200, calibrated by the
+        // harness), so the window is ALIGNED to counter updates: the device is kept busy
+        // with chunks of runs; the window opens at one update and closes at the first
+        // update after min_window_s.  P_avg = dE / dt over that window, and the
+        // energy per run = P_avg * t_run with t_run from CUDA events inside the window.
+        const int64_t chunk = std::max<int64_t>(1, (int64_t)std::ceil(10.0 / std::max(ms1, 1e-3f)));
+        constexpr int Q = 4;  // chunk events in flight (3 queued ahead)
+        cudaEvent_t cev[Q];
+        for (int i = 0; i < Q; i++) cudaEventCreateWithFlags(&cev[i], cudaEventDisableTiming);
+        int64_t launched = 0, inflight = 0, head = 0;
+        auto launch_chunk = [&]() {
+            for (int64_t k = 0; k < chunk && st == EATSS_OK; k++) st = eatss_run(d, t, buffers, s);
+            cudaEventRecord(cev[head % Q], s);
+            head++;
+            inflight++;
+            launched += chunk;
+        };
+        auto pump = [&]() {
+            while (inflight > 0 && cudaEventQuery(cev[(head - inflight) % Q]) == cudaSuccess) inflight--;
+            while (inflight < Q - 1 && st == EATSS_OK) launch_chunk();
+        };
+        using clk = std::chrono::steady_clock;
         Sampler smp;
-        unsigned long long e0 = 0, e1 = 0;
+        unsigned long long ea = 0, eb = 0, cur = 0;
+        clk::time_point ta, tb;
+        int64_t runs_a = 0, runs_b = 0;
+        pump();
         if (have_nvml) {
             smp.start(h);
-            nvml().energy(h, &e0);
+            nvml().energy(h, &cur);
+            const unsigned long long start = cur;
+            const auto t_guard = clk::now();
+            while (cur == start && st == EATSS_OK &&
+                   std::chrono::duration<double>(clk::now() - t_guard).count() < 2.0) {
+                pump();
+                std::this_thread::sleep_for(std::chrono::microseconds(200));
+                nvml().energy(h, &cur);
+            }
+            ea = cur;
         }
-        cudaEventRecord(ev0, s);
-        for (int64_t k = 0; k < runs && st == EATSS_OK; k++) st = eatss_run(d, t, buffers, s);
+        ta = clk::now();
+        cudaEventRecord(ev0, s);  // start of the timed runs (launched from here on)
+        runs_a = launched;
+        while (st == EATSS_OK) {
+            pump();
+            const double el = std::chrono::duration<double>(clk::now() - ta).count();
+            if (el >= min_window_s) {
+                if (!have_nvml) break;
+                nvml().energy(h, &cur);
+                if (cur != ea && cur != eb) {
+                    if (eb == 0) eb = cur;  // first update after the minimum window closes it
+                }
+                if (eb != 0) break;
+                if (el > min_window_s + 2.0) break;  // counter stalled: give up on energy
+            }
+            std::this_thread::sleep_for(std::chrono::microseconds(200));
+        }
+        tb = clk::now();
+        runs_b = launched;
         cudaEventRecord(ev1, s);
         cudaError_t se = cudaEventSynchronize(ev1);
-        if (have_nvml) {
-            nvml().energy(h, &e1);
-            smp.finish();
-        }
+        if (have_nvml) smp.finish();
+        for (int i = 0; i < Q; i++) cudaEventDestroy(cev[i]);
         if (st != EATSS_OK || se != cudaSuccess) {
             r.status = st != EATSS_OK ? st : EATSS_E_CUDA;
             cudaGetLastError();
@@ -178,16 +226,18 @@ extern "C" eatss_status eatss_sweep(const eatss_kernel_desc *d, const int64_t *v
         }
         float ms = 0;
         cudaEventElapsedTime(&ms, ev0, ev1);
+        const int64_t runs = std::max<int64_t>(1, runs_b - runs_a);
         r.runs = runs;
         r.ms_per_run = ms / runs;
         r.tflops = flops / (r.ms_per_run * 1e-3) / 1e12;
-        if (have_nvml && e1 > e0) {
-            r.joules_per_run = (double)(e1 - e0) * 1e-3 / runs;
-            r.avg_watts = r.joules_per_run / (r.ms_per_run * 1e-3);
+        const double win_s = std::chrono::duration<double>(tb - ta).count();
+        if (have_nvml && eb > ea && win_s > 0) {
+            r.avg_watts = (double)(eb - ea) * 1e-3 / win_s;
+            r.joules_per_run = r.avg_watts * r.ms_per_run * 1e-3;
             r.gflops_per_watt = flops / r.joules_per_run / 1e9;  // FLOP/J == (FLOP/s)/W
         }
         r.sm_mhz_median = median(smp.mhz);
-        r.status = have_nvml ? EATSS_OK : EATSS_E_NVML;
+        r.status = (have_nvml && eb > ea) ? EATSS_OK : EATSS_E_NVML;
     }
     cudaEventDestroy(ev0);
     cudaEventDestroy(ev1);

@@ -1,6 +1,3 @@
 cd $GRAFT_REPO_ROOT
-timeout 600 python -m pytest tests/test_gpu_parity.py -q -k "ccsd" --timeout 300 -p no:cacheprovider 2>&1 | tail -2
-T="timeout 120 python scripts/time_kernel.py ccsd_t_d1 48"
-$T 4,4,4,4,4,32,4 --iters 3; EATSS_CCSD_GROUP=2 $T 4,4,4,4,4,32,4 --iters 3; EATSS_CCSD_GROUP=1 $T 4,4,4,4,4,32,4 --iters 3
-EATSS_CCSD_NOPREFETCH=1 $T 4,4,4,4,4,32,4 --iters 3
-$T 8,4,4,4,4,16,8 --iters 3
+timeout 900 python harness/sweep.py --limit 60 --window 0.5 --out gpurun_out/sweep_cal2.jsonl 2>&1 | tail -2
+python harness/report.py gpurun_out/sweep_cal2.jsonl | python -c "import json,sys; d=json.load(sys.stdin); [print(k, d.get(k)) for k in ['measured_ok','perf_optimal','energy_optimal','anchor_default','anchor_eatss','ppw_noise_rel','finding_energy_beats_perf_on_ppw','eatss_rank_ppw','eatss_rank_perf']]"
