@@ -1,0 +1,274 @@
+#!/usr/bin/env python
+"""Multi-GPU runner for the sharded configs (BASELINE configs 3 and 5).
+
+    torchrun --nproc-per-node G --master-addr 127.0.0.1 harness/multigpu.py --kind 3mm [--n 4000]
+
+One process per GPU, NCCL over NVLink.  The paper is single-GPU; the north star
+partitions each problem:
+  * gemm / 2mm / syrk -- independent row blocks of the output (boundaries are multiples
+    of Ti, so every element sees exactly the 1-GPU operation sequence: bit-equal);
+  * 3mm -- E = A*B and F = C*D row-sharded, ONE exchange (all_gather of F), then
+    G = E*F row-sharded: the only data collective of the path;
+  * ccsd_t_d1 -- h3 slabs (t2 replicated, v2 sliced by h3, no reduction: h7 is local).
+Timing is the device time of the slowest rank (barrier + synchronize on both sides);
+energy is the sum of the ranks' NVML counters; parity is checked per shard on sampled
+entries against the fp64 oracle and reduced to rank 0.
+
+The sharding / exchange logic (``plan``, ``run_shard``) is backend-agnostic so the CPU
+test suite exercises it with the oracle under a gloo process group.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+
+def shard_rows(M: int, G: int, Ti: int, rank: int):
+    """Row range [r0, r1) of `rank`: whole i-tiles, split as evenly as possible."""
+    nt = -(-M // Ti)
+    t0, t1 = (rank * nt) // G, ((rank + 1) * nt) // G
+    return min(M, t0 * Ti), min(M, t1 * Ti)
+
+
+def dims_of(kind: str, n: int):
+    return {"gemm": (n, n, n), "2mm": (n, n, n, n), "3mm": (n, n, n, n, n), "syrk": (n, n),
+            "ccsd_t_d1": (n,) * 7}[kind]
+
+
+def make_inputs(kind: str, dims, seed0: int = 0, small_int: bool = False):
+    """Full host inputs (identical on every rank: same seeded generator)."""
+    import synth
+    gen = (lambda s, seed: synth.small_int(s, seed, -1, 1)) if small_int else (lambda s, seed: synth.uniform(s, seed))
+    if kind == "gemm":
+        ni, nj, nk = dims
+        return {"A": gen((ni, nk), seed0), "B": gen((nk, nj), seed0 + 1), "C": gen((ni, nj), seed0 + 2)}
+    if kind == "2mm":
+        ni, nj, nk, nl = dims
+        return {"A": gen((ni, nk), seed0), "B": gen((nk, nj), seed0 + 1), "C": gen((nj, nl), seed0 + 2),
+                "D": gen((ni, nl), seed0 + 3)}
+    if kind == "3mm":
+        ni, nj, nk, nl, nm = dims
+        return {"A": gen((ni, nk), seed0), "B": gen((nk, nj), seed0 + 1), "C": gen((nj, nm), seed0 + 2),
+                "D": gen((nm, nl), seed0 + 3)}
+    if kind == "syrk":
+        ni, nj = dims
+        return {"A": gen((ni, nj), seed0), "C": gen((ni, ni), seed0 + 1)}
+    if kind == "ccsd_t_d1":
+        H3, H2, H1, P6, P5, P4, H7 = dims
+        return {"t2": gen((H7, P4, P5, H1), seed0), "v2": gen((H3, H2, P6, H7), seed0 + 1)}
+    raise ValueError(kind)
+
+
+def run_shard(kind, dims, tiles, rank, world, X, backend, alpha=1.5, beta=1.2):
+    """Compute this rank's shard.  `backend` provides:
+         gemm(alpha, beta, C, A, B, init_zero)  -> C (row block)   [C := beta*C + alpha*A*B]
+         syrk_rows(alpha, beta, Crows, Afull, r0) -> Crows   [rows r0.. of a*A*A^T + b*C]
+         ccsd(t3slab, t2, v2slab) -> t3slab
+         all_gather_rows(local, total_rows, row_ranges) -> full
+       Returns (outputs dict, row range)."""
+    Ti = tiles[0]
+    if kind == "gemm":
+        ni = dims[0]
+        r0, r1 = shard_rows(ni, world, Ti, rank)
+        C = backend.gemm(alpha, beta, X["C"][r0:r1], X["A"][r0:r1], X["B"], False)
+        return {"C": C}, (r0, r1)
+    if kind == "2mm":
+        ni, nj, nk, nl = dims
+        r0, r1 = shard_rows(ni, world, Ti, rank)
+        tmp = backend.gemm(alpha, 0.0, np.zeros((r1 - r0, nj), np.float32), X["A"][r0:r1], X["B"], True)
+        D = backend.gemm(1.0, beta, X["D"][r0:r1], tmp, X["C"], False)
+        return {"tmp": tmp, "D": D}, (r0, r1)
+    if kind == "3mm":
+        ni, nj, nk, nl, nm = dims
+        r0, r1 = shard_rows(ni, world, Ti, rank)
+        f0, f1 = shard_rows(nj, world, Ti, rank)
+        E = backend.gemm(1.0, 0.0, np.zeros((r1 - r0, nj), np.float32), X["A"][r0:r1], X["B"], True)
+        Floc = backend.gemm(1.0, 0.0, np.zeros((f1 - f0, nl), np.float32), X["C"][f0:f1], X["D"], True)
+        ranges = [shard_rows(nj, world, Ti, r) for r in range(world)]
+        F = backend.all_gather_rows(Floc, nj, ranges)  # the one exchange step (NCCL all_gather)
+        G = backend.gemm(1.0, 0.0, np.zeros((r1 - r0, nl), np.float32), E, F, True)
+        return {"E": E, "F": F, "G": G}, (r0, r1)
+    if kind == "syrk":
+        ni, nj = dims
+        r0, r1 = shard_rows(ni, world, Ti, rank)
+        C = backend.syrk_rows(alpha, beta, X["C"][r0:r1], X["A"], r0)
+        return {"C": C}, (r0, r1)
+    if kind == "ccsd_t_d1":
+        H3 = dims[0]
+        h0, h1 = shard_rows(H3, world, tiles[0], rank)
+        t3 = backend.ccsd(X["t3"][h0:h1], X["t2"], X["v2"][h0:h1])
+        return {"t3": t3}, (h0, h1)
+    raise ValueError(kind)
+
+
+# ------------------------------------------------------------------ GPU backend (libeatss)
+class CudaBackend:
+    """Shard compute through libeatss.so; arrays are host numpy in / device tensors inside."""
+
+    def __init__(self, dev, tiles, dist=None, timing=False):
+        import torch
+        import paper_conf_cgo_jayaweerakwk24_b200 as E
+        self.torch, self.E, self.dev, self.tiles, self.dist = torch, E, dev, tiles, dist
+
+    def _t(self, x):
+        if isinstance(x, np.ndarray):
+            return self.torch.from_numpy(np.ascontiguousarray(x)).to(self.dev)
+        return x
+
+    def gemm(self, alpha, beta, C, A, B, init_zero):
+        C, A, B = self._t(C), self._t(A), self._t(B)
+        M, K = A.shape
+        N = B.shape[1]
+        d = self.E.desc_builtin("gemm", (M, N, K))
+        d.set_scalars(alpha, 0.0 if init_zero else beta)
+        if init_zero:
+            C.zero_()
+        self.E.run(d, self.tiles, [C, A, B])
+        return C
+
+    def syrk_rows(self, alpha, beta, Crows, Afull, r0):
+        Crows, Afull = self._t(Crows), self._t(Afull)
+        ni, nj = Afull.shape
+        rows = Crows.shape[0]
+        d = self.E.desc_builtin("syrk", (ni, nj, r0, rows))  # rows [r0, r0+rows) of C = a*A*A^T + b*C
+        d.set_scalars(alpha, beta)
+        self.E.run(d, self.tiles, [Crows, Afull])
+        return Crows
+
+    def ccsd(self, t3, t2, v2):
+        t3, t2, v2 = self._t(t3), self._t(t2), self._t(v2)
+        H3 = v2.shape[0]
+        H7, P4, P5, H1 = t2.shape
+        _, H2, P6, _ = v2.shape
+        d = self.E.desc_builtin("ccsd_t_d1", (H3, H2, H1, P6, P5, P4, H7))
+        self.E.run(d, self.tiles, [t3, t2, v2])
+        return t3
+
+    def all_gather_rows(self, local, total_rows, ranges):
+        torch = self.torch
+        local = self._t(local)
+        maxr = max(r1 - r0 for r0, r1 in ranges)
+        buf = torch.zeros((maxr,) + tuple(local.shape[1:]), dtype=local.dtype, device=self.dev)
+        buf[: local.shape[0]] = local
+        out = torch.empty((len(ranges) * maxr,) + tuple(local.shape[1:]), dtype=local.dtype, device=self.dev)
+        self.dist.all_gather_into_tensor(out, buf)
+        parts = [out[i * maxr: i * maxr + (r1 - r0)] for i, (r0, r1) in enumerate(ranges)]
+        return torch.cat(parts, 0)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--kind", default="3mm", choices=["gemm", "2mm", "3mm", "syrk", "ccsd_t_d1"])
+    ap.add_argument("--n", type=int, default=0)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--split", type=int, default=50)
+    a = ap.parse_args()
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_cgo_jayaweerakwk24_b200 as E
+    from oracle import numeric as O
+
+    ws, rank, local = int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("RANK", 0)), int(os.environ.get("LOCAL_RANK", 0))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if ws > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    n = a.n or (48 if a.kind == "ccsd_t_d1" else 4000)
+    dims = dims_of(a.kind, n)
+    d_full = E.desc_builtin(a.kind, dims)
+    waf = 4 if a.kind == "ccsd_t_d1" else 16
+    tiles, _ = E.select_tiles(d_full, E.gpu_params_query(local), a.split, waf)
+    X = make_inputs(a.kind, dims)
+    if a.kind == "ccsd_t_d1":
+        X["t3"] = np.zeros((n,) * 6, np.float32)
+    be = CudaBackend(dev, tiles, dist if ws > 1 else None)
+
+    def once():
+        return run_shard(a.kind, dims, tiles, rank, ws, X, be)
+
+    for _ in range(a.warmup):
+        out, rr = once()
+    torch.cuda.synchronize()
+    if ws > 1:
+        dist.barrier()
+    s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    mj0 = E.energy_mj(local)
+    s.record()
+    for _ in range(a.steps):
+        out, rr = once()
+    e.record()
+    torch.cuda.synchronize()
+    mj1 = E.energy_mj(local)
+    ms = s.elapsed_time(e) / a.steps
+    # parity on sampled entries of this shard (fp32 tolerance vs fp64 oracle)
+    err = parity_sample(a.kind, dims, X, out, rr, O)
+    v = torch.tensor([ms, (mj1 - mj0) / 1e3 / a.steps, err], dtype=torch.float64, device=dev)
+    if ws > 1:
+        mx = v.clone(); dist.all_reduce(mx, op=dist.ReduceOp.MAX)
+        sm = v.clone(); dist.all_reduce(sm, op=dist.ReduceOp.SUM)
+        ms_max, joules, err_max = mx[0].item(), sm[1].item(), mx[2].item()
+    else:
+        ms_max, joules, err_max = ms, v[1].item(), err
+    if rank == 0:
+        flops = d_full.flops
+        print(json.dumps({"kind": a.kind, "dims": dims, "tiles": list(tiles), "gpus": ws, "ms": ms_max,
+                          "tflops": flops / (ms_max * 1e-3) / 1e12, "joules": joules,
+                          "gflops_per_watt": flops / joules / 1e9 if joules > 0 else None,
+                          "parity_rel_err_max": err_max, "exchange": "all_gather(F)" if a.kind == "3mm" else None}))
+    if ws > 1:
+        dist.destroy_process_group()
+
+
+def parity_sample(kind, dims, X, out, rr, O, k=256, seed=5):
+    """Normwise relative error of sampled shard entries vs exact fp64 dots."""
+    g = np.random.default_rng(seed)
+    r0, r1 = rr
+    if r1 <= r0:
+        return 0.0
+    if kind in ("gemm",):
+        C = out["C"].double().cpu().numpy()
+        ii = g.integers(0, r1 - r0, k); jj = g.integers(0, C.shape[1], k)
+        ref = O.gemm_entries(ii + r0, jj, X["C"], X["A"], X["B"], 1.5, 1.2)
+        return O.normwise_rel_err(C[ii, jj], ref)
+    if kind == "3mm":
+        G = out["G"].double().cpu().numpy()
+        ii = g.integers(0, r1 - r0, k); jj = g.integers(0, G.shape[1], k)
+        A = X["A"].astype(np.float64); B = X["B"].astype(np.float64)
+        F = X["C"].astype(np.float64) @ X["D"].astype(np.float64)
+        ref = np.einsum("ij,ji->i", (A[ii + r0] @ B), F[:, jj])
+        return O.normwise_rel_err(G[ii, jj], ref)
+    if kind == "2mm":
+        D = out["D"].double().cpu().numpy()
+        ii = g.integers(0, r1 - r0, k); jj = g.integers(0, D.shape[1], k)
+        tmp = 1.5 * (X["A"][ii + r0].astype(np.float64) @ X["B"].astype(np.float64))
+        ref = np.einsum("ij,ji->i", tmp, X["C"].astype(np.float64)[:, jj]) + 1.2 * X["D"][ii + r0, jj]
+        return O.normwise_rel_err(D[ii, jj], ref)
+    if kind == "syrk":
+        C = out["C"].double().cpu().numpy()
+        ii = g.integers(0, r1 - r0, k); jj = g.integers(0, C.shape[1], k)
+        A = X["A"].astype(np.float64)
+        ref = 1.5 * np.einsum("ij,ij->i", A[ii + r0], A[jj]) + 1.2 * X["C"][ii + r0, jj]
+        return O.normwise_rel_err(C[ii, jj], ref)
+    if kind == "ccsd_t_d1":
+        t3 = out["t3"].reshape(-1)
+        n6 = t3.numel()
+        idx = g.integers(0, n6, 4096)
+        got = t3[__import__("torch").from_numpy(idx).to(t3.device)].double().cpu().numpy()
+        dims_s = (r1 - r0,) + tuple(dims[1:])
+        ref = O.ccsd_t_d1_entries(dims_s, idx, np.zeros(len(idx)), X["t2"], X["v2"][r0:r1])
+        return O.normwise_rel_err(got, ref)
+    return float("nan")
+
+
+if __name__ == "__main__":
+    main()

@@ -71,6 +71,8 @@ typedef enum { EATSS_F32 = 1, EATSS_F64 = 2 } eatss_dtype;
  *                   E := A*B; F := C*D; G := E*F
  *   EATSS_SYRK      dims (ni, nj)              buffers {C[ni][ni] (in/out), A[ni][nj]}
  *                   C := alpha*A*A^T + beta*C (full square, PolyBench 3.2)
+ *                   or dims (ni, nj, r0, rows): only rows [r0, r0+rows) of C (a row-block shard,
+ *                   SURVEY §8(e)); buffers {C rows x ni (in/out), the full A[ni][nj]}
  *   EATSS_JACOBI2D  dims (n), tsteps           buffers {A[n][n] (in/out), B[n][n] (in/out)}
  *                   tsteps x { B = 0.2*(5-point of A); A = B } on the interior (PolyBench 3.2)
  *   EATSS_HEAT3D    dims (n), tsteps           buffers {A[n][n][n] (in/out), B[n][n][n] (in/out)}

@@ -88,10 +88,11 @@ static eatss_status build(eatss_kernel_desc *d) {
             d->buffer_elems = {x[0] * x[1], x[0] * x[2], x[2] * x[1], x[1] * x[3],
                                x[1] * x[4], x[4] * x[3], x[0] * x[3]};
             break;
-        case EATSS_SYRK: {  // C A ; dims ni nj
-            d->nests = {N3(x[0], x[0], x[1], false,
+        case EATSS_SYRK: {  // C A ; dims (ni, nj) or (ni, nj, r0, rows): rows [r0, r0+rows) of C
+            const int64_t rows = x.size() == 4 ? x[3] : x[0];
+            d->nests = {N3(rows, x[0], x[1], false,
                            {R(0, {S(I), S(J)}, true), R(0, {S(I), S(J)}), R(1, {S(I), S(K)}), R(1, {S(J), S(K)})})};
-            d->buffer_elems = {x[0] * x[0], x[0] * x[1]};
+            d->buffer_elems = {rows * x[0], x[0] * x[1]};
             break;
         }
         case EATSS_JACOBI2D: {  // A B ; dims n ; interior extent n-2, time loop excluded
@@ -175,9 +176,12 @@ static std::vector<ContractNest> contraction_nests(const eatss_kernel_desc *d, v
             v.push_back(mk(x[1], x[3], x[4], b[4], x[4], b[5], x[3], false, b[3], x[3], 1.0, 0.0, true));
             v.push_back(mk(x[0], x[3], x[1], b[0], x[1], b[3], x[3], false, b[6], x[3], 1.0, 0.0, true));
             break;
-        case EATSS_SYRK:
-            v.push_back(mk(x[0], x[0], x[1], b[1], x[1], b[1], x[1], true, b[0], x[0], d->alpha, d->beta, false));
+        case EATSS_SYRK: {
+            const int64_t r0 = x.size() == 4 ? x[2] : 0, rows = x.size() == 4 ? x[3] : x[0];
+            const void *Ar = static_cast<const char *>(b[1]) + r0 * x[1] * (f64 ? 8 : 4);
+            v.push_back(mk(rows, x[0], x[1], Ar, x[1], b[1], x[1], true, b[0], x[0], d->alpha, d->beta, false));
             break;
+        }
         default:
             break;
     }
@@ -299,10 +303,13 @@ eatss_status eatss_desc_builtin(eatss_builtin k, const int64_t *dims, int ndims,
     const int want = kDimsPerBuiltin[k];
     std::vector<int64_t> dv;
     if (k == EATSS_CCSD_T_D1 && ndims == 1) dv.assign(7, dims[0]);
-    else if (ndims == want) dv.assign(dims, dims + ndims);
+    else if (ndims == want || (k == EATSS_SYRK && ndims == 4)) dv.assign(dims, dims + ndims);
     else return fail(EATSS_E_INVALID, "eatss_desc_builtin: wrong number of dims");
-    for (int64_t v : dv)
-        if (v <= 0) return fail(EATSS_E_INVALID, "eatss_desc_builtin: dims must be >= 1");
+    for (size_t i = 0; i < dv.size(); i++)
+        if (dv[i] <= 0 && !(k == EATSS_SYRK && i == 2 && dv[i] == 0))
+            return fail(EATSS_E_INVALID, "eatss_desc_builtin: dims must be >= 1");
+    if (k == EATSS_SYRK && dv.size() == 4 && dv[2] + dv[3] > dv[0])
+        return fail(EATSS_E_INVALID, "eatss_desc_builtin: syrk row block exceeds ni");
     if ((k == EATSS_JACOBI2D || k == EATSS_HEAT3D) && (dv[0] < 3 || tsteps < 0))
         return fail(EATSS_E_INVALID, "eatss_desc_builtin: stencils need n >= 3 and tsteps >= 0");
     if (k == EATSS_CCSD_T_D1 && dt != EATSS_F32)
@@ -346,7 +353,7 @@ double eatss_desc_flops(const eatss_kernel_desc *d) {
         case EATSS_2MM: return 2 * D(x[0]) * D(x[1]) * D(x[2]) + 2 * D(x[0]) * D(x[3]) * D(x[1]);
         case EATSS_3MM:
             return 2 * (D(x[0]) * D(x[1]) * D(x[2]) + D(x[1]) * D(x[3]) * D(x[4]) + D(x[0]) * D(x[3]) * D(x[1]));
-        case EATSS_SYRK: return 2 * D(x[0]) * D(x[0]) * D(x[1]);
+        case EATSS_SYRK: return 2 * D(x.size() == 4 ? x[3] : x[0]) * D(x[0]) * D(x[1]);
         case EATSS_JACOBI2D: return 5 * D(x[0] - 2) * D(x[0] - 2) * D(d->tsteps);
         case EATSS_HEAT3D: return 15 * D(x[0] - 2) * D(x[0] - 2) * D(x[0] - 2) * 2 * D(d->tsteps);
         case EATSS_CCSD_T_D1: return 2 * D(x[0]) * D(x[1]) * D(x[2]) * D(x[3]) * D(x[4]) * D(x[5]) * D(x[6]);
@@ -369,7 +376,7 @@ double eatss_desc_bytes(const eatss_kernel_desc *d) {
             for (int i = 0; i < 7; i++) s += D(d->buffer_elems[i]);
             return e * (s + D(d->buffer_elems[0]) + D(d->buffer_elems[3]));  // E, F re-read by G
         }
-        case EATSS_SYRK: return e * (D(x[0]) * D(x[1]) + 2 * D(x[0]) * D(x[0]));
+        case EATSS_SYRK: return e * (D(x[0]) * D(x[1]) + 2 * D(x.size() == 4 ? x[3] : x[0]) * D(x[0]));
         case EATSS_JACOBI2D:  // per sweep (no time tiling): read src + write dst; + final copy
             return e * 2 * D(x[0]) * D(x[0]) * (D(d->tsteps) + (d->tsteps > 0 ? 1 : 0));
         case EATSS_HEAT3D: return e * 2 * D(x[0]) * D(x[0]) * D(x[0]) * 2 * D(d->tsteps);
