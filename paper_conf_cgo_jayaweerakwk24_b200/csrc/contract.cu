@@ -533,15 +533,23 @@ ContractPlan plan_contraction(const ContractNest &n, const int64_t *tiles, int s
     p.smem_bytes = (int)(p.nbuf * ((p.a_smem ? a_bytes : 0) + (p.b_smem ? b_bytes : 0)));
     if (!p.stream) {
         // register-resident: stage both operand slices per k-tile through an S-stage cp.async ring
+        // The ring holds S stages of kst k-rows each; a k-tile of Tk rows is staged as
+        // ceil(Tk/kst) sub-stages (numerically identical: accumulators are resident and k
+        // stays ascending).  Default: the deepest ring (S = 3) whose footprint still lets two
+        // CTAs share an SM, halving kst until it fits; else one full-k-tile stage.
         const int64_t aip = ((p.Ti + 3) / 4) * 4, bjp = ((p.Tj + 3) / 4) * 4;
-        const int64_t stage_bytes = p.Tk * (aip + bjp) * esz;
-        int64_t s_fit = smem_limit / std::max<int64_t>(stage_bytes + 16, 1);
-        int want_s = 1;  // measured best for the EATSS tile with 2 co-resident CTAs (profiles/)
-        if (const char *e = getenv("EATSS_STAGES")) want_s = std::max(1, atoi(e));
-        const int64_t S = std::min<int64_t>(want_s, s_fit);
-        if (S >= 1 && !(getenv("EATSS_NO_STAGED") && atoi(getenv("EATSS_NO_STAGED")))) {
+        const int64_t half = smem_limit / 2 - 1024;
+        int64_t kst = p.Tk, S = 3;
+        while (kst > 1 && S * (kst * (aip + bjp) * esz + 16) > half) kst = (kst + 1) / 2;
+        if (S * (kst * (aip + bjp) * esz + 16) > half) { kst = p.Tk; S = 1; }
+        if (const char *e = getenv("EATSS_STAGES")) S = std::max(1, atoi(e));
+        if (const char *e = getenv("EATSS_KSUB")) kst = std::max<int64_t>(1, (p.Tk + atoi(e) - 1) / std::max(1, atoi(e)));
+        const int64_t stage_bytes = kst * (aip + bjp) * esz;
+        if (S * (stage_bytes + 16) > smem_limit) S = std::max<int64_t>(1, smem_limit / (stage_bytes + 16));
+        if (S * (stage_bytes + 16) <= smem_limit && !(getenv("EATSS_NO_STAGED") && atoi(getenv("EATSS_NO_STAGED")))) {
             p.staged = true;
             p.nbuf = (int)S;
+            p.kst = (int)kst;
             p.tkp = (int)aip;
             p.tjp = (int)bjp;
             p.a_smem = true;
@@ -666,7 +674,8 @@ static cudaError_t launch_typed(const ContractNest &n, const ContractPlan &p, in
     a.C = static_cast<T *>(n.C); a.ldc = n.ldc;
     a.alpha = (T)n.alpha; a.beta = (T)n.beta;
     a.init_zero = n.init_zero ? 1 : 0;
-    a.Ti = (int)p.Ti; a.Tj = (int)p.Tj; a.Tk = (int)p.Tk;
+    a.Ti = (int)p.Ti; a.Tj = (int)p.Tj;
+    a.Tk = p.staged ? p.kst : (int)p.Tk;  // the staged kernel walks k in ring stages of kst rows
     a.a_smem = p.a_smem; a.b_smem = p.b_smem; a.nbuf = p.nbuf;
     a.tkp = p.tkp; a.tjp = p.tjp;
     a.passes_i = p.passes_i; a.passes_j = p.passes_j;

@@ -32,6 +32,7 @@ struct ContractPlan {
     bool staged = false;  // resident fast path: both operand slices staged via cp.async ring (nbuf stages)
     bool a_smem = true, b_smem = false;
     int nbuf = 1;
+    int kst = 0;  // staged path: k-rows per ring stage
     int tkp = 0, tjp = 0;  // shared-memory pitches (elements)
     int smem_bytes = 0;
     int64_t grid_x = 1, grid_y = 1;

@@ -134,12 +134,14 @@ struct Args {
     int bjp;      // raw B row pitch (floats)
     uint32_t tmem_cols;
     int a_bulk;   // A rows by bulk copy (1) or by converter loads (0)
+    int R;        // stages per accumulator chunk
 };
 
 constexpr int KS = 8;            // k per stage = one tf32 MMA
 constexpr int NCONV = 8;         // converter warps (4..11): two per TMEM lane quarter
 constexpr int NTHREADS = (4 + NCONV) * 32;
 
+template <int NMT>  // MMA N (= Ti rounded up to 16), compile-time so the fp32 chunk sums stay in registers
 __global__ void __launch_bounds__(NTHREADS, 1) tc3_gemm_kernel(const Args p) {
     extern __shared__ __align__(1024) unsigned char smem[];
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -159,7 +161,9 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc3_gemm_kernel(const Args p) {
     uint64_t *opnd_full = empty + p.S;   // [2]
     uint64_t *opnd_empty = opnd_full + 2; // [2]
     uint64_t *acc_done = opnd_empty + 2;
-    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(acc_done + 1);
+    uint64_t *dfull = acc_done + 1;   // [2] accumulator chunk ready (MMA commit)
+    uint64_t *dempty = dfull + 2;     // [2] accumulator chunk drained (converter warps)
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(dempty + 2);
 
     if (warp == 2) {
         asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;\n" ::"r"(su32(tmem_slot)),
@@ -177,14 +181,23 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc3_gemm_kernel(const Args p) {
             mbar_init(opnd_empty + b, 1);
         }
         mbar_init(acc_done, 1);
+        for (int b = 0; b < 2; b++) {
+            mbar_init(dfull + b, 1);
+            mbar_init(dempty + b, NCONV);
+        }
         asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
     }
     fence_before();
     __syncthreads();
     fence_after();
     const uint32_t tmem = *tmem_slot;
-    // TMEM columns: [0, MB*NM) accumulators D; then 2 buffers x MB x 16 (8 hi + 8 lo) operand columns
-    const uint32_t acol0 = (uint32_t)(p.MB * p.NM);
+    // TMEM columns: 2 accumulator buffers [0, 2*MB*NM) (the k-loop is split into chunks of R
+    // stages accumulated in alternate buffers and summed in fp32 registers: the tensor core
+    // accumulates with truncation, so a single K=4000 accumulation drifts by ~K*2^-24);
+    // then 2 operand buffers x MB x 16 (8 hi + 8 lo) columns
+    const uint32_t acol0 = (uint32_t)(2 * p.MB * p.NM);
+    const int R = p.R;
+    const int nchunks = (nst + R - 1) / R;
     const bool bulk_b = (cols & 3) == 0;
     const bool a_bulk_enabled = p.a_bulk != 0;
 
@@ -214,20 +227,23 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc3_gemm_kernel(const Args p) {
             const uint32_t idesc = idesc_tf32(p.NM);
             for (int t = 0; t < nst; t++) {
                 const int b = t & 1;
+                const int ch = t / R, bd = ch & 1;
+                const bool first = (t % R) == 0;
+                if (first && ch >= 2) mbar_wait(dempty + bd, (unsigned)(((ch - 2) >> 1) & 1));
                 mbar_wait(opnd_full + b, (unsigned)((t >> 1) & 1));
                 fence_after();
                 const unsigned char *nhi = nside + (size_t)b * 2 * nbuf_bytes;
                 const uint64_t dhi = smem_desc(nhi, 128, 256), dlo = smem_desc(nhi + nbuf_bytes, 128, 256);
                 for (int mb = 0; mb < p.MB; mb++) {
-                    const uint32_t d = tmem + (uint32_t)(mb * p.NM);
+                    const uint32_t d = tmem + (uint32_t)((bd * p.MB + mb) * p.NM);
                     const uint32_t ahi = tmem + acol0 + (uint32_t)(b * p.MB * 16 + mb * 16), alo = ahi + 8;
-                    mma_tf32_ts(d, ahi, dhi, idesc, t > 0 ? 1u : 0u);
+                    mma_tf32_ts(d, ahi, dhi, idesc, first ? 0u : 1u);
                     mma_tf32_ts(d, ahi, dlo, idesc, 1u);
                     mma_tf32_ts(d, alo, dhi, idesc, 1u);
                 }
                 mma_commit(opnd_empty + b);  // operand buffer b may be overwritten once these MMAs finish
+                if ((t % R) == R - 1 || t == nst - 1) mma_commit(dfull + bd);  // chunk ready for draining
             }
-            mma_commit(acc_done);  // all MMAs of the tile
         }
     } else if (warp >= 4) {
         // ------------------------------------------------------------ converters
@@ -235,6 +251,37 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc3_gemm_kernel(const Args p) {
         const int q = warp & 3;       // TMEM lane quarter (warp id within its warpgroup)
         const int mg = c >> 2, ngroups = NCONV / 4;
         const int ctid = c * 32 + lane;
+        // fp32 register sums of the drained accumulator chunks: [my M-blocks][NM columns]
+        constexpr int MW = 64 / NMT;  // M-blocks per converter warp (host guarantees ceil(MB/2) <= MW)
+        float acc[MW][NMT];
+#pragma unroll
+        for (int m = 0; m < MW; m++)
+#pragma unroll
+            for (int x = 0; x < NMT; x++) acc[m][x] = 0.f;
+        int next_drain = 0;
+        auto drain = [&](int ch) {
+            const int bd = ch & 1;
+            mbar_wait(dfull + bd, (unsigned)((ch >> 1) & 1));
+            fence_after();
+#pragma unroll
+            for (int m = 0; m < MW; m++) {
+                const int mb = mg + m * ngroups;
+                if (mb < p.MB) {
+#pragma unroll
+                    for (int c0 = 0; c0 < NMT; c0 += 16) {
+                        uint32_t v[16];
+                        tmem_ld16(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)((bd * p.MB + mb) * NMT + c0), v);
+                        wait_ld();
+#pragma unroll
+                        for (int cc = 0; cc < 16; cc++) acc[m][c0 + cc] += __uint_as_float(v[cc]);
+                    }
+                }
+            }
+            fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(dempty + bd);
+        };
+        auto chunk_end = [&](int ch) { return min((ch + 1) * R, nst) - 1; };
         for (int t = 0; t < nst; t++) {
             const int s = t % p.S, b = t & 1;
             const int64_t k0 = (int64_t)t * KS;
@@ -279,25 +326,22 @@ __global__ void __launch_bounds__(NTHREADS, 1) tc3_gemm_kernel(const Args p) {
                 mbar_arrive(opnd_full + b);
                 mbar_arrive(empty + s);
             }
+            // drain every chunk whose last stage was fed at least one stage ago
+            while (next_drain < nchunks && chunk_end(next_drain) <= t - 1) drain(next_drain++);
         }
+        while (next_drain < nchunks) drain(next_drain++);
         // ------------------------------------------------------------ epilogue
-        mbar_wait(acc_done, 0u);
-        fence_after();
-        for (int mb = mg; mb < p.MB; mb += ngroups) {
-            const int jl = mb * 128 + q * 32 + lane;
-            for (int c0 = 0; c0 < p.NM; c0 += 16) {
-                uint32_t v[16];
-                tmem_ld16(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(mb * p.NM + c0), v);
-                wait_ld();
-                if (jl < cols) {
 #pragma unroll
-                    for (int cc = 0; cc < 16; cc++) {
-                        const int il = c0 + cc;
-                        if (il < rows) {
-                            float *cp = p.C + (i0 + il) * p.ldc + j0 + jl;
-                            const float o = p.init_zero ? 0.f : p.beta * *cp;
-                            *cp = fmaf(p.alpha, __uint_as_float(v[cc]), o);
-                        }
+        for (int m = 0; m < MW; m++) {
+            const int mb = mg + m * ngroups;
+            const int jl = mb * 128 + q * 32 + lane;
+            if (mb < p.MB && jl < cols) {
+#pragma unroll
+                for (int il = 0; il < NMT; il++) {
+                    if (il < rows) {
+                        float *cp = p.C + (i0 + il) * p.ldc + j0 + jl;
+                        const float o = p.init_zero ? 0.f : p.beta * *cp;
+                        *cp = fmaf(p.alpha, acc[m][il], o);
                     }
                 }
             }
@@ -329,11 +373,11 @@ static int tc_stages() {
 // Applicability + smem size of the tensor-core executor for a plan.
 bool tc_plan(const ContractNest &n, const ContractPlan &p, int *smem_bytes, int *tmem_cols) {
     if (n.f64 || n.transB) return false;
-    if (p.Ti > 256) return false;
     const int NM = (int)(((p.Ti + 15) / 16) * 16);
     const int MB = (int)((p.Tj + 127) / 128);
-    if (MB < 1 || MB > 16) return false;
-    const uint32_t cols = (uint32_t)(MB * NM + 2 * MB * 16);
+    if (NM > 64 || MB < 1) return false;
+    if (((MB + 1) / 2) * NM > 64) return false;  // fp32 chunk sums per converter thread
+    const uint32_t cols = (uint32_t)(2 * MB * NM + 2 * MB * 16);  // 2 accumulator + 2 operand buffers
     if (cols > 512) return false;
     if ((n.lda % 4) || (n.ldb % 4) || (reinterpret_cast<uintptr_t>(n.A) & 15) ||
         (reinterpret_cast<uintptr_t>(n.B) & 15))
@@ -341,7 +385,7 @@ bool tc_plan(const ContractNest &n, const ContractPlan &p, int *smem_bytes, int 
     const int bjp = (int)(((p.Tj + 3) / 4) * 4);
     const int S = tc_stages();
     const int64_t slot = (int64_t)(tc::KS * bjp + NM * tc::KS) * 4;
-    const int64_t bytes = ((S * slot + 127) & ~127LL) + 4 * NM * 32 + 8 * (2 * S + 5) + 16;
+    const int64_t bytes = ((S * slot + 127) & ~127LL) + 4 * NM * 32 + 8 * (2 * S + 9) + 16;
     if (bytes > 232448) return false;
     *smem_bytes = (int)bytes;
     *tmem_cols = (int)pow2_cols(cols);
@@ -365,7 +409,16 @@ cudaError_t launch_tc_contraction(const ContractNest &n, const ContractPlan &p, 
     a.tmem_cols = (uint32_t)tcols;
     a.a_bulk = 0;
     if (const char *e = getenv("EATSS_TC_ABULK")) a.a_bulk = atoi(e);
-    auto k = tc::tc3_gemm_kernel;
+    a.R = 16;  // stages per accumulator chunk (128 k): drift ~128 * 2^-24 per chunk
+    if (const char *e = getenv("EATSS_TC_CHUNK")) a.R = std::max(2, atoi(e));
+    void (*k)(const tc::Args) = nullptr;
+    switch (a.NM) {
+        case 16: k = tc::tc3_gemm_kernel<16>; break;
+        case 32: k = tc::tc3_gemm_kernel<32>; break;
+        case 48: k = tc::tc3_gemm_kernel<48>; break;
+        case 64: k = tc::tc3_gemm_kernel<64>; break;
+        default: return cudaErrorNotSupported;
+    }
     cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
     (void)carveout;
