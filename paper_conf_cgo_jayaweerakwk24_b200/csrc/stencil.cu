@@ -44,6 +44,56 @@ __global__ void __launch_bounds__(256) jacobi2d_sweep(T *__restrict__ dst, const
         const bool b = (i == 0) | (i == n - 1) | (j == 0) | (j == n - 1);
         return b ? bsrc[i * n + j] : src[i * n + j];
     };
+    if constexpr (V == 4 && !COVER) {
+        // Fast column walk for tiles whose every group and row neighbour is interior: a
+        // thread walks a contiguous run of rows of one 16-byte column group keeping rows
+        // i-1 and i in registers, so each output row costs one new 16-byte load (+ two
+        // scalars for the j-1 / j+4 neighbours), four rows in flight per iteration.
+        const bool tile_fast = (tj0 >= 2) && (g0 * 4 >= jlo) && ((g1 - 1) * 4 + 3 < jhi) && (g1 * 4 <= n - 2) &&
+                               (ilo >= 2) && (ihi <= n - 2);
+        if (tile_fast) {
+            const int64_t rows = ihi - ilo;
+            const int64_t chunk = (rows + blockDim.y - 1) / blockDim.y;
+            const int64_t r0 = ilo + threadIdx.y * chunk, r1 = smin64(ihi, r0 + chunk);
+            for (int64_t g = g0 + threadIdx.x; g < g1; g += blockDim.x) {
+                if (r0 >= r1) break;
+                const int64_t j = g * 4;
+                const float *col = src + j;
+                float *ocol = dst + j;
+                auto ld4 = [&](int64_t i) { return *reinterpret_cast<const float4 *>(col + i * n); };
+                auto out = [&](int64_t i, const float4 &u, const float4 &c, const float4 &d, float l, float r) {
+                    float4 o;
+                    o.x = c02 * ((((c.x + l) + c.y) + d.x) + u.x);
+                    o.y = c02 * ((((c.y + c.x) + c.z) + d.y) + u.y);
+                    o.z = c02 * ((((c.z + c.y) + c.w) + d.z) + u.z);
+                    o.w = c02 * ((((c.w + c.z) + r) + d.w) + u.w);
+                    *reinterpret_cast<float4 *>(ocol + i * n) = o;
+                };
+                float4 u = ld4(r0 - 1), c = ld4(r0);
+                int64_t i = r0;
+                for (; i + 4 <= r1; i += 4) {
+                    const float4 d0 = ld4(i + 1), d1 = ld4(i + 2), d2 = ld4(i + 3), d3 = ld4(i + 4);
+                    const float l0 = col[i * n - 1], q0 = col[i * n + 4];
+                    const float l1 = col[(i + 1) * n - 1], q1 = col[(i + 1) * n + 4];
+                    const float l2 = col[(i + 2) * n - 1], q2 = col[(i + 2) * n + 4];
+                    const float l3 = col[(i + 3) * n - 1], q3 = col[(i + 3) * n + 4];
+                    out(i, u, c, d0, l0, q0);
+                    out(i + 1, c, d0, d1, l1, q1);
+                    out(i + 2, d0, d1, d2, l2, q2);
+                    out(i + 3, d1, d2, d3, l3, q3);
+                    u = d2;
+                    c = d3;
+                }
+                for (; i < r1; i++) {
+                    const float4 d = ld4(i + 1);
+                    out(i, u, c, d, col[i * n - 1], col[i * n + 4]);
+                    u = c;
+                    c = d;
+                }
+            }
+            return;
+        }
+    }
     for (int64_t i = ilo + threadIdx.y; i < ihi; i += blockDim.y) {
         for (int64_t g = g0 + threadIdx.x; g < g1; g += blockDim.x) {
             const int64_t j = g * V;
@@ -110,6 +160,38 @@ __global__ void __launch_bounds__(256) heat3d_sweep(T *__restrict__ dst, const T
     const int64_t total = ni * nj * ng;
     const T c = T(0.125), two = T(2.0);
     const int64_t nn = n * n;
+    if constexpr (V == 4 && !COVER) {
+        // Fast column walk along i (stride n^2): a thread owns one (j, 16-byte k-group) and
+        // keeps planes i-1 and i in registers -- per output: one new 16-byte load (plane i+1),
+        // the j+-1 neighbours and two scalars for k-1 / k+4.  All reads stay in bounds.
+        const bool tile_fast = (g0 * 4 >= klo) && ((g1 - 1) * 4 + 3 < khi) && (g0 * 4 >= 1) && (g1 * 4 <= n - 1);
+        if (tile_fast) {
+            for (int64_t e = threadIdx.x; e < nj * ng; e += blockDim.x) {
+                const int64_t g = g0 + e % ng, j = jlo + e / ng, k = g * 4;
+                const float *col = src + j * n + k;
+                float *ocol = dst + j * n + k;
+                auto ld4 = [&](int64_t off) { return *reinterpret_cast<const float4 *>(col + off); };
+                float4 u = ld4((ilo - 1) * nn), x = ld4(ilo * nn);
+                for (int64_t i = ilo; i < ihi; i++) {
+                    const int64_t b = i * nn;
+                    const float4 ip = ld4(b + nn), jp = ld4(b + n), jm = ld4(b - n);
+                    const float km1 = col[b - 1], kp4 = col[b + 4];
+                    float4 o;
+#define HEAT_PT2(X, IP, IM, JP, JM, KP, KM) \
+    (c * (IP - two * X + IM) + c * (JP - two * X + JM) + c * (KP - two * X + KM) + X)
+                    o.x = HEAT_PT2(x.x, ip.x, u.x, jp.x, jm.x, x.y, km1);
+                    o.y = HEAT_PT2(x.y, ip.y, u.y, jp.y, jm.y, x.z, x.x);
+                    o.z = HEAT_PT2(x.z, ip.z, u.z, jp.z, jm.z, x.w, x.y);
+                    o.w = HEAT_PT2(x.w, ip.w, u.w, jp.w, jm.w, kp4, x.z);
+#undef HEAT_PT2
+                    *reinterpret_cast<float4 *>(ocol + b) = o;
+                    u = x;
+                    x = ip;
+                }
+            }
+            return;
+        }
+    }
     for (int64_t e = threadIdx.x; e < total; e += blockDim.x) {
         const int64_t g = g0 + e % ng;
         const int64_t r = e / ng;
@@ -179,7 +261,8 @@ StencilPlan plan_heat3d(int64_t n, int64_t Ti, int64_t Tj, int64_t Tk, bool f64)
     p.gx = cdiv(n - 1, Tk);
     const int64_t nbi = cdiv(n - 1, Ti), nbj = cdiv(n - 1, Tj);
     p.gy = nbi * nbj;
-    const int64_t pts = Ti * Tj * (cdiv(Tk, p.vec) + 1);
+    // vector path: one thread per (j, k-group) walking i; scalar path: one per point
+    const int64_t pts = (p.vec == 4 ? 1 : Ti) * Tj * (cdiv(Tk, p.vec) + 1);
     p.bx = (int)std::min<int64_t>(256, ((pts + 31) / 32) * 32);
     p.by = 1;
     return p;
