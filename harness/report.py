@@ -71,6 +71,27 @@ def summarise(path):
     if d:
         out["share_beating_default_perf"] = float(np.mean([r["tflops"] > d["tflops_median"] for r in ok]))
         out["share_beating_default_ppw"] = float(np.mean([r["gflops_per_watt"] > d["ppw_median"] for r in ok]))
+    # drift correction: scale each variant's PPW / TFLOP/s by the EATSS anchor interpolated
+    # at its measurement time (DVFS / thermal drift over the ~50 min sweep)
+    ae = sorted([r for r in anc["anchor_eatss"] if r.get("status") == 0 and (r.get("joules") or 0) > 0],
+                key=lambda r: r["t"])
+    if len(ae) >= 2:
+        ts = np.array([r["t"] for r in ae])
+        pp = np.array([r["gflops_per_watt"] for r in ae])
+        tf = np.array([r["tflops"] for r in ae])
+        p_med, t_med = float(np.median(pp)), float(np.median(tf))
+        for r in ok:
+            r["ppw_drift_corr"] = r["gflops_per_watt"] * p_med / float(np.interp(r["t"], ts, pp))
+            r["tflops_drift_corr"] = r["tflops"] * t_med / float(np.interp(r["t"], ts, tf))
+        perf_c = max(ok, key=lambda r: r["tflops_drift_corr"])
+        ener_c = max(ok, key=lambda r: r["ppw_drift_corr"])
+        out["drift_corrected"] = {
+            "perf_optimal": {"tile": perf_c["tile"], "tflops": perf_c["tflops_drift_corr"], "ppw": perf_c["ppw_drift_corr"]},
+            "energy_optimal": {"tile": ener_c["tile"], "tflops": ener_c["tflops_drift_corr"], "ppw": ener_c["ppw_drift_corr"]},
+            "ppw_gain": ener_c["ppw_drift_corr"] / perf_c["ppw_drift_corr"],
+            "top10_ppw": [r["tile"] for r in sorted(ok, key=lambda r: -r["ppw_drift_corr"])[:10]],
+            "top10_perf": [r["tile"] for r in sorted(ok, key=lambda r: -r["tflops_drift_corr"])[:10]],
+        }
     out["top5_ppw"] = [{"tile": r["tile"], "gflops_per_watt": r["gflops_per_watt"], "tflops": r["tflops"],
                         "watts": r["watts"]} for r in ppw[:5]]
     out["top5_perf"] = [{"tile": r["tile"], "gflops_per_watt": r["gflops_per_watt"], "tflops": r["tflops"],
@@ -78,12 +99,45 @@ def summarise(path):
     return out
 
 
+T975 = {2: 12.71, 3: 4.30, 4: 3.18, 5: 2.78, 6: 2.57, 7: 2.45, 8: 2.36, 9: 2.31, 10: 2.26}
+
+
+def confirm_summary(path):
+    """Per-tile mean and 95% CI (Student t) of repeated interleaved measurements."""
+    by = {}
+    for line in open(path):
+        r = json.loads(line)
+        if r.get("kind") == "confirm" and r.get("status") == 0 and (r.get("joules") or 0) > 0:
+            by.setdefault(tuple(r["tile"]), []).append(r)
+    rows = []
+    for tile, rs in by.items():
+        n = len(rs)
+        stats = {"tile": list(tile), "n": n}
+        for key in ("gflops_per_watt", "tflops", "watts"):
+            v = np.array([r[key] for r in rs])
+            half = T975.get(n, 1.96) * v.std(ddof=1) / np.sqrt(n) if n > 1 else float("nan")
+            stats[key] = {"mean": float(v.mean()), "ci95": [float(v.mean() - half), float(v.mean() + half)]}
+        rows.append(stats)
+    rows.sort(key=lambda s: -s["gflops_per_watt"]["mean"])
+    if not rows:
+        return {"file": path, "tiles": []}
+    best_ppw = rows[0]
+    best_perf = max(rows, key=lambda s: s["tflops"]["mean"])
+    sep = best_ppw["gflops_per_watt"]["ci95"][0] > best_perf["gflops_per_watt"]["ci95"][1]
+    return {"file": path, "energy_optimal": best_ppw["tile"], "perf_optimal": best_perf["tile"],
+            "ppw_energy_opt": best_ppw["gflops_per_watt"], "ppw_perf_opt": best_perf["gflops_per_watt"],
+            "tflops_energy_opt": best_ppw["tflops"], "tflops_perf_opt": best_perf["tflops"],
+            "finding_energy_beats_perf_on_ppw_ci_separated": bool(best_ppw["tile"] != best_perf["tile"] and sep),
+            "tiles": rows}
+
+
 if __name__ == "__main__":
     ap = argparse.ArgumentParser()
     ap.add_argument("path")
     ap.add_argument("--json", default="")
+    ap.add_argument("--confirm", action="store_true")
     a = ap.parse_args()
-    s = summarise(a.path)
+    s = confirm_summary(a.path) if a.confirm else summarise(a.path)
     txt = json.dumps(s, indent=1)
     print(txt)
     if a.json:

@@ -51,6 +51,8 @@ def parse():
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "sweep_gemm.jsonl"))
     ap.add_argument("--resume", default="", help="existing JSONL whose variants are skipped")
     ap.add_argument("--no-parity", action="store_true")
+    ap.add_argument("--tiles", default="", help="confirmation mode: 'a,b,c;d,e,f' measured --repeats times, interleaved")
+    ap.add_argument("--repeats", type=int, default=5)
     return ap.parse_args()
 
 
@@ -154,6 +156,16 @@ def main():
         return rec
 
     t0 = time.time()
+    if a.tiles:
+        # confirmation mode: the candidate tiles, re-measured round-robin
+        conf = [tuple(int(x) for x in s.split(",")) for s in a.tiles.split(";") if s]
+        for rep_i in range(a.repeats):
+            for tile in conf:
+                r = measure(tile, "confirm")
+        out.close()
+        if rank == 0:
+            print(f"[sweep] confirmation: {len(conf)} tiles x {a.repeats} in {time.time() - t0:.0f} s", flush=True)
+        return
     measure(default_tile, "anchor_default"); measure(eatss_tile, "anchor_eatss")
     for k, v in enumerate(mine):
         measure(v, "variant")

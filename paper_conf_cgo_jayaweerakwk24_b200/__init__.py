@@ -81,7 +81,8 @@ class Desc:
     def __del__(self):
         h = getattr(self, "_h", None)
         if h is not None and h.value:
-            _lib.eatss_desc_destroy(h)
+            if _lib is not None:  # interpreter shutdown may have cleared module globals
+                _lib.eatss_desc_destroy(h)
             self._h = ctypes.c_void_p(0)
 
     @property

@@ -535,13 +535,12 @@ ContractPlan plan_contraction(const ContractNest &n, const int64_t *tiles, int s
         // register-resident: stage both operand slices per k-tile through an S-stage cp.async ring
         // The ring holds S stages of kst k-rows each; a k-tile of Tk rows is staged as
         // ceil(Tk/kst) sub-stages (numerically identical: accumulators are resident and k
-        // stays ascending).  Default: the deepest ring (S = 3) whose footprint still lets two
-        // CTAs share an SM, halving kst until it fits; else one full-k-tile stage.
+        // stays ascending).  Default (measured, profiles/): one stage per whole k-tile
+        // (S = 1) so two CTAs share an SM and overlap each other's copies; kst is halved only
+        // when a k-tile does not fit.  EATSS_STAGES / EATSS_KSUB override for experiments.
         const int64_t aip = ((p.Ti + 3) / 4) * 4, bjp = ((p.Tj + 3) / 4) * 4;
-        const int64_t half = smem_limit / 2 - 1024;
-        int64_t kst = p.Tk, S = 3;
-        while (kst > 1 && S * (kst * (aip + bjp) * esz + 16) > half) kst = (kst + 1) / 2;
-        if (S * (kst * (aip + bjp) * esz + 16) > half) { kst = p.Tk; S = 1; }
+        int64_t kst = p.Tk, S = 1;
+        while (kst > 1 && S * (kst * (aip + bjp) * esz + 16) > smem_limit) kst = (kst + 1) / 2;
         if (const char *e = getenv("EATSS_STAGES")) S = std::max(1, atoi(e));
         if (const char *e = getenv("EATSS_KSUB")) kst = std::max<int64_t>(1, (p.Tk + atoi(e) - 1) / std::max(1, atoi(e)));
         const int64_t stage_bytes = kst * (aip + bjp) * esz;

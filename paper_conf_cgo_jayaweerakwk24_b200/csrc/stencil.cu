@@ -144,11 +144,15 @@ __global__ void __launch_bounds__(256) interior_copy2d(T *__restrict__ dst, cons
 
 // ------------------------------------------------------------------ heat-3d
 // dst = 0.125*(s[i+1]-2s+s[i-1]) + 0.125*(s[j+1]-2s+s[j-1]) + 0.125*(s[k+1]-2s+s[k-1]) + s
+// Grids of n >= kHeatWalkMinN use the i-walk (one thread per (j, k-group)); smaller,
+// L2-resident grids (the paper-size n = 120) keep one thread per point group for parallelism.
+constexpr int64_t kHeatWalkMinN = 256;
 template <typename T, int V, bool COVER>
 __global__ void __launch_bounds__(256) heat3d_sweep(T *__restrict__ dst, const T *__restrict__ src,
                                                     int64_t n, int Ti, int Tj, int Tk, int nbj,
                                                     int32_t *counts) {
     // blockIdx.x -> k-tile, blockIdx.y -> (i-tile, j-tile)
+    const bool walk = n >= kHeatWalkMinN;
     const int64_t tk0 = (int64_t)blockIdx.x * Tk;
     const int64_t ti0 = (int64_t)(blockIdx.y / nbj) * Ti, tj0 = (int64_t)(blockIdx.y % nbj) * Tj;
     const int64_t ilo = smax64(ti0, 1), ihi = smin64(ti0 + Ti, n - 1);
@@ -164,7 +168,9 @@ __global__ void __launch_bounds__(256) heat3d_sweep(T *__restrict__ dst, const T
         // Fast column walk along i (stride n^2): a thread owns one (j, 16-byte k-group) and
         // keeps planes i-1 and i in registers -- per output: one new 16-byte load (plane i+1),
         // the j+-1 neighbours and two scalars for k-1 / k+4.  All reads stay in bounds.
-        const bool tile_fast = (g0 * 4 >= klo) && ((g1 - 1) * 4 + 3 < khi) && (g0 * 4 >= 1) && (g1 * 4 <= n - 1);
+        // (only when the grid is large enough that one thread per (j, k-group) still fills the GPU)
+        const bool tile_fast = walk && (g0 * 4 >= klo) && ((g1 - 1) * 4 + 3 < khi) && (g0 * 4 >= 1) &&
+                               (g1 * 4 <= n - 1);
         if (tile_fast) {
             for (int64_t e = threadIdx.x; e < nj * ng; e += blockDim.x) {
                 const int64_t g = g0 + e % ng, j = jlo + e / ng, k = g * 4;
@@ -262,7 +268,7 @@ StencilPlan plan_heat3d(int64_t n, int64_t Ti, int64_t Tj, int64_t Tk, bool f64)
     const int64_t nbi = cdiv(n - 1, Ti), nbj = cdiv(n - 1, Tj);
     p.gy = nbi * nbj;
     // vector path: one thread per (j, k-group) walking i; scalar path: one per point
-    const int64_t pts = (p.vec == 4 ? 1 : Ti) * Tj * (cdiv(Tk, p.vec) + 1);
+    const int64_t pts = ((p.vec == 4 && n >= kHeatWalkMinN) ? 1 : Ti) * Tj * (cdiv(Tk, p.vec) + 1);
     p.bx = (int)std::min<int64_t>(256, ((pts + 31) / 32) * 32);
     p.by = 1;
     return p;

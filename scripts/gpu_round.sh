@@ -1,9 +1,6 @@
 cd $GRAFT_REPO_ROOT
-timeout 1200 python -m pytest tests -m gpu -q --timeout 600 -p no:cacheprovider 2>&1 | tail -4
+timeout 900 python harness/sweep.py --tiles "64,256,128;32,384,48;32,512,48;24,512,32;48,256,64;24,512,48;32,384,64;32,512,24;48,192,64;16,1024,16;32,32,32;48,256,48" --repeats 7 --window 1.0 --no-parity --out gpurun_out/sweep_confirm_r01.jsonl 2>&1 | tail -2
+python harness/report.py --confirm gpurun_out/sweep_confirm_r01.jsonl --json gpurun_out/sweep_confirm_r01.summary.json | head -40
+timeout 1200 python -m pytest tests -m gpu -q --timeout 600 -p no:cacheprovider 2>&1 | tail -3
 T="timeout 120 python scripts/time_kernel.py"
-$T gemm 4000,4000,4000 16,1024,16; EATSS_KSUB=1 EATSS_STAGES=1 $T gemm 4000,4000,4000 16,1024,16
-EATSS_STAGES=2 $T gemm 4000,4000,4000 16,1024,16; EATSS_KSUB=4 $T gemm 4000,4000,4000 16,1024,16
-timeout 120 python scripts/debug_tc.py 4000 16,1024,16
-$T gemm 4000,4000,4000 16,1024,16 --engine 2
-$T jacobi-2d 16384 16,1024 --tsteps 20 --iters 3; $T jacobi-2d 4000 16,1024 --tsteps 500 --iters 3
-$T heat-3d 512 16,16,32 --tsteps 10 --iters 3; $T heat-3d 120 16,16,32 --tsteps 500 --iters 3
+$T heat-3d 512 16,16,32 --tsteps 10 --iters 3; $T heat-3d 120 16,16,32 --tsteps 500 --iters 3; $T gemm 4000,4000,4000 16,1024,16

@@ -20,7 +20,15 @@ def host(t):
     return t.double().cpu().numpy()
 
 
-TILES = [(16, 1024, 16), (16, 128, 8), (32, 512, 16), (16, 256, 32), (48, 384, 8), (64, 128, 16)]
+TILES = [(16, 1024, 16), (16, 128, 8), (32, 512, 16), (16, 256, 32), (48, 256, 8), (64, 128, 16)]
+
+
+def test_tc_inapplicable_tile_is_reported_not_faked(cuda_device):
+    # (48, 384): 2 M-blocks per converter warp x 48 columns > the 64 fp32 chunk sums per thread
+    d = E.desc_builtin("gemm", (64, 384, 64)); d.set_exec(50, TENSOR)
+    with pytest.raises(E.EatssError) as ei:
+        E.run(d, (48, 384, 8), [dev(np.zeros((64, 384))), dev(np.zeros((64, 64))), dev(np.zeros((64, 384)))])
+    assert ei.value.status == -5  # EATSS_E_UNSUPPORTED
 
 
 @pytest.mark.parametrize("tiles", TILES)
