@@ -83,7 +83,7 @@ class Desc:
         if h is not None and h.value:
             if _lib is not None:  # interpreter shutdown may have cleared module globals
                 _lib.eatss_desc_destroy(h)
-            self._h = ctypes.c_void_p(0)
+            self._h = None
 
     @property
     def num_loops(self) -> int:

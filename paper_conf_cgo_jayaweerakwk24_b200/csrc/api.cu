@@ -513,11 +513,15 @@ static eatss_status run_impl(const eatss_kernel_desc *cd, int only_nest, const i
             if (only_nest >= 0 && i != only_nest) continue;
             ContractPlan p = plan_contraction(cn[i], tiles, sl);
             int tsm = 0, tcols = 0;
-            const bool tc = d->exec.engine == EATSS_ENGINE_TENSOR && tc_plan(cn[i], p, &tsm, &tcols);
-            if (d->exec.engine == EATSS_ENGINE_TENSOR && !tc)
+            const bool want_tc = d->exec.engine == EATSS_ENGINE_TENSOR;
+            // MMA-legal tiles (Ti = 128) take the TMA/SS-UMMA GEMM; narrow tiles the transposed TS kernel
+            const bool tcm = want_tc && tcm_applicable(cn[i], p);
+            const bool tc = want_tc && !tcm && tc_plan(cn[i], p, &tsm, &tcols);
+            if (want_tc && !tc && !tcm)
                 return fail(EATSS_E_UNSUPPORTED, "eatss_run: tensor engine not applicable to this tile/operand layout");
-            cudaError_t e = tc ? launch_tc_contraction(cn[i], p, d->exec.split_pct, s)
-                               : launch_contraction(cn[i], p, d->exec.split_pct, nullptr, s);
+            cudaError_t e = tcm  ? launch_tcm_contraction(cn[i], p, s)
+                            : tc ? launch_tc_contraction(cn[i], p, d->exec.split_pct, s)
+                                 : launch_contraction(cn[i], p, d->exec.split_pct, nullptr, s);
             if (e != cudaSuccess) return cuda_fail(e, "eatss_run(contraction)");
         }
         return EATSS_OK;

@@ -42,6 +42,9 @@ ContractPlan plan_contraction(const ContractNest &n, const int64_t *tiles, int s
 // tensor-core (tcgen05, 3xTF32) executor: applicability / launch (tc_gemm.cu)
 bool tc_plan(const ContractNest &n, const ContractPlan &p, int *smem_bytes, int *tmem_cols);
 cudaError_t launch_tc_contraction(const ContractNest &n, const ContractPlan &p, int carveout, cudaStream_t s);
+// tcgen05 3xTF32 GEMM for MMA-legal tiles (Ti = 128, Tj in 32..256 step 32) (tc_mma.cu)
+bool tcm_applicable(const ContractNest &n, const ContractPlan &p);
+cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p, cudaStream_t s);
 cudaError_t launch_contraction(const ContractNest &n, const ContractPlan &p, int carveout_pct,
                                int32_t *coverage_counts, cudaStream_t s);
 

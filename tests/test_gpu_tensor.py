@@ -77,3 +77,41 @@ def test_tc_2mm_3mm(cuda_device):
     tmp = torch.zeros((ni, nj), device="cuda"); Dd = dev(D)
     E.run(d, (16, 1024, 16), [tmp, dev(A), dev(B), dev(C), Dd])
     assert O.normwise_rel_err(host(tmp), tmp_ref) <= 1e-5 and O.normwise_rel_err(host(Dd), D_ref) <= 1e-5
+
+
+# ---- MMA-legal tiles (Ti = 128): TMA + SS-UMMA GEMM (tc_mma.cu)
+MMA_TILES = [(128, 256, 32), (128, 128, 32), (128, 64, 8), (128, 192, 16), (128, 32, 32)]
+
+
+@pytest.mark.parametrize("tiles", MMA_TILES)
+def test_tcm_small_int_bit_exact(cuda_device, tiles):
+    ni, nj, nk = 300, 1100, 204  # ragged everywhere: TMA zero-fill at the i/j/k edges
+    A = synth.small_int((ni, nk), 10); B = synth.small_int((nk, nj), 11); C = synth.small_int((ni, nj), 12)
+    ref = O.gemm(1.0, 1.0, C, A, B)
+    d = E.desc_builtin("gemm", (ni, nj, nk)); d.set_scalars(1.0, 1.0); d.set_exec(50, TENSOR)
+    Cd = dev(C)
+    E.run(d, tiles, [Cd, dev(A), dev(B)])
+    assert np.array_equal(host(Cd), ref)
+
+
+@pytest.mark.parametrize("tiles", MMA_TILES[:3])
+def test_tcm_random_tolerance(cuda_device, tiles):
+    ni, nj, nk = 260, 516, 1000
+    A = synth.uniform((ni, nk), 20); B = synth.uniform((nk, nj), 21); C = synth.uniform((ni, nj), 22)
+    ref = O.gemm(1.5, 1.2, C, A, B)
+    d = E.desc_builtin("gemm", (ni, nj, nk)); d.set_scalars(1.5, 1.2); d.set_exec(50, TENSOR)
+    Cd = dev(C)
+    E.run(d, tiles, [Cd, dev(A), dev(B)])
+    assert O.normwise_rel_err(host(Cd), ref) <= 1e-5
+
+
+def test_tcm_full_size_sampled(cuda_device):
+    n = 4000
+    d = E.desc_builtin("gemm", (n, n, n)); d.set_scalars(1.5, 1.2); d.set_exec(50, TENSOR)
+    A = synth.uniform((n, n), 4); B = synth.uniform((n, n), 5); C = synth.uniform((n, n), 6)
+    Cd = dev(C)
+    E.run(d, (128, 256, 32), [Cd, dev(A), dev(B)])
+    out = host(Cd)
+    g = synth.rng(7)
+    ii = g.integers(0, n, 2048); jj = g.integers(0, n, 2048)
+    assert O.normwise_rel_err(out[ii, jj], O.gemm_entries(ii, jj, C, A, B, 1.5, 1.2)) <= 1e-5
