@@ -331,10 +331,76 @@ def extents(prog: Program) -> List[int]:
     return ex
 
 
+# ------------------------------------------------------------- tensor-core mode (mode 2)
+# Reading T: the same objective (Eq. 2) and tie-break,
+# over MMA-legal tiles of the tcgen05 executor, with the register / L1 / SH capacities
+# replaced by the resources that executor actually uses:
+#   T1  applies to nests of depth 3 with one serial (reduction) loop and l_s1 parallel;
+#   T2  domain: l_s1 (UMMA N) in {32, 64, ..., min(256, roundup32(N))}; the other B-set loop
+#       (UMMA M) in {128}; the serial loop (one 128-byte TMA atom of fp32) in {32};
+#   T3  TMEM: two fp32 accumulator buffers of T_{l_s1} columns, 2*T_{l_s1} <= 512;
+#       SMEM: 2 stages x {hi, lo} x e x (sum of the input footprints) <= max_smem_per_block.
+
+TMEM_COLS = 512
+
+
+def tensor_applicable(prog: Program) -> bool:
+    for nest in prog.nests:
+        if len(nest.loops) != 3 or sum(1 for l in nest.loops if not l.parallel) != 1:
+            return False
+        d = derive(nest, 16)
+        if not nest.loops[[l.name for l in nest.loops].index(d.ls1)].parallel:
+            return False
+    return True
+
+
+def tensor_domains(prog: Program):
+    n0 = prog.nests[0]
+    d = derive(n0, 16)
+    doms = []
+    ex = extents(prog)
+    for p, l in enumerate(n0.loops):
+        if l.name == d.ls1:
+            hi = min(256, -(-ex[p] // 32) * 32)
+            doms.append(list(range(32, hi + 1, 32)))
+        elif l.parallel:
+            doms.append([128])
+        else:
+            doms.append([32])
+    return doms
+
+
+def evaluate_tensor(prog: Program, gpu: Gpu, opts: Opts, T):
+    e = prog.dtype_bytes
+    feas = np.ones(T[0].shape, dtype=bool)
+    obj = np.zeros(T[0].shape, dtype=np.int64)
+    for nest in prog.nests:
+        d = derive(nest, opts.waf)
+        pos = {l.name: p for p, l in enumerate(nest.loops)}
+        written = {r.array for r in nest.refs if r.write}
+        inputs = []
+        for r in d.refs:
+            f = (r.array, r.iters())
+            if r.array not in written and f not in inputs:
+                inputs.append(f)
+        feas &= 2 * T[pos[d.ls1]] <= TMEM_COLS                                  # T3 TMEM
+        vin = sum((_prod(T, f[1], pos) for f in inputs), np.zeros_like(T[0]))
+        feas &= 2 * 2 * e * vin <= gpu.max_smem_per_block                      # T3 SMEM
+        obj = obj + _prod(T, d.bset, pos)                                       # Eq. 2
+        for l in nest.loops:
+            if d.H[l.name]:
+                obj = obj + d.H[l.name] * T[pos[l.name]]
+    return feas, obj
+
+
 def select_tiles(prog: Program, gpu: Gpu, opts: Opts, keep_ties: bool = True) -> Result:
     """Exhaustive maximisation of OBJ over the whole domain (no pruning)."""
     L = prog.L
-    doms = [np.array(domain(n, gpu, opts.waf), dtype=np.int64) for n in extents(prog)]
+    tensor = opts.mode == 2
+    if tensor and not tensor_applicable(prog):
+        return Result(None, 0, 0, 0, [])
+    doms = ([np.array(v, dtype=np.int64) for v in tensor_domains(prog)] if tensor else
+            [np.array(domain(n, gpu, opts.waf), dtype=np.int64) for n in extents(prog)])
     free = objective_free_positions(prog, opts.waf)
     ls1_pos = [l.name for l in prog.nests[0].loops].index(derive(prog.nests[0], opts.waf).ls1)
     best_key, best, ties, n_feas = None, None, [], 0
@@ -343,7 +409,7 @@ def select_tiles(prog: Program, gpu: Gpu, opts: Opts, keep_ties: bool = True) ->
     rest = [r.ravel() for r in rest]
     for t0 in doms[0]:
         T = [np.full(rest[0].shape if rest else (1,), t0, dtype=np.int64)] + rest
-        feas, obj = evaluate(prog, gpu, opts, T)
+        feas, obj = (evaluate_tensor if tensor else evaluate)(prog, gpu, opts, T)
         n_feas += int(feas.sum())
         if not feas.any():
             continue

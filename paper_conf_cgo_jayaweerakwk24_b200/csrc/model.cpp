@@ -148,7 +148,28 @@ Caps capacities(const eatss_gpu_params &g, const eatss_model_opts &o, int e) {
 struct NestEval {
     const Nest *nest;
     NestModel m;
+    std::vector<uint32_t> in_fp;  // tensor mode: footprints of the arrays the nest only reads
 };
+
+// Tensor-core mode (reading T): the executor stages every input footprint in
+// shared memory (2 stages x {hi, lo}) and keeps two fp32 accumulators of T_{l_s1} TMEM columns.
+std::vector<uint32_t> input_footprints(const Nest &n) {
+    std::vector<int> written;
+    for (const Ref &r : n.refs)
+        if (r.write) written.push_back(r.array);
+    std::vector<std::pair<int, uint32_t>> seen;
+    for (const Ref &r : n.refs) {
+        if (std::find(written.begin(), written.end(), r.array) != written.end()) continue;
+        uint32_t it = 0;
+        for (const Sub &s : r.subs) it |= s.iters;
+        std::pair<int, uint32_t> f{r.array, it};
+        if (std::find(seen.begin(), seen.end(), f) == seen.end()) seen.push_back(f);
+    }
+    std::vector<uint32_t> out;
+    for (auto &f : seen) out.push_back(f.second);
+    return out;
+}
+constexpr int64_t kTmemCols = 512;
 
 struct Search {
     int L = 0;
@@ -171,7 +192,20 @@ struct Search {
         return v;
     }
 
+    bool tensor = false;
+    int64_t smem_cap = 0;
+    int esz = 4;
+
     bool feasible(const std::vector<int64_t> &T) const {
+        if (tensor) {
+            for (const NestEval &ne : nests) {
+                if (2 * T[ne.m.ls1] > kTmemCols) return false;  // two fp32 accumulator buffers
+                int64_t vin = 0;
+                for (uint32_t f : ne.in_fp) vin += prod(T, f);
+                if (2 * 2 * esz * vin > smem_cap) return false;  // 2 stages x {hi, lo}
+            }
+            return true;
+        }
         for (const NestEval &ne : nests) {
             const NestModel &m = ne.m;
             const int64_t B = prod(T, m.bset);
@@ -263,15 +297,41 @@ extern "C" eatss_status eatss_select_tiles(const eatss_kernel_desc *d, const eat
     s.fpf = (e == 8) ? 2 : 1;  // FP_factor
     s.regs = g->regs_per_sm;
     s.caps = capacities(*g, *o, e);
-    // rule 10 -- domain: multiples of WAF in [WAF, min(T_P_B, N)]; N < WAF -> {N}
-    for (int p = 0; p < s.L; p++) {
-        std::vector<int64_t> dm;
-        const int64_t hi = std::min<int64_t>(g->threads_per_block, ext[p]);
-        for (int64_t v = o->warp_align; v <= hi; v += o->warp_align) dm.push_back(v);
-        if (dm.empty()) dm.push_back(ext[p]);
-        s.dom.push_back(dm);
+    for (const Nest &n : d->nests) s.nests.push_back({&n, derive_nest(n, o->warp_align), input_footprints(n)});
+    if (o->mode == 2) {
+        // tensor-core mode: depth-3 nests with one serial loop and a parallel l_s1 only
+        for (const NestEval &ne : s.nests) {
+            int serial = 0;
+            for (const Loop &l : ne.nest->loops) serial += l.parallel ? 0 : 1;
+            if (ne.nest->loops.size() != 3 || serial != 1 || !ne.nest->loops[ne.m.ls1].parallel)
+                return fail(EATSS_E_UNSUPPORTED, "eatss_select_tiles: tensor mode needs depth-3 contraction nests");
+        }
+        s.tensor = true;
+        s.esz = e;
+        s.smem_cap = g->max_smem_per_block;
+        const Nest &n0 = d->nests[0];
+        for (int p = 0; p < s.L; p++) {
+            std::vector<int64_t> dm;
+            if (p == s.nests[0].m.ls1) {  // UMMA N: 32-multiples up to 256 (TMA boxes of 32 columns)
+                const int64_t hi = std::min<int64_t>(256, ((ext[p] + 31) / 32) * 32);
+                for (int64_t v = 32; v <= hi; v += 32) dm.push_back(v);
+            } else if (n0.loops[p].parallel) {
+                dm.push_back(128);  // UMMA M (cta_group::1)
+            } else {
+                dm.push_back(32);  // one 128-byte TMA atom of the reduction loop
+            }
+            s.dom.push_back(dm);
+        }
+    } else {
+        // rule 10 -- domain: multiples of WAF in [WAF, min(T_P_B, N)]; N < WAF -> {N}
+        for (int p = 0; p < s.L; p++) {
+            std::vector<int64_t> dm;
+            const int64_t hi = std::min<int64_t>(g->threads_per_block, ext[p]);
+            for (int64_t v = o->warp_align; v <= hi; v += o->warp_align) dm.push_back(v);
+            if (dm.empty()) dm.push_back(ext[p]);
+            s.dom.push_back(dm);
+        }
     }
-    for (const Nest &n : d->nests) s.nests.push_back({&n, derive_nest(n, o->warp_align)});
     // objective-free positions: H == 0 and outside the B-set in every nest
     for (int p = 0; p < s.L; p++) {
         bool fr = true;

@@ -43,6 +43,14 @@ for waf in (4, 8, 16, 32):
 for waf in (4, 8, 16, 32):
     for split in (0, 50, 100):
         add("heat-3d", (120,), 8, "GA100", split, waf, 0)
+# tensor-core mode (reading T)
+add("gemm", (4000, 4000, 4000), 4, "B200", 50, 16, 2)
+add("2mm", (4000, 4000, 4000, 4000), 4, "B200", 50, 16, 2)
+add("3mm", (4000, 4000, 4000, 4000, 4000), 4, "B200", 50, 16, 2)
+add("syrk", (4000, 4000), 4, "B200", 50, 16, 2)
+add("gemm", (100, 40, 20), 4, "B200", 50, 16, 2)
+add("gemm", (300, 1100, 204), 4, "B200", 50, 16, 2)
+add("gemm", (4000, 4000, 4000), 4, "GA100", 50, 16, 2)
 add("ccsd_t_d1", (48,), 4, "B200", 50, 4, 1)
 add("ccsd_t_d1", (48,), 4, "B200", 50, 8, 1)
 add("ccsd_t_d1", (16,), 4, "B200", 50, 4, 1)

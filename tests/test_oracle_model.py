@@ -146,3 +146,16 @@ def test_model_golden_regenerates():
         r = M.select_tiles(prog, gpu, M.Opts(case["split_pct"], case["waf"], case["mode"]))
         assert (list(r.tiles) if r.tiles else None) == case["tiles"]
         assert r.obj == case["obj"] and r.n_ties == case["n_ties"] and r.n_feasible == case["n_feasible"]
+
+
+def test_tensor_mode_hand_checked():
+    """Reading T on gemm 4000 fp32, B200: domain Ti = {128}, Tk = {32}, Tj = {32, 64, ..., 256}.
+
+    TMEM 2*Tj <= 512 and SMEM 2*2*4*(128*32 + 32*Tj) <= 232448 (Tj <= 326) hold for all 8
+    points; OBJ = Ti*Tj + 2*16*Tj = 160*Tj is maximal and unique at Tj = 256 -> (128, 256, 32).
+    With GA100's 48 KB shared memory per block no point fits (16*(4096+32*Tj) > 49152).
+    """
+    r = M.select_tiles(M.gemm(), M.B200, M.Opts(50, 16, 2))
+    assert r.n_feasible == 8 and r.n_ties == 1 and r.tiles == (128, 256, 32) and r.obj == 160 * 256
+    assert M.select_tiles(M.gemm(), M.GA100, M.Opts(50, 16, 2)).tiles is None
+    assert M.select_tiles(M.heat3d(), M.B200, M.Opts(50, 16, 2)).tiles is None  # not a contraction
