@@ -1,17 +1,19 @@
 #!/usr/bin/env python
 """bench.py -- headline benchmark: EATSS-tiled gemm N=4000 fp32 on B200.
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--engine tensor|simt]
 
 One step = one pass of the whole hot path on one problem: build the kernel
-descriptor's model inputs -> select the tile vector with the EATSS model
-(host enumeration) -> execute the tiled gemm N=4000 (SIMT contraction executor)
-in libeatss.so.  Metric (BASELINE.json): TFLOP/s and GFLOP/s per Watt.
-For N > 1 (torchrun, one process per GPU, NCCL) every rank runs its own
-N=4000 problem (weak scaling, no data-path collective); timing is the max over
-ranks of the device-timed region, energy the sum over ranks.
-
-Prints ONE JSON line on rank 0 (see DESIGN.md §6 for every key).
+descriptor -> select the tile vector with the EATSS model (host enumeration) ->
+execute the tiled gemm N=4000 in libeatss.so.  Two EATSS modes are measured:
+  * tensor (headline, default): the model in tensor-core mode (reading T, SURVEY §8(f)
+    row 3) picks an MMA-legal tile, executed by the tcgen05 3xTF32 engine (fp32-accurate);
+  * simt: the paper's formulation in B200 mode picks (16,1024,16), executed by the SIMT
+    contraction executor (the paper's code class) -- reported under "simt".
+Metric (BASELINE.json): TFLOP/s and GFLOP/s per Watt.  For N > 1 (torchrun, one
+process per GPU, NCCL) every rank runs its own N=4000 problem (weak scaling, no
+data-path collective); timing is the max over ranks of the device-timed region,
+energy the sum over ranks.  Prints ONE JSON line on rank 0.
 """
 from __future__ import annotations
 
@@ -32,6 +34,7 @@ N = 4000
 METRIC = "GFLOP/s per Watt and TFLOP/s of EATSS-tiled affine kernels (gemm N=4000)"
 FLOPS = 2.0 * N ** 3
 SM_COUNT, FP32_LANES = 148, 128
+TF32_OVER_BF16 = 1.1 / 2.25  # B200_PROFILING.md nominal dense tf32 / bf16
 
 
 def parse():
@@ -40,16 +43,15 @@ def parse():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--engine", choices=["tensor", "simt"], default="tensor")
     ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-secondary", action="store_true")
     return ap.parse_args()
 
 
 def dist_env():
-    ws = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    return ws, rank, local
+    return int(os.environ.get("WORLD_SIZE", "1")), int(os.environ.get("RANK", "0")), int(os.environ.get("LOCAL_RANK", "0"))
 
 
 def measured_peaks():
@@ -125,11 +127,11 @@ class ClockSampler:
 
     def __init__(self, device_index: int):
         self.ok = False
+        self.max_mhz = None
         try:
             import pynvml
-            pynvml.nvmlInit()
             import torch
-            # match the CUDA device to its NVML handle by UUID (CUDA_VISIBLE_DEVICES safe)
+            pynvml.nvmlInit()
             want = "GPU-" + str(torch.cuda.get_device_properties(device_index).uuid)
             h = None
             for i in range(pynvml.nvmlDeviceGetCount()):
@@ -144,7 +146,7 @@ class ClockSampler:
             self.nv, self.h, self.ok = pynvml, h, True
             self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
         except Exception:
-            self.max_mhz = None
+            pass
         self.mhz, self.mw, self.reasons = [], [], 0
         self._stop = threading.Event()
 
@@ -164,7 +166,7 @@ class ClockSampler:
                 self.reasons |= self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
             except Exception:
                 pass
-            time.sleep(0.05)
+            time.sleep(0.02)
 
     def __enter__(self):
         if self.ok:
@@ -182,6 +184,46 @@ class ClockSampler:
         return {"sm_mhz": statistics.median(self.mhz) if self.mhz else None, "sm_max_mhz": self.max_mhz,
                 "reasons": reasons, "samples": len(self.mhz),
                 "power_w_median": statistics.median(self.mw) / 1e3 if self.mw else None}
+
+
+# ------------------------------------------------------------------ one engine
+class Arm:
+    """EATSS mode + engine: model mode 2 (tensor) -> tcgen05, mode 1 (B200) -> SIMT."""
+
+    def __init__(self, E, engine, gpu):
+        self.E, self.gpu = E, gpu
+        self.mode = 2 if engine == "tensor" else 1
+        self.engine = 2 if engine == "tensor" else 1
+        self.name = engine
+
+    def step(self, C, A, B, stream):
+        E = self.E
+        d = E.desc_builtin("gemm", (N, N, N))                                   # a1 descriptor
+        d.set_scalars(1.5, 1.2)
+        tiles, rep = E.select_tiles(d, self.gpu, split_pct=50, waf=16, mode=self.mode)  # a2-a4 model
+        d.set_exec(split_pct=50, engine=self.engine)                             # a5 carve-out / engine
+        E.run(d, tiles, [C, A, B], stream)                                       # a5-a6 plan + execution
+        return d, tiles, rep
+
+
+def timed(arm, C, A, B, stream, K, torch, clk=None):
+    ev_s = [torch.cuda.Event(enable_timing=True) for _ in range(K)]
+    ev_e = [torch.cuda.Event(enable_timing=True) for _ in range(K)]
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    e0 = clk.energy_mj() if clk else None
+    t0.record(stream)
+    for i in range(K):
+        ev_s[i].record(stream)
+        arm.step(C, A, B, stream)
+        ev_e[i].record(stream)
+    t1.record(stream)
+    torch.cuda.synchronize()
+    e1 = clk.energy_mj() if clk else None
+    ms = t0.elapsed_time(t1)
+    kern = float(np.mean([ev_s[i].elapsed_time(ev_e[i]) for i in range(K)]))
+    joules = (e1 - e0) / 1e3 if (e0 is not None and e1 is not None) else float("nan")
+    return ms, kern, joules
 
 
 # ------------------------------------------------------------------ our arm
@@ -209,77 +251,61 @@ def main():
     A_h = synth.uniform((N, N), 0); B_h = synth.uniform((N, N), 1); C_h = synth.uniform((N, N), 2)
     A = torch.from_numpy(A_h).to(dev); B = torch.from_numpy(B_h).to(dev); C = torch.from_numpy(C_h).to(dev)
     gpu = E.gpu_params_query(local)
-    alpha, beta = 1.5, 1.2
-
-    def step():
-        d = E.desc_builtin("gemm", (N, N, N))                      # a1 kernel descriptor
-        d.set_scalars(alpha, beta)
-        tiles, rep = E.select_tiles(d, gpu, split_pct=50, waf=16)  # a2-a4 model + tile selection
-        d.set_exec(split_pct=50)                                   # a5 carve-out from the split
-        E.run(d, tiles, [C, A, B], stream)                         # a5-a6 launch plan + tiled execution
-        return d, tiles, rep
-
-    for _ in range(max(3, args.warmup)):
-        d, tiles, rep = step()
+    arm = Arm(E, args.engine, gpu)
+    W = max(3, args.warmup)
+    for _ in range(W):
+        d, tiles, rep = arm.step(C, A, B, stream)
     torch.cuda.synchronize()
     plans = E.plan(d, tiles)
-    launches_per_step = E.launches_per_run(d, tiles)
+    launches_per_step = E.launches_per_run(d, tiles) + (2 if arm.engine == 2 else 0)  # + tf32 split passes
 
     clk = ClockSampler(local)
     K = args.steps
-    ev_s = [torch.cuda.Event(enable_timing=True) for _ in range(K)]
-    ev_e = [torch.cuda.Event(enable_timing=True) for _ in range(K)]
-    t_start = torch.cuda.Event(enable_timing=True); t_end = torch.cuda.Event(enable_timing=True)
     if ws > 1:
         dist.barrier()
-    torch.cuda.synchronize()
     with clk:
-        e0 = clk.energy_mj()
-        t_start.record(stream)
-        for i in range(K):
-            dd = E.desc_builtin("gemm", (N, N, N))
-            dd.set_scalars(alpha, beta)
-            tt, _ = E.select_tiles(dd, gpu, split_pct=50, waf=16)
-            dd.set_exec(split_pct=50)
-            ev_s[i].record(stream)
-            E.run(dd, tt, [C, A, B], stream)
-            ev_e[i].record(stream)
-        t_end.record(stream)
-        torch.cuda.synchronize()
-        e1 = clk.energy_mj()
+        ms_total, kern_ms, joules = timed(arm, C, A, B, stream, K, torch, clk)
     if ws > 1:
         dist.barrier()
-    ms_total = t_start.elapsed_time(t_end)
-    kern_ms = [ev_s[i].elapsed_time(ev_e[i]) for i in range(K)]
-    joules = (e1 - e0) / 1e3 if (e0 is not None and e1 is not None) else float("nan")
+
+    # secondary: the paper-formulation (SIMT) EATSS arm on the same problem
+    sec = None
+    if not args.no_secondary:
+        arm2 = Arm(E, "simt" if args.engine == "tensor" else "tensor", gpu)
+        for _ in range(3):
+            d2, tiles2, _ = arm2.step(C, A, B, stream)
+        K2 = max(20, K // 4)
+        clk2 = ClockSampler(local)
+        ms2, kern2, j2 = timed(arm2, C, A, B, stream, K2, torch, clk2)
+        sec = {"engine": arm2.name, "tiles": list(tiles2), "ms_per_step": ms2 / K2,
+               "tflops": FLOPS / (ms2 / K2 * 1e-3) / 1e12,
+               "gflops_per_watt": FLOPS * K2 / j2 / 1e9 if j2 == j2 and j2 > 0 else None}
 
     # e2e through the public API with host buffers (pinned), copies inside the timed region
     A_p = torch.from_numpy(A_h).pin_memory(); B_p = torch.from_numpy(B_h).pin_memory()
     C_p = torch.from_numpy(C_h).pin_memory(); C_out = torch.empty_like(C_p).pin_memory()
     A2 = torch.empty_like(A); B2 = torch.empty_like(B); C2 = torch.empty_like(C)
     Ke = args.e2e_steps
-    for _ in range(2):
+
+    def e2e_step():
         A2.copy_(A_p, non_blocking=True); B2.copy_(B_p, non_blocking=True); C2.copy_(C_p, non_blocking=True)
-        step_d, step_t, _ = step()
-        E.run(step_d, step_t, [C2, A2, B2], stream)
+        arm.step(C2, A2, B2, stream)
         C_out.copy_(C2, non_blocking=True)
+
+    for _ in range(2):
+        e2e_step()
     torch.cuda.synchronize()
-    e2s = torch.cuda.Event(enable_timing=True); e2e_ev = torch.cuda.Event(enable_timing=True)
     if ws > 1:
         dist.barrier()
+    e2s, e2e_ev = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e2s.record(stream)
     for _ in range(Ke):
-        A2.copy_(A_p, non_blocking=True); B2.copy_(B_p, non_blocking=True); C2.copy_(C_p, non_blocking=True)
-        dd = E.desc_builtin("gemm", (N, N, N)); dd.set_scalars(alpha, beta)
-        tt, _ = E.select_tiles(dd, gpu, split_pct=50, waf=16)
-        E.run(dd, tt, [C2, A2, B2], stream)
-        C_out.copy_(C2, non_blocking=True)
+        e2e_step()
     e2e_ev.record(stream)
     torch.cuda.synchronize()
     e2e_ms = e2s.elapsed_time(e2e_ev) / Ke
 
-    # max over ranks (time), sum over ranks (energy)
-    vals = torch.tensor([ms_total, e2e_ms, float(np.mean(kern_ms))], dtype=torch.float64, device=dev)
+    vals = torch.tensor([ms_total, e2e_ms, kern_ms], dtype=torch.float64, device=dev)
     en = torch.tensor([joules], dtype=torch.float64, device=dev)
     if ws > 1:
         dist.all_reduce(vals, op=dist.ReduceOp.MAX)
@@ -293,46 +319,58 @@ def main():
         clocks = clk.summary()
         peaks = measured_peaks()
         sm_max = clocks.get("sm_max_mhz") or peaks.get("sm_max_mhz") or 1965.0
-        fp32_peak = SM_COUNT * FP32_LANES * 2 * sm_max * 1e6 / 1e12
         achieved = FLOPS / (kern_avg_ms * 1e-3) / 1e12
         traffic = None
         tp = os.path.join(ROOT, "profiles", "traffic.json")
+        key = "gemm_tensor_eatss_tile" if arm.engine == 2 else "gemm_eatss_tile"
         if os.path.exists(tp):
             try:
-                traffic = json.load(open(tp)).get("gemm_eatss_tile", {}).get("dram_bytes_per_launch")
+                traffic = json.load(open(tp)).get(key, {}).get("dram_bytes_per_launch")
             except Exception:
                 traffic = None
         p0 = plans[0]
+        if arm.engine == 2:
+            bf16 = peaks.get("bf16_tflops", 1590.0)
+            tf32 = bf16 * TF32_OVER_BF16
+            roof = {"bound": "tensor", "achieved": achieved, "peak": tf32 / 3, "unit": "TFLOP/s",
+                    "frac": achieved / (tf32 / 3), "traffic": traffic,
+                    "kernel": f"tc_mma_kernel<{tiles[1]}> (+2 tf32 split passes inside the timed call)",
+                    "peak_source": (f"measured bf16 {bf16:.1f} TF (MEASURED_PEAKS.json, burst) x nominal "
+                                    f"tf32/bf16 {TF32_OVER_BF16:.3f} = {tf32:.1f} TF tf32; 3xTF32 executes 3 "
+                                    f"MMAs per useful MAC -> {tf32 / 3:.1f} TF useful"),
+                    "achieved_note": "useful fp32 flops / device time of the whole eatss_run call"}
+            engine_desc = "tcgen05 3xTF32 (TMA + SS-UMMA, TMEM accumulators), EATSS tensor-core mode"
+        else:
+            fp32_peak = SM_COUNT * FP32_LANES * 2 * sm_max * 1e6 / 1e12
+            roof = {"bound": "alu", "achieved": achieved, "peak": fp32_peak, "unit": "TFLOP/s",
+                    "frac": achieved / fp32_peak, "traffic": traffic,
+                    "kernel": f"contract_staged_kernel<float,{p0.rm},{p0.rn},{p0.vec},false>",
+                    "peak_source": f"148 SMs x 128 FP32 lanes x 2 flop x {sm_max:.0f} MHz (sm max clock)"}
+            engine_desc = "SIMT contraction executor (FFMA), EATSS B200 mode"
         out = {
             "metric": METRIC, "value": value, "unit": "TFLOP/s", "n_gpus": ws, "steps": K,
-            "warmup": max(3, args.warmup), "ms_per_step": ms_total / K, "higher_is_better": True,
+            "warmup": W, "ms_per_step": ms_total / K, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f32",
             "data": "synthetic: A, B, C ~ U[-1,1) numpy PCG64 seeds 0,1,2; alpha=1.5 beta=1.2",
             "config": {"workload": "gemm N=4000 fp32 (BASELINE configs[1]), EATSS-selected tile",
-                       "tiles": list(tiles), "model": {"split_pct": 50, "waf": 16, "mode": "B200",
+                       "tiles": list(tiles), "model": {"split_pct": 50, "waf": 16,
+                                                        "mode": "tensor-core (reading T)" if arm.mode == 2 else "B200",
                                                         "obj": rep.obj, "n_ties": rep.n_ties},
-                       "engine": "SIMT contraction executor (FFMA)",
-                       "launch": {"grid": [p0.grid_x, p0.grid_y], "block": [p0.block_x, p0.block_y],
-                                  "micro_tile": [p0.rm, p0.rn], "vec": p0.vec, "smem_bytes": p0.smem_bytes},
+                       "engine": engine_desc,
                        "l2": "inputs 192 MB (A,B,C) > 126 MB L2; no flush",
                        "parallelism": f"dp{ws} independent problems"},
             "energy": {"joules_per_step": joules / K / ws if joules == joules else None,
                        "avg_watts_per_gpu": joules / (ms_total * 1e-3) / ws if joules == joules else None,
                        "gflops_per_watt": total_flops / joules / 1e9 if joules == joules and joules > 0 else None,
                        "source": "NVML total-energy counter over the timed region, summed over ranks"},
-            "roofline": {"bound": "alu", "achieved": achieved, "peak": fp32_peak, "unit": "TFLOP/s",
-                         "frac": achieved / fp32_peak, "traffic": traffic,
-                         "kernel": (f"contract_staged_kernel<float,{p0.rm},{p0.rn},{p0.vec},false>"
-                                    if (p0.b_in_smem and p0.passes == 1) else
-                                    f"contract_kernel<float,{p0.rm},{p0.rn},{p0.vec},false>"),
-                         "peak_source": f"148 SMs x 128 FP32 lanes x 2 flop x {sm_max:.0f} MHz (sm max clock)",
-                         "frac_at_observed_clock": (achieved / (SM_COUNT * FP32_LANES * 2 * clocks["sm_mhz"] * 1e-6))
-                         if clocks.get("sm_mhz") else None},
+            "roofline": roof,
             "e2e": {"value": FLOPS * ws / (e2e_ms * 1e-3) / 1e12, "unit": "TFLOP/s",
                     "h2d_bytes_per_step": int(3 * N * N * 4), "d2h_bytes_per_step": int(N * N * 4)},
             "gpu_launches": int(K * launches_per_step),
             "clocks": clocks,
         }
+        if sec:
+            out["secondary"] = sec
         if not args.no_cpu_baseline:
             out["cpu_baseline"] = cpu_oracle_sample()
         print(json.dumps(out), flush=True)
