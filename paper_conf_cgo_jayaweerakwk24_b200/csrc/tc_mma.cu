@@ -1,19 +1,31 @@
 // tc_mma.cu -- tcgen05 3xTF32 GEMM for MMA-legal tiles (the
-// "tensor-core EATSS mode"): Ti = 128 rows of i per CTA (UMMA M), Tj <= 256 columns of j
-// (UMMA N, multiple of 16), k in blocks of 32 (one 128-byte swizzle atom of fp32/tf32).
+// "tensor-core EATSS mode", DESIGN.md §2.5 / §4.1c): Ti = 128 rows of i per CTA (UMMA M per
+// SM), Tj <= 256 columns of j (UMMA N), k in blocks of 32 (one 128-byte swizzle atom of fp32).
 //
-// Same loop-nest semantics as the SIMT executor (Fig. 4: ti -> blockIdx.y,
-// tj -> blockIdx.x, k sequential); fp32-accurate via 3xTF32 (reading Q26):
+// Same loop-nest semantics as the SIMT executor (Fig. 4: each CTA owns one Ti x Tj
+// tile of C, k sequential); fp32-accurate via 3xTF32 (reading Q26):
 //   C = beta*C + alpha * sum_k (Ahi*Bhi + Ahi*Blo + Alo*Bhi),
 //   hi = rna_tf32(x), lo = rna_tf32(x - hi), computed once per operand by split_kernel.
+//
+// B200-specific structure (what differs from the paper's one-tile-per-block CUDA code):
+//  * CTA pairs (cta_group::2, cluster of 2 along i): the pair issues M = 256 MMAs; each CTA
+//    keeps its own 128 x Tj accumulator tile but stages only HALF of the B tile, so shared
+//    memory traffic per SM drops from 12 KB to 8 KB per MMA (the single-CTA kernel was
+//    shared-memory-bandwidth bound at ~74% tensor-pipe activity).  Used when Tj/2 is a whole
+//    number of 32-column swizzle atoms (or B is K-major); otherwise one CTA per tile.
+//  * persistent clusters over a grouped (L2-friendly) tile order; the accumulator is drained
+//    chunk by chunk (two TMEM buffers), so one tile's epilogue overlaps the next tile's MMAs.
+//  * wave-quantisation tail: when the last wave would leave clusters idle, the remaining tiles
+//    are split along k into `sp` parts whose partial sums are added to C with fp32 atomics
+//    (C pre-scaled by beta once by tail_prepass_kernel).
 // Pipeline (warp-specialised, mbarrier hand-off, one CTA per SM):
-//   warp 0  TMA producer: 2-D tensor-map loads (SWIZZLE_128B) of Ahi/Alo (K-major, 128 x 32)
-//           and Bhi/Blo (MN-major, 32 x Tj) into an S-stage ring;
-//   warp 1  MMA issuer: per 8-k step three kind::tf32 MMAs (M=128, N=Tj) from shared-memory
-//           descriptors into a TMEM accumulator; tcgen05.commit frees the ring slot;
-//   warps 4..11 epilogue: the k loop is split into chunks of R k-blocks accumulated in two
-//           alternating TMEM buffers (the tensor core accumulates with truncation); each
-//           chunk is drained with tcgen05.ld into fp32 registers, then C is updated.
+//   warp 0  TMA producer: Ahi/Alo (K-major, 128 x 32, SWIZZLE_128B) and Bhi/Blo (MN-major
+//           32 x Tj/CG in 32-column SWIZZLE_128B_ATOM_32B boxes, or K-major Tj/CG x 32 when B
+//           is transposed, as in syrk) into an S-stage ring;
+//   warp 1  MMA issuer (leader CTA only): per 8-k step three kind::tf32 MMAs;
+//           tcgen05.commit (multicast to the pair) frees ring slots / publishes chunks;
+//   warp 2  TMEM allocation (512 columns = two accumulator buffers of up to 256);
+//   warps 4..11 epilogue: tcgen05.ld of each finished chunk into fp32 registers, then C.
 #include <cuda.h>
 #include <cuda_runtime.h>
 
@@ -21,6 +33,7 @@
 #include <cstdint>
 #include <cstdlib>
 #include <mutex>
+#include <string>
 
 #include "contract.cuh"
 
@@ -28,6 +41,20 @@ namespace eatss {
 namespace tcm {
 
 __device__ __forceinline__ uint32_t su32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ uint32_t cta_rank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;\n" : "=r"(r));
+    return r;
+}
+// shared::cluster address of the same smem location in CTA `rank` of the cluster
+__device__ __forceinline__ uint32_t mapa(uint32_t a, uint32_t rank) {
+    uint32_t r;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;\n" : "=r"(r) : "r"(a), "r"(rank));
+    return r;
+}
+__device__ __forceinline__ void cluster_sync() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;\n" ::: "memory");
+}
 __device__ __forceinline__ void mbar_init(uint64_t *b, unsigned c) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(su32(b)), "r"(c) : "memory");
 }
@@ -37,6 +64,9 @@ __device__ __forceinline__ void mbar_expect_tx(uint64_t *b, unsigned bytes) {
 __device__ __forceinline__ void mbar_arrive(uint64_t *b) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(su32(b)) : "memory");
 }
+__device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_addr) {
+    asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];\n" ::"r"(cluster_addr) : "memory");
+}
 __device__ __forceinline__ void mbar_wait(uint64_t *b, unsigned parity) {
     asm volatile(
         "{\n.reg .pred p;\nW_%=:\n"
@@ -45,12 +75,30 @@ __device__ __forceinline__ void mbar_wait(uint64_t *b, unsigned parity) {
         "r"(parity)
         : "memory");
 }
-__device__ __forceinline__ void tma_2d(void *dst, const CUtensorMap *map, int c0, int c1, uint64_t *bar) {
+__device__ __forceinline__ void mbar_wait_cluster(uint64_t *b, unsigned parity) {
     asm volatile(
-        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];\n" ::"r"(
-            su32(dst)),
-        "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(su32(bar))
+        "{\n.reg .pred p;\nW_%=:\n"
+        "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%0], %1;\n"
+        "@!p bra W_%=;\n}\n" ::"r"(su32(b)),
+        "r"(parity)
         : "memory");
+}
+// 2-D TMA load into this CTA's smem; completion bytes signalled on `bar` (a shared::cluster
+// address: this CTA's barrier for CG = 1, the leader CTA's for CG = 2)
+template <int CG>
+__device__ __forceinline__ void tma_2d(void *dst, const CUtensorMap *map, int c0, int c1, uint32_t bar) {
+    if constexpr (CG == 1)
+        asm volatile(
+            "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];\n" ::"r"(
+                su32(dst)),
+            "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(bar)
+            : "memory");
+    else
+        asm volatile(
+            "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, "
+            "%3}], [%4];\n" ::"r"(su32(dst)),
+            "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(bar)
+            : "memory");
 }
 __device__ __forceinline__ void fence_before() { asm volatile("tcgen05.fence::before_thread_sync;\n" ::: "memory"); }
 __device__ __forceinline__ void fence_after() { asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory"); }
@@ -64,20 +112,38 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&v)[16]) {
         : "r"(taddr)
         : "memory");
 }
+template <int CG>
 __device__ __forceinline__ void mma_ss(uint32_t d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
-    asm volatile(
-        "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
-        "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(d),
-        "l"(a), "l"(b), "r"(idesc), "r"(acc)
-        : "memory");
+    if constexpr (CG == 1)
+        asm volatile(
+            "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
+            "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(d),
+            "l"(a), "l"(b), "r"(idesc), "r"(acc)
+            : "memory");
+    else
+        asm volatile(
+            "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
+            "tcgen05.mma.cta_group::2.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(d),
+            "l"(a), "l"(b), "r"(idesc), "r"(acc)
+            : "memory");
 }
+// arrive on `bar` (same smem offset in every CTA of the pair for CG = 2) when all prior MMAs finish
+template <int CG>
 __device__ __forceinline__ void mma_commit(uint64_t *bar) {
-    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(su32(bar))
-                 : "memory");
+    if constexpr (CG == 1)
+        asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(
+                         su32(bar))
+                     : "memory");
+    else
+        asm volatile(
+            "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;\n" ::"r"(
+                su32(bar)),
+            "h"((uint16_t)3)
+            : "memory");
 }
-// UMMA smem descriptor with SWIZZLE_128B (layout type 2), sm_100 version bit
-// layout type 2 = SWIZZLE_128B (K-major A), 1 = SWIZZLE_128B_BASE32B (the only smem layout
-// UMMA accepts for MN-major tf32 operands: 32-byte chunks XOR-swizzled over 4-row atoms)
+// UMMA smem descriptor, sm_100 version bit 46.  layout type 2 = SWIZZLE_128B (K-major
+// operands), 1 = SWIZZLE_128B_BASE32B (the only smem layout UMMA accepts for MN-major tf32:
+// 32-byte chunks XOR-swizzled over 4-row atoms)
 __device__ __forceinline__ uint64_t desc_sw128(const void *p, uint32_t lbo, uint32_t sbo, uint32_t layout = 2) {
     uint64_t d = 0;
     d |= (uint64_t)((su32(p) >> 4) & 0x3FFF);
@@ -87,15 +153,18 @@ __device__ __forceinline__ uint64_t desc_sw128(const void *p, uint32_t lbo, uint
     d |= (uint64_t)layout << 61;
     return d;
 }
-// kind::tf32: D f32, A tf32 K-major, B tf32 MN-major, M = 128, N = n
-__host__ __device__ constexpr uint32_t idesc(int n) {
-    return (1u << 4) | (2u << 7) | (2u << 10) | (1u << 16) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+// kind::tf32 instruction descriptor: D f32, A tf32 K-major, B tf32 (MN-major unless kmajor_b),
+// M = 128 * CG, N = n
+__host__ __device__ constexpr uint32_t idesc(int n, int cg, bool kmajor_b) {
+    return (1u << 4) | (2u << 7) | (2u << 10) | (kmajor_b ? 0u : (1u << 16)) | ((uint32_t)(n >> 3) << 17) |
+           ((uint32_t)((128 * cg) >> 4) << 24);
 }
 
-constexpr int BK = 32;         // k per stage (128-byte swizzle atom of fp32)
-constexpr int BM = 128;        // rows of i per CTA (UMMA M)
-constexpr int NEPI = 8;        // epilogue warps (4..11): two per TMEM lane quarter
+constexpr int BK = 32;   // k per stage (128-byte swizzle atom of fp32)
+constexpr int BM = 128;  // rows of i per CTA (UMMA M per SM)
+constexpr int NEPI = 8;  // epilogue warps (4..11): two per TMEM lane quarter
 constexpr int NTHREADS = (4 + NEPI) * 32;
+constexpr int GROUP_ROWS = 8;  // tile-order grouping (pair-rows per group) for L2 reuse
 
 struct Args {
     int64_t M, N, K;
@@ -103,37 +172,67 @@ struct Args {
     int64_t ldc;
     float alpha, beta;
     int init_zero;
-    int BN;   // Tj (multiple of 16, <= 256)
-    int S;    // ring stages
-    int R;    // k-blocks per accumulator chunk
-    int debug;
+    int S;   // ring stages
+    int R;   // k-blocks per accumulator chunk
+    // persistent schedule
+    int PI, TJ;   // row groups (of CG*128 rows) x column tiles
+    int T;        // PI * TJ tiles
+    int nfull;    // tiles done whole by one cluster
+    int sp;       // k-parts per tail tile (1 = no split)
+    int nunits;   // nfull + (T - nfull) * sp
+    int nkb;      // k-blocks of 32
 };
 
-template <int BNT>  // columns of j per CTA (compile-time: per-thread chunk sums live in registers)
+__host__ __device__ inline void tile_coords(int t, int PI, int TJ, int &pi, int &tj) {
+    const int g = t / (GROUP_ROWS * TJ), r = t % (GROUP_ROWS * TJ);
+    const int rows = PI - g * GROUP_ROWS < GROUP_ROWS ? PI - g * GROUP_ROWS : GROUP_ROWS;
+    pi = g * GROUP_ROWS + r % rows;
+    tj = r / rows;
+}
+
+struct Unit {
+    int pi, tj, kb0, kb1;
+    bool split;
+};
+__device__ __forceinline__ Unit unit_of(const Args &p, int u) {
+    Unit w;
+    int t;
+    if (u < p.nfull) {
+        t = u;
+        w.kb0 = 0;
+        w.kb1 = p.nkb;
+        w.split = false;
+    } else {
+        const int v = u - p.nfull, part = v % p.sp;
+        t = p.nfull + v / p.sp;
+        w.kb0 = (int)((int64_t)part * p.nkb / p.sp);
+        w.kb1 = (int)((int64_t)(part + 1) * p.nkb / p.sp);
+        w.split = p.sp > 1;
+    }
+    tile_coords(t, p.PI, p.TJ, w.pi, w.tj);
+    return w;
+}
+
+template <int BNT, bool TB, int CG>
 __global__ void __launch_bounds__(NTHREADS, 1)
     tc_mma_kernel(const __grid_constant__ CUtensorMap mAhi, const __grid_constant__ CUtensorMap mAlo,
                   const __grid_constant__ CUtensorMap mBhi, const __grid_constant__ CUtensorMap mBlo, const Args p) {
     extern __shared__ __align__(1024) unsigned char smem_raw[];
     unsigned char *smem = reinterpret_cast<unsigned char *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const int64_t i0 = (int64_t)blockIdx.y * BM, j0 = (int64_t)blockIdx.x * BNT;
-    const int nkb = (int)((p.K + BK - 1) / BK);
-    const int R = p.R, nchunks = (nkb + R - 1) / R;
-    constexpr int A_BYTES = BM * BK * 4;        // 16 KB
-    constexpr int B_BYTES = BK * BNT * 4;       // <= 32 KB
+    const uint32_t rank = CG == 2 ? cta_rank() : 0u;
+    const int cid = (int)blockIdx.x / CG, ncl = (int)gridDim.x / CG;
+    constexpr int BNH = BNT / CG;                // B columns (rows, if TB) staged by this CTA
+    constexpr int A_BYTES = BM * BK * 4;         // 16 KB
+    constexpr int B_BYTES = BK * BNH * 4;        // <= 32 KB
     constexpr int STAGE = 2 * A_BYTES + 2 * B_BYTES;
+    const int R = p.R;
     uint64_t *full = reinterpret_cast<uint64_t *>(smem + (size_t)p.S * STAGE);
     uint64_t *empty = full + p.S;
     uint64_t *dfull = empty + p.S;
     uint64_t *dempty = dfull + 2;
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(dempty + 2);
 
-    if (warp == 2) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;\n" ::"r"(su32(tmem_slot)),
-                     "r"(512)
-                     : "memory");
-        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;\n" ::: "memory");
-    }
     if (tid == 0) {
         for (int s = 0; s < p.S; s++) {
             mbar_init(full + s, 1);
@@ -141,154 +240,253 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         }
         for (int b = 0; b < 2; b++) {
             mbar_init(dfull + b, 1);
-            mbar_init(dempty + b, NEPI);
+            mbar_init(dempty + b, NEPI * CG);
         }
         asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
         asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&mAhi)) : "memory");
         asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&mBhi)) : "memory");
     }
+    if (warp == 2) {
+        if constexpr (CG == 1) {
+            asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;\n" ::"r"(su32(tmem_slot)),
+                         "r"(512)
+                         : "memory");
+            asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;\n" ::: "memory");
+        } else {
+            asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;\n" ::"r"(su32(tmem_slot)),
+                         "r"(512)
+                         : "memory");
+            asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;\n" ::: "memory");
+        }
+    }
     fence_before();
-    __syncthreads();
+    if constexpr (CG == 2) cluster_sync(); else __syncthreads();
     fence_after();
     const uint32_t tmem = *tmem_slot;
 
     if (warp == 0) {
         if (lane == 0) {  // ---------------------------------------------- TMA producer
-            for (int kb = 0; kb < nkb; kb++) {
-                const int s = kb % p.S;
-                if (kb >= p.S) mbar_wait(empty + s, (unsigned)(((kb / p.S) - 1) & 1));
-                unsigned char *st = smem + (size_t)s * STAGE;
-                mbar_expect_tx(full + s, STAGE);
-                const int k0 = kb * BK;
-                tma_2d(st, &mAhi, k0, (int)i0, full + s);
-                tma_2d(st + A_BYTES, &mAlo, k0, (int)i0, full + s);
+            const uint32_t fbar0 = CG == 2 ? mapa(su32(full), 0) : su32(full);
+            int it = 0;
+            for (int u = cid; u < p.nunits; u += ncl) {
+                const Unit w = unit_of(p, u);
+                const int i0 = (w.pi * CG + (int)rank) * BM;
+                const int jb = w.tj * BNT + (int)rank * BNH;
+                for (int kb = w.kb0; kb < w.kb1; kb++, it++) {
+                    const int s = it % p.S;
+                    if (it >= p.S) mbar_wait(empty + s, (unsigned)(((it / p.S) - 1) & 1));
+                    unsigned char *st = smem + (size_t)s * STAGE;
+                    if (rank == 0) mbar_expect_tx(full + s, CG * STAGE);
+                    const uint32_t fb = fbar0 + 8u * (uint32_t)s;
+                    const int k0 = kb * BK;
+                    tma_2d<CG>(st, &mAhi, k0, i0, fb);
+                    tma_2d<CG>(st + A_BYTES, &mAlo, k0, i0, fb);
+                    if constexpr (TB) {
+                        tma_2d<CG>(st + 2 * A_BYTES, &mBhi, k0, jb, fb);
+                        tma_2d<CG>(st + 2 * A_BYTES + B_BYTES, &mBlo, k0, jb, fb);
+                    } else {
 #pragma unroll
-                for (int g = 0; g < BNT / 32; g++) {
-                    tma_2d(st + 2 * A_BYTES + g * (BK * 128), &mBhi, (int)j0 + 32 * g, k0, full + s);
-                    tma_2d(st + 2 * A_BYTES + B_BYTES + g * (BK * 128), &mBlo, (int)j0 + 32 * g, k0, full + s);
+                        for (int g = 0; g < BNH / 32; g++) {
+                            tma_2d<CG>(st + 2 * A_BYTES + g * (BK * 128), &mBhi, jb + 32 * g, k0, fb);
+                            tma_2d<CG>(st + 2 * A_BYTES + B_BYTES + g * (BK * 128), &mBlo, jb + 32 * g, k0, fb);
+                        }
+                    }
                 }
             }
         }
     } else if (warp == 1) {
-        if (lane == 0) {  // ---------------------------------------------- MMA issuer
-            constexpr uint32_t ID = idesc(BNT);
-            // A: K-major SW128, SBO = 8 rows x 128 B.  B: MN-major SW128_BASE32B, LBO = stride of the
-            // 32-column groups (BK rows x 128 B), SBO = stride of the 4-row swizzle atoms (512 B)
-            constexpr uint32_t a_lbo = 16u, b_lbo = (uint32_t)(BK * 128), b_sbo = 512u;
-            for (int kb = 0; kb < nkb; kb++) {
-                const int s = kb % p.S;
-                const int ch = kb / R, bd = ch & 1;
-                const bool first = (kb % R) == 0;
-                if (first && ch >= 2) mbar_wait(dempty + bd, (unsigned)(((ch - 2) >> 1) & 1));
-                mbar_wait(full + s, (unsigned)((kb / p.S) & 1));
-                fence_after();
-                unsigned char *st = smem + (size_t)s * STAGE;
-                if (p.debug && kb == 0 && blockIdx.x == 0 && blockIdx.y == 0) {
-                    // debug: dump raw stage words (Ahi then Bhi) into C's first row(s)
-                    const float *w = reinterpret_cast<const float *>(st);
-                    for (int x = 0; x < 256; x++) p.C[x] = w[x];
-                    const float *wb = reinterpret_cast<const float *>(st + 2 * A_BYTES);
-                    for (int x = 0; x < 256; x++) p.C[256 + x] = wb[x];
-                }
-                const uint32_t d = tmem + (uint32_t)(bd * 256);
+        if (lane == 0 && rank == 0) {  // -------------------------------- MMA issuer (leader)
+            constexpr uint32_t ID = idesc(BNT, CG, TB);
+            // A (and K-major B): SW128 K-major, SBO = 8 rows x 128 B, +32 B per 8-k step.
+            // MN-major B: SW128_BASE32B, LBO = stride of 32-column groups (BK rows x 128 B),
+            // SBO = stride of the 4-row swizzle atoms (512 B), +1 KB per 8-k step.
+            int it = 0, gc = 0;
+            for (int u = cid; u < p.nunits; u += ncl) {
+                const Unit w = unit_of(p, u);
+                const int nk = w.kb1 - w.kb0;
+                for (int x = 0; x < nk; x++, it++) {
+                    const int s = it % p.S, bd = gc & 1;
+                    const bool first = (x % R) == 0;
+                    if (first && gc >= 2) mbar_wait_cluster(dempty + bd, (unsigned)(((gc - 2) >> 1) & 1));
+                    mbar_wait(full + s, (unsigned)((it / p.S) & 1));
+                    fence_after();
+                    unsigned char *st = smem + (size_t)s * STAGE;
+                    const uint32_t d = tmem + (uint32_t)(bd * 256);
 #pragma unroll
-                for (int ks = 0; ks < BK / 8; ks++) {
-                    // A K-major: 8 tf32 = 32 B into each 128-B row; B MN-major: one 8-k atom = 1 KB
-                    const uint64_t ahi = desc_sw128(st + ks * 32, a_lbo, 1024);
-                    const uint64_t alo = desc_sw128(st + A_BYTES + ks * 32, a_lbo, 1024);
-                    const uint64_t bhi = desc_sw128(st + 2 * A_BYTES + ks * 1024, b_lbo, b_sbo, 1);
-                    const uint64_t blo = desc_sw128(st + 2 * A_BYTES + B_BYTES + ks * 1024, b_lbo, b_sbo, 1);
-                    mma_ss(d, ahi, bhi, ID, (first && ks == 0) ? 0u : 1u);
-                    mma_ss(d, ahi, blo, ID, 1u);
-                    mma_ss(d, alo, bhi, ID, 1u);
+                    for (int ks = 0; ks < BK / 8; ks++) {
+                        const uint64_t ahi = desc_sw128(st + ks * 32, 16u, 1024u);
+                        const uint64_t alo = desc_sw128(st + A_BYTES + ks * 32, 16u, 1024u);
+                        uint64_t bhi, blo;
+                        if constexpr (TB) {
+                            bhi = desc_sw128(st + 2 * A_BYTES + ks * 32, 16u, 1024u);
+                            blo = desc_sw128(st + 2 * A_BYTES + B_BYTES + ks * 32, 16u, 1024u);
+                        } else {
+                            bhi = desc_sw128(st + 2 * A_BYTES + ks * 1024, (uint32_t)(BK * 128), 512u, 1);
+                            blo = desc_sw128(st + 2 * A_BYTES + B_BYTES + ks * 1024, (uint32_t)(BK * 128), 512u, 1);
+                        }
+                        mma_ss<CG>(d, ahi, bhi, ID, (first && ks == 0) ? 0u : 1u);
+                        mma_ss<CG>(d, ahi, blo, ID, 1u);
+                        mma_ss<CG>(d, alo, bhi, ID, 1u);
+                    }
+                    mma_commit<CG>(empty + s);
+                    if ((x % R) == R - 1 || x == nk - 1) {
+                        mma_commit<CG>(dfull + bd);
+                        gc++;
+                    }
                 }
-                mma_commit(empty + s);
-                if ((kb % R) == R - 1 || kb == nkb - 1) mma_commit(dfull + bd);
             }
         }
     } else if (warp >= 4) {  // ---------------------------------------- epilogue warps
         const int e = warp - 4, q = warp & 3, half = e >> 2;
         constexpr int CW = BNT / 2;  // columns per epilogue warp
-        float acc[CW];
+        const uint32_t demp0 = CG == 2 ? mapa(su32(dempty), 0) : su32(dempty);
+        int gc = 0;
+        for (int u = cid; u < p.nunits; u += ncl) {
+            const Unit w = unit_of(p, u);
+            const int nch = (w.kb1 - w.kb0 + R - 1) / R;
+            float acc[CW];
 #pragma unroll
-        for (int c = 0; c < CW; c++) acc[c] = 0.f;
-        for (int ch = 0; ch < nchunks; ch++) {
-            const int bd = ch & 1;
-            mbar_wait(dfull + bd, (unsigned)((ch >> 1) & 1));
-            fence_after();
+            for (int c = 0; c < CW; c++) acc[c] = 0.f;
+            for (int ch = 0; ch < nch; ch++, gc++) {
+                const int bd = gc & 1;
+                mbar_wait(dfull + bd, (unsigned)((gc >> 1) & 1));
+                fence_after();
 #pragma unroll
-            for (int c0 = 0; c0 < CW; c0 += 16) {
-                uint32_t v[16];
-                tmem_ld16(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(bd * 256 + half * CW + c0), v);
-                wait_ld();
+                for (int c0 = 0; c0 < CW; c0 += 16) {
+                    uint32_t v[16];
+                    tmem_ld16(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(bd * 256 + half * CW + c0), v);
+                    wait_ld();
 #pragma unroll
-                for (int c = 0; c < 16; c++) acc[c0 + c] += __uint_as_float(v[c]);
-            }
-            fence_before();
-            __syncwarp();
-            if (lane == 0) mbar_arrive(dempty + bd);
-        }
-        // C = beta*C + alpha*acc for row i = i0 + 32q + lane, columns j0 + half*CW + c
-        const int64_t i = i0 + q * 32 + lane;
-        if (i < p.M && !(p.debug && i < 16)) {
-            float *crow = p.C + i * p.ldc + j0 + half * CW;
-            const int64_t jb = j0 + half * CW;
-            const bool vec = ((p.ldc & 3) == 0) && (jb + CW <= p.N);
-            if (vec) {
-#pragma unroll
-                for (int c = 0; c < CW; c += 4) {
-                    float4 *cp = reinterpret_cast<float4 *>(crow + c);
-                    float4 o = p.init_zero ? make_float4(0.f, 0.f, 0.f, 0.f) : *cp;
-                    if (!p.init_zero) { o.x *= p.beta; o.y *= p.beta; o.z *= p.beta; o.w *= p.beta; }
-                    o.x = fmaf(p.alpha, acc[c], o.x);
-                    o.y = fmaf(p.alpha, acc[c + 1], o.y);
-                    o.z = fmaf(p.alpha, acc[c + 2], o.z);
-                    o.w = fmaf(p.alpha, acc[c + 3], o.w);
-                    *cp = o;
+                    for (int c = 0; c < 16; c++) acc[c0 + c] += __uint_as_float(v[c]);
                 }
-            } else {
+                fence_before();
+                __syncwarp();
+                if (lane == 0) {
+                    if constexpr (CG == 2) mbar_arrive_cluster(demp0 + 8u * (uint32_t)bd);
+                    else mbar_arrive(dempty + bd);
+                }
+            }
+            // C(i, j) for row i = i0 + 32q + lane, columns jb .. jb + CW - 1
+            const int64_t i = (int64_t)(w.pi * CG + (int)rank) * BM + q * 32 + lane;
+            const int64_t jb = (int64_t)w.tj * BNT + half * CW;
+            if (i < p.M && jb < p.N) {
+                float *crow = p.C + i * p.ldc + jb;
+                const bool vec = ((p.ldc & 3) == 0) && (jb + CW <= p.N);
+                if (w.split) {  // C already holds beta*C (tail_prepass_kernel): add the partial sum
+                    if (vec) {
 #pragma unroll
-                for (int c = 0; c < CW; c++) {
-                    if (jb + c < p.N) {
-                        const float o = p.init_zero ? 0.f : p.beta * crow[c];
-                        crow[c] = fmaf(p.alpha, acc[c], o);
+                        for (int c = 0; c < CW; c += 4)
+                            atomicAdd(reinterpret_cast<float4 *>(crow + c),
+                                      make_float4(p.alpha * acc[c], p.alpha * acc[c + 1], p.alpha * acc[c + 2],
+                                                  p.alpha * acc[c + 3]));
+                    } else {
+#pragma unroll
+                        for (int c = 0; c < CW; c++)
+                            if (jb + c < p.N) atomicAdd(crow + c, p.alpha * acc[c]);
+                    }
+                } else if (vec) {
+#pragma unroll
+                    for (int c = 0; c < CW; c += 4) {
+                        float4 *cp = reinterpret_cast<float4 *>(crow + c);
+                        float4 o = p.init_zero ? make_float4(0.f, 0.f, 0.f, 0.f) : *cp;
+                        if (!p.init_zero) { o.x *= p.beta; o.y *= p.beta; o.z *= p.beta; o.w *= p.beta; }
+                        o.x = fmaf(p.alpha, acc[c], o.x);
+                        o.y = fmaf(p.alpha, acc[c + 1], o.y);
+                        o.z = fmaf(p.alpha, acc[c + 2], o.z);
+                        o.w = fmaf(p.alpha, acc[c + 3], o.w);
+                        *cp = o;
+                    }
+                } else {
+#pragma unroll
+                    for (int c = 0; c < CW; c++) {
+                        if (jb + c < p.N) {
+                            const float o = p.init_zero ? 0.f : p.beta * crow[c];
+                            crow[c] = fmaf(p.alpha, acc[c], o);
+                        }
                     }
                 }
             }
         }
     }
+    __syncwarp();
     fence_before();
-    __syncthreads();
+    if constexpr (CG == 2) cluster_sync(); else __syncthreads();
     if (warp == 2) {
         fence_after();
-        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;\n" ::"r"(tmem), "r"(512) : "memory");
+        if constexpr (CG == 1)
+            asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;\n" ::"r"(tmem), "r"(512) : "memory");
+        else
+            asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;\n" ::"r"(tmem), "r"(512) : "memory");
     }
 }
 
-// hi = rna_tf32(x), lo = rna_tf32(x - hi)  (elementwise, 16-byte vectors)
-__global__ void split_kernel(const float *__restrict__ x, float *__restrict__ hi, float *__restrict__ lo, int64_t n) {
-    const int64_t n4 = n / 4;
-    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n4; v += (int64_t)gridDim.x * blockDim.x) {
-        const float4 a = reinterpret_cast<const float4 *>(x)[v];
-        float4 h, l;
-        float *ap = (float *)&a, *hp = (float *)&h, *lp = (float *)&l;
-#pragma unroll
-        for (int q = 0; q < 4; q++) {
-            uint32_t hb, lb;
-            asm("cvt.rna.tf32.f32 %0, %1;\n" : "=r"(hb) : "f"(ap[q]));
-            asm("cvt.rna.tf32.f32 %0, %1;\n" : "=r"(lb) : "f"(ap[q] - __uint_as_float(hb)));
-            hp[q] = __uint_as_float(hb);
-            lp[q] = __uint_as_float(lb);
+// C := init_zero ? 0 : beta*C over the tiles that are split along k (their parts then add
+// alpha * partial sums atomically).  One CTA per (tail tile, 8-row slab).
+__global__ void tail_prepass_kernel(const Args p, int rows_per_tile, int bn) {
+    const int ntail = p.T - p.nfull;
+    const int slabs = rows_per_tile / 8;
+    for (int b = blockIdx.x; b < ntail * slabs; b += gridDim.x) {
+        int pi, tj;
+        tile_coords(p.nfull + b / slabs, p.PI, p.TJ, pi, tj);
+        const int64_t r0 = (int64_t)pi * rows_per_tile + (b % slabs) * 8, j0 = (int64_t)tj * bn;
+        for (int x = threadIdx.x; x < 8 * bn; x += blockDim.x) {
+            const int64_t i = r0 + x / bn, j = j0 + x % bn;
+            if (i < p.M && j < p.N) {
+                float *c = p.C + i * p.ldc + j;
+                *c = p.init_zero ? 0.f : p.beta * *c;
+            }
         }
-        reinterpret_cast<float4 *>(hi)[v] = h;
-        reinterpret_cast<float4 *>(lo)[v] = l;
     }
-    for (int64_t t = n4 * 4 + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < n; t += (int64_t)gridDim.x * blockDim.x) {
-        uint32_t hb, lb;
-        asm("cvt.rna.tf32.f32 %0, %1;\n" : "=r"(hb) : "f"(x[t]));
-        asm("cvt.rna.tf32.f32 %0, %1;\n" : "=r"(lb) : "f"(x[t] - __uint_as_float(hb)));
-        hi[t] = __uint_as_float(hb);
-        lo[t] = __uint_as_float(lb);
+}
+
+// Operand split for 3xTF32 (reading Q26).  mode 0: hi = rna_tf32(x), lo = rna_tf32(x - hi).
+// mode 1 ("raw hi"): the tensor core reads only the tf32 bits of an fp32 container (it truncates),
+// so the untouched operand already serves as hi = rz_tf32(x) and only lo = rna_tf32(x - rz_tf32(x))
+// is materialised (hi == nullptr) -- one third less split traffic.  Rows of `cols` values at
+// pitch ldx are written at pitch ldp (ldp = ldx: flat 16-byte vectors; else padded scalar copy).
+__device__ __forceinline__ void split1(float v, int mode, float &h, float &l) {
+    uint32_t hb, lb;
+    if (mode == 0) {
+        asm("cvt.rna.tf32.f32 %0, %1;\n" : "=r"(hb) : "f"(v));
+    } else {
+        hb = __float_as_uint(v) & 0xFFFFE000u;
+    }
+    asm("cvt.rna.tf32.f32 %0, %1;\n" : "=r"(lb) : "f"(v - __uint_as_float(hb)));
+    h = mode == 0 ? __uint_as_float(hb) : v;
+    l = __uint_as_float(lb);
+}
+__global__ void split_kernel(const float *__restrict__ x, int64_t ldx, int64_t rows, int64_t cols,
+                             float *__restrict__ hi, float *__restrict__ lo, int64_t ldp, int mode) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x, t0 = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (ldx == ldp) {  // flat over (rows - 1) * ld + cols elements
+        const int64_t n = (rows - 1) * ldx + cols;
+        const bool v4 = ((reinterpret_cast<uintptr_t>(x) | reinterpret_cast<uintptr_t>(lo) |
+                          reinterpret_cast<uintptr_t>(hi)) & 15) == 0;
+        const int64_t n4 = v4 ? n / 4 : 0;
+        for (int64_t v = t0; v < n4; v += stride) {
+            const float4 a = reinterpret_cast<const float4 *>(x)[v];
+            float4 h, l;
+            split1(a.x, mode, h.x, l.x);
+            split1(a.y, mode, h.y, l.y);
+            split1(a.z, mode, h.z, l.z);
+            split1(a.w, mode, h.w, l.w);
+            if (hi) reinterpret_cast<float4 *>(hi)[v] = h;
+            reinterpret_cast<float4 *>(lo)[v] = l;
+        }
+        for (int64_t e = n4 * 4 + t0; e < n; e += stride) {
+            float h, l;
+            split1(x[e], mode, h, l);
+            if (hi) hi[e] = h;
+            lo[e] = l;
+        }
+    } else {
+        for (int64_t e = t0; e < rows * ldp; e += stride) {
+            const int64_t r = e / ldp, c = e % ldp;
+            float h = 0.f, l = 0.f;
+            if (c < cols) split1(x[r * ldx + c], mode, h, l);
+            hi[e] = h;
+            lo[e] = l;
+        }
     }
 }
 
@@ -354,69 +552,170 @@ static float *workspace(size_t elems) {
     return g_ws;
 }
 
-static int tcm_stages(int bn) {
-    const int stage = 2 * tcm::BM * tcm::BK * 4 + 2 * tcm::BK * bn * 4;
-    int S = (int)((232448 - 2048) / stage);
+// CTA pairs whenever each CTA's half of the B tile is whole swizzle atoms (EATSS_TCM_PAIR=0 disables)
+static int tcm_cg(const ContractNest &n, int bn) {
+    static const int env = getenv("EATSS_TCM_PAIR") ? atoi(getenv("EATSS_TCM_PAIR")) : 1;
+    if (!env) return 1;
+    return n.transB ? ((bn / 2) % 8 == 0 ? 2 : 1) : ((bn / 2) % 32 == 0 ? 2 : 1);
+}
+static int tcm_stage_bytes(int bn, int cg) { return 2 * tcm::BM * tcm::BK * 4 + 2 * tcm::BK * (bn / cg) * 4; }
+static int tcm_stages(int bn, int cg) {
+    int S = (int)((232448 - 2048) / tcm_stage_bytes(bn, cg));
     if (const char *e = getenv("EATSS_TCM_STAGES")) S = atoi(e);
     return std::max(2, std::min(S, 8));
 }
 
 bool tcm_applicable(const ContractNest &n, const ContractPlan &p) {
-    if (n.f64 || n.transB) return false;
+    if (n.f64) return false;
     if (p.Ti != tcm::BM || p.Tj < 32 || p.Tj > 256 || (p.Tj % 32) != 0) return false;
-    if ((n.lda % 4) || (n.ldb % 4)) return false;
-    if (n.M > INT32_MAX || n.N > INT32_MAX || n.K > INT32_MAX) return false;
-    const int stage = 2 * tcm::BM * tcm::BK * 4 + 2 * tcm::BK * (int)p.Tj * 4;
-    return 2 * stage + 2048 <= 232448 && tcm::encode_fn() != nullptr;
+    if (n.M > INT32_MAX / 2 || n.N > INT32_MAX / 2 || n.K > INT32_MAX / 2) return false;
+    return 2 * tcm_stage_bytes((int)p.Tj, 1) + 2048 <= 232448 && tcm::encode_fn() != nullptr;
 }
+
+template <int BN, bool TB, int CG>
+static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int nsm, cudaStream_t s) {
+    auto k = tcm::tc_mma_kernel<BN, TB, CG>;
+    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    // persistent: as many clusters as fit at once (one CTA per SM), never more than tiles
+    int ncl = nsm / CG;
+    cudaLaunchConfig_t cfg = {};
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = CG;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.blockDim = dim3(tcm::NTHREADS);
+    cfg.dynamicSmemBytes = (size_t)smem;
+    cfg.stream = s;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    if (CG == 2) {
+        cfg.gridDim = dim3((unsigned)(2 * ncl));
+        int active = 0;
+        if (cudaOccupancyMaxActiveClusters(&active, k, &cfg) == cudaSuccess && active > 0) ncl = std::min(ncl, active);
+        cudaGetLastError();
+    }
+    // schedule: full tiles in waves of ncl, the last partial wave split along k
+    a.T = a.PI * a.TJ;
+    ncl = std::max(1, std::min(ncl, a.T));
+    const int rem = a.T % ncl;
+    a.sp = 1;
+    a.nfull = a.T;
+    if (const char *ev = getenv("EATSS_TCM_SPLITK"); rem > 0 && !(ev && atoi(ev) == 0)) {
+        const int sp = std::min(std::min(4, ncl / rem), a.nkb);
+        if (sp >= 2) {
+            a.sp = sp;
+            a.nfull = a.T - rem;
+        }
+    }
+    a.nunits = a.nfull + (a.T - a.nfull) * a.sp;
+    if (a.sp > 1 && (a.init_zero || a.beta != 1.f)) {
+        tcm::tail_prepass_kernel<<<std::min(4096, (a.T - a.nfull) * (CG * tcm::BM / 8)), 256, 0, s>>>(
+            a, CG * tcm::BM, BN);
+        if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    }
+    cfg.gridDim = dim3((unsigned)(CG * ncl));
+    return cudaLaunchKernelEx(&cfg, k, m[0], m[1], m[2], m[3], a);
+}
+
+template <bool TB, int CG>
+static cudaError_t launch_bn(int bn, const CUtensorMap *m, const tcm::Args &a, int smem, int nsm, cudaStream_t s) {
+    switch (bn) {
+        case 32: return launch_one<32, TB, CG>(m, a, smem, nsm, s);
+        case 64: return launch_one<64, TB, CG>(m, a, smem, nsm, s);
+        case 96: return launch_one<96, TB, CG>(m, a, smem, nsm, s);
+        case 128: return launch_one<128, TB, CG>(m, a, smem, nsm, s);
+        case 160: return launch_one<160, TB, CG>(m, a, smem, nsm, s);
+        case 192: return launch_one<192, TB, CG>(m, a, smem, nsm, s);
+        case 224: return launch_one<224, TB, CG>(m, a, smem, nsm, s);
+        case 256: return launch_one<256, TB, CG>(m, a, smem, nsm, s);
+        default: return cudaErrorNotSupported;
+    }
+}
+
+namespace {
+struct Operand {
+    const float *x;  // source, rows x cols at pitch ld
+    int64_t rows, cols, ld;
+    const float *hi = nullptr, *lo = nullptr;  // split halves handed to TMA
+    int64_t ldp = 0;
+    bool raw_hi = false;  // hi is the source itself (mode 1, aligned)
+    int64_t need = 0;     // workspace elements
+};
+int split_mode() {
+    static const int m = [] {
+        const char *e = getenv("EATSS_TCM_SPLIT");
+        return e && std::string(e) == "rna" ? 0 : 1;
+    }();
+    return m;
+}
+void size_operand(Operand &o, int mode) {
+    const bool aligned = (o.ld % 4) == 0 && (reinterpret_cast<uintptr_t>(o.x) & 15) == 0;
+    o.ldp = aligned ? o.ld : (o.cols + 3) / 4 * 4;
+    o.raw_hi = aligned && mode == 1;
+    const int64_t span = aligned ? (o.rows - 1) * o.ld + o.cols : o.rows * o.ldp;
+    o.need = (o.raw_hi ? 1 : 2) * ((span + 3) / 4 * 4);
+}
+void split_operand(Operand &o, float *ws, int mode, cudaStream_t s) {
+    const int64_t span = o.need / (o.raw_hi ? 1 : 2);
+    float *lo = ws, *hi = o.raw_hi ? nullptr : ws + span;
+    tcm::split_kernel<<<148 * 8, 256, 0, s>>>(o.x, o.ld, o.rows, o.cols, hi, lo, o.ldp, mode);
+    o.lo = lo;
+    o.hi = o.raw_hi ? o.x : hi;
+}
+}  // namespace
 
 cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p, cudaStream_t s) {
     if (!tcm_applicable(n, p)) return cudaErrorNotSupported;
-    const int64_t a_elems = n.M * n.lda, b_elems = n.K * n.ldb;
-    float *ws = workspace((size_t)(2 * a_elems + 2 * b_elems + 64));
-    if (!ws) return cudaErrorMemoryAllocation;
-    float *Ahi = ws, *Alo = Ahi + a_elems, *Bhi = Alo + a_elems, *Blo = Bhi + b_elems;
+    const int bn = (int)p.Tj, cg = tcm_cg(n, bn), mode = split_mode();
     const float *A = static_cast<const float *>(n.A), *B = static_cast<const float *>(n.B);
-    tcm::split_kernel<<<148 * 8, 256, 0, s>>>(A, Ahi, Alo, a_elems);
-    tcm::split_kernel<<<148 * 8, 256, 0, s>>>(B, Bhi, Blo, b_elems);
+    Operand oa{A, n.M, n.K, n.lda}, ob{B, n.transB ? n.N : n.K, n.transB ? n.K : n.N, n.ldb};
+    size_operand(oa, mode);
+    size_operand(ob, mode);
+    // syrk: A is a row block of B (both row-major over k) -> split B once and point into it
+    const bool share = n.transB && n.lda == n.ldb && A >= B && (A - B) % n.ldb == 0 &&
+                       (A - B) / n.ldb + n.M <= ob.rows;
+    float *ws = workspace((size_t)(ob.need + (share ? 0 : oa.need) + 64));
+    if (!ws) return cudaErrorMemoryAllocation;
+    split_operand(ob, ws, mode, s);
+    if (share) {
+        const int64_t r = (A - B) / n.ldb;
+        oa.hi = ob.hi + r * ob.ldp;
+        oa.lo = ob.lo + r * ob.ldp;
+        oa.ldp = ob.ldp;
+    } else {
+        split_operand(oa, ws + ob.need, mode, s);
+    }
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
-    CUtensorMap mAhi, mAlo, mBhi, mBlo;
-    const int bn = (int)p.Tj;
-    const CUtensorMapSwizzle swA = CU_TENSOR_MAP_SWIZZLE_128B, swB = CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B;
-    if (!tcm::make_map(&mAhi, Ahi, n.M, n.K, n.lda, tcm::BK, tcm::BM, swA) ||
-        !tcm::make_map(&mAlo, Alo, n.M, n.K, n.lda, tcm::BK, tcm::BM, swA) ||
-        !tcm::make_map(&mBhi, Bhi, n.K, n.N, n.ldb, 32, tcm::BK, swB) ||
-        !tcm::make_map(&mBlo, Blo, n.K, n.N, n.ldb, 32, tcm::BK, swB))
-        return cudaErrorInvalidValue;
+    CUtensorMap m[4];
+    const CUtensorMapSwizzle swK = CU_TENSOR_MAP_SWIZZLE_128B, swMN = CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B;
+    bool ok = tcm::make_map(&m[0], oa.hi, n.M, n.K, oa.ldp, tcm::BK, tcm::BM, swK) &&
+              tcm::make_map(&m[1], oa.lo, n.M, n.K, oa.ldp, tcm::BK, tcm::BM, swK);
+    if (n.transB)  // B(k, j) = B[j*ldb + k]: rows j, K-major boxes of bn/cg rows x 32 k
+        ok = ok && tcm::make_map(&m[2], ob.hi, n.N, n.K, ob.ldp, tcm::BK, bn / cg, swK) &&
+             tcm::make_map(&m[3], ob.lo, n.N, n.K, ob.ldp, tcm::BK, bn / cg, swK);
+    else  // B(k, j) = B[k*ldb + j]: MN-major boxes of 32 k x 32 j
+        ok = ok && tcm::make_map(&m[2], ob.hi, n.K, n.N, ob.ldp, 32, tcm::BK, swMN) &&
+             tcm::make_map(&m[3], ob.lo, n.K, n.N, ob.ldp, 32, tcm::BK, swMN);
+    if (!ok) return cudaErrorInvalidValue;
     tcm::Args a;
     a.M = n.M; a.N = n.N; a.K = n.K;
     a.C = static_cast<float *>(n.C); a.ldc = n.ldc;
     a.alpha = (float)n.alpha; a.beta = (float)n.beta; a.init_zero = n.init_zero ? 1 : 0;
-    a.BN = bn;
-    a.S = tcm_stages(bn);
+    a.S = tcm_stages(bn, cg);
     a.R = 16;  // 16 k-blocks = 512 k per accumulator chunk
     if (const char *ev = getenv("EATSS_TCM_CHUNK")) a.R = std::max(1, atoi(ev));
-    a.debug = getenv("EATSS_TCM_DEBUG") ? atoi(getenv("EATSS_TCM_DEBUG")) : 0;
-    const int stage = 2 * tcm::BM * tcm::BK * 4 + 2 * tcm::BK * bn * 4;
-    const int smem = a.S * stage + 1024 /*align*/ + 8 * (2 * a.S + 4) + 16;
-    void (*k)(const CUtensorMap, const CUtensorMap, const CUtensorMap, const CUtensorMap, const tcm::Args) = nullptr;
-    switch (bn) {
-        case 32: k = tcm::tc_mma_kernel<32>; break;
-        case 64: k = tcm::tc_mma_kernel<64>; break;
-        case 96: k = tcm::tc_mma_kernel<96>; break;
-        case 128: k = tcm::tc_mma_kernel<128>; break;
-        case 160: k = tcm::tc_mma_kernel<160>; break;
-        case 192: k = tcm::tc_mma_kernel<192>; break;
-        case 224: k = tcm::tc_mma_kernel<224>; break;
-        case 256: k = tcm::tc_mma_kernel<256>; break;
-        default: return cudaErrorNotSupported;
-    }
-    e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    if (e != cudaSuccess) return e;
-    dim3 grid((unsigned)((n.N + bn - 1) / bn), (unsigned)((n.M + tcm::BM - 1) / tcm::BM));
-    k<<<grid, tcm::NTHREADS, smem, s>>>(mAhi, mAlo, mBhi, mBlo, a);
-    return cudaGetLastError();
+    a.nkb = (int)((n.K + tcm::BK - 1) / tcm::BK);
+    a.PI = (int)((n.M + cg * tcm::BM - 1) / (cg * tcm::BM));
+    a.TJ = (int)((n.N + bn - 1) / bn);
+    const int smem = a.S * tcm_stage_bytes(bn, cg) + 1024 /*align*/ + 8 * (2 * a.S + 4) + 16;
+    int dev = 0, nsm = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    if (n.transB) return cg == 2 ? launch_bn<true, 2>(bn, m, a, smem, nsm, s) : launch_bn<true, 1>(bn, m, a, smem, nsm, s);
+    return cg == 2 ? launch_bn<false, 2>(bn, m, a, smem, nsm, s) : launch_bn<false, 1>(bn, m, a, smem, nsm, s);
 }
 
 }  // namespace eatss

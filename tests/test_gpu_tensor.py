@@ -115,3 +115,93 @@ def test_tcm_full_size_sampled(cuda_device):
     g = synth.rng(7)
     ii = g.integers(0, n, 2048); jj = g.integers(0, n, 2048)
     assert O.normwise_rel_err(out[ii, jj], O.gemm_entries(ii, jj, C, A, B, 1.5, 1.2)) <= 1e-5
+
+
+# ---- syrk on the tensor pipe: B(k, j) = A(j, k) is K-major (same operand layout as A)
+SYRK_TILES = [(128, 256, 32), (128, 224, 16), (128, 96, 32), (128, 32, 8)]
+
+
+@pytest.mark.parametrize("tiles", SYRK_TILES)
+def test_tcm_syrk_small_int_exact_and_random(cuda_device, tiles):
+    ni, nj = 403, 157  # odd pitch: operands are re-pitched to 16-byte rows for TMA
+    Ai = synth.small_int((ni, nj), 72); Ci = synth.small_int((ni, ni), 73)
+    d = E.desc_builtin("syrk", (ni, nj)); d.set_scalars(1.0, 1.0); d.set_exec(50, TENSOR)
+    Cd = dev(Ci)
+    E.run(d, tiles, [Cd, dev(Ai)])
+    assert np.array_equal(host(Cd), O.syrk(1.0, 1.0, Ci, Ai))
+    A = synth.uniform((ni, nj), 70); C = synth.uniform((ni, ni), 71)
+    d.set_scalars(1.5, 1.2)
+    Cd = dev(C)
+    E.run(d, tiles, [Cd, dev(A)])
+    assert O.normwise_rel_err(host(Cd), O.syrk(1.5, 1.2, C, A)) <= 1e-5
+
+
+def test_tcm_syrk_row_block(cuda_device):
+    # rows [r0, r0 + rows) of C only (the multi-GPU shard form): A operand is a row block of B
+    ni, nj, r0, rows = 300, 200, 77, 150
+    A = synth.uniform((ni, nj), 80); C = synth.uniform((ni, ni), 81)
+    ref = O.syrk(1.5, 1.2, C, A)
+    d = E.desc_builtin("syrk", (ni, nj, r0, rows)); d.set_scalars(1.5, 1.2); d.set_exec(50, TENSOR)
+    Cb = dev(C[r0:r0 + rows])
+    E.run(d, (128, 128, 32), [Cb, dev(A)])
+    assert O.normwise_rel_err(host(Cb), ref[r0:r0 + rows]) <= 1e-5
+
+
+def test_tcm_syrk_full_size_sampled(cuda_device):
+    n = 4000
+    A = synth.uniform((n, n), 8); C = synth.uniform((n, n), 9)
+    d = E.desc_builtin("syrk", (n, n)); d.set_scalars(1.5, 1.2); d.set_exec(50, TENSOR)
+    Cd = dev(C)
+    E.run(d, (128, 256, 32), [Cd, dev(A)])
+    out = host(Cd)
+    g = synth.rng(10)
+    ii = g.integers(0, n, 2048); jj = g.integers(0, n, 2048)
+    want = O.gemm_entries(ii, jj, C, A, np.ascontiguousarray(A.T), 1.5, 1.2)
+    assert O.normwise_rel_err(out[ii, jj], want) <= 1e-5
+
+
+@pytest.mark.parametrize("splitk", ["0", "1"])
+def test_tcm_tail_split_on_and_off(cuda_device, monkeypatch, splitk):
+    # 600 x 1300 with (128, 256): 3 pair-rows x 6 column tiles = 18 tiles < the clusters of one
+    # wave, so with split-k on every tile is split along k (atomics on a beta-prescaled C)
+    monkeypatch.setenv("EATSS_TCM_SPLITK", splitk)
+    ni, nj, nk = 600, 1300, 2000
+    A = synth.small_int((ni, nk), 30); B = synth.small_int((nk, nj), 31); C = synth.small_int((ni, nj), 32)
+    d = E.desc_builtin("gemm", (ni, nj, nk)); d.set_scalars(1.0, 2.0); d.set_exec(50, TENSOR)
+    Cd = dev(C)
+    E.run(d, (128, 256, 32), [Cd, dev(A), dev(B)])
+    assert np.array_equal(host(Cd), O.gemm(1.0, 2.0, C, A, B))
+
+
+@pytest.mark.parametrize("tiles", [(128, 256, 32), (128, 160, 32)])
+def test_tcm_2mm_3mm(cuda_device, tiles):
+    ni, nj, nk, nl, nm = 331, 260, 296, 300, 140
+    A = synth.uniform((ni, nk), 50); B = synth.uniform((nk, nj), 51)
+    C = synth.uniform((nj, nl), 52); D = synth.uniform((ni, nl), 53)
+    tmp_ref, D_ref = O.two_mm(1.5, 1.2, A, B, C, D)
+    d = E.desc_builtin("2mm", (ni, nj, nk, nl)); d.set_scalars(1.5, 1.2); d.set_exec(50, TENSOR)
+    tmp = torch.full((ni, nj), float("nan"), device="cuda"); Dd = dev(D)  # init_zero: never read
+    E.run(d, tiles, [tmp, dev(A), dev(B), dev(C), Dd])
+    assert O.normwise_rel_err(host(tmp), tmp_ref) <= 1e-5 and O.normwise_rel_err(host(Dd), D_ref) <= 1e-5
+    C3 = synth.uniform((nj, nm), 54); D3 = synth.uniform((nm, nl), 55)
+    E_ref, F_ref, G_ref = O.three_mm(A, B, C3, D3)
+    d = E.desc_builtin("3mm", (ni, nj, nk, nl, nm)); d.set_exec(50, TENSOR)
+    Eb, Fb, Gb = (torch.full(s, float("nan"), device="cuda") for s in ((ni, nj), (nj, nl), (ni, nl)))
+    E.run(d, tiles, [Eb, dev(A), dev(B), Fb, dev(C3), dev(D3), Gb])
+    for got, want in ((Eb, E_ref), (Fb, F_ref), (Gb, G_ref)):
+        assert O.normwise_rel_err(host(got), want) <= 1e-5
+
+
+@pytest.mark.parametrize("tiles", [(128, 256, 32), (128, 96, 32)])
+def test_tcm_split_exact_for_22_bit_values(cuda_device, tiles):
+    # hi + lo reproduces every fp32 value with <= 22 significant bits exactly, whichever split
+    # mode is active (rna hi, or the raw operand read by the truncating tensor core): A @ I == A
+    n = 300
+    g = synth.rng(90)
+    A = (g.integers(2 ** 21, 2 ** 22, (n, n)) * g.choice([-1.0, 1.0], (n, n))) * 2.0 ** -21
+    A = A * 2.0 ** g.integers(-6, 6, (n, n))
+    A = A.astype(np.float32).astype(np.float64)
+    d = E.desc_builtin("gemm", (n, n, n)); d.set_scalars(1.0, 0.0); d.set_exec(50, TENSOR)
+    Cd = torch.zeros((n, n), device="cuda")
+    E.run(d, tiles, [Cd, dev(A), dev(np.eye(n))])
+    assert np.array_equal(host(Cd), A)
