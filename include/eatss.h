@@ -138,7 +138,8 @@ typedef struct {
     int32_t split_pct;  /* shared-memory carve-out preference, percent of max (sigma) */
     int32_t engine;     /* eatss_engine; AUTO = SIMT unless the tensor-core path applies */
     int32_t use_graph;  /* stencils: replay the time loop as one CUDA graph (default 1) */
-    int32_t reserved;
+    int32_t time_kernels; /* 1: record CUDA events around each nest's main compute kernel on the
+                             run's stream (read back with eatss_last_kernel_ms); default 0 */
 } eatss_exec_opts;
 
 /* Launch plan of one nest (tile -> GPU mapping, Fig. 4). */
@@ -225,8 +226,16 @@ EATSS_API eatss_status eatss_run_nest(const eatss_kernel_desc *d, int nest, cons
  * iteration point executed.  Contraction nests and stencil sweeps only. */
 EATSS_API eatss_status eatss_coverage(const eatss_kernel_desc *d, int nest, const int64_t *tiles,
                             int32_t *counts, void *stream);
-/* Number of kernel launches one eatss_run issues (graph nodes counted individually). */
+/* Number of kernel launches one eatss_run issues with the descriptor's current exec options
+ * (graph nodes counted individually; tensor engine: + operand split passes and the split-k
+ * tail pre-pass).  -1 on a bad argument. */
 EATSS_API int64_t eatss_launches_per_run(const eatss_kernel_desc *d, const int64_t *tiles);
+/* Device time in ms of the main compute kernel of each nest in the LAST eatss_run on `d`
+ * issued with exec.time_kernels = 1 (tensor engine: the tcgen05 GEMM kernel alone, without
+ * the operand split passes; SIMT / ccsd: the nest's kernel; stencils: the whole time loop).
+ * Writes min(cap, #nests) values to ms and the count to *n.  Blocks until those kernels have
+ * finished.  E_INVALID if no timed run has been issued on `d`. */
+EATSS_API eatss_status eatss_last_kernel_ms(const eatss_kernel_desc *d, float *ms, int32_t cap, int32_t *n);
 
 /* ------------------------------------------------------------ energy */
 /* NVML total-energy counter of `device` in millijoules since driver load. */

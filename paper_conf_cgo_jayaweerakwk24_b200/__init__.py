@@ -21,7 +21,7 @@ _lib = _abi.load()
 
 __all__ = [
     "EatssError", "Desc", "desc_builtin", "gpu_params_query", "gpu_params_b200", "gpu_params_ga100",
-    "select_tiles", "plan", "run", "run_nest", "coverage", "launches_per_run", "energy_mj",
+    "select_tiles", "plan", "run", "run_nest", "coverage", "launches_per_run", "last_kernel_ms", "energy_mj",
     "power_sample", "sweep", "last_error", "abi_version", "lib_path",
 ]
 
@@ -111,8 +111,8 @@ class Desc:
     def set_scalars(self, alpha: float, beta: float) -> None:
         _check(_lib.eatss_desc_set_scalars(self._h, float(alpha), float(beta)), "desc_set_scalars")
 
-    def set_exec(self, split_pct: int = 50, engine: int = 0, use_graph: int = 1) -> None:
-        o = _abi.ExecOpts(split_pct, engine, use_graph, 0)
+    def set_exec(self, split_pct: int = 50, engine: int = 0, use_graph: int = 1, time_kernels: int = 0) -> None:
+        o = _abi.ExecOpts(split_pct, engine, use_graph, time_kernels)
         _check(_lib.eatss_desc_set_exec(self._h, ctypes.byref(o)), "desc_set_exec")
 
     def model_info(self, nest: int = 0, waf: int = 16):
@@ -190,6 +190,14 @@ def coverage(d: Desc, nest: int, tiles: Sequence[int], counts, stream=None) -> N
 
 def launches_per_run(d: Desc, tiles: Sequence[int]) -> int:
     return int(_lib.eatss_launches_per_run(d.handle, _i64s(tiles)))
+
+
+def last_kernel_ms(d: Desc) -> List[float]:
+    """Device ms of each nest's main compute kernel in the last run with time_kernels=1 (blocks)."""
+    cap = max(1, d.num_nests)
+    ms = (ctypes.c_float * cap)(); n = ctypes.c_int32()
+    _check(_lib.eatss_last_kernel_ms(d.handle, ms, cap, ctypes.byref(n)), "last_kernel_ms")
+    return list(ms)[: n.value]
 
 
 def energy_mj(device: int = 0) -> int:

@@ -286,6 +286,26 @@ using namespace eatss;
 
 eatss_kernel_desc::~eatss_kernel_desc() {
     for (auto &kv : graphs) cudaGraphExecDestroy((cudaGraphExec_t)kv.second);
+    for (void *e : kev) cudaEventDestroy((cudaEvent_t)e);
+}
+
+// exec.time_kernels: a {start, stop} event pair per nest on the current device (nullptr if off)
+static cudaEvent_t *kernel_events(eatss_kernel_desc *d, int nest) {
+    if (!d->exec.time_kernels) return nullptr;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (d->kev_dev != dev) {
+        for (void *e : d->kev) cudaEventDestroy((cudaEvent_t)e);
+        d->kev.clear();
+        d->kev_dev = dev;
+    }
+    while ((int)d->kev.size() < 2 * (int)d->nests.size()) {
+        cudaEvent_t e;
+        if (cudaEventCreate(&e) != cudaSuccess) return nullptr;
+        d->kev.push_back(e);
+    }
+    d->kev_valid = (int)d->nests.size();
+    return reinterpret_cast<cudaEvent_t *>(&d->kev[2 * nest]);
 }
 
 extern "C" {
@@ -519,19 +539,29 @@ static eatss_status run_impl(const eatss_kernel_desc *cd, int only_nest, const i
             const bool tc = want_tc && !tcm && tc_plan(cn[i], p, &tsm, &tcols);
             if (want_tc && !tc && !tcm)
                 return fail(EATSS_E_UNSUPPORTED, "eatss_run: tensor engine not applicable to this tile/operand layout");
-            cudaError_t e = tcm  ? launch_tcm_contraction(cn[i], p, s)
+            cudaEvent_t *ev = kernel_events(d, i);
+            if (ev && !tcm) cudaEventRecord(ev[0], s);
+            cudaError_t e = tcm  ? launch_tcm_contraction(cn[i], p, s, ev)
                             : tc ? launch_tc_contraction(cn[i], p, d->exec.split_pct, s)
                                  : launch_contraction(cn[i], p, d->exec.split_pct, nullptr, s);
+            if (ev && !tcm) cudaEventRecord(ev[1], s);
             if (e != cudaSuccess) return cuda_fail(e, "eatss_run(contraction)");
         }
         return EATSS_OK;
     }
     if (d->kind == EATSS_JACOBI2D || d->kind == EATSS_HEAT3D) {
         if (only_nest >= 0) return fail(EATSS_E_UNSUPPORTED, "eatss_run_nest: stencils run whole time loops");
-        return stencil_run(d, tiles, buffers, s);
+        cudaEvent_t *ev = kernel_events(d, 0);
+        if (ev) cudaEventRecord(ev[0], s);
+        const eatss_status r = stencil_run(d, tiles, buffers, s);
+        if (ev) cudaEventRecord(ev[1], s);
+        return r;
     }
+    cudaEvent_t *ev = kernel_events(d, 0);
+    if (ev) cudaEventRecord(ev[0], s);
     cudaError_t e = launch_ccsd_d1((float *)buffers[0], (const float *)buffers[1], (const float *)buffers[2],
                                    d->dims.data(), tiles, 0, d->dims[0], d->exec.split_pct, nullptr, s);
+    if (ev) cudaEventRecord(ev[1], s);
     return e == cudaSuccess ? EATSS_OK : cuda_fail(e, "eatss_run(ccsd_t_d1)");
 }
 
@@ -578,8 +608,21 @@ eatss_status eatss_coverage(const eatss_kernel_desc *d, int nest, const int64_t 
 }
 
 int64_t eatss_launches_per_run(const eatss_kernel_desc *d, const int64_t *tiles) {
-    (void)tiles;
     if (!d) return -1;
+    if (is_contraction(d->kind) && d->exec.engine == EATSS_ENGINE_TENSOR) {
+        if (!tiles || check_tiles(d, tiles) != EATSS_OK) return -1;
+        void *b[EATSS_MAX_BUFFERS];  // layout only: aligned dummies, never dereferenced
+        for (int i = 0; i < EATSS_MAX_BUFFERS; i++) b[i] = (void *)((uintptr_t)(1 << 20) * (uintptr_t)(i + 1));
+        auto cn = contraction_nests(d, b);
+        const int sl = smem_limit_bytes();
+        int64_t total = 0;
+        for (auto &n : cn) {
+            ContractPlan p = plan_contraction(n, tiles, sl);
+            int tsm = 0, tcols = 0;
+            total += tcm_applicable(n, p) ? tcm_launches(n, p) : tc_plan(n, p, &tsm, &tcols) ? 1 : 0;
+        }
+        return total;
+    }
     switch (d->kind) {
         case EATSS_GEMM: case EATSS_SYRK: case EATSS_CCSD_T_D1: return 1;
         case EATSS_2MM: return 2;
@@ -588,6 +631,25 @@ int64_t eatss_launches_per_run(const eatss_kernel_desc *d, const int64_t *tiles)
         case EATSS_HEAT3D: return 2 * d->tsteps;
     }
     return -1;
+}
+
+eatss_status eatss_last_kernel_ms(const eatss_kernel_desc *cd, float *ms, int32_t cap, int32_t *n) {
+    auto *d = const_cast<eatss_kernel_desc *>(cd);
+    if (!d || !n || (cap > 0 && !ms)) return fail(EATSS_E_INVALID, "eatss_last_kernel_ms: bad argument");
+    if (!d->kev_valid) return fail(EATSS_E_INVALID, "eatss_last_kernel_ms: no run with exec.time_kernels = 1");
+    int cnt = 0;
+    for (int i = 0; i < d->kev_valid; i++) {
+        cudaEvent_t a = (cudaEvent_t)d->kev[2 * i], b = (cudaEvent_t)d->kev[2 * i + 1];
+        float t = 0.f;
+        cudaError_t e = cudaEventSynchronize(b);
+        if (e == cudaSuccess) e = cudaEventElapsedTime(&t, a, b);
+        if (e == cudaErrorNotReady || e == cudaErrorInvalidResourceHandle) t = -1.f, e = cudaSuccess;
+        if (e != cudaSuccess) return cuda_fail(e, "eatss_last_kernel_ms");
+        if (cnt < cap) ms[cnt] = t;
+        cnt++;
+    }
+    *n = cnt;
+    return EATSS_OK;
 }
 
 }  // extern "C"

@@ -44,7 +44,10 @@ bool tc_plan(const ContractNest &n, const ContractPlan &p, int *smem_bytes, int 
 cudaError_t launch_tc_contraction(const ContractNest &n, const ContractPlan &p, int carveout, cudaStream_t s);
 // tcgen05 3xTF32 GEMM for MMA-legal tiles (Ti = 128, Tj in 32..256 step 32) (tc_mma.cu)
 bool tcm_applicable(const ContractNest &n, const ContractPlan &p);
-cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p, cudaStream_t s);
+// ev: optional {start, stop} events recorded around the GEMM kernel alone
+cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p, cudaStream_t s,
+                                   cudaEvent_t *ev = nullptr);
+int tcm_launches(const ContractNest &n, const ContractPlan &p);  // kernels one launch_tcm_contraction issues
 cudaError_t launch_contraction(const ContractNest &n, const ContractPlan &p, int carveout_pct,
                                int32_t *coverage_counts, cudaStream_t s);
 

@@ -65,6 +65,9 @@ struct eatss_kernel_desc {
     // cached stencil time-loop graphs (cudaGraphExec_t as void*)
     std::mutex graph_mu;
     std::map<eatss::GraphKey, void *> graphs;
+    // exec.time_kernels: start/stop events per nest of the last timed run (cudaEvent_t as void*)
+    std::vector<void *> kev;
+    int kev_dev = -1, kev_valid = 0;
     ~eatss_kernel_desc();
 };
 

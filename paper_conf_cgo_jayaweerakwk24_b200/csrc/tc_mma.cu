@@ -32,6 +32,7 @@
 #include <algorithm>
 #include <cstdint>
 #include <cstdlib>
+#include <map>
 #include <mutex>
 #include <string>
 
@@ -421,21 +422,25 @@ __global__ void __launch_bounds__(NTHREADS, 1)
 }
 
 // C := init_zero ? 0 : beta*C over the tiles that are split along k (their parts then add
-// alpha * partial sums atomically).  One CTA per (tail tile, 8-row slab).
+// alpha * partial sums atomically).  One CTA per row of a tail tile.
 __global__ void tail_prepass_kernel(const Args p, int rows_per_tile, int bn) {
-    const int ntail = p.T - p.nfull;
-    const int slabs = rows_per_tile / 8;
-    for (int b = blockIdx.x; b < ntail * slabs; b += gridDim.x) {
-        int pi, tj;
-        tile_coords(p.nfull + b / slabs, p.PI, p.TJ, pi, tj);
-        const int64_t r0 = (int64_t)pi * rows_per_tile + (b % slabs) * 8, j0 = (int64_t)tj * bn;
-        for (int x = threadIdx.x; x < 8 * bn; x += blockDim.x) {
-            const int64_t i = r0 + x / bn, j = j0 + x % bn;
-            if (i < p.M && j < p.N) {
-                float *c = p.C + i * p.ldc + j;
-                *c = p.init_zero ? 0.f : p.beta * *c;
-            }
+    const int t = p.nfull + (int)blockIdx.x / rows_per_tile, r = (int)blockIdx.x % rows_per_tile;
+    int pi, tj;
+    tile_coords(t, p.PI, p.TJ, pi, tj);
+    const int64_t i = (int64_t)pi * rows_per_tile + r, j0 = (int64_t)tj * bn;
+    if (i >= p.M) return;
+    float *c = p.C + i * p.ldc + j0;
+    const int64_t w = p.N - j0 < bn ? p.N - j0 : bn;
+    if ((reinterpret_cast<uintptr_t>(c) & 15) == 0) {
+        for (int x = threadIdx.x; x < w / 4; x += blockDim.x) {
+            float4 v = reinterpret_cast<float4 *>(c)[x];
+            v = p.init_zero ? make_float4(0.f, 0.f, 0.f, 0.f)
+                            : make_float4(p.beta * v.x, p.beta * v.y, p.beta * v.z, p.beta * v.w);
+            reinterpret_cast<float4 *>(c)[x] = v;
         }
+        for (int64_t x = w / 4 * 4 + threadIdx.x; x < w; x += blockDim.x) c[x] = p.init_zero ? 0.f : p.beta * c[x];
+    } else {
+        for (int64_t x = threadIdx.x; x < w; x += blockDim.x) c[x] = p.init_zero ? 0.f : p.beta * c[x];
     }
 }
 
@@ -572,12 +577,55 @@ bool tcm_applicable(const ContractNest &n, const ContractPlan &p) {
     return 2 * tcm_stage_bytes((int)p.Tj, 1) + 2048 <= 232448 && tcm::encode_fn() != nullptr;
 }
 
+// Persistent schedule: full tiles in waves of ncl clusters, the last partial wave split along k
+// into sp parts (so idle clusters take k-slices instead of waiting).  nsm / CG clusters of one
+// CTA per SM (shared memory admits one); the CTA-pair count is capped by the occupancy query.
+static void schedule(tcm::Args &a, int ncl) {
+    a.T = a.PI * a.TJ;
+    ncl = std::max(1, std::min(ncl, a.T));
+    const int rem = a.T % ncl;
+    a.sp = 1;
+    a.nfull = a.T;
+    const char *ev = getenv("EATSS_TCM_SPLITK");
+    if (rem > 0 && !(ev && atoi(ev) == 0)) {
+        const int sp = std::min(std::min(4, ncl / rem), a.nkb);
+        if (sp >= 2) {
+            a.sp = sp;
+            a.nfull = a.T - rem;
+        }
+    }
+    a.nunits = a.nfull + (a.T - a.nfull) * a.sp;
+}
+static bool needs_prepass(const tcm::Args &a) { return a.sp > 1 && (a.init_zero || a.beta != 1.f); }
+
+// per (kernel, device): the dynamic-smem attribute already set and the CTA-pair occupancy, so
+// repeated launches do not pay for cudaFuncSetAttribute / the occupancy query on the host
+namespace {
+struct KernelState {
+    int smem = -1;
+    int active = 0;
+};
+std::mutex g_ks_mu;
+std::map<std::pair<const void *, int>, KernelState> g_ks;
+}  // namespace
+
 template <int BN, bool TB, int CG>
-static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int nsm, cudaStream_t s) {
+static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int nsm, cudaStream_t s,
+                              cudaEvent_t *ev) {
     auto k = tcm::tc_mma_kernel<BN, TB, CG>;
-    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    if (e != cudaSuccess) return e;
-    // persistent: as many clusters as fit at once (one CTA per SM), never more than tiles
+    int dev = 0;
+    cudaGetDevice(&dev);
+    KernelState *ks;
+    {
+        std::lock_guard<std::mutex> lk(g_ks_mu);
+        ks = &g_ks[{reinterpret_cast<const void *>(k), dev}];
+    }
+    cudaError_t e;
+    const bool fresh = ks->smem < smem;
+    if (fresh) {
+        if ((e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
+        ks->smem = smem;
+    }
     int ncl = nsm / CG;
     cudaLaunchConfig_t cfg = {};
     cudaLaunchAttribute attr[1];
@@ -591,45 +639,41 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
     cfg.attrs = attr;
     cfg.numAttrs = 1;
     if (CG == 2) {
-        cfg.gridDim = dim3((unsigned)(2 * ncl));
-        int active = 0;
-        if (cudaOccupancyMaxActiveClusters(&active, k, &cfg) == cudaSuccess && active > 0) ncl = std::min(ncl, active);
-        cudaGetLastError();
-    }
-    // schedule: full tiles in waves of ncl, the last partial wave split along k
-    a.T = a.PI * a.TJ;
-    ncl = std::max(1, std::min(ncl, a.T));
-    const int rem = a.T % ncl;
-    a.sp = 1;
-    a.nfull = a.T;
-    if (const char *ev = getenv("EATSS_TCM_SPLITK"); rem > 0 && !(ev && atoi(ev) == 0)) {
-        const int sp = std::min(std::min(4, ncl / rem), a.nkb);
-        if (sp >= 2) {
-            a.sp = sp;
-            a.nfull = a.T - rem;
+        if (fresh || ks->active <= 0) {
+            cfg.gridDim = dim3((unsigned)(2 * ncl));
+            int active = 0;
+            if (cudaOccupancyMaxActiveClusters(&active, k, &cfg) != cudaSuccess) active = 0;
+            cudaGetLastError();
+            ks->active = active;
         }
+        if (ks->active > 0) ncl = std::min(ncl, ks->active);
     }
-    a.nunits = a.nfull + (a.T - a.nfull) * a.sp;
-    if (a.sp > 1 && (a.init_zero || a.beta != 1.f)) {
-        tcm::tail_prepass_kernel<<<std::min(4096, (a.T - a.nfull) * (CG * tcm::BM / 8)), 256, 0, s>>>(
-            a, CG * tcm::BM, BN);
+    schedule(a, ncl);
+    ncl = std::max(1, std::min(ncl, a.T));
+    if (needs_prepass(a)) {
+        const int rows = CG * tcm::BM, blocks = (a.T - a.nfull) * rows;
+        tcm::tail_prepass_kernel<<<blocks, std::max(32, BN / 4), 0, s>>>(a, rows, BN);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
     }
     cfg.gridDim = dim3((unsigned)(CG * ncl));
-    return cudaLaunchKernelEx(&cfg, k, m[0], m[1], m[2], m[3], a);
+    if (ev) cudaEventRecord(ev[0], s);
+    e = cudaLaunchKernelEx(&cfg, k, m[0], m[1], m[2], m[3], a);
+    if (ev) cudaEventRecord(ev[1], s);
+    return e;
 }
 
 template <bool TB, int CG>
-static cudaError_t launch_bn(int bn, const CUtensorMap *m, const tcm::Args &a, int smem, int nsm, cudaStream_t s) {
+static cudaError_t launch_bn(int bn, const CUtensorMap *m, const tcm::Args &a, int smem, int nsm, cudaStream_t s,
+                             cudaEvent_t *ev) {
     switch (bn) {
-        case 32: return launch_one<32, TB, CG>(m, a, smem, nsm, s);
-        case 64: return launch_one<64, TB, CG>(m, a, smem, nsm, s);
-        case 96: return launch_one<96, TB, CG>(m, a, smem, nsm, s);
-        case 128: return launch_one<128, TB, CG>(m, a, smem, nsm, s);
-        case 160: return launch_one<160, TB, CG>(m, a, smem, nsm, s);
-        case 192: return launch_one<192, TB, CG>(m, a, smem, nsm, s);
-        case 224: return launch_one<224, TB, CG>(m, a, smem, nsm, s);
-        case 256: return launch_one<256, TB, CG>(m, a, smem, nsm, s);
+        case 32: return launch_one<32, TB, CG>(m, a, smem, nsm, s, ev);
+        case 64: return launch_one<64, TB, CG>(m, a, smem, nsm, s, ev);
+        case 96: return launch_one<96, TB, CG>(m, a, smem, nsm, s, ev);
+        case 128: return launch_one<128, TB, CG>(m, a, smem, nsm, s, ev);
+        case 160: return launch_one<160, TB, CG>(m, a, smem, nsm, s, ev);
+        case 192: return launch_one<192, TB, CG>(m, a, smem, nsm, s, ev);
+        case 224: return launch_one<224, TB, CG>(m, a, smem, nsm, s, ev);
+        case 256: return launch_one<256, TB, CG>(m, a, smem, nsm, s, ev);
         default: return cudaErrorNotSupported;
     }
 }
@@ -666,7 +710,7 @@ void split_operand(Operand &o, float *ws, int mode, cudaStream_t s) {
 }
 }  // namespace
 
-cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p, cudaStream_t s) {
+cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p, cudaStream_t s, cudaEvent_t *ev) {
     if (!tcm_applicable(n, p)) return cudaErrorNotSupported;
     const int bn = (int)p.Tj, cg = tcm_cg(n, bn), mode = split_mode();
     const float *A = static_cast<const float *>(n.A), *B = static_cast<const float *>(n.B);
@@ -714,8 +758,27 @@ cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p,
     int dev = 0, nsm = 148;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-    if (n.transB) return cg == 2 ? launch_bn<true, 2>(bn, m, a, smem, nsm, s) : launch_bn<true, 1>(bn, m, a, smem, nsm, s);
-    return cg == 2 ? launch_bn<false, 2>(bn, m, a, smem, nsm, s) : launch_bn<false, 1>(bn, m, a, smem, nsm, s);
+    if (n.transB)
+        return cg == 2 ? launch_bn<true, 2>(bn, m, a, smem, nsm, s, ev) : launch_bn<true, 1>(bn, m, a, smem, nsm, s, ev);
+    return cg == 2 ? launch_bn<false, 2>(bn, m, a, smem, nsm, s, ev) : launch_bn<false, 1>(bn, m, a, smem, nsm, s, ev);
+}
+
+int tcm_launches(const ContractNest &n, const ContractPlan &p) {
+    const int bn = (int)p.Tj, cg = tcm_cg(n, bn);
+    const float *A = static_cast<const float *>(n.A), *B = static_cast<const float *>(n.B);
+    const bool share = n.transB && n.lda == n.ldb && A >= B && (A - B) % n.ldb == 0 &&
+                       (A - B) / n.ldb + n.M <= n.N;
+    tcm::Args a{};
+    a.init_zero = n.init_zero ? 1 : 0;
+    a.beta = (float)n.beta;
+    a.nkb = (int)((n.K + tcm::BK - 1) / tcm::BK);
+    a.PI = (int)((n.M + cg * tcm::BM - 1) / (cg * tcm::BM));
+    a.TJ = (int)((n.N + bn - 1) / bn);
+    int dev = 0, nsm = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    schedule(a, nsm / cg);  // (the occupancy cap of CTA pairs is nsm / 2 on B200)
+    return (share ? 1 : 2) + (needs_prepass(a) ? 1 : 0) + 1;
 }
 
 }  // namespace eatss

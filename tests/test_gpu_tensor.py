@@ -205,3 +205,27 @@ def test_tcm_split_exact_for_22_bit_values(cuda_device, tiles):
     Cd = torch.zeros((n, n), device="cuda")
     E.run(d, tiles, [Cd, dev(A), dev(np.eye(n))])
     assert np.array_equal(host(Cd), A)
+
+
+def test_kernel_timing_and_launch_count(cuda_device):
+    # exec.time_kernels: events around the GEMM launch alone; launches_per_run counts the split
+    # passes (A and B; syrk shares one), the split-k tail pre-pass (beta != 1) and the GEMM
+    n = 2500
+    d = E.desc_builtin("gemm", (n, n, n)); d.set_scalars(1.5, 1.2); d.set_exec(50, TENSOR, time_kernels=1)
+    bufs = [torch.rand(n, n, device="cuda") for _ in range(3)]
+    s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    E.run(d, (128, 256, 32), bufs)
+    s.record(); E.run(d, (128, 256, 32), bufs); e.record()
+    torch.cuda.synchronize()
+    (k,) = E.last_kernel_ms(d)
+    assert 0 < k < s.elapsed_time(e)
+    # 2500/256 -> 10 pair-rows x 10 column tiles = 100 tiles on 74 clusters: the 26-tile tail is
+    # split along k (pre-pass needed for beta != 1)
+    assert E.launches_per_run(d, (128, 256, 32)) == 4
+    d.set_scalars(1.5, 1.0)
+    assert E.launches_per_run(d, (128, 256, 32)) == 3
+    ds = E.desc_builtin("syrk", (n, n)); ds.set_exec(50, TENSOR)
+    assert E.launches_per_run(ds, (128, 256, 32)) == 3
+    d2 = E.desc_builtin("gemm", (n, n, n))
+    with pytest.raises(E.EatssError):
+        E.last_kernel_ms(d2)
