@@ -35,6 +35,9 @@ void stencil_plan_dims(bool heat, int64_t n, const int64_t *t, bool f64, int64_t
 cudaError_t launch_ccsd_d1(float *t3, const float *t2, const float *v2, const int64_t *dims,
                            const int64_t *tiles, int64_t h3_begin, int64_t h3_count, int carveout,
                            int32_t *counts, cudaStream_t s);
+bool ccsd_tc_applicable(const int64_t *dims, const int64_t *tiles);
+cudaError_t launch_ccsd_tc(float *t3, const float *t2, const float *v2, const int64_t *dims, const int64_t *tiles,
+                           int64_t h3_begin, int64_t h3_count, cudaStream_t s, cudaEvent_t *ev);
 void ccsd_plan_dims(const int64_t *dims, const int64_t *tiles, int64_t *gx, int64_t *gy, int *bx,
                     int *by, int *rm, int *rn, int *passes, int *smem);
 
@@ -558,6 +561,15 @@ static eatss_status run_impl(const eatss_kernel_desc *cd, int only_nest, const i
         return r;
     }
     cudaEvent_t *ev = kernel_events(d, 0);
+    if (d->exec.engine == EATSS_ENGINE_TENSOR) {  // tcgen05 3xTF32 with TMA-streamed t3 (ccsd_tc.cu)
+        if (!ccsd_tc_applicable(d->dims.data(), tiles))
+            return fail(EATSS_E_UNSUPPORTED, "eatss_run: tensor engine needs a ccsd tile (1,1,Th1,Tp6,Tp5,Tp4,>=H7) "
+                                             "with Th1*Tp5*Tp4 <= 128, Tp6 % 16 == 0, Tp4 % 4 == 0, "
+                                             "P4 % 4 == 0, H7 % 4 == 0, H7 <= 64");
+        cudaError_t e = launch_ccsd_tc((float *)buffers[0], (const float *)buffers[1], (const float *)buffers[2],
+                                       d->dims.data(), tiles, 0, d->dims[0], s, ev);
+        return e == cudaSuccess ? EATSS_OK : cuda_fail(e, "eatss_run(ccsd_t_d1, tensor)");
+    }
     if (ev) cudaEventRecord(ev[0], s);
     cudaError_t e = launch_ccsd_d1((float *)buffers[0], (const float *)buffers[1], (const float *)buffers[2],
                                    d->dims.data(), tiles, 0, d->dims[0], d->exec.split_pct, nullptr, s);
@@ -623,6 +635,7 @@ int64_t eatss_launches_per_run(const eatss_kernel_desc *d, const int64_t *tiles)
         }
         return total;
     }
+    if (d->kind == EATSS_CCSD_T_D1 && d->exec.engine == EATSS_ENGINE_TENSOR) return 2;  // prep + contraction
     switch (d->kind) {
         case EATSS_GEMM: case EATSS_SYRK: case EATSS_CCSD_T_D1: return 1;
         case EATSS_2MM: return 2;

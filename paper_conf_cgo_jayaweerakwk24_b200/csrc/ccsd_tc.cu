@@ -1,0 +1,550 @@
+// ccsd_tc.cu -- the 6-D CCSD(T) d1 contraction (BASELINE config 5) on
+// the tensor pipe (tcgen05 3xTF32), streaming t3 through TMA:
+//
+//   t3[h3][h2][h1][p6][p5][p4] -= sum_h7 t2[h7][p4][p5][h1] * v2[h3][h2][p6][h7]
+//
+// The update has AI = 12 flop/B (t3 is read and written once, K = H7 = 48), so on B200 it is
+// HBM-bound once the arithmetic leaves the FFMA pipe: this executor makes the t3 stream the only
+// thing the SMs wait for.  Tile vector (Th3, Th2, Th1, Tp6, Tp5, Tp4, Th7) with Th3 = Th2 = 1,
+// Th7 = H7 (whole reduction per tile), M = Th1*Tp5*Tp4 <= 128 output rows on the MMA M axis and
+// N = Tp6 (multiple of 16, <= 256) on the MMA N axis:
+//   D[(h1,p5,p4)][p6] = sum_h7 t2[h7][p4][p5][h1] * v2[h3][h2][p6][h7]   (UMMA M=128, A in TMEM)
+//   X = t3 tile [h1][p6][p5][p4] (TMA 5-D box) ;  X -= D^T  (epilogue) ;  TMA store X.
+// The A operand depends on (h1,p5,p4) only: the epilogue warps write its tf32 hi/lo halves into
+// TMEM once per A tile (lane = output row, 16 columns per 8-k step) and the CTA then walks every
+// (h3,h2) unit that reuses it, so the MMAs read only the small v2 tile from shared memory (the
+// shared-memory port, not HBM, was the bound while A came from shared memory too).
+// 3xTF32 with the raw-hi split (tc_mma.cu): hi = the operand itself (the tensor core truncates to
+// tf32), lo = rna_tf32(x - rz_tf32(x)); v2's lo half is materialised once per call (21 MB).
+//
+// Warp roles (persistent, one CTA per SM): warp 0 streams t3 tiles from HBM into an SX-stage ring
+// (evict-first L2 policy); warp 3 loads the per-unit v2 tile into an SV-stage ring; warp 1 issues
+// the MMAs; warp 2 owns TMEM and issues the t3-tile TMA stores; warps 4..11 are the epilogue
+// (lane = output row m; t3 tile RMW in shared memory; ring slot released two stores later).
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdint>
+#include <cstdlib>
+#include <mutex>
+
+#include "tc_ptx.cuh"
+
+namespace eatss {
+namespace ccsdtc {
+
+using namespace tcm;
+
+constexpr int NEPI = 8;  // epilogue warps
+constexpr int NTHREADS = (4 + NEPI) * 32;
+constexpr int MROWS = 128;  // UMMA M
+
+struct Args {
+    int H3, H2, H1, P6, P5, P4, H7;
+    int Th1, Tp6, Tp5, Tp4;
+    int n_h1t, n_p5t, n_p4t, n_p6t;
+    int hh0, nhh;     // (h3,h2) flattened range of this launch
+    int64_t units;    // n_a * nhh * n_p6t
+    int nkb;          // ceil(H7 / 32)
+    int SV, SX;       // V ring stages, t3-tile ring stages
+    int bstride, NB;  // TMEM accumulator buffers (columns per buffer, count)
+    int nks;          // 8-k MMA steps: ceil(H7 / 8)
+    int a_col;        // TMEM column of A (hi at a_col + 16 ks, lo at + 8)
+    int v_kb_bytes;   // Tp6 * 128
+    int v_stage;      // 2 * nkb * v_kb_bytes
+    int x_bytes;      // Th1*Tp6*Tp5*Tp4*4
+    int x_stage;      // x_bytes rounded up to 1 KB
+    int order;        // 1: A tiles round-robin over CTAs (concurrent CTAs sweep whole t3 blocks)
+    int dbg;          // development only (EATSS_CCSD_TC_DBG): 1 no MMA, 2 no t3 traffic, 4 no v2 loads
+};
+
+struct Unit {
+    int a, hh, p6t;
+};
+__device__ __forceinline__ float lo_of(float x) {
+    const float hi = __uint_as_float(__float_as_uint(x) & 0xFFFFE000u);
+    uint32_t lb;
+    asm("cvt.rna.tf32.f32 %0, %1;\n" : "=r"(lb) : "f"(x - hi));
+    return __uint_as_float(lb);
+}
+__device__ __forceinline__ Unit decode(const Args &p, int64_t u) {
+    Unit w;
+    w.p6t = (int)(u % p.n_p6t);
+    const int64_t r = u / p.n_p6t;
+    w.hh = p.hh0 + (int)(r % p.nhh);
+    w.a = (int)(r / p.nhh);
+    return w;
+}
+// The units of CTA c.  Every A tile owns R = nhh * n_p6t units (all (h3,h2) for fixed
+// (h1,p5,p4) rows).  order 1: A tiles c, c+G, c+2G, ... whole, then an even share of the
+// remaining n_a mod G tiles' units -- so at any moment the G CTAs update adjacent row blocks
+// of the same (h3,h2,h1) t3 blocks (DRAM page locality) while each keeps its A tile resident.
+// order 0: one contiguous range of the unit space per CTA.
+struct Sched {
+    int64_t n1, lo, n, R;
+    int c, G, K1;
+};
+__device__ __forceinline__ Sched sched_of(const Args &p, int c, int G) {
+    Sched sc;
+    sc.c = c;
+    sc.G = G;
+    sc.R = (int64_t)p.nhh * p.n_p6t;
+    const int n_a = p.n_h1t * p.n_p5t * p.n_p4t;
+    if (p.order == 1) {
+        sc.K1 = n_a / G;
+        sc.n1 = (int64_t)sc.K1 * sc.R;
+        const int64_t rem = (int64_t)(n_a - sc.K1 * G) * sc.R;
+        sc.lo = rem * c / G;
+        sc.n = sc.n1 + rem * (c + 1) / G - sc.lo;
+    } else {
+        sc.K1 = 0;
+        sc.n1 = 0;
+        sc.lo = p.units * c / G;
+        sc.n = p.units * (c + 1) / G - sc.lo;
+    }
+    return sc;
+}
+__device__ __forceinline__ Unit unit_at(const Args &p, const Sched &sc, int64_t i) {
+    if (i < sc.n1) {
+        const int64_t k = i / sc.R, r2 = i % sc.R;
+        Unit w;
+        w.a = sc.c + (int)k * sc.G;
+        w.hh = p.hh0 + (int)(r2 / p.n_p6t);
+        w.p6t = (int)(r2 % p.n_p6t);
+        return w;
+    }
+    return decode(p, (int64_t)sc.K1 * sc.G * sc.R + sc.lo + (i - sc.n1));
+}
+__device__ __forceinline__ void a_coords(const Args &p, int a, int &h1_0, int &p5_0, int &p4_0) {
+    const int p4t = a % p.n_p4t;
+    a /= p.n_p4t;
+    const int p5t = a % p.n_p5t;
+    const int h1t = a / p.n_p5t;
+    h1_0 = h1t * p.Th1;
+    p5_0 = p5t * p.Tp5;
+    p4_0 = p4t * p.Tp4;
+}
+
+// Incremental walk over a CTA's units (no 64-bit divisions in the loops): region 1 = whole A
+// tiles c, c+G, ..., region 2 = the CTA's share of the remainder in plain unit order.
+struct UnitIter {
+    int a, hh, p6t;
+    int64_t left1;
+    bool r1;
+};
+__device__ __forceinline__ void iter_region2(const Args &p, const Sched &sc, UnitIter &w) {
+    const Unit u = decode(p, (int64_t)sc.K1 * sc.G * sc.R + sc.lo);
+    w.a = u.a;
+    w.hh = u.hh;
+    w.p6t = u.p6t;
+    w.r1 = false;
+}
+__device__ __forceinline__ UnitIter iter_begin(const Args &p, const Sched &sc) {
+    UnitIter w;
+    w.left1 = sc.n1;
+    if (sc.n1 > 0) {
+        w.a = sc.c;
+        w.hh = p.hh0;
+        w.p6t = 0;
+        w.r1 = true;
+    } else {
+        iter_region2(p, sc, w);
+    }
+    return w;
+}
+__device__ __forceinline__ void iter_next(const Args &p, const Sched &sc, UnitIter &w) {
+    if (++w.p6t == p.n_p6t) {
+        w.p6t = 0;
+        if (++w.hh == p.hh0 + p.nhh) {
+            w.hh = p.hh0;
+            w.a += w.r1 ? sc.G : 1;
+        }
+    }
+    if (w.r1 && --w.left1 == 0) iter_region2(p, sc, w);
+}
+// ring position: stage index and the parity of the current round
+struct Ring {
+    int s = 0;
+    unsigned ph = 0;
+    __device__ __forceinline__ void next(int S) {
+        if (++s == S) {
+            s = 0;
+            ph ^= 1u;
+        }
+    }
+};
+
+// warps: 0 t3-tile producer, 1 MMA issuer, 2 TMEM owner + t3-tile store issuer, 3 A/V producer,
+// 4..11 epilogue (two groups of four: TMEM lane quarter = warp % 4, column half = group)
+__global__ void __launch_bounds__(NTHREADS, 1)
+    ccsd_tc_kernel(const float *__restrict__ t2, const __grid_constant__ CUtensorMap mV,
+                   const __grid_constant__ CUtensorMap mVlo, const __grid_constant__ CUtensorMap mX, const Args p) {
+    extern __shared__ __align__(1024) unsigned char smem_raw[];
+    unsigned char *smem = reinterpret_cast<unsigned char *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    // layout: V ring [SV] {hi [nkb], lo [nkb]}, X ring [SX], barriers
+    unsigned char *vring = smem;
+    unsigned char *xring = vring + (size_t)p.SV * p.v_stage;
+    uint64_t *xfull = reinterpret_cast<uint64_t *>(xring + (size_t)p.SX * p.x_stage);
+    uint64_t *xempty = xfull + p.SX;
+    uint64_t *xdone = xempty + p.SX;
+    uint64_t *vfull = xdone + p.SX;
+    uint64_t *vempty = vfull + p.SV;
+    uint64_t *dfull = vempty + p.SV;
+    uint64_t *dempty = dfull + 4;
+    uint64_t *afull = dempty + 4;
+    uint64_t *aempty = afull + 1;
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(aempty + 1);
+    const Sched sc = sched_of(p, (int)blockIdx.x, (int)gridDim.x);
+
+    if (tid == 0) {
+        for (int s = 0; s < p.SX; s++) {
+            mbar_init(xfull + s, 1);
+            mbar_init(xempty + s, 1);
+            mbar_init(xdone + s, NEPI);
+        }
+        for (int s = 0; s < p.SV; s++) {
+            mbar_init(vfull + s, 1);
+            mbar_init(vempty + s, 1);
+        }
+        for (int b = 0; b < 4; b++) {
+            mbar_init(dfull + b, 1);
+            mbar_init(dempty + b, NEPI);
+        }
+        mbar_init(afull, NEPI);  // the epilogue warps write A into TMEM
+        mbar_init(aempty, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+        asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&mX)) : "memory");
+    }
+    if (warp == 2) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;\n" ::"r"(su32(tmem_slot)),
+                     "r"(512)
+                     : "memory");
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;\n" ::: "memory");
+    }
+    fence_before();
+    __syncthreads();
+    fence_after();
+    const uint32_t tmem = *tmem_slot;
+
+    if (warp == 0) {
+        if (lane == 0) {  // ------------------------------------ t3-tile producer (HBM stream)
+            const uint64_t pol = policy_evict_first();  // t3 is touched once: keep T2P / v2 in L2
+            UnitIter w = iter_begin(p, sc);
+            Ring r;
+            for (int64_t u = 0; u < sc.n; u++, iter_next(p, sc, w), r.next(p.SX)) {
+                int h1_0, p5_0, p4_0;
+                a_coords(p, w.a, h1_0, p5_0, p4_0);
+                if (u >= p.SX) mbar_wait(xempty + r.s, r.ph ^ 1u);
+                if (p.dbg & 2) { mbar_arrive(xfull + r.s); continue; }
+                mbar_expect_tx(xfull + r.s, p.x_bytes);
+                tma_5d_hint(xring + (size_t)r.s * p.x_stage, &mX, p4_0, p5_0, w.p6t * p.Tp6, h1_0, w.hh, xfull + r.s,
+                            pol);
+            }
+        }
+    } else if (warp == 3) {
+        if (lane == 0) {  // ------------------------------------ v2 tile producer (L2-resident)
+            UnitIter w = iter_begin(p, sc);
+            Ring r;
+            for (int64_t u = 0; u < sc.n; u++, iter_next(p, sc, w), r.next(p.SV)) {
+                if (u >= p.SV) mbar_wait(vempty + r.s, r.ph ^ 1u);
+                unsigned char *st = vring + (size_t)r.s * p.v_stage;
+                if (p.dbg & 4) { mbar_arrive(vfull + r.s); continue; }
+                mbar_expect_tx(vfull + r.s, p.v_stage);
+                const int vrow = w.hh * p.P6 + w.p6t * p.Tp6;
+                for (int kb = 0; kb < p.nkb; kb++) {
+                    tma_2d<1>(st + kb * p.v_kb_bytes, &mV, kb * 32, vrow, su32(vfull + r.s));
+                    tma_2d<1>(st + (p.nkb + kb) * p.v_kb_bytes, &mVlo, kb * 32, vrow, su32(vfull + r.s));
+                }
+            }
+        }
+    } else if (warp == 1) {
+        if (lane == 0) {  // ------------------------------------------------ MMA issuer
+            const uint32_t ID = idesc(p.Tp6, 1, true);  // M = 128, N = Tp6, A and B K-major
+            int a_prev = -1, na = 0;
+            UnitIter w = iter_begin(p, sc);
+            Ring rv, rd;
+            for (int64_t u = 0; u < sc.n; u++, iter_next(p, sc, w), rv.next(p.SV), rd.next(p.NB)) {
+                if (w.a != a_prev) {
+                    if (na > 0) mma_commit<1>(aempty);  // fires when every MMA on the old A is done
+                    mbar_wait(afull, (unsigned)(na & 1));
+                    a_prev = w.a;
+                    na++;
+                }
+                if (u >= p.NB) mbar_wait(dempty + rd.s, rd.ph ^ 1u);
+                mbar_wait(vfull + rv.s, rv.ph);
+                fence_after();
+                unsigned char *st = vring + (size_t)rv.s * p.v_stage;
+                const uint32_t d = tmem + (uint32_t)(rd.s * p.bstride);
+                bool first = true;
+                for (int k8 = 0; k8 < (p.dbg & 1 ? 0 : p.nks); k8++) {
+                    const int kb = k8 >> 2, ks = k8 & 3;
+                    const uint32_t ah = tmem + (uint32_t)(p.a_col + 16 * k8), al = ah + 8;
+                    const uint64_t vh = desc_sw128(st + kb * p.v_kb_bytes + ks * 32, 16u, 1024u);
+                    const uint64_t vl = desc_sw128(st + (p.nkb + kb) * p.v_kb_bytes + ks * 32, 16u, 1024u);
+                    mma_ts(d, ah, vh, ID, first ? 0u : 1u);
+                    mma_ts(d, ah, vl, ID, 1u);
+                    mma_ts(d, al, vh, ID, 1u);
+                    first = false;
+                }
+                mma_commit<1>(dfull + rd.s);
+                mma_commit<1>(vempty + rv.s);
+            }
+        }
+    } else if (warp == 2) {
+        if (lane == 0) {  // ------------------------------------ t3-tile store issuer
+            const uint64_t pol = policy_evict_first();
+            UnitIter w = iter_begin(p, sc);
+            Ring r;
+            int pend[3] = {-1, -1, -1};  // stages of the last stores, oldest first
+            for (int64_t u = 0; u < sc.n; u++, iter_next(p, sc, w), r.next(p.SX)) {
+                int h1_0, p5_0, p4_0;
+                a_coords(p, w.a, h1_0, p5_0, p4_0);
+                mbar_wait(xdone + r.s, r.ph);
+                if (p.dbg & 2) { mbar_arrive(xempty + r.s); continue; }
+                tma_store_5d_hint(&mX, xring + (size_t)r.s * p.x_stage, p4_0, p5_0, w.p6t * p.Tp6, h1_0, w.hh, pol);
+                bulk_commit();
+                bulk_wait_read<2>();  // all but the 2 newest stores have read their slots
+                if (pend[0] >= 0) mbar_arrive(xempty + pend[0]);
+                pend[0] = pend[1];
+                pend[1] = r.s;
+            }
+            bulk_wait_all();
+        }
+    } else if (warp >= 4) {  // ------------------------------------------------ epilogue
+        const int q = warp & 3, g = (warp - 4) >> 2, m = q * 32 + lane;
+        const int Mrows = p.Th1 * p.Tp5 * p.Tp4;
+        const int p4l = m % p.Tp4, p5l = (m / p.Tp4) % p.Tp5, h1l = m / (p.Tp4 * p.Tp5);
+        const bool live = m < Mrows;
+        const int xrow0 = (h1l * p.Tp6 * p.Tp5 + p5l) * p.Tp4 + p4l, xstep = p.Tp5 * p.Tp4;  // + p6 * xstep
+        const uint32_t trow = tmem + ((uint32_t)(q * 32) << 16);
+        UnitIter w = iter_begin(p, sc);
+        int a_prev = -1, na = 0;
+        Ring rx, rd;
+        for (int64_t u = 0; u < sc.n; u++, iter_next(p, sc, w), rx.next(p.SX), rd.next(p.NB)) {
+            if (w.a != a_prev) {  // new A tile: row m of t2 (as [h1][p5][p4] x h7) into TMEM
+                int h1_0, p5_0, p4_0;
+                a_coords(p, w.a, h1_0, p5_0, p4_0);
+                const int h1 = h1_0 + h1l, p5 = p5_0 + p5l, p4 = p4_0 + p4l;
+                const bool in = live && h1 < p.H1 && p5 < p.P5 && p4 < p.P4;
+                const float *src = t2 + (((int64_t)p4 * p.P5 + p5) * p.H1 + h1);
+                const int64_t hstride = (int64_t)p.P4 * p.P5 * p.H1;
+                if (na > 0) mbar_wait(aempty, (unsigned)((na - 1) & 1));  // MMAs on the old A are done
+                for (int k8 = g; k8 < p.nks; k8 += 2) {
+                    uint32_t hi[8], lo[8];
+#pragma unroll
+                    for (int c = 0; c < 8; c++) {
+                        const int h7 = 8 * k8 + c;
+                        const float x = (in && h7 < p.H7) ? __ldg(src + h7 * hstride) : 0.f;
+                        hi[c] = __float_as_uint(x);
+                        lo[c] = __float_as_uint(lo_of(x));
+                    }
+                    tmem_st8(trow + (uint32_t)(p.a_col + 16 * k8), hi);
+                    tmem_st8(trow + (uint32_t)(p.a_col + 16 * k8 + 8), lo);
+                }
+                wait_st();
+                fence_before();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(afull);
+                a_prev = w.a;
+                na++;
+            }
+            mbar_wait(xfull + rx.s, rx.ph);
+            mbar_wait(dfull + rd.s, rd.ph);
+            fence_after();
+            float *xs = reinterpret_cast<float *>(xring + (size_t)rx.s * p.x_stage) + xrow0;
+            // columns (p6) in chunks of 8, alternating between the two epilogue groups; up to three
+            // chunks per batch: all TMEM loads, then all shared loads, then the stores (no
+            // load-store serialisation through possibly-aliasing addresses)
+            for (int c0 = 8 * g; c0 < p.Tp6; c0 += 48) {
+                uint32_t v[3][8];
+                const int nc = min(3, (p.Tp6 - c0 + 15) / 16);
+                tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0), v[0]);
+                if (nc > 1) tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0 + 16), v[1]);
+                if (nc > 2) tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0 + 32), v[2]);
+                wait_ld();
+                if (live) {
+                    float x[3][8];
+#pragma unroll
+                    for (int j = 0; j < 3; j++)
+#pragma unroll
+                        for (int c = 0; c < 8; c++)
+                            if (j < nc) x[j][c] = xs[(c0 + 16 * j + c) * xstep];
+#pragma unroll
+                    for (int j = 0; j < 3; j++)
+#pragma unroll
+                        for (int c = 0; c < 8; c++)
+                            if (j < nc) xs[(c0 + 16 * j + c) * xstep] = x[j][c] - __uint_as_float(v[j][c]);
+                }
+            }
+            fence_before();
+            fence_proxy_async_smem();  // generic-proxy writes -> visible to the TMA store
+            __syncwarp();
+            if (lane == 0) {
+                mbar_arrive(dempty + rd.s);
+                mbar_arrive(xdone + rx.s);
+            }
+        }
+    }
+    fence_before();
+    __syncthreads();
+    if (warp == 2) {
+        fence_after();
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;\n" ::"r"(tmem), "r"(512) : "memory");
+    }
+}
+
+// v2lo = lo(v2)  (raw-hi split: v2 itself is the hi half)
+__global__ void prep_kernel(const float *__restrict__ v2, float *__restrict__ v2_lo, int64_t n_v2) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < n_v2; e += stride) v2_lo[e] = lo_of(v2[e]);
+}
+
+// n-D fp32 tensor map, dims/strides innermost first (strides in bytes for dims 1..n-1)
+static bool make_map_nd(CUtensorMap *m, const float *base, int rank, const uint64_t *dims, const uint64_t *strides,
+                        const uint32_t *box, CUtensorMapSwizzle sw) {
+    EncodeTiled enc = encode_fn();
+    if (!enc) return false;
+    cuuint64_t d[5], st[4];
+    cuuint32_t b[5], es[5];
+    for (int i = 0; i < rank; i++) {
+        d[i] = dims[i];
+        b[i] = box[i];
+        es[i] = 1;
+        if (i > 0) st[i - 1] = strides[i - 1];
+    }
+    return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, (cuuint32_t)rank, const_cast<float *>(base), d, st, b, es,
+               CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+}  // namespace ccsdtc
+
+namespace {
+std::mutex g_cws_mu;
+float *g_cws = nullptr;
+size_t g_cws_elems = 0;
+int g_cws_dev = -1;
+float *ccsd_workspace(size_t elems) {
+    std::lock_guard<std::mutex> lk(g_cws_mu);
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (g_cws && (g_cws_elems < elems || g_cws_dev != dev)) {
+        cudaFree(g_cws);
+        g_cws = nullptr;
+    }
+    if (!g_cws) {
+        if (cudaMalloc(&g_cws, elems * 4) != cudaSuccess) return g_cws = nullptr;
+        g_cws_elems = elems;
+        g_cws_dev = dev;
+    }
+    return g_cws;
+}
+
+struct CcsdTcPlan {
+    bool ok = false;
+    ccsdtc::Args a{};
+    int smem = 0;
+};
+
+CcsdTcPlan plan_ccsd_tc(const int64_t *dims, const int64_t *tiles) {
+    CcsdTcPlan pl;
+    int64_t T[7];
+    for (int i = 0; i < 7; i++) T[i] = std::min(tiles[i], dims[i]);
+    const int64_t H3 = dims[0], H2 = dims[1], H1 = dims[2], P6 = dims[3], P5 = dims[4], P4 = dims[5], H7 = dims[6];
+    if (T[0] != 1 || T[1] != 1 || T[6] < H7) return pl;  // one (h3,h2) per unit, whole h7 reduction
+    if (H7 > 64 || (H7 % 4) || (P4 % 4) || (T[5] % 4)) return pl;  // 16-byte TMA strides / boxes
+    if (T[2] * T[4] * T[5] > ccsdtc::MROWS || (T[3] % 16) || T[3] > 256) return pl;
+    if (H3 * H2 > INT32_MAX || H3 * H2 * P6 > INT32_MAX || H1 * P5 * P4 * H7 > INT32_MAX) return pl;
+    ccsdtc::Args &a = pl.a;
+    a.H3 = (int)H3; a.H2 = (int)H2; a.H1 = (int)H1; a.P6 = (int)P6; a.P5 = (int)P5; a.P4 = (int)P4; a.H7 = (int)H7;
+    a.Th1 = (int)T[2]; a.Tp6 = (int)T[3]; a.Tp5 = (int)T[4]; a.Tp4 = (int)T[5];
+    a.n_h1t = (int)((H1 + a.Th1 - 1) / a.Th1); a.n_p5t = (int)((P5 + a.Tp5 - 1) / a.Tp5);
+    a.n_p4t = (int)((P4 + a.Tp4 - 1) / a.Tp4); a.n_p6t = (int)((P6 + a.Tp6 - 1) / a.Tp6);
+    a.nkb = (int)((H7 + 31) / 32);
+    a.order = getenv("EATSS_CCSD_TC_ORDER") ? atoi(getenv("EATSS_CCSD_TC_ORDER")) : 1;
+    a.dbg = getenv("EATSS_CCSD_TC_DBG") ? atoi(getenv("EATSS_CCSD_TC_DBG")) : 0;
+    a.nks = (int)((H7 + 7) / 8);
+    a.bstride = 32;
+    while (a.bstride < a.Tp6) a.bstride *= 2;
+    a.a_col = 384;                            // TMEM: D buffers in [0, 384), A in [384, 512)
+    a.NB = std::min(4, 384 / a.bstride);
+    if (a.NB < 1) return pl;
+    a.v_kb_bytes = a.Tp6 * 128;
+    a.v_stage = 2 * a.nkb * a.v_kb_bytes;
+    a.x_bytes = a.Th1 * a.Tp6 * a.Tp5 * a.Tp4 * 4;
+    a.x_stage = (a.x_bytes + 1023) / 1024 * 1024;
+    const int fixed = 1024 /*align*/ + 512 /*barriers*/;
+    a.SV = 4;
+    const int avail = 232448 - fixed - a.SV * a.v_stage;
+    a.SX = std::min(8, avail / a.x_stage);
+    if (const char *e = getenv("EATSS_CCSD_TC_XSTAGES")) a.SX = std::max(3, std::min(a.SX, atoi(e)));
+    if (a.SX < 3) {  // big tiles: shallower operand ring
+        a.SV = 2;
+        a.SX = std::min(8, (232448 - fixed - a.SV * a.v_stage) / a.x_stage);
+    }
+    // SX >= 3: the store issuer releases a slot two stores after it was written
+    if (a.SX < 3) return pl;
+    pl.smem = fixed + a.SV * a.v_stage + a.SX * a.x_stage;
+    pl.ok = true;
+    return pl;
+}
+}  // namespace
+
+bool ccsd_tc_applicable(const int64_t *dims, const int64_t *tiles) {
+    return plan_ccsd_tc(dims, tiles).ok && tcm::encode_fn() != nullptr;
+}
+
+cudaError_t launch_ccsd_tc(float *t3, const float *t2, const float *v2, const int64_t *dims, const int64_t *tiles,
+                           int64_t h3_begin, int64_t h3_count, cudaStream_t s, cudaEvent_t *ev) {
+    CcsdTcPlan pl = plan_ccsd_tc(dims, tiles);
+    if (!pl.ok || !tcm::encode_fn()) return cudaErrorNotSupported;
+    ccsdtc::Args a = pl.a;
+    const int64_t H2 = dims[1], H1 = dims[2], P6 = dims[3], P5 = dims[4], P4 = dims[5], H7 = dims[6];
+    a.hh0 = (int)(h3_begin * H2);
+    a.nhh = (int)(h3_count * H2);
+    a.units = (int64_t)a.n_h1t * a.n_p5t * a.n_p4t * a.nhh * a.n_p6t;
+    if (a.units == 0) return cudaSuccess;
+    const int64_t n_v2 = (int64_t)a.H3 * H2 * P6 * H7;
+    float *v2_lo = ccsd_workspace((size_t)(n_v2 + 64));
+    if (!v2_lo) return cudaErrorMemoryAllocation;
+    ccsdtc::prep_kernel<<<148 * 4, 256, 0, s>>>(v2, v2_lo, n_v2);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return e;
+    CUtensorMap mV, mVlo, mX;
+    // V: v2 as [(h3,h2,p6)][h7], box {32, Tp6}, SWIZZLE_128B (K-major UMMA operand)
+    const uint64_t vdims[2] = {(uint64_t)H7, (uint64_t)((int64_t)a.H3 * H2 * P6)};
+    const uint64_t vstr[1] = {(uint64_t)H7 * 4};
+    const uint32_t vbox[2] = {32, (uint32_t)a.Tp6};
+    // X: t3 as [(h3,h2)][h1][p6][p5][p4], box {Tp4, Tp5, Tp6, Th1, 1}
+    const uint64_t xdims[5] = {(uint64_t)P4, (uint64_t)P5, (uint64_t)P6, (uint64_t)H1, (uint64_t)((int64_t)a.H3 * H2)};
+    const uint64_t xstr[4] = {(uint64_t)P4 * 4, (uint64_t)(P5 * P4) * 4, (uint64_t)(P6 * P5 * P4) * 4,
+                              (uint64_t)(H1 * P6 * P5 * P4) * 4};
+    const uint32_t xbox[5] = {(uint32_t)a.Tp4, (uint32_t)a.Tp5, (uint32_t)a.Tp6, (uint32_t)a.Th1, 1};
+    if (!ccsdtc::make_map_nd(&mV, v2, 2, vdims, vstr, vbox, CU_TENSOR_MAP_SWIZZLE_128B) ||
+        !ccsdtc::make_map_nd(&mVlo, v2_lo, 2, vdims, vstr, vbox, CU_TENSOR_MAP_SWIZZLE_128B) ||
+        !ccsdtc::make_map_nd(&mX, t3, 5, xdims, xstr, xbox, CU_TENSOR_MAP_SWIZZLE_NONE))
+        return cudaErrorInvalidValue;
+    static std::mutex mu;
+    static int smem_set = -1;
+    {
+        std::lock_guard<std::mutex> lk(mu);
+        if (smem_set < pl.smem) {
+            e = cudaFuncSetAttribute(ccsdtc::ccsd_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, pl.smem);
+            if (e != cudaSuccess) return e;
+            smem_set = pl.smem;
+        }
+    }
+    int dev = 0, nsm = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    const int grid = (int)std::min<int64_t>(nsm, a.units);
+    if (ev) cudaEventRecord(ev[0], s);
+    ccsdtc::ccsd_tc_kernel<<<grid, ccsdtc::NTHREADS, pl.smem, s>>>(t2, mV, mVlo, mX, a);
+    e = cudaGetLastError();
+    if (ev) cudaEventRecord(ev[1], s);
+    return e;
+}
+
+}  // namespace eatss

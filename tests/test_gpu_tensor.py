@@ -229,3 +229,50 @@ def test_kernel_timing_and_launch_count(cuda_device):
     d2 = E.desc_builtin("gemm", (n, n, n))
     with pytest.raises(E.EatssError):
         E.last_kernel_ms(d2)
+
+
+# ---- ccsd_t_d1 on the tensor pipe (ccsd_tc.cu): tile (1, 1, Th1, Tp6, Tp5, Tp4, >= H7)
+CCSD_TC = [((16,) * 7, (1, 1, 1, 16, 8, 16, 16)), ((16,) * 7, (1, 1, 2, 16, 4, 16, 16)),
+           ((16,) * 7, (1, 1, 1, 16, 2, 16, 16)),
+           ((3, 5, 6, 20, 7, 12, 20), (1, 1, 2, 16, 3, 12, 20)),   # ragged h1/p5/p6 tiles, h7 pad
+           ((2, 3, 4, 32, 4, 8, 48), (1, 1, 2, 32, 4, 8, 48)),    # two k-blocks (H7 = 48)
+           ((2, 2, 3, 160, 2, 16, 16), (1, 1, 1, 160, 2, 16, 16))]  # N = 160: one TMEM accumulator
+
+
+@pytest.mark.parametrize("dims,tiles", CCSD_TC)
+def test_ccsd_tc(cuda_device, dims, tiles):
+    H3, H2, H1, P6, P5, P4, H7 = dims
+    d = E.desc_builtin("ccsd_t_d1", dims); d.set_exec(50, TENSOR)
+    t3i = synth.small_int((H3, H2, H1, P6, P5, P4), 103)
+    t2i = synth.small_int((H7, P4, P5, H1), 104); v2i = synth.small_int((H3, H2, P6, H7), 105)
+    t3d = dev(t3i)
+    E.run(d, tiles, [t3d, dev(t2i), dev(v2i)])
+    assert np.array_equal(host(t3d), O.ccsd_t_d1(t3i, t2i, v2i))
+    t3 = synth.uniform(t3i.shape, 100); t2 = synth.uniform(t2i.shape, 101); v2 = synth.uniform(v2i.shape, 102)
+    t3d = dev(t3)
+    E.run(d, tiles, [t3d, dev(t2), dev(v2)])
+    assert O.normwise_rel_err(host(t3d), O.ccsd_t_d1(t3, t2, v2)) <= 1e-5
+
+
+def test_ccsd_tc_rejects_non_mma_tiles(cuda_device):
+    d = E.desc_builtin("ccsd_t_d1", (16,)); d.set_exec(50, TENSOR)
+    bufs = [torch.zeros(d.buffer_elems(i), device="cuda") for i in range(3)]
+    for tiles in [(4, 4, 4, 4, 4, 32, 4), (1, 1, 1, 16, 16, 16, 16), (1, 1, 1, 8, 8, 16, 16), (1, 1, 1, 16, 8, 16, 8)]:
+        with pytest.raises(E.EatssError) as ei:
+            E.run(d, tiles, bufs)
+        assert ei.value.status == -5
+
+
+def test_ccsd_tc_full_size_dims48_sampled(cuda_device):
+    n = 48
+    d = E.desc_builtin("ccsd_t_d1", (n,)); d.set_exec(50, TENSOR)
+    t2 = synth.uniform((n, n, n, n), 110); v2 = synth.uniform((n, n, n, n), 111)
+    t3d = torch.zeros(n ** 6, dtype=torch.float32, device="cuda")
+    E.run(d, (1, 1, 1, 48, 2, 48, 48), [t3d, dev(t2), dev(v2)])
+    g = synth.rng(112)
+    idx = np.concatenate([g.integers(0, n ** 6, 100000), np.arange(n ** 4) + 7 * n ** 5 + 3 * n ** 4])
+    got = t3d[torch.from_numpy(idx).cuda()].double().cpu().numpy()
+    ref = O.ccsd_t_d1_entries((n,) * 7, idx, np.zeros(len(idx)), t2, v2)
+    assert O.normwise_rel_err(got, ref) <= 1e-5
+    del t3d
+    torch.cuda.empty_cache()
