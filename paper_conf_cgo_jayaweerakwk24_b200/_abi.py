@@ -105,7 +105,7 @@ DECLS = [
 def load(path: str = LIB_PATH) -> ctypes.CDLL:
     if not os.path.exists(path):
         raise ImportError(
-            f"{path} not found: build it with `python -m paper_conf_cgo_jayaweerakwk24_b200.build` "
+            f"{path} not found: build it with `python paper_conf_cgo_jayaweerakwk24_b200/build.py` "
             "(there is no CPU fallback)")
     lib = ctypes.CDLL(path)
     for name, res, args in DECLS:

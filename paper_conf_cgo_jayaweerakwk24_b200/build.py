@@ -1,6 +1,6 @@
 """Build libeatss.so in-tree with nvcc for sm_100a (no torch extension machinery).
 
-    python -m paper_conf_cgo_jayaweerakwk24_b200.build [--force] [-j N]
+    python paper_conf_cgo_jayaweerakwk24_b200/build.py [--force] [-j N]
 
 Every source under csrc/ is compiled to an object in build/ (parallel), then
 linked into paper_conf_cgo_jayaweerakwk24_b200/libeatss.so.  Objects are rebuilt
