@@ -1,0 +1,132 @@
+#!/usr/bin/env python
+"""EATSS candidate protocol across shared-memory splits and warp fractions.
+
+    python harness/candidates.py [--kinds gemm,2mm,...] [--window 0.6] [--out cand.jsonl]
+
+The paper does not use one EATSS tile per kernel: it generates candidates over the L1/shared
+split (SPLIT_FACTOR; "three configurations", "0%, 50% or 67%, and 100%")
+and the warp fraction (WARP_ALIGNMENT_FACTOR = warp_frac * 32, "as small as 4"),
+runs each candidate with the matching carve-out, and keeps the best measured PPW (Figs. 8, 10).
+This harness does that on B200 with the library's own model (B200 mode, mode = 1) and the SIMT
+executor family the sweep uses (engine = SIMT; the paper's code class):
+
+  * candidates: sigma in {0, 50, 100} % (reading Q17) x WAF in {4, 8, 16, 32}; infeasible
+    pairs are recorded (e.g. heat-3d at WAF 32; the 6-D contraction at WAF >= 8);
+  * each distinct (tile, sigma) is measured with eatss_sweep (warm-up, then back-to-back runs
+    for >= --window s, CUDA-event time, NVML energy counter) at carve-out sigma;
+  * baseline: PPCG's default tile (32 per tiled loop) at the same three carve-outs.
+
+The summary gives, per kernel, the best candidate's PPW (GFLOP/s/W = FLOP/J) over
+the best default's PPW -- the quantity behind the paper's "median 1.5x / 1.2x, peak 6.3x" PPW
+gains over PPCG (context only: other GPUs, other code generator).
+Inputs are U[-1,1) on the device (energy must be measured on random data).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+SPLITS = (0, 50, 100)
+WAFS = (4, 8, 16, 32)
+# BASELINE.json configs (reading Q22 sizes)
+KINDS = {
+    "gemm": dict(dims=(4000, 4000, 4000)),
+    "2mm": dict(dims=(4000, 4000, 4000, 4000)),
+    "3mm": dict(dims=(4000, 4000, 4000, 4000, 4000)),
+    "syrk": dict(dims=(4000, 4000)),
+    "jacobi-2d": dict(dims=(4000,), tsteps=500),
+    "heat-3d": dict(dims=(120,), tsteps=500),
+    "ccsd_t_d1": dict(dims=(48,)),
+}
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--kinds", default=",".join(KINDS))
+    ap.add_argument("--window", type=float, default=0.6)
+    ap.add_argument("--warmup", type=int, default=2)
+    ap.add_argument("--device", type=int, default=0)
+    ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "candidates.jsonl"))
+    return ap.parse_args()
+
+
+def candidates(E, d, gpu):
+    """{(tile, sigma): [(sigma, waf), ...]} plus the infeasible (sigma, waf) pairs."""
+    out, infeasible = {}, []
+    for s in SPLITS:
+        for w in WAFS:
+            try:
+                t, rep = E.select_tiles(d, gpu, split_pct=s, waf=w, mode=1)
+            except E.EatssError as e:
+                if e.status != -2:
+                    raise
+                infeasible.append((s, w))
+                continue
+            out.setdefault((tuple(t), s), []).append((s, w, int(rep.obj)))
+    return out, infeasible
+
+
+def measure(E, d, tiles, split, bufs, a):
+    d.set_exec(split_pct=split, engine=1)
+    m = E.sweep(d, [tiles], bufs, device=a.device, warmup=a.warmup, min_window_s=a.window)[0]
+    return dict(ms=m.ms_per_run, joules=m.joules_per_run, watts=m.avg_watts, tflops=m.tflops,
+                ppw=m.gflops_per_watt, sm_mhz=m.sm_mhz_median, status=m.status)
+
+
+def main():
+    a = parse()
+    import torch
+
+    import paper_conf_cgo_jayaweerakwk24_b200 as E
+
+    torch.cuda.set_device(a.device)
+    gpu = E.gpu_params_query(a.device)
+    os.makedirs(os.path.dirname(a.out), exist_ok=True)
+    summary = {}
+    with open(a.out, "a") as f:
+        for kind in a.kinds.split(","):
+            cfg = KINDS[kind]
+            d = E.desc_builtin(kind, cfg["dims"], tsteps=cfg.get("tsteps", 0))
+            gen = torch.Generator(device="cuda").manual_seed(0)
+            bufs = [torch.rand(d.buffer_elems(i), device="cuda", generator=gen) * 2 - 1 for i in range(d.num_buffers)]
+            cands, infeasible = candidates(E, d, gpu)
+            default = tuple([32] * d.num_loops)
+            rows = []
+            for (tiles, s), origin in sorted(cands.items(), key=lambda kv: (kv[0][1], kv[0][0])):
+                r = measure(E, d, tiles, s, bufs, a)
+                rec = dict(kind=kind, role="eatss", tiles=list(tiles), split=s, origin=origin, **r)
+                rows.append(rec)
+                f.write(json.dumps(rec) + "\n"); f.flush()
+            for s in SPLITS:
+                r = measure(E, d, default, s, bufs, a)
+                rec = dict(kind=kind, role="default", tiles=list(default), split=s, **r)
+                rows.append(rec)
+                f.write(json.dumps(rec) + "\n"); f.flush()
+            ok = [r for r in rows if r["status"] == 0 and r["ppw"] > 0]
+            ea = [r for r in ok if r["role"] == "eatss"]
+            de = [r for r in ok if r["role"] == "default"]
+            if ea and de:
+                be = max(ea, key=lambda r: r["ppw"]); bd = max(de, key=lambda r: r["ppw"])
+                pe = max(ea, key=lambda r: r["tflops"])
+                summary[kind] = dict(
+                    best_candidate=dict(tiles=be["tiles"], split=be["split"], origin=be["origin"],
+                                        ppw=be["ppw"], tflops=be["tflops"], watts=be["watts"]),
+                    fastest_candidate=dict(tiles=pe["tiles"], split=pe["split"], ppw=pe["ppw"], tflops=pe["tflops"]),
+                    best_default=dict(split=bd["split"], ppw=bd["ppw"], tflops=bd["tflops"], watts=bd["watts"]),
+                    ppw_gain_vs_default=be["ppw"] / bd["ppw"],
+                    n_candidates=len(ea), infeasible=infeasible)
+            print(kind, json.dumps(summary.get(kind)), flush=True)
+            del bufs
+            torch.cuda.empty_cache()
+    with open(a.out.replace(".jsonl", ".summary.json"), "w") as g:
+        json.dump(dict(created=time.time(), window_s=a.window, splits=SPLITS, wafs=WAFS, kinds=summary), g, indent=1)
+
+
+if __name__ == "__main__":
+    main()

@@ -36,7 +36,8 @@ namespace ccsdtc {
 
 using namespace tcm;
 
-constexpr int NEPI = 8;  // epilogue warps
+constexpr int NGRP = 3;          // epilogue groups; group g owns the units u with u % NGRP == g
+constexpr int NEPI = 4 * NGRP;   // epilogue warps (a group = one warp per TMEM lane quarter)
 constexpr int NTHREADS = (4 + NEPI) * 32;
 constexpr int MROWS = 128;  // UMMA M
 
@@ -181,7 +182,9 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     ccsd_tc_kernel(const float *__restrict__ t2, const __grid_constant__ CUtensorMap mV,
                    const __grid_constant__ CUtensorMap mVlo, const __grid_constant__ CUtensorMap mX, const Args p) {
     extern __shared__ __align__(1024) unsigned char smem_raw[];
-    unsigned char *smem = reinterpret_cast<unsigned char *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
+    // align by pointer arithmetic on the shared array (an integer round trip would make every
+    // access through `smem` a generic-address access)
+    unsigned char *smem = smem_raw + ((1024u - (su32(smem_raw) & 1023u)) & 1023u);
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     // layout: V ring [SV] {hi [nkb], lo [nkb]}, X ring [SX], barriers
     unsigned char *vring = smem;
@@ -202,7 +205,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         for (int s = 0; s < p.SX; s++) {
             mbar_init(xfull + s, 1);
             mbar_init(xempty + s, 1);
-            mbar_init(xdone + s, NEPI);
+            mbar_init(xdone + s, 4);
         }
         for (int s = 0; s < p.SV; s++) {
             mbar_init(vfull + s, 1);
@@ -210,9 +213,9 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         }
         for (int b = 0; b < 4; b++) {
             mbar_init(dfull + b, 1);
-            mbar_init(dempty + b, NEPI);
+            mbar_init(dempty + b, 4);
         }
-        mbar_init(afull, NEPI);  // the epilogue warps write A into TMEM
+        mbar_init(afull, 4);  // the owning epilogue group writes A into TMEM
         mbar_init(aempty, 1);
         asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
         asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&mX)) : "memory");
@@ -313,6 +316,8 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             bulk_wait_all();
         }
     } else if (warp >= 4) {  // ------------------------------------------------ epilogue
+        // group g = (warp - 4) / 4 takes every NGRP-th unit, so NGRP units are in their epilogue
+        // at once (the per-unit chain -- wait, TMEM load, shared RMW, release -- is latency-bound)
         const int q = warp & 3, g = (warp - 4) >> 2, m = q * 32 + lane;
         const int Mrows = p.Th1 * p.Tp5 * p.Tp4;
         const int p4l = m % p.Tp4, p5l = (m / p.Tp4) % p.Tp5, h1l = m / (p.Tp4 * p.Tp5);
@@ -320,62 +325,67 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         const int xrow0 = (h1l * p.Tp6 * p.Tp5 + p5l) * p.Tp4 + p4l, xstep = p.Tp5 * p.Tp4;  // + p6 * xstep
         const uint32_t trow = tmem + ((uint32_t)(q * 32) << 16);
         UnitIter w = iter_begin(p, sc);
-        int a_prev = -1, na = 0;
+        int a_prev = -1, na = 0, own = g;  // own: units until this group's next unit
         Ring rx, rd;
-        for (int64_t u = 0; u < sc.n; u++, iter_next(p, sc, w), rx.next(p.SX), rd.next(p.NB)) {
-            if (w.a != a_prev) {  // new A tile: row m of t2 (as [h1][p5][p4] x h7) into TMEM
-                int h1_0, p5_0, p4_0;
-                a_coords(p, w.a, h1_0, p5_0, p4_0);
-                const int h1 = h1_0 + h1l, p5 = p5_0 + p5l, p4 = p4_0 + p4l;
-                const bool in = live && h1 < p.H1 && p5 < p.P5 && p4 < p.P4;
-                const float *src = t2 + (((int64_t)p4 * p.P5 + p5) * p.H1 + h1);
-                const int64_t hstride = (int64_t)p.P4 * p.P5 * p.H1;
-                if (na > 0) mbar_wait(aempty, (unsigned)((na - 1) & 1));  // MMAs on the old A are done
-                for (int k8 = g; k8 < p.nks; k8 += 2) {
-                    uint32_t hi[8], lo[8];
+        for (int64_t u = 0; u < sc.n; u++, iter_next(p, sc, w), rx.next(p.SX), rd.next(p.NB), own--) {
+            const bool mine = own == 0;
+            if (mine) own = NGRP;
+            if (w.a != a_prev) {  // new A tile: the group owning this unit writes row m of t2 into TMEM
+                if (mine) {
+                    int h1_0, p5_0, p4_0;
+                    a_coords(p, w.a, h1_0, p5_0, p4_0);
+                    const int h1 = h1_0 + h1l, p5 = p5_0 + p5l, p4 = p4_0 + p4l;
+                    const bool in = live && h1 < p.H1 && p5 < p.P5 && p4 < p.P4;
+                    const float *src = t2 + (((int64_t)p4 * p.P5 + p5) * p.H1 + h1);
+                    const int64_t hstride = (int64_t)p.P4 * p.P5 * p.H1;
+                    if (na > 0) mbar_wait(aempty, (unsigned)((na - 1) & 1));  // MMAs on the old A are done
+                    for (int k8 = 0; k8 < p.nks; k8++) {
+                        uint32_t hi[8], lo[8];
 #pragma unroll
-                    for (int c = 0; c < 8; c++) {
-                        const int h7 = 8 * k8 + c;
-                        const float x = (in && h7 < p.H7) ? __ldg(src + h7 * hstride) : 0.f;
-                        hi[c] = __float_as_uint(x);
-                        lo[c] = __float_as_uint(lo_of(x));
+                        for (int c = 0; c < 8; c++) {
+                            const int h7 = 8 * k8 + c;
+                            const float x = (in && h7 < p.H7) ? __ldg(src + h7 * hstride) : 0.f;
+                            hi[c] = __float_as_uint(x);
+                            lo[c] = __float_as_uint(lo_of(x));
+                        }
+                        tmem_st8(trow + (uint32_t)(p.a_col + 16 * k8), hi);
+                        tmem_st8(trow + (uint32_t)(p.a_col + 16 * k8 + 8), lo);
                     }
-                    tmem_st8(trow + (uint32_t)(p.a_col + 16 * k8), hi);
-                    tmem_st8(trow + (uint32_t)(p.a_col + 16 * k8 + 8), lo);
+                    wait_st();
+                    fence_before();
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(afull);
                 }
-                wait_st();
-                fence_before();
-                __syncwarp();
-                if (lane == 0) mbar_arrive(afull);
                 a_prev = w.a;
                 na++;
             }
+            if (!mine) continue;
             mbar_wait(xfull + rx.s, rx.ph);
             mbar_wait(dfull + rd.s, rd.ph);
             fence_after();
             float *xs = reinterpret_cast<float *>(xring + (size_t)rx.s * p.x_stage) + xrow0;
-            // columns (p6) in chunks of 8, alternating between the two epilogue groups; up to three
-            // chunks per batch: all TMEM loads, then all shared loads, then the stores (no
-            // load-store serialisation through possibly-aliasing addresses)
-            for (int c0 = 8 * g; c0 < p.Tp6; c0 += 48) {
-                uint32_t v[3][8];
-                const int nc = min(3, (p.Tp6 - c0 + 15) / 16);
+            // columns (p6) in batches of up to four 8-column chunks: all TMEM loads, then all
+            // shared loads, then the stores (no serialisation through possibly-aliasing addresses)
+            for (int c0 = 0; c0 < p.Tp6; c0 += 32) {
+                uint32_t v[4][8];
+                const int nc = min(4, (p.Tp6 - c0 + 7) / 8);
                 tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0), v[0]);
-                if (nc > 1) tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0 + 16), v[1]);
-                if (nc > 2) tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0 + 32), v[2]);
+                if (nc > 1) tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0 + 8), v[1]);
+                if (nc > 2) tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0 + 16), v[2]);
+                if (nc > 3) tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0 + 24), v[3]);
                 wait_ld();
                 if (live) {
-                    float x[3][8];
+                    float x[4][8];
 #pragma unroll
-                    for (int j = 0; j < 3; j++)
-#pragma unroll
-                        for (int c = 0; c < 8; c++)
-                            if (j < nc) x[j][c] = xs[(c0 + 16 * j + c) * xstep];
-#pragma unroll
-                    for (int j = 0; j < 3; j++)
+                    for (int j = 0; j < 4; j++)
 #pragma unroll
                         for (int c = 0; c < 8; c++)
-                            if (j < nc) xs[(c0 + 16 * j + c) * xstep] = x[j][c] - __uint_as_float(v[j][c]);
+                            if (j < nc) x[j][c] = xs[(c0 + 8 * j + c) * xstep];
+#pragma unroll
+                    for (int j = 0; j < 4; j++)
+#pragma unroll
+                        for (int c = 0; c < 8; c++)
+                            if (j < nc) xs[(c0 + 8 * j + c) * xstep] = x[j][c] - __uint_as_float(v[j][c]);
                 }
             }
             fence_before();

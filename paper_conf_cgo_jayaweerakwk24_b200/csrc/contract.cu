@@ -42,6 +42,7 @@ struct CArgs {
     int Ti, Tj, Tk;
     int a_smem, b_smem, nbuf;
     int tkp, tjp;
+    int bkp;  // staged transposed operand: B slice kept as [j][k] with this k-pitch (0 = [k][j] layout)
     int passes_i, passes_j;
     int32_t *counts;  // coverage mode
 };
@@ -539,11 +540,23 @@ ContractPlan plan_contraction(const ContractNest &n, const int64_t *tiles, int s
         // (S = 1) so two CTAs share an SM and overlap each other's copies; kst is halved only
         // when a k-tile does not fit.  EATSS_STAGES / EATSS_KSUB override for experiments.
         const int64_t aip = ((p.Ti + 3) / 4) * 4, bjp = ((p.Tj + 3) / 4) * 4;
-        int64_t kst = p.Tk, S = 1;
-        while (kst > 1 && S * (kst * (aip + bjp) * esz + 16) > smem_limit) kst = (kst + 1) / 2;
+        // transposed operand (syrk: B(k, j) = A(j, k)), fp32: stage it untransposed as [j][k] rows
+        // with 16-byte copies (k-pitch kst + 4: conflict-free 16-byte reads along k)
+        const uintptr_t bb = reinterpret_cast<uintptr_t>(n.B);
+        const bool bt4 = n.transB && !n.f64 && n.ldb % 4 == 0 && bb % 16 == 0 &&
+                         !(getenv("EATSS_TRANSB_LEGACY") && atoi(getenv("EATSS_TRANSB_LEGACY")));
+        auto stage_of = [&](int64_t ks) {
+            const int64_t b = bt4 ? bjp * (ks + 4) : ks * bjp;
+            return (ks * aip + b) * esz;
+        };
+        int64_t kst = bt4 ? ((p.Tk + 3) / 4) * 4 : p.Tk, S = 1;
+        const int64_t kmin = bt4 ? 4 : 1;
+        while (kst > kmin && S * (stage_of(kst) + 16) > smem_limit)
+            kst = bt4 ? std::max<int64_t>(4, ((kst / 2 + 3) / 4) * 4) : (kst + 1) / 2;
         if (const char *e = getenv("EATSS_STAGES")) S = std::max(1, atoi(e));
         if (const char *e = getenv("EATSS_KSUB")) kst = std::max<int64_t>(1, (p.Tk + atoi(e) - 1) / std::max(1, atoi(e)));
-        const int64_t stage_bytes = kst * (aip + bjp) * esz;
+        if (bt4) kst = ((kst + 3) / 4) * 4;
+        const int64_t stage_bytes = stage_of(kst);
         if (S * (stage_bytes + 16) > smem_limit) S = std::max<int64_t>(1, smem_limit / (stage_bytes + 16));
         if (S * (stage_bytes + 16) <= smem_limit && !(getenv("EATSS_NO_STAGED") && atoi(getenv("EATSS_NO_STAGED")))) {
             p.staged = true;
@@ -551,6 +564,7 @@ ContractPlan plan_contraction(const ContractNest &n, const int64_t *tiles, int s
             p.kst = (int)kst;
             p.tkp = (int)aip;
             p.tjp = (int)bjp;
+            p.bkp = bt4 ? (int)(kst + 4) : 0;
             p.a_smem = true;
             p.b_smem = true;
             p.smem_bytes = (int)(S * stage_bytes + 16 * S);  // + one mbarrier per stage
@@ -676,7 +690,7 @@ static cudaError_t launch_typed(const ContractNest &n, const ContractPlan &p, in
     a.Ti = (int)p.Ti; a.Tj = (int)p.Tj;
     a.Tk = p.staged ? p.kst : (int)p.Tk;  // the staged kernel walks k in ring stages of kst rows
     a.a_smem = p.a_smem; a.b_smem = p.b_smem; a.nbuf = p.nbuf;
-    a.tkp = p.tkp; a.tjp = p.tjp;
+    a.tkp = p.tkp; a.tjp = p.tjp; a.bkp = p.bkp;
     a.passes_i = p.passes_i; a.passes_j = p.passes_j;
     a.counts = counts;
     if (counts) return by_variant<T, MODE_COVER>(a, p, n.transB, carveout, s);

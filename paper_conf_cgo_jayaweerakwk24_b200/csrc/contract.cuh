@@ -34,6 +34,7 @@ struct ContractPlan {
     int nbuf = 1;
     int kst = 0;  // staged path: k-rows per ring stage
     int tkp = 0, tjp = 0;  // shared-memory pitches (elements)
+    int bkp = 0;           // staged transposed operand kept as [j][k] rows of this k-pitch (0 = [k][j])
     int smem_bytes = 0;
     int64_t grid_x = 1, grid_y = 1;
 };

@@ -51,7 +51,10 @@ __global__ void __launch_bounds__((16384 / (RM * RN)) < 1024 ? (16384 / (RM * RN
     T *const sm = reinterpret_cast<T *>(smem_raw);
     const int aip = p.tkp;  // A^T pitch (>= Ti, multiple of 4)
     const int bjp = p.tjp;  // B pitch (>= Tj, multiple of 4)
-    const int stage_elems = p.Tk * (aip + bjp);
+    // B slice: [k][j] (pitch bjp), or for a transposed operand with p.bkp > 0 untransposed [j][k]
+    // rows (pitch bkp, 16-byte aligned) filled by 16-byte copies and read 4 k at a time
+    const bool BT4 = TRANSB && sizeof(T) == 4 && p.bkp > 0;
+    const int stage_elems = p.Tk * aip + (BT4 ? bjp * p.bkp : p.Tk * bjp);
     const int S = p.nbuf;
     uint64_t *bars = reinterpret_cast<uint64_t *>(sm + S * stage_elems);  // 8-byte aligned (elems % 2 == 0)
 
@@ -83,7 +86,7 @@ __global__ void __launch_bounds__((16384 / (RM * RN)) < 1024 ? (16384 / (RM * RN
         return w;
     };
     const Walk wa = mkwalk(p.Tk);  // A: (row, k), k fastest -> coalesced reads
-    const Walk wb = TRANSB ? mkwalk(p.Tk) : mkwalk(V == 4 ? cols >> 2 : cols);
+    const Walk wb = TRANSB ? mkwalk(BT4 ? p.Tk >> 2 : p.Tk) : mkwalk(V == 4 ? cols >> 2 : cols);
 
     auto stage = [&](int t) {
         if (t < nk) {
@@ -105,7 +108,19 @@ __global__ void __launch_bounds__((16384 / (RM * RN)) < 1024 ? (16384 / (RM * RN
                 kk += wa.dI;
                 if (kk >= wa.inner) { kk -= wa.inner; r++; }
             }
-            if constexpr (TRANSB) {
+            if (BT4) {  // row jj of B^T: k0 .. k0 + kt, 16-byte chunks (scalar tail chunk)
+                for (int jj = wb.o0, c = wb.i0; jj < cols;) {
+                    const T *src = p.B + (j0 + jj) * p.ldb + k0 + 4 * c;
+                    T *dst = Bs + jj * p.bkp + 4 * c;
+                    if (4 * c + 4 <= kt) cp_async16(dst, src);
+                    else
+                        for (int e = 0; e < 4; e++)
+                            if (4 * c + e < kt) cp_elem(dst + e, src + e);
+                    jj += wb.dO;
+                    c += wb.dI;
+                    if (c >= wb.inner) { c -= wb.inner; jj++; }
+                }
+            } else if constexpr (TRANSB) {
                 for (int jj = wb.o0, kk = wb.i0; jj < cols;) {
                     if (kk < kt) cp_elem(Bs + kk * bjp + jj, p.B + (j0 + jj) * p.ldb + k0 + kk);
                     jj += wb.dO;
@@ -163,6 +178,51 @@ __global__ void __launch_bounds__((16384 / (RM * RN)) < 1024 ? (16384 / (RM * RN
             for (int c = 0; c < RN; c++) acc[r][c] = fma(a[r], b[c], acc[r][c]);
     };
 
+    // transposed operand in [j][k] rows: four k per pass, one 16-byte read per owned column
+    auto loada = [&](const T *As, int kk, T (&a)[RM]) {
+        if constexpr (sizeof(T) == 4 && RM % 4 == 0) {
+#pragma unroll
+            for (int r = 0; r < RM; r += 4) {
+                const float4 v = *reinterpret_cast<const float4 *>(As + kk * aip + r0 + r);
+                a[r] = v.x; a[r + 1] = v.y; a[r + 2] = v.z; a[r + 3] = v.w;
+            }
+        } else {
+#pragma unroll
+            for (int r = 0; r < RM; r++) a[r] = As[kk * aip + r0 + r];
+        }
+    };
+    auto body4t = [&](const T *As, const T *Bs, int kk) {
+        if constexpr (TRANSB && sizeof(T) == 4 && V == 1) {
+            float b[RN][4];
+#pragma unroll
+            for (int c = 0; c < RN; c++) {
+                const float4 v = *reinterpret_cast<const float4 *>(Bs + cc[c] * p.bkp + kk);
+                b[c][0] = v.x; b[c][1] = v.y; b[c][2] = v.z; b[c][3] = v.w;
+            }
+#pragma unroll
+            for (int q = 0; q < 4; q++) {
+                T a[RM];
+                loada(As, kk + q, a);
+#pragma unroll
+                for (int r = 0; r < RM; r++)
+#pragma unroll
+                    for (int c = 0; c < RN; c++) acc[r][c] = fma(a[r], b[c][q], acc[r][c]);
+            }
+        }
+    };
+    auto body1t = [&](const T *As, const T *Bs, int kk) {
+        if constexpr (TRANSB && V == 1) {
+            T a[RM], b[RN];
+            loada(As, kk, a);
+#pragma unroll
+            for (int c = 0; c < RN; c++) b[c] = Bs[cc[c] * p.bkp + kk];
+#pragma unroll
+            for (int r = 0; r < RM; r++)
+#pragma unroll
+                for (int c = 0; c < RN; c++) acc[r][c] = fma(a[r], b[c], acc[r][c]);
+        }
+    };
+
     for (int s = 0; s < S - 1; s++) stage(s);
     for (int t = 0; t < nk; t++) {
         stage(t + S - 1);
@@ -175,11 +235,16 @@ __global__ void __launch_bounds__((16384 / (RM * RN)) < 1024 ? (16384 / (RM * RN
         const T *Bs = As + p.Tk * aip;
         const int kt = (int)imin64(p.Tk, p.K - (int64_t)t * p.Tk);
         int kk = 0;
-        for (; kk + 4 <= kt; kk += 4) {
+        if (BT4) {
+            for (; kk + 4 <= kt; kk += 4) body4t(As, Bs, kk);
+            for (; kk < kt; kk++) body1t(As, Bs, kk);
+        } else {
+            for (; kk + 4 <= kt; kk += 4) {
 #pragma unroll
-            for (int q = 0; q < 4; q++) body(As, Bs, kk + q);
+                for (int q = 0; q < 4; q++) body(As, Bs, kk + q);
+            }
+            for (; kk < kt; kk++) body(As, Bs, kk);
         }
-        for (; kk < kt; kk++) body(As, Bs, kk);
         __syncthreads();
     }
     cp_async_wait<0>();

@@ -20,6 +20,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <cstdlib>
 
 namespace eatss {
 
@@ -240,6 +241,17 @@ __global__ void __launch_bounds__(256) heat3d_sweep(T *__restrict__ dst, const T
 }
 
 // ------------------------------------------------------------------ launchers
+// shared-memory-staged fast path (stencil_staged.cu); EATSS_STENCIL_STAGED=0 selects the column walks
+bool jacobi2d_staged_applicable(int64_t n, int64_t Ti, int64_t Tj, bool f64);
+bool heat3d_staged_applicable(int64_t n, int64_t Ti, int64_t Tj, int64_t Tk, bool f64);
+cudaError_t launch_jacobi2d_staged(float *dst, const float *src, const float *bsrc, int64_t n, int64_t Ti, int64_t Tj,
+                                   int split_pct, int32_t *counts, cudaStream_t s);
+cudaError_t launch_heat3d_staged(float *dst, const float *src, int64_t n, int64_t Ti, int64_t Tj, int64_t Tk,
+                                 int split_pct, int32_t *counts, cudaStream_t s);
+static bool stencil_staged_enabled() {
+    static const bool on = !(getenv("EATSS_STENCIL_STAGED") && atoi(getenv("EATSS_STENCIL_STAGED")) == 0);
+    return on;
+}
 static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
 struct StencilPlan {
@@ -276,6 +288,9 @@ StencilPlan plan_heat3d(int64_t n, int64_t Ti, int64_t Tj, int64_t Tk, bool f64)
 
 cudaError_t launch_jacobi2d_sweep(void *dst, const void *src, const void *bsrc, int64_t n, int64_t Ti,
                                   int64_t Tj, bool f64, int carveout, int32_t *counts, cudaStream_t s) {
+    if (stencil_staged_enabled() && jacobi2d_staged_applicable(n, Ti, Tj, f64))
+        return launch_jacobi2d_staged((float *)dst, (const float *)src, (const float *)bsrc, n, Ti, Tj, carveout,
+                                      counts, s);
     StencilPlan p = plan_jacobi2d(n, Ti, Tj, f64);
     dim3 grid((unsigned)p.gx, (unsigned)p.gy), block(p.bx, p.by);
     if (p.gy > 65535) return cudaErrorInvalidConfiguration;
@@ -310,6 +325,8 @@ cudaError_t launch_interior_copy2d(void *dst, const void *src, int64_t n, bool f
 
 cudaError_t launch_heat3d_sweep(void *dst, const void *src, int64_t n, int64_t Ti, int64_t Tj,
                                 int64_t Tk, bool f64, int carveout, int32_t *counts, cudaStream_t s) {
+    if (stencil_staged_enabled() && heat3d_staged_applicable(n, Ti, Tj, Tk, f64))
+        return launch_heat3d_staged((float *)dst, (const float *)src, n, Ti, Tj, Tk, carveout, counts, s);
     StencilPlan p = plan_heat3d(n, Ti, Tj, Tk, f64);
     if (p.gy > 65535) return cudaErrorInvalidConfiguration;
     const int nbj = (int)cdiv(n - 1, Tj);

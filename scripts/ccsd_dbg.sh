@@ -1,14 +1,18 @@
 cd $GRAFT_REPO_ROOT
-for dbg in 0 1 2 4 3 5 6 7; do echo "== dbg $dbg"; EATSS_CCSD_TC_DBG=$dbg timeout 300 python scripts/time_kernel.py ccsd_t_d1 48 1,1,1,48,2,48,48 --engine 2 --iters 5 2>&1 | tail -1; done
-echo "== M48 dbg 2"; EATSS_CCSD_TC_DBG=2 timeout 300 python scripts/time_kernel.py ccsd_t_d1 48 1,1,1,48,1,48,48 --engine 2 --iters 5 2>&1 | tail -1
-echo "== M48 dbg 6"; EATSS_CCSD_TC_DBG=6 timeout 300 python scripts/time_kernel.py ccsd_t_d1 48 1,1,1,48,1,48,48 --engine 2 --iters 5 2>&1 | tail -1
+# dbg bits (development only): 1 no MMA, 2 no t3 traffic, 4 no v2 loads
+for dbg in 0 1 2 4 5 6 7; do echo "== dbg $dbg"; EATSS_CCSD_TC_DBG=$dbg timeout 300 python scripts/time_kernel.py ccsd_t_d1 48 1,1,1,48,2,48,48 --engine 2 --iters 5 2>&1 | tail -1; done
+for xs in 3 4 5; do echo "== xstages $xs"; EATSS_CCSD_TC_XSTAGES=$xs timeout 300 python scripts/time_kernel.py ccsd_t_d1 48 1,1,1,48,2,48,48 --engine 2 --iters 5 2>&1 | tail -1; done
+echo "== order 0"; EATSS_CCSD_TC_ORDER=0 timeout 300 python scripts/time_kernel.py ccsd_t_d1 48 1,1,1,48,2,48,48 --engine 2 --iters 5 2>&1 | tail -1
 python - <<'PY'
-import torch, time
-x = torch.empty(12 * 1024**3 // 4, device="cuda"); y = torch.empty_like(x)
-for _ in range(3): y.copy_(x)
+import torch
+x = torch.empty(48**6, device="cuda")
+x.uniform_()
+for _ in range(2): x.sub_(0.5)
 s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
 torch.cuda.synchronize(); s.record()
-for _ in range(5): y.copy_(x)
+for _ in range(5): x.sub_(0.5)
 e.record(); torch.cuda.synchronize()
-print("copy 12 GiB: %.2f TB/s" % (2 * x.numel() * 4 * 5 / (s.elapsed_time(e) * 1e-3) / 1e12))
+ms = s.elapsed_time(e) / 5
+print("torch in-place RMW over t3 (48.9 GB): %.2f ms, %.2f TB/s" % (ms, 2 * x.numel() * 4 / ms / 1e9))
 PY
+timeout 900 python scripts/ccsd_variants.py
