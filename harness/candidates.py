@@ -111,15 +111,18 @@ def main():
             ok = [r for r in rows if r["status"] == 0 and r["ppw"] > 0]
             ea = [r for r in ok if r["role"] == "eatss"]
             de = [r for r in ok if r["role"] == "default"]
-            if ea and de:
-                be = max(ea, key=lambda r: r["ppw"]); bd = max(de, key=lambda r: r["ppw"])
+            if ea:
+                be = max(ea, key=lambda r: r["ppw"])
                 pe = max(ea, key=lambda r: r["tflops"])
+                bd = max(de, key=lambda r: r["ppw"]) if de else None
                 summary[kind] = dict(
                     best_candidate=dict(tiles=be["tiles"], split=be["split"], origin=be["origin"],
                                         ppw=be["ppw"], tflops=be["tflops"], watts=be["watts"]),
                     fastest_candidate=dict(tiles=pe["tiles"], split=pe["split"], ppw=pe["ppw"], tflops=pe["tflops"]),
-                    best_default=dict(split=bd["split"], ppw=bd["ppw"], tflops=bd["tflops"], watts=bd["watts"]),
-                    ppw_gain_vs_default=be["ppw"] / bd["ppw"],
+                    best_default=(dict(split=bd["split"], ppw=bd["ppw"], tflops=bd["tflops"], watts=bd["watts"])
+                                  if bd else "default tile not executable (launch configuration rejected)"),
+                    ppw_gain_vs_default=be["ppw"] / bd["ppw"] if bd else None,
+                    ppw_spread_over_candidates=be["ppw"] / min(r["ppw"] for r in ea),
                     n_candidates=len(ea), infeasible=infeasible)
             print(kind, json.dumps(summary.get(kind)), flush=True)
             del bufs

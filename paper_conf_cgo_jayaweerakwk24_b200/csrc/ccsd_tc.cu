@@ -45,16 +45,19 @@ struct Args {
     int H3, H2, H1, P6, P5, P4, H7;
     int Th1, Tp6, Tp5, Tp4;
     int n_h1t, n_p5t, n_p4t, n_p6t;
-    int hh0, nhh;     // (h3,h2) flattened range of this launch
+    int Th2, n_h2t;   // h2 tile: Th2 > 1 blocks Th2 consecutive h2 into one unit (needs Tp6 = P6, Tp4 = P4)
+    int NV;           // MMA N = Th2 * Tp6 output columns (h2, p6) per unit
+    int hh0, nhh;     // range of (h3, h2-tile) blocks of this launch (Th2 = 1: flattened (h3, h2))
     int64_t units;    // n_a * nhh * n_p6t
     int nkb;          // ceil(H7 / 32)
     int SV, SX;       // V ring stages, t3-tile ring stages
     int bstride, NB;  // TMEM accumulator buffers (columns per buffer, count)
     int nks;          // 8-k MMA steps: ceil(H7 / 8)
     int a_col;        // TMEM column of A (hi at a_col + 16 ks, lo at + 8)
-    int v_kb_bytes;   // Tp6 * 128
+    int v_kb_bytes;   // NV * 128
     int v_stage;      // 2 * nkb * v_kb_bytes
-    int x_bytes;      // Th1*Tp6*Tp5*Tp4*4
+    int x_bytes;      // Th2*Th1*Tp6*Tp5*Tp4*4
+    int pend;         // t3 stores kept in flight before their ring slot is released
     int x_stage;      // x_bytes rounded up to 1 KB
     int order;        // 1: A tiles round-robin over CTAs (concurrent CTAs sweep whole t3 blocks)
     int dbg;          // development only (EATSS_CCSD_TC_DBG): 1 no MMA, 2 no t3 traffic, 4 no v2 loads
@@ -125,6 +128,23 @@ __device__ __forceinline__ void a_coords(const Args &p, int a, int &h1_0, int &p
     h1_0 = h1t * p.Th1;
     p5_0 = p5t * p.Tp5;
     p4_0 = p4t * p.Tp4;
+}
+
+// t3 tile coordinates of a unit in the 5-D tensor map: Th2 = 1 -> dims (p4, p5, p6, h1, (h3,h2));
+// Th2 > 1 -> dims ((p5,p4), p6, h1, h2, h3) (Tp4 = P4), so a tile never straddles two h3
+__device__ __forceinline__ void x_coords(const Args &p, int hb, int p6t, int h1_0, int p5_0, int p4_0, int (&c)[5]) {
+    if (p.Th2 == 1) {
+        c[0] = p4_0; c[1] = p5_0; c[2] = p6t * p.Tp6; c[3] = h1_0; c[4] = hb;
+    } else {
+        const int h3 = hb / p.n_h2t, h2_0 = (hb - h3 * p.n_h2t) * p.Th2;
+        c[0] = p5_0 * p.P4 + p4_0; c[1] = p6t * p.Tp6; c[2] = h1_0; c[3] = h2_0; c[4] = h3;
+    }
+}
+// first row of the unit's v2 tile in v2 viewed as [(h3, h2, p6)][h7]
+__device__ __forceinline__ int v_row(const Args &p, int hb, int p6t) {
+    if (p.Th2 == 1) return hb * p.P6 + p6t * p.Tp6;
+    const int h3 = hb / p.n_h2t, h2_0 = (hb - h3 * p.n_h2t) * p.Th2;
+    return (h3 * p.H2 + h2_0) * p.P6 + p6t * p.Tp6;
 }
 
 // Incremental walk over a CTA's units (no 64-bit divisions in the loops): region 1 = whole A
@@ -242,8 +262,9 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                 if (u >= p.SX) mbar_wait(xempty + r.s, r.ph ^ 1u);
                 if (p.dbg & 2) { mbar_arrive(xfull + r.s); continue; }
                 mbar_expect_tx(xfull + r.s, p.x_bytes);
-                tma_5d_hint(xring + (size_t)r.s * p.x_stage, &mX, p4_0, p5_0, w.p6t * p.Tp6, h1_0, w.hh, xfull + r.s,
-                            pol);
+                int c[5];
+                x_coords(p, w.hh, w.p6t, h1_0, p5_0, p4_0, c);
+                tma_5d_hint(xring + (size_t)r.s * p.x_stage, &mX, c[0], c[1], c[2], c[3], c[4], xfull + r.s, pol);
             }
         }
     } else if (warp == 3) {
@@ -255,7 +276,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                 unsigned char *st = vring + (size_t)r.s * p.v_stage;
                 if (p.dbg & 4) { mbar_arrive(vfull + r.s); continue; }
                 mbar_expect_tx(vfull + r.s, p.v_stage);
-                const int vrow = w.hh * p.P6 + w.p6t * p.Tp6;
+                const int vrow = v_row(p, w.hh, w.p6t);
                 for (int kb = 0; kb < p.nkb; kb++) {
                     tma_2d<1>(st + kb * p.v_kb_bytes, &mV, kb * 32, vrow, su32(vfull + r.s));
                     tma_2d<1>(st + (p.nkb + kb) * p.v_kb_bytes, &mVlo, kb * 32, vrow, su32(vfull + r.s));
@@ -264,7 +285,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         }
     } else if (warp == 1) {
         if (lane == 0) {  // ------------------------------------------------ MMA issuer
-            const uint32_t ID = idesc(p.Tp6, 1, true);  // M = 128, N = Tp6, A and B K-major
+            const uint32_t ID = idesc(p.NV, 1, true);  // M = 128, N = NV = Th2 * Tp6, A and B K-major
             int a_prev = -1, na = 0;
             UnitIter w = iter_begin(p, sc);
             Ring rv, rd;
@@ -300,18 +321,26 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             const uint64_t pol = policy_evict_first();
             UnitIter w = iter_begin(p, sc);
             Ring r;
-            int pend[3] = {-1, -1, -1};  // stages of the last stores, oldest first
+            int pend[3] = {-1, -1, -1};  // stages of the last p.pend stores, oldest first
             for (int64_t u = 0; u < sc.n; u++, iter_next(p, sc, w), r.next(p.SX)) {
                 int h1_0, p5_0, p4_0;
                 a_coords(p, w.a, h1_0, p5_0, p4_0);
                 mbar_wait(xdone + r.s, r.ph);
                 if (p.dbg & 2) { mbar_arrive(xempty + r.s); continue; }
-                tma_store_5d_hint(&mX, xring + (size_t)r.s * p.x_stage, p4_0, p5_0, w.p6t * p.Tp6, h1_0, w.hh, pol);
+                int c[5];
+                x_coords(p, w.hh, w.p6t, h1_0, p5_0, p4_0, c);
+                tma_store_5d_hint(&mX, xring + (size_t)r.s * p.x_stage, c[0], c[1], c[2], c[3], c[4], pol);
                 bulk_commit();
-                bulk_wait_read<2>();  // all but the 2 newest stores have read their slots
-                if (pend[0] >= 0) mbar_arrive(xempty + pend[0]);
-                pend[0] = pend[1];
-                pend[1] = r.s;
+                if (p.pend == 2) {
+                    bulk_wait_read<2>();  // all but the 2 newest stores have read their slots
+                    if (pend[0] >= 0) mbar_arrive(xempty + pend[0]);
+                    pend[0] = pend[1];
+                    pend[1] = r.s;
+                } else {
+                    bulk_wait_read<1>();
+                    if (pend[0] >= 0) mbar_arrive(xempty + pend[0]);
+                    pend[0] = r.s;
+                }
             }
             bulk_wait_all();
         }
@@ -364,28 +393,34 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             mbar_wait(dfull + rd.s, rd.ph);
             fence_after();
             float *xs = reinterpret_cast<float *>(xring + (size_t)rx.s * p.x_stage) + xrow0;
-            // columns (p6) in batches of up to four 8-column chunks: all TMEM loads, then all
-            // shared loads, then the stores (no serialisation through possibly-aliasing addresses)
-            for (int c0 = 0; c0 < p.Tp6; c0 += 32) {
+            // columns n = (h2l, p6) in batches of up to four 8-column chunks (a chunk never straddles
+            // two h2, Tp6 % 16 == 0): all TMEM loads, then all shared loads, then the stores
+            for (int c0 = 0; c0 < p.NV; c0 += 32) {
                 uint32_t v[4][8];
-                const int nc = min(4, (p.Tp6 - c0 + 7) / 8);
+                const int nc = min(4, (p.NV - c0 + 7) / 8);
                 tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0), v[0]);
                 if (nc > 1) tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0 + 8), v[1]);
                 if (nc > 2) tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0 + 16), v[2]);
                 if (nc > 3) tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0 + 24), v[3]);
                 wait_ld();
                 if (live) {
+                    int cb[4];  // shared offset of each chunk's first column
+#pragma unroll
+                    for (int j = 0; j < 4; j++) {
+                        const int n = c0 + 8 * j, hl = n / p.Tp6;
+                        cb[j] = (hl * p.Th1 * p.Tp6 + (n - hl * p.Tp6)) * xstep;
+                    }
                     float x[4][8];
 #pragma unroll
                     for (int j = 0; j < 4; j++)
 #pragma unroll
                         for (int c = 0; c < 8; c++)
-                            if (j < nc) x[j][c] = xs[(c0 + 8 * j + c) * xstep];
+                            if (j < nc) x[j][c] = xs[cb[j] + c * xstep];
 #pragma unroll
                     for (int j = 0; j < 4; j++)
 #pragma unroll
                         for (int c = 0; c < 8; c++)
-                            if (j < nc) xs[(c0 + 8 * j + c) * xstep] = x[j][c] - __uint_as_float(v[j][c]);
+                            if (j < nc) xs[cb[j] + c * xstep] = x[j][c] - __uint_as_float(v[j][c]);
                 }
             }
             fence_before();
@@ -463,13 +498,16 @@ CcsdTcPlan plan_ccsd_tc(const int64_t *dims, const int64_t *tiles) {
     int64_t T[7];
     for (int i = 0; i < 7; i++) T[i] = std::min(tiles[i], dims[i]);
     const int64_t H3 = dims[0], H2 = dims[1], H1 = dims[2], P6 = dims[3], P5 = dims[4], P4 = dims[5], H7 = dims[6];
-    if (T[0] != 1 || T[1] != 1 || T[6] < H7) return pl;  // one (h3,h2) per unit, whole h7 reduction
+    if (T[0] != 1 || T[6] < H7) return pl;  // one h3 per unit, whole h7 reduction
+    // Th2 > 1: Th2 consecutive h2 per unit (MMA N = Th2 * P6); needs whole p6 and p4 ranges
+    if (T[1] > 1 && (T[3] != P6 || T[5] != P4 || T[1] * P6 > 256 || (T[1] * P6) % 16)) return pl;
     if (H7 > 64 || (H7 % 4) || (P4 % 4) || (T[5] % 4)) return pl;  // 16-byte TMA strides / boxes
     if (T[2] * T[4] * T[5] > ccsdtc::MROWS || (T[3] % 16) || T[3] > 256) return pl;
     if (H3 * H2 > INT32_MAX || H3 * H2 * P6 > INT32_MAX || H1 * P5 * P4 * H7 > INT32_MAX) return pl;
     ccsdtc::Args &a = pl.a;
     a.H3 = (int)H3; a.H2 = (int)H2; a.H1 = (int)H1; a.P6 = (int)P6; a.P5 = (int)P5; a.P4 = (int)P4; a.H7 = (int)H7;
     a.Th1 = (int)T[2]; a.Tp6 = (int)T[3]; a.Tp5 = (int)T[4]; a.Tp4 = (int)T[5];
+    a.Th2 = (int)T[1]; a.n_h2t = (int)((H2 + a.Th2 - 1) / a.Th2); a.NV = a.Th2 * a.Tp6;
     a.n_h1t = (int)((H1 + a.Th1 - 1) / a.Th1); a.n_p5t = (int)((P5 + a.Tp5 - 1) / a.Tp5);
     a.n_p4t = (int)((P4 + a.Tp4 - 1) / a.Tp4); a.n_p6t = (int)((P6 + a.Tp6 - 1) / a.Tp6);
     a.nkb = (int)((H7 + 31) / 32);
@@ -477,13 +515,13 @@ CcsdTcPlan plan_ccsd_tc(const int64_t *dims, const int64_t *tiles) {
     a.dbg = getenv("EATSS_CCSD_TC_DBG") ? atoi(getenv("EATSS_CCSD_TC_DBG")) : 0;
     a.nks = (int)((H7 + 7) / 8);
     a.bstride = 32;
-    while (a.bstride < a.Tp6) a.bstride *= 2;
+    while (a.bstride < a.NV) a.bstride *= 2;
     a.a_col = 384;                            // TMEM: D buffers in [0, 384), A in [384, 512)
     a.NB = std::min(4, 384 / a.bstride);
     if (a.NB < 1) return pl;
-    a.v_kb_bytes = a.Tp6 * 128;
+    a.v_kb_bytes = a.NV * 128;
     a.v_stage = 2 * a.nkb * a.v_kb_bytes;
-    a.x_bytes = a.Th1 * a.Tp6 * a.Tp5 * a.Tp4 * 4;
+    a.x_bytes = a.Th2 * a.Th1 * a.Tp6 * a.Tp5 * a.Tp4 * 4;
     a.x_stage = (a.x_bytes + 1023) / 1024 * 1024;
     const int fixed = 1024 /*align*/ + 512 /*barriers*/;
     a.SV = 4;
@@ -496,6 +534,7 @@ CcsdTcPlan plan_ccsd_tc(const int64_t *dims, const int64_t *tiles) {
     }
     // SX >= 3: the store issuer releases a slot two stores after it was written
     if (a.SX < 3) return pl;
+    a.pend = a.SX >= 4 ? 2 : 1;
     pl.smem = fixed + a.SV * a.v_stage + a.SX * a.x_stage;
     pl.ok = true;
     return pl;
@@ -512,8 +551,8 @@ cudaError_t launch_ccsd_tc(float *t3, const float *t2, const float *v2, const in
     if (!pl.ok || !tcm::encode_fn()) return cudaErrorNotSupported;
     ccsdtc::Args a = pl.a;
     const int64_t H2 = dims[1], H1 = dims[2], P6 = dims[3], P5 = dims[4], P4 = dims[5], H7 = dims[6];
-    a.hh0 = (int)(h3_begin * H2);
-    a.nhh = (int)(h3_count * H2);
+    a.hh0 = (int)(h3_begin * (a.Th2 == 1 ? H2 : a.n_h2t));
+    a.nhh = (int)(h3_count * (a.Th2 == 1 ? H2 : a.n_h2t));
     a.units = (int64_t)a.n_h1t * a.n_p5t * a.n_p4t * a.nhh * a.n_p6t;
     if (a.units == 0) return cudaSuccess;
     const int64_t n_v2 = (int64_t)a.H3 * H2 * P6 * H7;
@@ -526,12 +565,20 @@ cudaError_t launch_ccsd_tc(float *t3, const float *t2, const float *v2, const in
     // V: v2 as [(h3,h2,p6)][h7], box {32, Tp6}, SWIZZLE_128B (K-major UMMA operand)
     const uint64_t vdims[2] = {(uint64_t)H7, (uint64_t)((int64_t)a.H3 * H2 * P6)};
     const uint64_t vstr[1] = {(uint64_t)H7 * 4};
-    const uint32_t vbox[2] = {32, (uint32_t)a.Tp6};
+    const uint32_t vbox[2] = {32, (uint32_t)a.NV};
     // X: t3 as [(h3,h2)][h1][p6][p5][p4], box {Tp4, Tp5, Tp6, Th1, 1}
-    const uint64_t xdims[5] = {(uint64_t)P4, (uint64_t)P5, (uint64_t)P6, (uint64_t)H1, (uint64_t)((int64_t)a.H3 * H2)};
-    const uint64_t xstr[4] = {(uint64_t)P4 * 4, (uint64_t)(P5 * P4) * 4, (uint64_t)(P6 * P5 * P4) * 4,
-                              (uint64_t)(H1 * P6 * P5 * P4) * 4};
-    const uint32_t xbox[5] = {(uint32_t)a.Tp4, (uint32_t)a.Tp5, (uint32_t)a.Tp6, (uint32_t)a.Th1, 1};
+    uint64_t xdims[5] = {(uint64_t)P4, (uint64_t)P5, (uint64_t)P6, (uint64_t)H1, (uint64_t)((int64_t)a.H3 * H2)};
+    uint64_t xstr[4] = {(uint64_t)P4 * 4, (uint64_t)(P5 * P4) * 4, (uint64_t)(P6 * P5 * P4) * 4,
+                        (uint64_t)(H1 * P6 * P5 * P4) * 4};
+    uint32_t xbox[5] = {(uint32_t)a.Tp4, (uint32_t)a.Tp5, (uint32_t)a.Tp6, (uint32_t)a.Th1, 1};
+    if (a.Th2 > 1) {  // dims ((p5,p4), p6, h1, h2, h3)
+        const uint64_t d2[5] = {(uint64_t)(P5 * P4), (uint64_t)P6, (uint64_t)H1, (uint64_t)H2, (uint64_t)a.H3};
+        const uint64_t s2[4] = {(uint64_t)(P5 * P4) * 4, (uint64_t)(P6 * P5 * P4) * 4, (uint64_t)(H1 * P6 * P5 * P4) * 4,
+                                (uint64_t)(H2 * H1 * P6 * P5 * P4) * 4};
+        const uint32_t b2[5] = {(uint32_t)(a.Tp5 * a.Tp4), (uint32_t)a.Tp6, (uint32_t)a.Th1, (uint32_t)a.Th2, 1};
+        for (int i = 0; i < 5; i++) { xdims[i] = d2[i]; xbox[i] = b2[i]; }
+        for (int i = 0; i < 4; i++) xstr[i] = s2[i];
+    }
     if (!ccsdtc::make_map_nd(&mV, v2, 2, vdims, vstr, vbox, CU_TENSOR_MAP_SWIZZLE_128B) ||
         !ccsdtc::make_map_nd(&mVlo, v2_lo, 2, vdims, vstr, vbox, CU_TENSOR_MAP_SWIZZLE_128B) ||
         !ccsdtc::make_map_nd(&mX, t3, 5, xdims, xstr, xbox, CU_TENSOR_MAP_SWIZZLE_NONE))

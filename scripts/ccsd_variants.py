@@ -9,8 +9,8 @@ dims = (int(os.environ.get("H3", n)),) + (n,) * 6
 d = E.desc_builtin("ccsd_t_d1", dims)
 bufs = [torch.rand(d.buffer_elems(i), device="cuda") * 2 - 1 for i in range(3)]
 flops = d.flops
-variants = [(2, t) for t in [(1, 1, 1, 48, 2, 48, 48), (1, 1, 1, 48, 8, 16, 48), (1, 1, 1, 48, 4, 32, 48),
-                             (1, 1, 2, 48, 1, 48, 48), (1, 1, 1, 48, 1, 48, 48)]]
+variants = [(2, t) for t in [(1, 1, 1, 48, 2, 48, 48), (1, 2, 1, 48, 2, 48, 48), (1, 2, 2, 48, 1, 48, 48),
+                             (1, 1, 2, 48, 1, 48, 48)]]
 if os.environ.get("SIMT"):
     variants.append((1, (4, 4, 4, 4, 4, 32, 4)))
 res = {}

@@ -236,7 +236,10 @@ CCSD_TC = [((16,) * 7, (1, 1, 1, 16, 8, 16, 16)), ((16,) * 7, (1, 1, 2, 16, 4, 1
            ((16,) * 7, (1, 1, 1, 16, 2, 16, 16)),
            ((3, 5, 6, 20, 7, 12, 20), (1, 1, 2, 16, 3, 12, 20)),   # ragged h1/p5/p6 tiles, h7 pad
            ((2, 3, 4, 32, 4, 8, 48), (1, 1, 2, 32, 4, 8, 48)),    # two k-blocks (H7 = 48)
-           ((2, 2, 3, 160, 2, 16, 16), (1, 1, 1, 160, 2, 16, 16))]  # N = 160: one TMEM accumulator
+           ((2, 2, 3, 160, 2, 16, 16), (1, 1, 1, 160, 2, 16, 16)),  # N = 160: one TMEM accumulator
+           ((16,) * 7, (1, 2, 1, 16, 4, 16, 16)),                  # Th2 = 2: N = (h2, p6) = 32
+           ((2, 3, 4, 32, 4, 8, 48), (1, 2, 2, 32, 4, 8, 48)),      # ragged h2 tile (H2 = 3), two k-blocks
+           ((3, 5, 3, 16, 5, 12, 20), (1, 4, 2, 16, 3, 12, 20))]   # N = 64, ragged h1/p5, h7 pad
 
 
 @pytest.mark.parametrize("dims,tiles", CCSD_TC)
@@ -263,12 +266,15 @@ def test_ccsd_tc_rejects_non_mma_tiles(cuda_device):
         assert ei.value.status == -5
 
 
+CCSD_TC_TILE48 = (1, 2, 1, 48, 2, 48, 48)  # the tile bench-style timings use at dims 48
+
+
 def test_ccsd_tc_full_size_dims48_sampled(cuda_device):
     n = 48
     d = E.desc_builtin("ccsd_t_d1", (n,)); d.set_exec(50, TENSOR)
     t2 = synth.uniform((n, n, n, n), 110); v2 = synth.uniform((n, n, n, n), 111)
     t3d = torch.zeros(n ** 6, dtype=torch.float32, device="cuda")
-    E.run(d, (1, 1, 1, 48, 2, 48, 48), [t3d, dev(t2), dev(v2)])
+    E.run(d, CCSD_TC_TILE48, [t3d, dev(t2), dev(v2)])
     g = synth.rng(112)
     idx = np.concatenate([g.integers(0, n ** 6, 100000), np.arange(n ** 4) + 7 * n ** 5 + 3 * n ** 4])
     got = t3d[torch.from_numpy(idx).cuda()].double().cpu().numpy()
