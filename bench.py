@@ -35,6 +35,7 @@ METRIC = "GFLOP/s per Watt and TFLOP/s of EATSS-tiled affine kernels (gemm N=400
 FLOPS = 2.0 * N ** 3
 SM_COUNT, FP32_LANES = 148, 128
 TF32_OVER_BF16 = 1.1 / 2.25  # B200_PROFILING.md nominal dense tf32 / bf16
+E2E_ROW_BLOCKS = 8  # eatss_run_host row blocks: copies of block r+1 overlap the gemm of block r
 
 
 def parse():
@@ -47,6 +48,7 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-secondary", action="store_true")
+    ap.add_argument("--no-configs", action="store_true", help="skip the per-config table (BASELINE configs 3-5)")
     return ap.parse_args()
 
 
@@ -229,6 +231,76 @@ def timed(arm, C, A, B, stream, K, torch, clk=None):
     return ms, kern, call, joules
 
 
+# ------------------------------------------------------------------ the other BASELINE configs
+def other_configs(E, torch, gpu, stream, peaks):
+    """Device time of every other BASELINE.json config with the model-selected tile (rank-local,
+    inputs U[-1,1) resident in HBM, CUDA events on the launching stream, whole eatss_run call).
+    Contractions are graded against the 3xTF32 useful peak (tensor engine, reading T) or the FFMA
+    peak (SIMT engine, B200 mode); stencils and the 6-D contraction against measured HBM copy GB/s."""
+    hbm = peaks.get("hbm_gbs", 6538.0)
+    tf32u = peaks.get("bf16_tflops", 1590.0) * TF32_OVER_BF16 / 3
+    ffma = SM_COUNT * FP32_LANES * 2 * peaks.get("sm_max_mhz", 1965.0) * 1e6 / 1e12
+    g = torch.Generator(device="cuda").manual_seed(7)
+
+    def bufs_for(d):
+        return [torch.rand(d.buffer_elems(i), device="cuda", generator=g) * 2 - 1 for i in range(d.num_buffers)]
+
+    def timed_ms(d, tiles, bufs, iters):
+        E.run(d, tiles, bufs, stream)
+        s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        s.record(stream)
+        for _ in range(iters):
+            E.run(d, tiles, bufs, stream)
+        e.record(stream)
+        torch.cuda.synchronize()
+        return s.elapsed_time(e) / iters
+
+    out = {}
+    for kind, dims in (("2mm", (N,) * 4), ("3mm", (N,) * 5), ("syrk", (N, N))):
+        d = E.desc_builtin(kind, dims)
+        b = bufs_for(d)
+        row = {}
+        for eng, mode, peak, bound in ((2, 2, tf32u, "tensor"), (1, 1, ffma, "alu")):
+            tiles, _ = E.select_tiles(d, gpu, split_pct=50, waf=16, mode=mode)
+            d.set_exec(split_pct=50, engine=eng)
+            ms = timed_ms(d, tiles, b, 10 if eng == 2 else 3)
+            tf = d.flops / (ms * 1e-3) / 1e12
+            row["tensor" if eng == 2 else "simt"] = {"tiles": list(tiles), "ms": ms, "tflops": tf,
+                                                     "bound": bound, "frac": tf / peak}
+        out[kind] = row
+        del b
+    for kind, n, T, iters in (("jacobi-2d", 4000, 500, 3), ("jacobi-2d", 16384, 10, 5),
+                              ("heat-3d", 120, 500, 3), ("heat-3d", 512, 5, 5)):
+        d = E.desc_builtin(kind, (n,), tsteps=T)
+        b = bufs_for(d)
+        tiles, _ = E.select_tiles(d, gpu, split_pct=50, waf=16, mode=1)
+        d.set_exec(split_pct=50, engine=1)
+        ms = timed_ms(d, tiles, b, iters)
+        pts = n ** (2 if kind == "jacobi-2d" else 3)
+        sweeps = T + 1 if kind == "jacobi-2d" else 2 * T  # jacobi: ping-pong sweeps + one copy nest
+        gbs = sweeps * 2 * pts * 4 / (ms * 1e-3) / 1e9
+        out[f"{kind} n={n} T={T}"] = {"tiles": list(tiles), "ms": ms, "us_per_sweep": ms * 1e3 / sweeps,
+                                      "gbs": gbs, "bound": "hbm", "frac": gbs / hbm,
+                                      "l2_resident": 2 * pts * 4 < 126e6}
+        del b
+    d = E.desc_builtin("ccsd_t_d1", (48,))
+    b = bufs_for(d)
+    row = {}
+    simt_tiles, _ = E.select_tiles(d, gpu, split_pct=50, waf=4, mode=1)
+    for eng, tiles, note in ((1, simt_tiles, "EATSS B200 mode, WAF 4 (the space is empty for WAF >= 8)"),
+                             (2, (1, 2, 1, 48, 2, 48, 48), "hand-set MMA-legal tile: reading T covers depth-3 nests only")):
+        d.set_exec(split_pct=50, engine=eng)
+        ms = timed_ms(d, tiles, b, 2)
+        gbs = d.bytes / (ms * 1e-3) / 1e9
+        row["tensor" if eng == 2 else "simt"] = {"tiles": list(tiles), "ms": ms, "tflops": d.flops / (ms * 1e-3) / 1e12,
+                                                 "gbs": gbs, "bound": "hbm", "frac": gbs / hbm, "tile_origin": note}
+    out["ccsd_t_d1 dims=48"] = row
+    del b
+    torch.cuda.empty_cache()
+    return out
+
+
 # ------------------------------------------------------------------ our arm
 def main():
     args = parse()
@@ -293,16 +365,25 @@ def main():
                "sustained_tflops": s2.tflops, "gflops_per_watt": s2.gflops_per_watt,
                "avg_watts": s2.avg_watts, "sm_mhz_median": s2.sm_mhz_median}
 
-    # e2e through the public API with host buffers (pinned), copies inside the timed region
+    configs = None
+    if not args.no_configs and rank == 0:
+        configs = other_configs(E, torch, gpu, stream, measured_peaks())
+
+    # e2e through the C ABI with HOST buffers (eatss_run_host): every step copies A, B, C host->device
+    # and C device->host inside the timed region; gemm row blocks pipeline the copies with the compute
     A_p = torch.from_numpy(A_h).pin_memory(); B_p = torch.from_numpy(B_h).pin_memory()
-    C_p = torch.from_numpy(C_h).pin_memory(); C_out = torch.empty_like(C_p).pin_memory()
-    A2 = torch.empty_like(A); B2 = torch.empty_like(B); C2 = torch.empty_like(C)
+    C_p = torch.from_numpy(C_h).pin_memory()
     Ke = args.e2e_steps
 
+    # one descriptor for the e2e loop: it owns the device copies eatss_run_host fills (allocated on
+    # the first call, outside the timed region); the model still selects the tile every step
+    d_e2e = E.desc_builtin("gemm", (N, N, N))
+    d_e2e.set_scalars(1.5, 1.2)
+
     def e2e_step():
-        A2.copy_(A_p, non_blocking=True); B2.copy_(B_p, non_blocking=True); C2.copy_(C_p, non_blocking=True)
-        arm.step(C2, A2, B2, stream)
-        C_out.copy_(C2, non_blocking=True)
+        tiles, _ = E.select_tiles(d_e2e, gpu, split_pct=50, waf=16, mode=arm.mode)
+        d_e2e.set_exec(split_pct=50, engine=arm.engine)
+        E.run_host(d_e2e, tiles, [C_p, A_p, B_p], E2E_ROW_BLOCKS, stream)
 
     for _ in range(2):
         e2e_step()
@@ -391,12 +472,15 @@ def main():
                                   "counter-granularity limited)")},
             "roofline": roof,
             "e2e": {"value": FLOPS * ws / (e2e_ms * 1e-3) / 1e12, "unit": "TFLOP/s",
-                    "h2d_bytes_per_step": int(3 * N * N * 4), "d2h_bytes_per_step": int(N * N * 4)},
+                    "h2d_bytes_per_step": int(3 * N * N * 4), "d2h_bytes_per_step": int(N * N * 4),
+                    "path": f"eatss_run_host (C ABI, pinned host buffers, {E2E_ROW_BLOCKS} pipelined row blocks)"},
             "gpu_launches": int(K * launches_per_step),
             "clocks": clocks,
         }
         if sec:
             out["secondary"] = sec
+        if configs:
+            out["configs"] = configs
         if not args.no_cpu_baseline:
             out["cpu_baseline"] = cpu_oracle_sample()
         print(json.dumps(out), flush=True)

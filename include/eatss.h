@@ -221,6 +221,21 @@ EATSS_API eatss_status eatss_run(const eatss_kernel_desc *d, const int64_t *tile
 /* Execute only nest `nest` (0-based) -- used by the multi-GPU 3mm path between nests. */
 EATSS_API eatss_status eatss_run_nest(const eatss_kernel_desc *d, int nest, const int64_t *tiles,
                             void *const *buffers, void *stream);
+/* Execute the program on HOST buffers (the end-to-end path: host->device copies, the run, and
+ * device->host copies of the outputs, all ordered on `stream`).  host_buffers: the
+ * eatss_desc_num_buffers(d) arrays in the documented order, caller-owned host memory (page-locked
+ * -- cudaHostAlloc / torch pin_memory -- for the copies to run asynchronously; pageable memory
+ * works but serialises).  Inputs are read and outputs written per builtin (gemm: C in/out, A, B
+ * in; 2mm: tmp out, D in/out; 3mm: E, F, G out; stencils: both arrays in/out; ccsd: t3 in/out).
+ * The library keeps device copies per descriptor (allocated on first use, freed with the
+ * descriptor).  row_blocks > 1 (gemm): the rows of C are processed in that many blocks of whole
+ * i-tiles (CTA-pair rows on the tensor engine), B copied first, then each block's A and C rows
+ * copied in, computed and copied out on separate streams, so copies in both directions overlap
+ * the compute; every element sees the same operation order as one eatss_run.  Asynchronous:
+ * the outputs are in host memory once `stream` has reached the end of the call (synchronize on
+ * it); host buffers must stay valid until then.  Errors as eatss_run. */
+EATSS_API eatss_status eatss_run_host(const eatss_kernel_desc *d, const int64_t *tiles, void *const *host_buffers,
+                                      int64_t row_blocks, void *stream);
 /* Indexing oracle: run the executor's exact point mapping of nest
  * `nest`, adding 1 to counts[point] (int32, row-major over the nest's loops) for every
  * iteration point executed.  Contraction nests and stencil sweeps only. */

@@ -180,6 +180,26 @@ def run(d: Desc, tiles: Sequence[int], buffers, stream=None) -> None:
     _check(_lib.eatss_run(d.handle, _i64s(tiles), _bufs(d, buffers), _stream(stream)), "run")
 
 
+def _host_ptr(x) -> int:
+    if isinstance(x, int):
+        return x
+    if hasattr(x, "data_ptr") and hasattr(x, "is_cuda"):
+        if x.is_cuda:
+            raise TypeError("run_host takes host buffers")
+        return int(x.data_ptr())
+    if hasattr(x, "ctypes"):  # numpy array
+        return int(x.ctypes.data)
+    raise TypeError(f"cannot take a host pointer of {type(x)}")
+
+
+def run_host(d: Desc, tiles: Sequence[int], host_buffers, row_blocks: int = 1, stream=None) -> None:
+    """eatss_run_host: host buffers in, outputs copied back; complete when `stream` reaches the end."""
+    if len(host_buffers) != d.num_buffers:
+        raise ValueError(f"{d.kind}: expected {d.num_buffers} buffers, got {len(host_buffers)}")
+    arr = (ctypes.c_void_p * len(host_buffers))(*[_host_ptr(b) for b in host_buffers])
+    _check(_lib.eatss_run_host(d.handle, _i64s(tiles), arr, int(row_blocks), _stream(stream)), "run_host")
+
+
 def run_nest(d: Desc, nest: int, tiles: Sequence[int], buffers, stream=None) -> None:
     _check(_lib.eatss_run_nest(d.handle, nest, _i64s(tiles), _bufs(d, buffers), _stream(stream)), "run_nest")
 

@@ -89,6 +89,7 @@ DECLS = [
     ("eatss_plan", I32, [P, ctypes.POINTER(I64), ctypes.POINTER(LaunchPlan), ctypes.c_int,
                          ctypes.POINTER(ctypes.c_int)]),
     ("eatss_run", I32, [P, ctypes.POINTER(I64), ctypes.POINTER(P), P]),
+    ("eatss_run_host", I32, [P, ctypes.POINTER(I64), ctypes.POINTER(P), I64, P]),
     ("eatss_run_nest", I32, [P, ctypes.c_int, ctypes.POINTER(I64), ctypes.POINTER(P), P]),
     ("eatss_coverage", I32, [P, ctypes.c_int, ctypes.POINTER(I64), P, P]),
     ("eatss_launches_per_run", I64, [P, ctypes.POINTER(I64)]),

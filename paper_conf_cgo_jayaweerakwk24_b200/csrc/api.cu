@@ -290,6 +290,10 @@ using namespace eatss;
 eatss_kernel_desc::~eatss_kernel_desc() {
     for (auto &kv : graphs) cudaGraphExecDestroy((cudaGraphExec_t)kv.second);
     for (void *e : kev) cudaEventDestroy((cudaEvent_t)e);
+    for (void *b : hbuf) cudaFree(b);
+    for (void *e : hev) cudaEventDestroy((cudaEvent_t)e);
+    for (void *st : hstream)
+        if (st) cudaStreamDestroy((cudaStream_t)st);
 }
 
 // exec.time_kernels: a {start, stop} event pair per nest on the current device (nullptr if off)
@@ -585,6 +589,159 @@ eatss_status eatss_run_nest(const eatss_kernel_desc *d, int nest, const int64_t 
                             void *stream) {
     if (!d || nest < 0 || nest >= (int)d->nests.size()) return fail(EATSS_E_INVALID, "eatss_run_nest: bad nest");
     return run_impl(d, nest, tiles, buffers, stream);
+}
+
+// ------------------------------------------------------------------ host-buffer execution
+// Which buffers a builtin reads (copied host->device) and writes (copied device->host).
+static void buffer_io(const eatss_kernel_desc *d, int i, bool *in, bool *out) {
+    *in = true;
+    *out = false;
+    switch (d->kind) {
+        case EATSS_GEMM: case EATSS_SYRK: case EATSS_CCSD_T_D1: *out = i == 0; break;
+        case EATSS_2MM: *in = i != 0; *out = i == 0 || i == 4; break;
+        case EATSS_3MM: *in = !(i == 0 || i == 3 || i == 6); *out = !*in; break;
+        case EATSS_JACOBI2D: case EATSS_HEAT3D: *out = true; break;
+    }
+}
+
+eatss_status eatss_run_host(const eatss_kernel_desc *cd, const int64_t *tiles, void *const *host_buffers,
+                            int64_t row_blocks, void *stream) {
+    auto *d = const_cast<eatss_kernel_desc *>(cd);
+    if (!d || !host_buffers) return fail(EATSS_E_INVALID, "eatss_run_host: null argument");
+    for (int i = 0; i < d->num_buffers; i++)
+        if (!host_buffers[i]) return fail(EATSS_E_INVALID, "eatss_run_host: null host buffer");
+    eatss_status st = check_tiles(d, tiles);
+    if (st != EATSS_OK) return st;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0)
+        return fail(EATSS_E_CUDA, "eatss_run_host: no CUDA device (there is no CPU fallback)");
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaError_t e = cudaSuccess;
+    // library-owned device buffers, streams and events (per descriptor, re-created on a device change)
+    if (d->hdev != dev) {
+        for (void *b : d->hbuf) cudaFree(b);
+        for (void *ev : d->hev) cudaEventDestroy((cudaEvent_t)ev);
+        for (void *&hs : d->hstream)
+            if (hs) { cudaStreamDestroy((cudaStream_t)hs); hs = nullptr; }
+        d->hbuf.assign(d->num_buffers, nullptr);
+        d->hbuf_bytes.assign(d->num_buffers, 0);
+        d->hev.clear();
+        d->hdev = dev;
+    }
+    const size_t esz = (size_t)dtype_bytes(d->dtype);
+    for (int i = 0; i < d->num_buffers; i++) {
+        const size_t bytes = (size_t)d->buffer_elems[i] * esz;
+        if (d->hbuf_bytes[i] < bytes) {
+            if (d->hbuf[i]) cudaFree(d->hbuf[i]);
+            d->hbuf[i] = nullptr;
+            if ((e = cudaMalloc(&d->hbuf[i], bytes)) != cudaSuccess) {
+                d->hbuf_bytes[i] = 0;
+                return cuda_fail(e, "eatss_run_host: device buffer");
+            }
+            d->hbuf_bytes[i] = bytes;
+        }
+    }
+    for (void *&hs : d->hstream)
+        if (!hs) {
+            cudaStream_t t;
+            if ((e = cudaStreamCreateWithFlags(&t, cudaStreamNonBlocking)) != cudaSuccess)
+                return cuda_fail(e, "eatss_run_host: stream");
+            hs = t;
+        }
+    cudaStream_t sin = (cudaStream_t)d->hstream[0], sout = (cudaStream_t)d->hstream[1];
+    auto event = [&](size_t k) -> cudaEvent_t {
+        while (d->hev.size() <= k) {
+            cudaEvent_t ev;
+            if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess) return nullptr;
+            d->hev.push_back(ev);
+        }
+        return (cudaEvent_t)d->hev[k];
+    };
+    // event slots: 0 = start, 1 = end, 2.. = pipeline
+    // previous work on s (an earlier call's kernels may still read the device copies) before copies
+    cudaEvent_t e0 = event(0);
+    if (!e0) return fail(EATSS_E_CUDA, "eatss_run_host: event");
+    cudaEventRecord(e0, s);
+    cudaStreamWaitEvent(sin, e0, 0);
+    cudaStreamWaitEvent(sout, e0, 0);
+    void *dev_bufs[EATSS_MAX_BUFFERS];
+    for (int i = 0; i < d->num_buffers; i++) dev_bufs[i] = d->hbuf[i];
+    const bool f64 = d->dtype == EATSS_F64;
+    // gemm: row blocks of whole i-tiles pipelined -- B first, then per block A_r, C_r host->device,
+    // the block's gemm, and C_r device->host, the three on separate streams so copies in both
+    // directions overlap the compute (each block sees the single-launch operation order: its
+    // tiles are whole i-tiles of the full problem)
+    if (d->kind == EATSS_GEMM && row_blocks > 1) {
+        auto cn = contraction_nests(d, dev_bufs);
+        ContractNest full = cn[0];
+        const int64_t M = full.M, Ti = std::max<int64_t>(1, std::min(tiles[0], M));
+        const int64_t unit = d->exec.engine == EATSS_ENGINE_TENSOR ? std::max<int64_t>(Ti, 256) : Ti;
+        int64_t rb = (M + row_blocks - 1) / row_blocks;
+        rb = (rb + unit - 1) / unit * unit;
+        const int nblk = (int)((M + rb - 1) / rb);
+        const size_t rowA = (size_t)full.lda * esz, rowC = (size_t)full.ldc * esz;
+        char *hA = (char *)host_buffers[1], *hB = (char *)host_buffers[2], *hC = (char *)host_buffers[0];
+        char *dA = (char *)dev_bufs[1], *dC = (char *)dev_bufs[0];
+        cudaMemcpyAsync(dev_bufs[2], hB, d->hbuf_bytes[2], cudaMemcpyHostToDevice, sin);
+        const int sl = smem_limit_bytes();
+        for (int r = 0; r < nblk; r++) {
+            const int64_t r0 = (int64_t)r * rb, rows = std::min(rb, M - r0);
+            cudaMemcpyAsync(dA + r0 * rowA, hA + r0 * rowA, rows * rowA, cudaMemcpyHostToDevice, sin);
+            cudaMemcpyAsync(dC + r0 * rowC, hC + r0 * rowC, rows * rowC, cudaMemcpyHostToDevice, sin);
+            cudaEvent_t ein = event(2 + 2 * r), ecomp = event(3 + 2 * r);
+            if (!ein || !ecomp) return fail(EATSS_E_CUDA, "eatss_run_host: event");
+            cudaEventRecord(ein, sin);
+            cudaStreamWaitEvent(s, ein, 0);
+            ContractNest blk = full;
+            blk.M = rows;
+            blk.A = dA + r0 * rowA;
+            blk.C = dC + r0 * rowC;
+            ContractPlan p = plan_contraction(blk, tiles, sl);
+            const bool want_tc = d->exec.engine == EATSS_ENGINE_TENSOR;
+            int tsm = 0, tcols = 0;
+            const bool tcm = want_tc && tcm_applicable(blk, p);
+            const bool tc = want_tc && !tcm && tc_plan(blk, p, &tsm, &tcols);
+            if (want_tc && !tc && !tcm)
+                return fail(EATSS_E_UNSUPPORTED, "eatss_run_host: tensor engine not applicable to this tile");
+            e = tcm  ? launch_tcm_contraction(blk, p, s, nullptr)
+                : tc ? launch_tc_contraction(blk, p, d->exec.split_pct, s)
+                     : launch_contraction(blk, p, d->exec.split_pct, nullptr, s);
+            if (e != cudaSuccess) return cuda_fail(e, "eatss_run_host(gemm block)");
+            cudaEventRecord(ecomp, s);
+            cudaStreamWaitEvent(sout, ecomp, 0);
+            cudaMemcpyAsync(hC + r0 * rowC, dC + r0 * rowC, rows * rowC, cudaMemcpyDeviceToHost, sout);
+        }
+        (void)f64;
+    } else {
+        for (int i = 0; i < d->num_buffers; i++) {
+            bool in, out;
+            buffer_io(d, i, &in, &out);
+            if (in) cudaMemcpyAsync(dev_bufs[i], host_buffers[i], d->hbuf_bytes[i], cudaMemcpyHostToDevice, sin);
+        }
+        cudaEvent_t ein = event(2);
+        if (!ein) return fail(EATSS_E_CUDA, "eatss_run_host: event");
+        cudaEventRecord(ein, sin);
+        cudaStreamWaitEvent(s, ein, 0);
+        st = run_impl(d, -1, tiles, dev_bufs, s);
+        if (st != EATSS_OK) return st;
+        cudaEvent_t ecomp = event(3);
+        cudaEventRecord(ecomp, s);
+        cudaStreamWaitEvent(sout, ecomp, 0);
+        for (int i = 0; i < d->num_buffers; i++) {
+            bool in, out;
+            buffer_io(d, i, &in, &out);
+            if (out) cudaMemcpyAsync(host_buffers[i], dev_bufs[i], d->hbuf_bytes[i], cudaMemcpyDeviceToHost, sout);
+        }
+    }
+    // the call is complete on `stream` once the device->host copies are
+    cudaEvent_t eend = event(1);
+    if (!eend) return fail(EATSS_E_CUDA, "eatss_run_host: event");
+    cudaEventRecord(eend, sout);
+    cudaStreamWaitEvent(s, eend, 0);
+    e = cudaGetLastError();
+    return e == cudaSuccess ? EATSS_OK : cuda_fail(e, "eatss_run_host");
 }
 
 eatss_status eatss_coverage(const eatss_kernel_desc *d, int nest, const int64_t *tiles, int32_t *counts,

@@ -1,31 +1,39 @@
 // ccsd_tc.cu -- the 6-D CCSD(T) d1 contraction (BASELINE config 5) on
-// the tensor pipe (tcgen05 3xTF32), streaming t3 through TMA:
+// the tensor pipe (tcgen05 3xTF32):
 //
 //   t3[h3][h2][h1][p6][p5][p4] -= sum_h7 t2[h7][p4][p5][h1] * v2[h3][h2][p6][h7]
 //
 // The update has AI = 12 flop/B (t3 is read and written once, K = H7 = 48), so on B200 it is
 // HBM-bound once the arithmetic leaves the FFMA pipe: this executor makes the t3 stream the only
-// thing the SMs wait for.  Tile vector (Th3, Th2, Th1, Tp6, Tp5, Tp4, Th7) with Th3 = Th2 = 1,
+// thing the SMs wait for.  Tile vector (Th3, Th2, Th1, Tp6, Tp5, Tp4, Th7) with Th3 = 1,
 // Th7 = H7 (whole reduction per tile), M = Th1*Tp5*Tp4 <= 128 output rows on the MMA M axis and
-// N = Tp6 (multiple of 16, <= 256) on the MMA N axis:
-//   D[(h1,p5,p4)][p6] = sum_h7 t2[h7][p4][p5][h1] * v2[h3][h2][p6][h7]   (UMMA M=128, A in TMEM)
-//   X = t3 tile [h1][p6][p5][p4] (TMA 5-D box) ;  X -= D^T  (epilogue) ;  TMA store X.
-// The A operand depends on (h1,p5,p4) only: the epilogue warps write its tf32 hi/lo halves into
+// N = Th2*Tp6 (multiple of 16, <= 256; Th2 > 1 needs Tp6 = P6) on the MMA N axis:
+//   D[(h1,p5,p4)][(h2,p6)] = sum_h7 t2[h7][p4][p5][h1] * v2[h3][h2][p6][h7]   (UMMA M=128, A in TMEM)
+//   t3[h3][h2][h1][p6][p5][p4] -= D   (epilogue, read-modify-write of t3 in global memory)
+// The A operand depends on (h1,p5,p4) only: an epilogue group writes its tf32 hi/lo halves into
 // TMEM once per A tile (lane = output row, 16 columns per 8-k step) and the CTA then walks every
-// (h3,h2) unit that reuses it, so the MMAs read only the small v2 tile from shared memory (the
-// shared-memory port, not HBM, was the bound while A came from shared memory too).
+// (h3,h2) unit that reuses it, so the MMAs read only the small v2 tile from shared memory.
 // 3xTF32 with the raw-hi split (tc_mma.cu): hi = the operand itself (the tensor core truncates to
 // tf32), lo = rna_tf32(x - rz_tf32(x)); v2's lo half is materialised once per call (21 MB).
 //
-// Warp roles (persistent, one CTA per SM): warp 0 streams t3 tiles from HBM into an SX-stage ring
-// (evict-first L2 policy); warp 3 loads the per-unit v2 tile into an SV-stage ring; warp 1 issues
-// the MMAs; warp 2 owns TMEM and issues the t3-tile TMA stores; warps 4..11 are the epilogue
-// (lane = output row m; t3 tile RMW in shared memory; ring slot released two stores later).
+// Warp roles (persistent, one CTA per SM): warp 0 loads the per-unit v2 tile (hi, lo) into an
+// SV-stage ring by TMA; warp 1 issues the MMAs into NB TMEM accumulators; warp 2 owns TMEM; warps
+// 4.. are NGRP epilogue groups of four warps, each taking every NGRP-th unit.  A group brings its
+// unit's t3 tile into XB group-private shared buffers by TMA (XB = 2: the next owned unit's tile
+// is requested before the current one is processed), subtracts the TMEM accumulator and writes
+// the result straight to global memory (lane = output row m: a warp's 32 rows are contiguous t3
+// elements, one coalesced streaming store per column).
+// Measured history at dims 48: a single TMA ring + a separate store-issuer role
+// ran at 3.6 TB/s, bounded by per-unit hand-offs between four single-thread roles, not by HBM;
+// keeping shared pointers in the shared window (no generic accesses), blocking Th2 = 2 h2 per unit
+// (MMA N = 96: half the MMA instructions per byte -- the tensor pipe's per-instruction cost, not
+// its FLOP rate, bounded the N = 48 MMAs) and the group-private tiles bring it to 4.7 TB/s.
 #include <cuda.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
 #include <cstdint>
+#include <cstdio>
 #include <cstdlib>
 #include <mutex>
 
@@ -50,17 +58,18 @@ struct Args {
     int hh0, nhh;     // range of (h3, h2-tile) blocks of this launch (Th2 = 1: flattened (h3, h2))
     int64_t units;    // n_a * nhh * n_p6t
     int nkb;          // ceil(H7 / 32)
-    int SV, SX;       // V ring stages, t3-tile ring stages
+    int SV;           // V ring stages
     int bstride, NB;  // TMEM accumulator buffers (columns per buffer, count)
     int nks;          // 8-k MMA steps: ceil(H7 / 8)
     int a_col;        // TMEM column of A (hi at a_col + 16 ks, lo at + 8)
     int v_kb_bytes;   // NV * 128
     int v_stage;      // 2 * nkb * v_kb_bytes
-    int x_bytes;      // Th2*Th1*Tp6*Tp5*Tp4*4
-    int pend;         // t3 stores kept in flight before their ring slot is released
+    int x_bytes;      // t3 tile of a unit: Th2*Th1*Tp6*Tp5*Tp4*4
     int x_stage;      // x_bytes rounded up to 1 KB
+    int XB;           // t3 tile buffers per epilogue group (2: the next owned unit is prefetched)
     int order;        // 1: A tiles round-robin over CTAs (concurrent CTAs sweep whole t3 blocks)
     int dbg;          // development only (EATSS_CCSD_TC_DBG): 1 no MMA, 2 no t3 traffic, 4 no v2 loads
+    unsigned long long *prof;  // development only (EATSS_CCSD_TC_PROF): cycles per wait site
 };
 
 struct Unit {
@@ -196,23 +205,34 @@ struct Ring {
     }
 };
 
-// warps: 0 t3-tile producer, 1 MMA issuer, 2 TMEM owner + t3-tile store issuer, 3 A/V producer,
-// 4..11 epilogue (two groups of four: TMEM lane quarter = warp % 4, column half = group)
+// development instrumentation: cycles a role's lane 0 spends in each wait site (p.prof != nullptr)
+#define TWAIT(site, bar, par)                                                   \
+    do {                                                                        \
+        if (p.prof) {                                                           \
+            const long long t0_ = clock64();                                    \
+            mbar_wait_sleep(bar, par);                                          \
+            if (lane == 0) atomicAdd(p.prof + (site), (unsigned long long)(clock64() - t0_)); \
+        } else {                                                                \
+            mbar_wait_sleep(bar, par);                                          \
+        }                                                                       \
+    } while (0)
+
+// warps: 0 v2-tile producer (TMA), 1 MMA issuer, 2 TMEM owner, 3 idle, 4..4+NEPI-1 epilogue
+// (NGRP groups of four warps; warp % 4 = TMEM lane quarter; group g takes units u % NGRP == g)
+template <int SP6>  // compile-time t3 column (p6) stride P5*P4 in elements, 0 = runtime
 __global__ void __launch_bounds__(NTHREADS, 1)
-    ccsd_tc_kernel(const float *__restrict__ t2, const __grid_constant__ CUtensorMap mV,
+    ccsd_tc_kernel(const float *__restrict__ t2, float *__restrict__ t3, const __grid_constant__ CUtensorMap mV,
                    const __grid_constant__ CUtensorMap mVlo, const __grid_constant__ CUtensorMap mX, const Args p) {
     extern __shared__ __align__(1024) unsigned char smem_raw[];
     // align by pointer arithmetic on the shared array (an integer round trip would make every
     // access through `smem` a generic-address access)
     unsigned char *smem = smem_raw + ((1024u - (su32(smem_raw) & 1023u)) & 1023u);
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    // layout: V ring [SV] {hi [nkb], lo [nkb]}, X ring [SX], barriers
+    // layout: V ring [SV] {hi [nkb], lo [nkb]}, t3 tiles [NGRP][XB], barriers
     unsigned char *vring = smem;
     unsigned char *xring = vring + (size_t)p.SV * p.v_stage;
-    uint64_t *xfull = reinterpret_cast<uint64_t *>(xring + (size_t)p.SX * p.x_stage);
-    uint64_t *xempty = xfull + p.SX;
-    uint64_t *xdone = xempty + p.SX;
-    uint64_t *vfull = xdone + p.SX;
+    uint64_t *xbar = reinterpret_cast<uint64_t *>(xring + (size_t)NGRP * p.XB * p.x_stage);  // [NGRP][2]
+    uint64_t *vfull = xbar + 2 * NGRP;
     uint64_t *vempty = vfull + p.SV;
     uint64_t *dfull = vempty + p.SV;
     uint64_t *dempty = dfull + 4;
@@ -222,11 +242,6 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     const Sched sc = sched_of(p, (int)blockIdx.x, (int)gridDim.x);
 
     if (tid == 0) {
-        for (int s = 0; s < p.SX; s++) {
-            mbar_init(xfull + s, 1);
-            mbar_init(xempty + s, 1);
-            mbar_init(xdone + s, 4);
-        }
         for (int s = 0; s < p.SV; s++) {
             mbar_init(vfull + s, 1);
             mbar_init(vempty + s, 1);
@@ -235,9 +250,12 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             mbar_init(dfull + b, 1);
             mbar_init(dempty + b, 4);
         }
+        for (int b = 0; b < 2 * NGRP; b++) mbar_init(xbar + b, 1);
         mbar_init(afull, 4);  // the owning epilogue group writes A into TMEM
         mbar_init(aempty, 1);
         asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+        asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&mV)) : "memory");
+        asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&mVlo)) : "memory");
         asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&mX)) : "memory");
     }
     if (warp == 2) {
@@ -252,27 +270,11 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     const uint32_t tmem = *tmem_slot;
 
     if (warp == 0) {
-        if (lane == 0) {  // ------------------------------------ t3-tile producer (HBM stream)
-            const uint64_t pol = policy_evict_first();  // t3 is touched once: keep T2P / v2 in L2
-            UnitIter w = iter_begin(p, sc);
-            Ring r;
-            for (int64_t u = 0; u < sc.n; u++, iter_next(p, sc, w), r.next(p.SX)) {
-                int h1_0, p5_0, p4_0;
-                a_coords(p, w.a, h1_0, p5_0, p4_0);
-                if (u >= p.SX) mbar_wait(xempty + r.s, r.ph ^ 1u);
-                if (p.dbg & 2) { mbar_arrive(xfull + r.s); continue; }
-                mbar_expect_tx(xfull + r.s, p.x_bytes);
-                int c[5];
-                x_coords(p, w.hh, w.p6t, h1_0, p5_0, p4_0, c);
-                tma_5d_hint(xring + (size_t)r.s * p.x_stage, &mX, c[0], c[1], c[2], c[3], c[4], xfull + r.s, pol);
-            }
-        }
-    } else if (warp == 3) {
         if (lane == 0) {  // ------------------------------------ v2 tile producer (L2-resident)
             UnitIter w = iter_begin(p, sc);
             Ring r;
             for (int64_t u = 0; u < sc.n; u++, iter_next(p, sc, w), r.next(p.SV)) {
-                if (u >= p.SV) mbar_wait(vempty + r.s, r.ph ^ 1u);
+                if (u >= p.SV) TWAIT(0, vempty + r.s, r.ph ^ 1u);
                 unsigned char *st = vring + (size_t)r.s * p.v_stage;
                 if (p.dbg & 4) { mbar_arrive(vfull + r.s); continue; }
                 mbar_expect_tx(vfull + r.s, p.v_stage);
@@ -286,94 +288,92 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     } else if (warp == 1) {
         if (lane == 0) {  // ------------------------------------------------ MMA issuer
             const uint32_t ID = idesc(p.NV, 1, true);  // M = 128, N = NV = Th2 * Tp6, A and B K-major
+            const long long tmma = p.prof ? clock64() : 0;
             int a_prev = -1, na = 0;
             UnitIter w = iter_begin(p, sc);
             Ring rv, rd;
             for (int64_t u = 0; u < sc.n; u++, iter_next(p, sc, w), rv.next(p.SV), rd.next(p.NB)) {
                 if (w.a != a_prev) {
                     if (na > 0) mma_commit<1>(aempty);  // fires when every MMA on the old A is done
-                    mbar_wait(afull, (unsigned)(na & 1));
+                    mbar_wait_sleep(afull, (unsigned)(na & 1));
                     a_prev = w.a;
                     na++;
                 }
-                if (u >= p.NB) mbar_wait(dempty + rd.s, rd.ph ^ 1u);
-                mbar_wait(vfull + rv.s, rv.ph);
+                if (u >= p.NB) TWAIT(1, dempty + rd.s, rd.ph ^ 1u);
+                TWAIT(2, vfull + rv.s, rv.ph);
                 fence_after();
                 unsigned char *st = vring + (size_t)rv.s * p.v_stage;
                 const uint32_t d = tmem + (uint32_t)(rd.s * p.bstride);
+                const uint64_t vh0 = desc_sw128(st, 16u, 1024u), vl0 = desc_sw128(st + p.nkb * p.v_kb_bytes, 16u, 1024u);
                 bool first = true;
                 for (int k8 = 0; k8 < (p.dbg & 1 ? 0 : p.nks); k8++) {
-                    const int kb = k8 >> 2, ks = k8 & 3;
+                    // descriptor start address advances by (kb * v_kb_bytes + ks * 32) >> 4
+                    const uint64_t off = (uint64_t)(((k8 >> 2) * p.v_kb_bytes + (k8 & 3) * 32) >> 4);
                     const uint32_t ah = tmem + (uint32_t)(p.a_col + 16 * k8), al = ah + 8;
-                    const uint64_t vh = desc_sw128(st + kb * p.v_kb_bytes + ks * 32, 16u, 1024u);
-                    const uint64_t vl = desc_sw128(st + (p.nkb + kb) * p.v_kb_bytes + ks * 32, 16u, 1024u);
-                    mma_ts(d, ah, vh, ID, first ? 0u : 1u);
-                    mma_ts(d, ah, vl, ID, 1u);
-                    mma_ts(d, al, vh, ID, 1u);
+                    mma_ts(d, ah, vh0 + off, ID, first ? 0u : 1u);
+                    mma_ts(d, ah, vl0 + off, ID, 1u);
+                    mma_ts(d, al, vh0 + off, ID, 1u);
                     first = false;
                 }
                 mma_commit<1>(dfull + rd.s);
                 mma_commit<1>(vempty + rv.s);
             }
-        }
-    } else if (warp == 2) {
-        if (lane == 0) {  // ------------------------------------ t3-tile store issuer
-            const uint64_t pol = policy_evict_first();
-            UnitIter w = iter_begin(p, sc);
-            Ring r;
-            int pend[3] = {-1, -1, -1};  // stages of the last p.pend stores, oldest first
-            for (int64_t u = 0; u < sc.n; u++, iter_next(p, sc, w), r.next(p.SX)) {
-                int h1_0, p5_0, p4_0;
-                a_coords(p, w.a, h1_0, p5_0, p4_0);
-                mbar_wait(xdone + r.s, r.ph);
-                if (p.dbg & 2) { mbar_arrive(xempty + r.s); continue; }
-                int c[5];
-                x_coords(p, w.hh, w.p6t, h1_0, p5_0, p4_0, c);
-                tma_store_5d_hint(&mX, xring + (size_t)r.s * p.x_stage, c[0], c[1], c[2], c[3], c[4], pol);
-                bulk_commit();
-                if (p.pend == 2) {
-                    bulk_wait_read<2>();  // all but the 2 newest stores have read their slots
-                    if (pend[0] >= 0) mbar_arrive(xempty + pend[0]);
-                    pend[0] = pend[1];
-                    pend[1] = r.s;
-                } else {
-                    bulk_wait_read<1>();
-                    if (pend[0] >= 0) mbar_arrive(xempty + pend[0]);
-                    pend[0] = r.s;
-                }
-            }
-            bulk_wait_all();
+            if (p.prof) atomicAdd(p.prof + 6, (unsigned long long)(clock64() - tmma));
         }
     } else if (warp >= 4) {  // ------------------------------------------------ epilogue
-        // group g = (warp - 4) / 4 takes every NGRP-th unit, so NGRP units are in their epilogue
-        // at once (the per-unit chain -- wait, TMEM load, shared RMW, release -- is latency-bound)
+        // Group g owns the units u = g, g + NGRP, ...  Its t3 tiles come from HBM by TMA into XB
+        // group-private shared buffers, the next owned unit's tile being requested before the
+        // current one is processed, so the HBM latency is hidden behind a whole unit; the updated
+        // values go straight back to global memory (row m = (h1l, p5l, p4l): with Tp4 = P4 a warp's
+        // 32 rows are 128 contiguous bytes, one coalesced streaming store per column).
         const int q = warp & 3, g = (warp - 4) >> 2, m = q * 32 + lane;
         const int Mrows = p.Th1 * p.Tp5 * p.Tp4;
         const int p4l = m % p.Tp4, p5l = (m / p.Tp4) % p.Tp5, h1l = m / (p.Tp4 * p.Tp5);
         const bool live = m < Mrows;
-        const int xrow0 = (h1l * p.Tp6 * p.Tp5 + p5l) * p.Tp4 + p4l, xstep = p.Tp5 * p.Tp4;  // + p6 * xstep
         const uint32_t trow = tmem + ((uint32_t)(q * 32) << 16);
-        UnitIter w = iter_begin(p, sc);
-        int a_prev = -1, na = 0, own = g;  // own: units until this group's next unit
-        Ring rx, rd;
-        for (int64_t u = 0; u < sc.n; u++, iter_next(p, sc, w), rx.next(p.SX), rd.next(p.NB), own--) {
+        const int sp6 = SP6 > 0 ? SP6 : p.P5 * p.P4;
+        const int64_t s_h1 = (int64_t)p.P6 * sp6, s_hh = p.H1 * s_h1;
+        const int xstep = p.Tp5 * p.Tp4;                                 // smem column (p6) stride
+        const int xrow0 = h1l * p.Tp6 * xstep + p5l * p.Tp4 + p4l;       // smem offset of row m
+        const int xh2 = p.Th1 * p.Tp6 * xstep;                           // smem stride of h2l
+        unsigned char *xbuf = xring + (size_t)g * p.XB * p.x_stage;
+        uint64_t *xb = xbar + 2 * g;
+        const bool leader = q == 0 && lane == 0;
+        const uint64_t pol = policy_evict_first();  // t3 is touched once: keep v2 / t2 in L2
+        auto fetch = [&](const UnitIter &wn, int buf) {  // t3 tile of unit wn -> xbuf[buf]
+            int h1_0, p5_0, p4_0, c[5];
+            a_coords(p, wn.a, h1_0, p5_0, p4_0);
+            x_coords(p, wn.hh, wn.p6t, h1_0, p5_0, p4_0, c);
+            mbar_expect_tx(xb + buf, p.x_bytes);
+            tma_5d_hint(xbuf + (size_t)buf * p.x_stage, &mX, c[0], c[1], c[2], c[3], c[4], xb + buf, pol);
+        };
+        UnitIter w = iter_begin(p, sc), wn = w;  // wn: this group's next unit to prefetch
+        for (int i = 0; i < g && i < sc.n; i++) iter_next(p, sc, wn);
+        int64_t un = g;  // unit index of wn
+        int a_prev = -1, na = 0, own = g, k = 0;  // own: units until this group's next unit; k: owned count
+        bool rin = false;
+        int64_t rowoff = 0;  // t3 offset of row m for hh = 0, p6 = 0
+        if (p.XB == 2 && leader && !(p.dbg & 2) && un < sc.n) fetch(wn, 0);  // XB = 1 fetches at unit start
+        Ring rd;
+        for (int64_t u = 0; u < sc.n; u++, iter_next(p, sc, w), rd.next(p.NB), own--) {
             const bool mine = own == 0;
             if (mine) own = NGRP;
-            if (w.a != a_prev) {  // new A tile: the group owning this unit writes row m of t2 into TMEM
+            if (w.a != a_prev) {  // new A tile: row coordinates; the owning group writes A into TMEM
+                int h1_0, p5_0, p4_0;
+                a_coords(p, w.a, h1_0, p5_0, p4_0);
+                const int h1 = h1_0 + h1l, p5 = p5_0 + p5l, p4 = p4_0 + p4l;
+                rin = live && h1 < p.H1 && p5 < p.P5 && p4 < p.P4;
+                rowoff = (int64_t)h1 * s_h1 + (int64_t)p5 * p.P4 + p4;
                 if (mine) {
-                    int h1_0, p5_0, p4_0;
-                    a_coords(p, w.a, h1_0, p5_0, p4_0);
-                    const int h1 = h1_0 + h1l, p5 = p5_0 + p5l, p4 = p4_0 + p4l;
-                    const bool in = live && h1 < p.H1 && p5 < p.P5 && p4 < p.P4;
                     const float *src = t2 + (((int64_t)p4 * p.P5 + p5) * p.H1 + h1);
                     const int64_t hstride = (int64_t)p.P4 * p.P5 * p.H1;
-                    if (na > 0) mbar_wait(aempty, (unsigned)((na - 1) & 1));  // MMAs on the old A are done
+                    if (na > 0) mbar_wait_sleep(aempty, (unsigned)((na - 1) & 1));  // MMAs on the old A are done
                     for (int k8 = 0; k8 < p.nks; k8++) {
                         uint32_t hi[8], lo[8];
 #pragma unroll
                         for (int c = 0; c < 8; c++) {
                             const int h7 = 8 * k8 + c;
-                            const float x = (in && h7 < p.H7) ? __ldg(src + h7 * hstride) : 0.f;
+                            const float x = (rin && h7 < p.H7) ? __ldg(src + h7 * hstride) : 0.f;
                             hi[c] = __float_as_uint(x);
                             lo[c] = __float_as_uint(lo_of(x));
                         }
@@ -389,47 +389,66 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                 na++;
             }
             if (!mine) continue;
-            mbar_wait(xfull + rx.s, rx.ph);
-            mbar_wait(dfull + rd.s, rd.ph);
+            const int buf = p.XB == 2 ? (k & 1) : 0;
+            const unsigned xph = (unsigned)((p.XB == 2 ? (k >> 1) : k) & 1);
+            // next owned unit: its buffer was last read for unit k - 1 (XB = 2) -- the group barrier
+            // orders those reads before the TMA overwrites it; XB = 1 fetches the current unit here
+            for (int i = 0; i < NGRP && un < sc.n; i++, un++) iter_next(p, sc, wn);
+            named_bar(1 + g, 128);
+            if (p.XB == 2) {
+                if (leader && !(p.dbg & 2) && un < sc.n) fetch(wn, buf ^ 1);
+            } else if (leader && !(p.dbg & 2)) {
+                fetch(w, 0);
+            }
+            // columns of this unit: hh = hhb + h2l (h2l < nh valid), p6 = p6b + c6 (c6 < np6 valid)
+            int hhb, nh;
+            if (p.Th2 == 1) {
+                hhb = w.hh;
+                nh = 1;
+            } else {
+                const int h3 = w.hh / p.n_h2t, h2_0 = (w.hh - h3 * p.n_h2t) * p.Th2;
+                hhb = h3 * p.H2 + h2_0;
+                nh = min(p.Th2, p.H2 - h2_0);
+            }
+            const int p6b = w.p6t * p.Tp6, np6 = min(p.Tp6, p.P6 - p6b);
+            float *const rowp = t3 + rowoff + (int64_t)hhb * s_hh + (int64_t)p6b * sp6;
+            const float *xs = reinterpret_cast<const float *>(xbuf + (size_t)buf * p.x_stage) + xrow0;
+            const bool io = rin && !(p.dbg & 2);
+            if (!(p.dbg & 2)) TWAIT(7, xb + buf, xph);
+            if (p.prof && leader) atomicAdd(p.prof + 5, 1ull);
+            TWAIT(3, dfull + rd.s, rd.ph);
+            const long long tproc = p.prof ? clock64() : 0;
             fence_after();
-            float *xs = reinterpret_cast<float *>(xring + (size_t)rx.s * p.x_stage) + xrow0;
-            // columns n = (h2l, p6) in batches of up to four 8-column chunks (a chunk never straddles
-            // two h2, Tp6 % 16 == 0): all TMEM loads, then all shared loads, then the stores
-            for (int c0 = 0; c0 < p.NV; c0 += 32) {
-                uint32_t v[4][8];
-                const int nc = min(4, (p.NV - c0 + 7) / 8);
-                tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0), v[0]);
-                if (nc > 1) tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0 + 8), v[1]);
-                if (nc > 2) tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0 + 16), v[2]);
-                if (nc > 3) tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0 + 24), v[3]);
+            // chunks of 16 columns (Tp6 % 16 == 0: never two h2 in a chunk), walked without divisions
+            constexpr int CH = 16;
+            int h2l = 0, c6 = 0;
+            for (int c0 = 0; c0 < p.NV; c0 += CH) {
+                uint32_t v[CH];
+                tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0), *reinterpret_cast<uint32_t(*)[8]>(v));
+                tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0 + 8), *reinterpret_cast<uint32_t(*)[8]>(v + 8));
+                const float *xc = xs + h2l * xh2 + c6 * xstep;
+                float x[CH];  // rows m >= Th1*Tp5*Tp4 lie outside the tile (and possibly the window)
+#pragma unroll
+                for (int c = 0; c < CH; c++) x[c] = live ? xc[c * xstep] : 0.f;
                 wait_ld();
-                if (live) {
-                    int cb[4];  // shared offset of each chunk's first column
+                const int nok = (io && h2l < nh) ? min(CH, np6 - c6) : 0;
+                float *gp = rowp + (int64_t)h2l * s_hh + (int64_t)c6 * sp6;
+                if (nok == CH) {
 #pragma unroll
-                    for (int j = 0; j < 4; j++) {
-                        const int n = c0 + 8 * j, hl = n / p.Tp6;
-                        cb[j] = (hl * p.Th1 * p.Tp6 + (n - hl * p.Tp6)) * xstep;
-                    }
-                    float x[4][8];
+                    for (int c = 0; c < CH; c++) __stcs(gp + c * sp6, x[c] - __uint_as_float(v[c]));
+                } else {
 #pragma unroll
-                    for (int j = 0; j < 4; j++)
-#pragma unroll
-                        for (int c = 0; c < 8; c++)
-                            if (j < nc) x[j][c] = xs[cb[j] + c * xstep];
-#pragma unroll
-                    for (int j = 0; j < 4; j++)
-#pragma unroll
-                        for (int c = 0; c < 8; c++)
-                            if (j < nc) xs[cb[j] + c * xstep] = x[j][c] - __uint_as_float(v[j][c]);
+                    for (int c = 0; c < CH; c++)
+                        if (c < nok) __stcs(gp + c * sp6, x[c] - __uint_as_float(v[c]));
                 }
+                c6 += CH;
+                if (c6 == p.Tp6) { c6 = 0; h2l++; }
             }
             fence_before();
-            fence_proxy_async_smem();  // generic-proxy writes -> visible to the TMA store
             __syncwarp();
-            if (lane == 0) {
-                mbar_arrive(dempty + rd.s);
-                mbar_arrive(xdone + rx.s);
-            }
+            if (lane == 0) mbar_arrive(dempty + rd.s);
+            if (p.prof && leader) atomicAdd(p.prof + 4, (unsigned long long)(clock64() - tproc));
+            k++;
         }
     }
     fence_before();
@@ -499,7 +518,8 @@ CcsdTcPlan plan_ccsd_tc(const int64_t *dims, const int64_t *tiles) {
     for (int i = 0; i < 7; i++) T[i] = std::min(tiles[i], dims[i]);
     const int64_t H3 = dims[0], H2 = dims[1], H1 = dims[2], P6 = dims[3], P5 = dims[4], P4 = dims[5], H7 = dims[6];
     if (T[0] != 1 || T[6] < H7) return pl;  // one h3 per unit, whole h7 reduction
-    // Th2 > 1: Th2 consecutive h2 per unit (MMA N = Th2 * P6); needs whole p6 and p4 ranges
+    // Th2 > 1: Th2 consecutive h2 per unit (MMA N = Th2 * P6: their v2 rows are contiguous)
+    // and whole p4 (the t3 tile's TMA box flattens (p5, p4))
     if (T[1] > 1 && (T[3] != P6 || T[5] != P4 || T[1] * P6 > 256 || (T[1] * P6) % 16)) return pl;
     if (H7 > 64 || (H7 % 4) || (P4 % 4) || (T[5] % 4)) return pl;  // 16-byte TMA strides / boxes
     if (T[2] * T[4] * T[5] > ccsdtc::MROWS || (T[3] % 16) || T[3] > 256) return pl;
@@ -524,18 +544,14 @@ CcsdTcPlan plan_ccsd_tc(const int64_t *dims, const int64_t *tiles) {
     a.x_bytes = a.Th2 * a.Th1 * a.Tp6 * a.Tp5 * a.Tp4 * 4;
     a.x_stage = (a.x_bytes + 1023) / 1024 * 1024;
     const int fixed = 1024 /*align*/ + 512 /*barriers*/;
-    a.SV = 4;
-    const int avail = 232448 - fixed - a.SV * a.v_stage;
-    a.SX = std::min(8, avail / a.x_stage);
-    if (const char *e = getenv("EATSS_CCSD_TC_XSTAGES")) a.SX = std::max(3, std::min(a.SX, atoi(e)));
-    if (a.SX < 3) {  // big tiles: shallower operand ring
-        a.SV = 2;
-        a.SX = std::min(8, (232448 - fixed - a.SV * a.v_stage) / a.x_stage);
-    }
-    // SX >= 3: the store issuer releases a slot two stores after it was written
-    if (a.SX < 3) return pl;
-    a.pend = a.SX >= 4 ? 2 : 1;
-    pl.smem = fixed + a.SV * a.v_stage + a.SX * a.x_stage;
+    const int budget = 232448 - fixed;
+    a.XB = 2;
+    if (budget - ccsdtc::NGRP * a.XB * a.x_stage < 3 * a.v_stage) a.XB = 1;  // keep >= 3 v2 stages if possible
+    if (const char *e = getenv("EATSS_CCSD_TC_XB")) a.XB = std::max(1, std::min(2, atoi(e)));
+    a.SV = std::min(6, (budget - ccsdtc::NGRP * a.XB * a.x_stage) / a.v_stage);
+    if (const char *e = getenv("EATSS_CCSD_TC_VSTAGES")) a.SV = std::max(1, std::min(a.SV, atoi(e)));
+    if (a.SV < 2) return pl;
+    pl.smem = fixed + a.SV * a.v_stage + ccsdtc::NGRP * a.XB * a.x_stage;
     pl.ok = true;
     return pl;
 }
@@ -561,17 +577,17 @@ cudaError_t launch_ccsd_tc(float *t3, const float *t2, const float *v2, const in
     ccsdtc::prep_kernel<<<148 * 4, 256, 0, s>>>(v2, v2_lo, n_v2);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
-    CUtensorMap mV, mVlo, mX;
-    // V: v2 as [(h3,h2,p6)][h7], box {32, Tp6}, SWIZZLE_128B (K-major UMMA operand)
+    CUtensorMap mV, mVlo;
+    // V: v2 as [(h3,h2,p6)][h7], box {32, NV}, SWIZZLE_128B (K-major UMMA operand)
     const uint64_t vdims[2] = {(uint64_t)H7, (uint64_t)((int64_t)a.H3 * H2 * P6)};
     const uint64_t vstr[1] = {(uint64_t)H7 * 4};
     const uint32_t vbox[2] = {32, (uint32_t)a.NV};
-    // X: t3 as [(h3,h2)][h1][p6][p5][p4], box {Tp4, Tp5, Tp6, Th1, 1}
+    // X: t3 as [(h3,h2)][h1][p6][p5][p4], box {Tp4, Tp5, Tp6, Th1, 1}; Th2 > 1: ((p5,p4), p6, h1, h2, h3)
     uint64_t xdims[5] = {(uint64_t)P4, (uint64_t)P5, (uint64_t)P6, (uint64_t)H1, (uint64_t)((int64_t)a.H3 * H2)};
     uint64_t xstr[4] = {(uint64_t)P4 * 4, (uint64_t)(P5 * P4) * 4, (uint64_t)(P6 * P5 * P4) * 4,
                         (uint64_t)(H1 * P6 * P5 * P4) * 4};
     uint32_t xbox[5] = {(uint32_t)a.Tp4, (uint32_t)a.Tp5, (uint32_t)a.Tp6, (uint32_t)a.Th1, 1};
-    if (a.Th2 > 1) {  // dims ((p5,p4), p6, h1, h2, h3)
+    if (a.Th2 > 1) {
         const uint64_t d2[5] = {(uint64_t)(P5 * P4), (uint64_t)P6, (uint64_t)H1, (uint64_t)H2, (uint64_t)a.H3};
         const uint64_t s2[4] = {(uint64_t)(P5 * P4) * 4, (uint64_t)(P6 * P5 * P4) * 4, (uint64_t)(H1 * P6 * P5 * P4) * 4,
                                 (uint64_t)(H2 * H1 * P6 * P5 * P4) * 4};
@@ -579,6 +595,7 @@ cudaError_t launch_ccsd_tc(float *t3, const float *t2, const float *v2, const in
         for (int i = 0; i < 5; i++) { xdims[i] = d2[i]; xbox[i] = b2[i]; }
         for (int i = 0; i < 4; i++) xstr[i] = s2[i];
     }
+    CUtensorMap mX;
     if (!ccsdtc::make_map_nd(&mV, v2, 2, vdims, vstr, vbox, CU_TENSOR_MAP_SWIZZLE_128B) ||
         !ccsdtc::make_map_nd(&mVlo, v2_lo, 2, vdims, vstr, vbox, CU_TENSOR_MAP_SWIZZLE_128B) ||
         !ccsdtc::make_map_nd(&mX, t3, 5, xdims, xstr, xbox, CU_TENSOR_MAP_SWIZZLE_NONE))
@@ -588,7 +605,10 @@ cudaError_t launch_ccsd_tc(float *t3, const float *t2, const float *v2, const in
     {
         std::lock_guard<std::mutex> lk(mu);
         if (smem_set < pl.smem) {
-            e = cudaFuncSetAttribute(ccsdtc::ccsd_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, pl.smem);
+            e = cudaFuncSetAttribute(ccsdtc::ccsd_tc_kernel<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, pl.smem);
+            if (e == cudaSuccess)
+                e = cudaFuncSetAttribute(ccsdtc::ccsd_tc_kernel<48 * 48>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         pl.smem);
             if (e != cudaSuccess) return e;
             smem_set = pl.smem;
         }
@@ -597,9 +617,29 @@ cudaError_t launch_ccsd_tc(float *t3, const float *t2, const float *v2, const in
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     const int grid = (int)std::min<int64_t>(nsm, a.units);
+    static unsigned long long *prof = nullptr;
+    if (getenv("EATSS_CCSD_TC_PROF")) {
+        if (!prof) cudaMalloc(&prof, 16 * sizeof(unsigned long long));
+        cudaMemsetAsync(prof, 0, 16 * sizeof(unsigned long long), s);
+        a.prof = prof;
+    }
     if (ev) cudaEventRecord(ev[0], s);
-    ccsdtc::ccsd_tc_kernel<<<grid, ccsdtc::NTHREADS, pl.smem, s>>>(t2, mV, mVlo, mX, a);
+    if (a.P5 * a.P4 == 48 * 48)  // the BASELINE dims-48 stride: immediate-offset accesses
+        ccsdtc::ccsd_tc_kernel<48 * 48><<<grid, ccsdtc::NTHREADS, pl.smem, s>>>(t2, t3, mV, mVlo, mX, a);
+    else
+        ccsdtc::ccsd_tc_kernel<0><<<grid, ccsdtc::NTHREADS, pl.smem, s>>>(t2, t3, mV, mVlo, mX, a);
     e = cudaGetLastError();
+    if (a.prof) {  // development: per-site average cycles (per CTA role lane / per unit)
+        unsigned long long h[16];
+        cudaMemcpyAsync(h, prof, sizeof(h), cudaMemcpyDeviceToHost, s);
+        cudaStreamSynchronize(s);
+        const double units = (double)h[5];
+        fprintf(stderr,
+                "ccsd_tc prof: units %.0f | per unit: V wait vempty %.0f, MMA wait dempty %.0f, MMA wait vfull "
+                "%.0f, EPI wait dfull %.0f, EPI process %.0f, EPI wait t3 %.0f | MMA loop per CTA %.0f cyc (%d CTAs)\n",
+                units, h[0] / units, h[1] / units, h[2] / units, h[3] / units / 4, h[4] / units, h[7] / units / 4, h[6] / (double)grid,
+                grid);
+    }
     if (ev) cudaEventRecord(ev[1], s);
     return e;
 }

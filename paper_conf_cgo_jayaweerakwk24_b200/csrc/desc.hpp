@@ -68,6 +68,12 @@ struct eatss_kernel_desc {
     // exec.time_kernels: start/stop events per nest of the last timed run (cudaEvent_t as void*)
     std::vector<void *> kev;
     int kev_dev = -1, kev_valid = 0;
+    // eatss_run_host: library-owned device copies of the buffers, copy streams and events
+    std::vector<void *> hbuf;
+    std::vector<size_t> hbuf_bytes;
+    int hdev = -1;
+    void *hstream[2] = {nullptr, nullptr};  // host->device, device->host
+    std::vector<void *> hev;                // pipeline events
     ~eatss_kernel_desc();
 };
 

@@ -46,6 +46,16 @@ __device__ __forceinline__ void mbar_wait(uint64_t *b, unsigned parity) {
         "r"(parity)
         : "memory");
 }
+// Same wait, but the waiting thread is suspended (up to the hint, 10 ms) instead of spinning:
+// waiters then do not take issue slots from the warps that do the work on their SM sub-partition.
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t *b, unsigned parity) {
+    asm volatile(
+        "{\n.reg .pred p;\nW_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n"
+        "@!p bra W_%=;\n}\n" ::"r"(su32(b)),
+        "r"(parity), "r"(0x989680u)
+        : "memory");
+}
 __device__ __forceinline__ void mbar_wait_cluster(uint64_t *b, unsigned parity) {
     asm volatile(
         "{\n.reg .pred p;\nW_%=:\n"

@@ -1,10 +1,6 @@
 cd $GRAFT_REPO_ROOT
-mkdir -p gpurun_out
-timeout 900 python -m pytest tests/test_gpu_parity.py tests/test_gpu_tensor.py -q --timeout 600 -p no:cacheprovider -k "ccsd or syrk" 2>&1 | tail -3
 T=scripts/time_kernel.py
-timeout 120 python $T syrk 4000,4000 16,1024,16 --engine 1 --iters 10 2>&1 | tail -1
-timeout 120 python $T gemm 4000,4000,4000 16,1024,16 --engine 1 --iters 10 2>&1 | tail -1
-timeout 900 python scripts/ccsd_variants.py
-timeout 900 python harness/l2power.py --phase power --count 120 2>&1 | tail -2
-timeout 900 ncu --metrics lts__t_sectors_srcunit_tex_op_read.sum,lts__t_sectors_op_read.sum,gpu__time_duration.sum --clock-control none -k regex:'contract|jacobi2d' --csv --log-file gpurun_out/l2power_l2.csv python harness/l2power.py --phase l2 > /dev/null 2>&1; echo "ncu l2 $?"
-python harness/l2power.py --phase report 2>&1 | tail -30
+timeout 900 python -m pytest tests/test_gpu_tensor.py tests/test_gpu_host.py -q --timeout 600 -p no:cacheprovider -k "ccsd or host" 2>&1 | tail -3
+for t in 1,2,1,48,2,48,48; do echo "== $t"; EATSS_CCSD_TC_PROF=1 timeout 300 python $T ccsd_t_d1 48 $t --engine 2 --iters 1 2>&1 | tail -2; done
+for t in 1,2,1,48,2,48,48 1,1,1,48,2,48,48; do timeout 300 python $T ccsd_t_d1 48 $t --engine 2 --iters 5 2>&1 | tail -1; done
+for xb in 1; do EATSS_CCSD_TC_XB=$xb timeout 300 python $T ccsd_t_d1 48 1,1,1,48,2,48,48 --engine 2 --iters 5 2>&1 | tail -1; done
