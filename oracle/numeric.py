@@ -56,10 +56,15 @@ def _declare(L):
     L.oracle_heat3d.argtypes = [_I, _I, _P, _P]
     L.oracle_ccsd_t_d1.argtypes = [_P, _P, _P, _P]
     L.oracle_ccsd_t_d1_entries.argtypes = [_P, _I, _P, _P, _P, _P, _P]
+    L.oracle_mvt.argtypes = [_I, _P, _P, _P, _P, _P]
+    L.oracle_atax.argtypes = [_I, _I, _P, _P, _P, _P]
+    L.oracle_bicg.argtypes = [_I, _I, _P, _P, _P, _P, _P]
+    L.oracle_gemver.argtypes = [_I, _D, _D, _P, _P, _P, _P, _P, _P, _P, _P, _P]
     L.oracle_num_threads.restype = ctypes.c_int
     for f in ("oracle_gemm", "oracle_gemm_ijk", "oracle_gemm_entries", "oracle_2mm",
               "oracle_3mm", "oracle_syrk", "oracle_jacobi2d", "oracle_heat3d",
-              "oracle_ccsd_t_d1", "oracle_ccsd_t_d1_entries"):
+              "oracle_ccsd_t_d1", "oracle_ccsd_t_d1_entries", "oracle_mvt", "oracle_atax", "oracle_bicg",
+              "oracle_gemver"):
         getattr(L, f).restype = None
 
 
@@ -166,6 +171,41 @@ def ccsd_t_d1_entries(dims, idx, t3_0, t2, v2) -> np.ndarray:
     out = np.empty(len(idx), dtype=np.float64)
     lib().oracle_ccsd_t_d1_entries(_p(d), len(idx), _p(idx), _p(t3_0), _p(t2), _p(v2), _p(out))
     return out
+
+
+def mvt(x1, x2, y1, y2, A):
+    """PolyBench 3.2 mvt. Returns (x1, x2)."""
+    x1 = _f64(x1).copy(); x2 = _f64(x2).copy(); A = _f64(A)
+    n = x1.shape[0]
+    assert A.shape == (n, n)
+    lib().oracle_mvt(n, _p(x1), _p(x2), _p(_f64(y1)), _p(_f64(y2)), _p(A))
+    return x1, x2
+
+
+def atax(A, x):
+    """PolyBench 3.2 atax: tmp = A x, y = A^T tmp (fused loop order). Returns (y, tmp)."""
+    A = _f64(A); nx, ny = A.shape
+    y = np.zeros(ny); tmp = np.zeros(nx)
+    lib().oracle_atax(nx, ny, _p(y), _p(tmp), _p(A), _p(_f64(x)))
+    return y, tmp
+
+
+def bicg(A, r, p):
+    """PolyBench 3.2 bicg: s = A^T r, q = A p. Returns (s, q)."""
+    A = _f64(A); nx, ny = A.shape
+    s = np.zeros(ny); q = np.zeros(nx)
+    lib().oracle_bicg(nx, ny, _p(s), _p(q), _p(A), _p(_f64(r)), _p(_f64(p)))
+    return s, q
+
+
+def gemver(alpha, beta, A, x, w, u1, v1, u2, v2, y, z):
+    """PolyBench 3.2 gemver. Returns (A, x, w)."""
+    A = _f64(A).copy(); x = _f64(x).copy(); w = _f64(w).copy()
+    n = x.shape[0]
+    assert A.shape == (n, n)
+    lib().oracle_gemver(n, float(alpha), float(beta), _p(A), _p(x), _p(w), _p(_f64(u1)), _p(_f64(v1)),
+                        _p(_f64(u2)), _p(_f64(v2)), _p(_f64(y)), _p(_f64(z)))
+    return A, x, w
 
 
 def normwise_rel_err(x, ref) -> float:

@@ -248,6 +248,66 @@ void oracle_ccsd_t_d1_entries(const int64_t *d, int64_t n, const int64_t *idx,
     }
 }
 
+/* ------------------------------------------- low-dimensional kernels --- */
+/* the paper's low-dimensional PolyBench kernels (atax, bicg, mvt, gemver:
+ * PAPER.md:240, :248, Fig. 7; mvt in Fig. 9).  PolyBench/C 3.2 bodies, recalled (not printed in
+ * PAPER.md, reading R-N7), literal loop order, float64.                          */
+
+/* mvt:  for i, j: x1[i] = x1[i] + A[i][j] * y_1[j];   for i, j: x2[i] = x2[i] + A[j][i] * y_2[j] */
+void oracle_mvt(int64_t n, double *x1, double *x2, const double *y1, const double *y2, const double *A)
+{
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < n; i++)
+        for (int64_t j = 0; j < n; j++) x1[i] = x1[i] + A[IDX2(i, j, n)] * y1[j];
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < n; i++)
+        for (int64_t j = 0; j < n; j++) x2[i] = x2[i] + A[IDX2(j, i, n)] * y2[j];
+}
+
+/* atax:  y[j] = 0;  for i: { tmp[i] = 0; for j: tmp[i] = tmp[i] + A[i][j] * x[j];
+ *                            for j: y[j] = y[j] + A[i][j] * tmp[i]; }                          */
+void oracle_atax(int64_t nx, int64_t ny, double *y, double *tmp, const double *A, const double *x)
+{
+    for (int64_t j = 0; j < ny; j++) y[j] = 0.0;
+    for (int64_t i = 0; i < nx; i++) {
+        tmp[i] = 0.0;
+        for (int64_t j = 0; j < ny; j++) tmp[i] = tmp[i] + A[IDX2(i, j, ny)] * x[j];
+        for (int64_t j = 0; j < ny; j++) y[j] = y[j] + A[IDX2(i, j, ny)] * tmp[i];
+    }
+}
+
+/* bicg:  s[j] = 0;  for i: { q[i] = 0; for j: { s[j] = s[j] + r[i] * A[i][j];
+ *                                                q[i] = q[i] + A[i][j] * p[j]; } }               */
+void oracle_bicg(int64_t nx, int64_t ny, double *s, double *q, const double *A, const double *r, const double *p)
+{
+    for (int64_t j = 0; j < ny; j++) s[j] = 0.0;
+    for (int64_t i = 0; i < nx; i++) {
+        q[i] = 0.0;
+        for (int64_t j = 0; j < ny; j++) {
+            s[j] = s[j] + r[i] * A[IDX2(i, j, ny)];
+            q[i] = q[i] + A[IDX2(i, j, ny)] * p[j];
+        }
+    }
+}
+
+/* gemver:  A[i][j] = A[i][j] + u1[i]*v1[j] + u2[i]*v2[j];
+ *          x[i] = x[i] + beta * A[j][i] * y[j];   x[i] = x[i] + z[i];
+ *          w[i] = w[i] + alpha * A[i][j] * x[j]                                                  */
+void oracle_gemver(int64_t n, double alpha, double beta, double *A, double *x, double *w, const double *u1,
+                   const double *v1, const double *u2, const double *v2, const double *y, const double *z)
+{
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < n; i++)
+        for (int64_t j = 0; j < n; j++) A[IDX2(i, j, n)] = A[IDX2(i, j, n)] + u1[i] * v1[j] + u2[i] * v2[j];
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < n; i++)
+        for (int64_t j = 0; j < n; j++) x[i] = x[i] + beta * A[IDX2(j, i, n)] * y[j];
+    for (int64_t i = 0; i < n; i++) x[i] = x[i] + z[i];
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < n; i++)
+        for (int64_t j = 0; j < n; j++) w[i] = w[i] + alpha * A[IDX2(i, j, n)] * x[j];
+}
+
 /* Number of OpenMP threads the oracle uses (reported as cpu_baseline.cores). */
 #ifdef _OPENMP
 #include <omp.h>
