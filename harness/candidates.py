@@ -43,6 +43,11 @@ KINDS = {
     "jacobi-2d": dict(dims=(4000,), tsteps=500),
     "heat-3d": dict(dims=(120,), tsteps=500),
     "ccsd_t_d1": dict(dims=(48,)),
+    # low-dimensional PolyBench kernels (PolyBench EXTRALARGE-like n = 4000)
+    "mvt": dict(dims=(4000,)),
+    "atax": dict(dims=(4000, 4000)),
+    "bicg": dict(dims=(4000, 4000)),
+    "gemver": dict(dims=(4000,)),
 }
 
 

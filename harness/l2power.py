@@ -11,7 +11,7 @@ correlation (P:264-268, Fig. 9: '0.85 and 0.75 for 2mm and gemm, respectively').
      (warm-up, >= --window s of back-to-back runs, NVML energy counter, P:225);
   2. ``--phase l2`` (run under ncu, one launch per variant and nest):
         ncu --metrics lts__t_sectors_srcunit_tex_op_read.sum,lts__t_sectors_op_read.sum,gpu__time_duration.sum \
-            -k regex:'contract|jacobi2d' --csv --log-file l2.csv python harness/l2power.py --phase l2 ...
+            -k regex:'contract|jacobi2d|lowdim_kernel' --csv --log-file l2.csv python harness/l2power.py --phase l2 ...
   3. ``--phase report``: join both, Pearson r of power vs L2 read sectors per second (and per run).
 
 Power comes only from phase 1 (ncu serialises and replays kernels, so it never measures time
@@ -33,13 +33,14 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
 SIZES = [4, 8, 16, 24, 32, 48, 64, 96, 128, 192, 256, 384, 512, 768, 1024]
-KINDS = {"gemm": ((4000, 4000, 4000), 0), "2mm": ((4000, 4000, 4000, 4000), 0), "jacobi-2d": ((4000,), 1)}
+KINDS = {"gemm": ((4000, 4000, 4000), 0), "2mm": ((4000, 4000, 4000, 4000), 0), "jacobi-2d": ((4000,), 1),
+         "mvt": ((4000,), 0)}
 
 
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--phase", choices=["power", "l2", "report"], required=True)
-    ap.add_argument("--kinds", default="gemm,2mm,jacobi-2d")
+    ap.add_argument("--kinds", default="gemm,2mm,jacobi-2d,mvt")
     ap.add_argument("--count", type=int, default=120, help="variants per kind (jacobi-2d: at most 225)")
     ap.add_argument("--seed", type=int, default=0)
     ap.add_argument("--window", type=float, default=0.5)
@@ -52,7 +53,7 @@ def parse():
 
 def variants(kind, count, seed):
     dims, _ = KINDS[kind]
-    depth = 2 if kind == "jacobi-2d" else 3
+    depth = 2 if kind in ("jacobi-2d", "mvt") else 3
     space = list(itertools.product(SIZES, repeat=depth))
     random.Random(seed).shuffle(space)
     return space[: min(count, len(space))]
@@ -60,7 +61,7 @@ def variants(kind, count, seed):
 
 def nest_kernels(kind):
     """Kernel launches matched by the ncu filter per run of one variant."""
-    return {"gemm": 1, "2mm": 2, "jacobi-2d": 1}[kind]
+    return {"gemm": 1, "2mm": 2, "jacobi-2d": 1, "mvt": 1}[kind]
 
 
 def make(E, torch, kind):
@@ -158,7 +159,7 @@ def phase_report(a):
                          r_power_vs_sectors_per_run=pearson(w, [p[1] for p in pts]),
                          r_power_vs_all_l2_read_sectors_per_s=pearson(w, [p[5] for p in pts]),
                          watts_range=[min(w), max(w)],
-                         paper_r={"gemm": 0.75, "2mm": 0.85, "jacobi-2d": "no correlation"}.get(kind))
+                         paper_r={"gemm": 0.75, "2mm": 0.85, "jacobi-2d": "no correlation", "mvt": "no correlation"}.get(kind))
     out["launches_parsed"] = len(launches)
     out["launches_used"] = pos
     json.dump(out, open(a.out, "w"), indent=1)

@@ -44,7 +44,7 @@ extern "C" {
 #define EATSS_ABI_VERSION 1
 #define EATSS_MAX_LOOPS 8
 #define EATSS_MAX_NESTS 4
-#define EATSS_MAX_BUFFERS 8
+#define EATSS_MAX_BUFFERS 16
 
 typedef enum {
     EATSS_OK = 0,
@@ -80,8 +80,19 @@ typedef enum { EATSS_F32 = 1, EATSS_F64 = 2 } eatss_dtype;
  *   EATSS_CCSD_T_D1 dims (h3,h2,h1,p6,p5,p4,h7) or (d) buffers {t3 (in/out), t2[h7][p4][p5][h1],
  *                                                              v2[h3][h2][p6][h7]}
  *                   t3[h3][h2][h1][p6][p5][p4] -= sum_h7 t2[h7][p4][p5][h1]*v2[h3][h2][p6][h7]
+ * Low-dimensional PolyBench 3.2 kernels (Fig. 7, Fig. 9),
+ * fp32; one executor pass streams the matrix once and may serve two products (reading R-N7):
+ *   EATSS_MVT       dims (n)                   buffers {x1[n] (in/out), x2[n] (in/out), y_1[n], y_2[n], A[n][n]}
+ *                   x1[i] += A[i][j]*y_1[j];  x2[i] += A[j][i]*y_2[j]
+ *   EATSS_ATAX      dims (nx, ny)              buffers {y[ny] (out), tmp[nx] (out), A[nx][ny], x[ny]}
+ *                   tmp = A x;  y = A^T tmp
+ *   EATSS_BICG      dims (nx, ny)              buffers {s[ny] (out), q[nx] (out), A[nx][ny], r[nx], p[ny]}
+ *                   s = A^T r;  q = A p
+ *   EATSS_GEMVER    dims (n)                   buffers {A[n][n] (in/out), x (in/out), w (in/out),
+ *                                                       u1, v1, u2, v2, y, z} (vectors of n)
+ *                   A += u1 v1^T + u2 v2^T;  x += beta A^T y;  x += z;  w += alpha A x
  * The tile vector has one entry per loop depth position (reading Q15): 3 for the
- * gemm family, 2 for jacobi-2d, 3 for heat-3d, 7 for ccsd_t_d1
+ * gemm family, 2 for jacobi-2d and the low-dimensional kernels, 3 for heat-3d, 7 for ccsd_t_d1
  * (h3,h2,h1,p6,p5,p4,h7).  Stencil time loops are not tiled.
  */
 typedef enum {
@@ -91,7 +102,11 @@ typedef enum {
     EATSS_SYRK = 3,
     EATSS_JACOBI2D = 4,
     EATSS_HEAT3D = 5,
-    EATSS_CCSD_T_D1 = 6
+    EATSS_CCSD_T_D1 = 6,
+    EATSS_MVT = 7,
+    EATSS_ATAX = 8,
+    EATSS_BICG = 9,
+    EATSS_GEMVER = 10
 } eatss_builtin;
 
 /* GPU parameters of the model: Table I + SM count + the

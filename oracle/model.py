@@ -531,7 +531,45 @@ def fdtd2d(nx=1000, ny=1000, dtype_bytes=8) -> Program:
     return P("fdtd-2d", [n1, n2, n3], dtype_bytes)
 
 
+# Low-dimensional PolyBench 3.2 kernels (Fig. 7): 2-deep nests
+# (i, j), the reduction loop not parallel (reading R-N7).
+def mvt(n=4000, dtype_bytes=4) -> Program:
+    loops = [Loop("i", n, True), Loop("j", n, False)]
+    n1 = Nest(list(loops), [ref("x1", "i", write=True), ref("x1", "i"), ref("A", "i", "j"), ref("y_1", "j")])
+    n2 = Nest(list(loops), [ref("x2", "i", write=True), ref("x2", "i"), ref("A", "j", "i"), ref("y_2", "j")])
+    return P("mvt", [n1, n2], dtype_bytes)
+
+
+def atax(nx=4000, ny=4000, dtype_bytes=4) -> Program:
+    n1 = Nest([Loop("i", nx, True), Loop("j", ny, False)],
+              [ref("tmp", "i", write=True), ref("tmp", "i"), ref("A", "i", "j"), ref("x", "j")])
+    n2 = Nest([Loop("i", nx, False), Loop("j", ny, True)],
+              [ref("y", "j", write=True), ref("y", "j"), ref("A", "i", "j"), ref("tmp", "i")])
+    return P("atax", [n1, n2], dtype_bytes)
+
+
+def bicg(nx=4000, ny=4000, dtype_bytes=4) -> Program:
+    n1 = Nest([Loop("i", nx, False), Loop("j", ny, True)],
+              [ref("s", "j", write=True), ref("s", "j"), ref("r", "i"), ref("A", "i", "j")])
+    n2 = Nest([Loop("i", nx, True), Loop("j", ny, False)],
+              [ref("q", "i", write=True), ref("q", "i"), ref("A", "i", "j"), ref("p", "j")])
+    return P("bicg", [n1, n2], dtype_bytes)
+
+
+def gemver(n=4000, dtype_bytes=4) -> Program:
+    n1 = Nest([Loop("i", n, True), Loop("j", n, True)],
+              [ref("A", "i", "j", write=True), ref("A", "i", "j"), ref("u1", "i"), ref("v1", "j"),
+               ref("u2", "i"), ref("v2", "j")])
+    n2 = Nest([Loop("i", n, True), Loop("j", n, False)],
+              [ref("x", "i", write=True), ref("x", "i"), ref("A", "j", "i"), ref("y", "j")])
+    n3 = Nest([Loop("i", n, True)], [ref("x", "i", write=True), ref("x", "i"), ref("z", "i")])
+    n4 = Nest([Loop("i", n, True), Loop("j", n, False)],
+              [ref("w", "i", write=True), ref("w", "i"), ref("A", "i", "j"), ref("x", "j")])
+    return P("gemver", [n1, n2, n3, n4], dtype_bytes)
+
+
 BUILTINS = {
     "gemm": gemm, "2mm": two_mm, "3mm": three_mm, "syrk": syrk,
     "jacobi-2d": jacobi2d, "heat-3d": heat3d, "ccsd_t_d1": ccsd_t_d1,
+    "mvt": mvt, "atax": atax, "bicg": bicg, "gemver": gemver,
 }

@@ -41,6 +41,24 @@ cudaError_t launch_ccsd_tc(float *t3, const float *t2, const float *v2, const in
 void ccsd_plan_dims(const int64_t *dims, const int64_t *tiles, int64_t *gx, int64_t *gy, int *bx,
                     int *by, int *rm, int *rn, int *passes, int *smem);
 
+// lowdim.cu entry points (mvt, atax, bicg, gemver)
+struct LowdimArgs {
+    const float *A;
+    float *Aout;
+    int64_t nx, ny;
+    int Ti, Tj;
+    float *rowout;
+    const float *vr;
+    float ar;
+    float *colout;
+    const float *vc;
+    float ac;
+    const float *u1, *v1, *u2, *v2;
+};
+cudaError_t launch_lowdim(const LowdimArgs &a, bool row, bool col, bool upd, cudaStream_t s, int64_t *launched);
+cudaError_t launch_lowdim_axpy(float *out, const float *add, float scale, int64_t n, cudaStream_t s,
+                               int64_t *launched);
+
 // ------------------------------------------------------------------ builtin nests
 // Loop positions are bits: the model only needs which loops a subscript uses.
 static Sub S(uint32_t iters, int off = 0) {
@@ -137,6 +155,54 @@ static eatss_status build(eatss_kernel_desc *d) {
                                x[0] * x[1] * x[3] * x[6]};
             break;
         }
+        // low-dimensional PolyBench 3.2 kernels (reading R-N7): 2-deep nests
+        // (i, j); a reduction loop is marked not parallel
+        case EATSS_MVT: {  // x1 x2 y_1 y_2 A ; dims n
+            const int64_t n = x[0];
+            Nest a, b;
+            a.loops = b.loops = {{n, true}, {n, false}};
+            a.refs = {R(0, {S(I)}, true), R(0, {S(I)}), R(4, {S(I), S(J)}), R(2, {S(J)})};
+            b.refs = {R(1, {S(I)}, true), R(1, {S(I)}), R(4, {S(J), S(I)}), R(3, {S(J)})};
+            d->nests = {a, b};
+            d->buffer_elems = {n, n, n, n, n * n};
+            break;
+        }
+        case EATSS_ATAX: {  // y tmp A x ; dims (nx, ny)
+            Nest a, b;
+            a.loops = {{x[0], true}, {x[1], false}};
+            a.refs = {R(1, {S(I)}, true), R(1, {S(I)}), R(2, {S(I), S(J)}), R(3, {S(J)})};
+            b.loops = {{x[0], false}, {x[1], true}};
+            b.refs = {R(0, {S(J)}, true), R(0, {S(J)}), R(2, {S(I), S(J)}), R(1, {S(I)})};
+            d->nests = {a, b};
+            d->buffer_elems = {x[1], x[0], x[0] * x[1], x[1]};
+            break;
+        }
+        case EATSS_BICG: {  // s q A r p ; dims (nx, ny)
+            Nest a, b;
+            a.loops = {{x[0], false}, {x[1], true}};
+            a.refs = {R(0, {S(J)}, true), R(0, {S(J)}), R(3, {S(I)}), R(2, {S(I), S(J)})};
+            b.loops = {{x[0], true}, {x[1], false}};
+            b.refs = {R(1, {S(I)}, true), R(1, {S(I)}), R(2, {S(I), S(J)}), R(4, {S(J)})};
+            d->nests = {a, b};
+            d->buffer_elems = {x[1], x[0], x[0] * x[1], x[0], x[1]};
+            break;
+        }
+        case EATSS_GEMVER: {  // A x w u1 v1 u2 v2 y z ; dims n
+            const int64_t n = x[0];
+            Nest a, b, c, e;
+            a.loops = {{n, true}, {n, true}};
+            a.refs = {R(0, {S(I), S(J)}, true), R(0, {S(I), S(J)}), R(3, {S(I)}), R(4, {S(J)}), R(5, {S(I)}),
+                      R(6, {S(J)})};
+            b.loops = {{n, true}, {n, false}};
+            b.refs = {R(1, {S(I)}, true), R(1, {S(I)}), R(0, {S(J), S(I)}), R(7, {S(J)})};
+            c.loops = {{n, true}};
+            c.refs = {R(1, {S(I)}, true), R(1, {S(I)}), R(8, {S(I)})};
+            e.loops = {{n, true}, {n, false}};
+            e.refs = {R(2, {S(I)}, true), R(2, {S(I)}), R(0, {S(I), S(J)}), R(1, {S(J)})};
+            d->nests = {a, b, c, e};
+            d->buffer_elems = {n * n, n, n, n, n, n, n, n, n};
+            break;
+        }
         default:
             return fail(EATSS_E_INVALID, "eatss_desc_builtin: unknown builtin");
     }
@@ -144,7 +210,11 @@ static eatss_status build(eatss_kernel_desc *d) {
     return EATSS_OK;
 }
 
-static const int kDimsPerBuiltin[] = {3, 4, 5, 2, 1, 1, 7};
+static const int kDimsPerBuiltin[] = {3, 4, 5, 2, 1, 1, 7, 1, 2, 2, 1};
+
+static bool is_lowdim(eatss_builtin k) {
+    return k == EATSS_MVT || k == EATSS_ATAX || k == EATSS_BICG || k == EATSS_GEMVER;
+}
 
 // ------------------------------------------------------------------ execution helpers
 static int smem_limit_bytes() {
@@ -324,7 +394,7 @@ eatss_status eatss_desc_builtin(eatss_builtin k, const int64_t *dims, int ndims,
                                 int64_t tsteps, eatss_kernel_desc **out) {
     if (!out) return fail(EATSS_E_INVALID, "eatss_desc_builtin: out is null");
     *out = nullptr;
-    if ((int)k < 0 || (int)k > (int)EATSS_CCSD_T_D1) return fail(EATSS_E_INVALID, "eatss_desc_builtin: bad builtin");
+    if ((int)k < 0 || (int)k > (int)EATSS_GEMVER) return fail(EATSS_E_INVALID, "eatss_desc_builtin: bad builtin");
     if (dt != EATSS_F32 && dt != EATSS_F64) return fail(EATSS_E_INVALID, "eatss_desc_builtin: bad dtype");
     if (!dims) return fail(EATSS_E_INVALID, "eatss_desc_builtin: dims is null");
     const int want = kDimsPerBuiltin[k];
@@ -384,6 +454,9 @@ double eatss_desc_flops(const eatss_kernel_desc *d) {
         case EATSS_JACOBI2D: return 5 * D(x[0] - 2) * D(x[0] - 2) * D(d->tsteps);
         case EATSS_HEAT3D: return 15 * D(x[0] - 2) * D(x[0] - 2) * D(x[0] - 2) * 2 * D(d->tsteps);
         case EATSS_CCSD_T_D1: return 2 * D(x[0]) * D(x[1]) * D(x[2]) * D(x[3]) * D(x[4]) * D(x[5]) * D(x[6]);
+        case EATSS_MVT: return 4 * D(x[0]) * D(x[0]);
+        case EATSS_ATAX: case EATSS_BICG: return 4 * D(x[0]) * D(x[1]);
+        case EATSS_GEMVER: return 10 * D(x[0]) * D(x[0]) + D(x[0]);  // 4 + 3 + 3 per (i, j), + per i
     }
     return 0;
 }
@@ -409,6 +482,13 @@ double eatss_desc_bytes(const eatss_kernel_desc *d) {
         case EATSS_HEAT3D: return e * 2 * D(x[0]) * D(x[0]) * D(x[0]) * 2 * D(d->tsteps);
         case EATSS_CCSD_T_D1:
             return e * (2 * D(d->buffer_elems[0]) + D(d->buffer_elems[1]) + D(d->buffer_elems[2]));
+        // the matrix once (mvt, bicg: both products from one read -- the fused pass) or twice (atax:
+        // tmp = A x must be complete before y = A^T tmp); gemver: A read + written by the update,
+        // read again by w = A' x; vectors once each (read, + write for outputs)
+        case EATSS_MVT: return e * (D(x[0]) * D(x[0]) + 6 * D(x[0]));
+        case EATSS_ATAX: return e * (2 * D(x[0]) * D(x[1]) + 2 * D(x[1]) + D(x[0]));
+        case EATSS_BICG: return e * (D(x[0]) * D(x[1]) + 2 * D(x[0]) + 2 * D(x[1]));
+        case EATSS_GEMVER: return e * (3 * D(x[0]) * D(x[0]) + 11 * D(x[0]));
     }
     return 0;
 }
@@ -507,6 +587,19 @@ eatss_status eatss_plan(const eatss_kernel_desc *d, const int64_t *tiles, eatss_
             for (int p = 0; p < L; p++) o.tile[p] = t[p];
         }
         *n_plans = nn;
+    } else if (is_lowdim(d->kind)) {  // one CTA per (Ti, Tj) block of the matrix, 256 threads
+        const int64_t nx = d->dims[0], ny = d->kind == EATSS_ATAX || d->kind == EATSS_BICG ? d->dims[1] : d->dims[0];
+        for (int i = 0; i < nn; i++) {
+            eatss_launch_plan &o = plans[i];
+            std::memset(&o, 0, sizeof(o));
+            o.nest = i; o.engine = 1;
+            const int64_t ti = std::min(tiles[0], nx), tj = std::min(tiles[1], ny);
+            o.grid_x = (ny + tj - 1) / tj; o.grid_y = (nx + ti - 1) / ti; o.grid_z = 1;
+            o.block_x = 256; o.block_y = 1; o.rm = 1; o.rn = 4; o.vec = (ny % 4 == 0 && tj % 4 == 0) ? 4 : 1;
+            o.passes = 1; o.carveout_pct = d->exec.split_pct; o.simt_x = 32;
+            o.tile[0] = ti; o.tile[1] = tj;
+        }
+        *n_plans = nn;
     } else {
         eatss_launch_plan &o = plans[0];
         std::memset(&o, 0, sizeof(o));
@@ -519,6 +612,58 @@ eatss_status eatss_plan(const eatss_kernel_desc *d, const int64_t *tiles, eatss_
         *n_plans = 1;
     }
     return EATSS_OK;
+}
+
+// mvt / atax / bicg / gemver as passes of the tiled matrix-vector executor (lowdim.cu); the tile
+// (Ti, Tj) maps rows x columns of the matrix for every pass.  `launched` counts kernels (may be null).
+static cudaError_t lowdim_run(const eatss_kernel_desc *d, const int64_t *t, void *const *b, cudaStream_t s,
+                              int64_t *launched) {
+    auto F = [&](int i) { return static_cast<float *>(b[i]); };
+    const auto &x = d->dims;
+    LowdimArgs a{};
+    a.Ti = (int)std::min<int64_t>(t[0], INT32_MAX);
+    a.Tj = (int)std::min<int64_t>(t[1], INT32_MAX);
+    cudaError_t e;
+    auto zero = [&](int i) { return cudaMemsetAsync(b[i], 0, (size_t)d->buffer_elems[i] * 4, s); };
+    switch (d->kind) {
+        case EATSS_MVT:  // x1 += A y_1 (row form), x2 += A^T y_2 (col form): one pass over A
+            a.A = F(4); a.nx = a.ny = x[0];
+            a.rowout = F(0); a.vr = F(2); a.ar = 1.f;
+            a.colout = F(1); a.vc = F(3); a.ac = 1.f;
+            return launch_lowdim(a, true, true, false, s, launched);
+        case EATSS_ATAX:  // tmp = A x; y = A^T tmp (tmp complete first)
+            if ((e = zero(0)) != cudaSuccess || (e = zero(1)) != cudaSuccess) return e;
+            a.A = F(2); a.nx = x[0]; a.ny = x[1];
+            a.rowout = F(1); a.vr = F(3); a.ar = 1.f;
+            if ((e = launch_lowdim(a, true, false, false, s, launched)) != cudaSuccess) return e;
+            a.colout = F(0); a.vc = F(1); a.ac = 1.f;
+            return launch_lowdim(a, false, true, false, s, launched);
+        case EATSS_BICG:  // s = A^T r (col form), q = A p (row form): one pass over A
+            if ((e = zero(0)) != cudaSuccess || (e = zero(1)) != cudaSuccess) return e;
+            a.A = F(2); a.nx = x[0]; a.ny = x[1];
+            a.colout = F(0); a.vc = F(3); a.ac = 1.f;
+            a.rowout = F(1); a.vr = F(4); a.ar = 1.f;
+            return launch_lowdim(a, true, true, false, s, launched);
+        case EATSS_GEMVER: {  // A' = A + u1 v1^T + u2 v2^T fused with x += beta A'^T y; x += z; w += alpha A' x
+            // the fused pass carries nest 2 (x[i] += beta A[j][i] y[j]): its loop i runs along A's
+            // columns, so that pass maps tile position 0 to columns and position 1 to rows
+            a.Ti = (int)std::min<int64_t>(t[1], INT32_MAX);
+            a.Tj = (int)std::min<int64_t>(t[0], INT32_MAX);
+            a.A = F(0); a.Aout = F(0); a.nx = a.ny = x[0];
+            a.u1 = F(3); a.v1 = F(4); a.u2 = F(5); a.v2 = F(6);
+            a.colout = F(1); a.vc = F(7); a.ac = (float)d->beta;
+            if ((e = launch_lowdim(a, false, true, true, s, launched)) != cudaSuccess) return e;
+            if ((e = launch_lowdim_axpy(F(1), F(8), 1.f, x[0], s, launched)) != cudaSuccess) return e;
+            LowdimArgs w{};
+            w.A = F(0); w.nx = w.ny = x[0];
+            w.Ti = (int)std::min<int64_t>(t[0], INT32_MAX);  // nest 4: i rows, j columns
+            w.Tj = (int)std::min<int64_t>(t[1], INT32_MAX);
+            w.rowout = F(2); w.vr = F(1); w.ar = (float)d->alpha;
+            return launch_lowdim(w, true, false, false, s, launched);
+        }
+        default:
+            return cudaErrorInvalidValue;
+    }
 }
 
 static eatss_status run_impl(const eatss_kernel_desc *cd, int only_nest, const int64_t *tiles,
@@ -555,6 +700,16 @@ static eatss_status run_impl(const eatss_kernel_desc *cd, int only_nest, const i
             if (e != cudaSuccess) return cuda_fail(e, "eatss_run(contraction)");
         }
         return EATSS_OK;
+    }
+    if (is_lowdim(d->kind)) {
+        if (only_nest >= 0) return fail(EATSS_E_UNSUPPORTED, "eatss_run_nest: low-dimensional kernels run whole");
+        if (d->dtype != EATSS_F32)  // fp64 descriptors serve the model (paper-mode tables) only
+            return fail(EATSS_E_UNSUPPORTED, "eatss_run: the low-dimensional executor is fp32 only");
+        cudaEvent_t *ev = kernel_events(d, 0);
+        if (ev) cudaEventRecord(ev[0], s);
+        const cudaError_t e = lowdim_run(d, tiles, buffers, s, nullptr);
+        if (ev) cudaEventRecord(ev[1], s);
+        return e == cudaSuccess ? EATSS_OK : cuda_fail(e, "eatss_run(low-dimensional kernel)");
     }
     if (d->kind == EATSS_JACOBI2D || d->kind == EATSS_HEAT3D) {
         if (only_nest >= 0) return fail(EATSS_E_UNSUPPORTED, "eatss_run_nest: stencils run whole time loops");
@@ -601,6 +756,10 @@ static void buffer_io(const eatss_kernel_desc *d, int i, bool *in, bool *out) {
         case EATSS_2MM: *in = i != 0; *out = i == 0 || i == 4; break;
         case EATSS_3MM: *in = !(i == 0 || i == 3 || i == 6); *out = !*in; break;
         case EATSS_JACOBI2D: case EATSS_HEAT3D: *out = true; break;
+        case EATSS_MVT: *out = i <= 1; break;
+        case EATSS_ATAX: *in = i >= 2; *out = i <= 1; break;
+        case EATSS_BICG: *in = i >= 2; *out = i <= 1; break;
+        case EATSS_GEMVER: *out = i <= 2; break;
     }
 }
 
@@ -764,6 +923,8 @@ eatss_status eatss_coverage(const eatss_kernel_desc *d, int nest, const int64_t 
         cudaError_t e = launch_contraction(cn[nest], p, d->exec.split_pct, counts, s);
         return e == cudaSuccess ? EATSS_OK : cuda_fail(e, "eatss_coverage");
     }
+    if (is_lowdim(d->kind))
+        return fail(EATSS_E_UNSUPPORTED, "eatss_coverage: the low-dimensional kernels have no visit-count mode");
     const int64_t n = d->dims[0];
     cudaError_t e;
     if (d->kind == EATSS_JACOBI2D)
@@ -799,6 +960,9 @@ int64_t eatss_launches_per_run(const eatss_kernel_desc *d, const int64_t *tiles)
         case EATSS_3MM: return 3;
         case EATSS_JACOBI2D: return d->tsteps + (d->tsteps > 0 ? 1 : 0);
         case EATSS_HEAT3D: return 2 * d->tsteps;
+        case EATSS_MVT: case EATSS_BICG: return 1;  // one fused pass over the matrix
+        case EATSS_ATAX: return 2;
+        case EATSS_GEMVER: return 3;
     }
     return -1;
 }

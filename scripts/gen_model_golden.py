@@ -54,6 +54,12 @@ add("gemm", (4000, 4000, 4000), 4, "GA100", 50, 16, 2)
 add("ccsd_t_d1", (48,), 4, "B200", 50, 4, 1)
 add("ccsd_t_d1", (48,), 4, "B200", 50, 8, 1)
 add("ccsd_t_d1", (16,), 4, "B200", 50, 4, 1)
+# low-dimensional PolyBench kernels
+for kern, dims in (("mvt", (4000,)), ("atax", (4000, 4000)), ("bicg", (4000, 4000)), ("gemver", (4000,)),
+                   ("atax", (1900, 2100)), ("bicg", (2100, 1900))):
+    for split, waf in ((50, 16), (0, 4), (100, 32)):
+        add(kern, dims, 4, "B200", split, waf, 1)
+add("gemver", (4000,), 8, "GA100", 50, 16, 0)
 
 
 def main():

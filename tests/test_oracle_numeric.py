@@ -174,3 +174,65 @@ def test_ccsd_t_d1_small_int_exact_and_entries():
 def test_normwise_error_definition():
     ref = np.array([3.0, 4.0]); x = np.array([3.0, 4.5])
     assert O.normwise_rel_err(x, ref) == pytest.approx(0.5 / 5.0)
+
+
+# ---------------------------------------------------------------- low-dimensional kernels
+# (PolyBench 3.2 mvt / atax / bicg / gemver, reading R-N7).  Pins: closed forms
+# on rank-1 integer matrices (every value an exact integer in fp64), and integer-matrix identities.
+
+def _ints(shape, seed, lo=-4, hi=5):
+    return np.random.default_rng(seed).integers(lo, hi, size=shape).astype(np.float64)
+
+
+def test_mvt_rank1_closed_form():
+    n = 37
+    u, v = _ints(n, 1), _ints(n, 2)
+    A = np.outer(u, v)
+    x1, x2, y1, y2 = _ints(n, 3), _ints(n, 4), _ints(n, 5), _ints(n, 6)
+    r1, r2 = O.mvt(x1, x2, y1, y2, A)
+    # x1 += A y1 = u (v . y1);  x2 += A^T y2 = v (u . y2)
+    assert np.array_equal(r1, x1 + u * float(v @ y1))
+    assert np.array_equal(r2, x2 + v * float(u @ y2))
+
+
+def test_mvt_transposed_operand_is_not_swapped():
+    """A non-symmetric integer matrix: x2 must use A^T (a swapped index fails here)."""
+    A = np.triu(np.ones((5, 5)))
+    y = np.arange(1.0, 6.0)
+    r1, r2 = O.mvt(np.zeros(5), np.zeros(5), y, y, A)
+    assert np.array_equal(r1, np.array([15.0, 14.0, 12.0, 9.0, 5.0]))   # row suffix sums
+    assert np.array_equal(r2, np.array([1.0, 3.0, 6.0, 10.0, 15.0]))    # column prefix sums
+
+
+def test_atax_rank1_closed_form_and_rectangular():
+    nx, ny = 23, 31
+    u, v, x = _ints(nx, 7), _ints(ny, 8), _ints(ny, 9)
+    y, tmp = O.atax(np.outer(u, v), x)
+    assert np.array_equal(tmp, u * float(v @ x))
+    assert np.array_equal(y, v * float(u @ u) * float(v @ x))
+    A = _ints((nx, ny), 10)
+    y2, tmp2 = O.atax(A, x)
+    assert np.array_equal(tmp2, A.astype(np.int64) @ x.astype(np.int64))
+    assert np.array_equal(y2, A.T.astype(np.int64) @ (A.astype(np.int64) @ x.astype(np.int64)))
+
+
+def test_bicg_integer_identities():
+    nx, ny = 19, 29
+    A, r, p = _ints((nx, ny), 11), _ints(nx, 12), _ints(ny, 13)
+    s, q = O.bicg(A, r, p)
+    Ai = A.astype(np.int64)
+    assert np.array_equal(s, Ai.T @ r.astype(np.int64))
+    assert np.array_equal(q, Ai @ p.astype(np.int64))
+
+
+def test_gemver_closed_form_on_integers():
+    n = 17
+    A = _ints((n, n), 14)
+    x, w, u1, v1, u2, v2, y, z = (_ints(n, 15 + k) for k in range(8))
+    alpha, beta = 2.0, -1.0
+    An, xn, wn = O.gemver(alpha, beta, A, x, w, u1, v1, u2, v2, y, z)
+    Ap = A + np.outer(u1, v1) + np.outer(u2, v2)
+    xp = x + beta * (Ap.T @ y) + z
+    assert np.array_equal(An, Ap)
+    assert np.array_equal(xn, xp)
+    assert np.array_equal(wn, w + alpha * (Ap @ xp))   # w uses the UPDATED x (nest order)
