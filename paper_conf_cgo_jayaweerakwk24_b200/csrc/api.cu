@@ -954,10 +954,17 @@ int64_t eatss_launches_per_run(const eatss_kernel_desc *d, const int64_t *tiles)
         return total;
     }
     if (d->kind == EATSS_CCSD_T_D1 && d->exec.engine == EATSS_ENGINE_TENSOR) return 2;  // prep + contraction
+    if (is_contraction(d->kind)) {  // SIMT: one kernel per nest (+ the tail pre-pass when it splits)
+        if (!tiles || check_tiles(d, tiles) != EATSS_OK) return -1;
+        void *b[EATSS_MAX_BUFFERS];
+        for (int i = 0; i < EATSS_MAX_BUFFERS; i++) b[i] = (void *)((uintptr_t)(1 << 20) * (uintptr_t)(i + 1));
+        int64_t total = 0;
+        const int sl = smem_limit_bytes();
+        for (auto &n : contraction_nests(d, b)) total += contraction_launches(n, plan_contraction(n, tiles, sl));
+        return total;
+    }
     switch (d->kind) {
-        case EATSS_GEMM: case EATSS_SYRK: case EATSS_CCSD_T_D1: return 1;
-        case EATSS_2MM: return 2;
-        case EATSS_3MM: return 3;
+        case EATSS_CCSD_T_D1: return 1;
         case EATSS_JACOBI2D: return d->tsteps + (d->tsteps > 0 ? 1 : 0);
         case EATSS_HEAT3D: return 2 * d->tsteps;
         case EATSS_MVT: case EATSS_BICG: return 1;  // one fused pass over the matrix

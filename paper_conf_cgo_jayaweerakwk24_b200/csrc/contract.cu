@@ -43,6 +43,9 @@ struct CArgs {
     int a_smem, b_smem, nbuf;
     int tkp, tjp;
     int bkp;  // staged transposed operand: B slice kept as [j][k] with this k-pitch (0 = [k][j] layout)
+    int64_t gx;      // staged: j-tiles of the grid (tile index t = ti * gx + tj)
+    int64_t nfull;   // staged: tiles run whole; tiles >= nfull are split along k into sp parts
+    int sp;          // staged: 1 = 2-D grid, no split
     int passes_i, passes_j;
     int32_t *counts;  // coverage mode
 };
@@ -593,6 +596,9 @@ static cudaError_t launch_one(const CArgs<T> &a, const ContractPlan &p, int carv
     return cudaGetLastError();
 }
 
+// contraction_launches(): set while counting the kernels a launch would issue (no launch happens)
+static thread_local int *g_dry_launches = nullptr;
+
 template <typename T, int RM, int RN, int V, bool TB>
 static cudaError_t launch_staged(const CArgs<T> &a, const ContractPlan &p, int carveout, cudaStream_t s) {
     auto k = contract_staged_kernel<T, RM, RN, V, TB>;
@@ -612,8 +618,40 @@ static cudaError_t launch_staged(const CArgs<T> &a, const ContractPlan &p, int c
     }
     e = cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, carveout);
     if (e != cudaSuccess) return e;
-    dim3 grid((unsigned)p.grid_x, (unsigned)p.grid_y, 1), block(p.bx, p.by, 1);
-    k<<<grid, block, p.smem_bytes, s>>>(a);
+    dim3 block(p.bx, p.by, 1);
+    // wave-quantisation tail: when the last wave would leave at least half of the resident-CTA
+    // slots idle, its tiles are split along k (EATSS_SIMT_SPLITK=0 disables)
+    CArgs<T> b = a;
+    b.sp = 1;
+    b.gx = p.grid_x;
+    const int64_t T_ = p.grid_x * p.grid_y;
+    static const bool splitk = !(getenv("EATSS_SIMT_SPLITK") && atoi(getenv("EATSS_SIMT_SPLITK")) == 0);
+    int nb = 0, dev = 0, nsm = 148;
+    if (splitk && cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k, p.bx * p.by, p.smem_bytes) == cudaSuccess &&
+        nb > 0) {
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+        const int64_t slots = (int64_t)nb * nsm, rem = T_ % slots;
+        const int64_t nk = (a.K + a.Tk - 1) / a.Tk;
+        if (T_ > slots && rem > 0 && 2 * rem <= slots) {
+            b.sp = (int)std::min<int64_t>(std::min<int64_t>(4, slots / rem), nk);
+            b.nfull = T_ - rem;
+        }
+    }
+    cudaGetLastError();
+    if (g_dry_launches) {
+        *g_dry_launches += b.sp > 1 ? 2 : 1;
+        return cudaSuccess;
+    }
+    if (b.sp > 1) {
+        const int64_t ntail = T_ - b.nfull;
+        staged_tail_prepass<T><<<(unsigned)(ntail * b.Ti), 256, 0, s>>>(b);
+        if ((e = cudaGetLastError()) != cudaSuccess) return e;
+        k<<<(unsigned)(b.nfull + ntail * b.sp), block, p.smem_bytes, s>>>(b);
+    } else {
+        dim3 grid((unsigned)p.grid_x, (unsigned)p.grid_y, 1);
+        k<<<grid, block, p.smem_bytes, s>>>(b);
+    }
     return cudaGetLastError();
 }
 
@@ -691,6 +729,7 @@ static cudaError_t launch_typed(const ContractNest &n, const ContractPlan &p, in
     a.Tk = p.staged ? p.kst : (int)p.Tk;  // the staged kernel walks k in ring stages of kst rows
     a.a_smem = p.a_smem; a.b_smem = p.b_smem; a.nbuf = p.nbuf;
     a.tkp = p.tkp; a.tjp = p.tjp; a.bkp = p.bkp;
+    a.gx = p.grid_x; a.nfull = 0; a.sp = 1;
     a.passes_i = p.passes_i; a.passes_j = p.passes_j;
     a.counts = counts;
     if (counts) return by_variant<T, MODE_COVER>(a, p, n.transB, carveout, s);
@@ -711,6 +750,15 @@ cudaError_t launch_contraction(const ContractNest &n, const ContractPlan &p, int
     if (p.grid_y > 65535) return cudaErrorInvalidConfiguration;
     if (n.f64) return launch_typed<double>(n, p, carveout_pct, coverage_counts, s);
     return launch_typed<float>(n, p, carveout_pct, coverage_counts, s);
+}
+
+int contraction_launches(const ContractNest &n, const ContractPlan &p) {
+    if (!p.staged || n.M <= 0 || n.N <= 0) return 1;
+    int c = 0;
+    g_dry_launches = &c;
+    launch_contraction(n, p, 50, nullptr, nullptr);
+    g_dry_launches = nullptr;
+    return c > 0 ? c : 1;
 }
 
 }  // namespace eatss

@@ -51,5 +51,8 @@ cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p,
 int tcm_launches(const ContractNest &n, const ContractPlan &p);  // kernels one launch_tcm_contraction issues
 cudaError_t launch_contraction(const ContractNest &n, const ContractPlan &p, int carveout_pct,
                                int32_t *coverage_counts, cudaStream_t s);
+// kernels one launch_contraction issues (the SIMT staged path adds a pre-pass when it splits the
+// wave tail along k)
+int contraction_launches(const ContractNest &n, const ContractPlan &p);
 
 }  // namespace eatss

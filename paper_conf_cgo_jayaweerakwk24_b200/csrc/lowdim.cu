@@ -5,8 +5,8 @@
 // one of two forms (reading R-N7):
 //   row form   rowout[i] (+)= ar * sum_j A[i][j] * vr[j]   (i parallel, j reduction: stride-1 j)
 //   col form   colout[j] (+)= ac * sum_i A[i][j] * vc[i]   (j parallel, i reduction)
-// One tile (Ti, Tj) is one CTA (tj -> blockIdx.x, ti -> blockIdx.y), clipped with min()
-// (reading Q25).  A CTA streams its Ti x Tj block of A once, with 16-byte loads along j (the CMA
+// One tile (Ti, Tj) is executed whole by one CTA (tj -> blockIdx.x; a CTA walks the row
+// tiles ti = blockIdx.y, + gridDim.y, ... in turn), clipped with min() (reading Q25).  A CTA streams its Ti x Tj block of A once, with 16-byte loads along j (the CMA
 // loop), and evaluates BOTH forms from that single read when both are requested: PolyBench's bicg
 // loop computes s = A^T r and q = A p in one sweep, and mvt's two nests read the same matrix, so
 // on B200 each becomes one pass over A instead of two (A is the only O(n^2) traffic: the kernels
@@ -48,9 +48,12 @@ template <bool ROW, bool COL, bool UPD, int V>
 __global__ void __launch_bounds__(LD_THREADS) lowdim_kernel(const LowdimArgs p) {
     __shared__ float colred[LD_THREADS / 32][32 * V * LD_MAXG];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
-    const int64_t i0 = (int64_t)blockIdx.y * p.Ti, j0 = (int64_t)blockIdx.x * p.Tj;
-    const int64_t i1 = min(i0 + (int64_t)p.Ti, p.nx), j1 = min(j0 + (int64_t)p.Tj, p.ny);
-    if (i0 >= i1 || j0 >= j1) return;
+    // a CTA executes the tiles (ti, tj = blockIdx.x) for ti = blockIdx.y, + gridDim.y, ... one after
+    // the other (each tile whole, by this CTA), carrying its column partial sums across them, so a
+    // column costs one atomic per CTA instead of one per row tile
+    const int64_t j0 = (int64_t)blockIdx.x * p.Tj, j1 = min(j0 + (int64_t)p.Tj, p.ny);
+    const int64_t ntile_i = (p.nx + p.Ti - 1) / p.Ti;
+    if (j0 >= j1 || (int64_t)blockIdx.y >= ntile_i) return;
     const int ng = (int)((j1 - j0 + 32 * V - 1) / (32 * V));  // column groups per lane (<= LD_MAXG)
     float vrr[LD_MAXG][V], v1r[LD_MAXG][V], v2r[LD_MAXG][V], cacc[LD_MAXG][V];
 #pragma unroll
@@ -64,6 +67,8 @@ __global__ void __launch_bounds__(LD_THREADS) lowdim_kernel(const LowdimArgs p) 
             v2r[g][e] = (UPD && ok) ? __ldg(p.v2 + j) : 0.f;
             cacc[g][e] = 0.f;
         }
+    for (int64_t ti = blockIdx.y; ti < ntile_i; ti += gridDim.y) {
+    const int64_t i0 = ti * p.Ti, i1 = min(i0 + (int64_t)p.Ti, p.nx);
     for (int64_t i = i0 + warp; i < i1; i += nw) {
         const float *arow = p.A + i * p.ny;
         const float vci = COL ? __ldg(p.vc + i) : 0.f;
@@ -113,6 +118,7 @@ __global__ void __launch_bounds__(LD_THREADS) lowdim_kernel(const LowdimArgs p) 
             if (lane == 0) atomicAdd(p.rowout + i, p.ar * racc);
         }
     }
+    }
     if constexpr (COL) {  // reduce the column partials of the CTA's warps, one atomic per column
 #pragma unroll
         for (int g = 0; g < LD_MAXG; g++)
@@ -147,8 +153,14 @@ cudaError_t launch_lowdim(const LowdimArgs &a0, bool row, bool col, bool upd, cu
     const int V = v4 ? 4 : 1;
     a.Tj = (int)std::min<int64_t>(a.Tj, (int64_t)LD_MAXG * 32 * V);
     a.Ti = (int)std::min<int64_t>(a.Ti, a.nx);
-    const int64_t gx = (a.ny + a.Tj - 1) / a.Tj, gy = (a.nx + a.Ti - 1) / a.Ti;
-    if (gy > 65535 || gx > INT32_MAX) return cudaErrorInvalidConfiguration;
+    const int64_t gx = (a.ny + a.Tj - 1) / a.Tj, ntile_i = (a.nx + a.Ti - 1) / a.Ti;
+    // enough CTAs to keep every SM streaming (8 per SM), each walking several row tiles
+    int dev = 0, nsm = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    const int64_t gy = std::min<int64_t>(std::min<int64_t>(ntile_i, 65535),
+                                         std::max<int64_t>(1, ((int64_t)nsm * 8 + gx - 1) / gx));
+    if (gx > INT32_MAX) return cudaErrorInvalidConfiguration;
     dim3 grid((unsigned)gx, (unsigned)gy), block(LD_THREADS);
 #define LDK(R, C, U)                                                                   \
     do {                                                                               \

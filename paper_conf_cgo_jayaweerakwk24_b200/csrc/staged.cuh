@@ -61,10 +61,31 @@ __global__ void __launch_bounds__((16384 / (RM * RN)) < 1024 ? (16384 / (RM * RN
 
     const int tx = threadIdx.x, ty = threadIdx.y, BX = blockDim.x;
     const int tid = ty * BX + tx, nthr = BX * blockDim.y;
-    const int64_t i0 = (int64_t)blockIdx.y * p.Ti, j0 = (int64_t)blockIdx.x * p.Tj;
+    // tile of this CTA (Fig. 4 mapping); with a split wave tail (p.sp > 1, 1-D grid) the last
+    // tiles are cut along k into sp parts whose partial sums are added to C atomically
+    const int nk = (int)((p.K + p.Tk - 1) / p.Tk);
+    int64_t tile_i, tile_j;
+    int ks0 = 0, nloc = nk;
+    bool split = false;
+    if (p.sp > 1) {
+        int64_t t = blockIdx.x;
+        if (t >= p.nfull) {
+            const int64_t v = t - p.nfull;
+            const int part = (int)(v % p.sp);
+            t = p.nfull + v / p.sp;
+            ks0 = (int)((int64_t)part * nk / p.sp);
+            nloc = (int)((int64_t)(part + 1) * nk / p.sp) - ks0;
+            split = true;
+        }
+        tile_i = t / p.gx;
+        tile_j = t - tile_i * p.gx;
+    } else {
+        tile_i = blockIdx.y;
+        tile_j = blockIdx.x;
+    }
+    const int64_t i0 = tile_i * p.Ti, j0 = tile_j * p.Tj;
     const int rows = (int)imin64(p.Ti, p.M - i0);
     const int cols = (int)imin64(p.Tj, p.N - j0);
-    const int nk = (int)((p.K + p.Tk - 1) / p.Tk);
 
     if constexpr (BULK) {
         if (tid == 0)
@@ -89,12 +110,12 @@ __global__ void __launch_bounds__((16384 / (RM * RN)) < 1024 ? (16384 / (RM * RN
     const Walk wa = mkwalk(p.Tk);  // A: (row, k), k fastest -> coalesced reads
     const Walk wb = TRANSB ? mkwalk(BT4 ? p.Tk >> 2 : p.Tk) : mkwalk(V == 4 ? cols >> 2 : cols);
 
-    auto stage = [&](int t) {
-        if (t < nk) {
+    auto stage = [&](int t) {  // local stage t = global k-stage ks0 + t, ring slot t % S
+        if (t < nloc) {
             const int s = t % S;
             T *As = sm + s * stage_elems;
             T *Bs = As + p.Tk * aip;
-            const int64_t k0 = (int64_t)t * p.Tk;
+            const int64_t k0 = (int64_t)(ks0 + t) * p.Tk;
             const int kt = (int)imin64(p.Tk, p.K - k0);
             if constexpr (BULK) {
                 if (tid == 0) {
@@ -225,7 +246,7 @@ __global__ void __launch_bounds__((16384 / (RM * RN)) < 1024 ? (16384 / (RM * RN
     };
 
     for (int s = 0; s < S - 1; s++) stage(s);
-    for (int t = 0; t < nk; t++) {
+    for (int t = 0; t < nloc; t++) {
         stage(t + S - 1);
         if (S == 1) cp_async_wait<0>();
         else if (S == 2) cp_async_wait<1>();
@@ -234,7 +255,7 @@ __global__ void __launch_bounds__((16384 / (RM * RN)) < 1024 ? (16384 / (RM * RN
         __syncthreads();
         const T *As = sm + (t % S) * stage_elems;
         const T *Bs = As + p.Tk * aip;
-        const int kt = (int)imin64(p.Tk, p.K - (int64_t)t * p.Tk);
+        const int kt = (int)imin64(p.Tk, p.K - (int64_t)(ks0 + t) * p.Tk);
         int kk = 0;
         if (BT4) {
             for (; kk + 4 <= kt; kk += 4) body4t(As, Bs, kk);
@@ -250,7 +271,25 @@ __global__ void __launch_bounds__((16384 / (RM * RN)) < 1024 ? (16384 / (RM * RN
     }
     cp_async_wait<0>();
 
-    // epilogue: C = (init_zero ? 0 : beta*C) + alpha*acc
+    // epilogue: C = (init_zero ? 0 : beta*C) + alpha*acc; a k-part of a split tile adds alpha*acc to
+    // C, which staged_tail_prepass has already set to (init_zero ? 0 : beta*C)
+    if (split) {
+#pragma unroll
+        for (int r = 0; r < RM; r++) {
+            const int rl = ty * RM + r;
+            if (rl >= rows) continue;
+            T *crow = p.C + (i0 + rl) * p.ldc + j0;
+#pragma unroll
+            for (int c = 0; c < VN; c++) {
+#pragma unroll
+                for (int e = 0; e < V; e++) {
+                    const int cl = (tx + c * BX) * V + e;
+                    if (cl < cols) atomicAdd(crow + cl, p.alpha * acc[r][c * V + e]);
+                }
+            }
+        }
+        return;
+    }
 #pragma unroll
     for (int r = 0; r < RM; r++) {
         const int rl = ty * RM + r;
@@ -275,4 +314,16 @@ __global__ void __launch_bounds__((16384 / (RM * RN)) < 1024 ? (16384 / (RM * RN
             }
         }
     }
+}
+
+// C := init_zero ? 0 : beta*C on the tiles t >= nfull (the split wave tail); one CTA per tile row.
+template <typename T>
+__global__ void staged_tail_prepass(const CArgs<T> p) {
+    const int64_t t = p.nfull + (int64_t)blockIdx.x / p.Ti, r = (int64_t)blockIdx.x % p.Ti;
+    const int64_t ti = t / p.gx, tj = t - ti * p.gx;
+    const int64_t i = ti * p.Ti + r, j0 = tj * p.Tj;
+    if (i >= p.M) return;
+    T *c = p.C + i * p.ldc + j0;
+    const int64_t w = p.N - j0 < p.Tj ? p.N - j0 : p.Tj;
+    for (int64_t x = threadIdx.x; x < w; x += blockDim.x) c[x] = p.init_zero ? T(0) : p.beta * c[x];
 }

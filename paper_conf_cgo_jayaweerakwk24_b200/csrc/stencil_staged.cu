@@ -16,6 +16,7 @@
 
 #include <algorithm>
 #include <cstdint>
+#include <cstdlib>
 
 #include "tc_ptx.cuh"
 
@@ -127,44 +128,27 @@ __global__ void __launch_bounds__(256) jacobi2d_staged(float *__restrict__ dst, 
 // Window: box {Tk+8, Tj+2, Ti+2} at (tk0-4, tj0-1, ti0-1) of the 3-D tensor map over src
 // (out-of-range cells zero-filled by TMA; they are never used by an interior output).
 // A thread owns (j, 16-byte k-group) columns and walks i with planes i-1, i in registers.
-template <bool COVER>
-__global__ void __launch_bounds__(256) heat3d_staged(float *__restrict__ dst, const __grid_constant__ CUtensorMap msrc,
-                                                     int64_t n, int Ti, int Tj, int Tk, int nbj, int32_t *counts) {
-    extern __shared__ __align__(128) unsigned char win_raw[];
-    // TMA destinations must be 128-byte aligned: align the dynamic window by hand
-    float *win = reinterpret_cast<float *>(win_raw + ((128u - (su32(win_raw) & 127u)) & 127u));
-    __shared__ uint64_t bar;
-    const int64_t tk0 = (int64_t)blockIdx.x * Tk;
-    const int64_t ti0 = (int64_t)(blockIdx.y / nbj) * Ti, tj0 = (int64_t)(blockIdx.y % nbj) * Tj;
+// One tile of a heat-3d sweep: tile (bx = k-tile, by = (i-tile, j-tile)); `win` is the CTA's
+// 128-byte-aligned window, `bar` its mbarrier in phase `phase`.  Returns false (no window traffic,
+// barrier untouched) when the tile is empty.  Ends with __syncthreads(): the window may be reused.
+__device__ __forceinline__ bool heat_tile(float *__restrict__ dst, const CUtensorMap *msrc, int64_t n, int Ti,
+                                          int Tj, int Tk, int nbj, int64_t bx, int64_t by, float *win,
+                                          uint64_t *bar, unsigned phase) {
+    const int64_t tk0 = bx * Tk;
+    const int64_t ti0 = (by / nbj) * Ti, tj0 = (by % nbj) * Tj;
     const int64_t ilo = ti0 > 1 ? ti0 : 1, ihi = ti0 + Ti < n - 1 ? ti0 + Ti : n - 1;
     const int64_t jlo = tj0 > 1 ? tj0 : 1, jhi = tj0 + Tj < n - 1 ? tj0 + Tj : n - 1;
     const int64_t klo = tk0 > 1 ? tk0 : 1, khi = tk0 + Tk < n - 1 ? tk0 + Tk : n - 1;
-    if (ilo >= ihi || jlo >= jhi || klo >= khi) return;
+    if (ilo >= ihi || jlo >= jhi || klo >= khi) return false;
     const int KW = Tk + 8, JW = Tj + 2;  // window pitches (elements)
     const int64_t g0 = klo >> 2, g1 = ((khi - 1) >> 2) + 1;
     const int ng = (int)(g1 - g0), nj = (int)(jhi - jlo), ni = (int)(ihi - ilo);
     const int tid = threadIdx.x;
-    if constexpr (COVER) {
-        for (int e = tid; e < nj * ng * ni; e += blockDim.x) {
-            const int gi = e % ng, jj = (e / ng) % nj, ii = e / (ng * nj);
-            for (int q = 0; q < 4; q++) {
-                const int64_t k = 4 * (g0 + gi) + q;
-                if (k >= klo && k < khi) atomicAdd(counts + ((ilo + ii) * n + jlo + jj) * n + k, 1);
-            }
-        }
-        return;
-    }
     if (tid == 0) {
-        mbar_init(&bar, 1);
-        asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
-        asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&msrc)) : "memory");
+        mbar_expect_tx(bar, (unsigned)((Ti + 2) * JW * KW * 4));
+        tcm::tma_3d(win, msrc, (int)(tk0 - 4), (int)(tj0 - 1), (int)(ti0 - 1), bar);
     }
-    __syncthreads();
-    if (tid == 0) {
-        mbar_expect_tx(&bar, (unsigned)((Ti + 2) * JW * KW * 4));
-        tcm::tma_3d(win, &msrc, (int)(tk0 - 4), (int)(tj0 - 1), (int)(ti0 - 1), &bar);
-    }
-    mbar_wait(&bar, 0);
+    mbar_wait(bar, phase);
     const float c = 0.125f, two = 2.0f;
     const int64_t nn = n * n;
     // work items: (i-chunk, j, k-group); i is split when the columns alone do not fill the CTA
@@ -212,6 +196,42 @@ __global__ void __launch_bounds__(256) heat3d_staged(float *__restrict__ dst, co
             x = ip;
         }
     }
+    __syncthreads();
+    return true;
+}
+
+template <bool COVER>
+__global__ void __launch_bounds__(256) heat3d_staged(float *__restrict__ dst, const __grid_constant__ CUtensorMap msrc,
+                                                     int64_t n, int Ti, int Tj, int Tk, int nbj, int32_t *counts) {
+    extern __shared__ __align__(128) unsigned char win_raw[];
+    // TMA destinations must be 128-byte aligned: align the dynamic window by hand
+    float *win = reinterpret_cast<float *>(win_raw + ((128u - (su32(win_raw) & 127u)) & 127u));
+    __shared__ uint64_t bar;
+    if constexpr (COVER) {
+        const int64_t tk0 = (int64_t)blockIdx.x * Tk;
+        const int64_t ti0 = (int64_t)(blockIdx.y / nbj) * Ti, tj0 = (int64_t)(blockIdx.y % nbj) * Tj;
+        const int64_t ilo = ti0 > 1 ? ti0 : 1, ihi = ti0 + Ti < n - 1 ? ti0 + Ti : n - 1;
+        const int64_t jlo = tj0 > 1 ? tj0 : 1, jhi = tj0 + Tj < n - 1 ? tj0 + Tj : n - 1;
+        const int64_t klo = tk0 > 1 ? tk0 : 1, khi = tk0 + Tk < n - 1 ? tk0 + Tk : n - 1;
+        if (ilo >= ihi || jlo >= jhi || klo >= khi) return;
+        const int64_t g0 = klo >> 2, g1 = ((khi - 1) >> 2) + 1;
+        const int ng = (int)(g1 - g0), nj = (int)(jhi - jlo), ni = (int)(ihi - ilo);
+        for (int e = threadIdx.x; e < nj * ng * ni; e += blockDim.x) {
+            const int gi = e % ng, jj = (e / ng) % nj, ii = e / (ng * nj);
+            for (int q = 0; q < 4; q++) {
+                const int64_t k = 4 * (g0 + gi) + q;
+                if (k >= klo && k < khi) atomicAdd(counts + ((ilo + ii) * n + jlo + jj) * n + k, 1);
+            }
+        }
+        return;
+    }
+    if (threadIdx.x == 0) {
+        mbar_init(&bar, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+        asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&msrc)) : "memory");
+    }
+    __syncthreads();
+    heat_tile(dst, &msrc, n, Ti, Tj, Tk, nbj, blockIdx.x, blockIdx.y, win, &bar, 0);
 }
 
 constexpr int kSmemTarget = 113 * 1024;  // at least two resident CTAs per SM

@@ -114,8 +114,13 @@ def test_gemm_full_size_eatss_tile_sampled(cuda_device):
     n = 4000
     d = E.desc_builtin("gemm", (n, n, n))
     tiles, _ = E.select_tiles(d, E.gpu_params_query(0), 50, 16)
+    # 1000 tiles on 2 x 148 resident CTAs: the last wave's tiles are split along k (tail pre-pass +
+    # atomic k-parts), which these samples reach (tail rows >= 3552 get their own 512 samples)
+    d.set_exec(50, 1)
+    assert E.launches_per_run(d, tiles) == 2
     g = synth.rng(7)
-    ii = g.integers(0, n, 2048); jj = g.integers(0, n, 2048)
+    ii = np.concatenate([g.integers(0, n, 2048), g.integers(3552, n, 512)])
+    jj = g.integers(0, n, len(ii))
     # small-int pass: every output must be exact (checked on 2048 sampled entries)
     A = synth.small_int((n, n), 1); B = synth.small_int((n, n), 2); C = synth.small_int((n, n), 3)
     d.set_scalars(1.0, 1.0)
