@@ -58,6 +58,9 @@ def parse():
     ap.add_argument("--warmup", type=int, default=2)
     ap.add_argument("--device", type=int, default=0)
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "candidates.jsonl"))
+    ap.add_argument("--confirm", type=int, default=5,
+                    help="when the PPW-best and the fastest candidate differ, re-measure both this many "
+                         "times, interleaved, and report mean and 95%% interval of the PPW (0 = off)")
     return ap.parse_args()
 
 
@@ -82,6 +85,28 @@ def measure(E, d, tiles, split, bufs, a):
     m = E.sweep(d, [tiles], bufs, device=a.device, warmup=a.warmup, min_window_s=a.window)[0]
     return dict(ms=m.ms_per_run, joules=m.joules_per_run, watts=m.avg_watts, tflops=m.tflops,
                 ppw=m.gflops_per_watt, sm_mhz=m.sm_mhz_median, status=m.status)
+
+
+def confirm(E, d, bufs, a, cands):
+    """Interleaved repeats of the given candidates (DVFS / thermal drift hits both alike)."""
+    import numpy as np
+
+    ppw = {i: [] for i in range(len(cands))}
+    tf = {i: [] for i in range(len(cands))}
+    for _ in range(a.confirm):
+        for i, c in enumerate(cands):
+            r = measure(E, d, tuple(c["tiles"]), c["split"], bufs, a)
+            if r["status"] == 0 and r["ppw"] > 0:
+                ppw[i].append(r["ppw"]); tf[i].append(r["tflops"])
+    out = []
+    for i, c in enumerate(cands):
+        x = np.array(ppw[i]); t = np.array(tf[i])
+        half = 1.96 * x.std(ddof=1) / np.sqrt(len(x)) if len(x) > 1 else float("nan")
+        out.append(dict(tiles=c["tiles"], split=c["split"], role="ppw-best" if i == 0 else "fastest",
+                        ppw_mean=float(x.mean()) if len(x) else None, ppw_ci95=[float(x.mean() - half), float(x.mean() + half)]
+                        if len(x) > 1 else None, tflops_mean=float(t.mean()) if len(t) else None, n=len(x)))
+    lo0, hi1 = (out[0]["ppw_ci95"] or [None])[0], (out[1]["ppw_ci95"] or [None, None])[1]
+    return dict(repeats=out, ppw_best_separated=(lo0 is not None and hi1 is not None and lo0 > hi1))
 
 
 def main():
@@ -129,6 +154,10 @@ def main():
                     ppw_gain_vs_default=be["ppw"] / bd["ppw"] if bd else None,
                     ppw_spread_over_candidates=be["ppw"] / min(r["ppw"] for r in ea),
                     n_candidates=len(ea), infeasible=infeasible)
+            if ea and a.confirm > 0:
+                be = max(ea, key=lambda r: r["ppw"]); pe = max(ea, key=lambda r: r["tflops"])
+                if (be["tiles"], be["split"]) != (pe["tiles"], pe["split"]):
+                    summary[kind]["confirm"] = confirm(E, d, bufs, a, [be, pe])
             print(kind, json.dumps(summary.get(kind)), flush=True)
             del bufs
             torch.cuda.empty_cache()

@@ -252,6 +252,20 @@ def test_heat3d(cuda_device, n, tiles, T):
     assert O.normwise_rel_err(host(Ad), Ar) <= TOL32 and O.normwise_rel_err(host(Bd), Br) <= TOL32
 
 
+@pytest.mark.parametrize("kind,n,T", [("jacobi-2d", 4000, 500), ("heat-3d", 120, 500)])
+def test_stencil_baseline_config_full(cuda_device, kind, n, T):
+    """BASELINE config 4 at full size and full time-step count, with the model-selected tile (the
+    tile bench.py times), random U[-1,1) fields, every output element compared."""
+    d = E.desc_builtin(kind, (n,), tsteps=T)
+    tiles, _ = E.select_tiles(d, E.gpu_params_query(0), 50, 16)
+    shape = (n, n) if kind == "jacobi-2d" else (n, n, n)
+    A = synth.uniform(shape, 95); B = synth.uniform(shape, 96)
+    Ar, Br = (O.jacobi2d if kind == "jacobi-2d" else O.heat3d)(A, B, T)
+    Ad, Bd = dev(A), dev(B)
+    run(d, tiles, [Ad, Bd])
+    assert O.normwise_rel_err(host(Ad), Ar) <= TOL32 and O.normwise_rel_err(host(Bd), Br) <= TOL32
+
+
 def test_heat3d_linear_field_exact(cuda_device):
     n = 120
     A = synth.linear_field((n, n, n), (2, -3, 1), 5)
