@@ -568,8 +568,29 @@ def gemver(n=4000, dtype_bytes=4) -> Program:
     return P("gemver", [n1, n2, n3, n4], dtype_bytes)
 
 
+# Non-PolyBench 4-D kernels (Figs. 10-11): our restatement
+# (reading R-N8, R-N9).  Reduction loops are not parallel.
+def mttkrp(ni=512, nj=32, nk=512, nl=512, dtype_bytes=4) -> Program:
+    """A[i][j] += B[i][k][l] * C[k][j] * D[l][j]  (mode-1 MTTKRP, loops i, j, k, l)."""
+    return P("mttkrp", [Nest(
+        [Loop("i", ni, True), Loop("j", nj, True), Loop("k", nk, False), Loop("l", nl, False)],
+        [ref("A", "i", "j", write=True), ref("A", "i", "j"), ref("B", "i", "k", "l"),
+         ref("C", "k", "j"), ref("D", "l", "j")],
+    )], dtype_bytes)
+
+
+def conv2d(n=8192, f=5, dtype_bytes=4) -> Program:
+    """out[i][j] += inp[i+p][j+q] * W[p][q]  (valid 2-D cross-correlation, loops i, j, p, q)."""
+    m = n - f + 1
+    return P("conv-2d", [Nest(
+        [Loop("i", m, True), Loop("j", m, True), Loop("p", f, False), Loop("q", f, False)],
+        [ref("out", "i", "j", write=True), ref("out", "i", "j"), ref("inp", "i+p", "j+q"), ref("W", "p", "q")],
+    )], dtype_bytes)
+
+
 BUILTINS = {
     "gemm": gemm, "2mm": two_mm, "3mm": three_mm, "syrk": syrk,
     "jacobi-2d": jacobi2d, "heat-3d": heat3d, "ccsd_t_d1": ccsd_t_d1,
     "mvt": mvt, "atax": atax, "bicg": bicg, "gemver": gemver,
+    "mttkrp": mttkrp, "conv-2d": conv2d,
 }

@@ -60,11 +60,14 @@ def _declare(L):
     L.oracle_atax.argtypes = [_I, _I, _P, _P, _P, _P]
     L.oracle_bicg.argtypes = [_I, _I, _P, _P, _P, _P, _P]
     L.oracle_gemver.argtypes = [_I, _D, _D, _P, _P, _P, _P, _P, _P, _P, _P, _P]
+    L.oracle_mttkrp.argtypes = [_I, _I, _I, _I, _P, _P, _P, _P]
+    L.oracle_mttkrp_entries.argtypes = [_I, _P, _P, _P, _I, _I, _I, _P, _P, _P, _P]
+    L.oracle_conv2d.argtypes = [_I, _I, _P, _P, _P]
     L.oracle_num_threads.restype = ctypes.c_int
     for f in ("oracle_gemm", "oracle_gemm_ijk", "oracle_gemm_entries", "oracle_2mm",
               "oracle_3mm", "oracle_syrk", "oracle_jacobi2d", "oracle_heat3d",
               "oracle_ccsd_t_d1", "oracle_ccsd_t_d1_entries", "oracle_mvt", "oracle_atax", "oracle_bicg",
-              "oracle_gemver"):
+              "oracle_gemver", "oracle_mttkrp", "oracle_mttkrp_entries", "oracle_conv2d"):
         getattr(L, f).restype = None
 
 
@@ -206,6 +209,35 @@ def gemver(alpha, beta, A, x, w, u1, v1, u2, v2, y, z):
     lib().oracle_gemver(n, float(alpha), float(beta), _p(A), _p(x), _p(w), _p(_f64(u1)), _p(_f64(v1)),
                         _p(_f64(u2)), _p(_f64(v2)), _p(_f64(y)), _p(_f64(z)))
     return A, x, w
+
+
+def mttkrp(A, B, C, D):
+    """A[i][j] += sum_k sum_l B[i][k][l]*C[k][j]*D[l][j] (reading R-N8). Returns the new A."""
+    A = _f64(A).copy(); B = _f64(B); C = _f64(C); D = _f64(D)
+    ni, nk, nl = B.shape; nj = A.shape[1]
+    assert A.shape == (ni, nj) and C.shape == (nk, nj) and D.shape == (nl, nj)
+    lib().oracle_mttkrp(ni, nj, nk, nl, _p(A), _p(B), _p(C), _p(D))
+    return A
+
+
+def mttkrp_entries(ii, jj, A0, B, C, D) -> np.ndarray:
+    """Sampled mttkrp outputs at (ii[s], jj[s]) (full-size parity)."""
+    ii = _i64(ii); jj = _i64(jj); B = _f64(B); C = _f64(C); D = _f64(D)
+    a0 = _f64(np.asarray(A0)[ii, jj])
+    ni, nk, nl = B.shape; nj = C.shape[1]
+    out = np.empty(len(ii), dtype=np.float64)
+    lib().oracle_mttkrp_entries(len(ii), _p(ii), _p(jj), _p(a0), nj, nk, nl, _p(B), _p(C), _p(D), _p(out))
+    return out
+
+
+def conv2d(inp, W) -> np.ndarray:
+    """Valid 2-D cross-correlation out[i][j] = sum_p sum_q inp[i+p][j+q]*W[p][q] (reading R-N9)."""
+    inp = _f64(inp); W = _f64(W)
+    n = inp.shape[0]; f = W.shape[0]
+    assert inp.shape == (n, n) and W.shape == (f, f) and f <= n
+    out = np.empty((n - f + 1, n - f + 1), dtype=np.float64)
+    lib().oracle_conv2d(n, f, _p(out), _p(inp), _p(W))
+    return out
 
 
 def normwise_rel_err(x, ref) -> float:

@@ -308,6 +308,62 @@ void oracle_gemver(int64_t n, double alpha, double beta, double *A, double *x, d
         for (int64_t j = 0; j < n; j++) w[i] = w[i] + alpha * A[IDX2(i, j, n)] * x[j];
 }
 
+/* ------------------------------------------- non-PolyBench 4-D kernels --- */
+/* the paper's non-PolyBench kernels mttkrp and convolution-2d (PAPER.md:191,
+ * :272-284, Figs. 10-11, Fig. 13).  The paper prints neither body nor size; it states they are 4-D
+ * loop nests ("higher loop dimensionality (4D)", Fig. 10 note on depth > 3).  The
+ * bodies below are OUR restatement (readings R-N8, R-N9), literal loop order,
+ * float64, the statement evaluated left to right as written.                                     */
+
+/* mttkrp (mode-1 matricized tensor times Khatri-Rao product):
+ *   for i < ni, j < nj, k < nk, l < nl:  A[i][j] = A[i][j] + B[i][k][l] * C[k][j] * D[l][j]
+ * A: ni x nj (in/out), B: ni x nk x nl, C: nk x nj, D: nl x nj, row-major.                      */
+void oracle_mttkrp(int64_t ni, int64_t nj, int64_t nk, int64_t nl, double *A, const double *B,
+                   const double *C, const double *D)
+{
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < ni; i++)
+        for (int64_t j = 0; j < nj; j++) {
+            double a = A[IDX2(i, j, nj)];
+            for (int64_t k = 0; k < nk; k++)
+                for (int64_t l = 0; l < nl; l++)
+                    a = a + B[(i * nk + k) * nl + l] * C[IDX2(k, j, nj)] * D[IDX2(l, j, nj)];
+            A[IDX2(i, j, nj)] = a;
+        }
+}
+
+/* Sampled mttkrp outputs (full-size parity): out[s] = A0[s] + the sum above at (ii[s], jj[s]). */
+void oracle_mttkrp_entries(int64_t n, const int64_t *ii, const int64_t *jj, const double *a0, int64_t nj,
+                           int64_t nk, int64_t nl, const double *B, const double *C, const double *D, double *out)
+{
+#pragma omp parallel for schedule(static)
+    for (int64_t s = 0; s < n; s++) {
+        const int64_t i = ii[s], j = jj[s];
+        double a = a0[s];
+        for (int64_t k = 0; k < nk; k++)
+            for (int64_t l = 0; l < nl; l++)
+                a = a + B[(i * nk + k) * nl + l] * C[IDX2(k, j, nj)] * D[IDX2(l, j, nj)];
+        out[s] = a;
+    }
+}
+
+/* convolution-2d ("valid" cross-correlation of an n x n image with an f x f filter):
+ *   for i < n-f+1, j < n-f+1:  out[i][j] = 0;
+ *                              for p < f, q < f:  out[i][j] = out[i][j] + inp[i+p][j+q] * W[p][q]
+ * out: (n-f+1) x (n-f+1) (out), inp: n x n, W: f x f, row-major.                                 */
+void oracle_conv2d(int64_t n, int64_t f, double *out, const double *inp, const double *W)
+{
+    const int64_t m = n - f + 1;
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < m; i++)
+        for (int64_t j = 0; j < m; j++) {
+            double o = 0.0;
+            for (int64_t p = 0; p < f; p++)
+                for (int64_t q = 0; q < f; q++) o = o + inp[IDX2(i + p, j + q, n)] * W[IDX2(p, q, f)];
+            out[IDX2(i, j, m)] = o;
+        }
+}
+
 /* Number of OpenMP threads the oracle uses (reported as cpu_baseline.cores). */
 #ifdef _OPENMP
 #include <omp.h>

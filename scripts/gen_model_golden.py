@@ -60,6 +60,16 @@ for kern, dims in (("mvt", (4000,)), ("atax", (4000, 4000)), ("bicg", (4000, 400
     for split, waf in ((50, 16), (0, 4), (100, 32)):
         add(kern, dims, 4, "B200", split, waf, 1)
 add("gemver", (4000,), 8, "GA100", 50, 16, 0)
+# non-PolyBench 4-D kernels (readings R-N8, R-N9): B200 at the config sizes,
+# GA100 paper mode over the P:282 space (warp_frac x shared-memory quota)
+for waf in (4, 8, 16, 32):
+    add("mttkrp", (512, 32, 512, 512), 4, "B200", 50, waf, 1)
+    add("conv-2d", (8192, 5), 4, "B200", 50, waf, 1)
+    for split in (0, 50, 100):
+        add("mttkrp", (512, 32, 512, 512), 4, "GA100", split, waf, 0)
+        add("conv-2d", (8192, 5), 4, "GA100", split, waf, 0)
+add("mttkrp", (60, 20, 36, 44), 4, "B200", 0, 4, 1)
+add("conv-2d", (514, 3), 4, "B200", 100, 8, 1)
 
 
 def main():

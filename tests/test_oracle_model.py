@@ -159,3 +159,52 @@ def test_tensor_mode_hand_checked():
     assert r.n_feasible == 8 and r.n_ties == 1 and r.tiles == (128, 256, 32) and r.obj == 160 * 256
     assert M.select_tiles(M.gemm(), M.GA100, M.Opts(50, 16, 2)).tiles is None
     assert M.select_tiles(M.heat3d(), M.B200, M.Opts(50, 16, 2)).tiles is None  # not a contraction
+
+
+def _p282_space(prog):
+    feas = {}
+    for wf in (0.125, 0.25, 0.5, 1.0):
+        for split in (0, 50, 100):
+            r = M.select_tiles(prog, M.GA100, M.Opts(split, int(wf * 32), 0), keep_ties=False)
+            feas[(wf, split)] = r.tiles is not None
+    return feas
+
+
+@pytest.mark.parametrize("prog", [
+    M.mttkrp(512, 32, 512, 512), M.mttkrp(256, 64, 256, 256), M.mttkrp(64, 32, 64, 64),
+    M.conv2d(8192, 5), M.conv2d(1024, 5), M.conv2d(2048, 6),
+], ids=["mttkrp512", "mttkrp256", "mttkrp64", "conv8192f5", "conv1024f5", "conv2048f6"])
+def test_mttkrp_conv2d_feasible_configurations_on_ga100(prog):
+    """11 of the 12 (warp_frac x shared quota) configurations are feasible for conv-2d and
+    mttkrp; the missing one is warp_frac 1.0 with 50% shared memory.  Under reading R with fp32
+    elements this holds for mttkrp at every size >= 32 per loop; for conv-2d it fixes the filter at
+    5x5 or 6x6 (3x3 and 4x4 leave all 12 feasible, 7x7 loses warp_frac 1.0 at 0% too) -- a reading
+    chosen to agree with P:282, recorded in DESIGN.md §2.7 (R-N9), not an independent pin."""
+    f = _load("paper_facts.json")["mttkrp_conv2d_feasible_configs"]
+    feas = _p282_space(prog)
+    assert sum(feas.values()) == f["value"]
+    assert [k for k, v in feas.items() if not v] == [(x["warp_frac"], x["shared_pct"]) for x in f["infeasible"]]
+
+
+def test_mttkrp_count_depends_on_element_size():
+    """With fp64 elements (reading Q3's precision of the PolyBench runs) mttkrp loses every
+    warp_frac 1.0 configuration (9/12), so P:282's 11/12 is evidence the non-PolyBench kernels ran
+    in fp32; heat-3d's 9/12 holds for both element sizes."""
+    feas = _p282_space(M.mttkrp(512, 32, 512, 512, dtype_bytes=8))
+    assert sum(feas.values()) == 9
+    for e in (4, 8):
+        assert sum(_p282_space(M.heat3d(120, e)).values()) == 9
+
+
+def test_mttkrp_conv2d_derivation():
+    """Rules 2-8 on the 4-D nests: mttkrp groups {A(i;j), B(i,k;l), C(k;j), D(l;j)} -> nrefs 4,
+    cnt(j) = 3 -> l_s1 = j, SH = {B} with footprint Ti*Tk*Tl; conv-2d groups {out(i;j),
+    inp(i+p;j+q), W(p;q)} -> nrefs 3, cnt(j) = cnt(q) = 2, l_s1 = j (parallel), SH = {W}."""
+    d = M.derive(M.mttkrp().nests[0], 16)
+    assert (d.ls1, d.nrefs, d.bset) == ("j", 4, ["j", "i"])
+    assert d.H == {"i": 0, "j": 48, "k": 0, "l": 0}
+    assert d.sh_fp == [frozenset("ikl")]
+    c = M.derive(M.conv2d().nests[0], 16)
+    assert (c.ls1, c.nrefs, c.bset) == ("j", 3, ["j", "i"])
+    assert c.H == {"i": 0, "j": 32, "p": 0, "q": 0}
+    assert c.sh_fp == [frozenset("pq")] and frozenset("ijpq") in c.l1_fp

@@ -236,3 +236,86 @@ def test_gemver_closed_form_on_integers():
     assert np.array_equal(An, Ap)
     assert np.array_equal(xn, xp)
     assert np.array_equal(wn, w + alpha * (Ap @ xp))   # w uses the UPDATED x (nest order)
+
+
+# ------------------------------------------------------------------ mttkrp (reading R-N8)
+def _khatri_rao(C, D):
+    """Column-wise Kronecker product: row k*L + l, column j = C[k][j] * D[l][j] (textbook definition)."""
+    K, J = C.shape
+    L = D.shape[0]
+    return (C[:, None, :] * D[None, :, :]).reshape(K * L, J)
+
+
+def test_mttkrp_equals_unfolding_times_khatri_rao_on_integers():
+    """MTTKRP's textbook closed form A + B_(1) (C ⊙ D) with the mode-1 unfolding B_(1) (I x KL):
+    a swapped C/D, a transposed factor or a wrong unfolding order fails (K != L != J)."""
+    I, J, K, L = 7, 5, 6, 4
+    A0, B, C, D = _ints((I, J), 1), _ints((I, K, L), 2), _ints((K, J), 3), _ints((L, J), 4)
+    got = O.mttkrp(A0, B, C, D)
+    want = A0 + B.reshape(I, K * L) @ _khatri_rao(C, D)
+    assert np.array_equal(got, want)
+    swapped = A0 + B.reshape(I, K * L) @ _khatri_rao(np.zeros((K, J)) + C[:, ::-1], D)
+    assert not np.array_equal(got, swapped)
+
+
+def test_mttkrp_rank1_tensor_closed_form():
+    """B = a ∘ b ∘ c (rank 1): A[i][j] = A0[i][j] + a_i (b . C[:, j]) (c . D[:, j]), exact on integers."""
+    I, J, K, L = 9, 6, 8, 5
+    a, b, c = _ints(I, 5), _ints(K, 6), _ints(L, 7)
+    B = a[:, None, None] * b[None, :, None] * c[None, None, :]
+    A0, C, D = _ints((I, J), 8), _ints((K, J), 9), _ints((L, J), 10)
+    got = O.mttkrp(A0, B, C, D)
+    assert np.array_equal(got, A0 + np.outer(a, (b @ C) * (c @ D)))
+
+
+def test_mttkrp_brute_force_tiny_and_entries():
+    I, J, K, L = 3, 4, 2, 3
+    A0, B, C, D = (synth.uniform(s, seed) for s, seed in (((I, J), 1), ((I, K, L), 2), ((K, J), 3), ((L, J), 4)))
+    want = A0.astype(np.float64).copy()
+    for i in range(I):
+        for j in range(J):
+            for k in range(K):
+                for l in range(L):
+                    want[i, j] = want[i, j] + float(B[i, k, l]) * float(C[k, j]) * float(D[l, j])
+    got = O.mttkrp(A0, B, C, D)
+    assert np.array_equal(got, want)  # same operation order as written: bit-identical
+    ii, jj = np.array([0, 2, 1]), np.array([3, 0, 1])
+    assert np.array_equal(O.mttkrp_entries(ii, jj, A0, B, C, D), got[ii, jj])
+
+
+# ------------------------------------------------------------------ conv-2d (reading R-N9)
+def test_conv2d_matches_scipy_valid_correlation():
+    """scipy.signal.correlate2d(mode='valid') is the textbook definition; a flipped filter
+    (true convolution) or a transposed index fails on a non-symmetric filter."""
+    inp = synth.uniform((23, 23), 3).astype(np.float64)
+    W = synth.uniform((5, 5), 4).astype(np.float64)
+    got = O.conv2d(inp, W)
+    assert got.shape == (19, 19)
+    np.testing.assert_allclose(got, signal.correlate2d(inp, W, mode="valid"), rtol=0, atol=1e-13)
+    assert not np.allclose(got, signal.convolve2d(inp, W, mode="valid"))
+
+
+def test_conv2d_delta_filter_is_an_exact_shift():
+    inp = _ints((12, 12), 11)
+    for p0, q0 in ((0, 0), (2, 1), (1, 3)):
+        W = np.zeros((4, 4))
+        W[p0, q0] = 1.0
+        assert np.array_equal(O.conv2d(inp, W), inp[p0:p0 + 9, q0:q0 + 9])
+
+
+def test_conv2d_linear_field_closed_form():
+    """inp = a*i + b*j + d: out[i][j] = (a*i + b*j + d)*sum(W) + a*sum_p p*W[p,:] + b*sum_q q*W[:,q]."""
+    n, f, a, b, d = 17, 3, 3.0, -2.0, 5.0
+    i, j = np.meshgrid(np.arange(n), np.arange(n), indexing="ij")
+    inp = a * i + b * j + d
+    W = _ints((f, f), 12)
+    m = n - f + 1
+    ii, jj = np.meshgrid(np.arange(m), np.arange(m), indexing="ij")
+    p = np.arange(f)
+    want = (a * ii + b * jj + d) * W.sum() + a * (p @ W.sum(axis=1)) + b * (p @ W.sum(axis=0))
+    assert np.array_equal(O.conv2d(inp, W), want)
+
+
+def test_conv2d_filter_equal_to_image_is_one_dot_product():
+    inp, W = _ints((6, 6), 13), _ints((6, 6), 14)
+    assert np.array_equal(O.conv2d(inp, W), np.array([[float((inp * W).sum())]]))
