@@ -91,9 +91,16 @@ typedef enum { EATSS_F32 = 1, EATSS_F64 = 2 } eatss_dtype;
  *   EATSS_GEMVER    dims (n)                   buffers {A[n][n] (in/out), x (in/out), w (in/out),
  *                                                       u1, v1, u2, v2, y, z} (vectors of n)
  *                   A += u1 v1^T + u2 v2^T;  x += beta A^T y;  x += z;  w += alpha A x
+ * Non-PolyBench 4-D kernels (Figs. 10-11, 13), fp32; bodies and
+ * sizes are our restatement (readings R-N8, R-N9):
+ *   EATSS_MTTKRP    dims (ni, nj, nk, nl)      buffers {A[ni][nj] (in/out), B[ni][nk][nl], C[nk][nj], D[nl][nj]}
+ *                   A[i][j] += sum_k sum_l B[i][k][l]*C[k][j]*D[l][j]  (mode-1 MTTKRP, loops i, j, k, l)
+ *   EATSS_CONV2D    dims (n, f)                buffers {out[m][m] (out), inp[n][n], W[f][f]}, m = n - f + 1
+ *                   out[i][j] = sum_p sum_q inp[i+p][j+q]*W[p][q]  (valid cross-correlation, loops i, j, p, q)
  * The tile vector has one entry per loop depth position (reading Q15): 3 for the
  * gemm family, 2 for jacobi-2d and the low-dimensional kernels, 3 for heat-3d, 7 for ccsd_t_d1
- * (h3,h2,h1,p6,p5,p4,h7).  Stencil time loops are not tiled.
+ * (h3,h2,h1,p6,p5,p4,h7), 4 for mttkrp (i,j,k,l) and conv-2d (i,j,p,q).  Stencil time loops are not
+ * tiled.
  */
 typedef enum {
     EATSS_GEMM = 0,
@@ -106,7 +113,9 @@ typedef enum {
     EATSS_MVT = 7,
     EATSS_ATAX = 8,
     EATSS_BICG = 9,
-    EATSS_GEMVER = 10
+    EATSS_GEMVER = 10,
+    EATSS_MTTKRP = 11,
+    EATSS_CONV2D = 12
 } eatss_builtin;
 
 /* GPU parameters of the model: Table I + SM count + the

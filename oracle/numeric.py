@@ -62,7 +62,7 @@ def _declare(L):
     L.oracle_gemver.argtypes = [_I, _D, _D, _P, _P, _P, _P, _P, _P, _P, _P, _P]
     L.oracle_mttkrp.argtypes = [_I, _I, _I, _I, _P, _P, _P, _P]
     L.oracle_mttkrp_entries.argtypes = [_I, _P, _P, _P, _I, _I, _I, _P, _P, _P, _P]
-    L.oracle_conv2d.argtypes = [_I, _I, _P, _P, _P]
+    L.oracle_conv2d.argtypes = [_I, _I, _I, _P, _P, _P]
     L.oracle_num_threads.restype = ctypes.c_int
     for f in ("oracle_gemm", "oracle_gemm_ijk", "oracle_gemm_entries", "oracle_2mm",
               "oracle_3mm", "oracle_syrk", "oracle_jacobi2d", "oracle_heat3d",
@@ -231,12 +231,13 @@ def mttkrp_entries(ii, jj, A0, B, C, D) -> np.ndarray:
 
 
 def conv2d(inp, W) -> np.ndarray:
-    """Valid 2-D cross-correlation out[i][j] = sum_p sum_q inp[i+p][j+q]*W[p][q] (reading R-N9)."""
+    """Valid 2-D cross-correlation out[i][j] = sum_p sum_q inp[i+p][j+q]*W[p][q] (reading R-N9);
+    inp may be rectangular (row bands of a full-size check)."""
     inp = _f64(inp); W = _f64(W)
-    n = inp.shape[0]; f = W.shape[0]
-    assert inp.shape == (n, n) and W.shape == (f, f) and f <= n
-    out = np.empty((n - f + 1, n - f + 1), dtype=np.float64)
-    lib().oracle_conv2d(n, f, _p(out), _p(inp), _p(W))
+    nr, nc = inp.shape; f = W.shape[0]
+    assert W.shape == (f, f) and f <= min(nr, nc)
+    out = np.empty((nr - f + 1, nc - f + 1), dtype=np.float64)
+    lib().oracle_conv2d(nr, nc, f, _p(out), _p(inp), _p(W))
     return out
 
 

@@ -347,20 +347,21 @@ void oracle_mttkrp_entries(int64_t n, const int64_t *ii, const int64_t *jj, cons
     }
 }
 
-/* convolution-2d ("valid" cross-correlation of an n x n image with an f x f filter):
- *   for i < n-f+1, j < n-f+1:  out[i][j] = 0;
- *                              for p < f, q < f:  out[i][j] = out[i][j] + inp[i+p][j+q] * W[p][q]
- * out: (n-f+1) x (n-f+1) (out), inp: n x n, W: f x f, row-major.                                 */
-void oracle_conv2d(int64_t n, int64_t f, double *out, const double *inp, const double *W)
+/* convolution-2d ("valid" cross-correlation of an nr x nc image with an f x f filter):
+ *   for i < nr-f+1, j < nc-f+1:  out[i][j] = 0;
+ *                                for p < f, q < f:  out[i][j] = out[i][j] + inp[i+p][j+q] * W[p][q]
+ * out: (nr-f+1) x (nc-f+1) (out), inp: nr x nc, W: f x f, row-major.  The builtin is square
+ * (nr = nc = n); a rectangular inp serves row bands of a full-size check.                         */
+void oracle_conv2d(int64_t nr, int64_t nc, int64_t f, double *out, const double *inp, const double *W)
 {
-    const int64_t m = n - f + 1;
+    const int64_t mr = nr - f + 1, mc = nc - f + 1;
 #pragma omp parallel for schedule(static)
-    for (int64_t i = 0; i < m; i++)
-        for (int64_t j = 0; j < m; j++) {
+    for (int64_t i = 0; i < mr; i++)
+        for (int64_t j = 0; j < mc; j++) {
             double o = 0.0;
             for (int64_t p = 0; p < f; p++)
-                for (int64_t q = 0; q < f; q++) o = o + inp[IDX2(i + p, j + q, n)] * W[IDX2(p, q, f)];
-            out[IDX2(i, j, m)] = o;
+                for (int64_t q = 0; q < f; q++) o = o + inp[IDX2(i + p, j + q, nc)] * W[IDX2(p, q, f)];
+            out[IDX2(i, j, mc)] = o;
         }
 }
 

@@ -59,6 +59,16 @@ cudaError_t launch_lowdim(const LowdimArgs &a, bool row, bool col, bool upd, cud
 cudaError_t launch_lowdim_axpy(float *out, const float *add, float scale, int64_t n, cudaStream_t s,
                                int64_t *launched);
 
+// mttkrp.cu / conv2d.cu entry points (non-PolyBench 4-D kernels)
+bool mttkrp_plan(const int64_t *dims, const int64_t *tiles, int64_t *gx, int64_t *gy, int64_t *gz, int *bx, int *by,
+                 int *rm, int *smem, int *splits, int *sw_out = nullptr, int *ks_out = nullptr);
+cudaError_t launch_mttkrp(float *A, const float *B, const float *C, const float *D, const int64_t *dims,
+                          const int64_t *tiles, float *ws, int32_t *counts, cudaStream_t s, int64_t *launched);
+bool conv2d_plan(int64_t n, int64_t f, const int64_t *tiles, int64_t *gx, int64_t *gy, int *threads, int *smem,
+                 int *rc, int *wc, int *groups, int *segs);
+cudaError_t launch_conv2d(float *out, const float *inp, const float *W, int64_t n, int64_t f, const int64_t *tiles,
+                          int32_t *counts, cudaStream_t s, int64_t *launched);
+
 // ------------------------------------------------------------------ builtin nests
 // Loop positions are bits: the model only needs which loops a subscript uses.
 static Sub S(uint32_t iters, int off = 0) {
@@ -203,6 +213,27 @@ static eatss_status build(eatss_kernel_desc *d) {
             d->buffer_elems = {n * n, n, n, n, n, n, n, n, n};
             break;
         }
+        // non-PolyBench 4-D kernels (readings R-N8, R-N9): reduction loops serial
+        case EATSS_MTTKRP: {  // A B C D ; dims (ni, nj, nk, nl) ; loops i j k l
+            Nest n;
+            n.loops = {{x[0], true}, {x[1], true}, {x[2], false}, {x[3], false}};
+            const uint32_t i = 1, j = 2, k = 4, l = 8;
+            n.refs = {R(0, {S(i), S(j)}, true), R(0, {S(i), S(j)}), R(1, {S(i), S(k), S(l)}), R(2, {S(k), S(j)}),
+                      R(3, {S(l), S(j)})};
+            d->nests = {n};
+            d->buffer_elems = {x[0] * x[1], x[0] * x[2] * x[3], x[2] * x[1], x[3] * x[1]};
+            break;
+        }
+        case EATSS_CONV2D: {  // out inp W ; dims (n, f) ; loops i j p q over out[m][m], m = n - f + 1
+            const int64_t m = x[0] - x[1] + 1;
+            Nest n;
+            n.loops = {{m, true}, {m, true}, {x[1], false}, {x[1], false}};
+            const uint32_t i = 1, j = 2, p = 4, q = 8;
+            n.refs = {R(0, {S(i), S(j)}, true), R(0, {S(i), S(j)}), R(1, {S(i | p), S(j | q)}), R(2, {S(p), S(q)})};
+            d->nests = {n};
+            d->buffer_elems = {m * m, x[0] * x[0], x[1] * x[1]};
+            break;
+        }
         default:
             return fail(EATSS_E_INVALID, "eatss_desc_builtin: unknown builtin");
     }
@@ -210,7 +241,7 @@ static eatss_status build(eatss_kernel_desc *d) {
     return EATSS_OK;
 }
 
-static const int kDimsPerBuiltin[] = {3, 4, 5, 2, 1, 1, 7, 1, 2, 2, 1};
+static const int kDimsPerBuiltin[] = {3, 4, 5, 2, 1, 1, 7, 1, 2, 2, 1, 4, 2};
 
 static bool is_lowdim(eatss_builtin k) {
     return k == EATSS_MVT || k == EATSS_ATAX || k == EATSS_BICG || k == EATSS_GEMVER;
@@ -364,6 +395,7 @@ eatss_kernel_desc::~eatss_kernel_desc() {
     for (void *e : hev) cudaEventDestroy((cudaEvent_t)e);
     for (void *st : hstream)
         if (st) cudaStreamDestroy((cudaStream_t)st);
+    if (ws) cudaFree(ws);
 }
 
 // exec.time_kernels: a {start, stop} event pair per nest on the current device (nullptr if off)
@@ -394,7 +426,7 @@ eatss_status eatss_desc_builtin(eatss_builtin k, const int64_t *dims, int ndims,
                                 int64_t tsteps, eatss_kernel_desc **out) {
     if (!out) return fail(EATSS_E_INVALID, "eatss_desc_builtin: out is null");
     *out = nullptr;
-    if ((int)k < 0 || (int)k > (int)EATSS_GEMVER) return fail(EATSS_E_INVALID, "eatss_desc_builtin: bad builtin");
+    if ((int)k < 0 || (int)k > (int)EATSS_CONV2D) return fail(EATSS_E_INVALID, "eatss_desc_builtin: bad builtin");
     if (dt != EATSS_F32 && dt != EATSS_F64) return fail(EATSS_E_INVALID, "eatss_desc_builtin: bad dtype");
     if (!dims) return fail(EATSS_E_INVALID, "eatss_desc_builtin: dims is null");
     const int want = kDimsPerBuiltin[k];
@@ -409,6 +441,8 @@ eatss_status eatss_desc_builtin(eatss_builtin k, const int64_t *dims, int ndims,
         return fail(EATSS_E_INVALID, "eatss_desc_builtin: syrk row block exceeds ni");
     if ((k == EATSS_JACOBI2D || k == EATSS_HEAT3D) && (dv[0] < 3 || tsteps < 0))
         return fail(EATSS_E_INVALID, "eatss_desc_builtin: stencils need n >= 3 and tsteps >= 0");
+    if (k == EATSS_CONV2D && dv[1] > dv[0])
+        return fail(EATSS_E_INVALID, "eatss_desc_builtin: conv-2d needs f <= n");
     if (k == EATSS_CCSD_T_D1 && dt != EATSS_F32)
         return fail(EATSS_E_UNSUPPORTED, "eatss_desc_builtin: ccsd_t_d1 is fp32 only in this build");
     auto *d = new (std::nothrow) eatss_kernel_desc();
@@ -457,6 +491,10 @@ double eatss_desc_flops(const eatss_kernel_desc *d) {
         case EATSS_MVT: return 4 * D(x[0]) * D(x[0]);
         case EATSS_ATAX: case EATSS_BICG: return 4 * D(x[0]) * D(x[1]);
         case EATSS_GEMVER: return 10 * D(x[0]) * D(x[0]) + D(x[0]);  // 4 + 3 + 3 per (i, j), + per i
+        // one multiply-add per iteration point (the Khatri-Rao factor C[k][j]*D[l][j] formed once per
+        // (k, l, j), not per point)
+        case EATSS_MTTKRP: return 2 * D(x[0]) * D(x[1]) * D(x[2]) * D(x[3]);
+        case EATSS_CONV2D: return 2 * D(x[1]) * D(x[1]) * D(x[0] - x[1] + 1) * D(x[0] - x[1] + 1);
     }
     return 0;
 }
@@ -489,6 +527,10 @@ double eatss_desc_bytes(const eatss_kernel_desc *d) {
         case EATSS_ATAX: return e * (2 * D(x[0]) * D(x[1]) + 2 * D(x[1]) + D(x[0]));
         case EATSS_BICG: return e * (D(x[0]) * D(x[1]) + 2 * D(x[0]) + 2 * D(x[1]));
         case EATSS_GEMVER: return e * (3 * D(x[0]) * D(x[0]) + 11 * D(x[0]));
+        case EATSS_MTTKRP:  // A read + written, B, C, D read once
+            return e * (2 * D(x[0]) * D(x[1]) + D(x[0]) * D(x[2]) * D(x[3]) + D(x[2]) * D(x[1]) + D(x[3]) * D(x[1]));
+        case EATSS_CONV2D:  // inp, W read once, out written once
+            return e * (D(x[0]) * D(x[0]) + D(x[1]) * D(x[1]) + D(x[0] - x[1] + 1) * D(x[0] - x[1] + 1));
     }
     return 0;
 }
@@ -600,6 +642,29 @@ eatss_status eatss_plan(const eatss_kernel_desc *d, const int64_t *tiles, eatss_
             o.tile[0] = ti; o.tile[1] = tj;
         }
         *n_plans = nn;
+    } else if (d->kind == EATSS_MTTKRP || d->kind == EATSS_CONV2D) {
+        eatss_launch_plan &o = plans[0];
+        std::memset(&o, 0, sizeof(o));
+        o.engine = 1;
+        o.carveout_pct = d->exec.split_pct;
+        if (d->kind == EATSS_MTTKRP) {
+            int bx, by, rm, smem, sp;
+            const bool fast = mttkrp_plan(d->dims.data(), tiles, &o.grid_x, &o.grid_y, &o.grid_z, &bx, &by, &rm, &smem, &sp);
+            o.block_x = bx; o.block_y = by; o.rm = rm; o.rn = fast ? 4 : 1; o.vec = fast ? 4 : 1;
+            o.passes = sp;  // split-k factor (grid.z)
+            o.smem_bytes = smem; o.a_in_smem = 0; o.b_in_smem = fast;
+        } else {
+            int threads, smem, rc, wc, groups, segs;
+            const bool fast = conv2d_plan(d->dims[0], d->dims[1], tiles, &o.grid_x, &o.grid_y, &threads, &smem, &rc,
+                                          &wc, &groups, &segs);
+            o.grid_z = 1; o.block_x = threads; o.block_y = 1; o.rm = rc; o.rn = 4; o.vec = fast ? 4 : 1;
+            o.passes = 1; o.smem_bytes = smem; o.a_in_smem = fast; o.b_in_smem = 0;
+        }
+        o.simt_x = std::min(32, o.block_x);
+        const int64_t ex[4] = {d->nests[0].loops[0].extent, d->nests[0].loops[1].extent, d->nests[0].loops[2].extent,
+                               d->nests[0].loops[3].extent};
+        for (int p = 0; p < 4; p++) o.tile[p] = std::min(tiles[p], ex[p]);
+        *n_plans = 1;
     } else {
         eatss_launch_plan &o = plans[0];
         std::memset(&o, 0, sizeof(o));
@@ -711,6 +776,39 @@ static eatss_status run_impl(const eatss_kernel_desc *cd, int only_nest, const i
         if (ev) cudaEventRecord(ev[1], s);
         return e == cudaSuccess ? EATSS_OK : cuda_fail(e, "eatss_run(low-dimensional kernel)");
     }
+    if (d->kind == EATSS_MTTKRP || d->kind == EATSS_CONV2D) {
+        if (d->dtype != EATSS_F32)  // fp64 descriptors serve the model (paper-mode tables) only
+            return fail(EATSS_E_UNSUPPORTED, "eatss_run: the mttkrp / conv-2d executors are fp32 only");
+        cudaEvent_t *ev = kernel_events(d, 0);
+        cudaError_t e = cudaSuccess;
+        if (d->kind == EATSS_MTTKRP) {
+            int64_t gx, gy, gz;
+            int bx, by, rm, smem, sp;
+            mttkrp_plan(d->dims.data(), tiles, &gx, &gy, &gz, &bx, &by, &rm, &smem, &sp);
+            if (sp > 1) {  // split-k partials: library-owned workspace of sp x ni x nj floats
+                int dev = 0;
+                cudaGetDevice(&dev);
+                const size_t need = (size_t)sp * (size_t)d->buffer_elems[0] * 4;
+                if (d->ws_dev != dev || d->ws_bytes < need) {
+                    if (d->ws && d->ws_dev == dev) cudaFree(d->ws);  // never free another device's pointer here
+                    d->ws = nullptr;
+                    d->ws_bytes = 0;
+                    if ((e = cudaMalloc(&d->ws, need)) != cudaSuccess) return cuda_fail(e, "eatss_run(mttkrp workspace)");
+                    d->ws_bytes = need;
+                    d->ws_dev = dev;
+                }
+            }
+            if (ev) cudaEventRecord(ev[0], s);
+            e = launch_mttkrp((float *)buffers[0], (const float *)buffers[1], (const float *)buffers[2],
+                              (const float *)buffers[3], d->dims.data(), tiles, (float *)d->ws, nullptr, s, nullptr);
+        } else {
+            if (ev) cudaEventRecord(ev[0], s);
+            e = launch_conv2d((float *)buffers[0], (const float *)buffers[1], (const float *)buffers[2], d->dims[0],
+                              d->dims[1], tiles, nullptr, s, nullptr);
+        }
+        if (ev) cudaEventRecord(ev[1], s);
+        return e == cudaSuccess ? EATSS_OK : cuda_fail(e, "eatss_run(mttkrp / conv-2d)");
+    }
     if (d->kind == EATSS_JACOBI2D || d->kind == EATSS_HEAT3D) {
         if (only_nest >= 0) return fail(EATSS_E_UNSUPPORTED, "eatss_run_nest: stencils run whole time loops");
         cudaEvent_t *ev = kernel_events(d, 0);
@@ -760,6 +858,8 @@ static void buffer_io(const eatss_kernel_desc *d, int i, bool *in, bool *out) {
         case EATSS_ATAX: *in = i >= 2; *out = i <= 1; break;
         case EATSS_BICG: *in = i >= 2; *out = i <= 1; break;
         case EATSS_GEMVER: *out = i <= 2; break;
+        case EATSS_MTTKRP: *out = i == 0; break;
+        case EATSS_CONV2D: *in = i != 0; *out = i == 0; break;
     }
 }
 
@@ -925,6 +1025,15 @@ eatss_status eatss_coverage(const eatss_kernel_desc *d, int nest, const int64_t 
     }
     if (is_lowdim(d->kind))
         return fail(EATSS_E_UNSUPPORTED, "eatss_coverage: the low-dimensional kernels have no visit-count mode");
+    if (d->kind == EATSS_MTTKRP) {
+        cudaError_t e = launch_mttkrp(nullptr, nullptr, nullptr, nullptr, d->dims.data(), tiles, nullptr, counts, s,
+                                      nullptr);
+        return e == cudaSuccess ? EATSS_OK : cuda_fail(e, "eatss_coverage");
+    }
+    if (d->kind == EATSS_CONV2D) {
+        cudaError_t e = launch_conv2d(nullptr, nullptr, nullptr, d->dims[0], d->dims[1], tiles, counts, s, nullptr);
+        return e == cudaSuccess ? EATSS_OK : cuda_fail(e, "eatss_coverage");
+    }
     const int64_t n = d->dims[0];
     cudaError_t e;
     if (d->kind == EATSS_JACOBI2D)
@@ -970,6 +1079,14 @@ int64_t eatss_launches_per_run(const eatss_kernel_desc *d, const int64_t *tiles)
         case EATSS_MVT: case EATSS_BICG: return 1;  // one fused pass over the matrix
         case EATSS_ATAX: return 2;
         case EATSS_GEMVER: return 3;
+        case EATSS_CONV2D: return 1;
+        case EATSS_MTTKRP: {  // the kernel, + the split-order reduction when k is split across CTAs
+            if (!tiles || check_tiles(d, tiles) != EATSS_OK) return -1;
+            int64_t gx, gy, gz;
+            int bx, by, rm, smem, sp;
+            mttkrp_plan(d->dims.data(), tiles, &gx, &gy, &gz, &bx, &by, &rm, &smem, &sp);
+            return sp > 1 ? 2 : 1;
+        }
     }
     return -1;
 }

@@ -74,6 +74,10 @@ struct eatss_kernel_desc {
     int hdev = -1;
     void *hstream[2] = {nullptr, nullptr};  // host->device, device->host
     std::vector<void *> hev;                // pipeline events
+    // library-owned scratch (mttkrp split-k partials), grown on demand, freed with the descriptor
+    void *ws = nullptr;
+    size_t ws_bytes = 0;
+    int ws_dev = -1;
     ~eatss_kernel_desc();
 };
 

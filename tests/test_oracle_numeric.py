@@ -319,3 +319,11 @@ def test_conv2d_linear_field_closed_form():
 def test_conv2d_filter_equal_to_image_is_one_dot_product():
     inp, W = _ints((6, 6), 13), _ints((6, 6), 14)
     assert np.array_equal(O.conv2d(inp, W), np.array([[float((inp * W).sum())]]))
+
+
+def test_conv2d_rectangular_band_equals_rows_of_the_square_result():
+    inp, W = synth.uniform((30, 30), 15), synth.uniform((5, 5), 16)
+    full = O.conv2d(inp, W)
+    assert np.array_equal(O.conv2d(inp[7:7 + 10 + 4, :], W), full[7:17])
+    np.testing.assert_allclose(O.conv2d(inp[:, 3:20], W), signal.correlate2d(inp[:, 3:20].astype(np.float64),
+                               W.astype(np.float64), mode="valid"), rtol=0, atol=1e-13)
