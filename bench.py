@@ -297,6 +297,19 @@ def other_configs(E, torch, gpu, stream, peaks):
                                                  "gbs": gbs, "bound": "hbm", "frac": gbs / hbm, "tile_origin": note}
     out["ccsd_t_d1 dims=48"] = row
     del b
+    # non-PolyBench 4-D kernels (readings R-N8, R-N9): mttkrp is graded against
+    # the FFMA peak (one FFMA per iteration point), conv-2d against HBM (8 B per output)
+    for kind, dims, bound in (("mttkrp", (512, 32, 512, 512), "alu"), ("conv-2d", (8192, 5), "hbm")):
+        d = E.desc_builtin(kind, dims)
+        b = bufs_for(d)
+        tiles, _ = E.select_tiles(d, gpu, split_pct=50, waf=16, mode=1)
+        d.set_exec(split_pct=50, engine=1)
+        ms = timed_ms(d, tiles, b, 10)
+        tf = d.flops / (ms * 1e-3) / 1e12
+        gbs = d.bytes / (ms * 1e-3) / 1e9
+        out[kind] = {"dims": list(dims), "tiles": list(tiles), "ms": ms, "tflops": tf, "gbs": gbs, "bound": bound,
+                     "frac": tf / ffma if bound == "alu" else gbs / hbm}
+        del b
     torch.cuda.empty_cache()
     return out
 

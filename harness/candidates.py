@@ -48,6 +48,9 @@ KINDS = {
     "atax": dict(dims=(4000, 4000)),
     "bicg": dict(dims=(4000, 4000)),
     "gemver": dict(dims=(4000,)),
+    # non-PolyBench 4-D kernels of Figs. 10-11 (readings R-N8, R-N9: our sizes)
+    "mttkrp": dict(dims=(512, 32, 512, 512)),
+    "conv-2d": dict(dims=(8192, 5)),
 }
 
 

@@ -66,11 +66,11 @@ struct Cursor {
     int64_t kt, lt;
     int kk, sub;
 };
-__device__ __forceinline__ void advance(Cursor &c, const MtArgs &a, int spt, int64_t nlt) {
+__device__ __forceinline__ void advance(Cursor &c, const MtArgs &a, int spt, int64_t nlt, int ks) {
     if (++c.sub < spt) return;
     c.sub = 0;
     const int64_t tkl = min((int64_t)a.Tk, a.nk - c.kt * a.Tk);
-    if ((c.kk += a.ks) < tkl) return;
+    if ((c.kk += ks) < tkl) return;
     c.kk = 0;
     if (++c.lt < nlt) return;
     c.lt = 0;
@@ -80,40 +80,46 @@ __device__ __forceinline__ void advance(Cursor &c, const MtArgs &a, int spt, int
 // Fast path: nj % 4 == 0, nl % 4 == 0, Tj % 4 == 0, Tl % 4 == 0 (mttkrp_plan).  128 threads; each
 // owns RM rows x 4 consecutive columns of A per row pass.  A stage holds B[R rows][ks k][sw l] and
 // D[sw l][4 bx columns].
-template <int RM, bool COVER>
+// SW, BXT, KS > 0: compile-time stage width, threads along j and k per stage (shared-memory
+// addresses become immediates); 0: the runtime values of MtArgs.
+template <int RM, bool COVER, int SW = 0, int BXT = 0, int KS = 0>
 __global__ void __launch_bounds__(128, RM <= 4 ? 4 : 2) mttkrp_kernel(MtArgs a) {
     extern __shared__ __align__(16) float sm[];
-    const int tx = threadIdx.x % a.bx, ty = threadIdx.x / a.bx;
-    const int nthr = a.bx * a.by;
-    const int R = a.by * RM;             // rows per row pass
-    const int bpitch = a.sw + 4;         // B stage row pitch (floats), staggers banks
-    const int rpitch = a.ks * bpitch;    // one row's ks k-slices
-    const int dw = a.bx * 4;             // D stage row width (floats)
-    const int stage_f = R * rpitch + a.sw * dw;
+    const int sw = SW > 0 ? SW : a.sw;
+    const int bxv = BXT > 0 ? BXT : a.bx;
+    const int byv = BXT > 0 ? kThreads / BXT : a.by;
+    const int ksv = KS > 0 ? KS : a.ks;
+    const int tx = threadIdx.x % bxv, ty = threadIdx.x / bxv;
+    const int nthr = bxv * byv;
+    const int R = byv * RM;             // rows per row pass
+    const int bpitch = sw + 4;         // B stage row pitch (floats), staggers banks
+    const int rpitch = ksv * bpitch;    // one row's ks k-slices
+    const int dw = bxv * 4;             // D stage row width (floats)
+    const int stage_f = R * rpitch + sw * dw;
     const int64_t ti0 = (int64_t)blockIdx.y * a.Ti, tj0 = (int64_t)blockIdx.x * a.Tj;
     const int64_t ihi = min(ti0 + a.Ti, a.ni), jhi = min(tj0 + a.Tj, a.nj);
     const int64_t nkt = (a.nk + a.Tk - 1) / a.Tk, nlt = (a.nl + a.Tl - 1) / a.Tl;
-    const int spt = (a.Tl + a.sw - 1) / a.sw;  // sub-stages per l-tile
+    const int spt = (a.Tl + sw - 1) / sw;  // sub-stages per l-tile
     const int64_t p0 = (int64_t)blockIdx.z * a.pps, p1 = min(p0 + a.pps, nkt * nlt);
     if (p0 >= p1) return;  // (a.S > 1: its partial plane is never read -- reduce covers z < S only)
     // stages of this CTA per pass: sum over its pairs of ceil(k in the pair's k-tile / ks) x spt
     int64_t nst;
     {
         const int64_t kf = p0 / nlt, kl = (p1 - 1) / nlt;
-        auto grp = [&](int64_t kt) { return (min((int64_t)a.Tk, a.nk - kt * a.Tk) + a.ks - 1) / a.ks; };
+        auto grp = [&](int64_t kt) { return (min((int64_t)a.Tk, a.nk - kt * a.Tk) + ksv - 1) / ksv; };
         if (kf == kl) nst = (p1 - p0) * grp(kf);
         else nst = (nlt - p0 % nlt) * grp(kf) + (kl - kf - 1) * nlt * grp(kf) + ((p1 - 1) % nlt + 1) * grp(kl);
         nst *= spt;
     }
     const int64_t nknl = a.nk * a.nl;
-    const int cpr = a.sw >> 2, lgc = a.lgc;  // 16-byte chunks per staged B row slice
+    const int cpr = sw >> 2, lgc = SW > 0 ? (SW == 4 ? 0 : SW == 8 ? 1 : SW == 16 ? 2 : 3) : a.lgc;  // 16-byte chunks per staged B row slice
     for (int64_t jp = tj0; jp < jhi; jp += dw) {                   // column passes (Tj > 4*bx)
         const int64_t j = jp + 4 * tx;
         const bool jok = j < jhi;
         for (int64_t ip = ti0; ip < ihi; ip += R) {                // row passes (Ti > R)
             if constexpr (COVER) {
                 for (int r = 0; r < RM; r++) {
-                    const int64_t i = ip + ty + (int64_t)a.by * r;
+                    const int64_t i = ip + ty + (int64_t)byv * r;
                     if (i >= ihi || !jok) continue;
                     for (int64_t p = p0; p < p1; p++) {
                         const int64_t kt = p / nlt, lt = p % nlt;
@@ -143,16 +149,16 @@ __global__ void __launch_bounds__(128, RM <= 4 ? 4 : 2) mttkrp_kernel(MtArgs a) 
 #pragma unroll
             for (int m = 0; m < kMaxDChunks; m++) {
                 const int c = threadIdx.x + m * nthr;
-                const int l = c / a.bx, q = c - l * a.bx;
-                dl[m] = (c < a.sw * a.bx && jp + 4 * q < jhi) ? l : -1;
+                const int l = c / bxv, q = c - l * bxv;
+                dl[m] = (c < sw * bxv && jp + 4 * q < jhi) ? l : -1;
                 dso[m] = l * dw + 4 * q;
             }
             auto issue = [&](int64_t s) {
                 float *st = sm + (int)(s % kStages) * stage_f;
                 const int64_t k = ci.kt * a.Tk + ci.kk;
-                const int kc = (int)min((int64_t)a.ks, min((ci.kt + 1) * a.Tk, a.nk) - k);
-                const int64_t l0 = ci.lt * a.Tl + (int64_t)ci.sub * a.sw;
-                const int w = (int)min((int64_t)a.sw, min((ci.lt + 1) * a.Tl, a.nl) - l0);
+                const int kc = (int)min((int64_t)ksv, min((ci.kt + 1) * a.Tk, a.nk) - k);
+                const int64_t l0 = ci.lt * a.Tl + (int64_t)ci.sub * sw;
+                const int w = (int)min((int64_t)sw, min((ci.lt + 1) * a.Tl, a.nl) - l0);
                 const float *bk = a.B + k * a.nl + l0;
                 for (int kk = 0; kk < kc; kk++, bk += a.nl) {
 #pragma unroll
@@ -171,7 +177,7 @@ __global__ void __launch_bounds__(128, RM <= 4 ? 4 : 2) mttkrp_kernel(MtArgs a) 
                     const bool v = dl[m] < w;
                     cp16(ds + dso[m], v ? dk + (int64_t)dl[m] * a.nj + (dso[m] - dl[m] * dw) : a.D, v);
                 }
-                advance(ci, a, spt, nlt);
+                advance(ci, a, spt, nlt, ksv);
             };
             float acc[RM][4], t[RM][4];
 #pragma unroll
@@ -190,16 +196,19 @@ __global__ void __launch_bounds__(128, RM <= 4 ? 4 : 2) mttkrp_kernel(MtArgs a) 
                 const float *st = sm + (int)(s % kStages) * stage_f;
                 const float *ds = st + R * rpitch + 4 * tx;
                 const int64_t k0s = cc.kt * a.Tk + cc.kk;
-                const int kc = (int)min((int64_t)a.ks, min((cc.kt + 1) * a.Tk, a.nk) - k0s);
+                const int kc = (int)min((int64_t)ksv, min((cc.kt + 1) * a.Tk, a.nk) - k0s);
                 const bool fold = cc.sub == spt - 1;  // (k, l-tile) complete after this stage
                 for (int kk = 0; kk < kc; kk++) {
                     const float *brow = st + ty * rpitch + kk * bpitch;
-#pragma unroll 2
-                    for (int l = 0; l < a.sw; l += 4) {
+                    // C[k][j] of this k-slice, loaded before the slice's FFMAs hide its latency
+                    float4 c = make_float4(0.f, 0.f, 0.f, 0.f);
+                    if (fold && jok) c = __ldg(reinterpret_cast<const float4 *>(a.C + (k0s + kk) * a.nj + j));
+#pragma unroll
+                    for (int l = 0; l < sw; l += 4) {
                         float b[RM][4], d[4][4];
 #pragma unroll
                         for (int r = 0; r < RM; r++) {
-                            const float4 v = *reinterpret_cast<const float4 *>(brow + a.by * r * rpitch + l);
+                            const float4 v = *reinterpret_cast<const float4 *>(brow + byv * r * rpitch + l);
                             b[r][0] = v.x; b[r][1] = v.y; b[r][2] = v.z; b[r][3] = v.w;
                         }
 #pragma unroll
@@ -217,8 +226,6 @@ __global__ void __launch_bounds__(128, RM <= 4 ? 4 : 2) mttkrp_kernel(MtArgs a) 
                                 for (int c = 0; c < 4; c++) t[r][c] = fmaf(b[r][u], d[u][c], t[r][c]);
                     }
                     if (fold) {  // fold C[k][j] in
-                        float4 c = make_float4(0.f, 0.f, 0.f, 0.f);
-                        if (jok) c = __ldg(reinterpret_cast<const float4 *>(a.C + (k0s + kk) * a.nj + j));
 #pragma unroll
                         for (int r = 0; r < RM; r++) {
                             acc[r][0] = fmaf(c.x, t[r][0], acc[r][0]); acc[r][1] = fmaf(c.y, t[r][1], acc[r][1]);
@@ -227,14 +234,14 @@ __global__ void __launch_bounds__(128, RM <= 4 ? 4 : 2) mttkrp_kernel(MtArgs a) 
                         }
                     }
                 }
-                advance(cc, a, spt, nlt);
+                advance(cc, a, spt, nlt, ksv);
             }
             cp_wait<0>();
             __syncthreads();  // the ring is reused by the next pass
             if (!jok) continue;
 #pragma unroll
             for (int r = 0; r < RM; r++) {
-                const int64_t i = ip + ty + (int64_t)a.by * r;
+                const int64_t i = ip + ty + (int64_t)byv * r;
                 if (i >= ihi) continue;
                 const float4 v = make_float4(acc[r][0], acc[r][1], acc[r][2], acc[r][3]);
                 if (a.S > 1) {
@@ -321,12 +328,13 @@ bool mttkrp_plan(const int64_t *dims, const int64_t *tiles, int64_t *gx, int64_t
     }
     const int b_x = (int)std::min<int64_t>(Tj / 4, 32);
     const int b_y = kThreads / b_x;
-    // rows per thread: at most 4 (128 registers: four CTAs of 128 threads per SM keep 16 warps
-    // resident -- measured faster than 8 rows at 232 registers and 8 warps); EATSS_MT_MAXRM overrides
+    // rows per thread: up to 8 (two CTAs of 128 threads per SM at ~230 registers: measured faster
+    // than 4 rows at 128 registers and four CTAs -- 0.40 vs 0.46 ms at the config); EATSS_MT_MAXRM
+    // (1, 2, 4, 8) overrides for experiments
     static const int max_rm = [] {
         const char *e = getenv("EATSS_MT_MAXRM");
-        const int v = e ? atoi(e) : 4;
-        return v == 1 || v == 2 || v == 8 ? v : 4;
+        const int v = e ? atoi(e) : 8;
+        return v == 1 || v == 2 || v == 4 ? v : 8;
     }();
     int r = 1;
     while (r < max_rm && (int64_t)b_y * r < Ti) r *= 2;
@@ -402,7 +410,25 @@ cudaError_t launch_mttkrp(float *A, const float *B, const float *C, const float 
             mttkrp_kernel<RMV, false><<<grid, threads, sm, s>>>(a);                                     \
         }                                                                                               \
     }
-    EATSS_MT(1) EATSS_MT(2) EATSS_MT(4) EATSS_MT(8)
+#define EATSS_MTS(RMV, SWV, KSV)                                                                        \
+    if (!done && rm == RMV && a.sw == SWV && a.ks == KSV) {                                             \
+        e = cudaFuncSetAttribute(mttkrp_kernel<RMV, false, SWV, 8, KSV>,                                 \
+                                 cudaFuncAttributeMaxDynamicSharedMemorySize, sm);                      \
+        if (e != cudaSuccess) return e;                                                                 \
+        mttkrp_kernel<RMV, false, SWV, 8, KSV><<<grid, threads, sm, s>>>(a);                            \
+        done = true;                                                                                    \
+    }
+    bool done = false;
+    if (!counts && bx == 8) {  // Tj = 32 (the rank of the config, every EATSS tile of it): specialised
+        EATSS_MTS(8, 16, 2) EATSS_MTS(8, 32, 2) EATSS_MTS(8, 8, 2) EATSS_MTS(8, 4, 2)
+        EATSS_MTS(8, 16, 1) EATSS_MTS(8, 32, 1) EATSS_MTS(8, 8, 1) EATSS_MTS(8, 4, 1)
+        EATSS_MTS(4, 16, 2) EATSS_MTS(4, 32, 2) EATSS_MTS(4, 8, 2) EATSS_MTS(4, 4, 2)
+        EATSS_MTS(4, 16, 1) EATSS_MTS(4, 32, 1) EATSS_MTS(4, 8, 1) EATSS_MTS(4, 4, 1)
+    }
+    if (!done) {
+        EATSS_MT(1) EATSS_MT(2) EATSS_MT(4) EATSS_MT(8)
+    }
+#undef EATSS_MTS
 #undef EATSS_MT
     if (launched) (*launched)++;
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
