@@ -309,6 +309,14 @@ def other_configs(E, torch, gpu, stream, peaks):
         gbs = d.bytes / (ms * 1e-3) / 1e9
         out[kind] = {"dims": list(dims), "tiles": list(tiles), "ms": ms, "tflops": tf, "gbs": gbs, "bound": bound,
                      "frac": tf / ffma if bound == "alu" else gbs / hbm}
+        if kind == "mttkrp":  # the tcgen05 3xTF32 path at its MMA-legal tile: HBM-bound (B read once)
+            tt = (1, dims[1], 128, 32)
+            d.set_exec(split_pct=50, engine=2)
+            ms = timed_ms(d, tt, b, 10)
+            gbs = d.bytes / (ms * 1e-3) / 1e9
+            out[kind] = {"simt": out[kind], "tensor": {"tiles": list(tt), "ms": ms, "tflops": d.flops / (ms * 1e-3) / 1e12,
+                                                       "gbs": gbs, "bound": "hbm", "frac": gbs / hbm,
+                                                       "tile_origin": "MMA-legal point of the mttkrp space"}}
         del b
     torch.cuda.empty_cache()
     return out

@@ -54,7 +54,7 @@ def main():
             dims = KINDS[kind]
             d = E.desc_builtin(kind, dims)
             d.set_exec(split_pct=50, engine=1)
-            ext = [d.plan([1 << 30] * 4)[0].tile[p] for p in range(4)]  # loop extents (tiles clip to them)
+            ext = [E.plan(d, [1 << 30] * 4)[0].tile[p] for p in range(4)]  # loop extents (tiles clip to them)
             doms = [sorted({min(s, e) for s in SIZES}) for e in ext]
             space = [tuple(v) for v in np.array(np.meshgrid(*doms, indexing="ij")).reshape(4, -1).T.tolist()]
             rng = random.Random(a.seed)

@@ -64,6 +64,10 @@ bool mttkrp_plan(const int64_t *dims, const int64_t *tiles, int64_t *gx, int64_t
                  int *rm, int *smem, int *splits, int *sw_out = nullptr, int *ks_out = nullptr);
 cudaError_t launch_mttkrp(float *A, const float *B, const float *C, const float *D, const int64_t *dims,
                           const int64_t *tiles, float *ws, int32_t *counts, cudaStream_t s, int64_t *launched);
+bool mttkrp_tc_applicable(const int64_t *dims, const int64_t *tiles);
+size_t mttkrp_tc_ws_floats(const int64_t *dims);
+cudaError_t launch_mttkrp_tc(float *A, const float *B, const float *C, const float *D, const int64_t *dims, float *ws,
+                             cudaStream_t s, cudaEvent_t *ev, int64_t *launched);
 bool conv2d_plan(int64_t n, int64_t f, const int64_t *tiles, int64_t *gx, int64_t *gy, int *threads, int *smem,
                  int *rc, int *wc, int *groups, int *segs);
 cudaError_t launch_conv2d(float *out, const float *inp, const float *W, int64_t n, int64_t f, const int64_t *tiles,
@@ -782,13 +786,18 @@ static eatss_status run_impl(const eatss_kernel_desc *cd, int only_nest, const i
         cudaEvent_t *ev = kernel_events(d, 0);
         cudaError_t e = cudaSuccess;
         if (d->kind == EATSS_MTTKRP) {
+            const bool tc = d->exec.engine == EATSS_ENGINE_TENSOR;
+            if (tc && !mttkrp_tc_applicable(d->dims.data(), tiles))
+                return fail(EATSS_E_UNSUPPORTED, "eatss_run: the mttkrp tensor engine needs the tile (1, nj, 128, 32) "
+                                                 "with nj in {32, 64, 128}, nk % 128 == 0, nl % 32 == 0");
             int64_t gx, gy, gz;
             int bx, by, rm, smem, sp;
             mttkrp_plan(d->dims.data(), tiles, &gx, &gy, &gz, &bx, &by, &rm, &smem, &sp);
-            if (sp > 1) {  // split-k partials: library-owned workspace of sp x ni x nj floats
+            if (tc || sp > 1) {  // split partials (SIMT) / D lo + block partials (tensor): library-owned
                 int dev = 0;
                 cudaGetDevice(&dev);
-                const size_t need = (size_t)sp * (size_t)d->buffer_elems[0] * 4;
+                const size_t need = tc ? mttkrp_tc_ws_floats(d->dims.data()) * 4
+                                       : (size_t)sp * (size_t)d->buffer_elems[0] * 4;
                 if (d->ws_dev != dev || d->ws_bytes < need) {
                     if (d->ws && d->ws_dev == dev) cudaFree(d->ws);  // never free another device's pointer here
                     d->ws = nullptr;
@@ -797,6 +806,11 @@ static eatss_status run_impl(const eatss_kernel_desc *cd, int only_nest, const i
                     d->ws_bytes = need;
                     d->ws_dev = dev;
                 }
+            }
+            if (tc) {  // events around the tcgen05 kernel alone (the D split and the block reduction outside)
+                e = launch_mttkrp_tc((float *)buffers[0], (const float *)buffers[1], (const float *)buffers[2],
+                                     (const float *)buffers[3], d->dims.data(), (float *)d->ws, s, ev, nullptr);
+                return e == cudaSuccess ? EATSS_OK : cuda_fail(e, "eatss_run(mttkrp, tensor)");
             }
             if (ev) cudaEventRecord(ev[0], s);
             e = launch_mttkrp((float *)buffers[0], (const float *)buffers[1], (const float *)buffers[2],
@@ -1082,6 +1096,8 @@ int64_t eatss_launches_per_run(const eatss_kernel_desc *d, const int64_t *tiles)
         case EATSS_CONV2D: return 1;
         case EATSS_MTTKRP: {  // the kernel, + the split-order reduction when k is split across CTAs
             if (!tiles || check_tiles(d, tiles) != EATSS_OK) return -1;
+            if (d->exec.engine == EATSS_ENGINE_TENSOR)  // D lo split, tcgen05 kernel, block reduction
+                return mttkrp_tc_applicable(d->dims.data(), tiles) ? 3 : -1;
             int64_t gx, gy, gz;
             int bx, by, rm, smem, sp;
             mttkrp_plan(d->dims.data(), tiles, &gx, &gy, &gz, &bx, &by, &rm, &smem, &sp);

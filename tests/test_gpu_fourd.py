@@ -160,3 +160,41 @@ def test_conv2d_coverage(cuda_device, tiles, n, f):
     E.coverage(d, 0, tiles, counts)
     torch.cuda.synchronize()
     assert int(counts.min()) == 1 and int(counts.max()) == 1
+
+
+# ------------------------------------------------------------------ mttkrp on the tensor pipe
+@pytest.mark.parametrize("kind,dims", [("int", (3, 32, 256, 64)), ("rand", (5, 32, 128, 96)),
+                                       ("int", (2, 64, 384, 32)), ("rand", (3, 128, 128, 64))])
+def test_mttkrp_tensor(cuda_device, kind, dims):
+    """tcgen05 3xTF32 path at its MMA-legal tile (1, nj, 128, 32): small integers exact (|B| <= 2
+    stays exact in tf32 hi; lo = 0), random data within the fp32 normwise bar."""
+    ni, nj, nk, nl = dims
+    A0, B, C, D = gen(kind, (ni, nj), 1), gen(kind, (ni, nk, nl), 2), gen(kind, (nk, nj), 3), gen(kind, (nl, nj), 4)
+    d = E.desc_builtin("mttkrp", dims)
+    d.set_exec(split_pct=50, engine=2)
+    tiles = (1, nj, 128, 32)
+    assert E.launches_per_run(d, tiles) == 3
+    b = [dev(A0), dev(B), dev(C), dev(D)]
+    E.run(d, tiles, b)
+    check(kind, host(b[0]), O.mttkrp(A0, B, C, D))
+    b2 = [dev(A0)] + b[1:]
+    E.run(d, tiles, b2)
+    assert torch.equal(b[0], b2[0])  # deterministic block-order reduction
+    with pytest.raises(E.EatssError):
+        E.run(d, (128, 32, 16, 16), b)  # not an MMA-legal tile: refused, no silent fallback
+
+
+def test_mttkrp_tensor_full_size(cuda_device):
+    dims = (512, 32, 512, 512)
+    ni, nj, nk, nl = dims
+    d = E.desc_builtin("mttkrp", dims)
+    d.set_exec(split_pct=50, engine=2)
+    A0, B, C, D = synth.uniform((ni, nj), 1), synth.uniform((ni, nk, nl), 2), synth.uniform((nk, nj), 3), \
+        synth.uniform((nl, nj), 4)
+    b = [dev(A0), dev(B), dev(C), dev(D)]
+    E.run(d, (1, nj, 128, 32), b)
+    got = host(b[0])
+    g = np.random.default_rng(8)
+    ii, jj = g.integers(0, ni, 600), g.integers(0, nj, 600)
+    ref = O.mttkrp_entries(ii, jj, A0, B, C, D)
+    assert np.linalg.norm(got[ii, jj] - ref) / np.linalg.norm(ref) <= 1e-5
