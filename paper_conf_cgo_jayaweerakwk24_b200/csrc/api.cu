@@ -245,6 +245,40 @@ static eatss_status build(eatss_kernel_desc *d) {
     return EATSS_OK;
 }
 
+// Library-owned scratch of a descriptor (grown on demand, on the current device).
+static eatss_status ensure_ws(eatss_kernel_desc *d, size_t need) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (d->ws_dev == dev && d->ws_bytes >= need) return EATSS_OK;
+    if (d->ws && d->ws_dev == dev) cudaFree(d->ws);  // never free another device's pointer here
+    d->ws = nullptr;
+    d->ws_bytes = 0;
+    cudaError_t e = cudaMalloc(&d->ws, need);
+    if (e != cudaSuccess) return cuda_fail(e, "eatss_run(workspace)");
+    d->ws_bytes = need;
+    d->ws_dev = dev;
+    return EATSS_OK;
+}
+
+// SIMT syrk: its transposed operand B(k, j) = A[j][k] is laid out as A^T once per run (a layout pass
+// into the descriptor's workspace, ~2 x 64 MB of traffic at N = 4000) so the executor runs its
+// non-transposed staged path; every element keeps the same k-ascending sum.  EATSS_SYRK_TRANSB=1
+// keeps the strided transposed-operand path (for comparison).
+static bool simt_untranspose(const eatss_kernel_desc *d) {
+    static const bool off = [] {
+        const char *e = getenv("EATSS_SYRK_TRANSB");
+        return e && atoi(e) != 0;
+    }();
+    return d->kind == EATSS_SYRK && d->dtype == EATSS_F32 && d->exec.engine != EATSS_ENGINE_TENSOR && !off;
+}
+static void untranspose_nests(const eatss_kernel_desc *d, std::vector<ContractNest> &cn, const void *at) {
+    for (auto &n : cn) {
+        n.B = at;
+        n.ldb = d->dims[0];  // A^T is nj x ni
+        n.transB = false;
+    }
+}
+
 static const int kDimsPerBuiltin[] = {3, 4, 5, 2, 1, 1, 7, 1, 2, 2, 1, 4, 2};
 
 static bool is_lowdim(eatss_builtin k) {
@@ -606,6 +640,7 @@ eatss_status eatss_plan(const eatss_kernel_desc *d, const int64_t *tiles, eatss_
         void *b[EATSS_MAX_BUFFERS];
         for (int i = 0; i < EATSS_MAX_BUFFERS; i++) b[i] = (void *)(uintptr_t)(256 * (i + 1));
         auto cn = contraction_nests(d, b);
+        if (simt_untranspose(d)) untranspose_nests(d, cn, b[EATSS_MAX_BUFFERS - 1]);
         for (int i = 0; i < (int)cn.size(); i++) {
             ContractPlan p = plan_contraction(cn[i], tiles, 232448);
             eatss_launch_plan &o = plans[i];
@@ -750,6 +785,13 @@ static eatss_status run_impl(const eatss_kernel_desc *cd, int only_nest, const i
     if (is_contraction(d->kind)) {
         auto cn = contraction_nests(d, buffers);
         const int sl = smem_limit_bytes();
+        if (simt_untranspose(d)) {
+            const int64_t ni = d->dims[0], nj = d->dims[1];
+            if ((st = ensure_ws(d, (size_t)ni * nj * 4)) != EATSS_OK) return st;
+            cudaError_t e = launch_transpose((const float *)buffers[1], ni, nj, nj, (float *)d->ws, s);
+            if (e != cudaSuccess) return cuda_fail(e, "eatss_run(syrk layout pass)");
+            untranspose_nests(d, cn, d->ws);
+        }
         for (int i = 0; i < (int)cn.size(); i++) {
             if (only_nest >= 0 && i != only_nest) continue;
             ContractPlan p = plan_contraction(cn[i], tiles, sl);
@@ -794,18 +836,10 @@ static eatss_status run_impl(const eatss_kernel_desc *cd, int only_nest, const i
             int bx, by, rm, smem, sp;
             mttkrp_plan(d->dims.data(), tiles, &gx, &gy, &gz, &bx, &by, &rm, &smem, &sp);
             if (tc || sp > 1) {  // split partials (SIMT) / D lo + block partials (tensor): library-owned
-                int dev = 0;
-                cudaGetDevice(&dev);
                 const size_t need = tc ? mttkrp_tc_ws_floats(d->dims.data()) * 4
                                        : (size_t)sp * (size_t)d->buffer_elems[0] * 4;
-                if (d->ws_dev != dev || d->ws_bytes < need) {
-                    if (d->ws && d->ws_dev == dev) cudaFree(d->ws);  // never free another device's pointer here
-                    d->ws = nullptr;
-                    d->ws_bytes = 0;
-                    if ((e = cudaMalloc(&d->ws, need)) != cudaSuccess) return cuda_fail(e, "eatss_run(mttkrp workspace)");
-                    d->ws_bytes = need;
-                    d->ws_dev = dev;
-                }
+                eatss_status ws_st = ensure_ws(d, need);
+                if (ws_st != EATSS_OK) return ws_st;
             }
             if (tc) {  // events around the tcgen05 kernel alone (the D split and the block reduction outside)
                 e = launch_mttkrp_tc((float *)buffers[0], (const float *)buffers[1], (const float *)buffers[2],
@@ -1083,7 +1117,12 @@ int64_t eatss_launches_per_run(const eatss_kernel_desc *d, const int64_t *tiles)
         for (int i = 0; i < EATSS_MAX_BUFFERS; i++) b[i] = (void *)((uintptr_t)(1 << 20) * (uintptr_t)(i + 1));
         int64_t total = 0;
         const int sl = smem_limit_bytes();
-        for (auto &n : contraction_nests(d, b)) total += contraction_launches(n, plan_contraction(n, tiles, sl));
+        auto cn = contraction_nests(d, b);
+        if (simt_untranspose(d)) {
+            untranspose_nests(d, cn, b[EATSS_MAX_BUFFERS - 1]);
+            total += 1;  // the layout pass
+        }
+        for (auto &n : cn) total += contraction_launches(n, plan_contraction(n, tiles, sl));
         return total;
     }
     switch (d->kind) {

@@ -752,6 +752,31 @@ cudaError_t launch_contraction(const ContractNest &n, const ContractPlan &p, int
     return launch_typed<float>(n, p, carveout_pct, coverage_counts, s);
 }
 
+// dst[c][r] = src[r][c] (rows x cols fp32, row pitch lds; dst pitch rows): 32 x 32 shared tiles,
+// coalesced both ways.  The SIMT executor's layout pass for a transposed operand (syrk's A^T).
+__global__ void transpose_kernel(const float *__restrict__ src, int64_t rows, int64_t cols, int64_t lds,
+                                 float *__restrict__ dst) {
+    __shared__ float t[32][33];
+    const int64_t c0 = (int64_t)blockIdx.x * 32, r0 = (int64_t)blockIdx.y * 32;
+    for (int y = threadIdx.y; y < 32; y += blockDim.y) {
+        const int64_t r = r0 + y, c = c0 + threadIdx.x;
+        if (r < rows && c < cols) t[y][threadIdx.x] = src[r * lds + c];
+    }
+    __syncthreads();
+    for (int y = threadIdx.y; y < 32; y += blockDim.y) {
+        const int64_t c = c0 + y, r = r0 + threadIdx.x;
+        if (r < rows && c < cols) dst[c * rows + r] = t[threadIdx.x][y];
+    }
+}
+
+cudaError_t launch_transpose(const float *src, int64_t rows, int64_t cols, int64_t lds, float *dst, cudaStream_t s) {
+    if (rows <= 0 || cols <= 0) return cudaSuccess;
+    if ((rows + 31) / 32 > 65535) return cudaErrorInvalidConfiguration;
+    dim3 grid((unsigned)((cols + 31) / 32), (unsigned)((rows + 31) / 32)), block(32, 8);
+    transpose_kernel<<<grid, block, 0, s>>>(src, rows, cols, lds, dst);
+    return cudaGetLastError();
+}
+
 int contraction_launches(const ContractNest &n, const ContractPlan &p) {
     if (!p.staged || n.M <= 0 || n.N <= 0) return 1;
     int c = 0;

@@ -54,5 +54,7 @@ cudaError_t launch_contraction(const ContractNest &n, const ContractPlan &p, int
 // kernels one launch_contraction issues (the SIMT staged path adds a pre-pass when it splits the
 // wave tail along k)
 int contraction_launches(const ContractNest &n, const ContractPlan &p);
+// dst[c][r] = src[r][c]: fp32, rows x cols with row pitch lds -> cols x rows dense
+cudaError_t launch_transpose(const float *src, int64_t rows, int64_t cols, int64_t lds, float *dst, cudaStream_t s);
 
 }  // namespace eatss
