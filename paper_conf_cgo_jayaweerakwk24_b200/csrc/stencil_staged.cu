@@ -29,6 +29,12 @@ using tcm::su32;
 
 namespace {
 
+// Programmatic dependent launch (sweep t+1 of a time loop is launched while sweep t drains): the
+// dependent grid is scheduled early, then waits here until the previous grid has completed and its
+// writes are visible -- before any global access, since sweep t+1 writes the array sweep t reads.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;\n" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;\n" ::: "memory"); }
+
 __device__ __forceinline__ void bulk_row_g2s(void *dst, const void *src, unsigned bytes, uint64_t *bar) {
     asm volatile(
         "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n" ::"r"(su32(dst)),
@@ -70,6 +76,7 @@ __global__ void __launch_bounds__(256) jacobi2d_staged(float *__restrict__ dst, 
         mbar_init(&bar, 1);
         asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
     }
+    pdl_wait();
     __syncthreads();
     if (tid < 32) {
         if (tid == 0) mbar_expect_tx(&bar, (unsigned)(nr * W * 4));
@@ -230,11 +237,34 @@ __global__ void __launch_bounds__(256) heat3d_staged(float *__restrict__ dst, co
         asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
         asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&msrc)) : "memory");
     }
+    pdl_wait();
     __syncthreads();
     heat_tile(dst, &msrc, n, Ti, Tj, Tk, nbj, blockIdx.x, blockIdx.y, win, &bar, 0);
+    pdl_trigger();  // after this CTA's stores: the next sweep's launch overlaps this grid's tail
 }
 
 constexpr int kSmemTarget = 113 * 1024;  // at least two resident CTAs per SM
+
+// launch with programmatic stream serialization allowed (the kernel calls pdl_trigger / pdl_wait);
+// EATSS_STENCIL_PDL=0 launches normally (for comparison)
+template <typename... KArgs, typename... Args>
+cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, int smem, cudaStream_t s, Args... args) {
+    static const bool on = [] {
+        const char *e = getenv("EATSS_STENCIL_PDL");
+        return !(e && atoi(e) == 0);
+    }();
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = (size_t)smem;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = on ? 1 : 0;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
+}
 
 int jacobi_staged_smem(int64_t n, int64_t Ti, int64_t Tj) {
     const int64_t nr = std::min<int64_t>(Ti, n) + 2, W = std::min<int64_t>(Tj + 8, n);
@@ -276,8 +306,8 @@ cudaError_t launch_jacobi2d_staged(float *dst, const float *src, const float *bs
     cudaFuncSetAttribute(jacobi2d_staged<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     cudaFuncSetAttribute(jacobi2d_staged<false>, cudaFuncAttributePreferredSharedMemoryCarveout,
                          staged_carveout(smem, split_pct));
-    jacobi2d_staged<false><<<grid, block, smem, s>>>(dst, src, bsrc, n, (int)Ti, (int)Tj, nullptr);
-    return cudaGetLastError();
+    return launch_pdl(jacobi2d_staged<false>, grid, block, smem, s, dst, src, bsrc, n, (int)Ti, (int)Tj,
+                      (int32_t *)nullptr);
 }
 
 cudaError_t launch_heat3d_staged(float *dst, const float *src, int64_t n, int64_t Ti, int64_t Tj, int64_t Tk,
@@ -302,8 +332,8 @@ cudaError_t launch_heat3d_staged(float *dst, const float *src, int64_t n, int64_
     cudaFuncSetAttribute(heat3d_staged<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     cudaFuncSetAttribute(heat3d_staged<false>, cudaFuncAttributePreferredSharedMemoryCarveout,
                          staged_carveout(smem, split_pct));
-    heat3d_staged<false><<<grid, block, smem, s>>>(dst, m, n, (int)Ti, (int)Tj, (int)Tk, (int)nbj, nullptr);
-    return cudaGetLastError();
+    return launch_pdl(heat3d_staged<false>, grid, block, smem, s, dst, (const CUtensorMap)m, n, (int)Ti, (int)Tj,
+                      (int)Tk, (int)nbj, (int32_t *)nullptr);
 }
 
 }  // namespace eatss
