@@ -171,3 +171,68 @@ def test_eatss_pick_is_register_resident():
     tiles, _ = E.select_tiles(d, E.gpu_params_b200(), 50, 16)
     (p,) = E.plan(d, tiles)
     assert tiles == (16, 1024, 16) and p.passes == 1 and p.a_in_smem and p.vec == 4
+
+
+# ------------------------------------------------------------------ 4-D builtins (readings R-N8, R-N9)
+def test_fourd_descriptors_and_accounting():
+    d = E.desc_builtin("mttkrp", (512, 32, 512, 512))
+    assert d.num_loops == 4 and d.num_nests == 1 and d.num_buffers == 4
+    assert [d.buffer_elems(i) for i in range(4)] == [512 * 32, 512 ** 3, 512 * 32, 512 * 32]
+    assert d.flops == 2 * 512 * 32 * 512 * 512
+    assert d.bytes == 4 * (2 * 512 * 32 + 512 ** 3 + 2 * 512 * 32)
+    c = E.desc_builtin("conv-2d", (8192, 5))
+    assert c.num_loops == 4 and c.num_buffers == 3
+    assert [c.buffer_elems(i) for i in range(3)] == [8188 ** 2, 8192 ** 2, 25]
+    assert c.flops == 2 * 25 * 8188 ** 2
+    assert c.bytes == 4 * (8192 ** 2 + 25 + 8188 ** 2)
+    with pytest.raises(E.EatssError):
+        E.desc_builtin("conv-2d", (4, 5))  # filter larger than the image
+    # model view (rules 2-8, tests/test_oracle_model.py::test_mttkrp_conv2d_derivation)
+    assert d.model_info(0, 16) == (1, 4, [0, 48, 0, 0])
+    assert c.model_info(0, 16) == (1, 3, [0, 32, 0, 0])
+
+
+def test_mttkrp_plan_split_and_launches():
+    d = E.desc_builtin("mttkrp", (512, 32, 512, 512))
+    (p,) = E.plan(d, (128, 32, 16, 16))
+    assert (p.grid_x, p.grid_y) == (1, 4)
+    assert p.block_x * p.block_y == 128 and p.rm == 8 and p.vec == 4
+    # (k-tile, l-tile) pairs split until ~2 CTAs per SM: 32 x 32 pairs over 4 blocks
+    assert p.grid_z == p.passes and 1 < p.grid_z <= 32 * 32
+    assert E.launches_per_run(d, (128, 32, 16, 16)) == 2          # kernel + split-order reduction
+    (q,) = E.plan(d, (7, 12, 5, 9))                                # Tl % 4 != 0: general path
+    assert q.vec == 1 and q.grid_z == 1
+    d.set_exec(split_pct=50, engine=2)
+    # D lo, tcgen05 kernel, reduction (-1 only without a CUDA driver: no TMA descriptor encoder)
+    import torch
+    assert E.launches_per_run(d, (1, 32, 128, 32)) == (3 if torch.cuda.is_available() else -1)
+    assert E.launches_per_run(d, (128, 32, 16, 16)) == -1          # not MMA-legal on the tensor engine
+
+
+@pytest.mark.parametrize("tiles", [(16, 64, 5, 5), (8, 152, 5, 5), (1024, 1024, 5, 5), (7, 13, 3, 3)])
+def test_conv2d_plan_invariants(tiles):
+    n, f = 8192, 5
+    m = n - f + 1
+    d = E.desc_builtin("conv-2d", (n, f))
+    (p,) = E.plan(d, tiles)
+    Ti, Tj = min(tiles[0], m), min(tiles[1], m)
+    assert p.grid_x == -(-m // Tj) and p.grid_y == -(-m // Ti)
+    assert 1 <= p.block_x <= 256
+    assert (p.tile[2], p.tile[3]) == (min(tiles[2], f), min(tiles[3], f))
+    if Tj % 4 == 0:  # fast path: the (row chunk + halo) x window fits the per-CTA budget
+        assert p.vec == 4 and 0 < p.smem_bytes <= 2 * 64 * 1024 and p.rm >= 1
+    else:
+        assert p.vec == 1
+    assert E.launches_per_run(d, tiles) == 1
+
+
+def test_syrk_simt_layout_pass_counted():
+    d = E.desc_builtin("syrk", (4000, 4000))
+    d.set_exec(split_pct=50, engine=1)
+    g = E.desc_builtin("gemm", (4000, 4000, 4000))
+    g.set_exec(split_pct=50, engine=1)
+    # syrk = the gemm-shaped SIMT kernel(s) + the A -> A^T layout pass
+    assert E.launches_per_run(d, (16, 1024, 16)) == E.launches_per_run(g, (16, 1024, 16)) + 1
+    (ps,) = E.plan(d, (16, 1024, 16))
+    (pg,) = E.plan(g, (16, 1024, 16))
+    assert (ps.block_x, ps.block_y, ps.rm, ps.rn, ps.vec) == (pg.block_x, pg.block_y, pg.rm, pg.rn, pg.vec)
