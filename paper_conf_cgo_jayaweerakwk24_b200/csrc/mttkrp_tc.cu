@@ -12,7 +12,9 @@
 // its tf32 lo half is NOT materialised in HBM (that would triple the traffic) -- converter warps
 // form it in shared memory from the TMA-landed tile (same swizzled layout, elementwise), as
 //   hi = B itself (the tensor core truncates fp32 to tf32), lo = rna_tf32(B - rz_tf32(B)),
-// and D's lo half (64 KB) is formed once per call.  3xTF32: T = Bhi*Dhi + Bhi*Dlo + Blo*Dhi.
+// and D's lo half (64 KB) is formed once per call.  3xTF32: T = Bhi*Dhi + Bhi*Dlo + Blo*Dhi, issued as
+// two MMAs per 8-k step -- Bhi x [Dhi | Dlo] (N = 2 NJ) and Blo x Dhi (N = NJ) -- because the small-N
+// MMAs are bound by their per-instruction cost (measured: 12 -> 8 MMAs per stage).
 // Epilogue: a thread per TMEM lane (= one (i, k) row) scales its N accumulators by C[k][:], the
 // 128 rows are reduced across lanes (shuffle reduce-scatter) and warps (shared memory, fixed
 // order) and written as one partial row per block; a second kernel adds the nk/128 partials of
@@ -26,6 +28,7 @@
 
 #include <algorithm>
 #include <cstdint>
+#include <cstdlib>
 
 #include "tc_ptx.cuh"
 
@@ -44,6 +47,7 @@ struct Args {
     int nblk;   // ni * nk / 128 row blocks
     int nkb;    // nl / 32
     int S;      // ring stages
+    int dbg;    // development only (EATSS_MTC_DBG): 1 skip the lo conversion, 2 skip the MMAs
     const float *C;
     float *part;  // [nblk][nj]
 };
@@ -65,7 +69,9 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     constexpr int A_BYTES = BM * BK * 4;       // 16 KB
     constexpr int D_BYTES = BK * NJ * 4;       // NJ/32 groups of 32 l x 128 B
     constexpr int HSTAGE = 2 * A_BYTES + 2 * D_BYTES;  // ring stage: B hi tile, B lo tile, D hi, D lo
-    constexpr uint32_t ID = idesc(NJ, 1, false);
+    constexpr uint32_t ID = idesc(NJ, 1, false);       // A_lo x D_hi          (N = NJ)
+    constexpr uint32_t ID2 = idesc(2 * NJ, 1, false);  // A_hi x [D_hi | D_lo] (N = 2 NJ: both D tiles are
+                                                       // adjacent 32-column groups of one MN-major operand)
     const int SH = p.S;                        // ring depth
     // the lo tile of a stage is rewritten only after the TMA of a later use of that stage landed,
     // which the producer issues only after the MMAs of the earlier use finished
@@ -90,7 +96,8 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         }
         asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
     }
-    constexpr uint32_t TCOLS = 2 * NJ <= 32 ? 32 : 2 * NJ <= 64 ? 64 : 2 * NJ <= 128 ? 128 : 2 * NJ <= 256 ? 256 : 512;
+    // two accumulator buffers of 2 NJ columns: [hi*hi + lo*hi | hi*lo], summed by the epilogue
+    constexpr uint32_t TCOLS = 4 * NJ <= 32 ? 32 : 4 * NJ <= 64 ? 64 : 4 * NJ <= 128 ? 128 : 4 * NJ <= 256 ? 256 : 512;
     if (warp == 2) {
         asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;\n" ::"r"(su32(tmem_slot)),
                      "r"(TCOLS)
@@ -127,7 +134,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                 const int bd = gc & 1;
                 if (gc >= 2) mbar_wait(dempty + bd, (unsigned)(((gc - 2) >> 1) & 1));
                 fence_after();
-                const uint32_t d = tmem + (uint32_t)(bd * NJ);
+                const uint32_t d = tmem + (uint32_t)(bd * 2 * NJ);
                 for (int kb = 0; kb < p.nkb; kb++, it++) {
                     const int s = it % SH;
                     mbar_wait(full + s, (unsigned)((it / SH) & 1));
@@ -137,14 +144,13 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                     unsigned char *lo = st + A_BYTES;
 #pragma unroll
                     for (int ks = 0; ks < BK / 8; ks++) {
+                        if (p.dbg & 2) break;
                         const uint64_t ahi = desc_sw128(st + ks * 32, 16u, 1024u);
                         const uint64_t alo = desc_sw128(lo + ks * 32, 16u, 1024u);
-                        const uint64_t bhi = desc_sw128(st + 2 * A_BYTES + ks * 1024, (uint32_t)(BK * 128), 512u, 1);
-                        const uint64_t blo =
-                            desc_sw128(st + 2 * A_BYTES + D_BYTES + ks * 1024, (uint32_t)(BK * 128), 512u, 1);
-                        mma_ss<1>(d, ahi, bhi, ID, (kb == 0 && ks == 0) ? 0u : 1u);
-                        mma_ss<1>(d, ahi, blo, ID, 1u);
-                        mma_ss<1>(d, alo, bhi, ID, 1u);
+                        // the D hi groups, then the D lo groups: LBO = stride of 32-column groups
+                        const uint64_t bcat = desc_sw128(st + 2 * A_BYTES + ks * 1024, (uint32_t)(BK * 128), 512u, 1);
+                        mma_ss<1>(d, ahi, bcat, ID2, (kb == 0 && ks == 0) ? 0u : 1u);
+                        mma_ss<1>(d, alo, bcat, ID, 1u);
                     }
                     mma_commit<1>(empty + s);
                 }
@@ -162,6 +168,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                 float4 *dst = reinterpret_cast<float4 *>(smem + (size_t)s * HSTAGE + A_BYTES);
 #pragma unroll
                 for (int v = 0; v < A_BYTES / 16 / (NCONV * 32); v++) {
+                    if (p.dbg & 1) break;
                     const int e = ct + v * NCONV * 32;  // consecutive threads: consecutive 16-byte chunks
                     const float4 x = src[e];
                     dst[e] = make_float4(lo_of(x.x), lo_of(x.y), lo_of(x.z), lo_of(x.w));
@@ -186,10 +193,12 @@ __global__ void __launch_bounds__(NTHREADS, 1)
 #pragma unroll
             for (int c0 = 0; c0 < NJ; c0 += 16) {
                 uint32_t r[16];
-                tmem_ld16(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(bd * NJ + c0), r);
+                uint32_t r2[16];
+                tmem_ld16(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(bd * 2 * NJ + c0), r);
+                tmem_ld16(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(bd * 2 * NJ + NJ + c0), r2);
                 wait_ld();
 #pragma unroll
-                for (int c = 0; c < 16; c++) v[c0 + c] = __uint_as_float(r[c]);
+                for (int c = 0; c < 16; c++) v[c0 + c] = __uint_as_float(r[c]) + __uint_as_float(r2[c]);
             }
             fence_before();
             __syncwarp();
@@ -268,6 +277,7 @@ cudaError_t launch_mttkrp_tc(float *A, const float *B, const float *C, const flo
     p.nblk = (int)(p.ni * p.nk / BM);
     p.nkb = (int)(p.nl / BK);
     p.C = C;
+    p.dbg = getenv("EATSS_MTC_DBG") ? atoi(getenv("EATSS_MTC_DBG")) : 0;
     float *dlo = ws;
     p.part = ws + p.nj * p.nl;
     CUtensorMap mB, mDhi, mDlo;
