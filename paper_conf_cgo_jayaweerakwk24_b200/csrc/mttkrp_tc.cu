@@ -299,6 +299,7 @@ cudaError_t launch_mttkrp_tc(float *A, const float *B, const float *C, const flo
         cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
         auto bytes = [&](int sh) { return 1024 + sh * hstage + 256 + NEPI * nj * 4; };
         p.S = SMAX;
+        if (const char *ev_s = getenv("EATSS_MTC_STAGES")) p.S = std::max(2, std::min(8, atoi(ev_s)));  // development
         while (p.S > 2 && bytes(p.S) > optin) p.S--;
         const int smem = bytes(p.S);
         cudaError_t r = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
