@@ -18,6 +18,7 @@
 
 #include <algorithm>
 #include <cstdint>
+#include <cstdlib>
 
 #include "tc_ptx.cuh"
 
@@ -51,6 +52,7 @@ struct CvArgs {
     int64_t units;     // gy * cpt * gx work units (tile row-chunks)
     int slot_f;        // floats per window slot
     int nslot;         // 1: one CTA per unit; 2: persistent CTAs with a prefetching second slot
+    int tma;           // 1: the window is one 2-D TMA box {wc, rc + f - 1} (wc <= 256, rc + f - 1 <= 256)
     int32_t *counts;
 };
 
@@ -78,8 +80,10 @@ __device__ __forceinline__ Unit unit_of(const CvArgs &a, int64_t u) {
 // unit (the default: more CTAs resident per SM, no per-CTA unit loop).  F > 0: compile-time filter size with the
 // register ring; F == 0: runtime f, direct shared reads.
 template <int F, bool COVER>
-__global__ void __launch_bounds__(256) conv2d_kernel(CvArgs a) {
-    extern __shared__ __align__(16) float win[];
+__global__ void __launch_bounds__(256) conv2d_kernel(CvArgs a, const __grid_constant__ CUtensorMap wmap) {
+    extern __shared__ __align__(128) unsigned char win_raw[];
+    // TMA destinations must be 128-byte aligned
+    float *win = reinterpret_cast<float *>(win_raw + ((128u - (su32(win_raw) & 127u)) & 127u));
     __shared__ uint64_t bar[2];
     constexpr int NV = F > 0 ? (F + 6) / 4 : 1;  // float4 per row segment: 4 + F - 1 floats
     const int f = F > 0 ? F : a.f;
@@ -120,6 +124,13 @@ __global__ void __launch_bounds__(256) conv2d_kernel(CvArgs a) {
         const unsigned rowbytes = (unsigned)((ce - w.tj0) * 4);
         const int wr = w.rows + f - 1;  // window rows (c0 + wr <= n always)
         float *dst = win + slot * a.slot_f;
+        if (a.tma) {  // one box; rows / columns past the image are zero-filled (never used by an output)
+            if (tid == 0) {
+                mbar_expect_tx(&bar[slot], (unsigned)(a.wc * (a.rc + f - 1) * 4));
+                tcm::tma_2d<1>(dst, &wmap, (int)w.tj0, (int)w.c0, su32(&bar[slot]));
+            }
+            return;
+        }
         if (tid == 0) mbar_expect_tx(&bar[slot], rowbytes * (unsigned)wr);
         __syncwarp(nt == 32 ? 0xffffffffu : (1u << nt) - 1u);
         for (int r = tid; r < wr; r += nt)
@@ -278,16 +289,26 @@ cudaError_t launch_conv2d(float *out, const float *inp, const float *W, int64_t 
     a.units = gy * a.cpt * gx;
     a.slot_f = smem / 4;  // floats of the (single) slot
     a.nslot = 1;
+    CUtensorMap wmap{};
+    a.tma = 0;
+    static const bool tma_on = [] {
+        const char *e = getenv("EATSS_CONV_TMA");
+        return !(e && atoi(e) == 0);
+    }();
+    if (tma_on && !counts && wc <= 256 && rc + f - 1 <= 256 && tcm::encode_fn() &&
+        tcm::make_map(&wmap, inp, n, n, n, wc, (int)(rc + f - 1), CU_TENSOR_MAP_SWIZZLE_NONE))
+        a.tma = 1;
+    smem += 128;  // manual 128-byte alignment of the window
     if (a.units >= (int64_t)1 << 31) return cudaErrorInvalidConfiguration;
     if (launched) (*launched)++;
     cudaError_t e = cudaSuccess;
 #define EATSS_CV(FV)                                                                                       \
     if (counts) {                                                                                          \
-        conv2d_kernel<FV, true><<<(unsigned)std::min<int64_t>(a.units, 65535), threads, 0, s>>>(a);        \
+        conv2d_kernel<FV, true><<<(unsigned)std::min<int64_t>(a.units, 65535), threads, 0, s>>>(a, wmap);  \
     } else {                                                                                               \
         e = cudaFuncSetAttribute(conv2d_kernel<FV, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem); \
         if (e != cudaSuccess) return e;                                                                    \
-        conv2d_kernel<FV, false><<<(unsigned)a.units, threads, smem, s>>>(a);                              \
+        conv2d_kernel<FV, false><<<(unsigned)a.units, threads, smem, s>>>(a, wmap);                        \
     }
     switch (f) {
         case 3: EATSS_CV(3) break;
