@@ -4,3 +4,7 @@ timeout 600 python -m pytest tests/test_gpu_fourd.py -x -q -k "conv2d" --timeout
 tail -2 gpurun_out/pytest_conv.log; cat gpurun_out/conv_tma.txt
 timeout 2400 python harness/candidates.py --confirm 7 --out gpurun_out/candidates_r01g.jsonl > gpurun_out/candidates_r01g.log 2>&1; echo "cand $?"
 tail -15 gpurun_out/candidates_r01g.log | cut -c1-300
+T=scripts/time_kernel.py
+{ for at in 0 1; do EATSS_MTC_ATMEM=$at timeout 120 python $T mttkrp 512,32,512,512 1,32,128,32 --engine 2 --iters 20 2>&1 | tail -1 | sed "s/^/atmem$at /"; done; } > gpurun_out/mtc_atmem.txt 2>&1
+EATSS_MTC_ATMEM=1 timeout 600 python -m pytest tests/test_gpu_fourd.py -x -q -k "tensor" --timeout 300 -p no:cacheprovider > gpurun_out/pytest_atmem.log 2>&1; echo "pytest atmem rc=$?" >> gpurun_out/pytest_atmem.log
+cat gpurun_out/mtc_atmem.txt; tail -2 gpurun_out/pytest_atmem.log
