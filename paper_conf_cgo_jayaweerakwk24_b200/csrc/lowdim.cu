@@ -21,6 +21,7 @@
 
 #include <algorithm>
 #include <cstdint>
+#include <cstdlib>
 
 namespace eatss {
 
@@ -185,7 +186,25 @@ cudaError_t launch_lowdim(const LowdimArgs &a0, bool row, bool col, bool upd, cu
     a.Tj = (int)std::min<int64_t>(a.Tj, (int64_t)LD_MAXG * LPR * V);
     a.Ti = (int)std::min<int64_t>(a.Ti, a.nx);
     const int64_t gx = (a.ny + a.Tj - 1) / a.Tj, ntile_i = (a.nx + a.Ti - 1) / a.Ti;
-    const int64_t gy = std::min<int64_t>(ntile_i, 65535);  // > 65535 row tiles: CTAs walk several
+    int64_t gy = std::min<int64_t>(ntile_i, 65535);  // > 65535 row tiles: CTAs walk several
+    // column form: each CTA adds one atomic per column, so with narrow row tiles (the EATSS picks)
+    // the atomics, not the matrix stream, dominate; CTAs then walk several row tiles each, the grid
+    // sized to ~8 resident CTAs per SM (one atomic per column and CTA). EATSS_LOWDIM_WALK=0: one tile
+    // per CTA.
+    static const bool walk = [] {
+        const char *e = getenv("EATSS_LOWDIM_WALK");
+        return !(e && atoi(e) == 0);
+    }();
+    if (col && walk) {
+        static int nsm = 0;
+        if (!nsm) {
+            int dev = 0;
+            cudaGetDevice(&dev);
+            if (cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || nsm <= 0) nsm = 148;
+        }
+        const int64_t target = 8LL * nsm;
+        gy = std::max<int64_t>(1, std::min<int64_t>(gy, (target + gx - 1) / gx));
+    }
     if (gx > INT32_MAX) return cudaErrorInvalidConfiguration;
     dim3 grid((unsigned)gx, (unsigned)gy), block(LD_THREADS);
 #define LDK(R, C, U)                                                                   \
