@@ -48,7 +48,6 @@ struct Args {
     int nkb;    // nl / 32
     int S;      // ring stages
     int dbg;    // development only (EATSS_MTC_DBG): 1 skip the lo conversion, 2 skip the MMAs
-    int atmem;  // 1: B lo half in TMEM (converter thread = TMEM lane = row; A_lo x D_hi as a TS-MMA)
     const float *C;
     float *part;  // [nblk][nj]
 };
@@ -97,10 +96,8 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         }
         asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
     }
-    // two accumulator buffers of 2 NJ columns: [hi*hi + lo*hi | hi*lo], summed by the epilogue; with
-    // atmem the B lo tiles follow at column 4 NJ (32 columns per stage)
-    constexpr uint32_t TCOLS = 512;
-    const uint32_t lo_col0 = 4 * NJ;
+    // two accumulator buffers of 2 NJ columns: [hi*hi + lo*hi | hi*lo], summed by the epilogue
+    constexpr uint32_t TCOLS = 4 * NJ <= 32 ? 32 : 4 * NJ <= 64 ? 64 : 4 * NJ <= 128 ? 128 : 4 * NJ <= 256 ? 256 : 512;
     if (warp == 2) {
         asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;\n" ::"r"(su32(tmem_slot)),
                      "r"(TCOLS)
@@ -149,12 +146,11 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                     for (int ks = 0; ks < BK / 8; ks++) {
                         if (p.dbg & 2) break;
                         const uint64_t ahi = desc_sw128(st + ks * 32, 16u, 1024u);
-                        const uint64_t alo = p.atmem ? 0ull : desc_sw128(lo + ks * 32, 16u, 1024u);
+                        const uint64_t alo = desc_sw128(lo + ks * 32, 16u, 1024u);
                         // the D hi groups, then the D lo groups: LBO = stride of 32-column groups
                         const uint64_t bcat = desc_sw128(st + 2 * A_BYTES + ks * 1024, (uint32_t)(BK * 128), 512u, 1);
                         mma_ss<1>(d, ahi, bcat, ID2, (kb == 0 && ks == 0) ? 0u : 1u);
-                        if (p.atmem) mma_ts(d, tmem + lo_col0 + (uint32_t)(s * BK + ks * 8), bcat, ID, 1u);
-                        else mma_ss<1>(d, alo, bcat, ID, 1u);
+                        mma_ss<1>(d, alo, bcat, ID, 1u);
                     }
                     mma_commit<1>(empty + s);
                 }
@@ -170,27 +166,6 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                 mbar_wait(full + s, (unsigned)((it / SH) & 1));
                 const float4 *src = reinterpret_cast<const float4 *>(smem + (size_t)s * HSTAGE);
                 float4 *dst = reinterpret_cast<float4 *>(smem + (size_t)s * HSTAGE + A_BYTES);
-                if (p.atmem) {
-                    // this thread = row m = TMEM lane (warp quarter q): its 32 k-values are the row's eight
-                    // 16-byte chunks of the SW128 tile, chunk c stored at position c ^ (m & 7)
-                    const int m = ((warp & 3) << 5) + lane;
-                    uint32_t lv[32];
-#pragma unroll
-                    for (int c = 0; c < 8; c++) {
-                        const float4 x = src[m * 8 + (c ^ (m & 7))];
-                        lv[4 * c] = __float_as_uint(lo_of(x.x)); lv[4 * c + 1] = __float_as_uint(lo_of(x.y));
-                        lv[4 * c + 2] = __float_as_uint(lo_of(x.z)); lv[4 * c + 3] = __float_as_uint(lo_of(x.w));
-                    }
-                    const uint32_t ta = tmem + ((uint32_t)((warp & 3) * 32) << 16) + lo_col0 + (uint32_t)(s * BK);
-#pragma unroll
-                    for (int c = 0; c < 4; c++)
-                        tmem_st8(ta + 8 * c, *reinterpret_cast<const uint32_t(*)[8]>(lv + 8 * c));
-                    wait_st();
-                    fence_before();
-                    __syncwarp();
-                    if (lane == 0) mbar_arrive(conv + s);
-                    continue;
-                }
 #pragma unroll
                 for (int v = 0; v < A_BYTES / 16 / (NCONV * 32); v++) {
                     if (p.dbg & 1) break;
@@ -303,7 +278,6 @@ cudaError_t launch_mttkrp_tc(float *A, const float *B, const float *C, const flo
     p.nkb = (int)(p.nl / BK);
     p.C = C;
     p.dbg = getenv("EATSS_MTC_DBG") ? atoi(getenv("EATSS_MTC_DBG")) : 0;
-    p.atmem = getenv("EATSS_MTC_ATMEM") ? atoi(getenv("EATSS_MTC_ATMEM")) : 0;
     float *dlo = ws;
     p.part = ws + p.nj * p.nl;
     CUtensorMap mB, mDhi, mDlo;
@@ -328,7 +302,6 @@ cudaError_t launch_mttkrp_tc(float *A, const float *B, const float *C, const flo
         if (const char *ev_s = getenv("EATSS_MTC_STAGES")) p.S = std::max(2, std::min(8, atoi(ev_s)));  // development
         while (p.S > 2 && bytes(p.S) > optin) p.S--;
         const int smem = bytes(p.S);
-        if (p.atmem && 4 * nj + p.S * BK > 512) p.atmem = 0;  // TMEM: accumulators + per-stage lo tiles
         cudaError_t r = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
         if (r != cudaSuccess) return r;
         if (ev) cudaEventRecord(ev[0], s);
