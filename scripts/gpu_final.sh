@@ -9,3 +9,4 @@ timeout 600 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/b
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/launches.csv python bench.py --steps 5 --warmup 3 --e2e-steps 1 --no-cpu-baseline --no-secondary --no-configs > gpurun_out/bench_ncu.log 2>&1; echo "ncu list $?"
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:tc_mma -s 3 -c 1 -o gpurun_out/prof_tcm_r01g -f python bench.py --steps 3 --warmup 3 --e2e-steps 1 --no-cpu-baseline --no-secondary --no-configs > /dev/null 2>&1; echo "ncu tcm $?"
 tail -3 gpurun_out/pytest_gpu.log; tail -2 gpurun_out/smoke.log; tail -c 400 gpurun_out/bench.log
+timeout 120 python scripts/time_kernel.py mttkrp 512,32,512,512 1,32,128,32 --engine 2 --iters 20 > gpurun_out/mtc_final.txt 2>&1; cat gpurun_out/mtc_final.txt
