@@ -21,7 +21,11 @@
  *     row-major, contiguous, 16-byte aligned, non-aliasing, in the order documented
  *     per builtin below.  The library never frees them.
  *   - Descriptors are library-owned (create / destroy); a descriptor may be used by
- *     one thread at a time (eatss_run caches CUDA graphs inside it).
+ *     one thread at a time (eatss_run caches CUDA graphs inside it).  A descriptor may also
+ *     own device scratch, allocated on the first run that needs it and freed with the
+ *     descriptor: mttkrp's split partials / tensor-path block partials, SIMT syrk's A^T
+ *     layout copy, eatss_run_host's device buffers.  Runs of ONE descriptor on different
+ *     streams must therefore be ordered by the caller (they share that scratch).
  *   - eatss_run is asynchronous on `stream`: argument and launch-configuration
  *     errors are returned synchronously; device faults surface on the stream.
  *   - No CPU fallback exists: without a CUDA device eatss_run returns EATSS_E_CUDA.
