@@ -198,3 +198,34 @@ def test_mttkrp_tensor_full_size(cuda_device):
     ii, jj = g.integers(0, ni, 600), g.integers(0, nj, 600)
     ref = O.mttkrp_entries(ii, jj, A0, B, C, D)
     assert np.linalg.norm(got[ii, jj] - ref) / np.linalg.norm(ref) <= 1e-5
+
+
+# ------------------------------------------------------------------ degenerate cases
+@pytest.mark.parametrize("n,f,tiles", [(16, 1, (4, 8, 1, 1)), (12, 12, (16, 64, 5, 5)), (13, 12, (1, 4, 1, 1)),
+                                       (64, 5, (1024, 1024, 5, 5)), (8, 7, (16, 64, 7, 7)), (264, 5, (16, 64, 5, 5))])
+def test_conv2d_degenerate(cuda_device, n, f, tiles):
+    """1x1 filter (a scaled copy), filter = image (one output), two outputs per row, tiles larger than
+    the output, the TMA-window path with ragged last tiles (m = 260 = 4 * 64 + 4 columns, 16 * 16 + 4 rows)."""
+    inp, W = synth.small_int((n, n), 21), synth.small_int((f, f), 22)
+    m = n - f + 1
+    d = E.desc_builtin("conv-2d", (n, f))
+    out = dev(np.full((m, m), 7.0))
+    E.run(d, tiles, [out, dev(inp), dev(W)])
+    assert np.array_equal(host(out), O.conv2d(inp, W))
+
+
+@pytest.mark.parametrize("dims,tiles", [((1, 4, 1, 4), (128, 32, 16, 16)), ((5, 4, 1, 1), (1, 1, 1, 1)),
+                                        ((3, 8, 7, 4), (1024, 1024, 1024, 1024)), ((33, 4, 2, 8), (16, 4, 1, 4)),
+                                        ((2, 32, 3, 36), (128, 32, 16, 16))])
+def test_mttkrp_degenerate(cuda_device, dims, tiles):
+    """Single row / rank 4 / single-element reductions / tiles larger than every extent."""
+    ni, nj, nk, nl = dims
+    A0, B, C, D = (synth.small_int(s, 30 + i, -2, 2) for i, s in enumerate(((ni, nj), (ni, nk, nl), (nk, nj), (nl, nj))))
+    d = E.desc_builtin("mttkrp", dims)
+    b = [dev(A0), dev(B), dev(C), dev(D)]
+    E.run(d, tiles, b)
+    assert np.array_equal(host(b[0]), O.mttkrp(A0, B, C, D))
+    counts = torch.zeros(ni * nj * nk * nl, dtype=torch.int32, device="cuda")
+    E.coverage(d, 0, tiles, counts)
+    torch.cuda.synchronize()
+    assert int(counts.min()) == 1 and int(counts.max()) == 1
