@@ -73,7 +73,9 @@ def run_shard(kind, dims, tiles, rank, world, X, backend, alpha=1.5, beta=1.2):
          syrk_rows(alpha, beta, Crows, Afull, r0) -> Crows   [rows r0.. of a*A*A^T + b*C]
          ccsd(t3slab, t2, v2slab) -> t3slab
          all_gather_rows(local, total_rows, row_ranges) -> full
+         zeros(shape) -> a zero-initialised output block (optional: numpy when absent)
        Returns (outputs dict, row range)."""
+    zeros = getattr(backend, "zeros", lambda shape: np.zeros(shape, np.float32))
     Ti = tiles[0]
     if kind == "gemm":
         ni = dims[0]
@@ -83,18 +85,18 @@ def run_shard(kind, dims, tiles, rank, world, X, backend, alpha=1.5, beta=1.2):
     if kind == "2mm":
         ni, nj, nk, nl = dims
         r0, r1 = shard_rows(ni, world, Ti, rank)
-        tmp = backend.gemm(alpha, 0.0, np.zeros((r1 - r0, nj), np.float32), X["A"][r0:r1], X["B"], True)
+        tmp = backend.gemm(alpha, 0.0, zeros((r1 - r0, nj)), X["A"][r0:r1], X["B"], True)
         D = backend.gemm(1.0, beta, X["D"][r0:r1], tmp, X["C"], False)
         return {"tmp": tmp, "D": D}, (r0, r1)
     if kind == "3mm":
         ni, nj, nk, nl, nm = dims
         r0, r1 = shard_rows(ni, world, Ti, rank)
         f0, f1 = shard_rows(nj, world, Ti, rank)
-        E = backend.gemm(1.0, 0.0, np.zeros((r1 - r0, nj), np.float32), X["A"][r0:r1], X["B"], True)
-        Floc = backend.gemm(1.0, 0.0, np.zeros((f1 - f0, nl), np.float32), X["C"][f0:f1], X["D"], True)
+        E = backend.gemm(1.0, 0.0, zeros((r1 - r0, nj)), X["A"][r0:r1], X["B"], True)
+        Floc = backend.gemm(1.0, 0.0, zeros((f1 - f0, nl)), X["C"][f0:f1], X["D"], True)
         ranges = [shard_rows(nj, world, Ti, r) for r in range(world)]
         F = backend.all_gather_rows(Floc, nj, ranges)  # the one exchange step (NCCL all_gather)
-        G = backend.gemm(1.0, 0.0, np.zeros((r1 - r0, nl), np.float32), E, F, True)
+        G = backend.gemm(1.0, 0.0, zeros((r1 - r0, nl)), E, F, True)
         return {"E": E, "F": F, "G": G}, (r0, r1)
     if kind == "syrk":
         ni, nj = dims
@@ -111,12 +113,20 @@ def run_shard(kind, dims, tiles, rank, world, X, backend, alpha=1.5, beta=1.2):
 
 # ------------------------------------------------------------------ GPU backend (libeatss)
 class CudaBackend:
-    """Shard compute through libeatss.so; arrays are host numpy in / device tensors inside."""
+    """Shard compute through libeatss.so on device tensors (host numpy arrays are uploaded on use;
+    main() uploads the inputs once, outside the timed loop)."""
 
     def __init__(self, dev, tiles, dist=None, timing=False):
         import torch
         import paper_conf_cgo_jayaweerakwk24_b200 as E
         self.torch, self.E, self.dev, self.tiles, self.dist = torch, E, dev, tiles, dist
+        self._descs = {}  # one descriptor per shape: it owns device scratch (e.g. syrk's A^T copy)
+
+    def _desc(self, kind, dims):
+        key = (kind, tuple(dims))
+        if key not in self._descs:
+            self._descs[key] = self.E.desc_builtin(kind, dims)
+        return self._descs[key]
 
     def _t(self, x):
         if isinstance(x, np.ndarray):
@@ -127,7 +137,7 @@ class CudaBackend:
         C, A, B = self._t(C), self._t(A), self._t(B)
         M, K = A.shape
         N = B.shape[1]
-        d = self.E.desc_builtin("gemm", (M, N, K))
+        d = self._desc("gemm", (M, N, K))
         d.set_scalars(alpha, 0.0 if init_zero else beta)
         if init_zero:
             C.zero_()
@@ -138,7 +148,7 @@ class CudaBackend:
         Crows, Afull = self._t(Crows), self._t(Afull)
         ni, nj = Afull.shape
         rows = Crows.shape[0]
-        d = self.E.desc_builtin("syrk", (ni, nj, r0, rows))  # rows [r0, r0+rows) of C = a*A*A^T + b*C
+        d = self._desc("syrk", (ni, nj, r0, rows))  # rows [r0, r0+rows) of C = a*A*A^T + b*C
         d.set_scalars(alpha, beta)
         self.E.run(d, self.tiles, [Crows, Afull])
         return Crows
@@ -148,13 +158,18 @@ class CudaBackend:
         H3 = v2.shape[0]
         H7, P4, P5, H1 = t2.shape
         _, H2, P6, _ = v2.shape
-        d = self.E.desc_builtin("ccsd_t_d1", (H3, H2, H1, P6, P5, P4, H7))
+        d = self._desc("ccsd_t_d1", (H3, H2, H1, P6, P5, P4, H7))
         self.E.run(d, self.tiles, [t3, t2, v2])
         return t3
+
+    def zeros(self, shape):
+        return self.torch.zeros(shape, dtype=self.torch.float32, device=self.dev)
 
     def all_gather_rows(self, local, total_rows, ranges):
         torch = self.torch
         local = self._t(local)
+        if self.dist is None:  # one rank: its shard is the whole array
+            return local
         maxr = max(r1 - r0 for r0, r1 in ranges)
         buf = torch.zeros((maxr,) + tuple(local.shape[1:]), dtype=local.dtype, device=self.dev)
         buf[: local.shape[0]] = local
@@ -189,12 +204,14 @@ def main():
     waf = 4 if a.kind == "ccsd_t_d1" else 16
     tiles, _ = E.select_tiles(d_full, E.gpu_params_query(local), a.split, waf)
     X = make_inputs(a.kind, dims)
+    # inputs resident in HBM before the timed loop (only the shard compute and the exchange are timed)
+    Xd = {k: torch.from_numpy(np.ascontiguousarray(v)).to(dev) for k, v in X.items()}
     if a.kind == "ccsd_t_d1":
-        X["t3"] = np.zeros((n,) * 6, np.float32)
+        Xd["t3"] = torch.zeros((n,) * 6, dtype=torch.float32, device=dev)
     be = CudaBackend(dev, tiles, dist if ws > 1 else None)
 
-    def once():
-        return run_shard(a.kind, dims, tiles, rank, ws, X, be)
+    def once():  # in/out arrays (C, D, t3) keep accumulating across timed steps; parity re-uploads below
+        return run_shard(a.kind, dims, tiles, rank, ws, Xd, be)
 
     for _ in range(a.warmup):
         out, rr = once()
@@ -210,7 +227,13 @@ def main():
     torch.cuda.synchronize()
     mj1 = E.energy_mj(local)
     ms = s.elapsed_time(e) / a.steps
-    # parity on sampled entries of this shard (fp32 tolerance vs fp64 oracle)
+    # parity on sampled entries of this shard (fp32 tolerance vs fp64 oracle): one step from fresh inputs
+    for k, v in X.items():
+        Xd[k].copy_(torch.from_numpy(np.ascontiguousarray(v)))
+    if a.kind == "ccsd_t_d1":
+        Xd["t3"].zero_()
+    out, rr = once()
+    torch.cuda.synchronize()
     err = parity_sample(a.kind, dims, X, out, rr, O)
     v = torch.tensor([ms, (mj1 - mj0) / 1e3 / a.steps, err], dtype=torch.float64, device=dev)
     if ws > 1:
