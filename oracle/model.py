@@ -30,6 +30,15 @@ Rules (PAPER.md citation for each):
      shared memory per block (reading Q18).
  13  tie-break: max OBJ, then min sum of T on objective-free positions,
      then max T_{l_s1}, then lexicographically smallest T (reading Q16).
+
+Pin status (tests/test_oracle_model.py):
+  pinned    the worked example (unique optimum), Table II / l_s1 / nrefs,
+            heat-3d 9/12 and mttkrp / conv-2d 11/12 feasible configurations (conv-2d's filter
+            size chosen to agree, reading R-N9), Z3 driven as in P:179-181, a hand-solved space, the
+            infeasible spaces.
+  parity unpinned (our readings, held bit-exact against the C++ enumerator only): stencil H weights
+            and footprints (Q6, Q11), the 2-D H rule (Q7), the B-set order beyond three parallel loops
+            (Q12), the split levels (Q17), the sweep sizes (Q19), the tensor-core mode (reading T).
 """
 from __future__ import annotations
 

@@ -22,6 +22,12 @@
  * identical; tests/test_oracle_numeric.py pins that against the literal i-j-k
  * loop (oracle_gemm_ijk) on small sizes.
  *
+ * Pin status (tests/test_oracle_numeric.py): every function is pinned to something other than
+ * itself -- integer matmul / closed forms (identity, rank-1, Khatri-Rao unfolding, rank-1 tensor),
+ * numpy / scipy routines on non-square shapes (a transposed operand fails), exact stencil fixed
+ * points and impulse responses, brute force on tiny sizes, delta-filter shifts.  The loop bodies
+ * themselves (PolyBench 3.2 / 4.x, mttkrp, conv-2d) are our restatement: the paper prints none.
+ *
  * Compile: gcc -O2 -ffp-contract=off -fno-fast-math -fopenmp -shared -fPIC.
  * OpenMP only distributes the outermost parallel loop (rows are independent).
  */
