@@ -283,6 +283,11 @@ def other_configs(E, torch, gpu, stream, peaks):
         out[f"{kind} n={n} T={T}"] = {"tiles": list(tiles), "ms": ms, "us_per_sweep": ms * 1e3 / sweeps,
                                       "gbs": gbs, "bound": "hbm", "frac": gbs / hbm,
                                       "l2_resident": 2 * pts * 4 < 126e6}
+        if T == 500:  # BASELINE config 4: EATSS tiles vs untiled (the plain nest, one thread per point)
+            d.set_exec(split_pct=50, engine=3)
+            ms_u = timed_ms(d, tiles, b, iters)
+            out[f"{kind} n={n} T={T}"]["untiled"] = {"ms": ms_u, "eatss_speedup": ms_u / ms}
+            d.set_exec(split_pct=50, engine=1)
         del b
     d = E.desc_builtin("ccsd_t_d1", (48,))
     b = bufs_for(d)

@@ -161,10 +161,13 @@ typedef struct {
 } eatss_model_report;
 
 /* Execution options stored in a descriptor (eatss_desc_set_exec). */
-typedef enum { EATSS_ENGINE_AUTO = 0, EATSS_ENGINE_SIMT = 1, EATSS_ENGINE_TENSOR = 2 } eatss_engine;
+/* EATSS_ENGINE_UNTILED (jacobi-2d / heat-3d only; others return EATSS_E_UNSUPPORTED): the plain loop
+ * nest without tiling -- one thread per interior point, neighbours from global memory, the tile
+ * vector ignored -- the "untiled" baseline of BASELINE config 4 (same time loop and arithmetic). */
+typedef enum { EATSS_ENGINE_AUTO = 0, EATSS_ENGINE_SIMT = 1, EATSS_ENGINE_TENSOR = 2, EATSS_ENGINE_UNTILED = 3 } eatss_engine;
 typedef struct {
     int32_t split_pct;  /* shared-memory carve-out preference, percent of max (sigma) */
-    int32_t engine;     /* eatss_engine; AUTO = SIMT unless the tensor-core path applies */
+    int32_t engine;     /* eatss_engine; AUTO = SIMT unless the tensor-core path applies; UNTILED: stencils */
     int32_t use_graph;  /* stencils: replay the time loop as one CUDA graph (default 1) */
     int32_t time_kernels; /* 1: record CUDA events around each nest's main compute kernel on the
                              run's stream (read back with eatss_last_kernel_ms); default 0 */

@@ -28,6 +28,9 @@ static eatss_status cuda_fail(cudaError_t e, const char *where) {
 cudaError_t launch_jacobi2d_sweep(void *dst, const void *src, const void *bsrc, int64_t n, int64_t Ti,
                                   int64_t Tj, bool f64, int carveout, int32_t *counts, cudaStream_t s);
 cudaError_t launch_interior_copy2d(void *dst, const void *src, int64_t n, bool f64, cudaStream_t s);
+// stencil_untiled.cu: the untiled baseline (engine EATSS_ENGINE_UNTILED; tile vector ignored)
+cudaError_t launch_jacobi2d_untiled(void *dst, const void *src, const void *bsrc, int64_t n, bool f64, cudaStream_t s);
+cudaError_t launch_heat3d_untiled(void *dst, const void *src, int64_t n, bool f64, cudaStream_t s);
 cudaError_t launch_heat3d_sweep(void *dst, const void *src, int64_t n, int64_t Ti, int64_t Tj,
                                 int64_t Tk, bool f64, int carveout, int32_t *counts, cudaStream_t s);
 void stencil_plan_dims(bool heat, int64_t n, const int64_t *t, bool f64, int64_t *gx, int64_t *gy,
@@ -356,11 +359,13 @@ static cudaError_t stencil_issue(const eatss_kernel_desc *d, const int64_t *t, v
     const int cv = d->exec.split_pct;
     cudaError_t e = cudaSuccess;
     if (n < 3) return cudaSuccess;
+    const bool untiled = d->exec.engine == EATSS_ENGINE_UNTILED;
     if (d->kind == EATSS_JACOBI2D) {
         void *A = b[0], *B = b[1];
         for (int64_t step = 0; step < d->tsteps && e == cudaSuccess; step++) {
-            if (step % 2 == 0) e = launch_jacobi2d_sweep(B, A, A, n, t[0], t[1], f64, cv, nullptr, s);
-            else e = launch_jacobi2d_sweep(A, B, A, n, t[0], t[1], f64, cv, nullptr, s);
+            void *dst = step % 2 == 0 ? B : A, *src = step % 2 == 0 ? A : B;
+            e = untiled ? launch_jacobi2d_untiled(dst, src, A, n, f64, s)
+                        : launch_jacobi2d_sweep(dst, src, A, n, t[0], t[1], f64, cv, nullptr, s);
         }
         if (e == cudaSuccess && d->tsteps > 0) {
             // the literal copy nest of the last step (both interiors end equal to X_T)
@@ -370,8 +375,11 @@ static cudaError_t stencil_issue(const eatss_kernel_desc *d, const int64_t *t, v
     } else {
         void *A = b[0], *B = b[1];
         for (int64_t step = 0; step < d->tsteps && e == cudaSuccess; step++) {
-            e = launch_heat3d_sweep(B, A, n, t[0], t[1], t[2], f64, cv, nullptr, s);
-            if (e == cudaSuccess) e = launch_heat3d_sweep(A, B, n, t[0], t[1], t[2], f64, cv, nullptr, s);
+            e = untiled ? launch_heat3d_untiled(B, A, n, f64, s)
+                        : launch_heat3d_sweep(B, A, n, t[0], t[1], t[2], f64, cv, nullptr, s);
+            if (e == cudaSuccess)
+                e = untiled ? launch_heat3d_untiled(A, B, n, f64, s)
+                            : launch_heat3d_sweep(A, B, n, t[0], t[1], t[2], f64, cv, nullptr, s);
         }
     }
     return e;
@@ -384,6 +392,7 @@ static eatss_status stencil_run(eatss_kernel_desc *d, const int64_t *t, void *co
     }
     GraphKey key;
     key.tiles.assign(t, t + eatss_desc_num_loops(d));
+    key.tiles.push_back(d->exec.engine);  // a tiled and an untiled time loop are different graphs
     for (int i = 0; i < d->num_buffers; i++) key.bufs.push_back((uintptr_t)b[i]);
     key.stream = 0;  // graphs are stream-independent; launched on the caller's stream
     cudaGraphExec_t exec = nullptr;
@@ -583,7 +592,7 @@ eatss_status eatss_desc_set_scalars(eatss_kernel_desc *d, double alpha, double b
 eatss_status eatss_desc_set_exec(eatss_kernel_desc *d, const eatss_exec_opts *o) {
     if (!d || !o) return fail(EATSS_E_INVALID, "eatss_desc_set_exec: null argument");
     if (o->split_pct < 0 || o->split_pct > 100) return fail(EATSS_E_INVALID, "split_pct must be 0..100");
-    if (o->engine < 0 || o->engine > 2) return fail(EATSS_E_INVALID, "bad engine");
+    if (o->engine < 0 || o->engine > 3) return fail(EATSS_E_INVALID, "bad engine");
     d->exec = *o;
     return EATSS_OK;
 }
@@ -782,6 +791,8 @@ static eatss_status run_impl(const eatss_kernel_desc *cd, int only_nest, const i
     if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0)
         return fail(EATSS_E_CUDA, "eatss_run: no CUDA device (there is no CPU fallback)");
     cudaStream_t s = (cudaStream_t)stream;
+    if (d->exec.engine == EATSS_ENGINE_UNTILED && d->kind != EATSS_JACOBI2D && d->kind != EATSS_HEAT3D)
+        return fail(EATSS_E_UNSUPPORTED, "eatss_run: the untiled engine is the stencils' baseline only");
     if (is_contraction(d->kind)) {
         auto cn = contraction_nests(d, buffers);
         const int sl = smem_limit_bytes();

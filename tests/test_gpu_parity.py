@@ -343,3 +343,31 @@ def test_sweep_reports_energy(cuda_device):
         assert r.ms_per_run > 0 and r.tflops > 0 and r.runs >= 1
         if r.status == 0:
             assert r.joules_per_run > 0 and r.avg_watts > 50 and r.gflops_per_watt > 0
+
+
+# ------------------------------------------------------------------ untiled baseline (BASELINE config 4)
+@pytest.mark.parametrize("kind,n,T", [("jacobi-2d", 130, 21), ("jacobi-2d", 67, 6), ("heat-3d", 40, 6),
+                                      ("heat-3d", 23, 3)])
+def test_stencil_untiled_engine(cuda_device, kind, n, T):
+    """The untiled engine (one thread per interior point, tile vector ignored) against the oracle, and
+    the linear-field fixed point exactly; a tiled and an untiled run of one descriptor use separate
+    cached graphs."""
+    shape = (n, n) if kind == "jacobi-2d" else (n, n, n)
+    A = synth.uniform(shape, 97); B = synth.uniform(shape, 98)
+    Ar, Br = (O.jacobi2d if kind == "jacobi-2d" else O.heat3d)(A, B, T)
+    d = E.desc_builtin(kind, (n,), tsteps=T)
+    tiles = (16, 1024) if kind == "jacobi-2d" else (16, 16, 32)
+    for engine in (1, 3, 1, 3):  # alternate: graphs cached per engine
+        d.set_exec(split_pct=50, engine=engine)
+        Ad, Bd = dev(A), dev(B)
+        run(d, tiles, [Ad, Bd])
+        assert O.normwise_rel_err(host(Ad), Ar) <= TOL32 and O.normwise_rel_err(host(Bd), Br) <= TOL32
+    L = synth.linear_field(shape, (2, -3) if kind == "jacobi-2d" else (2, -3, 1), 5)
+    d.set_exec(split_pct=50, engine=3)
+    Ld = dev(L)
+    run(d, tiles, [Ld, dev(L.copy())])
+    assert np.array_equal(host(Ld), L)
+    g = E.desc_builtin("gemm", (64, 64, 64))
+    g.set_exec(split_pct=50, engine=3)
+    with pytest.raises(E.EatssError):
+        run(g, (16, 16, 16), [dev(np.zeros((64, 64))), dev(np.zeros((64, 64))), dev(np.zeros((64, 64)))])
