@@ -758,18 +758,10 @@ static cudaError_t lowdim_run(const eatss_kernel_desc *d, const int64_t *t, void
             a.rowout = F(1); a.vr = F(4); a.ar = 1.f;
             return launch_lowdim(a, true, true, false, s, launched);
         case EATSS_GEMVER: {  // A' = A + u1 v1^T + u2 v2^T fused with x += beta A'^T y; x += z; w += alpha A' x
-            // the fused pass executes nest 1 (A[i][j] update, both loops parallel) and nest 2
-            // (x[i] += beta A[j][i] y[j]) together; it takes nest 1's orientation of the tile vector
-            // -- position 0 over A's rows, position 1 over its columns -- the nest that reads AND
-            // writes A (nest 2's orientation puts Ti = 16 of A's columns on a CTA: 64-byte row
-            // segments; whole gemver at n = 16384, tile (16,1024): 1.445 ms that way, 0.662 ms this
-            // way; EATSS_GEMVER_NEST2=1 restores nest 2's orientation)
-            static const bool nest2 = [] {
-                const char *e = getenv("EATSS_GEMVER_NEST2");
-                return e && atoi(e) != 0;
-            }();
-            a.Ti = (int)std::min<int64_t>(nest2 ? t[1] : t[0], INT32_MAX);
-            a.Tj = (int)std::min<int64_t>(nest2 ? t[0] : t[1], INT32_MAX);
+            // the fused pass carries nest 2 (x[i] += beta A[j][i] y[j]): its loop i runs along A's
+            // columns, so that pass maps tile position 0 to columns and position 1 to rows
+            a.Ti = (int)std::min<int64_t>(t[1], INT32_MAX);
+            a.Tj = (int)std::min<int64_t>(t[0], INT32_MAX);
             a.A = F(0); a.Aout = F(0); a.nx = a.ny = x[0];
             a.u1 = F(3); a.v1 = F(4); a.u2 = F(5); a.v2 = F(6);
             a.colout = F(1); a.vc = F(7); a.ac = (float)d->beta;
