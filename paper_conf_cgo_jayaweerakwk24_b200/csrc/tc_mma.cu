@@ -350,15 +350,26 @@ __global__ void split_kernel(const float *__restrict__ x, int64_t ldx, int64_t r
         const bool v4 = ((reinterpret_cast<uintptr_t>(x) | reinterpret_cast<uintptr_t>(lo) |
                           reinterpret_cast<uintptr_t>(hi)) & 15) == 0;
         const int64_t n4 = v4 ? n / 4 : 0;
-        for (int64_t v = t0; v < n4; v += stride) {
-            const float4 a = reinterpret_cast<const float4 *>(x)[v];
-            float4 h, l;
-            split1(a.x, mode, h.x, l.x);
-            split1(a.y, mode, h.y, l.y);
-            split1(a.z, mode, h.z, l.z);
-            split1(a.w, mode, h.w, l.w);
-            if (hi) reinterpret_cast<float4 *>(hi)[v] = h;
-            reinterpret_cast<float4 *>(lo)[v] = l;
+        // SPLIT_U independent 16-byte loads in flight per thread before the first store
+        // (one load per thread leaves ~32 KB per SM in flight: below the HBM latency-bandwidth product)
+        constexpr int SPLIT_U = 4;
+        for (int64_t v0 = t0; v0 < n4; v0 += SPLIT_U * stride) {
+            float4 a[SPLIT_U];
+#pragma unroll
+            for (int u = 0; u < SPLIT_U; ++u)
+                if (v0 + u * stride < n4) a[u] = reinterpret_cast<const float4 *>(x)[v0 + u * stride];
+#pragma unroll
+            for (int u = 0; u < SPLIT_U; ++u) {
+                const int64_t v = v0 + u * stride;
+                if (v >= n4) break;
+                float4 h, l;
+                split1(a[u].x, mode, h.x, l.x);
+                split1(a[u].y, mode, h.y, l.y);
+                split1(a[u].z, mode, h.z, l.z);
+                split1(a[u].w, mode, h.w, l.w);
+                if (hi) reinterpret_cast<float4 *>(hi)[v] = h;
+                reinterpret_cast<float4 *>(lo)[v] = l;
+            }
         }
         for (int64_t e = n4 * 4 + t0; e < n; e += stride) {
             float h, l;
