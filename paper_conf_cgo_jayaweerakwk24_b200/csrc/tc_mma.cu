@@ -5,7 +5,7 @@
 // Same loop-nest semantics as the SIMT executor (Fig. 4: each CTA owns one Ti x Tj
 // tile of C, k sequential); fp32-accurate via 3xTF32 (reading Q26):
 //   C = beta*C + alpha * sum_k (Ahi*Bhi + Ahi*Blo + Alo*Bhi),
-//   hi = rna_tf32(x), lo = rna_tf32(x - hi), computed once per operand by split_kernel.
+//   hi = rna_tf32(x), lo = rna_tf32(x - hi), computed once per operand by prep_kernel.
 //
 // B200-specific structure (what differs from the paper's one-tile-per-block CUDA code):
 //  * CTA pairs (cta_group::2, cluster of 2 along i): the pair issues M = 256 MMAs; each CTA
@@ -17,7 +17,7 @@
 //    chunk by chunk (two TMEM buffers), so one tile's epilogue overlaps the next tile's MMAs.
 //  * wave-quantisation tail: when the last wave would leave clusters idle, the remaining tiles
 //    are split along k into `sp` parts whose partial sums are added to C with fp32 atomics
-//    (C pre-scaled by beta once by tail_prepass_kernel).
+//    (C pre-scaled by beta once by prep_kernel).
 // Pipeline (warp-specialised, mbarrier hand-off, one CTA per SM):
 //   warp 0  TMA producer: Ahi/Alo (K-major, 128 x 32, SWIZZLE_128B) and Bhi/Blo (MN-major
 //           32 x Tj/CG in 32-column SWIZZLE_128B_ATOM_32B boxes, or K-major Tj/CG x 32 when B
@@ -255,7 +255,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             if (i < p.M && jb < p.N) {
                 float *crow = p.C + i * p.ldc + jb;
                 const bool vec = ((p.ldc & 3) == 0) && (jb + CW <= p.N);
-                if (w.split) {  // C already holds beta*C (tail_prepass_kernel): add the partial sum
+                if (w.split) {  // C already holds beta*C (prep_kernel): add the partial sum
                     if (vec) {
 #pragma unroll
                         for (int c = 0; c < CW; c += 4)
@@ -303,29 +303,6 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     }
 }
 
-// C := init_zero ? 0 : beta*C over the tiles that are split along k (their parts then add
-// alpha * partial sums atomically).  One CTA per row of a tail tile.
-__global__ void tail_prepass_kernel(const Args p, int rows_per_tile, int bn) {
-    const int t = p.nfull + (int)blockIdx.x / rows_per_tile, r = (int)blockIdx.x % rows_per_tile;
-    int pi, tj;
-    tile_coords(t, p.PI, p.TJ, pi, tj);
-    const int64_t i = (int64_t)pi * rows_per_tile + r, j0 = (int64_t)tj * bn;
-    if (i >= p.M) return;
-    float *c = p.C + i * p.ldc + j0;
-    const int64_t w = p.N - j0 < bn ? p.N - j0 : bn;
-    if ((reinterpret_cast<uintptr_t>(c) & 15) == 0) {
-        for (int x = threadIdx.x; x < w / 4; x += blockDim.x) {
-            float4 v = reinterpret_cast<float4 *>(c)[x];
-            v = p.init_zero ? make_float4(0.f, 0.f, 0.f, 0.f)
-                            : make_float4(p.beta * v.x, p.beta * v.y, p.beta * v.z, p.beta * v.w);
-            reinterpret_cast<float4 *>(c)[x] = v;
-        }
-        for (int64_t x = w / 4 * 4 + threadIdx.x; x < w; x += blockDim.x) c[x] = p.init_zero ? 0.f : p.beta * c[x];
-    } else {
-        for (int64_t x = threadIdx.x; x < w; x += blockDim.x) c[x] = p.init_zero ? 0.f : p.beta * c[x];
-    }
-}
-
 // Operand split for 3xTF32 (reading Q26).  mode 0: hi = rna_tf32(x), lo = rna_tf32(x - hi).
 // mode 1 ("raw hi"): the tensor core reads only the tf32 bits of an fp32 container (it truncates),
 // so the untouched operand already serves as hi = rz_tf32(x) and only lo = rna_tf32(x - rz_tf32(x))
@@ -342,9 +319,17 @@ __device__ __forceinline__ void split1(float v, int mode, float &h, float &l) {
     h = mode == 0 ? __uint_as_float(hb) : v;
     l = __uint_as_float(lb);
 }
-__global__ void split_kernel(const float *__restrict__ x, int64_t ldx, int64_t rows, int64_t cols,
-                             float *__restrict__ hi, float *__restrict__ lo, int64_t ldp, int mode) {
-    const int64_t stride = (int64_t)gridDim.x * blockDim.x, t0 = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+struct SplitJob {
+    const float *x;  // nullptr: no job
+    int64_t ldx, rows, cols;
+    float *hi, *lo;  // hi == nullptr: raw hi (mode 1, flat)
+    int64_t ldp;
+};
+__device__ __forceinline__ void split_body(const SplitJob &j, int mode, int64_t t0, int64_t stride) {
+    const float *__restrict__ x = j.x;
+    float *__restrict__ hi = j.hi;
+    float *__restrict__ lo = j.lo;
+    const int64_t ldx = j.ldx, rows = j.rows, cols = j.cols, ldp = j.ldp;
     if (ldx == ldp) {  // flat over (rows - 1) * ld + cols elements
         const int64_t n = (rows - 1) * ldx + cols;
         const bool v4 = ((reinterpret_cast<uintptr_t>(x) | reinterpret_cast<uintptr_t>(lo) |
@@ -388,8 +373,52 @@ __global__ void split_kernel(const float *__restrict__ x, int64_t ldx, int64_t r
     }
 }
 
+// One launch before the GEMM: blocks [0, nb0) split operand j0, [nb0, nb0 + nb1) operand j1, the
+// rest run the tail prepass (C := init_zero ? 0 : beta*C over the k-split tail tiles; rows of
+// CG*128 per tile, bn columns) as a grid-stride loop over 4-column groups.  vecC: C and ldc allow
+// 16-byte accesses.
+__global__ void __launch_bounds__(256) prep_kernel(const SplitJob j0, const SplitJob j1, int nb0, int nb1, int mode,
+                                                   const Args p, int rows_per_tile, int bn, int vecC) {
+    const int b = (int)blockIdx.x;
+    if (b < nb0) {
+        split_body(j0, mode, (int64_t)b * blockDim.x + threadIdx.x, (int64_t)nb0 * blockDim.x);
+        return;
+    }
+    if (b < nb0 + nb1) {
+        split_body(j1, mode, (int64_t)(b - nb0) * blockDim.x + threadIdx.x, (int64_t)nb1 * blockDim.x);
+        return;
+    }
+    const int npb = (int)gridDim.x - nb0 - nb1, g4 = (bn + 3) / 4;
+    const int64_t total = (int64_t)(p.T - p.nfull) * rows_per_tile * g4;
+    for (int64_t e = (int64_t)(b - nb0 - nb1) * blockDim.x + threadIdx.x; e < total; e += (int64_t)npb * blockDim.x) {
+        const int64_t rowid = e / g4;
+        const int x = (int)(e % g4);
+        const int t = p.nfull + (int)(rowid / rows_per_tile), r = (int)(rowid % rows_per_tile);
+        int pi, tj;
+        tile_coords(t, p.PI, p.TJ, pi, tj);
+        const int64_t i = (int64_t)pi * rows_per_tile + r, j = (int64_t)tj * bn + 4 * x;
+        if (i >= p.M || j >= p.N) continue;
+        float *c = p.C + i * p.ldc + j;
+        if (vecC && j + 3 < p.N) {
+            float4 v = *reinterpret_cast<float4 *>(c);
+            v = p.init_zero ? make_float4(0.f, 0.f, 0.f, 0.f)
+                            : make_float4(p.beta * v.x, p.beta * v.y, p.beta * v.z, p.beta * v.w);
+            *reinterpret_cast<float4 *>(c) = v;
+        } else {
+            for (int q = 0; q < 4 && j + q < p.N; q++) c[q] = p.init_zero ? 0.f : p.beta * c[q];
+        }
+    }
+}
+
 // ------------------------------------------------------------------ host side
 }  // namespace tcm
+
+// The operand split jobs of one GEMM (j1.x == nullptr when B's split serves A too) and their
+// block counts in the fused prep launch.
+struct Prep {
+    tcm::SplitJob j0{}, j1{};
+    int nb0 = 0, nb1 = 0, mode = 1;
+};
 
 // Workspace for the split operands (library-owned, grown on demand, per device).
 namespace {
@@ -471,7 +500,7 @@ std::map<std::pair<const void *, int>, KernelState> g_ks;
 }  // namespace
 
 template <int BN, bool TB, int CG>
-static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int nsm, cudaStream_t s,
+static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int nsm, const Prep &pr, cudaStream_t s,
                               cudaEvent_t *ev) {
     auto k = tcm::tc_mma_kernel<BN, TB, CG>;
     int dev = 0;
@@ -511,9 +540,12 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
     }
     schedule(a, ncl);
     ncl = std::max(1, std::min(ncl, a.T));
-    if (needs_prepass(a)) {
-        const int rows = CG * tcm::BM, blocks = (a.T - a.nfull) * rows;
-        tcm::tail_prepass_kernel<<<blocks, std::max(32, BN / 4), 0, s>>>(a, rows, BN);
+    {  // operand splits + tail prepass: one launch
+        const int rows = CG * tcm::BM;
+        const int64_t tail4 = needs_prepass(a) ? (int64_t)(a.T - a.nfull) * rows * ((BN + 3) / 4) : 0;
+        const int npb = (int)std::min<int64_t>((tail4 + 255) / 256, 148 * 4);
+        const int vecC = (a.ldc % 4 == 0 && (reinterpret_cast<uintptr_t>(a.C) & 15) == 0) ? 1 : 0;
+        tcm::prep_kernel<<<pr.nb0 + pr.nb1 + npb, 256, 0, s>>>(pr.j0, pr.j1, pr.nb0, pr.nb1, pr.mode, a, rows, BN, vecC);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
     }
     cfg.gridDim = dim3((unsigned)(CG * ncl));
@@ -524,17 +556,17 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
 }
 
 template <bool TB, int CG>
-static cudaError_t launch_bn(int bn, const CUtensorMap *m, const tcm::Args &a, int smem, int nsm, cudaStream_t s,
-                             cudaEvent_t *ev) {
+static cudaError_t launch_bn(int bn, const CUtensorMap *m, const tcm::Args &a, int smem, int nsm, const Prep &pr,
+                             cudaStream_t s, cudaEvent_t *ev) {
     switch (bn) {
-        case 32: return launch_one<32, TB, CG>(m, a, smem, nsm, s, ev);
-        case 64: return launch_one<64, TB, CG>(m, a, smem, nsm, s, ev);
-        case 96: return launch_one<96, TB, CG>(m, a, smem, nsm, s, ev);
-        case 128: return launch_one<128, TB, CG>(m, a, smem, nsm, s, ev);
-        case 160: return launch_one<160, TB, CG>(m, a, smem, nsm, s, ev);
-        case 192: return launch_one<192, TB, CG>(m, a, smem, nsm, s, ev);
-        case 224: return launch_one<224, TB, CG>(m, a, smem, nsm, s, ev);
-        case 256: return launch_one<256, TB, CG>(m, a, smem, nsm, s, ev);
+        case 32: return launch_one<32, TB, CG>(m, a, smem, nsm, pr, s, ev);
+        case 64: return launch_one<64, TB, CG>(m, a, smem, nsm, pr, s, ev);
+        case 96: return launch_one<96, TB, CG>(m, a, smem, nsm, pr, s, ev);
+        case 128: return launch_one<128, TB, CG>(m, a, smem, nsm, pr, s, ev);
+        case 160: return launch_one<160, TB, CG>(m, a, smem, nsm, pr, s, ev);
+        case 192: return launch_one<192, TB, CG>(m, a, smem, nsm, pr, s, ev);
+        case 224: return launch_one<224, TB, CG>(m, a, smem, nsm, pr, s, ev);
+        case 256: return launch_one<256, TB, CG>(m, a, smem, nsm, pr, s, ev);
         default: return cudaErrorNotSupported;
     }
 }
@@ -562,12 +594,12 @@ void size_operand(Operand &o, int mode) {
     const int64_t span = aligned ? (o.rows - 1) * o.ld + o.cols : o.rows * o.ldp;
     o.need = (o.raw_hi ? 1 : 2) * ((span + 3) / 4 * 4);
 }
-void split_operand(Operand &o, float *ws, int mode, cudaStream_t s) {
+tcm::SplitJob split_job(Operand &o, float *ws) {  // the split is run by the fused prep launch
     const int64_t span = o.need / (o.raw_hi ? 1 : 2);
     float *lo = ws, *hi = o.raw_hi ? nullptr : ws + span;
-    tcm::split_kernel<<<148 * 8, 256, 0, s>>>(o.x, o.ld, o.rows, o.cols, hi, lo, o.ldp, mode);
     o.lo = lo;
     o.hi = o.raw_hi ? o.x : hi;
+    return tcm::SplitJob{o.x, o.ld, o.rows, o.cols, hi, lo, o.ldp};
 }
 }  // namespace
 
@@ -583,14 +615,20 @@ cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p,
                        (A - B) / n.ldb + n.M <= ob.rows;
     float *ws = workspace((size_t)(ob.need + (share ? 0 : oa.need) + 64));
     if (!ws) return cudaErrorMemoryAllocation;
-    split_operand(ob, ws, mode, s);
+    Prep pr;
+    pr.mode = mode;
+    pr.j0 = split_job(ob, ws);
+    constexpr int kSplitBlocks = 148 * 8;  // grid-stride split blocks over both operands
     if (share) {
         const int64_t r = (A - B) / n.ldb;
         oa.hi = ob.hi + r * ob.ldp;
         oa.lo = ob.lo + r * ob.ldp;
         oa.ldp = ob.ldp;
+        pr.nb0 = kSplitBlocks;
     } else {
-        split_operand(oa, ws + ob.need, mode, s);
+        pr.j1 = split_job(oa, ws + ob.need);
+        pr.nb0 = std::max(1, std::min(kSplitBlocks - 1, (int)((double)kSplitBlocks * ob.need / (ob.need + oa.need))));
+        pr.nb1 = kSplitBlocks - pr.nb0;
     }
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
@@ -620,26 +658,12 @@ cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p,
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     if (n.transB)
-        return cg == 2 ? launch_bn<true, 2>(bn, m, a, smem, nsm, s, ev) : launch_bn<true, 1>(bn, m, a, smem, nsm, s, ev);
-    return cg == 2 ? launch_bn<false, 2>(bn, m, a, smem, nsm, s, ev) : launch_bn<false, 1>(bn, m, a, smem, nsm, s, ev);
+        return cg == 2 ? launch_bn<true, 2>(bn, m, a, smem, nsm, pr, s, ev) : launch_bn<true, 1>(bn, m, a, smem, nsm, pr, s, ev);
+    return cg == 2 ? launch_bn<false, 2>(bn, m, a, smem, nsm, pr, s, ev) : launch_bn<false, 1>(bn, m, a, smem, nsm, pr, s, ev);
 }
 
-int tcm_launches(const ContractNest &n, const ContractPlan &p) {
-    const int bn = (int)p.Tj, cg = tcm_cg(n, bn);
-    const float *A = static_cast<const float *>(n.A), *B = static_cast<const float *>(n.B);
-    const bool share = n.transB && n.lda == n.ldb && A >= B && (A - B) % n.ldb == 0 &&
-                       (A - B) / n.ldb + n.M <= n.N;
-    tcm::Args a{};
-    a.init_zero = n.init_zero ? 1 : 0;
-    a.beta = (float)n.beta;
-    a.nkb = (int)((n.K + tcm::BK - 1) / tcm::BK);
-    a.PI = (int)((n.M + cg * tcm::BM - 1) / (cg * tcm::BM));
-    a.TJ = (int)((n.N + bn - 1) / bn);
-    int dev = 0, nsm = 148;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-    schedule(a, nsm / cg);  // (the occupancy cap of CTA pairs is nsm / 2 on B200)
-    return (share ? 1 : 2) + (needs_prepass(a) ? 1 : 0) + 1;
+int tcm_launches(const ContractNest &, const ContractPlan &) {
+    return 2;  // the fused prep launch (splits + tail prepass) and the GEMM
 }
 
 }  // namespace eatss

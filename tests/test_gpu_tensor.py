@@ -208,8 +208,9 @@ def test_tcm_split_exact_for_22_bit_values(cuda_device, tiles):
 
 
 def test_kernel_timing_and_launch_count(cuda_device):
-    # exec.time_kernels: events around the GEMM launch alone; launches_per_run counts the split
-    # passes (A and B; syrk shares one), the split-k tail pre-pass (beta != 1) and the GEMM
+    # exec.time_kernels: events around the GEMM launch alone; launches_per_run counts the fused
+    # prep launch (operand splits of A and B -- syrk shares one -- and the split-k tail pre-pass
+    # when beta != 1) and the GEMM
     n = 2500
     d = E.desc_builtin("gemm", (n, n, n)); d.set_scalars(1.5, 1.2); d.set_exec(50, TENSOR, time_kernels=1)
     bufs = [torch.rand(n, n, device="cuda") for _ in range(3)]
@@ -220,12 +221,12 @@ def test_kernel_timing_and_launch_count(cuda_device):
     (k,) = E.last_kernel_ms(d)
     assert 0 < k < s.elapsed_time(e)
     # 2500/256 -> 10 pair-rows x 10 column tiles = 100 tiles on 74 clusters: the 26-tile tail is
-    # split along k (pre-pass needed for beta != 1)
-    assert E.launches_per_run(d, (128, 256, 32)) == 4
+    # split along k (pre-pass needed for beta != 1, run inside the prep launch)
+    assert E.launches_per_run(d, (128, 256, 32)) == 2
     d.set_scalars(1.5, 1.0)
-    assert E.launches_per_run(d, (128, 256, 32)) == 3
+    assert E.launches_per_run(d, (128, 256, 32)) == 2
     ds = E.desc_builtin("syrk", (n, n)); ds.set_exec(50, TENSOR)
-    assert E.launches_per_run(ds, (128, 256, 32)) == 3
+    assert E.launches_per_run(ds, (128, 256, 32)) == 2
     d2 = E.desc_builtin("gemm", (n, n, n))
     with pytest.raises(E.EatssError):
         E.last_kernel_ms(d2)
