@@ -358,7 +358,7 @@ def main():
         d, tiles, rep = arm.step(C, A, B, stream)
     torch.cuda.synchronize()
     plans = E.plan(d, tiles)
-    launches_per_step = E.launches_per_run(d, tiles)  # tensor engine: + operand split passes + tail pre-pass
+    launches_per_step = E.launches_per_run(d, tiles)  # tensor engine: prep launch (operand splits + tail pre-pass) + GEMM
 
     clk = ClockSampler(local)
     K = args.steps
@@ -455,8 +455,8 @@ def main():
             tf32 = bf16 * TF32_OVER_BF16
             roof = {"bound": "tensor", "achieved": achieved, "peak": tf32 / 3, "unit": "TFLOP/s",
                     "frac": achieved / (tf32 / 3), "traffic": traffic,
-                    "kernel": f"tc_mma_kernel<{tiles[1]}> (tcgen05 GEMM alone; the operand split passes "
-                              f"are outside this window but inside every timed step)",
+                    "kernel": f"tc_mma_kernel<{tiles[1]}> (tcgen05 GEMM alone; the prep launch (operand "
+                              f"splits + split-k tail pre-pass) is outside this window but inside every timed step)",
                     "call_frac": FLOPS / (call_avg_ms * 1e-3) / 1e12 / (tf32 / 3),
                     "peak_source": (f"measured bf16 {bf16:.1f} TF (MEASURED_PEAKS.json, burst) x nominal "
                                     f"tf32/bf16 {TF32_OVER_BF16:.3f} = {tf32:.1f} TF tf32; 3xTF32 executes 3 "
