@@ -273,12 +273,12 @@ EATSS_API eatss_status eatss_run_host(const eatss_kernel_desc *d, const int64_t 
 EATSS_API eatss_status eatss_coverage(const eatss_kernel_desc *d, int nest, const int64_t *tiles,
                             int32_t *counts, void *stream);
 /* Number of kernel launches one eatss_run issues with the descriptor's current exec options
- * (graph nodes counted individually; tensor engine: + operand split passes and the split-k
- * tail pre-pass).  -1 on a bad argument. */
+ * (graph nodes counted individually; tensor engine: one prep launch -- the operand splits and
+ * the split-k tail pre-pass -- plus the GEMM).  -1 on a bad argument. */
 EATSS_API int64_t eatss_launches_per_run(const eatss_kernel_desc *d, const int64_t *tiles);
 /* Device time in ms of the main compute kernel of each nest in the LAST eatss_run on `d`
  * issued with exec.time_kernels = 1 (tensor engine: the tcgen05 GEMM kernel alone, without
- * the operand split passes; SIMT / ccsd: the nest's kernel; stencils: the whole time loop).
+ * the prep launch; SIMT / ccsd: the nest's kernel; stencils: the whole time loop).
  * Writes min(cap, #nests) values to ms and the count to *n.  Blocks until those kernels have
  * finished.  E_INVALID if no timed run has been issued on `d`. */
 EATSS_API eatss_status eatss_last_kernel_ms(const eatss_kernel_desc *d, float *ms, int32_t cap, int32_t *n);
