@@ -65,8 +65,20 @@ def measured_peaks():
 
 
 # ------------------------------------------------------------------ CPU oracle leg
+def cpu_model() -> str:
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    import platform
+    return platform.processor() or "unknown"
+
+
 def cpu_oracle_sample(target_s: float = 12.0):
-    """Time the fp64 oracle on a bounded row block of the same gemm N=4000."""
+    """Time the fp64 oracle on a bounded row block of the same gemm N=4000; returns (record, rows,
+    oracle rows) -- the rows also serve the headline's precision check (same inputs, one step)."""
     import synth
     from oracle import numeric as O
 
@@ -77,16 +89,30 @@ def cpu_oracle_sample(target_s: float = 12.0):
 
     def run_rows(r):
         t0 = time.perf_counter()
-        O.gemm(1.5, 1.2, C[:r], A[:r], B)
-        return time.perf_counter() - t0
+        out = O.gemm(1.5, 1.2, C[:r], A[:r], B)
+        return time.perf_counter() - t0, out
 
-    t = run_rows(16)
+    t, _ = run_rows(16)
     rows = int(min(N, max(16, 16 * target_s / max(t, 1e-3))))
-    t = run_rows(rows)
+    t, ref = run_rows(rows)
     flops = 2.0 * rows * N * N
-    return {"value": flops / t / 1e12, "unit": "TFLOP/s", "cores": O.num_threads(), "kind": "oracle",
-            "sample": f"fp64 oracle (oracle/oracle.c, OpenMP) on rows 0..{rows - 1} of gemm N=4000 "
-                      f"({flops:.3g} flop, {t:.2f} s)"}
+    rec = {"value": flops / t / 1e12, "unit": "TFLOP/s", "cores": O.num_threads(), "cpu_model": cpu_model(),
+           "kind": "oracle",
+           "sample": f"fp64 oracle (oracle/oracle.c, OpenMP) on rows 0..{rows - 1} of gemm N=4000 "
+                     f"({flops:.3g} flop, {t:.2f} s)"}
+    return rec, rows, ref
+
+
+def precision_of(out_rows, ref_rows, rows):
+    """Headline precision: one step's C (fresh inputs) against the fp64 oracle on the same rows."""
+    from oracle import numeric as O
+
+    x = np.asarray(out_rows, dtype=np.float64)
+    rms = float(np.sqrt(np.mean(ref_rows * ref_rows)))
+    return {"normwise_rel_err": O.normwise_rel_err(x, ref_rows),
+            "max_abs_err_over_rms": float(np.max(np.abs(x - ref_rows)) / rms),
+            "bar": 1e-5, "rows_checked": rows, "of": N,
+            "how": "one headline step on fresh U[-1,1) inputs vs the fp64 oracle (cpu_baseline leg)"}
 
 
 def reference_arm(args, ws, rank):
@@ -114,8 +140,8 @@ def reference_arm(args, ws, rank):
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
         "data": "synthetic U[-1,1) PCG64 seeds 0,1,2",
         "config": {"workload": "gemm N=4000 (row-block sample on host cores)", "rows_per_step": rows},
-        "cpu_baseline": {"value": value, "unit": "TFLOP/s", "cores": O.num_threads(), "kind": "oracle",
-                         "sample": sample},
+        "cpu_baseline": {"value": value, "unit": "TFLOP/s", "cores": O.num_threads(), "cpu_model": cpu_model(),
+                         "kind": "oracle", "sample": sample},
         "e2e": {"value": value, "unit": "TFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }), flush=True)
 
@@ -508,7 +534,14 @@ def main():
         if configs:
             out["configs"] = configs
         if not args.no_cpu_baseline:
-            out["cpu_baseline"] = cpu_oracle_sample()
+            rec, rows, ref_rows = cpu_oracle_sample()
+            out["cpu_baseline"] = rec
+            # one fresh headline step (same inputs as the oracle's) for the precision record
+            Cf = torch.from_numpy(C_h).to(dev)
+            arm.step(Cf, A, B, stream)
+            torch.cuda.synchronize()
+            out["precision"] = precision_of(Cf[:rows].double().cpu().numpy(), ref_rows, rows)
+            del Cf
         print(json.dumps(out), flush=True)
     if ws > 1:
         dist.barrier()

@@ -45,7 +45,7 @@ extern "C" {
 #define EATSS_API
 #endif
 
-#define EATSS_ABI_VERSION 1
+#define EATSS_ABI_VERSION 2
 #define EATSS_MAX_LOOPS 8
 #define EATSS_MAX_NESTS 4
 #define EATSS_MAX_BUFFERS 16
@@ -171,6 +171,15 @@ typedef struct {
     int32_t use_graph;  /* stencils: replay the time loop as one CUDA graph (default 1) */
     int32_t time_kernels; /* 1: record CUDA events around each nest's main compute kernel on the
                              run's stream (read back with eatss_last_kernel_ms); default 0 */
+    int32_t warp_align; /* SIMT contraction executor: lanes of every warp laid contiguously along the
+                           CMA loop l_s1 -- the "SIMT length as a fraction of the warp size" (P:25,
+                           P:125): WAF in {4, 8, 16, 32}, the remaining 32/WAF lanes of the warp
+                           on consecutive rows of the tile; 0 (default) = the executor's own layout
+                           (reported as eatss_launch_plan.simt_x).  Other values: EATSS_E_INVALID */
+    int32_t carveout_exact; /* 1: request exactly split_pct as the L1/shared carve-out (the model's
+                           sigma); 0 (default): split_pct is a lower bound that the SIMT
+                           executors raise as far as their register-limited resident CTAs need.  The
+                           value actually requested is reported by eatss_last_carveout */
 } eatss_exec_opts;
 
 /* Launch plan of one nest (tile -> GPU mapping, Fig. 4). */
@@ -184,8 +193,8 @@ typedef struct {
     int32_t smem_bytes;    /* dynamic shared memory per CTA */
     int32_t a_in_smem;     /* SH_set operand staged in shared memory */
     int32_t b_in_smem;
-    int32_t carveout_pct;
-    int32_t simt_x;        /* lanes of a warp laid along l_s1 */
+    int32_t carveout_pct;  /* exec.split_pct (the request; the effective value: eatss_last_carveout) */
+    int32_t simt_x;        /* lanes of a warp laid along l_s1 (= exec.warp_align when set) */
     int64_t tile[EATSS_MAX_LOOPS]; /* tile vector clipped to the extents */
 } eatss_launch_plan;
 
@@ -282,6 +291,11 @@ EATSS_API int64_t eatss_launches_per_run(const eatss_kernel_desc *d, const int64
  * Writes min(cap, #nests) values to ms and the count to *n.  Blocks until those kernels have
  * finished.  E_INVALID if no timed run has been issued on `d`. */
 EATSS_API eatss_status eatss_last_kernel_ms(const eatss_kernel_desc *d, float *ms, int32_t cap, int32_t *n);
+
+/* Carve-out (percent) each nest's main kernel requested in the LAST eatss_run on `d` (the effective
+ * value under exec.carveout_exact; -1 for kernels that set none, e.g. the tcgen05 engine, whose
+ * shared memory is fixed by its stage ring).  Writes min(cap, #nests) values, the count to *n. */
+EATSS_API eatss_status eatss_last_carveout(const eatss_kernel_desc *d, int32_t *pct, int32_t cap, int32_t *n);
 
 /* ------------------------------------------------------------ energy */
 /* NVML total-energy counter of `device` in millijoules since driver load. */

@@ -21,7 +21,8 @@ _lib = _abi.load()
 
 __all__ = [
     "EatssError", "Desc", "desc_builtin", "gpu_params_query", "gpu_params_b200", "gpu_params_ga100",
-    "select_tiles", "plan", "run", "run_nest", "coverage", "launches_per_run", "last_kernel_ms", "energy_mj",
+    "select_tiles", "plan", "run", "run_nest", "coverage", "launches_per_run", "last_kernel_ms", "last_carveout",
+    "energy_mj",
     "power_sample", "sweep", "last_error", "abi_version", "lib_path",
 ]
 
@@ -111,8 +112,9 @@ class Desc:
     def set_scalars(self, alpha: float, beta: float) -> None:
         _check(_lib.eatss_desc_set_scalars(self._h, float(alpha), float(beta)), "desc_set_scalars")
 
-    def set_exec(self, split_pct: int = 50, engine: int = 0, use_graph: int = 1, time_kernels: int = 0) -> None:
-        o = _abi.ExecOpts(split_pct, engine, use_graph, time_kernels)
+    def set_exec(self, split_pct: int = 50, engine: int = 0, use_graph: int = 1, time_kernels: int = 0,
+                 warp_align: int = 0, carveout_exact: int = 0) -> None:
+        o = _abi.ExecOpts(split_pct, engine, use_graph, time_kernels, warp_align, carveout_exact)
         _check(_lib.eatss_desc_set_exec(self._h, ctypes.byref(o)), "desc_set_exec")
 
     def model_info(self, nest: int = 0, waf: int = 16):
@@ -218,6 +220,14 @@ def last_kernel_ms(d: Desc) -> List[float]:
     ms = (ctypes.c_float * cap)(); n = ctypes.c_int32()
     _check(_lib.eatss_last_kernel_ms(d.handle, ms, cap, ctypes.byref(n)), "last_kernel_ms")
     return list(ms)[: n.value]
+
+
+def last_carveout(d: Desc) -> List[int]:
+    """Carve-out percent each nest's main kernel requested in the last run (-1: none set)."""
+    cap = max(1, d.num_nests)
+    v = (ctypes.c_int32 * cap)(); n = ctypes.c_int32()
+    _check(_lib.eatss_last_carveout(d.handle, v, cap, ctypes.byref(n)), "last_carveout")
+    return list(v)[: n.value]
 
 
 def energy_mj(device: int = 0) -> int:

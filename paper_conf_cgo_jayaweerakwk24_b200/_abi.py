@@ -51,7 +51,8 @@ class ModelReport(ctypes.Structure):
 
 
 class ExecOpts(ctypes.Structure):
-    _fields_ = [("split_pct", I32), ("engine", I32), ("use_graph", I32), ("time_kernels", I32)]
+    _fields_ = [("split_pct", I32), ("engine", I32), ("use_graph", I32), ("time_kernels", I32),
+                ("warp_align", I32), ("carveout_exact", I32)]
 
 
 class LaunchPlan(ctypes.Structure):
@@ -95,6 +96,7 @@ DECLS = [
     ("eatss_coverage", I32, [P, ctypes.c_int, ctypes.POINTER(I64), P, P]),
     ("eatss_launches_per_run", I64, [P, ctypes.POINTER(I64)]),
     ("eatss_last_kernel_ms", I32, [P, ctypes.POINTER(ctypes.c_float), I32, ctypes.POINTER(I32)]),
+    ("eatss_last_carveout", I32, [P, ctypes.POINTER(I32), I32, ctypes.POINTER(I32)]),
     ("eatss_energy_mj", I32, [ctypes.c_int, ctypes.POINTER(ctypes.c_uint64)]),
     ("eatss_power_sample", I32, [ctypes.c_int, ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(ctypes.c_uint32)]),
     ("eatss_sweep", I32, [P, ctypes.POINTER(I64), ctypes.c_int, ctypes.POINTER(P), ctypes.c_int, ctypes.c_int,

@@ -39,8 +39,10 @@ cudaError_t launch_ccsd_d1(float *t3, const float *t2, const float *v2, const in
                            const int64_t *tiles, int64_t h3_begin, int64_t h3_count, int carveout,
                            int32_t *counts, cudaStream_t s);
 bool ccsd_tc_applicable(const int64_t *dims, const int64_t *tiles);
+size_t ccsd_tc_ws_floats(const int64_t *dims);
 cudaError_t launch_ccsd_tc(float *t3, const float *t2, const float *v2, const int64_t *dims, const int64_t *tiles,
-                           int64_t h3_begin, int64_t h3_count, cudaStream_t s, cudaEvent_t *ev);
+                           int64_t h3_begin, int64_t h3_count, float *ws, size_t ws_floats, cudaStream_t s,
+                           cudaEvent_t *ev);
 void ccsd_plan_dims(const int64_t *dims, const int64_t *tiles, int64_t *gx, int64_t *gy, int *bx,
                     int *by, int *rm, int *rn, int *passes, int *smem);
 
@@ -249,12 +251,21 @@ static eatss_status build(eatss_kernel_desc *d) {
 }
 
 // Library-owned scratch of a descriptor (grown on demand, on the current device).
+static void free_ws(eatss_kernel_desc *d) {
+    if (!d->ws) return;
+    int cur = 0;
+    cudaGetDevice(&cur);
+    if (d->ws_dev >= 0 && d->ws_dev != cur) cudaSetDevice(d->ws_dev);  // free on the owning device
+    cudaFree(d->ws);  // synchronises that device: no queued launch still uses the old scratch
+    if (d->ws_dev >= 0 && d->ws_dev != cur) cudaSetDevice(cur);
+    d->ws = nullptr;
+    d->ws_bytes = 0;
+}
 static eatss_status ensure_ws(eatss_kernel_desc *d, size_t need) {
     int dev = 0;
     cudaGetDevice(&dev);
-    if (d->ws_dev == dev && d->ws_bytes >= need) return EATSS_OK;
-    if (d->ws && d->ws_dev == dev) cudaFree(d->ws);  // never free another device's pointer here
-    d->ws = nullptr;
+    if (d->ws && d->ws_dev == dev && d->ws_bytes >= need) return EATSS_OK;
+    free_ws(d);
     d->ws_bytes = 0;
     cudaError_t e = cudaMalloc(&d->ws, need);
     if (e != cudaSuccess) return cuda_fail(e, "eatss_run(workspace)");
@@ -352,11 +363,14 @@ static eatss_status check_bufs(const eatss_kernel_desc *d, void *const *b) {
     return EATSS_OK;
 }
 
+// The carve-out request of a descriptor's launches (sigma and exec.carveout_exact).
+static int exec_cv(const eatss_kernel_desc *d) { return cv_make(d->exec.split_pct, d->exec.carveout_exact != 0); }
+
 // Issue the stencil time loop on stream s (no graph).
 static cudaError_t stencil_issue(const eatss_kernel_desc *d, const int64_t *t, void *const *b, cudaStream_t s) {
     const bool f64 = d->dtype == EATSS_F64;
     const int64_t n = d->dims[0];
-    const int cv = d->exec.split_pct;
+    const int cv = exec_cv(d);
     cudaError_t e = cudaSuccess;
     if (n < 3) return cudaSuccess;
     const bool untiled = d->exec.engine == EATSS_ENGINE_UNTILED;
@@ -387,19 +401,29 @@ static cudaError_t stencil_issue(const eatss_kernel_desc *d, const int64_t *t, v
 
 static eatss_status stencil_run(eatss_kernel_desc *d, const int64_t *t, void *const *b, cudaStream_t s) {
     if (!d->exec.use_graph || d->tsteps <= 1) {
+        take_carveout();
         cudaError_t e = stencil_issue(d, t, b, s);
+        d->graph_cv = take_carveout();
         return e == cudaSuccess ? EATSS_OK : cuda_fail(e, "eatss_run(stencil)");
     }
     GraphKey key;
     key.tiles.assign(t, t + eatss_desc_num_loops(d));
     key.tiles.push_back(d->exec.engine);  // a tiled and an untiled time loop are different graphs
+    key.tiles.push_back(d->exec.split_pct);  // the carve-out is captured with each launch
+    key.tiles.push_back(d->exec.carveout_exact);
+    int gdev = 0;
+    cudaGetDevice(&gdev);
+    key.tiles.push_back(gdev);  // a graph is instantiated for one device
     for (int i = 0; i < d->num_buffers; i++) key.bufs.push_back((uintptr_t)b[i]);
     key.stream = 0;  // graphs are stream-independent; launched on the caller's stream
     cudaGraphExec_t exec = nullptr;
     {
         std::lock_guard<std::mutex> lk(d->graph_mu);
         auto it = d->graphs.find(key);
-        if (it != d->graphs.end()) exec = (cudaGraphExec_t)it->second;
+        if (it != d->graphs.end()) {
+            exec = (cudaGraphExec_t)it->second;
+            d->graph_cv = d->graph_cvs[key];
+        }
     }
     if (!exec) {
         // set function attributes outside capture by issuing nothing: attributes are
@@ -412,7 +436,9 @@ static eatss_status stencil_run(eatss_kernel_desc *d, const int64_t *t, void *co
             cudaStreamDestroy(cs);
             return cuda_fail(e, "cudaStreamBeginCapture");
         }
+        take_carveout();
         cudaError_t ei = stencil_issue(d, t, b, cs);
+        const int cap_cv = take_carveout();
         cudaGraph_t g = nullptr;
         e = cudaStreamEndCapture(cs, &g);
         cudaStreamDestroy(cs);
@@ -426,6 +452,8 @@ static eatss_status stencil_run(eatss_kernel_desc *d, const int64_t *t, void *co
         if (e != cudaSuccess) return cuda_fail(e, "cudaGraphInstantiate");
         std::lock_guard<std::mutex> lk(d->graph_mu);
         d->graphs[key] = exec;
+        d->graph_cvs[key] = cap_cv;
+        d->graph_cv = cap_cv;
     }
     cudaError_t e = cudaGraphLaunch(exec, s);
     return e == cudaSuccess ? EATSS_OK : cuda_fail(e, "cudaGraphLaunch");
@@ -442,7 +470,7 @@ eatss_kernel_desc::~eatss_kernel_desc() {
     for (void *e : hev) cudaEventDestroy((cudaEvent_t)e);
     for (void *st : hstream)
         if (st) cudaStreamDestroy((cudaStream_t)st);
-    if (ws) cudaFree(ws);
+    free_ws(this);
 }
 
 // exec.time_kernels: a {start, stop} event pair per nest on the current device (nullptr if off)
@@ -593,6 +621,9 @@ eatss_status eatss_desc_set_exec(eatss_kernel_desc *d, const eatss_exec_opts *o)
     if (!d || !o) return fail(EATSS_E_INVALID, "eatss_desc_set_exec: null argument");
     if (o->split_pct < 0 || o->split_pct > 100) return fail(EATSS_E_INVALID, "split_pct must be 0..100");
     if (o->engine < 0 || o->engine > 3) return fail(EATSS_E_INVALID, "bad engine");
+    if (o->warp_align != 0 && o->warp_align != 4 && o->warp_align != 8 && o->warp_align != 16 && o->warp_align != 32)
+        return fail(EATSS_E_INVALID, "warp_align must be 0, 4, 8, 16 or 32");
+    if (o->carveout_exact != 0 && o->carveout_exact != 1) return fail(EATSS_E_INVALID, "carveout_exact must be 0 or 1");
     d->exec = *o;
     return EATSS_OK;
 }
@@ -651,7 +682,7 @@ eatss_status eatss_plan(const eatss_kernel_desc *d, const int64_t *tiles, eatss_
         auto cn = contraction_nests(d, b);
         if (simt_untranspose(d)) untranspose_nests(d, cn, b[EATSS_MAX_BUFFERS - 1]);
         for (int i = 0; i < (int)cn.size(); i++) {
-            ContractPlan p = plan_contraction(cn[i], tiles, 232448);
+            ContractPlan p = plan_contraction(cn[i], tiles, 232448, d->exec.warp_align);
             eatss_launch_plan &o = plans[i];
             std::memset(&o, 0, sizeof(o));
             o.nest = i; o.engine = 1;
@@ -659,7 +690,7 @@ eatss_status eatss_plan(const eatss_kernel_desc *d, const int64_t *tiles, eatss_
             o.block_x = p.bx; o.block_y = p.by; o.rm = p.rm; o.rn = p.rn; o.vec = p.vec;
             o.passes = p.passes_i * p.passes_j; o.smem_bytes = p.smem_bytes;
             o.a_in_smem = p.a_smem; o.b_in_smem = p.b_smem; o.carveout_pct = d->exec.split_pct;
-            o.simt_x = std::min(32, p.bx);
+            o.simt_x = plan_simt_x(p);
             o.tile[0] = p.Ti; o.tile[1] = p.Tj; o.tile[2] = p.Tk;
         }
         *n_plans = (int)cn.size();
@@ -779,10 +810,19 @@ static cudaError_t lowdim_run(const eatss_kernel_desc *d, const int64_t *t, void
     }
 }
 
+static eatss_status run_body(eatss_kernel_desc *d, int only_nest, const int64_t *tiles, void *const *buffers,
+                             void *stream);
 static eatss_status run_impl(const eatss_kernel_desc *cd, int only_nest, const int64_t *tiles,
                              void *const *buffers, void *stream) {
     auto *d = const_cast<eatss_kernel_desc *>(cd);
     if (!d) return fail(EATSS_E_INVALID, "eatss_run: null descriptor");
+    d->last_cv.assign(d->nests.size(), -1);
+    take_carveout();
+    return run_body(d, only_nest, tiles, buffers, stream);
+}
+
+static eatss_status run_body(eatss_kernel_desc *d, int only_nest, const int64_t *tiles, void *const *buffers,
+                             void *stream) {
     eatss_status st = check_tiles(d, tiles);
     if (st != EATSS_OK) return st;
     st = check_bufs(d, buffers);
@@ -803,9 +843,17 @@ static eatss_status run_impl(const eatss_kernel_desc *cd, int only_nest, const i
             if (e != cudaSuccess) return cuda_fail(e, "eatss_run(syrk layout pass)");
             untranspose_nests(d, cn, d->ws);
         }
+        if (d->exec.engine == EATSS_ENGINE_TENSOR) {  // split-operand scratch for the tcgen05 GEMMs
+            size_t need = 0;
+            for (int i = 0; i < (int)cn.size(); i++) {
+                ContractPlan p = plan_contraction(cn[i], tiles, sl, d->exec.warp_align);
+                if (tcm_applicable(cn[i], p)) need = std::max(need, tcm_ws_floats(cn[i], p));
+            }
+            if (need && (st = ensure_ws(d, need * 4)) != EATSS_OK) return st;
+        }
         for (int i = 0; i < (int)cn.size(); i++) {
             if (only_nest >= 0 && i != only_nest) continue;
-            ContractPlan p = plan_contraction(cn[i], tiles, sl);
+            ContractPlan p = plan_contraction(cn[i], tiles, sl, d->exec.warp_align);
             int tsm = 0, tcols = 0;
             const bool want_tc = d->exec.engine == EATSS_ENGINE_TENSOR;
             // MMA-legal tiles (Ti = 128) take the TMA/SS-UMMA GEMM; narrow tiles the transposed TS kernel
@@ -815,10 +863,11 @@ static eatss_status run_impl(const eatss_kernel_desc *cd, int only_nest, const i
                 return fail(EATSS_E_UNSUPPORTED, "eatss_run: tensor engine not applicable to this tile/operand layout");
             cudaEvent_t *ev = kernel_events(d, i);
             if (ev && !tcm) cudaEventRecord(ev[0], s);
-            cudaError_t e = tcm  ? launch_tcm_contraction(cn[i], p, s, ev)
-                            : tc ? launch_tc_contraction(cn[i], p, d->exec.split_pct, s)
-                                 : launch_contraction(cn[i], p, d->exec.split_pct, nullptr, s);
+            cudaError_t e = tcm  ? launch_tcm_contraction(cn[i], p, (float *)d->ws, d->ws_bytes / 4, s, ev)
+                            : tc ? launch_tc_contraction(cn[i], p, exec_cv(d), s)
+                                 : launch_contraction(cn[i], p, exec_cv(d), nullptr, s);
             if (ev && !tcm) cudaEventRecord(ev[1], s);
+            d->last_cv[i] = take_carveout();
             if (e != cudaSuccess) return cuda_fail(e, "eatss_run(contraction)");
         }
         return EATSS_OK;
@@ -874,6 +923,7 @@ static eatss_status run_impl(const eatss_kernel_desc *cd, int only_nest, const i
         if (ev) cudaEventRecord(ev[0], s);
         const eatss_status r = stencil_run(d, tiles, buffers, s);
         if (ev) cudaEventRecord(ev[1], s);
+        for (auto &v : d->last_cv) v = d->graph_cv;  // set by the capture / direct issue
         return r;
     }
     cudaEvent_t *ev = kernel_events(d, 0);
@@ -882,14 +932,16 @@ static eatss_status run_impl(const eatss_kernel_desc *cd, int only_nest, const i
             return fail(EATSS_E_UNSUPPORTED, "eatss_run: tensor engine needs a ccsd tile (1,1,Th1,Tp6,Tp5,Tp4,>=H7) "
                                              "with Th1*Tp5*Tp4 <= 128, Tp6 % 16 == 0, Tp4 % 4 == 0, "
                                              "P4 % 4 == 0, H7 % 4 == 0, H7 <= 64");
+        if ((st = ensure_ws(d, ccsd_tc_ws_floats(d->dims.data()) * 4)) != EATSS_OK) return st;
         cudaError_t e = launch_ccsd_tc((float *)buffers[0], (const float *)buffers[1], (const float *)buffers[2],
-                                       d->dims.data(), tiles, 0, d->dims[0], s, ev);
+                                       d->dims.data(), tiles, 0, d->dims[0], (float *)d->ws, d->ws_bytes / 4, s, ev);
         return e == cudaSuccess ? EATSS_OK : cuda_fail(e, "eatss_run(ccsd_t_d1, tensor)");
     }
     if (ev) cudaEventRecord(ev[0], s);
     cudaError_t e = launch_ccsd_d1((float *)buffers[0], (const float *)buffers[1], (const float *)buffers[2],
-                                   d->dims.data(), tiles, 0, d->dims[0], d->exec.split_pct, nullptr, s);
+                                   d->dims.data(), tiles, 0, d->dims[0], exec_cv(d), nullptr, s);
     if (ev) cudaEventRecord(ev[1], s);
+    d->last_cv[0] = take_carveout();
     return e == cudaSuccess ? EATSS_OK : cuda_fail(e, "eatss_run(ccsd_t_d1)");
 }
 
@@ -1016,16 +1068,17 @@ eatss_status eatss_run_host(const eatss_kernel_desc *cd, const int64_t *tiles, v
             blk.M = rows;
             blk.A = dA + r0 * rowA;
             blk.C = dC + r0 * rowC;
-            ContractPlan p = plan_contraction(blk, tiles, sl);
+            ContractPlan p = plan_contraction(blk, tiles, sl, d->exec.warp_align);
             const bool want_tc = d->exec.engine == EATSS_ENGINE_TENSOR;
             int tsm = 0, tcols = 0;
             const bool tcm = want_tc && tcm_applicable(blk, p);
             const bool tc = want_tc && !tcm && tc_plan(blk, p, &tsm, &tcols);
             if (want_tc && !tc && !tcm)
                 return fail(EATSS_E_UNSUPPORTED, "eatss_run_host: tensor engine not applicable to this tile");
-            e = tcm  ? launch_tcm_contraction(blk, p, s, nullptr)
-                : tc ? launch_tc_contraction(blk, p, d->exec.split_pct, s)
-                     : launch_contraction(blk, p, d->exec.split_pct, nullptr, s);
+            if (tcm && (st = ensure_ws(d, tcm_ws_floats(blk, p) * 4)) != EATSS_OK) return st;
+            e = tcm  ? launch_tcm_contraction(blk, p, (float *)d->ws, d->ws_bytes / 4, s, nullptr)
+                : tc ? launch_tc_contraction(blk, p, exec_cv(d), s)
+                     : launch_contraction(blk, p, exec_cv(d), nullptr, s);
             if (e != cudaSuccess) return cuda_fail(e, "eatss_run_host(gemm block)");
             cudaEventRecord(ecomp, s);
             cudaStreamWaitEvent(sout, ecomp, 0);
@@ -1075,11 +1128,11 @@ eatss_status eatss_coverage(const eatss_kernel_desc *d, int nest, const int64_t 
         void *b[EATSS_MAX_BUFFERS];
         for (int i = 0; i < EATSS_MAX_BUFFERS; i++) b[i] = (void *)(uintptr_t)(256 * (i + 1));
         auto cn = contraction_nests(d, b);
-        ContractPlan p = plan_contraction(cn[nest], tiles, smem_limit_bytes());
+        ContractPlan p = plan_contraction(cn[nest], tiles, smem_limit_bytes(), d->exec.warp_align);
         p.a_smem = false;  // no operand traffic in coverage mode
         p.b_smem = false;
         p.smem_bytes = 0;
-        cudaError_t e = launch_contraction(cn[nest], p, d->exec.split_pct, counts, s);
+        cudaError_t e = launch_contraction(cn[nest], p, exec_cv(d), counts, s);
         return e == cudaSuccess ? EATSS_OK : cuda_fail(e, "eatss_coverage");
     }
     if (is_lowdim(d->kind))
@@ -1096,11 +1149,11 @@ eatss_status eatss_coverage(const eatss_kernel_desc *d, int nest, const int64_t 
     const int64_t n = d->dims[0];
     cudaError_t e;
     if (d->kind == EATSS_JACOBI2D)
-        e = launch_jacobi2d_sweep(nullptr, nullptr, nullptr, n, tiles[0], tiles[1], f64, d->exec.split_pct, counts, s);
+        e = launch_jacobi2d_sweep(nullptr, nullptr, nullptr, n, tiles[0], tiles[1], f64, exec_cv(d), counts, s);
     else if (d->kind == EATSS_HEAT3D)
-        e = launch_heat3d_sweep(nullptr, nullptr, n, tiles[0], tiles[1], tiles[2], f64, d->exec.split_pct, counts, s);
+        e = launch_heat3d_sweep(nullptr, nullptr, n, tiles[0], tiles[1], tiles[2], f64, exec_cv(d), counts, s);
     else
-        e = launch_ccsd_d1(nullptr, nullptr, nullptr, d->dims.data(), tiles, 0, d->dims[0], d->exec.split_pct,
+        e = launch_ccsd_d1(nullptr, nullptr, nullptr, d->dims.data(), tiles, 0, d->dims[0], exec_cv(d),
                            counts, s);
     return e == cudaSuccess ? EATSS_OK : cuda_fail(e, "eatss_coverage");
 }
@@ -1115,7 +1168,7 @@ int64_t eatss_launches_per_run(const eatss_kernel_desc *d, const int64_t *tiles)
         const int sl = smem_limit_bytes();
         int64_t total = 0;
         for (auto &n : cn) {
-            ContractPlan p = plan_contraction(n, tiles, sl);
+            ContractPlan p = plan_contraction(n, tiles, sl, d->exec.warp_align);
             int tsm = 0, tcols = 0;
             total += tcm_applicable(n, p) ? tcm_launches(n, p) : tc_plan(n, p, &tsm, &tcols) ? 1 : 0;
         }
@@ -1133,7 +1186,7 @@ int64_t eatss_launches_per_run(const eatss_kernel_desc *d, const int64_t *tiles)
             untranspose_nests(d, cn, b[EATSS_MAX_BUFFERS - 1]);
             total += 1;  // the layout pass
         }
-        for (auto &n : cn) total += contraction_launches(n, plan_contraction(n, tiles, sl));
+        for (auto &n : cn) total += contraction_launches(n, plan_contraction(n, tiles, sl, d->exec.warp_align));
         return total;
     }
     switch (d->kind) {
@@ -1155,6 +1208,14 @@ int64_t eatss_launches_per_run(const eatss_kernel_desc *d, const int64_t *tiles)
         }
     }
     return -1;
+}
+
+eatss_status eatss_last_carveout(const eatss_kernel_desc *d, int32_t *pct, int32_t cap, int32_t *n) {
+    if (!d || !n || (cap > 0 && !pct)) return fail(EATSS_E_INVALID, "eatss_last_carveout: bad argument");
+    const int cnt = (int)d->last_cv.size();
+    for (int i = 0; i < cnt && i < cap; i++) pct[i] = d->last_cv[i];
+    *n = cnt;
+    return EATSS_OK;
 }
 
 eatss_status eatss_last_kernel_ms(const eatss_kernel_desc *cd, float *ms, int32_t cap, int32_t *n) {

@@ -19,6 +19,9 @@
 #include <cstdint>
 #include <cstdlib>
 
+#include "contract.cuh"
+#include "devsw.hpp"
+
 namespace eatss {
 
 struct CcsdArgs {
@@ -230,8 +233,8 @@ static CcsdFastPlan plan_ccsd_fast(const int64_t *dims, const int *T, int Rt, in
     f.ctp = ((Ct + 3) / 4) * 4;
     f.S = 3;
     int group = std::max(1, (16 + T[6] - 1) / T[6]);
-    if (const char *e = getenv("EATSS_CCSD_GROUP")) group = std::max(1, atoi(e));
-    const bool want_prefetch = !(getenv("EATSS_CCSD_NOPREFETCH") && atoi(getenv("EATSS_CCSD_NOPREFETCH")));
+    if (devsw("EATSS_CCSD_GROUP", 0) > 0) group = devsw("EATSS_CCSD_GROUP", 0);
+    const bool want_prefetch = devsw("EATSS_CCSD_NOPREFETCH", 0) == 0;
     auto layout = [&](int kst, bool pre, int64_t *bytes, int *t3s_off) {
         const int64_t ring = (int64_t)f.S * kst * (f.rtp + f.ctp);
         const int64_t tab = ((ring + 1) & ~1LL);
@@ -269,7 +272,9 @@ static cudaError_t ccsd_fast_launch(const CcsdFastArgs &a, const CcsdFastPlan &f
     auto k = ccsd_fast_kernel<RM, RN, V>;
     cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, f.smem);
     if (e != cudaSuccess) return e;
-    cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, std::max(carveout, 50));
+    const int cvr = cv_resolve(carveout, 50);
+    cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, cvr);
+    note_carveout(cvr);
     k<<<dim3((unsigned)gx, (unsigned)gy), dim3(f.bx, f.by), f.smem, s>>>(a);
     return cudaGetLastError();
 }
@@ -343,7 +348,8 @@ static cudaError_t ccsd_launch(const CcsdArgs &a, const CcsdPlan &p, int carveou
     auto k = ccsd_d1_kernel<RM, RN, MODE>;
     cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem);
     if (e != cudaSuccess) return e;
-    cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, carveout);
+    cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, cv_resolve(carveout, 0));
+    note_carveout(cv_resolve(carveout, 0));
     k<<<dim3((unsigned)p.gx, (unsigned)p.gy), dim3(p.bx, p.by), p.smem, s>>>(a);
     return cudaGetLastError();
 }
@@ -372,7 +378,7 @@ cudaError_t launch_ccsd_d1(float *t3, const float *t2, const float *v2, const in
     d2[0] = h3_count;
     CcsdPlan p = plan_ccsd(d2, tiles);
     if (p.gy > 65535 || p.gx > 2147483647LL) return cudaErrorInvalidConfiguration;
-    if (!counts && !(getenv("EATSS_CCSD_SLOW") && atoi(getenv("EATSS_CCSD_SLOW")))) {
+    if (!counts && devsw("EATSS_CCSD_SLOW", 0) == 0) {
         CcsdFastPlan f = plan_ccsd_fast(d2, p.T, p.Rt, p.Ct);
         if (f.ok) {
             CcsdFastArgs a;

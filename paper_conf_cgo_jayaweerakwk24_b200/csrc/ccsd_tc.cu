@@ -486,26 +486,6 @@ static bool make_map_nd(CUtensorMap *m, const float *base, int rank, const uint6
 }  // namespace ccsdtc
 
 namespace {
-std::mutex g_cws_mu;
-float *g_cws = nullptr;
-size_t g_cws_elems = 0;
-int g_cws_dev = -1;
-float *ccsd_workspace(size_t elems) {
-    std::lock_guard<std::mutex> lk(g_cws_mu);
-    int dev = 0;
-    cudaGetDevice(&dev);
-    if (g_cws && (g_cws_elems < elems || g_cws_dev != dev)) {
-        cudaFree(g_cws);
-        g_cws = nullptr;
-    }
-    if (!g_cws) {
-        if (cudaMalloc(&g_cws, elems * 4) != cudaSuccess) return g_cws = nullptr;
-        g_cws_elems = elems;
-        g_cws_dev = dev;
-    }
-    return g_cws;
-}
-
 struct CcsdTcPlan {
     bool ok = false;
     ccsdtc::Args a{};
@@ -531,8 +511,13 @@ CcsdTcPlan plan_ccsd_tc(const int64_t *dims, const int64_t *tiles) {
     a.n_h1t = (int)((H1 + a.Th1 - 1) / a.Th1); a.n_p5t = (int)((P5 + a.Tp5 - 1) / a.Tp5);
     a.n_p4t = (int)((P4 + a.Tp4 - 1) / a.Tp4); a.n_p6t = (int)((P6 + a.Tp6 - 1) / a.Tp6);
     a.nkb = (int)((H7 + 31) / 32);
-    a.order = getenv("EATSS_CCSD_TC_ORDER") ? atoi(getenv("EATSS_CCSD_TC_ORDER")) : 1;
+    static const int order_env = getenv("EATSS_CCSD_TC_ORDER") ? atoi(getenv("EATSS_CCSD_TC_ORDER")) : 1;
+    a.order = order_env;
+#ifdef EATSS_DEVTOOLS  // component switches for cost isolation (results then wrong): never in the product build
     a.dbg = getenv("EATSS_CCSD_TC_DBG") ? atoi(getenv("EATSS_CCSD_TC_DBG")) : 0;
+#else
+    a.dbg = 0;
+#endif
     a.nks = (int)((H7 + 7) / 8);
     a.bstride = 32;
     while (a.bstride < a.NV) a.bstride *= 2;
@@ -547,9 +532,11 @@ CcsdTcPlan plan_ccsd_tc(const int64_t *dims, const int64_t *tiles) {
     const int budget = 232448 - fixed;
     a.XB = 2;
     if (budget - ccsdtc::NGRP * a.XB * a.x_stage < 3 * a.v_stage) a.XB = 1;  // keep >= 3 v2 stages if possible
-    if (const char *e = getenv("EATSS_CCSD_TC_XB")) a.XB = std::max(1, std::min(2, atoi(e)));
+    static const int xb_env = getenv("EATSS_CCSD_TC_XB") ? atoi(getenv("EATSS_CCSD_TC_XB")) : 0;  // development
+    if (xb_env > 0) a.XB = std::min(2, xb_env);
     a.SV = std::min(6, (budget - ccsdtc::NGRP * a.XB * a.x_stage) / a.v_stage);
-    if (const char *e = getenv("EATSS_CCSD_TC_VSTAGES")) a.SV = std::max(1, std::min(a.SV, atoi(e)));
+    static const int sv_env = getenv("EATSS_CCSD_TC_VSTAGES") ? atoi(getenv("EATSS_CCSD_TC_VSTAGES")) : 0;
+    if (sv_env > 0) a.SV = std::min(a.SV, sv_env);
     if (a.SV < 2) return pl;
     pl.smem = fixed + a.SV * a.v_stage + ccsdtc::NGRP * a.XB * a.x_stage;
     pl.ok = true;
@@ -561,8 +548,13 @@ bool ccsd_tc_applicable(const int64_t *dims, const int64_t *tiles) {
     return plan_ccsd_tc(dims, tiles).ok && tcm::encode_fn() != nullptr;
 }
 
+size_t ccsd_tc_ws_floats(const int64_t *dims) {  // v2's tf32 lo half (descriptor-owned scratch)
+    return (size_t)(dims[0] * dims[1] * dims[3] * dims[6] + 64);
+}
+
 cudaError_t launch_ccsd_tc(float *t3, const float *t2, const float *v2, const int64_t *dims, const int64_t *tiles,
-                           int64_t h3_begin, int64_t h3_count, cudaStream_t s, cudaEvent_t *ev) {
+                           int64_t h3_begin, int64_t h3_count, float *ws, size_t ws_floats, cudaStream_t s,
+                           cudaEvent_t *ev) {
     CcsdTcPlan pl = plan_ccsd_tc(dims, tiles);
     if (!pl.ok || !tcm::encode_fn()) return cudaErrorNotSupported;
     ccsdtc::Args a = pl.a;
@@ -572,9 +564,12 @@ cudaError_t launch_ccsd_tc(float *t3, const float *t2, const float *v2, const in
     a.units = (int64_t)a.n_h1t * a.n_p5t * a.n_p4t * a.nhh * a.n_p6t;
     if (a.units == 0) return cudaSuccess;
     const int64_t n_v2 = (int64_t)a.H3 * H2 * P6 * H7;
-    float *v2_lo = ccsd_workspace((size_t)(n_v2 + 64));
-    if (!v2_lo) return cudaErrorMemoryAllocation;
-    ccsdtc::prep_kernel<<<148 * 4, 256, 0, s>>>(v2, v2_lo, n_v2);
+    float *v2_lo = ws;
+    if (!v2_lo || ws_floats < (size_t)(n_v2 + 64)) return cudaErrorInvalidValue;
+    int dev = 0, nsm = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    ccsdtc::prep_kernel<<<nsm * 4, 256, 0, s>>>(v2, v2_lo, n_v2);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
     CUtensorMap mV, mVlo;
@@ -613,12 +608,10 @@ cudaError_t launch_ccsd_tc(float *t3, const float *t2, const float *v2, const in
             smem_set = pl.smem;
         }
     }
-    int dev = 0, nsm = 148;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     const int grid = (int)std::min<int64_t>(nsm, a.units);
     static unsigned long long *prof = nullptr;
-    if (getenv("EATSS_CCSD_TC_PROF")) {
+    static const bool prof_on = getenv("EATSS_CCSD_TC_PROF") != nullptr;  // development: wait profile
+    if (prof_on) {
         if (!prof) cudaMalloc(&prof, 16 * sizeof(unsigned long long));
         cudaMemsetAsync(prof, 0, 16 * sizeof(unsigned long long), s);
         a.prof = prof;

@@ -25,6 +25,7 @@
 #include <cstdlib>
 
 #include "contract.cuh"
+#include "devsw.hpp"
 
 namespace eatss {
 
@@ -47,8 +48,19 @@ struct CArgs {
     int64_t nfull;   // staged: tiles run whole; tiles >= nfull are split along k into sp parts
     int sp;          // staged: 1 = 2-D grid, no split
     int passes_i, passes_j;
+    int waf;          // lanes of each warp along j (0: linear layout, tx fastest)
     int32_t *counts;  // coverage mode
 };
+
+// Thread layout with WAF lanes of every warp along the CMA loop j (the SIMT length as a fraction of
+// the warp size): lane l of warp w owns column slot (w % wx)*WAF + l % WAF and row slot
+// (w / wx)*(32/WAF) + l / WAF, wx = BX / WAF.  The planner makes BX a multiple of WAF and BY a
+// multiple of 32/WAF, so this is a permutation of the (tx, ty) slots.
+__device__ __forceinline__ void warp_layout(int tid, int BX, int waf, int &tx, int &ty) {
+    const int w = tid >> 5, l = tid & 31, wx = BX / waf;
+    tx = (w % wx) * waf + (l % waf);
+    ty = (w / wx) * (32 / waf) + l / waf;
+}
 
 enum { MODE_RESIDENT = 0, MODE_STREAM = 1, MODE_COVER = 2 };
 
@@ -144,9 +156,10 @@ __global__ void __launch_bounds__((16384 / (RM * RN)) < 1024 ? (16384 / (RM * RN
     T *As = reinterpret_cast<T *>(smem_raw);
     T *Bs = As + (p.a_smem ? p.nbuf * p.Ti * p.tkp : 0);
 
-    const int tx = threadIdx.x, ty = threadIdx.y;
     const int BX = blockDim.x, BY = blockDim.y;
-    const int tid = ty * BX + tx, nthr = BX * BY;
+    const int tid = threadIdx.y * BX + threadIdx.x, nthr = BX * BY;
+    int tx = threadIdx.x, ty = threadIdx.y;
+    if (p.waf) warp_layout(tid, BX, p.waf, tx, ty);
     const int64_t i0 = (int64_t)blockIdx.y * p.Ti, j0 = (int64_t)blockIdx.x * p.Tj;
     const int rows = (int)imin64(p.Ti, p.M - i0);
     const int cols = (int)imin64(p.Tj, p.N - j0);
@@ -469,7 +482,7 @@ inline int maxthreads(int rm, int rn) { return std::min(1024, 16384 / (rm * rn))
 inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 }  // namespace
 
-ContractPlan plan_contraction(const ContractNest &n, const int64_t *tiles, int smem_limit) {
+ContractPlan plan_contraction(const ContractNest &n, const int64_t *tiles, int smem_limit, int waf_req) {
     ContractPlan p;
     p.Ti = std::max<int64_t>(1, std::min(tiles[0], n.M));
     p.Tj = std::max<int64_t>(1, std::min(tiles[1], n.N));
@@ -484,20 +497,41 @@ ContractPlan plan_contraction(const ContractNest &n, const int64_t *tiles, int s
     const int64_t rows = p.Ti, cols = p.Tj;
     const int64_t outputs = rows * cols;
     int target_threads = 256;
-    if (const char *e = getenv("EATSS_THREADS")) target_threads = std::max(32, atoi(e));
+    if (devsw("EATSS_THREADS", 0) > 0) target_threads = std::max(32, devsw("EATSS_THREADS", 0));
     const int64_t want = cdiv(outputs, target_threads);
-    // smallest micro-tile reaching `want` outputs/thread that does not exceed the tile
-    int pick = -1;
+    const int waf = (waf_req == 4 || waf_req == 8 || waf_req == 16 || waf_req == 32) ? waf_req : 0;
+    const int yq = waf ? 32 / waf : 1;  // rows of one warp
+    p.waf = waf;
+    auto rup = [](int64_t v, int64_t m) { return ((v + m - 1) / m) * m; };
+    // smallest micro-tile reaching `want` outputs/thread that does not exceed the tile; with a warp
+    // alignment the thread grid is rounded to whole warps of WAF x 32/WAF (idle slots predicated) and
+    // the first candidate that keeps >= 3/4 of the slots busy is taken (else the busiest one)
+    int pick = -1, best = -1;
+    double best_u = -1.0;
     for (int c = 0; c < ncand; c++) {
         if (cand[c].rm > std::max<int64_t>(rows, 1) && c > 0) continue;
         if (cand[c].rn > ((cols + p.vec - 1) / p.vec) * p.vec && c > 0) continue;
-        pick = c;
-        if (cand[c].rm * cand[c].rn >= want) break;
+        if (!waf) {
+            pick = c;
+            if (cand[c].rm * cand[c].rn >= want) break;
+            continue;
+        }
+        const int64_t by0 = cdiv(rows, cand[c].rm), bx0 = cdiv(cols, cand[c].rn);
+        const int64_t byr = rup(by0, yq), bxr = rup(bx0, waf);
+        if (bxr * byr > maxthreads(cand[c].rm, cand[c].rn)) continue;
+        const double u = (double)(by0 * bx0) / (double)(byr * bxr);
+        if (u > best_u) { best_u = u; best = c; }
+        if (cand[c].rm * cand[c].rn >= want && u >= 0.75) { pick = c; break; }
     }
+    if (waf && pick < 0) pick = best;
     if (pick < 0) pick = 0;
     p.rm = cand[pick].rm;
     p.rn = cand[pick].rn;
     int64_t by = cdiv(rows, p.rm), bx = cdiv(cols, p.rn);
+    if (waf) {
+        by = rup(by, yq);
+        bx = rup(bx, waf);
+    }
     const int mt = maxthreads(p.rm, p.rn);
     if (by * bx <= mt) {
         p.stream = false;
@@ -508,8 +542,10 @@ ContractPlan plan_contraction(const ContractNest &n, const int64_t *tiles, int s
         p.rm = 8;
         p.rn = 8;
         const int lim = maxthreads(8, 8);
-        p.bx = (int)std::min<int64_t>(cdiv(cols, p.rn), lim);
+        p.bx = (int)std::min<int64_t>(cdiv(cols, p.rn), lim / yq);
+        if (waf) p.bx = std::max(waf, p.bx / waf * waf);
         p.by = (int)std::max<int64_t>(1, std::min<int64_t>(cdiv(rows, p.rm), lim / p.bx));
+        if (waf) p.by = std::max(yq, p.by / yq * yq);
         p.stream = true;
         p.passes_i = (int)cdiv(rows, (int64_t)p.by * p.rm);
         p.passes_j = (int)cdiv(cols, (int64_t)p.bx * p.rn);
@@ -547,7 +583,7 @@ ContractPlan plan_contraction(const ContractNest &n, const int64_t *tiles, int s
         // with 16-byte copies (k-pitch kst + 4: conflict-free 16-byte reads along k)
         const uintptr_t bb = reinterpret_cast<uintptr_t>(n.B);
         const bool bt4 = n.transB && !n.f64 && n.ldb % 4 == 0 && bb % 16 == 0 &&
-                         !(getenv("EATSS_TRANSB_LEGACY") && atoi(getenv("EATSS_TRANSB_LEGACY")));
+                         devsw("EATSS_TRANSB_LEGACY", 0) == 0;
         auto stage_of = [&](int64_t ks) {
             const int64_t b = bt4 ? bjp * (ks + 4) : ks * bjp;
             return (ks * aip + b) * esz;
@@ -556,12 +592,12 @@ ContractPlan plan_contraction(const ContractNest &n, const int64_t *tiles, int s
         const int64_t kmin = bt4 ? 4 : 1;
         while (kst > kmin && S * (stage_of(kst) + 16) > smem_limit)
             kst = bt4 ? std::max<int64_t>(4, ((kst / 2 + 3) / 4) * 4) : (kst + 1) / 2;
-        if (const char *e = getenv("EATSS_STAGES")) S = std::max(1, atoi(e));
-        if (const char *e = getenv("EATSS_KSUB")) kst = std::max<int64_t>(1, (p.Tk + atoi(e) - 1) / std::max(1, atoi(e)));
+        if (devsw("EATSS_STAGES", 0) > 0) S = devsw("EATSS_STAGES", 0);
+        if (const int ksub = devsw("EATSS_KSUB", 0)) kst = std::max<int64_t>(1, (p.Tk + ksub - 1) / std::max(1, ksub));
         if (bt4) kst = ((kst + 3) / 4) * 4;
         const int64_t stage_bytes = stage_of(kst);
         if (S * (stage_bytes + 16) > smem_limit) S = std::max<int64_t>(1, smem_limit / (stage_bytes + 16));
-        if (S * (stage_bytes + 16) <= smem_limit && !(getenv("EATSS_NO_STAGED") && atoi(getenv("EATSS_NO_STAGED")))) {
+        if (S * (stage_bytes + 16) <= smem_limit && devsw("EATSS_NO_STAGED", 0) == 0) {
             p.staged = true;
             p.nbuf = (int)S;
             p.kst = (int)kst;
@@ -578,6 +614,24 @@ ContractPlan plan_contraction(const ContractNest &n, const int64_t *tiles, int s
     return p;
 }
 
+int plan_simt_x(const ContractPlan &p) {
+    if (p.waf) return p.waf;
+    // linear layout (tx fastest): a warp spans min(32, bx) consecutive column slots when bx divides 32
+    // or is a multiple of it; otherwise its lanes wrap over rows and the run along j is bx % 32
+    if (p.bx >= 32) return p.bx % 32 == 0 ? 32 : p.bx % 32;
+    return p.bx;
+}
+
+namespace {
+thread_local int g_last_cv = -1;
+}
+void note_carveout(int pct) { g_last_cv = pct; }
+int take_carveout() {
+    const int v = g_last_cv;
+    g_last_cv = -1;
+    return v;
+}
+
 // ------------------------------------------------------------------ dispatch
 
 template <typename T, int RM, int RN, int V, bool TB, int MODE>
@@ -589,8 +643,10 @@ static cudaError_t launch_one(const CArgs<T> &a, const ContractPlan &p, int carv
         e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem_bytes);
         if (e != cudaSuccess) return e;
     }
-    e = cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, carveout);
+    const int cv = cv_resolve(carveout, 0);
+    e = cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, cv);
     if (e != cudaSuccess) return e;
+    note_carveout(cv);
     dim3 grid((unsigned)p.grid_x, (unsigned)p.grid_y, 1), block(p.bx, p.by, 1);
     k<<<grid, block, p.smem_bytes, s>>>(a);
     return cudaGetLastError();
@@ -606,18 +662,20 @@ static cudaError_t launch_staged(const CArgs<T> &a, const ContractPlan &p, int c
     if (e != cudaSuccess) return e;
     // The staged path keeps its operand slices in shared memory: the split's carve-out is
     // honoured unless it would cut the co-resident CTAs below what registers allow
-    // (the sigma -> carve-out mapping).
+    // (the sigma -> carve-out mapping); exec.carveout_exact keeps sigma as is.
+    int need = 0;
     cudaFuncAttributes fa;
     if (cudaFuncGetAttributes(&fa, k) == cudaSuccess && fa.numRegs > 0) {
         const int threads = ((p.bx * p.by + 31) / 32) * 32;
         const int nb_regs = 65536 / (((fa.numRegs + 7) / 8) * 8 * threads);
         const int per_cta = p.smem_bytes + 1024;  // + per-CTA reservation
         const int nb = std::max(1, std::min(nb_regs, 233472 / per_cta));
-        const int need = (int)std::min<int64_t>(100, (100LL * nb * per_cta + 233471) / 233472);
-        carveout = std::max(carveout, need);
+        need = (int)std::min<int64_t>(100, (100LL * nb * per_cta + 233471) / 233472);
     }
-    e = cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, carveout);
+    const int cv = cv_resolve(carveout, need);
+    e = cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, cv);
     if (e != cudaSuccess) return e;
+    if (!g_dry_launches) note_carveout(cv);
     dim3 block(p.bx, p.by, 1);
     // wave-quantisation tail: when the last wave would leave at least half of the resident-CTA
     // slots idle, its tiles are split along k (EATSS_SIMT_SPLITK=0 disables)
@@ -625,7 +683,7 @@ static cudaError_t launch_staged(const CArgs<T> &a, const ContractPlan &p, int c
     b.sp = 1;
     b.gx = p.grid_x;
     const int64_t T_ = p.grid_x * p.grid_y;
-    static const bool splitk = !(getenv("EATSS_SIMT_SPLITK") && atoi(getenv("EATSS_SIMT_SPLITK")) == 0);
+    static const bool splitk = devsw("EATSS_SIMT_SPLITK", 1) != 0;
     int nb = 0, dev = 0, nsm = 148;
     if (splitk && cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k, p.bx * p.by, p.smem_bytes) == cudaSuccess &&
         nb > 0) {
@@ -731,6 +789,7 @@ static cudaError_t launch_typed(const ContractNest &n, const ContractPlan &p, in
     a.tkp = p.tkp; a.tjp = p.tjp; a.bkp = p.bkp;
     a.gx = p.grid_x; a.nfull = 0; a.sp = 1;
     a.passes_i = p.passes_i; a.passes_j = p.passes_j;
+    a.waf = p.waf;
     a.counts = counts;
     if (counts) return by_variant<T, MODE_COVER>(a, p, n.transB, carveout, s);
     if (p.staged) {

@@ -6,6 +6,18 @@
 
 namespace eatss {
 
+// Carve-out request handed to the SIMT launchers: the model's split sigma in percent,
+// bit 8 set when it must be honoured exactly (exec.carveout_exact); otherwise it is a lower bound
+// the launcher raises as far as its register-limited resident CTAs need.  The
+// launchers report what they requested through note_carveout (read back per nest by the API).
+inline int cv_make(int pct, bool exact) { return pct | (exact ? 0x100 : 0); }
+inline int cv_resolve(int cv, int need) {
+    const int pct = cv & 0xff;
+    return (cv & 0x100) ? pct : (pct > need ? pct : need);
+}
+void note_carveout(int pct);  // thread-local: the last carve-out a launcher requested
+int take_carveout();          // read and reset (-1 when none was requested)
+
 // One gemm-like nest of the gemm family (gemm, 2mm, 3mm, syrk):
 //   C(i,j) = [init_zero ? 0 : beta*C(i,j)] + alpha * sum_k A(i,k) * B(k,j)
 //   A(i,k) = A[i*lda + k];  B(k,j) = transB ? B[j*ldb + k] : B[k*ldb + j];  C(i,j) = C[i*ldc + j]
@@ -37,17 +49,24 @@ struct ContractPlan {
     int bkp = 0;           // staged transposed operand kept as [j][k] rows of this k-pitch (0 = [k][j])
     int smem_bytes = 0;
     int64_t grid_x = 1, grid_y = 1;
+    int waf = 0;  // lanes of each warp along j (exec.warp_align; 0 = linear thread layout)
 };
 
-ContractPlan plan_contraction(const ContractNest &n, const int64_t *tiles, int smem_limit);
+ContractPlan plan_contraction(const ContractNest &n, const int64_t *tiles, int smem_limit, int waf = 0);
+// lanes of one warp laid along j by a plan (the executor's SIMT length)
+int plan_simt_x(const ContractPlan &p);
 // tensor-core (tcgen05, 3xTF32) executor: applicability / launch (tc_gemm.cu)
 bool tc_plan(const ContractNest &n, const ContractPlan &p, int *smem_bytes, int *tmem_cols);
 cudaError_t launch_tc_contraction(const ContractNest &n, const ContractPlan &p, int carveout, cudaStream_t s);
 // tcgen05 3xTF32 GEMM for MMA-legal tiles (Ti = 128, Tj in 32..256 step 32) (tc_mma.cu)
 bool tcm_applicable(const ContractNest &n, const ContractPlan &p);
+// Split-operand workspace (floats) one launch needs: owned by the caller's descriptor, so
+// concurrent descriptors (streams, devices, host threads) never share it.
+size_t tcm_ws_floats(const ContractNest &n, const ContractPlan &p);
+// ws: >= tcm_ws_floats() floats on the current device, used in stream order by this launch;
 // ev: optional {start, stop} events recorded around the GEMM kernel alone
-cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p, cudaStream_t s,
-                                   cudaEvent_t *ev = nullptr);
+cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p, float *ws, size_t ws_floats,
+                                   cudaStream_t s, cudaEvent_t *ev = nullptr);
 int tcm_launches(const ContractNest &n, const ContractPlan &p);  // kernels one launch_tcm_contraction issues
 cudaError_t launch_contraction(const ContractNest &n, const ContractPlan &p, int carveout_pct,
                                int32_t *coverage_counts, cudaStream_t s);

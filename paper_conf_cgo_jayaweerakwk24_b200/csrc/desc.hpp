@@ -58,16 +58,20 @@ struct eatss_kernel_desc {
     std::vector<int64_t> dims;
     int64_t tsteps = 0;
     double alpha = 1.5, beta = 1.2;
-    eatss_exec_opts exec{50, EATSS_ENGINE_AUTO, 1, 0};
+    eatss_exec_opts exec{50, EATSS_ENGINE_AUTO, 1, 0, 0, 0};
     std::vector<eatss::Nest> nests;
     int num_buffers = 0;
     std::vector<int64_t> buffer_elems;
     // cached stencil time-loop graphs (cudaGraphExec_t as void*)
     std::mutex graph_mu;
     std::map<eatss::GraphKey, void *> graphs;
+    std::map<eatss::GraphKey, int> graph_cvs;  // carve-out each graph's launches were captured with
+    int graph_cv = -1;                         // carve-out of the last stencil issue / replay
     // exec.time_kernels: start/stop events per nest of the last timed run (cudaEvent_t as void*)
     std::vector<void *> kev;
     int kev_dev = -1, kev_valid = 0;
+    // carve-out (percent) requested by each nest's main kernel in the last run (-1: none)
+    std::vector<int> last_cv;
     // eatss_run_host: library-owned device copies of the buffers, copy streams and events
     std::vector<void *> hbuf;
     std::vector<size_t> hbuf_bytes;

@@ -277,7 +277,11 @@ cudaError_t launch_mttkrp_tc(float *A, const float *B, const float *C, const flo
     p.nblk = (int)(p.ni * p.nk / BM);
     p.nkb = (int)(p.nl / BK);
     p.C = C;
+#ifdef EATSS_DEVTOOLS  // cost-isolation switches (results then wrong): never in the product build
     p.dbg = getenv("EATSS_MTC_DBG") ? atoi(getenv("EATSS_MTC_DBG")) : 0;
+#else
+    p.dbg = 0;
+#endif
     float *dlo = ws;
     p.part = ws + p.nj * p.nl;
     CUtensorMap mB, mDhi, mDlo;
@@ -299,7 +303,8 @@ cudaError_t launch_mttkrp_tc(float *A, const float *B, const float *C, const flo
         cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
         auto bytes = [&](int sh) { return 1024 + sh * hstage + 256 + NEPI * nj * 4; };
         p.S = SMAX;
-        if (const char *ev_s = getenv("EATSS_MTC_STAGES")) p.S = std::max(2, std::min(8, atoi(ev_s)));  // development
+        static const int st_env = getenv("EATSS_MTC_STAGES") ? atoi(getenv("EATSS_MTC_STAGES")) : 0;  // development
+        if (st_env > 0) p.S = std::max(2, std::min(8, st_env));
         while (p.S > 2 && bytes(p.S) > optin) p.S--;
         const int smem = bytes(p.S);
         cudaError_t r = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);

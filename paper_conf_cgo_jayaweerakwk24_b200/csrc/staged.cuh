@@ -59,8 +59,10 @@ __global__ void __launch_bounds__((16384 / (RM * RN)) < 1024 ? (16384 / (RM * RN
     const int S = p.nbuf;
     uint64_t *bars = reinterpret_cast<uint64_t *>(sm + S * stage_elems);  // 8-byte aligned (elems % 2 == 0)
 
-    const int tx = threadIdx.x, ty = threadIdx.y, BX = blockDim.x;
-    const int tid = ty * BX + tx, nthr = BX * blockDim.y;
+    const int BX = blockDim.x;
+    const int tid = threadIdx.y * BX + threadIdx.x, nthr = BX * blockDim.y;
+    int tx = threadIdx.x, ty = threadIdx.y;
+    if (p.waf) warp_layout(tid, BX, p.waf, tx, ty);  // WAF lanes per warp along j
     // tile of this CTA (Fig. 4 mapping); with a split wave tail (p.sp > 1, 1-D grid) the last
     // tiles are cut along k into sp parts whose partial sums are added to C atomically
     const int nk = (int)((p.K + p.Tk - 1) / p.Tk);

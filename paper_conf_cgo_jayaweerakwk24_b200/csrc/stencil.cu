@@ -22,6 +22,8 @@
 #include <cstdint>
 #include <cstdlib>
 
+#include "contract.cuh"
+
 namespace eatss {
 
 __device__ __forceinline__ int64_t smin64(int64_t a, int64_t b) { return a < b ? a : b; }
@@ -286,20 +288,35 @@ StencilPlan plan_heat3d(int64_t n, int64_t Ti, int64_t Tj, int64_t Tk, bool f64)
     return p;
 }
 
+// launch with the carve-out as a launch attribute (captured into graph nodes with the launch)
+template <typename... KArgs, typename... Args>
+static void launch_cv(void (*kern)(KArgs...), dim3 grid, dim3 block, int cv, cudaStream_t s, Args... args) {
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributePreferredSharedMemoryCarveout;
+    at[0].val.sharedMemCarveout = (unsigned)cv;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    note_carveout(cv);
+    cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
+}
+
 cudaError_t launch_jacobi2d_sweep(void *dst, const void *src, const void *bsrc, int64_t n, int64_t Ti,
                                   int64_t Tj, bool f64, int carveout, int32_t *counts, cudaStream_t s) {
     if (stencil_staged_enabled() && jacobi2d_staged_applicable(n, Ti, Tj, f64))
         return launch_jacobi2d_staged((float *)dst, (const float *)src, (const float *)bsrc, n, Ti, Tj, carveout,
                                       counts, s);
     StencilPlan p = plan_jacobi2d(n, Ti, Tj, f64);
+    const int cv = cv_resolve(carveout, 0);
     dim3 grid((unsigned)p.gx, (unsigned)p.gy), block(p.bx, p.by);
     if (p.gy > 65535) return cudaErrorInvalidConfiguration;
 #define JL(T, V, C)                                                                               \
     do {                                                                                          \
-        cudaFuncSetAttribute(jacobi2d_sweep<T, V, C>, cudaFuncAttributePreferredSharedMemoryCarveout, \
-                             carveout);                                                           \
-        jacobi2d_sweep<T, V, C><<<grid, block, 0, s>>>((T *)dst, (const T *)src, (const T *)bsrc, n, \
-                                                       (int)Ti, (int)Tj, counts);                 \
+        launch_cv(jacobi2d_sweep<T, V, C>, grid, block, cv, s, (T *)dst, (const T *)src,          \
+                  (const T *)bsrc, n, (int)Ti, (int)Tj, counts);                                  \
     } while (0)
     if (counts) {
         if (f64) JL(double, 1, true);
@@ -330,13 +347,12 @@ cudaError_t launch_heat3d_sweep(void *dst, const void *src, int64_t n, int64_t T
     StencilPlan p = plan_heat3d(n, Ti, Tj, Tk, f64);
     if (p.gy > 65535) return cudaErrorInvalidConfiguration;
     const int nbj = (int)cdiv(n - 1, Tj);
+    const int cv = cv_resolve(carveout, 0);
     dim3 grid((unsigned)p.gx, (unsigned)p.gy), block(p.bx, 1);
 #define HL(T, V, C)                                                                              \
     do {                                                                                         \
-        cudaFuncSetAttribute(heat3d_sweep<T, V, C>, cudaFuncAttributePreferredSharedMemoryCarveout, \
-                             carveout);                                                          \
-        heat3d_sweep<T, V, C><<<grid, block, 0, s>>>((T *)dst, (const T *)src, n, (int)Ti, (int)Tj, \
-                                                     (int)Tk, nbj, counts);                      \
+        launch_cv(heat3d_sweep<T, V, C>, grid, block, cv, s, (T *)dst, (const T *)src, n, (int)Ti,  \
+                  (int)Tj, (int)Tk, nbj, counts);                                                \
     } while (0)
     if (counts) {
         if (f64) HL(double, 1, true);

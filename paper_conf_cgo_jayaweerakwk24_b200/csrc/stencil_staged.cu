@@ -18,6 +18,8 @@
 #include <cstdint>
 #include <cstdlib>
 
+#include "contract.cuh"
+
 #include "tc_ptx.cuh"
 
 namespace eatss {
@@ -248,7 +250,8 @@ constexpr int kSmemTarget = 113 * 1024;  // at least two resident CTAs per SM
 // launch with programmatic stream serialization allowed (the kernel calls pdl_trigger / pdl_wait);
 // EATSS_STENCIL_PDL=0 launches normally (for comparison)
 template <typename... KArgs, typename... Args>
-cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, int smem, cudaStream_t s, Args... args) {
+cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, int smem, int carveout, cudaStream_t s,
+                       Args... args) {
     static const bool on = [] {
         const char *e = getenv("EATSS_STENCIL_PDL");
         return !(e && atoi(e) == 0);
@@ -258,11 +261,16 @@ cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, int smem, 
     cfg.blockDim = block;
     cfg.dynamicSmemBytes = (size_t)smem;
     cfg.stream = s;
-    cudaLaunchAttribute at[1];
+    cudaLaunchAttribute at[2];
     at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
     at[0].val.programmaticStreamSerializationAllowed = on ? 1 : 0;
+    // the carve-out travels with the launch (and with a captured graph node), so a replayed time
+    // loop keeps the carve-out it was captured with
+    at[1].id = cudaLaunchAttributePreferredSharedMemoryCarveout;
+    at[1].val.sharedMemCarveout = (unsigned)carveout;
     cfg.attrs = at;
-    cfg.numAttrs = 1;
+    cfg.numAttrs = 2;
+    note_carveout(carveout);
     return cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
 }
 
@@ -273,14 +281,14 @@ int jacobi_staged_smem(int64_t n, int64_t Ti, int64_t Tj) {
 int heat_staged_smem(int64_t Ti, int64_t Tj, int64_t Tk) { return (int)((Ti + 2) * (Tj + 2) * (Tk + 8) * 4) + 128; }
 
 // carve-out (percent of the maximum shared memory) that keeps `ctas` CTAs of `smem` bytes resident,
-// never below the model's split (sigma) preference
-int staged_carveout(int smem, int split_pct) {
+// never below the model's split (sigma) preference -- or sigma itself under exec.carveout_exact
+int staged_carveout(int smem, int cv) {
     int dev = 0, maxsm = 228 * 1024;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&maxsm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev);
     const int ctas = std::max(1, std::min(4, (maxsm - 1024) / (smem + 1024 + 16)));
     const int need = (int)(((int64_t)ctas * (smem + 1024 + 16) * 100 + maxsm - 1) / maxsm);
-    return std::min(100, std::max(split_pct, need));
+    return cv_resolve(cv, std::min(100, need));
 }
 
 }  // namespace
@@ -304,10 +312,8 @@ cudaError_t launch_jacobi2d_staged(float *dst, const float *src, const float *bs
         return cudaGetLastError();
     }
     cudaFuncSetAttribute(jacobi2d_staged<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    cudaFuncSetAttribute(jacobi2d_staged<false>, cudaFuncAttributePreferredSharedMemoryCarveout,
-                         staged_carveout(smem, split_pct));
-    return launch_pdl(jacobi2d_staged<false>, grid, block, smem, s, dst, src, bsrc, n, (int)Ti, (int)Tj,
-                      (int32_t *)nullptr);
+    return launch_pdl(jacobi2d_staged<false>, grid, block, smem, staged_carveout(smem, split_pct), s, dst, src, bsrc,
+                      n, (int)Ti, (int)Tj, (int32_t *)nullptr);
 }
 
 cudaError_t launch_heat3d_staged(float *dst, const float *src, int64_t n, int64_t Ti, int64_t Tj, int64_t Tk,
@@ -330,10 +336,8 @@ cudaError_t launch_heat3d_staged(float *dst, const float *src, int64_t n, int64_
         return cudaErrorInvalidValue;
     const int smem = heat_staged_smem(Ti, Tj, Tk);
     cudaFuncSetAttribute(heat3d_staged<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    cudaFuncSetAttribute(heat3d_staged<false>, cudaFuncAttributePreferredSharedMemoryCarveout,
-                         staged_carveout(smem, split_pct));
-    return launch_pdl(heat3d_staged<false>, grid, block, smem, s, dst, (const CUtensorMap)m, n, (int)Ti, (int)Tj,
-                      (int)Tk, (int)nbj, (int32_t *)nullptr);
+    return launch_pdl(heat3d_staged<false>, grid, block, smem, staged_carveout(smem, split_pct), s, dst,
+                      (const CUtensorMap)m, n, (int)Ti, (int)Tj, (int)Tk, (int)nbj, (int32_t *)nullptr);
 }
 
 }  // namespace eatss

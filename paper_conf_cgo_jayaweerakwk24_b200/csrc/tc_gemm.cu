@@ -28,6 +28,7 @@
 #include <cstdlib>
 
 #include "contract.cuh"
+#include "devsw.hpp"
 
 namespace eatss {
 
@@ -366,7 +367,7 @@ static inline uint32_t pow2_cols(uint32_t c) {
 
 static int tc_stages() {
     int S = 4;
-    if (const char *e = getenv("EATSS_TC_STAGES")) S = std::max(2, atoi(e));
+    if (devsw("EATSS_TC_STAGES", 0) > 0) S = std::max(2, devsw("EATSS_TC_STAGES", 0));
     return S;
 }
 
@@ -408,9 +409,9 @@ cudaError_t launch_tc_contraction(const ContractNest &n, const ContractPlan &p, 
     a.bjp = (int)(((p.Tj + 3) / 4) * 4);
     a.tmem_cols = (uint32_t)tcols;
     a.a_bulk = 0;
-    if (const char *e = getenv("EATSS_TC_ABULK")) a.a_bulk = atoi(e);
+    a.a_bulk = devsw("EATSS_TC_ABULK", 0);
     a.R = 16;  // stages per accumulator chunk (128 k): drift ~128 * 2^-24 per chunk
-    if (const char *e = getenv("EATSS_TC_CHUNK")) a.R = std::max(2, atoi(e));
+    if (devsw("EATSS_TC_CHUNK", 0) > 0) a.R = std::max(2, devsw("EATSS_TC_CHUNK", 0));
     void (*k)(const tc::Args) = nullptr;
     switch (a.NM) {
         case 16: k = tc::tc3_gemm_kernel<16>; break;

@@ -420,33 +420,6 @@ struct Prep {
     int nb0 = 0, nb1 = 0, mode = 1;
 };
 
-// Workspace for the split operands (library-owned, grown on demand, per device).
-namespace {
-std::mutex g_ws_mu;
-float *g_ws = nullptr;
-size_t g_ws_elems = 0;
-int g_ws_dev = -1;
-}  // namespace
-
-static float *workspace(size_t elems) {
-    std::lock_guard<std::mutex> lk(g_ws_mu);
-    int dev = 0;
-    cudaGetDevice(&dev);
-    if (g_ws && (g_ws_elems < elems || g_ws_dev != dev)) {
-        cudaFree(g_ws);
-        g_ws = nullptr;
-    }
-    if (!g_ws) {
-        if (cudaMalloc(&g_ws, elems * 4) != cudaSuccess) {
-            g_ws = nullptr;
-            return nullptr;
-        }
-        g_ws_elems = elems;
-        g_ws_dev = dev;
-    }
-    return g_ws;
-}
-
 // CTA pairs whenever each CTA's half of the B tile is whole swizzle atoms (EATSS_TCM_PAIR=0 disables)
 static int tcm_cg(const ContractNest &n, int bn) {
     static const int env = getenv("EATSS_TCM_PAIR") ? atoi(getenv("EATSS_TCM_PAIR")) : 1;
@@ -455,8 +428,8 @@ static int tcm_cg(const ContractNest &n, int bn) {
 }
 static int tcm_stage_bytes(int bn, int cg) { return 2 * tcm::BM * tcm::BK * 4 + 2 * tcm::BK * (bn / cg) * 4; }
 static int tcm_stages(int bn, int cg) {
-    int S = (int)((232448 - 2048) / tcm_stage_bytes(bn, cg));
-    if (const char *e = getenv("EATSS_TCM_STAGES")) S = atoi(e);
+    static const int env = getenv("EATSS_TCM_STAGES") ? atoi(getenv("EATSS_TCM_STAGES")) : 0;  // development
+    const int S = env > 0 ? env : (int)((232448 - 2048) / tcm_stage_bytes(bn, cg));
     return std::max(2, std::min(S, 8));
 }
 
@@ -476,8 +449,8 @@ static void schedule(tcm::Args &a, int ncl) {
     const int rem = a.T % ncl;
     a.sp = 1;
     a.nfull = a.T;
-    const char *ev = getenv("EATSS_TCM_SPLITK");
-    if (rem > 0 && !(ev && atoi(ev) == 0)) {
+    static const bool splitk = !(getenv("EATSS_TCM_SPLITK") && atoi(getenv("EATSS_TCM_SPLITK")) == 0);
+    if (rem > 0 && splitk) {
         const int sp = std::min(std::min(4, ncl / rem), a.nkb);
         if (sp >= 2) {
             a.sp = sp;
@@ -505,17 +478,6 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
     auto k = tcm::tc_mma_kernel<BN, TB, CG>;
     int dev = 0;
     cudaGetDevice(&dev);
-    KernelState *ks;
-    {
-        std::lock_guard<std::mutex> lk(g_ks_mu);
-        ks = &g_ks[{reinterpret_cast<const void *>(k), dev}];
-    }
-    cudaError_t e;
-    const bool fresh = ks->smem < smem;
-    if (fresh) {
-        if ((e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
-        ks->smem = smem;
-    }
     int ncl = nsm / CG;
     cudaLaunchConfig_t cfg = {};
     cudaLaunchAttribute attr[1];
@@ -528,22 +490,30 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
     cfg.stream = s;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    if (CG == 2) {
-        if (fresh || ks->active <= 0) {
+    cudaError_t e;
+    {  // attribute and occupancy state of (kernel, device): checked and set under the lock
+        std::lock_guard<std::mutex> lk(g_ks_mu);
+        KernelState &ks = g_ks[{reinterpret_cast<const void *>(k), dev}];
+        const bool fresh = ks.smem < smem;
+        if (fresh) {
+            if ((e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
+            ks.smem = smem;
+        }
+        if (CG == 2 && (fresh || ks.active <= 0)) {
             cfg.gridDim = dim3((unsigned)(2 * ncl));
             int active = 0;
             if (cudaOccupancyMaxActiveClusters(&active, k, &cfg) != cudaSuccess) active = 0;
             cudaGetLastError();
-            ks->active = active;
+            ks.active = active;
         }
-        if (ks->active > 0) ncl = std::min(ncl, ks->active);
+        if (CG == 2 && ks.active > 0) ncl = std::min(ncl, ks.active);
     }
     schedule(a, ncl);
     ncl = std::max(1, std::min(ncl, a.T));
     {  // operand splits + tail prepass: one launch
         const int rows = CG * tcm::BM;
         const int64_t tail4 = needs_prepass(a) ? (int64_t)(a.T - a.nfull) * rows * ((BN + 3) / 4) : 0;
-        const int npb = (int)std::min<int64_t>((tail4 + 255) / 256, 148 * 4);
+        const int npb = (int)std::min<int64_t>((tail4 + 255) / 256, (int64_t)nsm * 4);
         const int vecC = (a.ldc % 4 == 0 && (reinterpret_cast<uintptr_t>(a.C) & 15) == 0) ? 1 : 0;
         tcm::prep_kernel<<<pr.nb0 + pr.nb1 + npb, 256, 0, s>>>(pr.j0, pr.j1, pr.nb0, pr.nb1, pr.mode, a, rows, BN, vecC);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
@@ -603,22 +573,41 @@ tcm::SplitJob split_job(Operand &o, float *ws) {  // the split is run by the fus
 }
 }  // namespace
 
-cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p, cudaStream_t s, cudaEvent_t *ev) {
+// The split operands of one GEMM (workspace sizing shared by tcm_ws_floats and the launcher).
+struct Operands {
+    Operand oa, ob;
+    bool share = false;  // syrk: A is a row block of B (both row-major over k): B's split serves A
+};
+static Operands operands(const ContractNest &n, int mode) {
+    const float *A = static_cast<const float *>(n.A), *B = static_cast<const float *>(n.B);
+    Operands o{Operand{A, n.M, n.K, n.lda}, Operand{B, n.transB ? n.N : n.K, n.transB ? n.K : n.N, n.ldb}};
+    size_operand(o.oa, mode);
+    size_operand(o.ob, mode);
+    o.share = n.transB && n.lda == n.ldb && A >= B && (A - B) % n.ldb == 0 && (A - B) / n.ldb + n.M <= o.ob.rows;
+    return o;
+}
+
+size_t tcm_ws_floats(const ContractNest &n, const ContractPlan &) {
+    const Operands o = operands(n, split_mode());
+    return (size_t)(o.ob.need + (o.share ? 0 : o.oa.need) + 64);
+}
+
+cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p, float *ws, size_t ws_floats,
+                                   cudaStream_t s, cudaEvent_t *ev) {
     if (!tcm_applicable(n, p)) return cudaErrorNotSupported;
     const int bn = (int)p.Tj, cg = tcm_cg(n, bn), mode = split_mode();
     const float *A = static_cast<const float *>(n.A), *B = static_cast<const float *>(n.B);
-    Operand oa{A, n.M, n.K, n.lda}, ob{B, n.transB ? n.N : n.K, n.transB ? n.K : n.N, n.ldb};
-    size_operand(oa, mode);
-    size_operand(ob, mode);
-    // syrk: A is a row block of B (both row-major over k) -> split B once and point into it
-    const bool share = n.transB && n.lda == n.ldb && A >= B && (A - B) % n.ldb == 0 &&
-                       (A - B) / n.ldb + n.M <= ob.rows;
-    float *ws = workspace((size_t)(ob.need + (share ? 0 : oa.need) + 64));
-    if (!ws) return cudaErrorMemoryAllocation;
+    Operands ops = operands(n, mode);
+    Operand &oa = ops.oa, &ob = ops.ob;
+    const bool share = ops.share;
+    if (!ws || ws_floats < (size_t)(ob.need + (share ? 0 : oa.need) + 64)) return cudaErrorInvalidValue;
     Prep pr;
     pr.mode = mode;
     pr.j0 = split_job(ob, ws);
-    constexpr int kSplitBlocks = 148 * 8;  // grid-stride split blocks over both operands
+    int dev = 0, nsm = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    const int kSplitBlocks = nsm * 8;  // grid-stride split blocks over both operands
     if (share) {
         const int64_t r = (A - B) / n.ldb;
         oa.hi = ob.hi + r * ob.ldp;
@@ -648,15 +637,12 @@ cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p,
     a.C = static_cast<float *>(n.C); a.ldc = n.ldc;
     a.alpha = (float)n.alpha; a.beta = (float)n.beta; a.init_zero = n.init_zero ? 1 : 0;
     a.S = tcm_stages(bn, cg);
-    a.R = 16;  // 16 k-blocks = 512 k per accumulator chunk
-    if (const char *ev = getenv("EATSS_TCM_CHUNK")) a.R = std::max(1, atoi(ev));
+    static const int chunk_env = getenv("EATSS_TCM_CHUNK") ? atoi(getenv("EATSS_TCM_CHUNK")) : 0;  // development
+    a.R = chunk_env > 0 ? chunk_env : 16;  // 16 k-blocks = 512 k per accumulator chunk
     a.nkb = (int)((n.K + tcm::BK - 1) / tcm::BK);
     a.PI = (int)((n.M + cg * tcm::BM - 1) / (cg * tcm::BM));
     a.TJ = (int)((n.N + bn - 1) / bn);
     const int smem = a.S * tcm_stage_bytes(bn, cg) + 1024 /*align*/ + 8 * (2 * a.S + 4) + 16;
-    int dev = 0, nsm = 148;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     if (n.transB)
         return cg == 2 ? launch_bn<true, 2>(bn, m, a, smem, nsm, pr, s, ev) : launch_bn<true, 1>(bn, m, a, smem, nsm, pr, s, ev);
     return cg == 2 ? launch_bn<false, 2>(bn, m, a, smem, nsm, pr, s, ev) : launch_bn<false, 1>(bn, m, a, smem, nsm, pr, s, ev);

@@ -30,7 +30,7 @@ def test_library_exports_every_declared_symbol():
 
 
 def test_abi_version():
-    assert E.abi_version() == 1
+    assert E.abi_version() == 2
 
 
 def _gpu(name):
@@ -236,3 +236,42 @@ def test_syrk_simt_layout_pass_counted():
     (ps,) = E.plan(d, (16, 1024, 16))
     (pg,) = E.plan(g, (16, 1024, 16))
     assert (ps.block_x, ps.block_y, ps.rm, ps.rn, ps.vec) == (pg.block_x, pg.block_y, pg.rm, pg.rn, pg.vec)
+
+
+# ------------------------------------------------------------------ warp alignment in the executor
+@pytest.mark.parametrize("waf", [4, 8, 16, 32])
+@pytest.mark.parametrize("tiles", [(16, 1024, 16), (32, 512, 48), (64, 64, 64), (4, 4, 4), (7, 13, 5),
+                                   (1024, 1024, 16)])
+def test_contraction_plan_honours_warp_alignment(waf, tiles):
+    """exec.warp_align = WAF lays WAF lanes of every warp along l_s1 = j: the plan reports
+    simt_x == WAF, the thread grid is whole warps of WAF x 32/WAF slots, and the tile is still
+    covered (passes x micro-tile >= tile)."""
+    d = E.desc_builtin("gemm", (4000, 4000, 4000))
+    d.set_exec(split_pct=50, engine=1, warp_align=waf)
+    (p,) = E.plan(d, tiles)
+    assert p.simt_x == waf
+    assert p.block_x % waf == 0 and p.block_y % (32 // waf) == 0
+    assert (p.block_x * p.block_y) % 32 == 0 and p.block_x * p.block_y <= 1024
+    Ti, Tj = min(tiles[0], 4000), min(tiles[1], 4000)
+    cover_i, cover_j = p.block_y * p.rm, p.block_x * p.rn
+    assert p.passes == (-(-Ti // cover_i)) * (-(-Tj // cover_j))
+
+
+def test_default_layout_simt_x():
+    d = E.desc_builtin("gemm", (4000, 4000, 4000))
+    (p,) = E.plan(d, (16, 1024, 16))
+    assert p.block_x % 32 == 0 and p.simt_x == 32
+    (q,) = E.plan(d, (32, 32, 32))  # 8 lanes along j, rows below
+    assert q.simt_x == q.block_x < 32
+
+
+def test_exec_opts_validation():
+    d = E.desc_builtin("gemm", (64, 64, 64))
+    for bad in (3, 12, 64, -4):
+        with pytest.raises(E.EatssError) as e:
+            d.set_exec(warp_align=bad)
+        assert e.value.status == _abi.EATSS_E_INVALID
+    with pytest.raises(E.EatssError):
+        d.set_exec(carveout_exact=2)
+    d.set_exec(split_pct=0, warp_align=8, carveout_exact=1)
+    assert E.last_carveout(d) == []  # no run yet
