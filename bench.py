@@ -481,7 +481,7 @@ def main():
             tf32 = bf16 * TF32_OVER_BF16
             roof = {"bound": "tensor", "achieved": achieved, "peak": tf32 / 3, "unit": "TFLOP/s",
                     "frac": achieved / (tf32 / 3), "traffic": traffic,
-                    "kernel": f"tc_mma_kernel<{tiles[1]}> (tcgen05 GEMM alone; the prep launch (operand "
+                    "kernel": f"tc_mma_kernel<{tiles[2]},false,{tiles[0] // 128}> (tile {tuple(tiles)}: tcgen05 GEMM alone; the prep launch (operand "
                               f"splits + split-k tail pre-pass) is outside this window but inside every timed step)",
                     "call_frac": FLOPS / (call_avg_ms * 1e-3) / 1e12 / (tf32 / 3),
                     "peak_source": (f"measured bf16 {bf16:.1f} TF (MEASURED_PEAKS.json, burst) x nominal "

@@ -4,9 +4,11 @@ on the tensor pipe?
 
     python harness/tensor_sweep.py [--kinds gemm,2mm,syrk] [--repeats 5] [--window 1.0] [--out ts.jsonl]
 
-The tcgen05 3xTF32 executor accepts the MMA-legal tiles of reading T: Ti = 128
-(UMMA M; CTA pairs cover 256 rows), Tj in {32, 64, ..., 256} (UMMA N), Tk = one 32-float TMA atom.
-Every legal vector of gemm / 2mm / syrk at N = 4000 is measured with the a9 protocol (eatss_sweep:
+The tcgen05 3xTF32 executor accepts the tiles Ti in {128 (one CTA), 256 (a CTA pair)}, Tj in
+{16, 32, ..., 256} (UMMA N), Tk in {8, 16, 32, 64} (k per pipeline stage) that fit its shared memory;
+reading T is the subset with Tk in {32, 64} (whole 128-byte swizzle atoms).
+Every executable vector of gemm (2mm / syrk: the reading-T subset) at N = 4000 is measured with the
+a9 protocol (eatss_sweep:
 warm-up, >= --window s of back-to-back runs, NVML energy counter) in --repeats interleaved
 rounds, so DVFS and thermal drift hit every variant alike; each variant is first checked for
 exactness on small-integer inputs (sampled entries vs the fp64 oracle).  The summary gives per
@@ -32,7 +34,7 @@ KINDS = {"gemm": (N, N, N), "2mm": (N, N, N, N), "syrk": (N, N)}
 
 def parse():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--kinds", default="gemm,2mm,syrk")
+    ap.add_argument("--kinds", default="gemm")
     ap.add_argument("--repeats", type=int, default=5)
     ap.add_argument("--window", type=float, default=1.0)
     ap.add_argument("--warmup", type=int, default=3)
@@ -73,7 +75,10 @@ def main():
             d = E.desc_builtin(kind, dims)
             d.set_exec(split_pct=50, engine=2)
             pick, _ = E.select_tiles(d, gpu, split_pct=50, waf=16, mode=2)
-            variants = [(128, tj, 32) for tj in range(32, 257, 32)]
+            space = [(ti, tj, tk) for ti in (128, 256) for tj in range(16, 257, 16) for tk in (8, 16, 32, 64)]
+            if kind != "gemm":
+                space = [v for v in space if v[2] >= 32]
+            variants = [v for v in space if E.launches_per_run(d, v) == 2]  # executable on tcgen05
             gen = torch.Generator(device="cuda").manual_seed(0)
             bufs = [torch.rand(d.buffer_elems(i), device="cuda", generator=gen) * 2 - 1 for i in range(d.num_buffers)]
             exact = {v: exact_gemm(E, torch, v) for v in variants} if kind == "gemm" else {}
@@ -87,7 +92,7 @@ def main():
                     rec = dict(kind=kind, tiles=list(v), rep=rep, ms=m.ms_per_run, tflops=m.tflops,
                                watts=m.avg_watts, ppw=m.gflops_per_watt, joules=m.joules_per_run,
                                sm_mhz=m.sm_mhz_median, status=m.status, eatss_pick=tuple(v) == tuple(pick),
-                               exact=exact.get(v))
+                               reading_t=v[2] >= 32, exact=exact.get(v))
                     f.write(json.dumps(rec) + "\n"); f.flush()
                     if m.status == 0 and m.gflops_per_watt > 0:
                         ppw[v].append(m.gflops_per_watt); tf[v].append(m.tflops); watts[v].append(m.avg_watts)
@@ -101,7 +106,7 @@ def main():
                     if ppw[v]}
             perf = max(rows, key=lambda v: rows[v]["tflops"][0])
             eff = max(rows, key=lambda v: rows[v]["ppw"][0])
-            s = dict(eatss_pick=list(pick), perf_optimal=dict(tiles=list(perf), **rows[perf]),
+            s = dict(eatss_pick=list(pick), n_variants=len(rows), perf_optimal=dict(tiles=list(perf), **rows[perf]),
                      ppw_optimal=dict(tiles=list(eff), **rows[eff]),
                      distinct=perf != eff,
                      separated=perf != eff and rows[eff]["ppw"][1][0] > rows[perf]["ppw"][1][1],

@@ -141,6 +141,43 @@ class Opts:
     mode: int = 1  # 0 = paper mode, 1 = B200 mode (SMEM clamp)
 
 
+@dataclass(frozen=True)
+class Reading:
+    """Alternative readings of the ambiguous model text.
+
+    Reading R (every default) is the library's; each field names the passage it reads and its
+    alternatives, so tests can show which alternatives the paper's own numbers exclude (P:121,
+    P:153) and the harness can measure what the rest would pick.
+      h_count   Q6  "number of times each loop iterator appears in the stride-1 dimension":
+                'group' (distinct cache-line groups, R), 'array' (arrays), 'ref' (deduped references)
+      nrefs     Q10 "references accessing distinct cache lines": 'group' (R), 'array', 'ref'
+      rule2d    Q7  2-D sub-case: 'R' (parallel loops 0, the serial loop unscaled),
+                'none' (no 2-D rule: the >=3-D rule applies), 'scaled' (as R, the serial loop x WAF)
+      waf_scale Q7  CMA scaling: 'waf' (R; "2 x 16") or 'warp' (T_P_W = 32)
+      footprint Q11 data tile of a reference: 'nohalo' (R: product of T over its iterators)
+                or 'halo' (per array dimension sum of T over its iterators - (n-1) + offset span)
+      bset      Q12 "up to the first three outer parallel loop dimensions":
+                'ls1_outer' (R: l_s1, then outermost others), 'outer' (the three outermost),
+                'ls1_inner' (l_s1, then innermost others)
+      split     Q4  sigma = 0 / 1: 'R' (0: one combined L1; 1: L1 bound by L2/#SM)
+                or 'literal' (the printed inequalities at every sigma)
+      units     Q2  KB / MB: 'KiB' (R) or 'KB' (powers of 1000)
+      tiebreak  Q16 Z3's arbitrary optimum: 'R' (rule 13), 'lexmin', 'lexmax'
+    """
+    h_count: str = "group"
+    nrefs: str = "group"
+    rule2d: str = "R"
+    waf_scale: str = "waf"
+    footprint: str = "nohalo"
+    bset: str = "ls1_outer"
+    split: str = "R"
+    units: str = "KiB"
+    tiebreak: str = "R"
+
+
+R = Reading()
+
+
 # ------------------------------------------------------------- derivation
 
 
@@ -158,9 +195,12 @@ class Derived:
     all_fp: List[frozenset]
     bset: List[str]
     H: Dict[str, int]
+    # per footprint (parallel to l1_fp / sh_fp): array dimensions as (iterator names, offset span)
+    l1_dims: List[tuple] = field(default_factory=list)
+    sh_dims: List[tuple] = field(default_factory=list)
 
 
-def derive(nest: Nest, waf: int) -> Derived:
+def derive(nest: Nest, waf: int, rd: Reading = R) -> Derived:
     loops = nest.loops
     depth = len(loops)
     # rule 1: dedupe
@@ -173,9 +213,16 @@ def derive(nest: Nest, waf: int) -> Derived:
     groups = set()
     for r in refs:
         groups.add((r.array, r.subs[:-1], r.last_iters()))
-    nrefs = len(groups)
-    # rule 3: counts over groups
-    cnt = {l.name: sum(1 for g in groups if l.name in g[2]) for l in loops}
+    arrays = {r.array for r in refs}
+    nrefs = {"group": len(groups), "array": len(arrays), "ref": len(refs)}[rd.nrefs]
+    # rule 3: counts (Q6: over groups, arrays or references)
+    if rd.h_count == "group":
+        cnt = {l.name: sum(1 for g in groups if l.name in g[2]) for l in loops}
+    elif rd.h_count == "array":
+        cnt = {l.name: sum(1 for a in arrays if any(r.array == a and l.name in r.last_iters() for r in refs))
+               for l in loops}
+    else:
+        cnt = {l.name: sum(1 for r in refs if l.name in r.last_iters()) for l in loops}
     # rule 4: CMA loop
     cands = [(cnt[l.name], d, l.name) for d, l in enumerate(loops) if l.parallel and cnt[l.name] > 0]
     if not cands:
@@ -186,31 +233,52 @@ def derive(nest: Nest, waf: int) -> Derived:
     sh_refs = [r for r in refs if ls1 not in r.last_iters()]
 
     def fps(rs):
-        out = []
+        out, dims = [], []
         for r in rs:
             f = (r.array, r.iters())
+            per_dim = [(its, off, off) for its, off in r.subs]
             if f not in out:
                 out.append(f)
-        return out
+                dims.append(per_dim)
+            else:  # widen the offset range of each dimension (halo reading, Q11)
+                k = out.index(f)
+                dims[k] = [(its, min(lo, off), max(hi, off)) for (its, lo, hi), (_, off) in zip(dims[k], r.subs)]
+        return out, [tuple((its, hi - lo) for its, lo, hi in dd) for dd in dims]
 
-    l1_fp = fps(l1_refs)
-    sh_fp = [f for f in fps(sh_refs) if f not in l1_fp]
+    l1_fp, l1_dims = fps(l1_refs)
+    sh_all, sh_dims_all = fps(sh_refs)
+    keep = [k for k, f in enumerate(sh_all) if f not in l1_fp]
+    sh_fp = [sh_all[k] for k in keep]
+    sh_dims = [sh_dims_all[k] for k in keep]
     all_fp = l1_fp + sh_fp
-    # rule 7: B-set
+    # rule 7: B-set (Q12)
     par = [l.name for l in loops if l.parallel]
-    bset = ([ls1] if ls1 in par else []) + [p for p in par if p != ls1]
-    bset = bset[:3]
-    # rule 8: weights
+    if rd.bset == "outer":
+        bset = par[:3]
+    elif rd.bset == "ls1_inner":
+        bset = ([ls1] if ls1 in par else []) + [p for p in reversed(par) if p != ls1]
+        bset = bset[:3]
+    else:
+        bset = ([ls1] if ls1 in par else []) + [p for p in par if p != ls1]
+        bset = bset[:3]
+    # rule 8: weights (Q7)
+    scale = waf if rd.waf_scale == "waf" else 32
     H = {}
     for l in loops:
-        h = cnt[l.name] * (waf if l.name == ls1 else 1)
+        h = cnt[l.name] * (scale if l.name == ls1 else 1)
         if depth >= 3 and not l.parallel:
             h = 0
-        if depth == 2 and l.parallel:
+        if depth == 2 and rd.rule2d != "none":
+            if l.parallel:
+                h = 0
+            elif rd.rule2d == "scaled":
+                h = cnt[l.name] * scale
+        if depth == 2 and rd.rule2d == "none" and not l.parallel:
             h = 0
         H[l.name] = h
     return Derived(loops, refs, nrefs, cnt, ls1, l1_refs, sh_refs,
-                   [f[1] for f in l1_fp], [f[1] for f in sh_fp], [f[1] for f in all_fp], bset, H)
+                   [f[1] for f in l1_fp], [f[1] for f in sh_fp], [f[1] for f in all_fp], bset, H,
+                   l1_dims, sh_dims)
 
 
 def table2(nest: Nest, waf: int = 16):
@@ -229,27 +297,34 @@ def table2(nest: Nest, waf: int = 16):
 # ------------------------------------------------------------- capacities
 
 
-def caps(gpu: Gpu, opts: Opts, e: int):
+def caps(gpu: Gpu, opts: Opts, e: int, rd: Reading = R):
     """Element-unit capacities (rule 12). Returns dict with possibly-None entries."""
     pct = opts.split_pct
+    L1_SH, L2 = gpu.L1_SH, gpu.L2
+    if rd.units == "KB":  # Q2: the printed KB / MB as powers of 1000
+        L1_SH, L2 = L1_SH // 1024 * 1000, L2 // (1024 * 1024) * 1000 * 1000
     c = {}
-    if pct == 0:
-        c["all_l1"] = (gpu.L1_SH) // e  # L1 u SH footprints share the whole L1
+    if rd.split == "literal":
+        c["all_l1"] = None
+        c["l1"] = ((100 - pct) * L1_SH) // (100 * e)
+        c["sh"] = (pct * L1_SH) // (100 * e)
+    elif pct == 0:
+        c["all_l1"] = (L1_SH) // e  # L1 u SH footprints share the whole L1
         c["l1"] = None
         c["sh"] = None
     elif pct == 100:
         c["all_l1"] = None
-        c["l1"] = gpu.L2 // (gpu.n_SM * e)
-        c["sh"] = gpu.L1_SH // e
+        c["l1"] = L2 // (gpu.n_SM * e)
+        c["sh"] = L1_SH // e
     else:
         c["all_l1"] = None
-        c["l1"] = ((100 - pct) * gpu.L1_SH) // (100 * e)
-        c["sh"] = (pct * gpu.L1_SH) // (100 * e)
-    c["l2"] = gpu.L2 // e
+        c["l1"] = ((100 - pct) * L1_SH) // (100 * e)
+        c["sh"] = (pct * L1_SH) // (100 * e)
+    c["l2"] = L2 // e
     if opts.mode == 1:
         clamp = gpu.max_smem_per_block // e
         c["sh"] = clamp if c["sh"] is None else min(c["sh"], clamp)
-        if pct == 0:
+        if pct == 0 and rd.split != "literal":
             c["sh"] = None  # SH set lives in L1 when no shared memory is carved out
     return c
 
@@ -281,24 +356,38 @@ def _prod(T, names, pos):
     return v
 
 
-def evaluate(prog: Program, gpu: Gpu, opts: Opts, T: Sequence[np.ndarray]):
+def _volume(T, pos, f, dims, rd: Reading):
+    """V^f: reading R -- product of T over the reference's iterators; halo reading (Q11) --
+    per array dimension the extent sum(T) - (n - 1) + offset span."""
+    if rd.footprint == "nohalo":
+        return _prod(T, f, pos)
+    v = np.ones_like(T[0])
+    for its, span in dims:
+        if not its:
+            continue
+        ext = sum(T[pos[n]] for n in its) - (len(its) - 1) + span
+        v = v * ext
+    return v
+
+
+def evaluate(prog: Program, gpu: Gpu, opts: Opts, T: Sequence[np.ndarray], rd: Reading = R):
     """Vectorised rules 6-12 over arrays of tile values T[p] (one array per position).
 
     Returns (feasible bool array, OBJ int64 array)."""
     e = prog.dtype_bytes
     fpf = 1 if e == 4 else 2
-    c = caps(gpu, opts, e)
+    c = caps(gpu, opts, e, rd)
     feas = np.ones(T[0].shape, dtype=bool)
     obj = np.zeros(T[0].shape, dtype=np.int64)
     for nest in prog.nests:
-        d = derive(nest, opts.waf)
+        d = derive(nest, opts.waf, rd)
         pos = {l.name: p for p, l in enumerate(nest.loops)}
         Bn = _prod(T, d.bset, pos)
         # rule 11
         feas &= Bn * d.nrefs * fpf <= gpu.R_P_S
         # rule 12
-        ml1 = sum((_prod(T, f, pos) for f in d.l1_fp), np.zeros_like(Bn))
-        msh = sum((_prod(T, f, pos) for f in d.sh_fp), np.zeros_like(Bn))
+        ml1 = sum((_volume(T, pos, f, dd, rd) for f, dd in zip(d.l1_fp, d.l1_dims)), np.zeros_like(Bn))
+        msh = sum((_volume(T, pos, f, dd, rd) for f, dd in zip(d.sh_fp, d.sh_dims)), np.zeros_like(Bn))
         mall = ml1 + msh
         if c["all_l1"] is not None:
             feas &= mall <= c["all_l1"]
@@ -315,14 +404,14 @@ def evaluate(prog: Program, gpu: Gpu, opts: Opts, T: Sequence[np.ndarray]):
     return feas, obj
 
 
-def objective_free_positions(prog: Program, waf: int) -> List[int]:
+def objective_free_positions(prog: Program, waf: int, rd: Reading = R) -> List[int]:
     free = []
     for p in range(prog.L):
         ok = True
         for nest in prog.nests:
             if p >= len(nest.loops):
                 continue
-            d = derive(nest, waf)
+            d = derive(nest, waf, rd)
             name = nest.loops[p].name
             if d.H[name] != 0 or name in d.bset:
                 ok = False
@@ -345,12 +434,19 @@ def extents(prog: Program) -> List[int]:
 # over MMA-legal tiles of the tcgen05 executor, with the register / L1 / SH capacities
 # replaced by the resources that executor actually uses:
 #   T1  applies to nests of depth 3 with one serial (reduction) loop and l_s1 parallel;
-#   T2  domain: l_s1 (UMMA N) in {32, 64, ..., min(256, roundup32(N))}; the other B-set loop
-#       (UMMA M) in {128}; the serial loop (one 128-byte TMA atom of fp32) in {32};
-#   T3  TMEM: two fp32 accumulator buffers of T_{l_s1} columns, 2*T_{l_s1} <= 512;
-#       SMEM: 2 stages x {hi, lo} x e x (sum of the input footprints) <= max_smem_per_block.
+#   T2  domain: l_s1 (UMMA N) in {16, 32, ..., min(256, roundup16(N))}; the other B-set loop
+#       (UMMA M rows: one CTA or a CTA pair) in {128, 256}; the serial loop (k per pipeline stage,
+#       whole 128-byte swizzle atoms of fp32) in {32, 64};
+#   T3  per nest, CG = T_M / 128 CTAs per tile:
+#       legality: T_{l_s1} / CG a multiple of 16 (UMMA N per CTA half);
+#       TMEM: two fp32 accumulator buffers of T_{l_s1} columns, 2*T_{l_s1} <= 512;
+#       SMEM: 2 stages x {hi, lo} x e x (sum of the per-CTA input footprints) <= max_smem_per_block
+#       - 2048, a footprint taken per CTA (T_M -> 128, T_{l_s1} -> T_{l_s1} / CG) and, for an
+#       operand whose last subscript is l_s1 (MN-major on the tensor core), its l_s1 extent
+#       rounded up to the 32-column swizzle atom.
 
 TMEM_COLS = 512
+SMEM_RESERVE = 2048  # barriers + 1024-byte alignment of the stage ring
 
 
 def tensor_applicable(prog: Program) -> bool:
@@ -370,12 +466,12 @@ def tensor_domains(prog: Program):
     ex = extents(prog)
     for p, l in enumerate(n0.loops):
         if l.name == d.ls1:
-            hi = min(256, -(-ex[p] // 32) * 32)
-            doms.append(list(range(32, hi + 1, 32)))
+            hi = min(256, -(-ex[p] // 16) * 16)
+            doms.append(list(range(16, hi + 1, 16)))
         elif l.parallel:
-            doms.append([128])
+            doms.append([128, 256])
         else:
-            doms.append([32])
+            doms.append([32, 64])
     return doms
 
 
@@ -386,39 +482,53 @@ def evaluate_tensor(prog: Program, gpu: Gpu, opts: Opts, T):
     for nest in prog.nests:
         d = derive(nest, opts.waf)
         pos = {l.name: p for p, l in enumerate(nest.loops)}
+        rows = [l.name for l in nest.loops if l.parallel and l.name != d.ls1][0]  # UMMA M loop
+        cg = T[pos[rows]] // 128
+        n_cta = T[pos[d.ls1]] // cg
+        feas &= (T[pos[d.ls1]] % cg == 0) & (n_cta % 16 == 0)                     # T3 legality
+        feas &= 2 * T[pos[d.ls1]] <= TMEM_COLS                                      # T3 TMEM
         written = {r.array for r in nest.refs if r.write}
         inputs = []
         for r in d.refs:
             f = (r.array, r.iters())
-            if r.array not in written and f not in inputs:
-                inputs.append(f)
-        feas &= 2 * T[pos[d.ls1]] <= TMEM_COLS                                  # T3 TMEM
-        vin = sum((_prod(T, f[1], pos) for f in inputs), np.zeros_like(T[0]))
-        feas &= 2 * 2 * e * vin <= gpu.max_smem_per_block                      # T3 SMEM
-        obj = obj + _prod(T, d.bset, pos)                                       # Eq. 2
+            if r.array not in written and f not in [x[:2] for x in inputs]:
+                inputs.append((r.array, r.iters(), d.ls1 in r.last_iters()))
+        vin = np.zeros_like(T[0])
+        for _, its, mn_major in inputs:
+            v = np.ones_like(T[0])
+            for it in its:
+                if it == rows:
+                    v = v * 128
+                elif it == d.ls1:
+                    v = v * (-(-n_cta // 32) * 32 if mn_major else n_cta)
+                else:
+                    v = v * T[pos[it]]
+            vin = vin + v
+        feas &= 2 * 2 * e * vin <= gpu.max_smem_per_block - SMEM_RESERVE           # T3 SMEM
+        obj = obj + _prod(T, d.bset, pos)                                           # Eq. 2
         for l in nest.loops:
             if d.H[l.name]:
                 obj = obj + d.H[l.name] * T[pos[l.name]]
     return feas, obj
 
 
-def select_tiles(prog: Program, gpu: Gpu, opts: Opts, keep_ties: bool = True) -> Result:
-    """Exhaustive maximisation of OBJ over the whole domain (no pruning)."""
+def select_tiles(prog: Program, gpu: Gpu, opts: Opts, keep_ties: bool = True, rd: Reading = R) -> Result:
+    """Exhaustive maximisation of OBJ over the whole domain (no pruning); `rd` selects the reading."""
     L = prog.L
     tensor = opts.mode == 2
     if tensor and not tensor_applicable(prog):
         return Result(None, 0, 0, 0, [])
     doms = ([np.array(v, dtype=np.int64) for v in tensor_domains(prog)] if tensor else
             [np.array(domain(n, gpu, opts.waf), dtype=np.int64) for n in extents(prog)])
-    free = objective_free_positions(prog, opts.waf)
-    ls1_pos = [l.name for l in prog.nests[0].loops].index(derive(prog.nests[0], opts.waf).ls1)
+    free = objective_free_positions(prog, opts.waf, rd)
+    ls1_pos = [l.name for l in prog.nests[0].loops].index(derive(prog.nests[0], opts.waf, rd).ls1)
     best_key, best, ties, n_feas = None, None, [], 0
     # iterate the first position in Python, the rest as one numpy meshgrid block
     rest = np.meshgrid(*doms[1:], indexing="ij") if L > 1 else []
     rest = [r.ravel() for r in rest]
     for t0 in doms[0]:
         T = [np.full(rest[0].shape if rest else (1,), t0, dtype=np.int64)] + rest
-        feas, obj = (evaluate_tensor if tensor else evaluate)(prog, gpu, opts, T)
+        feas, obj = evaluate_tensor(prog, gpu, opts, T) if tensor else evaluate(prog, gpu, opts, T, rd)
         n_feas += int(feas.sum())
         if not feas.any():
             continue
@@ -440,7 +550,12 @@ def select_tiles(prog: Program, gpu: Gpu, opts: Opts, keep_ties: bool = True) ->
     def key(t):
         return (sum(t[p] for p in free), -t[ls1_pos], t)
 
-    ties.sort(key=key)
+    if rd.tiebreak == "lexmin":
+        ties.sort()
+    elif rd.tiebreak == "lexmax":
+        ties.sort(reverse=True)
+    else:
+        ties.sort(key=key)
     return Result(ties[0], best, n_feas, len(ties), ties if keep_ties else [])
 
 

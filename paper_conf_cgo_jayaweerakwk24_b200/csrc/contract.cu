@@ -484,6 +484,7 @@ inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
 ContractPlan plan_contraction(const ContractNest &n, const int64_t *tiles, int smem_limit, int waf_req) {
     ContractPlan p;
+    p.rTi = tiles[0]; p.rTj = tiles[1]; p.rTk = tiles[2];
     p.Ti = std::max<int64_t>(1, std::min(tiles[0], n.M));
     p.Tj = std::max<int64_t>(1, std::min(tiles[1], n.N));
     p.Tk = std::max<int64_t>(1, std::min(tiles[2], n.K));

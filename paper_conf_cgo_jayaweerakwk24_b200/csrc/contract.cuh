@@ -37,6 +37,7 @@ struct ContractNest {
 
 struct ContractPlan {
     int64_t Ti = 0, Tj = 0, Tk = 0;  // clipped tile
+    int64_t rTi = 0, rTj = 0, rTk = 0;  // tile as requested (the tensor engine's MMA-legal shape)
     int rm = 1, rn = 1, vec = 1;
     int bx = 1, by = 1;
     int passes_i = 1, passes_j = 1;
@@ -58,7 +59,8 @@ int plan_simt_x(const ContractPlan &p);
 // tensor-core (tcgen05, 3xTF32) executor: applicability / launch (tc_gemm.cu)
 bool tc_plan(const ContractNest &n, const ContractPlan &p, int *smem_bytes, int *tmem_cols);
 cudaError_t launch_tc_contraction(const ContractNest &n, const ContractPlan &p, int carveout, cudaStream_t s);
-// tcgen05 3xTF32 GEMM for MMA-legal tiles (Ti = 128, Tj in 32..256 step 32) (tc_mma.cu)
+// tcgen05 3xTF32 GEMM for MMA-legal tiles (tc_mma.cu): Ti in {128, 256} (one CTA / a CTA pair),
+// Tj in 16..256 step 16, Tk in {8, 16, 32, 64}
 bool tcm_applicable(const ContractNest &n, const ContractPlan &p);
 // Split-operand workspace (floats) one launch needs: owned by the caller's descriptor, so
 // concurrent descriptors (streams, devices, host threads) never share it.

@@ -149,11 +149,14 @@ struct NestEval {
     const Nest *nest;
     NestModel m;
     std::vector<uint32_t> in_fp;  // tensor mode: footprints of the arrays the nest only reads
+    std::vector<char> in_mn;      // ... whose last subscript uses l_s1 (MN-major tensor-core operand)
+    int rows_pos = -1;            // tensor mode: the parallel loop that is not l_s1 (UMMA M)
 };
 
 // Tensor-core mode (reading T): the executor stages every input footprint in
 // shared memory (2 stages x {hi, lo}) and keeps two fp32 accumulators of T_{l_s1} TMEM columns.
-std::vector<uint32_t> input_footprints(const Nest &n) {
+void input_footprints(NestEval &ne) {
+    const Nest &n = *ne.nest;
     std::vector<int> written;
     for (const Ref &r : n.refs)
         if (r.write) written.push_back(r.array);
@@ -163,11 +166,16 @@ std::vector<uint32_t> input_footprints(const Nest &n) {
         uint32_t it = 0;
         for (const Sub &s : r.subs) it |= s.iters;
         std::pair<int, uint32_t> f{r.array, it};
-        if (std::find(seen.begin(), seen.end(), f) == seen.end()) seen.push_back(f);
+        if (std::find(seen.begin(), seen.end(), f) != seen.end()) continue;
+        seen.push_back(f);
+        ne.in_fp.push_back(it);
+        ne.in_mn.push_back((r.subs.back().iters >> ne.m.ls1) & 1u ? 1 : 0);
     }
-    std::vector<uint32_t> out;
-    for (auto &f : seen) out.push_back(f.second);
-    return out;
+    for (int p = 0; p < (int)n.loops.size(); p++)
+        if (n.loops[p].parallel && p != ne.m.ls1) {
+            ne.rows_pos = p;
+            break;
+        }
 }
 constexpr int64_t kTmemCols = 512;
 
@@ -197,12 +205,24 @@ struct Search {
     int esz = 4;
 
     bool feasible(const std::vector<int64_t> &T) const {
-        if (tensor) {
+        if (tensor) {  // reading T3
             for (const NestEval &ne : nests) {
-                if (2 * T[ne.m.ls1] > kTmemCols) return false;  // two fp32 accumulator buffers
+                const int64_t tn = T[ne.m.ls1], cg = T[ne.rows_pos] / 128;
+                if (cg < 1 || tn % cg || (tn / cg) % 16) return false;  // UMMA N per CTA half
+                if (2 * tn > kTmemCols) return false;                   // two fp32 accumulator buffers
+                const int64_t n_cta = tn / cg;
                 int64_t vin = 0;
-                for (uint32_t f : ne.in_fp) vin += prod(T, f);
-                if (2 * 2 * esz * vin > smem_cap) return false;  // 2 stages x {hi, lo}
+                for (size_t f = 0; f < ne.in_fp.size(); f++) {
+                    int64_t v = 1;
+                    for (int p = 0; p < L; p++) {
+                        if (!((ne.in_fp[f] >> p) & 1u)) continue;
+                        if (p == ne.rows_pos) v *= 128;  // per-CTA rows
+                        else if (p == ne.m.ls1) v *= ne.in_mn[f] ? (n_cta + 31) / 32 * 32 : n_cta;
+                        else v *= T[p];
+                    }
+                    vin += v;
+                }
+                if (2 * 2 * esz * vin > smem_cap - 2048) return false;  // 2 stages x {hi, lo}
             }
             return true;
         }
@@ -265,6 +285,14 @@ struct Search {
         }
         for (int64_t v : dom[p]) {
             T[p] = v;
+            if (tensor) {  // reading T's legality is not monotone: enumerate the (small) space whole
+                if (p + 1 == L) {
+                    if (feasible(T)) leaf();
+                } else {
+                    dfs(p + 1);
+                }
+                continue;
+            }
             // positions > p sit at their minimum; monotone constraints => break
             if (!feasible(T)) break;
             dfs(p + 1);
@@ -297,7 +325,13 @@ extern "C" eatss_status eatss_select_tiles(const eatss_kernel_desc *d, const eat
     s.fpf = (e == 8) ? 2 : 1;  // FP_factor
     s.regs = g->regs_per_sm;
     s.caps = capacities(*g, *o, e);
-    for (const Nest &n : d->nests) s.nests.push_back({&n, derive_nest(n, o->warp_align), input_footprints(n)});
+    for (const Nest &n : d->nests) {
+        NestEval ne;
+        ne.nest = &n;
+        ne.m = derive_nest(n, o->warp_align);
+        input_footprints(ne);
+        s.nests.push_back(ne);
+    }
     if (o->mode == 2) {
         // tensor-core mode: depth-3 nests with one serial loop and a parallel l_s1 only
         for (const NestEval &ne : s.nests) {
@@ -312,13 +346,13 @@ extern "C" eatss_status eatss_select_tiles(const eatss_kernel_desc *d, const eat
         const Nest &n0 = d->nests[0];
         for (int p = 0; p < s.L; p++) {
             std::vector<int64_t> dm;
-            if (p == s.nests[0].m.ls1) {  // UMMA N: 32-multiples up to 256 (TMA boxes of 32 columns)
-                const int64_t hi = std::min<int64_t>(256, ((ext[p] + 31) / 32) * 32);
-                for (int64_t v = 32; v <= hi; v += 32) dm.push_back(v);
+            if (p == s.nests[0].m.ls1) {  // UMMA N: multiples of 16 up to 256
+                const int64_t hi = std::min<int64_t>(256, ((ext[p] + 15) / 16) * 16);
+                for (int64_t v = 16; v <= hi; v += 16) dm.push_back(v);
             } else if (n0.loops[p].parallel) {
-                dm.push_back(128);  // UMMA M (cta_group::1)
+                dm = {128, 256};  // UMMA M rows: one CTA (cta_group::1) or a CTA pair (cta_group::2)
             } else {
-                dm.push_back(32);  // one 128-byte TMA atom of the reduction loop
+                dm = {32, 64};  // k per stage: whole 128-byte swizzle atoms of fp32
             }
             s.dom.push_back(dm);
         }

@@ -1,31 +1,36 @@
-// tc_mma.cu -- tcgen05 3xTF32 GEMM for MMA-legal tiles (the
-// "tensor-core EATSS mode", DESIGN.md §2.5 / §4.1c): Ti = 128 rows of i per CTA (UMMA M per
-// SM), Tj <= 256 columns of j (UMMA N), k in blocks of 32 (one 128-byte swizzle atom of fp32).
+// tc_mma.cu -- tcgen05 3xTF32 GEMM for MMA-legal tiles (the "tensor-core
+// EATSS mode", DESIGN.md §2.5 / §4.1c).  The tile vector (Ti, Tj, Tk) is honoured as written:
+//   Ti in {128, 256}  rows of i per cluster tile: 128 = one CTA (UMMA M = 128, cta_group::1),
+//                     256 = a CTA pair (cta_group::2, cluster of 2 along i: M = 256, each CTA keeps
+//                     its own 128 x Tj accumulator but stages only half of the B tile);
+//   Tj in 16..256, multiple of 16: UMMA N (columns of j per tile);
+//   Tk in {8, 16, 32, 64}: k per pipeline stage (one TMA box per operand and stage; 8 / 16 k are
+//                     one 32 / 64-byte swizzle row, 32 one 128-byte atom, 64 two atoms).
 //
-// Same loop-nest semantics as the SIMT executor (Fig. 4: each CTA owns one Ti x Tj
+// Same loop-nest semantics as the SIMT executor (Fig. 4: each cluster owns one Ti x Tj
 // tile of C, k sequential); fp32-accurate via 3xTF32 (reading Q26):
 //   C = beta*C + alpha * sum_k (Ahi*Bhi + Ahi*Blo + Alo*Bhi),
-//   hi = rna_tf32(x), lo = rna_tf32(x - hi), computed once per operand by prep_kernel.
+//   hi = the fp32 operand itself (the tensor core reads its tf32 bits), lo = rna_tf32(x - rz_tf32(x))
+//   materialised once per operand by prep_kernel.
+// The tensor core's own fp32 accumulation truncates, so the accumulator is drained into fp32
+// registers every CHUNK_K = 128 k (two TMEM buffers alternate; a drain overlaps the next chunk's
+// MMAs): 1.2e-6 normwise at N = 4000 (16 chunks of 512 k: 4.0e-6; one chunk: 2.8e-5;
+// profiles/r02/chunk_ab*.jsonl) -- chained products (3mm) need the fp32-level error.
 //
 // B200-specific structure (what differs from the paper's one-tile-per-block CUDA code):
-//  * CTA pairs (cta_group::2, cluster of 2 along i): the pair issues M = 256 MMAs; each CTA
-//    keeps its own 128 x Tj accumulator tile but stages only HALF of the B tile, so shared
-//    memory traffic per SM drops from 12 KB to 8 KB per MMA (the single-CTA kernel was
-//    shared-memory-bandwidth bound at ~74% tensor-pipe activity).  Used when Tj/2 is a whole
-//    number of 32-column swizzle atoms (or B is K-major); otherwise one CTA per tile.
-//  * persistent clusters over a grouped (L2-friendly) tile order; the accumulator is drained
-//    chunk by chunk (two TMEM buffers), so one tile's epilogue overlaps the next tile's MMAs.
+//  * persistent clusters over a grouped (L2-friendly) tile order; one CTA per SM;
 //  * wave-quantisation tail: when the last wave would leave clusters idle, the remaining tiles
 //    are split along k into `sp` parts whose partial sums are added to C with fp32 atomics
 //    (C pre-scaled by beta once by prep_kernel).
-// Pipeline (warp-specialised, mbarrier hand-off, one CTA per SM):
-//   warp 0  TMA producer: Ahi/Alo (K-major, 128 x 32, SWIZZLE_128B) and Bhi/Blo (MN-major
-//           32 x Tj/CG in 32-column SWIZZLE_128B_ATOM_32B boxes, or K-major Tj/CG x 32 when B
-//           is transposed, as in syrk) into an S-stage ring;
+// Pipeline (warp-specialised, mbarrier hand-off):
+//   warp 0  TMA producer: Ahi/Alo (K-major, 128 x Tk, swizzled) and Bhi/Blo (MN-major boxes of
+//           32 columns x Tk rows, SWIZZLE_128B_ATOM_32B -- UMMA SWIZZLE_128B_BASE32B -- or K-major
+//           Tj/CG x Tk when B is transposed, as in syrk) into an S-stage ring;
 //   warp 1  MMA issuer (leader CTA only): per 8-k step three kind::tf32 MMAs;
 //           tcgen05.commit (multicast to the pair) frees ring slots / publishes chunks;
 //   warp 2  TMEM allocation (512 columns = two accumulator buffers of up to 256);
-//   warps 4..11 epilogue: tcgen05.ld of each finished chunk into fp32 registers, then C.
+//   warps 4..19 epilogue: tcgen05.ld of each finished chunk into fp32 registers, then C (16 warps:
+//           a drain of Tj/4 columns per warp keeps short chunks cheap).
 #include <cuda.h>
 #include <cuda_runtime.h>
 
@@ -37,17 +42,17 @@
 #include <string>
 
 #include "contract.cuh"
+#include "devsw.hpp"
 #include "tc_ptx.cuh"
 
 namespace eatss {
 namespace tcm {
 
-
-constexpr int BK = 32;   // k per stage (128-byte swizzle atom of fp32)
-constexpr int BM = 128;  // rows of i per CTA (UMMA M per SM)
-constexpr int NEPI = 8;  // epilogue warps (4..11): two per TMEM lane quarter
+constexpr int BM = 128;      // rows of i per CTA (UMMA M per SM)
+constexpr int NEPI = 16;     // epilogue warps (4..19): four per TMEM lane quarter, a column quarter each
 constexpr int NTHREADS = (4 + NEPI) * 32;
-constexpr int GROUP_ROWS = 8;  // tile-order grouping (pair-rows per group) for L2 reuse
+constexpr int MAXBN = 256;   // UMMA N limit
+constexpr int CHUNK_K = 128; // k per accumulator chunk (fp32 drain of the truncating accumulation)
 
 struct Args {
     int64_t M, N, K;
@@ -55,21 +60,28 @@ struct Args {
     int64_t ldc;
     float alpha, beta;
     int init_zero;
-    int S;   // ring stages
-    int R;   // k-blocks per accumulator chunk
+    int S;        // ring stages
+    int R;        // k-blocks per accumulator chunk
+    int BNT;      // Tj: UMMA N of the cluster tile (multiple of 16, <= 256)
+    int BNH;      // B columns (rows, if K-major) staged by one CTA: BNT / CG
+    int bgroups;  // MN-major B: 32-column swizzle atoms per CTA and stage
+    int b_bytes;  // bytes of one B half (hi or lo) per CTA and stage
+    int stage;    // bytes per stage (per CTA)
+    uint32_t idesc;
     // persistent schedule
     int PI, TJ;   // row groups (of CG*128 rows) x column tiles
     int T;        // PI * TJ tiles
     int nfull;    // tiles done whole by one cluster
     int sp;       // k-parts per tail tile (1 = no split)
     int nunits;   // nfull + (T - nfull) * sp
-    int nkb;      // k-blocks of 32
+    int nkb;      // k-blocks of Tk
+    int group_rows;  // tile-order grouping (row groups per group) for L2 reuse
 };
 
-__host__ __device__ inline void tile_coords(int t, int PI, int TJ, int &pi, int &tj) {
-    const int g = t / (GROUP_ROWS * TJ), r = t % (GROUP_ROWS * TJ);
-    const int rows = PI - g * GROUP_ROWS < GROUP_ROWS ? PI - g * GROUP_ROWS : GROUP_ROWS;
-    pi = g * GROUP_ROWS + r % rows;
+__host__ __device__ inline void tile_coords(int t, int PI, int TJ, int G, int &pi, int &tj) {
+    const int g = t / (G * TJ), r = t % (G * TJ);
+    const int rows = PI - g * G < G ? PI - g * G : G;
+    pi = g * G + r % rows;
     tj = r / rows;
 }
 
@@ -92,23 +104,35 @@ __device__ __forceinline__ Unit unit_of(const Args &p, int u) {
         w.kb1 = (int)((int64_t)(part + 1) * p.nkb / p.sp);
         w.split = p.sp > 1;
     }
-    tile_coords(t, p.PI, p.TJ, w.pi, w.tj);
+    tile_coords(t, p.PI, p.TJ, p.group_rows, w.pi, w.tj);
     return w;
 }
 
-template <int BNT, bool TB, int CG>
+// K-major operand (rows x Tk of fp32, TMA box inner = min(Tk, 32) elements): swizzle span in bytes,
+// UMMA layout type, and the descriptor of 8-k step ks (atoms of 32 k are rows*128 bytes apart)
+template <int BK>
+struct KMajor {
+    static constexpr int SW = BK >= 32 ? 128 : BK * 4;                    // bytes per swizzled row
+    static constexpr uint32_t LAYOUT = SW == 128 ? 2u : SW == 64 ? 4u : 6u;  // SW128 / SW64 / SW32
+    static constexpr int NA = BK > 32 ? BK / 32 : 1;                      // 128-byte atoms along k
+    __device__ static uint64_t desc(const unsigned char *base, int rows, int ks) {
+        const unsigned char *p = base + (ks / 4) * rows * 128 + (ks % 4) * 32;
+        return desc_sw128(p, 16u, (uint32_t)(8 * SW), LAYOUT);
+    }
+};
+
+template <int BK, bool TB, int CG>
 __global__ void __launch_bounds__(NTHREADS, 1)
     tc_mma_kernel(const __grid_constant__ CUtensorMap mAhi, const __grid_constant__ CUtensorMap mAlo,
                   const __grid_constant__ CUtensorMap mBhi, const __grid_constant__ CUtensorMap mBlo, const Args p) {
     extern __shared__ __align__(1024) unsigned char smem_raw[];
     unsigned char *smem = smem_raw + ((1024u - (su32(smem_raw) & 1023u)) & 1023u);  // stays a shared pointer
+    using KA = KMajor<BK>;
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const uint32_t rank = CG == 2 ? cta_rank() : 0u;
     const int cid = (int)blockIdx.x / CG, ncl = (int)gridDim.x / CG;
-    constexpr int BNH = BNT / CG;                // B columns (rows, if TB) staged by this CTA
-    constexpr int A_BYTES = BM * BK * 4;         // 16 KB
-    constexpr int B_BYTES = BK * BNH * 4;        // <= 32 KB
-    constexpr int STAGE = 2 * A_BYTES + 2 * B_BYTES;
+    constexpr int A_BYTES = BM * BK * 4;  // one A half (hi or lo) per stage
+    const int BNH = p.BNH, B_BYTES = p.b_bytes, STAGE = p.stage;
     const int R = p.R;
     uint64_t *full = reinterpret_cast<uint64_t *>(smem + (size_t)p.S * STAGE);
     uint64_t *empty = full + p.S;
@@ -154,7 +178,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             for (int u = cid; u < p.nunits; u += ncl) {
                 const Unit w = unit_of(p, u);
                 const int i0 = (w.pi * CG + (int)rank) * BM;
-                const int jb = w.tj * BNT + (int)rank * BNH;
+                const int jb = w.tj * p.BNT + (int)rank * BNH;
                 for (int kb = w.kb0; kb < w.kb1; kb++, it++) {
                     const int s = it % p.S;
                     if (it >= p.S) mbar_wait(empty + s, (unsigned)(((it / p.S) - 1) & 1));
@@ -162,16 +186,22 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                     if (rank == 0) mbar_expect_tx(full + s, CG * STAGE);
                     const uint32_t fb = fbar0 + 8u * (uint32_t)s;
                     const int k0 = kb * BK;
-                    tma_2d<CG>(st, &mAhi, k0, i0, fb);
-                    tma_2d<CG>(st + A_BYTES, &mAlo, k0, i0, fb);
-                    if constexpr (TB) {
-                        tma_2d<CG>(st + 2 * A_BYTES, &mBhi, k0, jb, fb);
-                        tma_2d<CG>(st + 2 * A_BYTES + B_BYTES, &mBlo, k0, jb, fb);
-                    } else {
 #pragma unroll
-                        for (int g = 0; g < BNH / 32; g++) {
-                            tma_2d<CG>(st + 2 * A_BYTES + g * (BK * 128), &mBhi, jb + 32 * g, k0, fb);
-                            tma_2d<CG>(st + 2 * A_BYTES + B_BYTES + g * (BK * 128), &mBlo, jb + 32 * g, k0, fb);
+                    for (int a = 0; a < KA::NA; a++) {
+                        tma_2d<CG>(st + a * BM * 128, &mAhi, k0 + 32 * a, i0, fb);
+                        tma_2d<CG>(st + A_BYTES + a * BM * 128, &mAlo, k0 + 32 * a, i0, fb);
+                    }
+                    unsigned char *sb = st + 2 * A_BYTES;
+                    if constexpr (TB) {
+#pragma unroll
+                        for (int a = 0; a < KA::NA; a++) {
+                            tma_2d<CG>(sb + a * BNH * 128, &mBhi, k0 + 32 * a, jb, fb);
+                            tma_2d<CG>(sb + B_BYTES + a * BNH * 128, &mBlo, k0 + 32 * a, jb, fb);
+                        }
+                    } else {
+                        for (int g = 0; g < p.bgroups; g++) {
+                            tma_2d<CG>(sb + g * (BK * 128), &mBhi, jb + 32 * g, k0, fb);
+                            tma_2d<CG>(sb + B_BYTES + g * (BK * 128), &mBlo, jb + 32 * g, k0, fb);
                         }
                     }
                 }
@@ -179,10 +209,9 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         }
     } else if (warp == 1) {
         if (lane == 0 && rank == 0) {  // -------------------------------- MMA issuer (leader)
-            constexpr uint32_t ID = idesc(BNT, CG, TB);
-            // A (and K-major B): SW128 K-major, SBO = 8 rows x 128 B, +32 B per 8-k step.
-            // MN-major B: SW128_BASE32B, LBO = stride of 32-column groups (BK rows x 128 B),
-            // SBO = stride of the 4-row swizzle atoms (512 B), +1 KB per 8-k step.
+            const uint32_t ID = p.idesc;
+            // K-major operands: swizzled rows (SBO = 8 rows), atoms of 32 k; MN-major B: SW128_BASE32B,
+            // LBO = stride of 32-column groups (Tk rows x 128 B), SBO = 512 B, +1 KB per 8-k step.
             int it = 0, gc = 0;
             for (int u = cid; u < p.nunits; u += ncl) {
                 const Unit w = unit_of(p, u);
@@ -193,19 +222,20 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                     if (first && gc >= 2) mbar_wait_cluster(dempty + bd, (unsigned)(((gc - 2) >> 1) & 1));
                     mbar_wait(full + s, (unsigned)((it / p.S) & 1));
                     fence_after();
-                    unsigned char *st = smem + (size_t)s * STAGE;
+                    const unsigned char *st = smem + (size_t)s * STAGE;
+                    const unsigned char *sb = st + 2 * A_BYTES;
                     const uint32_t d = tmem + (uint32_t)(bd * 256);
 #pragma unroll
                     for (int ks = 0; ks < BK / 8; ks++) {
-                        const uint64_t ahi = desc_sw128(st + ks * 32, 16u, 1024u);
-                        const uint64_t alo = desc_sw128(st + A_BYTES + ks * 32, 16u, 1024u);
+                        const uint64_t ahi = KA::desc(st, BM, ks);
+                        const uint64_t alo = KA::desc(st + A_BYTES, BM, ks);
                         uint64_t bhi, blo;
                         if constexpr (TB) {
-                            bhi = desc_sw128(st + 2 * A_BYTES + ks * 32, 16u, 1024u);
-                            blo = desc_sw128(st + 2 * A_BYTES + B_BYTES + ks * 32, 16u, 1024u);
+                            bhi = KA::desc(sb, BNH, ks);
+                            blo = KA::desc(sb + B_BYTES, BNH, ks);
                         } else {
-                            bhi = desc_sw128(st + 2 * A_BYTES + ks * 1024, (uint32_t)(BK * 128), 512u, 1);
-                            blo = desc_sw128(st + 2 * A_BYTES + B_BYTES + ks * 1024, (uint32_t)(BK * 128), 512u, 1);
+                            bhi = desc_sw128(sb + ks * 1024, (uint32_t)(BK * 128), 512u, 1);
+                            blo = desc_sw128(sb + B_BYTES + ks * 1024, (uint32_t)(BK * 128), 512u, 1);
                         }
                         mma_ss<CG>(d, ahi, bhi, ID, (first && ks == 0) ? 0u : 1u);
                         mma_ss<CG>(d, ahi, blo, ID, 1u);
@@ -220,27 +250,38 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             }
         }
     } else if (warp >= 4) {  // ---------------------------------------- epilogue warps
-        const int e = warp - 4, q = warp & 3, half = e >> 2;
-        constexpr int CW = BNT / 2;  // columns per epilogue warp
+        const int e = warp - 4, q = warp & 3, cq = e >> 2;  // TMEM lane quarter, column quarter
+        const int CW = p.BNT / 4;  // columns per epilogue warp (multiple of 4)
+        constexpr int MAXCW = MAXBN / 4;
         const uint32_t demp0 = CG == 2 ? mapa(su32(dempty), 0) : su32(dempty);
         int gc = 0;
         for (int u = cid; u < p.nunits; u += ncl) {
             const Unit w = unit_of(p, u);
             const int nch = (w.kb1 - w.kb0 + R - 1) / R;
-            float acc[CW];
+            float acc[MAXCW];
 #pragma unroll
-            for (int c = 0; c < CW; c++) acc[c] = 0.f;
+            for (int c = 0; c < MAXCW; c++) acc[c] = 0.f;
             for (int ch = 0; ch < nch; ch++, gc++) {
                 const int bd = gc & 1;
                 mbar_wait(dfull + bd, (unsigned)((gc >> 1) & 1));
                 fence_after();
+                const uint32_t ta = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(bd * 256 + cq * CW);
+                // drain: four 4-column loads in flight per wait
 #pragma unroll
-                for (int c0 = 0; c0 < CW; c0 += 16) {
-                    uint32_t v[16];
-                    tmem_ld16(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(bd * 256 + half * CW + c0), v);
-                    wait_ld();
+                for (int c0 = 0; c0 < MAXCW; c0 += 16) {
+                    if (c0 < CW) {
+                        uint32_t v[4][4];
 #pragma unroll
-                    for (int c = 0; c < 16; c++) acc[c0 + c] += __uint_as_float(v[c]);
+                        for (int g = 0; g < 4; g++)
+                            if (c0 + 4 * g < CW) tmem_ld4(ta + (uint32_t)(c0 + 4 * g), v[g]);
+                        wait_ld();
+#pragma unroll
+                        for (int g = 0; g < 4; g++)
+                            if (c0 + 4 * g < CW) {
+#pragma unroll
+                                for (int c = 0; c < 4; c++) acc[c0 + 4 * g + c] += __uint_as_float(v[g][c]);
+                            }
+                    }
                 }
                 fence_before();
                 __syncwarp();
@@ -251,38 +292,52 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             }
             // C(i, j) for row i = i0 + 32q + lane, columns jb .. jb + CW - 1
             const int64_t i = (int64_t)(w.pi * CG + (int)rank) * BM + q * 32 + lane;
-            const int64_t jb = (int64_t)w.tj * BNT + half * CW;
+            const int64_t jb = (int64_t)w.tj * p.BNT + cq * CW;
             if (i < p.M && jb < p.N) {
                 float *crow = p.C + i * p.ldc + jb;
                 const bool vec = ((p.ldc & 3) == 0) && (jb + CW <= p.N);
                 if (w.split) {  // C already holds beta*C (prep_kernel): add the partial sum
                     if (vec) {
 #pragma unroll
-                        for (int c = 0; c < CW; c += 4)
-                            atomicAdd(reinterpret_cast<float4 *>(crow + c),
-                                      make_float4(p.alpha * acc[c], p.alpha * acc[c + 1], p.alpha * acc[c + 2],
-                                                  p.alpha * acc[c + 3]));
+                        for (int c = 0; c < MAXCW; c += 4)
+                            if (c < CW)
+                                atomicAdd(reinterpret_cast<float4 *>(crow + c),
+                                          make_float4(p.alpha * acc[c], p.alpha * acc[c + 1], p.alpha * acc[c + 2],
+                                                      p.alpha * acc[c + 3]));
                     } else {
 #pragma unroll
-                        for (int c = 0; c < CW; c++)
-                            if (jb + c < p.N) atomicAdd(crow + c, p.alpha * acc[c]);
+                        for (int c = 0; c < MAXCW; c++)
+                            if (c < CW && jb + c < p.N) atomicAdd(crow + c, p.alpha * acc[c]);
                     }
                 } else if (vec) {
+                    // four 16-byte loads of C in flight before their stores
 #pragma unroll
-                    for (int c = 0; c < CW; c += 4) {
-                        float4 *cp = reinterpret_cast<float4 *>(crow + c);
-                        float4 o = p.init_zero ? make_float4(0.f, 0.f, 0.f, 0.f) : *cp;
-                        if (!p.init_zero) { o.x *= p.beta; o.y *= p.beta; o.z *= p.beta; o.w *= p.beta; }
-                        o.x = fmaf(p.alpha, acc[c], o.x);
-                        o.y = fmaf(p.alpha, acc[c + 1], o.y);
-                        o.z = fmaf(p.alpha, acc[c + 2], o.z);
-                        o.w = fmaf(p.alpha, acc[c + 3], o.w);
-                        *cp = o;
+                    for (int c0 = 0; c0 < MAXCW; c0 += 16) {
+                        if (c0 < CW) {
+                            float4 o[4];
+#pragma unroll
+                            for (int g = 0; g < 4; g++)
+                                if (c0 + 4 * g < CW)
+                                    o[g] = p.init_zero ? make_float4(0.f, 0.f, 0.f, 0.f)
+                                                       : *reinterpret_cast<const float4 *>(crow + c0 + 4 * g);
+#pragma unroll
+                            for (int g = 0; g < 4; g++)
+                                if (c0 + 4 * g < CW) {
+                                    const int c = c0 + 4 * g;
+                                    float4 r = o[g];
+                                    if (!p.init_zero) { r.x *= p.beta; r.y *= p.beta; r.z *= p.beta; r.w *= p.beta; }
+                                    r.x = fmaf(p.alpha, acc[c], r.x);
+                                    r.y = fmaf(p.alpha, acc[c + 1], r.y);
+                                    r.z = fmaf(p.alpha, acc[c + 2], r.z);
+                                    r.w = fmaf(p.alpha, acc[c + 3], r.w);
+                                    *reinterpret_cast<float4 *>(crow + c) = r;
+                                }
+                        }
                     }
                 } else {
 #pragma unroll
-                    for (int c = 0; c < CW; c++) {
-                        if (jb + c < p.N) {
+                    for (int c = 0; c < MAXCW; c++) {
+                        if (c < CW && jb + c < p.N) {
                             const float o = p.init_zero ? 0.f : p.beta * crow[c];
                             crow[c] = fmaf(p.alpha, acc[c], o);
                         }
@@ -395,7 +450,7 @@ __global__ void __launch_bounds__(256) prep_kernel(const SplitJob j0, const Spli
         const int x = (int)(e % g4);
         const int t = p.nfull + (int)(rowid / rows_per_tile), r = (int)(rowid % rows_per_tile);
         int pi, tj;
-        tile_coords(t, p.PI, p.TJ, pi, tj);
+        tile_coords(t, p.PI, p.TJ, p.group_rows, pi, tj);
         const int64_t i = (int64_t)pi * rows_per_tile + r, j = (int64_t)tj * bn + 4 * x;
         if (i >= p.M || j >= p.N) continue;
         float *c = p.C + i * p.ldc + j;
@@ -420,25 +475,37 @@ struct Prep {
     int nb0 = 0, nb1 = 0, mode = 1;
 };
 
-// CTA pairs whenever each CTA's half of the B tile is whole swizzle atoms (EATSS_TCM_PAIR=0 disables)
-static int tcm_cg(const ContractNest &n, int bn) {
-    static const int env = getenv("EATSS_TCM_PAIR") ? atoi(getenv("EATSS_TCM_PAIR")) : 1;
-    if (!env) return 1;
-    return n.transB ? ((bn / 2) % 8 == 0 ? 2 : 1) : ((bn / 2) % 32 == 0 ? 2 : 1);
-}
-static int tcm_stage_bytes(int bn, int cg) { return 2 * tcm::BM * tcm::BK * 4 + 2 * tcm::BK * (bn / cg) * 4; }
-static int tcm_stages(int bn, int cg) {
-    static const int env = getenv("EATSS_TCM_STAGES") ? atoi(getenv("EATSS_TCM_STAGES")) : 0;  // development
-    const int S = env > 0 ? env : (int)((232448 - 2048) / tcm_stage_bytes(bn, cg));
-    return std::max(2, std::min(S, 8));
+// Geometry of one tile vector on this engine (shared by applicability, workspace and launch).
+struct TcmGeom {
+    bool ok = false;
+    int bk = 0, bn = 0, cg = 1, bnh = 0, bgroups = 0, a_bytes = 0, b_bytes = 0, stage = 0, S = 0, smem = 0;
+};
+static TcmGeom tcm_geom(const ContractNest &n, const ContractPlan &p) {
+    TcmGeom g;
+    const int64_t Ti = p.rTi, Tj = p.rTj, Tk = p.rTk;
+    if (n.f64 || (Ti != 128 && Ti != 256)) return g;
+    if (Tj < 16 || Tj > tcm::MAXBN || Tj % 16) return g;
+    if (Tk != 8 && Tk != 16 && Tk != 32 && Tk != 64) return g;
+    if (n.M > INT32_MAX / 2 || n.N > INT32_MAX / 2 || n.K > INT32_MAX / 2) return g;
+    g.bk = (int)Tk;
+    g.bn = (int)Tj;
+    g.cg = Ti == 256 ? 2 : 1;           // Ti = 256: a CTA pair (cta_group::2) per tile
+    g.bnh = g.bn / g.cg;
+    if (g.bnh % (n.transB ? 8 : 16)) return g;  // UMMA N per CTA half: K-major rows in 8s, MN-major in 16s
+    g.bgroups = (g.bnh + 31) / 32;
+    g.a_bytes = tcm::BM * g.bk * 4;
+    g.b_bytes = n.transB ? g.bnh * g.bk * 4 : g.bgroups * 32 * g.bk * 4;
+    g.stage = 2 * g.a_bytes + 2 * g.b_bytes;
+    static const int env_s = devsw("EATSS_TCM_STAGES", 0);  // development
+    g.S = std::min(8, (232448 - 2048) / g.stage);
+    if (env_s > 0) g.S = std::min(g.S, env_s);
+    if (g.S < 2) return g;
+    g.smem = g.S * g.stage + 1024 /*align*/ + 8 * (2 * g.S + 4) + 16;
+    g.ok = tcm::encode_fn() != nullptr;
+    return g;
 }
 
-bool tcm_applicable(const ContractNest &n, const ContractPlan &p) {
-    if (n.f64) return false;
-    if (p.Ti != tcm::BM || p.Tj < 32 || p.Tj > 256 || (p.Tj % 32) != 0) return false;
-    if (n.M > INT32_MAX / 2 || n.N > INT32_MAX / 2 || n.K > INT32_MAX / 2) return false;
-    return 2 * tcm_stage_bytes((int)p.Tj, 1) + 2048 <= 232448 && tcm::encode_fn() != nullptr;
-}
+bool tcm_applicable(const ContractNest &n, const ContractPlan &p) { return tcm_geom(n, p).ok; }
 
 // Persistent schedule: full tiles in waves of ncl clusters, the last partial wave split along k
 // into sp parts (so idle clusters take k-slices instead of waiting).  nsm / CG clusters of one
@@ -449,7 +516,7 @@ static void schedule(tcm::Args &a, int ncl) {
     const int rem = a.T % ncl;
     a.sp = 1;
     a.nfull = a.T;
-    static const bool splitk = !(getenv("EATSS_TCM_SPLITK") && atoi(getenv("EATSS_TCM_SPLITK")) == 0);
+    static const bool splitk = devsw("EATSS_TCM_SPLITK", 1) != 0;
     if (rem > 0 && splitk) {
         const int sp = std::min(std::min(4, ncl / rem), a.nkb);
         if (sp >= 2) {
@@ -472,10 +539,10 @@ std::mutex g_ks_mu;
 std::map<std::pair<const void *, int>, KernelState> g_ks;
 }  // namespace
 
-template <int BN, bool TB, int CG>
+template <int BK, bool TB, int CG>
 static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int nsm, const Prep &pr, cudaStream_t s,
                               cudaEvent_t *ev) {
-    auto k = tcm::tc_mma_kernel<BN, TB, CG>;
+    auto k = tcm::tc_mma_kernel<BK, TB, CG>;
     int dev = 0;
     cudaGetDevice(&dev);
     int ncl = nsm / CG;
@@ -512,10 +579,11 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
     ncl = std::max(1, std::min(ncl, a.T));
     {  // operand splits + tail prepass: one launch
         const int rows = CG * tcm::BM;
-        const int64_t tail4 = needs_prepass(a) ? (int64_t)(a.T - a.nfull) * rows * ((BN + 3) / 4) : 0;
+        const int64_t tail4 = needs_prepass(a) ? (int64_t)(a.T - a.nfull) * rows * ((a.BNT + 3) / 4) : 0;
         const int npb = (int)std::min<int64_t>((tail4 + 255) / 256, (int64_t)nsm * 4);
         const int vecC = (a.ldc % 4 == 0 && (reinterpret_cast<uintptr_t>(a.C) & 15) == 0) ? 1 : 0;
-        tcm::prep_kernel<<<pr.nb0 + pr.nb1 + npb, 256, 0, s>>>(pr.j0, pr.j1, pr.nb0, pr.nb1, pr.mode, a, rows, BN, vecC);
+        tcm::prep_kernel<<<pr.nb0 + pr.nb1 + npb, 256, 0, s>>>(pr.j0, pr.j1, pr.nb0, pr.nb1, pr.mode, a, rows, a.BNT,
+                                                               vecC);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
     }
     cfg.gridDim = dim3((unsigned)(CG * ncl));
@@ -526,17 +594,13 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
 }
 
 template <bool TB, int CG>
-static cudaError_t launch_bn(int bn, const CUtensorMap *m, const tcm::Args &a, int smem, int nsm, const Prep &pr,
+static cudaError_t launch_bk(int bk, const CUtensorMap *m, const tcm::Args &a, int smem, int nsm, const Prep &pr,
                              cudaStream_t s, cudaEvent_t *ev) {
-    switch (bn) {
+    switch (bk) {
+        case 8: return launch_one<8, TB, CG>(m, a, smem, nsm, pr, s, ev);
+        case 16: return launch_one<16, TB, CG>(m, a, smem, nsm, pr, s, ev);
         case 32: return launch_one<32, TB, CG>(m, a, smem, nsm, pr, s, ev);
         case 64: return launch_one<64, TB, CG>(m, a, smem, nsm, pr, s, ev);
-        case 96: return launch_one<96, TB, CG>(m, a, smem, nsm, pr, s, ev);
-        case 128: return launch_one<128, TB, CG>(m, a, smem, nsm, pr, s, ev);
-        case 160: return launch_one<160, TB, CG>(m, a, smem, nsm, pr, s, ev);
-        case 192: return launch_one<192, TB, CG>(m, a, smem, nsm, pr, s, ev);
-        case 224: return launch_one<224, TB, CG>(m, a, smem, nsm, pr, s, ev);
-        case 256: return launch_one<256, TB, CG>(m, a, smem, nsm, pr, s, ev);
         default: return cudaErrorNotSupported;
     }
 }
@@ -552,7 +616,7 @@ struct Operand {
 };
 int split_mode() {
     static const int m = [] {
-        const char *e = getenv("EATSS_TCM_SPLIT");
+        const char *e = getenv("EATSS_TCM_SPLIT");  // development: "rna" = hi = rna_tf32(x) materialised too
         return e && std::string(e) == "rna" ? 0 : 1;
     }();
     return m;
@@ -594,8 +658,9 @@ size_t tcm_ws_floats(const ContractNest &n, const ContractPlan &) {
 
 cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p, float *ws, size_t ws_floats,
                                    cudaStream_t s, cudaEvent_t *ev) {
-    if (!tcm_applicable(n, p)) return cudaErrorNotSupported;
-    const int bn = (int)p.Tj, cg = tcm_cg(n, bn), mode = split_mode();
+    const TcmGeom g = tcm_geom(n, p);
+    if (!g.ok) return cudaErrorNotSupported;
+    const int bn = g.bn, cg = g.cg, bk = g.bk, mode = split_mode();
     const float *A = static_cast<const float *>(n.A), *B = static_cast<const float *>(n.B);
     Operands ops = operands(n, mode);
     Operand &oa = ops.oa, &ob = ops.ob;
@@ -622,30 +687,38 @@ cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p,
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
     CUtensorMap m[4];
-    const CUtensorMapSwizzle swK = CU_TENSOR_MAP_SWIZZLE_128B, swMN = CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B;
-    bool ok = tcm::make_map(&m[0], oa.hi, n.M, n.K, oa.ldp, tcm::BK, tcm::BM, swK) &&
-              tcm::make_map(&m[1], oa.lo, n.M, n.K, oa.ldp, tcm::BK, tcm::BM, swK);
-    if (n.transB)  // B(k, j) = B[j*ldb + k]: rows j, K-major boxes of bn/cg rows x 32 k
-        ok = ok && tcm::make_map(&m[2], ob.hi, n.N, n.K, ob.ldp, tcm::BK, bn / cg, swK) &&
-             tcm::make_map(&m[3], ob.lo, n.N, n.K, ob.ldp, tcm::BK, bn / cg, swK);
-    else  // B(k, j) = B[k*ldb + j]: MN-major boxes of 32 k x 32 j
-        ok = ok && tcm::make_map(&m[2], ob.hi, n.K, n.N, ob.ldp, 32, tcm::BK, swMN) &&
-             tcm::make_map(&m[3], ob.lo, n.K, n.N, ob.ldp, 32, tcm::BK, swMN);
+    // K-major boxes: min(Tk, 32) k (one swizzled row: 32 / 64 / 128 bytes) x rows
+    const int kbox = std::min(bk, 32);
+    const CUtensorMapSwizzle swK = kbox == 32   ? CU_TENSOR_MAP_SWIZZLE_128B
+                                   : kbox == 16 ? CU_TENSOR_MAP_SWIZZLE_64B
+                                                : CU_TENSOR_MAP_SWIZZLE_32B;
+    const CUtensorMapSwizzle swMN = CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B;
+    bool ok = tcm::make_map(&m[0], oa.hi, n.M, n.K, oa.ldp, kbox, tcm::BM, swK) &&
+              tcm::make_map(&m[1], oa.lo, n.M, n.K, oa.ldp, kbox, tcm::BM, swK);
+    if (n.transB)  // B(k, j) = B[j*ldb + k]: rows j, K-major boxes of bn/cg rows x kbox k
+        ok = ok && tcm::make_map(&m[2], ob.hi, n.N, n.K, ob.ldp, kbox, g.bnh, swK) &&
+             tcm::make_map(&m[3], ob.lo, n.N, n.K, ob.ldp, kbox, g.bnh, swK);
+    else  // B(k, j) = B[k*ldb + j]: MN-major boxes of Tk k x 32 j
+        ok = ok && tcm::make_map(&m[2], ob.hi, n.K, n.N, ob.ldp, 32, bk, swMN) &&
+             tcm::make_map(&m[3], ob.lo, n.K, n.N, ob.ldp, 32, bk, swMN);
     if (!ok) return cudaErrorInvalidValue;
     tcm::Args a;
     a.M = n.M; a.N = n.N; a.K = n.K;
     a.C = static_cast<float *>(n.C); a.ldc = n.ldc;
     a.alpha = (float)n.alpha; a.beta = (float)n.beta; a.init_zero = n.init_zero ? 1 : 0;
-    a.S = tcm_stages(bn, cg);
-    static const int chunk_env = getenv("EATSS_TCM_CHUNK") ? atoi(getenv("EATSS_TCM_CHUNK")) : 0;  // development
-    a.R = chunk_env > 0 ? chunk_env : 16;  // 16 k-blocks = 512 k per accumulator chunk
-    a.nkb = (int)((n.K + tcm::BK - 1) / tcm::BK);
+    a.S = g.S;
+    static const int chunk_env = devsw("EATSS_TCM_CHUNK_K", 0);  // development: k per accumulator chunk
+    a.R = std::max(1, (chunk_env > 0 ? chunk_env : tcm::CHUNK_K) / bk);
+    a.BNT = bn; a.BNH = g.bnh; a.bgroups = g.bgroups; a.b_bytes = g.b_bytes; a.stage = g.stage;
+    a.idesc = tcm::idesc(bn, cg, n.transB);
+    a.nkb = (int)((n.K + bk - 1) / bk);
     a.PI = (int)((n.M + cg * tcm::BM - 1) / (cg * tcm::BM));
     a.TJ = (int)((n.N + bn - 1) / bn);
-    const int smem = a.S * tcm_stage_bytes(bn, cg) + 1024 /*align*/ + 8 * (2 * a.S + 4) + 16;
+    static const int group_env = devsw("EATSS_TCM_GROUP", 8);  // development: row groups per raster group
+    a.group_rows = std::max(1, group_env);
     if (n.transB)
-        return cg == 2 ? launch_bn<true, 2>(bn, m, a, smem, nsm, pr, s, ev) : launch_bn<true, 1>(bn, m, a, smem, nsm, pr, s, ev);
-    return cg == 2 ? launch_bn<false, 2>(bn, m, a, smem, nsm, pr, s, ev) : launch_bn<false, 1>(bn, m, a, smem, nsm, pr, s, ev);
+        return cg == 2 ? launch_bk<true, 2>(bk, m, a, g.smem, nsm, pr, s, ev) : launch_bk<true, 1>(bk, m, a, g.smem, nsm, pr, s, ev);
+    return cg == 2 ? launch_bk<false, 2>(bk, m, a, g.smem, nsm, pr, s, ev) : launch_bk<false, 1>(bk, m, a, g.smem, nsm, pr, s, ev);
 }
 
 int tcm_launches(const ContractNest &, const ContractPlan &) {

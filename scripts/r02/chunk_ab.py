@@ -1,5 +1,5 @@
 #!/usr/bin/env python
-"""A/B of the tcgen05 GEMM's accumulator chunk (k-blocks of 32 per TMEM drain, EATSS_TCM_CHUNK) at the
+"""A/B of the tcgen05 GEMM's accumulator chunk (k-blocks of 32 per TMEM drain, EATSS_TCM_CHUNK_K) at the
 headline size: device time and precision vs the fp64 oracle (development measurement, not the bench).
 
     python scripts/r02/chunk_ab.py            # runs one subprocess per chunk value
@@ -32,7 +32,7 @@ def one():
     d = E.desc_builtin("gemm", (n, n, n)); d.set_scalars(1.5, 1.2); d.set_exec(50, 2)
     Ad, Bd = torch.from_numpy(A).cuda(), torch.from_numpy(B).cuda()
     Cd = torch.from_numpy(C).cuda()
-    t = (128, 256, 32)
+    t = tuple(int(x) for x in os.environ.get("TILE", "256,256,32").split(","))
     E.run(d, t, [Cd, Ad, Bd]); torch.cuda.synchronize()
     out = Cd.double().cpu().numpy()
     err = O.normwise_rel_err(out, ref)
@@ -46,7 +46,7 @@ def one():
         E.run(d, t, [Cw, Ad, Bd])
     e.record(); torch.cuda.synchronize()
     ms = s.elapsed_time(e) / 50
-    print(json.dumps({"chunk": os.environ.get("EATSS_TCM_CHUNK", "16"), "ms": ms, "tflops": 2 * n ** 3 / ms / 1e9,
+    print(json.dumps({"tiles": t, "chunk_k": os.environ.get("EATSS_TCM_CHUNK_K", "128"), "ms": ms, "tflops": 2 * n ** 3 / ms / 1e9,
                       "normwise_rel_err": err, "max_abs_err_over_rms": mx}), flush=True)
 
 
@@ -54,6 +54,6 @@ if __name__ == "__main__":
     if len(sys.argv) > 1 and sys.argv[1] == "one":
         one()
     else:
-        for r in ("2", "4", "8", "16", "32", "125"):
-            env = dict(os.environ, EATSS_TCM_CHUNK=r)
+        for r in ("64", "128", "256", "512", "4000"):
+            env = dict(os.environ, EATSS_TCM_CHUNK_K=r)
             subprocess.run([sys.executable, __file__, "one"], env=env, check=False)

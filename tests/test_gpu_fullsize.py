@@ -6,7 +6,7 @@ both engines, comparing WHOLE output matrices with the fp64 oracle (no sampling)
 * Exact pass: small-integer / sparse-ternary inputs whose every partial sum the oracle certifies below
   2^24 (fp32) -- and, on the 3xTF32 tensor path, every MMA operand (chained products' intermediates)
   below 2^11 so that its lo half is exact -- must equal the oracle bit for bit.
-The tiles are the ones the bench times: the SIMT pick (16,1024,16) and the tensor-mode pick (128,256,32).
+The tiles are the ones the bench times: the SIMT pick (16,1024,16) and the tensor-mode pick (256,256,32).
 """
 import numpy as np
 import pytest
@@ -19,7 +19,7 @@ pytestmark = pytest.mark.gpu
 E = pytest.importorskip("paper_conf_cgo_jayaweerakwk24_b200")
 
 N = 4000
-ENGINES = [(1, (16, 1024, 16)), (2, (128, 256, 32))]
+ENGINES = [(1, (16, 1024, 16)), (2, (256, 256, 32))]
 IDS = ["simt", "tensor"]
 
 

@@ -21,7 +21,8 @@ def pinned(x):
 
 
 @pytest.mark.parametrize("engine,tiles,shape,rb", [
-    (2, (128, 256, 32), (1000, 520, 300), 3),   # tensor engine: CTA-pair row blocks, ragged last
+    (2, (256, 256, 32), (1000, 520, 300), 3),   # tensor engine: CTA-pair row blocks, ragged last
+    (2, (128, 208, 16), (700, 530, 300), 3),    # tensor engine: single-CTA tiles
     (2, (128, 128, 32), (700, 384, 96), 1),     # single block
     (1, (16, 1024, 16), (333, 1100, 70), 5),    # SIMT, ragged tiles
     (1, (32, 32, 32), (256, 256, 256), 8),

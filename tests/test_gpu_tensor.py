@@ -79,7 +79,8 @@ def test_tc_2mm_3mm(cuda_device):
 
 
 # ---- MMA-legal tiles (Ti = 128): TMA + SS-UMMA GEMM (tc_mma.cu)
-MMA_TILES = [(128, 256, 32), (128, 128, 32), (128, 64, 8), (128, 192, 16), (128, 32, 32)]
+MMA_TILES = [(256, 256, 32), (128, 256, 32), (128, 128, 32), (128, 64, 8), (128, 192, 16), (128, 32, 32),
+             (256, 96, 64), (128, 48, 16), (128, 208, 32), (256, 64, 8), (256, 160, 16), (128, 16, 64)]
 
 
 @pytest.mark.parametrize("tiles", MMA_TILES)
@@ -109,7 +110,7 @@ def test_tcm_full_size_sampled(cuda_device):
     d = E.desc_builtin("gemm", (n, n, n)); d.set_scalars(1.5, 1.2); d.set_exec(50, TENSOR)
     A = synth.uniform((n, n), 4); B = synth.uniform((n, n), 5); C = synth.uniform((n, n), 6)
     Cd = dev(C)
-    E.run(d, (128, 256, 32), [Cd, dev(A), dev(B)])
+    E.run(d, (256, 256, 32), [Cd, dev(A), dev(B)])
     out = host(Cd)
     g = synth.rng(7)
     ii = g.integers(0, n, 2048); jj = g.integers(0, n, 2048)
@@ -117,7 +118,8 @@ def test_tcm_full_size_sampled(cuda_device):
 
 
 # ---- syrk on the tensor pipe: B(k, j) = A(j, k) is K-major (same operand layout as A)
-SYRK_TILES = [(128, 256, 32), (128, 224, 16), (128, 96, 32), (128, 32, 8)]
+SYRK_TILES = [(256, 256, 32), (128, 256, 32), (128, 224, 16), (128, 96, 32), (128, 32, 8), (256, 48, 32),
+              (256, 80, 64), (128, 16, 16)]
 
 
 @pytest.mark.parametrize("tiles", SYRK_TILES)
@@ -151,7 +153,7 @@ def test_tcm_syrk_full_size_sampled(cuda_device):
     A = synth.uniform((n, n), 8); C = synth.uniform((n, n), 9)
     d = E.desc_builtin("syrk", (n, n)); d.set_scalars(1.5, 1.2); d.set_exec(50, TENSOR)
     Cd = dev(C)
-    E.run(d, (128, 256, 32), [Cd, dev(A)])
+    E.run(d, (256, 256, 32), [Cd, dev(A)])
     out = host(Cd)
     g = synth.rng(10)
     ii = g.integers(0, n, 2048); jj = g.integers(0, n, 2048)
@@ -168,11 +170,11 @@ def test_tcm_tail_split_on_and_off(cuda_device, monkeypatch, splitk):
     A = synth.small_int((ni, nk), 30); B = synth.small_int((nk, nj), 31); C = synth.small_int((ni, nj), 32)
     d = E.desc_builtin("gemm", (ni, nj, nk)); d.set_scalars(1.0, 2.0); d.set_exec(50, TENSOR)
     Cd = dev(C)
-    E.run(d, (128, 256, 32), [Cd, dev(A), dev(B)])
+    E.run(d, (256, 256, 32), [Cd, dev(A), dev(B)])
     assert np.array_equal(host(Cd), O.gemm(1.0, 2.0, C, A, B))
 
 
-@pytest.mark.parametrize("tiles", [(128, 256, 32), (128, 160, 32)])
+@pytest.mark.parametrize("tiles", [(256, 256, 32), (128, 256, 32), (128, 160, 32), (256, 96, 16)])
 def test_tcm_2mm_3mm(cuda_device, tiles):
     ni, nj, nk, nl, nm = 331, 260, 296, 300, 140
     A = synth.uniform((ni, nk), 50); B = synth.uniform((nk, nj), 51)
@@ -191,7 +193,7 @@ def test_tcm_2mm_3mm(cuda_device, tiles):
         assert O.normwise_rel_err(host(got), want) <= 1e-5
 
 
-@pytest.mark.parametrize("tiles", [(128, 256, 32), (128, 96, 32)])
+@pytest.mark.parametrize("tiles", [(256, 256, 32), (128, 96, 32), (128, 48, 8)])
 def test_tcm_split_exact_for_22_bit_values(cuda_device, tiles):
     # hi + lo reproduces every fp32 value with <= 22 significant bits exactly, whichever split
     # mode is active (rna hi, or the raw operand read by the truncating tensor core): A @ I == A
@@ -214,18 +216,18 @@ def test_kernel_timing_and_launch_count(cuda_device):
     d = E.desc_builtin("gemm", (n, n, n)); d.set_scalars(1.5, 1.2); d.set_exec(50, TENSOR, time_kernels=1)
     bufs = [torch.rand(n, n, device="cuda") for _ in range(3)]
     s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    E.run(d, (128, 256, 32), bufs)
-    s.record(); E.run(d, (128, 256, 32), bufs); e.record()
+    E.run(d, (256, 256, 32), bufs)
+    s.record(); E.run(d, (256, 256, 32), bufs); e.record()
     torch.cuda.synchronize()
     (k,) = E.last_kernel_ms(d)
     assert 0 < k < s.elapsed_time(e)
     # 2500/256 -> 10 pair-rows x 10 column tiles = 100 tiles on 74 clusters: the 26-tile tail is
     # split along k (pre-pass needed for beta != 1, run inside the prep launch)
-    assert E.launches_per_run(d, (128, 256, 32)) == 2
+    assert E.launches_per_run(d, (256, 256, 32)) == 2
     d.set_scalars(1.5, 1.0)
-    assert E.launches_per_run(d, (128, 256, 32)) == 2
+    assert E.launches_per_run(d, (256, 256, 32)) == 2
     ds = E.desc_builtin("syrk", (n, n)); ds.set_exec(50, TENSOR)
-    assert E.launches_per_run(ds, (128, 256, 32)) == 2
+    assert E.launches_per_run(ds, (256, 256, 32)) == 2
     d2 = E.desc_builtin("gemm", (n, n, n))
     with pytest.raises(E.EatssError):
         E.last_kernel_ms(d2)
@@ -282,3 +284,55 @@ def test_ccsd_tc_full_size_dims48_sampled(cuda_device):
     assert O.normwise_rel_err(got, ref) <= 1e-5
     del t3d
     torch.cuda.empty_cache()
+
+
+# ---- the whole tensor-engine tile space: Ti in {128, 256}, Tj in 16..256 step 16,
+# Tk in {8, 16, 32, 64}; every executable tile exact on small integers (gemm: MN-major B; syrk: K-major)
+def _space():
+    return [(ti, tj, tk) for ti in (128, 256) for tj in range(16, 257, 16) for tk in (8, 16, 32, 64)]
+
+
+@pytest.fixture(scope="module")
+def space_inputs():
+    ni, nj, nk = 300, 1100, 204
+    A = synth.small_int((ni, nk), 10); B = synth.small_int((nk, nj), 11); C = synth.small_int((ni, nj), 12)
+    As = synth.small_int((ni, nk), 13); Cs = synth.small_int((ni, ni), 14)
+    return (ni, nj, nk), (A, B, C, O.gemm(1.0, 1.0, C, A, B)), (As, Cs, O.syrk(1.0, 1.0, Cs, As))
+
+
+def test_tcm_whole_tile_space_exact(cuda_device, space_inputs):
+    (ni, nj, nk), (A, B, C, ref), (As, Cs, refs) = space_inputs
+    d = E.desc_builtin("gemm", (ni, nj, nk)); d.set_scalars(1.0, 1.0); d.set_exec(50, TENSOR)
+    ds = E.desc_builtin("syrk", (ni, nk)); ds.set_scalars(1.0, 1.0); ds.set_exec(50, TENSOR)
+    Ad, Bd, Asd = dev(A), dev(B), dev(As)
+    ran = {"gemm": 0, "syrk": 0}
+    for t in _space():
+        for name, dd, mk, r in (("gemm", d, lambda: [dev(C), Ad, Bd], ref), ("syrk", ds, lambda: [dev(Cs), Asd], refs)):
+            b = mk()
+            try:
+                E.run(dd, t, b)
+            except E.EatssError as err:
+                assert err.status == -5, (name, t)  # EATSS_E_UNSUPPORTED: shared memory / legal N only
+                ti, tj, tk = t
+                assert (name == "gemm" and ti == 256 and (tj // 2) % 16) or tk == 64, (name, t)
+                continue
+            assert np.array_equal(host(b[0]), r), (name, t)
+            ran[name] += 1
+    assert ran["gemm"] >= 80 and ran["syrk"] >= 80, ran
+
+
+def test_tcm_model_space_is_executable(cuda_device):
+    """Every tile reading T declares feasible (tensor mode of eatss_select_tiles) is one
+    the executor accepts: the model's T3 constraints are the executor's legality + shared memory."""
+    from oracle import model as M
+    doms = M.tensor_domains(M.gemm())
+    import itertools
+    feas = [t for t in itertools.product(*doms)
+            if M.evaluate_tensor(M.gemm(), M.B200, M.Opts(50, 16, 2), [np.array([v]) for v in t])[0][0]]
+    assert len(feas) == 36
+    n = 512
+    d = E.desc_builtin("gemm", (n, n, n)); d.set_exec(50, TENSOR)
+    bufs = [torch.zeros((n, n), device="cuda") for _ in range(3)]
+    for t in feas:
+        E.run(d, t, bufs)
+    torch.cuda.synchronize()

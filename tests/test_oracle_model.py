@@ -149,14 +149,18 @@ def test_model_golden_regenerates():
 
 
 def test_tensor_mode_hand_checked():
-    """Reading T on gemm 4000 fp32, B200: domain Ti = {128}, Tk = {32}, Tj = {32, 64, ..., 256}.
-
-    TMEM 2*Tj <= 512 and SMEM 2*2*4*(128*32 + 32*Tj) <= 232448 (Tj <= 326) hold for all 8
-    points; OBJ = Ti*Tj + 2*16*Tj = 160*Tj is maximal and unique at Tj = 256 -> (128, 256, 32).
-    With GA100's 48 KB shared memory per block no point fits (16*(4096+32*Tj) > 49152).
-    """
+    """Reading T on gemm 4000 fp32, B200 (max_smem 232448 B, 2048 B reserved -> 230400 B for the ring):
+    domain Ti in {128, 256} (one CTA / a CTA pair, CG = Ti/128), Tj in {16, ..., 256}, Tk in {32, 64}.
+    Per-CTA stage bytes x 2 stages = 2*2*4*(128*Tk + Tk*ceil32(Tj/CG)) <= 230400, i.e.
+    128*Tk + Tk*ceil32(Tj/CG) <= 14400:
+      Ti=128, Tk=32: ceil32(Tj) <= 322 -> all 16 Tj;  Tk=64: ceil32(Tj) <= 97 -> Tj <= 96: 6;
+      Ti=256 (Tj/2 must be a multiple of 16 -> Tj in 32N: 8 values), Tk=32: all 8;
+      Tk=64: ceil32(Tj/2) <= 97 -> Tj <= 192: 6.            n_feasible = 16 + 6 + 8 + 6 = 36.
+    TMEM 2*Tj <= 512 holds everywhere.  OBJ = Ti*Tj + 2*16*Tj = (Ti + 32)*Tj is maximal at Ti = 256,
+    Tj = 256 (73728); (256, 256, 64) needs 128*64 + 64*128 = 16384 > 14400, so the optimum is unique.
+    With GA100's 48 KB per block no point fits (even (128, 16, 32): 16*(4096 + 1024) = 81920 > 47104)."""
     r = M.select_tiles(M.gemm(), M.B200, M.Opts(50, 16, 2))
-    assert r.n_feasible == 8 and r.n_ties == 1 and r.tiles == (128, 256, 32) and r.obj == 160 * 256
+    assert r.n_feasible == 36 and r.n_ties == 1 and r.tiles == (256, 256, 32) and r.obj == 288 * 256
     assert M.select_tiles(M.gemm(), M.GA100, M.Opts(50, 16, 2)).tiles is None
     assert M.select_tiles(M.heat3d(), M.B200, M.Opts(50, 16, 2)).tiles is None  # not a contraction
 
