@@ -25,7 +25,10 @@
  *     own device scratch, allocated on the first run that needs it and freed with the
  *     descriptor: mttkrp's split partials / tensor-path block partials, SIMT syrk's A^T
  *     layout copy, eatss_run_host's device buffers.  Runs of ONE descriptor on different
- *     streams must therefore be ordered by the caller (they share that scratch).
+ *     streams must therefore be ordered by the caller (they share that scratch).  The tensor
+ *     engines' split operands (3xTF32 lo halves) are per-run scratch instead: allocated on the
+ *     run's stream from a library-owned pool of the current device (cudaMallocFromPoolAsync) and
+ *     freed on it after the run's launches, so they are never shared between runs.
  *   - eatss_run is asynchronous on `stream`: argument and launch-configuration
  *     errors are returned synchronously; device faults surface on the stream.
  *   - No CPU fallback exists: without a CUDA device eatss_run returns EATSS_E_CUDA.

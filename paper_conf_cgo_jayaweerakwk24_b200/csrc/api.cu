@@ -4,6 +4,8 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <map>
+#include <mutex>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -273,6 +275,47 @@ static eatss_status ensure_ws(eatss_kernel_desc *d, size_t need) {
     d->ws_dev = dev;
     return EATSS_OK;
 }
+
+// Stream-ordered scratch of ONE run (tensor engines' split operands): allocated from a library-owned
+// pool of the current device on the run's stream and freed on it after the run's launches, so runs on
+// different streams, devices or host threads never share it and nothing synchronises (the pool keeps
+// its memory: release threshold = max).
+static cudaMemPool_t scratch_pool() {
+    static std::mutex mu;
+    static std::map<int, cudaMemPool_t> pools;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = pools.find(dev);
+    if (it != pools.end()) return it->second;
+    cudaMemPoolProps props{};
+    props.allocType = cudaMemAllocationTypePinned;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = dev;
+    cudaMemPool_t pool = nullptr;
+    if (cudaMemPoolCreate(&pool, &props) != cudaSuccess) return nullptr;
+    uint64_t thr = UINT64_MAX;
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    pools[dev] = pool;
+    return pool;
+}
+struct RunScratch {  // freed (stream-ordered) when the run's launches have been issued
+    void *p = nullptr;
+    size_t bytes = 0;
+    cudaStream_t s = nullptr;
+    cudaError_t alloc(size_t n, cudaStream_t st) {
+        s = st;
+        cudaMemPool_t pool = scratch_pool();
+        if (!pool) return cudaErrorMemoryAllocation;
+        cudaError_t e = cudaMallocFromPoolAsync(&p, n, pool, st);
+        if (e == cudaSuccess) bytes = n;
+        else p = nullptr;
+        return e;
+    }
+    ~RunScratch() {
+        if (p) cudaFreeAsync(p, s);
+    }
+};
 
 // SIMT syrk: its transposed operand B(k, j) = A[j][k] is laid out as A^T once per run (a layout pass
 // into the descriptor's workspace, ~2 x 64 MB of traffic at N = 4000) so the executor runs its
@@ -843,13 +886,17 @@ static eatss_status run_body(eatss_kernel_desc *d, int only_nest, const int64_t 
             if (e != cudaSuccess) return cuda_fail(e, "eatss_run(syrk layout pass)");
             untranspose_nests(d, cn, d->ws);
         }
-        if (d->exec.engine == EATSS_ENGINE_TENSOR) {  // split-operand scratch for the tcgen05 GEMMs
+        RunScratch scratch;  // split-operand scratch of the tcgen05 GEMMs (stream-ordered, this run only)
+        if (d->exec.engine == EATSS_ENGINE_TENSOR) {
             size_t need = 0;
             for (int i = 0; i < (int)cn.size(); i++) {
                 ContractPlan p = plan_contraction(cn[i], tiles, sl, d->exec.warp_align);
                 if (tcm_applicable(cn[i], p)) need = std::max(need, tcm_ws_floats(cn[i], p));
             }
-            if (need && (st = ensure_ws(d, need * 4)) != EATSS_OK) return st;
+            if (need) {
+                cudaError_t e = scratch.alloc(need * 4, s);
+                if (e != cudaSuccess) return cuda_fail(e, "eatss_run(tensor scratch)");
+            }
         }
         for (int i = 0; i < (int)cn.size(); i++) {
             if (only_nest >= 0 && i != only_nest) continue;
@@ -863,7 +910,7 @@ static eatss_status run_body(eatss_kernel_desc *d, int only_nest, const int64_t 
                 return fail(EATSS_E_UNSUPPORTED, "eatss_run: tensor engine not applicable to this tile/operand layout");
             cudaEvent_t *ev = kernel_events(d, i);
             if (ev && !tcm) cudaEventRecord(ev[0], s);
-            cudaError_t e = tcm  ? launch_tcm_contraction(cn[i], p, (float *)d->ws, d->ws_bytes / 4, s, ev)
+            cudaError_t e = tcm  ? launch_tcm_contraction(cn[i], p, (float *)scratch.p, scratch.bytes / 4, s, ev)
                             : tc ? launch_tc_contraction(cn[i], p, exec_cv(d), s)
                                  : launch_contraction(cn[i], p, exec_cv(d), nullptr, s);
             if (ev && !tcm) cudaEventRecord(ev[1], s);
@@ -932,9 +979,11 @@ static eatss_status run_body(eatss_kernel_desc *d, int only_nest, const int64_t 
             return fail(EATSS_E_UNSUPPORTED, "eatss_run: tensor engine needs a ccsd tile (1,1,Th1,Tp6,Tp5,Tp4,>=H7) "
                                              "with Th1*Tp5*Tp4 <= 128, Tp6 % 16 == 0, Tp4 % 4 == 0, "
                                              "P4 % 4 == 0, H7 % 4 == 0, H7 <= 64");
-        if ((st = ensure_ws(d, ccsd_tc_ws_floats(d->dims.data()) * 4)) != EATSS_OK) return st;
-        cudaError_t e = launch_ccsd_tc((float *)buffers[0], (const float *)buffers[1], (const float *)buffers[2],
-                                       d->dims.data(), tiles, 0, d->dims[0], (float *)d->ws, d->ws_bytes / 4, s, ev);
+        RunScratch scratch;  // v2's lo half (stream-ordered, this run only)
+        cudaError_t e = scratch.alloc(ccsd_tc_ws_floats(d->dims.data()) * 4, s);
+        if (e != cudaSuccess) return cuda_fail(e, "eatss_run(ccsd tensor scratch)");
+        e = launch_ccsd_tc((float *)buffers[0], (const float *)buffers[1], (const float *)buffers[2], d->dims.data(),
+                           tiles, 0, d->dims[0], (float *)scratch.p, scratch.bytes / 4, s, ev);
         return e == cudaSuccess ? EATSS_OK : cuda_fail(e, "eatss_run(ccsd_t_d1, tensor)");
     }
     if (ev) cudaEventRecord(ev[0], s);
@@ -1056,6 +1105,16 @@ eatss_status eatss_run_host(const eatss_kernel_desc *cd, const int64_t *tiles, v
         char *dA = (char *)dev_bufs[1], *dC = (char *)dev_bufs[0];
         cudaMemcpyAsync(dev_bufs[2], hB, d->hbuf_bytes[2], cudaMemcpyHostToDevice, sin);
         const int sl = smem_limit_bytes();
+        RunScratch scratch;  // tensor engine: split operands of the largest block (blocks run in order on s)
+        if (d->exec.engine == EATSS_ENGINE_TENSOR) {
+            ContractNest b0 = full;
+            b0.M = std::min(rb, M);
+            ContractPlan p0 = plan_contraction(b0, tiles, sl, d->exec.warp_align);
+            if (tcm_applicable(b0, p0)) {
+                const cudaError_t ea = scratch.alloc(tcm_ws_floats(b0, p0) * 4, s);
+                if (ea != cudaSuccess) return cuda_fail(ea, "eatss_run_host(tensor scratch)");
+            }
+        }
         for (int r = 0; r < nblk; r++) {
             const int64_t r0 = (int64_t)r * rb, rows = std::min(rb, M - r0);
             cudaMemcpyAsync(dA + r0 * rowA, hA + r0 * rowA, rows * rowA, cudaMemcpyHostToDevice, sin);
@@ -1075,8 +1134,7 @@ eatss_status eatss_run_host(const eatss_kernel_desc *cd, const int64_t *tiles, v
             const bool tc = want_tc && !tcm && tc_plan(blk, p, &tsm, &tcols);
             if (want_tc && !tc && !tcm)
                 return fail(EATSS_E_UNSUPPORTED, "eatss_run_host: tensor engine not applicable to this tile");
-            if (tcm && (st = ensure_ws(d, tcm_ws_floats(blk, p) * 4)) != EATSS_OK) return st;
-            e = tcm  ? launch_tcm_contraction(blk, p, (float *)d->ws, d->ws_bytes / 4, s, nullptr)
+            e = tcm  ? launch_tcm_contraction(blk, p, (float *)scratch.p, scratch.bytes / 4, s, nullptr)
                 : tc ? launch_tc_contraction(blk, p, exec_cv(d), s)
                      : launch_contraction(blk, p, exec_cv(d), nullptr, s);
             if (e != cudaSuccess) return cuda_fail(e, "eatss_run_host(gemm block)");
