@@ -24,6 +24,8 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-std=c++17", "-O3", "-lineinfo", "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden",
          "-diag-suppress", "128", "-I", os.path.join(ROOT, "include")]
+# development builds only (e.g. -DEATSS_DEVTOOLS for cost-isolation switches); never set by build()
+FLAGS += os.environ.get("EATSS_DEV_NVCC_FLAGS", "").split()
 
 
 def _sources():

@@ -36,6 +36,7 @@
 
 #include <algorithm>
 #include <cstdint>
+#include <cstdio>
 #include <cstdlib>
 #include <map>
 #include <mutex>
@@ -76,6 +77,9 @@ struct Args {
     int nunits;   // nfull + (T - nfull) * sp
     int nkb;      // k-blocks of Tk
     int group_rows;  // tile-order grouping (row groups per group) for L2 reuse
+    unsigned long long *prof;  // development (EATSS_TCM_PROF): per-site cycle counters, else nullptr
+    int dbg;  // -DEATSS_DEVTOOLS builds only (EATSS_TCM_DBG; results then wrong): 1 no TMEM drain,
+              // 4 no accumulator reset at chunk starts
 };
 
 __host__ __device__ inline void tile_coords(int t, int PI, int TJ, int G, int &pi, int &tj) {
@@ -218,9 +222,15 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                 const int nk = w.kb1 - w.kb0;
                 for (int x = 0; x < nk; x++, it++) {
                     const int s = it % p.S, bd = gc & 1;
-                    const bool first = (x % R) == 0;
+                    const bool first = (p.dbg & 4) ? x == 0 : (x % R) == 0;
+                    const long long t0 = p.prof ? clock64() : 0;
                     if (first && gc >= 2) mbar_wait_cluster(dempty + bd, (unsigned)(((gc - 2) >> 1) & 1));
+                    const long long t1 = p.prof ? clock64() : 0;
                     mbar_wait(full + s, (unsigned)((it / p.S) & 1));
+                    if (p.prof) {
+                        atomicAdd(p.prof + 0, (unsigned long long)(t1 - t0));
+                        atomicAdd(p.prof + 1, (unsigned long long)(clock64() - t1));
+                    }
                     fence_after();
                     const unsigned char *st = smem + (size_t)s * STAGE;
                     const unsigned char *sb = st + 2 * A_BYTES;
@@ -263,13 +273,15 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             for (int c = 0; c < MAXCW; c++) acc[c] = 0.f;
             for (int ch = 0; ch < nch; ch++, gc++) {
                 const int bd = gc & 1;
+                const long long t0 = p.prof ? clock64() : 0;
                 mbar_wait(dfull + bd, (unsigned)((gc >> 1) & 1));
+                const long long t1 = p.prof ? clock64() : 0;
                 fence_after();
                 const uint32_t ta = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(bd * 256 + cq * CW);
                 // drain: four 4-column loads in flight per wait
 #pragma unroll
                 for (int c0 = 0; c0 < MAXCW; c0 += 16) {
-                    if (c0 < CW) {
+                    if (c0 < CW && !(p.dbg & 1)) {
                         uint32_t v[4][4];
 #pragma unroll
                         for (int g = 0; g < 4; g++)
@@ -288,8 +300,14 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                 if (lane == 0) {
                     if constexpr (CG == 2) mbar_arrive_cluster(demp0 + 8u * (uint32_t)bd);
                     else mbar_arrive(dempty + bd);
+                    if (p.prof) {
+                        atomicAdd(p.prof + 2, (unsigned long long)(t1 - t0));
+                        atomicAdd(p.prof + 3, (unsigned long long)(clock64() - t1));
+                        atomicAdd(p.prof + 4, 1ull);
+                    }
                 }
             }
+            const long long te = p.prof ? clock64() : 0;
             // C(i, j) for row i = i0 + 32q + lane, columns jb .. jb + CW - 1
             const int64_t i = (int64_t)(w.pi * CG + (int)rank) * BM + q * 32 + lane;
             const int64_t jb = (int64_t)w.tj * p.BNT + cq * CW;
@@ -343,6 +361,10 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                         }
                     }
                 }
+            }
+            if (p.prof && lane == 0) {
+                atomicAdd(p.prof + 5, (unsigned long long)(clock64() - te));
+                atomicAdd(p.prof + 6, 1ull);
             }
         }
     }
@@ -716,9 +738,34 @@ cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p,
     a.TJ = (int)((n.N + bn - 1) / bn);
     static const int group_env = devsw("EATSS_TCM_GROUP", 8);  // development: row groups per raster group
     a.group_rows = std::max(1, group_env);
+    a.prof = nullptr;
+#ifdef EATSS_DEVTOOLS
+    a.dbg = devsw("EATSS_TCM_DBG", 0);
+#else
+    a.dbg = 0;
+#endif
+    static unsigned long long *prof = nullptr;
+    if (devsw("EATSS_TCM_PROF", 0)) {  // development: wait / drain / epilogue cycle profile (printed)
+        if (!prof) cudaMalloc(&prof, 16 * sizeof(unsigned long long));
+        cudaMemsetAsync(prof, 0, 16 * sizeof(unsigned long long), s);
+        a.prof = prof;
+    }
+    cudaError_t r;
     if (n.transB)
-        return cg == 2 ? launch_bk<true, 2>(bk, m, a, g.smem, nsm, pr, s, ev) : launch_bk<true, 1>(bk, m, a, g.smem, nsm, pr, s, ev);
-    return cg == 2 ? launch_bk<false, 2>(bk, m, a, g.smem, nsm, pr, s, ev) : launch_bk<false, 1>(bk, m, a, g.smem, nsm, pr, s, ev);
+        r = cg == 2 ? launch_bk<true, 2>(bk, m, a, g.smem, nsm, pr, s, ev) : launch_bk<true, 1>(bk, m, a, g.smem, nsm, pr, s, ev);
+    else
+        r = cg == 2 ? launch_bk<false, 2>(bk, m, a, g.smem, nsm, pr, s, ev) : launch_bk<false, 1>(bk, m, a, g.smem, nsm, pr, s, ev);
+    if (a.prof) {
+        unsigned long long h[16];
+        cudaMemcpyAsync(h, a.prof, sizeof(h), cudaMemcpyDeviceToHost, s);
+        cudaStreamSynchronize(s);
+        const double nmma = (double)a.nunits * a.nkb;  // k-blocks issued (approx.)
+        fprintf(stderr,
+                "tc_mma prof: MMA wait dempty %.0f / wait full %.0f cycles per k-block | EPI wait dfull %.0f / "
+                "drain %.0f per chunk-warp (%llu) | C epilogue %.0f per tile-warp (%llu)\n",
+                h[0] / nmma, h[1] / nmma, h[2] / (double)h[4], h[3] / (double)h[4], h[4], h[5] / (double)h[6], h[6]);
+    }
+    return r;
 }
 
 int tcm_launches(const ContractNest &, const ContractPlan &) {
