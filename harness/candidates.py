@@ -12,8 +12,11 @@ executor family the sweep uses (engine = SIMT; the paper's code class):
 
   * candidates: sigma in {0, 50, 100} % (reading Q17) x WAF in {4, 8, 16, 32}; infeasible
     pairs are recorded (e.g. heat-3d at WAF 32, P:282; the 6-D contraction at WAF >= 8);
-  * each distinct (tile, sigma) is measured with eatss_sweep (warm-up, then back-to-back runs
-    for >= --window s, CUDA-event time, NVML energy counter, P:225) at carve-out sigma;
+  * each distinct (tile, sigma, WAF) is measured with eatss_sweep (warm-up, then back-to-back runs
+    for >= --window s, CUDA-event time, NVML energy counter) at carve-out sigma requested
+    EXACTLY (exec.carveout_exact; the carve-out each run requested is recorded from
+    eatss_last_carveout) and, for the gemm family, with WAF lanes of every warp along l_s1
+    (exec.warp_align: the executor's SIMT length, P:25);
   * baseline: PPCG's default tile (32 per tiled loop) at the same three carve-outs.
 
 The summary gives, per kernel, the best candidate's PPW (GFLOP/s/W = FLOP/J) over
@@ -67,8 +70,12 @@ def parse():
     return ap.parse_args()
 
 
+CONTRACTIONS = ("gemm", "2mm", "3mm", "syrk")
+
+
 def candidates(E, d, gpu):
-    """{(tile, sigma): [(sigma, waf), ...]} plus the infeasible (sigma, waf) pairs."""
+    """{(tile, sigma, waf): [(sigma, waf, obj), ...]} plus the infeasible (sigma, waf) pairs; the WAF is
+    part of the key only where the executor honours it (the gemm family)."""
     out, infeasible = {}, []
     for s in SPLITS:
         for w in WAFS:
@@ -79,15 +86,19 @@ def candidates(E, d, gpu):
                     raise
                 infeasible.append((s, w))
                 continue
-            out.setdefault((tuple(t), s), []).append((s, w, int(rep.obj)))
+            out.setdefault((tuple(t), s, w if d.kind in CONTRACTIONS else 0), []).append((s, w, int(rep.obj)))
     return out, infeasible
 
 
-def measure(E, d, tiles, split, bufs, a):
-    d.set_exec(split_pct=split, engine=1)
+def measure(E, d, tiles, split, bufs, a, waf=0):
+    d.set_exec(split_pct=split, engine=1, warp_align=waf, carveout_exact=1)
     m = E.sweep(d, [tiles], bufs, device=a.device, warmup=a.warmup, min_window_s=a.window)[0]
+    try:
+        cv = E.last_carveout(d)
+    except E.EatssError:
+        cv = None
     return dict(ms=m.ms_per_run, joules=m.joules_per_run, watts=m.avg_watts, tflops=m.tflops,
-                ppw=m.gflops_per_watt, sm_mhz=m.sm_mhz_median, status=m.status)
+                ppw=m.gflops_per_watt, sm_mhz=m.sm_mhz_median, status=m.status, carveout_requested=cv)
 
 
 def confirm(E, d, bufs, a, cands):
@@ -98,7 +109,7 @@ def confirm(E, d, bufs, a, cands):
     tf = {i: [] for i in range(len(cands))}
     for _ in range(a.confirm):
         for i, c in enumerate(cands):
-            r = measure(E, d, tuple(c["tiles"]), c["split"], bufs, a)
+            r = measure(E, d, tuple(c["tiles"]), c["split"], bufs, a, c.get("waf", 0))
             if r["status"] == 0 and r["ppw"] > 0:
                 ppw[i].append(r["ppw"]); tf[i].append(r["tflops"])
     out = []
@@ -131,9 +142,9 @@ def main():
             cands, infeasible = candidates(E, d, gpu)
             default = tuple([32] * d.num_loops)
             rows = []
-            for (tiles, s), origin in sorted(cands.items(), key=lambda kv: (kv[0][1], kv[0][0])):
-                r = measure(E, d, tiles, s, bufs, a)
-                rec = dict(kind=kind, role="eatss", tiles=list(tiles), split=s, origin=origin, **r)
+            for (tiles, s, w), origin in sorted(cands.items(), key=lambda kv: (kv[0][1], kv[0][2], kv[0][0])):
+                r = measure(E, d, tiles, s, bufs, a, w)
+                rec = dict(kind=kind, role="eatss", tiles=list(tiles), split=s, waf=w, origin=origin, **r)
                 rows.append(rec)
                 f.write(json.dumps(rec) + "\n"); f.flush()
             for s in SPLITS:
@@ -149,7 +160,7 @@ def main():
                 pe = max(ea, key=lambda r: r["tflops"])
                 bd = max(de, key=lambda r: r["ppw"]) if de else None
                 summary[kind] = dict(
-                    best_candidate=dict(tiles=be["tiles"], split=be["split"], origin=be["origin"],
+                    best_candidate=dict(tiles=be["tiles"], split=be["split"], waf=be["waf"], origin=be["origin"],
                                         ppw=be["ppw"], tflops=be["tflops"], watts=be["watts"]),
                     fastest_candidate=dict(tiles=pe["tiles"], split=pe["split"], ppw=pe["ppw"], tflops=pe["tflops"]),
                     best_default=(dict(split=bd["split"], ppw=bd["ppw"], tflops=bd["tflops"], watts=bd["watts"])
@@ -159,7 +170,7 @@ def main():
                     n_candidates=len(ea), infeasible=infeasible)
             if ea and a.confirm > 0:
                 be = max(ea, key=lambda r: r["ppw"]); pe = max(ea, key=lambda r: r["tflops"])
-                if (be["tiles"], be["split"]) != (pe["tiles"], pe["split"]):
+                if (be["tiles"], be["split"], be["waf"]) != (pe["tiles"], pe["split"], pe["waf"]):
                     summary[kind]["confirm"] = confirm(E, d, bufs, a, [be, pe])
             print(kind, json.dumps(summary.get(kind)), flush=True)
             del bufs

@@ -212,3 +212,66 @@ def test_mttkrp_conv2d_derivation():
     assert (c.ls1, c.nrefs, c.bset) == ("j", 3, ["j", "i"])
     assert c.H == {"i": 0, "j": 32, "p": 0, "q": 0}
     assert c.sh_fp == [frozenset("pq")] and frozenset("ijpq") in c.l1_fp
+
+
+# ------------------------------------------------------------------ alternative readings
+# tests/golden/reading_table.json was written by scripts/gen_reading_table.py (oracle/model.py only).
+# The paper prints four facts the model must reproduce: P:282 (heat-3d 9 of 12 configurations, all of
+# warp_frac 1.0 missing; conv-2d and mttkrp 11 of 12, the missing one warp_frac 1.0 at 50% shared
+# memory), P:153 (fdtd-2d no.references = 4), P:121 (the worked example's tile (16, 384, 16) and its
+# objective Ti*Tj + 2*16*Tj).  Each alternative reading either breaks one of them (excluded) or leaves
+# all four unchanged (unpinned: harness/readings.py measures what it would pick on B200).
+READINGS = _load("reading_table.json")["readings"]
+
+
+def _paper_facts_hold(rec, conv_f):
+    p = rec["p282"]
+    heat = all(p[k]["feasible"] == 9 and all(m[0] == 1.0 for m in p[k]["missing"])
+               for k in ("heat-3d n=120 fp64", "heat-3d n=120 fp32"))
+    mtt = all(p[k]["feasible"] == 11 and p[k]["missing"] == [[1.0, 50]]
+              for k in ("mttkrp 512x32x512x512", "mttkrp 64x32x64x64"))
+    conv = p[f"conv-2d n=8192 f={conv_f}"]["feasible"] == 11 and p[f"conv-2d n=8192 f={conv_f}"]["missing"] == [[1.0, 50]]
+    we = rec["worked_example"]
+    example = we["tiles"] == [16, 384, 16] and we["H"] == {"i": 0, "j": 32, "k": 0}
+    return heat and mtt and conv and example and rec["fdtd_nrefs"] == 4
+
+
+def test_reading_r_reproduces_every_paper_fact():
+    r = READINGS["R"]
+    # conv-2d's filter is not printed: under reading R the P:282 count holds for f = 5 or 6 only
+    assert [f for f in range(3, 12) if _paper_facts_hold(r, f)] == [5, 6]
+
+
+@pytest.mark.parametrize("name,why", [
+    ("footprint=halo", "P:282 conv-2d"), ("split=literal", "P:282 heat-3d / mttkrp / conv-2d"),
+    ("nrefs=array", "P:153 fdtd-2d and P:282 heat-3d fp32"), ("nrefs=ref", "P:153 fdtd-2d"),
+    ("units=KB", "P:121 tile"), ("waf_scale=warp", "P:121 objective 2 x 16"),
+])
+def test_excluded_readings_break_a_paper_fact_at_every_filter_size(name, why):
+    rec = READINGS[name]
+    assert not any(_paper_facts_hold(rec, f) for f in range(3, 12)), why
+    if name == "footprint=halo":  # the halo-inclusive footprint keeps all 12 conv-2d configurations
+        assert all(rec["p282"][f"conv-2d n=8192 f={f}"]["feasible"] == 12 for f in range(3, 12))
+
+
+@pytest.mark.parametrize("name", ["h_count=array", "h_count=ref", "rule2d=none", "rule2d=scaled", "bset=outer",
+                                  "bset=ls1_inner", "tiebreak=lexmin", "tiebreak=lexmax"])
+def test_unpinned_readings_keep_the_paper_facts_but_may_move_config_tiles(name):
+    rec = READINGS[name]
+    assert _paper_facts_hold(rec, 5)  # nothing in the paper separates them from R ...
+    r = {(t["kernel"], t["waf"]): t for t in READINGS["R"]["tiles"]}
+    moved = [(t["kernel"], t["waf"]) for t in rec["tiles"] if t["pick"] != r[(t["kernel"], t["waf"])]["pick"]]
+    expect = {"h_count=array": [("heat-3d", 8)], "h_count=ref": [], "rule2d=none": [], "rule2d=scaled": [],
+              "bset=outer": [("ccsd_t_d1", 4)], "bset=ls1_inner": [],
+              "tiebreak=lexmin": [], "tiebreak=lexmax": [("jacobi-2d", 16), ("heat-3d", 8), ("heat-3d", 4),
+                                                        ("ccsd_t_d1", 4)]}
+    assert moved == expect[name]  # ... so the tiles they move to are measured (harness/readings.py)
+
+
+def test_reading_table_regenerates_spot_checks():
+    rd = M.Reading(footprint="halo")
+    assert M.select_tiles(M.conv2d(8192, 5), M.GA100, M.Opts(50, 32, 0), keep_ties=False, rd=rd).tiles is not None
+    assert M.select_tiles(M.conv2d(8192, 5), M.GA100, M.Opts(50, 32, 0), keep_ties=False).tiles is None
+    r = M.select_tiles(M.ccsd_t_d1(48), M.B200, M.Opts(50, 4, 1), rd=M.Reading(bset="outer"), keep_ties=False)
+    want = next(t for t in READINGS["bset=outer"]["tiles"] if t["kernel"] == "ccsd_t_d1")
+    assert list(r.tiles) == want["pick"]
