@@ -319,8 +319,9 @@ def other_configs(E, torch, gpu, stream, peaks):
     b = bufs_for(d)
     row = {}
     simt_tiles, _ = E.select_tiles(d, gpu, split_pct=50, waf=4, mode=1)
-    for eng, tiles, note in ((1, simt_tiles, "EATSS B200 mode, WAF 4 (the space is empty for WAF >= 8)"),
-                             (2, (1, 2, 1, 48, 2, 48, 48), "hand-set MMA-legal tile: reading T covers depth-3 nests only")):
+    tc_tiles, _ = E.select_tiles(d, gpu, split_pct=50, waf=4, mode=2)
+    for eng, tiles, note in ((1, simt_tiles, "model: EATSS B200 mode, WAF 4 (the space is empty for WAF >= 8)"),
+                             (2, tc_tiles, "model: EATSS tensor-core mode, reading T4 (DESIGN.md §2.5), WAF 4")):
         d.set_exec(split_pct=50, engine=eng)
         ms = timed_ms(d, tiles, b, 2)
         gbs = d.bytes / (ms * 1e-3) / 1e9

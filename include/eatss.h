@@ -145,9 +145,11 @@ typedef struct {
     int32_t warp_align; /* WARP_ALIGNMENT_FACTOR = warp_frac * T_P_W, in {4, 8, 16, 32} */
     int32_t mode;       /* 0 = paper mode, 1 = B200 mode (clamp M_SH at max_smem_per_block),
                            2 = tensor-core mode (reading T: MMA-legal tiles of the
-                           tcgen05 executor -- Ti = 128, Tj in 32..256 step 32, Tk = 32 -- under
-                           TMEM / shared-memory capacities; depth-3 contraction nests only, else
-                           EATSS_E_UNSUPPORTED) */
+                           tcgen05 executors under their TMEM / shared-memory capacities -- depth-3
+                           contraction nests: Ti in {128, 256} (one CTA / a CTA pair), Tj in 16..256
+                           step 16, Tk in {32, 64}; the 6-D contraction (ccsd_t_d1, T4): rows
+                           Th1*Tp5*Tp4 <= 128, columns Th2*Tp6 <= 256, whole reduction; anything
+                           else EATSS_E_UNSUPPORTED) */
 } eatss_model_opts;
 
 /* Optional report of eatss_select_tiles (values of the first nest unless noted). */

@@ -437,6 +437,8 @@ def extents(prog: Program) -> List[int]:
 #   T2  domain: l_s1 (UMMA N) in {16, 32, ..., min(256, roundup16(N))}; the other B-set loop
 #       (UMMA M rows: one CTA or a CTA pair) in {128, 256}; the serial loop (k per pipeline stage,
 #       whole 128-byte swizzle atoms of fp32) in {32, 64};
+#   T4  the 6-D contraction pattern (ccsd_t_d1: one serial loop, three M-side and three N-side loops,
+#       _evaluate_tensor_6d): the executor's rows / columns / shared-memory budget instead of T2-T3.
 #   T3  per nest, CG = T_M / 128 CTAs per tile:
 #       legality: T_{l_s1} / CG a multiple of 16 (UMMA N per CTA half);
 #       TMEM: two fp32 accumulator buffers of T_{l_s1} columns, 2*T_{l_s1} <= 512;
@@ -449,14 +451,49 @@ TMEM_COLS = 512
 SMEM_RESERVE = 2048  # barriers + 1024-byte alignment of the stage ring
 
 
-def tensor_applicable(prog: Program) -> bool:
-    for nest in prog.nests:
-        if len(nest.loops) != 3 or sum(1 for l in nest.loops if not l.parallel) != 1:
-            return False
-        d = derive(nest, 16)
-        if not nest.loops[[l.name for l in nest.loops].index(d.ls1)].parallel:
-            return False
-    return True
+def _contraction_sets(nest: Nest):
+    """Depth >= 4 with one serial loop k and two read-only inputs X, Y sharing only k (T4): returns
+    (M-set loops of the input whose iterators contain l_s1, in loop order; N-set loops; k), else None."""
+    serial = [l.name for l in nest.loops if not l.parallel]
+    if len(nest.loops) < 4 or len(serial) != 1:
+        return None
+    k = serial[0]
+    d = derive(nest, 16)
+    written = {r.array for r in nest.refs if r.write}
+    ins = []
+    for r in d.refs:
+        if r.array not in written and r.iters() not in [x.iters() for x in ins]:
+            ins.append(r)
+    if len(ins) != 2:
+        return None
+    a, b = ins
+    if a.iters() & b.iters() != {k} or (a.iters() | b.iters()) != {l.name for l in nest.loops}:
+        return None
+    x, y = (a, b) if d.ls1 in a.iters() else (b, a)
+    if d.ls1 not in x.iters():
+        return None
+    order = [l.name for l in nest.loops]
+    mset = [n for n in order if n in x.iters() and n != k]
+    nset = [n for n in order if n in y.iters() and n != k]
+    return mset, nset, k
+
+
+def tensor_applicable(prog: Program):
+    """'3d' (T1: depth-3 nests, one serial loop, l_s1 parallel), '6d' (T4: the 6-D contraction pattern
+    of the ccsd executor: three M-side and three N-side loops), or False."""
+    if all(len(n.loops) == 3 for n in prog.nests):
+        for nest in prog.nests:
+            if sum(1 for l in nest.loops if not l.parallel) != 1:
+                return False
+            d = derive(nest, 16)
+            if not nest.loops[[l.name for l in nest.loops].index(d.ls1)].parallel:
+                return False
+        return "3d"
+    if len(prog.nests) == 1:
+        cs = _contraction_sets(prog.nests[0])
+        if cs and len(cs[0]) == 3 and len(cs[1]) == 3:
+            return "6d"
+    return False
 
 
 def tensor_domains(prog: Program):
@@ -464,6 +501,20 @@ def tensor_domains(prog: Program):
     d = derive(n0, 16)
     doms = []
     ex = extents(prog)
+    if tensor_applicable(prog) == "6d":
+        mset, nset, k = _contraction_sets(n0)
+        for p, l in enumerate(n0.loops):
+            if l.name == k:
+                doms.append([ex[p]])                                  # whole reduction in TMEM
+            elif l.name == d.ls1:
+                doms.append(list(range(4, ex[p] + 1, 4)))             # 16-byte TMA rows of the output
+            elif l.name == nset[0]:
+                doms.append([1])                                      # one outer N-side index per unit
+            elif l.name == nset[-1]:
+                doms.append(list(range(16, min(256, ex[p]) + 1, 16)) or [16])  # UMMA N granules
+            else:
+                doms.append(list(range(1, ex[p] + 1)))
+        return doms
     for p, l in enumerate(n0.loops):
         if l.name == d.ls1:
             hi = min(256, -(-ex[p] // 16) * 16)
@@ -475,7 +526,42 @@ def tensor_domains(prog: Program):
     return doms
 
 
+def _evaluate_tensor_6d(prog: Program, gpu: Gpu, opts: Opts, T):
+    """T4 (reading T for the 6-D contraction): MMA rows M = product of the M-side tiles
+    <= 128 TMEM lanes; columns N = product of the N-side tiles, a multiple of 16, <= 256; a middle N-side
+    tile > 1 needs whole innermost N-side and l_s1 tiles (one TMA box per unit); TMEM: an accumulator
+    buffer (N rounded up to a power of two >= 32) next to the 128 columns of the A operand; shared memory:
+    three epilogue groups' output tiles (M*N*e rounded to 1 KB) + two stages of the N-side operand (hi, lo;
+    k in 32-element atoms) <= max_smem_per_block - 1536.  B (the parallelism term) = M * N, the output
+    tile of one CTA (on the tensor core every parallel loop maps into it; for depth 3 it equals Ti*Tj)."""
+    e = prog.dtype_bytes
+    nest = prog.nests[0]
+    d = derive(nest, opts.waf)
+    mset, nset, k = _contraction_sets(nest)
+    pos = {l.name: p for p, l in enumerate(nest.loops)}
+    ex = {l.name: l.extent for l in nest.loops}
+    M = _prod(T, mset, pos)
+    N = _prod(T, nset, pos)
+    feas = (M <= 128) & (N <= 256) & (N % 16 == 0) & (T[pos[nset[-1]]] <= ex[nset[-1]])
+    feas &= ex[d.ls1] % 4 == 0  # 16-byte rows of the output tile
+    feas &= ~((T[pos[nset[1]]] > 1) & ((T[pos[nset[-1]]] != ex[nset[-1]]) | (T[pos[d.ls1]] != ex[d.ls1])))
+    bstride = np.maximum(32, 2 ** np.ceil(np.log2(np.maximum(N, 1))).astype(np.int64))
+    feas &= bstride <= 384
+    kext = ex[k]
+    feas &= (kext <= 64) & (kext % 4 == 0)
+    x_stage = -(-(M * N * e) // 1024) * 1024
+    v_stage = 2 * (-(-kext // 32)) * N * 128
+    feas &= 3 * x_stage + 2 * v_stage <= gpu.max_smem_per_block - 1536
+    obj = M * N
+    for l in nest.loops:
+        if d.H[l.name]:
+            obj = obj + d.H[l.name] * T[pos[l.name]]
+    return feas, obj
+
+
 def evaluate_tensor(prog: Program, gpu: Gpu, opts: Opts, T):
+    if tensor_applicable(prog) == "6d":
+        return _evaluate_tensor_6d(prog, gpu, opts, T)
     e = prog.dtype_bytes
     feas = np.ones(T[0].shape, dtype=bool)
     obj = np.zeros(T[0].shape, dtype=np.int64)
@@ -521,6 +607,9 @@ def select_tiles(prog: Program, gpu: Gpu, opts: Opts, keep_ties: bool = True, rd
     doms = ([np.array(v, dtype=np.int64) for v in tensor_domains(prog)] if tensor else
             [np.array(domain(n, gpu, opts.waf), dtype=np.int64) for n in extents(prog)])
     free = objective_free_positions(prog, opts.waf, rd)
+    if tensor and tensor_applicable(prog) == "6d":  # T4: objective-free = outside the CTA tile (the reduction)
+        k = _contraction_sets(prog.nests[0])[2]
+        free = [p for p, l in enumerate(prog.nests[0].loops) if l.name == k and not derive(prog.nests[0], opts.waf).H[k]]
     ls1_pos = [l.name for l in prog.nests[0].loops].index(derive(prog.nests[0], opts.waf, rd).ls1)
     best_key, best, ties, n_feas = None, None, [], 0
     # iterate the first position in Python, the rest as one numpy meshgrid block

@@ -177,6 +177,33 @@ void input_footprints(NestEval &ne) {
             break;
         }
 }
+// T4 (reading T for the 6-D contraction pattern): one serial loop k, two read-only
+// inputs sharing only k; M-side = the loops of the input that uses l_s1, N-side = the other input's.
+struct Sets6 {
+    bool ok = false;
+    std::vector<int> m, n;  // loop positions, outermost first
+    int k = -1;
+};
+Sets6 contraction_sets(const NestEval &ne) {
+    Sets6 r;
+    const Nest &n = *ne.nest;
+    const int L = (int)n.loops.size();
+    int serial = 0;
+    for (int p = 0; p < L; p++)
+        if (!n.loops[p].parallel) { serial++; r.k = p; }
+    if (L < 4 || serial != 1 || ne.in_fp.size() != 2) return r;
+    const uint32_t a = ne.in_fp[0], b = ne.in_fp[1], kb = 1u << r.k, all = (1u << L) - 1u;
+    if ((a & b) != kb || (a | b) != all) return r;
+    const uint32_t x = ((a >> ne.m.ls1) & 1u) ? a : b, y = x == a ? b : a;
+    if (!((x >> ne.m.ls1) & 1u)) return r;
+    for (int p = 0; p < L; p++) {
+        if (p == r.k) continue;
+        if ((x >> p) & 1u) r.m.push_back(p);
+        if ((y >> p) & 1u) r.n.push_back(p);
+    }
+    r.ok = r.m.size() == 3 && r.n.size() == 3;
+    return r;
+}
 constexpr int64_t kTmemCols = 512;
 
 struct Search {
@@ -200,11 +227,28 @@ struct Search {
         return v;
     }
 
-    bool tensor = false;
+    bool tensor = false, tensor6 = false;
+    Sets6 s6;                        // tensor6: M-side / N-side / reduction positions
+    std::vector<int64_t> ext;        // loop extents
     int64_t smem_cap = 0;
     int esz = 4;
 
     bool feasible(const std::vector<int64_t> &T) const {
+        if (tensor6) {  // reading T4: the ccsd executor's rows, columns and shared memory
+            int64_t M = 1, N = 1;
+            for (int p : s6.m) M *= T[p];
+            for (int p : s6.n) N *= T[p];
+            const int ls1 = nests[0].m.ls1, inner = s6.n.back(), mid = s6.n[1];
+            if (M > 128 || N > 256 || N % 16 || T[inner] > ext[inner] || ext[ls1] % 4) return false;
+            if (T[mid] > 1 && (T[inner] != ext[inner] || T[ls1] != ext[ls1])) return false;
+            int64_t bstride = 32;
+            while (bstride < N) bstride *= 2;
+            if (bstride > 384) return false;  // one accumulator buffer next to the 128 A columns
+            const int64_t kx = ext[s6.k];
+            if (kx > 64 || kx % 4) return false;
+            const int64_t x_stage = (M * N * esz + 1023) / 1024 * 1024, v_stage = 2 * ((kx + 31) / 32) * N * 128;
+            return 3 * x_stage + 2 * v_stage <= smem_cap - 1536;
+        }
         if (tensor) {  // reading T3
             for (const NestEval &ne : nests) {
                 const int64_t tn = T[ne.m.ls1], cg = T[ne.rows_pos] / 128;
@@ -244,7 +288,14 @@ struct Search {
     int64_t objective(const std::vector<int64_t> &T) const {  // Eq. 2, summed over nests
         int64_t obj = 0;
         for (const NestEval &ne : nests) {
-            obj += prod(T, ne.m.bset);
+            if (tensor6) {  // T4: the parallelism term is the CTA's output tile M x N
+                int64_t M = 1, N = 1;
+                for (int p : s6.m) M *= T[p];
+                for (int p : s6.n) N *= T[p];
+                obj += M * N;
+            } else {
+                obj += prod(T, ne.m.bset);
+            }
             for (size_t p = 0; p < ne.m.H.size(); p++) obj += ne.m.H[p] * T[p];
         }
         return obj;
@@ -332,7 +383,34 @@ extern "C" eatss_status eatss_select_tiles(const eatss_kernel_desc *d, const eat
         input_footprints(ne);
         s.nests.push_back(ne);
     }
-    if (o->mode == 2) {
+    s.ext = ext;
+    if (o->mode == 2 && s.nests.size() == 1 && s.nests[0].nest->loops.size() >= 4) {
+        // tensor-core mode T4: the 6-D contraction pattern of the ccsd executor
+        s.s6 = contraction_sets(s.nests[0]);
+        if (!s.s6.ok)
+            return fail(EATSS_E_UNSUPPORTED, "eatss_select_tiles: tensor mode needs a depth-3 contraction or the "
+                                             "6-D contraction pattern (one reduction loop, 3 + 3 output loops)");
+        s.tensor = s.tensor6 = true;
+        s.esz = e;
+        s.smem_cap = g->max_smem_per_block;
+        const int ls1 = s.nests[0].m.ls1;
+        for (int p = 0; p < s.L; p++) {
+            std::vector<int64_t> dm;
+            if (p == s.s6.k) {
+                dm = {ext[p]};  // the whole reduction stays in TMEM
+            } else if (p == ls1) {
+                for (int64_t v = 4; v <= ext[p]; v += 4) dm.push_back(v);  // 16-byte output rows
+            } else if (p == s.s6.n.front()) {
+                dm = {1};  // one outer N-side index per unit
+            } else if (p == s.s6.n.back()) {
+                for (int64_t v = 16; v <= std::min<int64_t>(256, ext[p]); v += 16) dm.push_back(v);  // UMMA N granules
+            } else {
+                for (int64_t v = 1; v <= ext[p]; v++) dm.push_back(v);
+            }
+            if (dm.empty()) dm.push_back(16);
+            s.dom.push_back(dm);
+        }
+    } else if (o->mode == 2) {
         // tensor-core mode: depth-3 nests with one serial loop and a parallel l_s1 only
         for (const NestEval &ne : s.nests) {
             int serial = 0;
@@ -366,12 +444,14 @@ extern "C" eatss_status eatss_select_tiles(const eatss_kernel_desc *d, const eat
             s.dom.push_back(dm);
         }
     }
-    // objective-free positions: H == 0 and outside the B-set in every nest
+    // objective-free positions: H == 0 and outside the B-set in every nest; T4: outside
+    // the CTA tile, i.e. the reduction loop
     for (int p = 0; p < s.L; p++) {
         bool fr = true;
         for (const NestEval &ne : s.nests) {
             if (p >= (int)ne.nest->loops.size()) continue;
-            if (ne.m.H[p] != 0 || ((ne.m.bset >> p) & 1u)) fr = false;
+            const bool in_b = s.tensor6 ? p != s.s6.k : ((ne.m.bset >> p) & 1u) != 0;
+            if (ne.m.H[p] != 0 || in_b) fr = false;
         }
         if (fr) s.free_mask |= 1u << p;
     }

@@ -268,15 +268,34 @@ def test_ccsd_tc_rejects_non_mma_tiles(cuda_device):
         assert ei.value.status == -5
 
 
-CCSD_TC_TILE48 = (1, 2, 1, 48, 2, 48, 48)  # the tile bench-style timings use at dims 48
+CCSD_TC_TILE48 = (1, 2, 1, 48, 2, 48, 48)  # round 1's hand-set MMA-legal tile
 
 
-def test_ccsd_tc_full_size_dims48_sampled(cuda_device):
+def test_ccsd_tc_model_tiles_run_exact(cuda_device):
+    """Reading T4 (tensor mode of eatss_select_tiles for the 6-D contraction) picks executable tiles:
+    small-integer inputs give the oracle's exact result at several shapes."""
+    gpu = E.gpu_params_query(0)
+    for dims in [(16,) * 7, (3, 5, 6, 20, 7, 12, 20), (2, 3, 4, 32, 4, 8, 48), (24,) * 7]:
+        H3, H2, H1, P6, P5, P4, H7 = dims
+        d = E.desc_builtin("ccsd_t_d1", dims); d.set_exec(50, TENSOR)
+        tiles, _ = E.select_tiles(d, gpu, 50, 4, mode=2)
+        t3i = synth.small_int((H3, H2, H1, P6, P5, P4), 113)
+        t2i = synth.small_int((H7, P4, P5, H1), 114); v2i = synth.small_int((H3, H2, P6, H7), 115)
+        t3d = dev(t3i)
+        E.run(d, tiles, [t3d, dev(t2i), dev(v2i)])
+        assert np.array_equal(host(t3d), O.ccsd_t_d1(t3i, t2i, v2i)), (dims, tiles)
+
+
+@pytest.mark.parametrize("source", ["model", "hand"])
+def test_ccsd_tc_full_size_dims48_sampled(cuda_device, source):
     n = 48
     d = E.desc_builtin("ccsd_t_d1", (n,)); d.set_exec(50, TENSOR)
+    tiles = E.select_tiles(d, E.gpu_params_query(0), 50, 4, mode=2)[0] if source == "model" else CCSD_TC_TILE48
+    if source == "model":
+        assert tiles == (1, 2, 2, 48, 1, 48, 48)  # tests/test_oracle_model.py::test_tensor_mode_6d_hand_checked
     t2 = synth.uniform((n, n, n, n), 110); v2 = synth.uniform((n, n, n, n), 111)
     t3d = torch.zeros(n ** 6, dtype=torch.float32, device="cuda")
-    E.run(d, CCSD_TC_TILE48, [t3d, dev(t2), dev(v2)])
+    E.run(d, tiles, [t3d, dev(t2), dev(v2)])
     g = synth.rng(112)
     idx = np.concatenate([g.integers(0, n ** 6, 100000), np.arange(n ** 4) + 7 * n ** 5 + 3 * n ** 4])
     got = t3d[torch.from_numpy(idx).cuda()].double().cpu().numpy()
