@@ -11,9 +11,12 @@ execute the tiled gemm N=4000 in libeatss.so.  Two EATSS modes are measured:
   * simt: the paper's formulation in B200 mode picks (16,1024,16), executed by the SIMT
     contraction executor (the paper's code class) -- reported under "simt".
 Metric (BASELINE.json): TFLOP/s and GFLOP/s per Watt.  For N > 1 (torchrun, one
-process per GPU, NCCL) every rank runs its own N=4000 problem (weak scaling, no
+process per GPU, NCCL) every rank runs its own N=4000 problem for the headline (weak scaling, no
 data-path collective); timing is the max over ranks of the device-timed region,
-energy the sum over ranks.  Prints ONE JSON line on rank 0.
+energy the sum over ranks.  At N > 1 the line also carries configs.sharded: BASELINE configs 3
+(2mm, 3mm with its all_gather of F, syrk at N=4000) and 5 (ccsd_t_d1 dims 48, h3 slabs) split over
+the N ranks (harness/sharded.py: max-over-ranks time, summed energy, speedup over rank 0 alone,
+bit-equality on exact inputs).  Prints ONE JSON line on rank 0.
 """
 from __future__ import annotations
 
@@ -49,6 +52,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-secondary", action="store_true")
     ap.add_argument("--no-configs", action="store_true", help="skip the per-config table (BASELINE configs 3-5)")
+    ap.add_argument("--sharded", choices=["auto", "on", "off"], default="auto",
+                    help="BASELINE configs 3 and 5 sharded over the N ranks (SURVEY §8(e)); auto = when N > 1")
     return ap.parse_args()
 
 
@@ -421,6 +426,12 @@ def main():
     configs = None
     if not args.no_configs and rank == 0:
         configs = other_configs(E, torch, gpu, stream, measured_peaks())
+    sharded = None
+    if args.sharded == "on" or (args.sharded == "auto" and ws > 1):
+        # configs 3 and 5 split over the ranks (row blocks / h3 slabs, 3mm's all_gather of F over NCCL):
+        # time (max over ranks), energy (sum), speedup vs the same problem on rank 0 alone, bit-equality
+        from harness.sharded import sharded_configs
+        sharded = sharded_configs(E, torch, dist, rank, ws, dev, gpu)
 
     # e2e through the C ABI with HOST buffers (eatss_run_host): every step copies A, B, C host->device
     # and C device->host inside the timed region; gemm row blocks pipeline the copies with the compute
@@ -534,6 +545,8 @@ def main():
             out["secondary"] = sec
         if configs:
             out["configs"] = configs
+        if sharded:
+            out.setdefault("configs", {})["sharded"] = sharded
         if not args.no_cpu_baseline:
             rec, rows, ref_rows = cpu_oracle_sample()
             out["cpu_baseline"] = rec

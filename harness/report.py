@@ -71,26 +71,34 @@ def summarise(path):
     if d:
         out["share_beating_default_perf"] = float(np.mean([r["tflops"] > d["tflops_median"] for r in ok]))
         out["share_beating_default_ppw"] = float(np.mean([r["gflops_per_watt"] > d["ppw_median"] for r in ok]))
-    # drift correction: scale each variant's PPW / TFLOP/s by the EATSS anchor interpolated
-    # at its measurement time (DVFS / thermal drift over the ~50 min sweep)
-    ae = sorted([r for r in anc["anchor_eatss"] if r.get("status") == 0 and (r.get("joules") or 0) > 0],
-                key=lambda r: r["t"])
-    if len(ae) >= 2:
-        ts = np.array([r["t"] for r in ae])
-        pp = np.array([r["gflops_per_watt"] for r in ae])
-        tf = np.array([r["tflops"] for r in ae])
-        p_med, t_med = float(np.median(pp)), float(np.median(tf))
-        for r in ok:
+    # drift correction: scale each variant's PPW / TFLOP/s by the EATSS anchor interpolated at its
+    # measurement time (DVFS / thermal drift over the ~50 min sweep) -- on the variant's OWN GPU when the
+    # sweep ran on several (per-GPU anchor normalisation: GPUs differ in clocks, power and drift)
+    ae_all = [r for r in anc["anchor_eatss"] if r.get("status") == 0 and (r.get("joules") or 0) > 0]
+    ranks = sorted({r.get("rank", 0) for r in ae_all})
+    per_rank = {}
+    for rk in ranks:
+        ae = sorted([r for r in ae_all if r.get("rank", 0) == rk], key=lambda r: r["t"])
+        if len(ae) >= 2:
+            per_rank[rk] = (np.array([r["t"] for r in ae]), np.array([r["gflops_per_watt"] for r in ae]),
+                            np.array([r["tflops"] for r in ae]))
+    if per_rank:
+        p_med = float(np.median([r["gflops_per_watt"] for r in ae_all]))
+        t_med = float(np.median([r["tflops"] for r in ae_all]))
+        corr = [r for r in ok if r.get("rank", 0) in per_rank]
+        for r in corr:
+            ts, pp, tf = per_rank[r.get("rank", 0)]
             r["ppw_drift_corr"] = r["gflops_per_watt"] * p_med / float(np.interp(r["t"], ts, pp))
             r["tflops_drift_corr"] = r["tflops"] * t_med / float(np.interp(r["t"], ts, tf))
-        perf_c = max(ok, key=lambda r: r["tflops_drift_corr"])
-        ener_c = max(ok, key=lambda r: r["ppw_drift_corr"])
+        perf_c = max(corr, key=lambda r: r["tflops_drift_corr"])
+        ener_c = max(corr, key=lambda r: r["ppw_drift_corr"])
         out["drift_corrected"] = {
+            "per_gpu_anchors": {str(k): int(len(v[0])) for k, v in per_rank.items()},
             "perf_optimal": {"tile": perf_c["tile"], "tflops": perf_c["tflops_drift_corr"], "ppw": perf_c["ppw_drift_corr"]},
             "energy_optimal": {"tile": ener_c["tile"], "tflops": ener_c["tflops_drift_corr"], "ppw": ener_c["ppw_drift_corr"]},
             "ppw_gain": ener_c["ppw_drift_corr"] / perf_c["ppw_drift_corr"],
-            "top10_ppw": [r["tile"] for r in sorted(ok, key=lambda r: -r["ppw_drift_corr"])[:10]],
-            "top10_perf": [r["tile"] for r in sorted(ok, key=lambda r: -r["tflops_drift_corr"])[:10]],
+            "top10_ppw": [r["tile"] for r in sorted(corr, key=lambda r: -r["ppw_drift_corr"])[:10]],
+            "top10_perf": [r["tile"] for r in sorted(corr, key=lambda r: -r["tflops_drift_corr"])[:10]],
         }
     out["top5_ppw"] = [{"tile": r["tile"], "gflops_per_watt": r["gflops_per_watt"], "tflops": r["tflops"],
                         "watts": r["watts"]} for r in ppw[:5]]

@@ -53,7 +53,42 @@ def parse():
     ap.add_argument("--no-parity", action="store_true")
     ap.add_argument("--tiles", default="", help="confirmation mode: 'a,b,c;d,e,f' measured --repeats times, interleaved")
     ap.add_argument("--repeats", type=int, default=5)
+    ap.add_argument("--dtype", choices=["f32", "f64"], default="f32",
+                    help="f64: the paper's precision (P:117 FP_factor 2, P:202): model and executor in fp64")
     return ap.parse_args()
+
+
+REC_FIELDS = ["ms", "joules", "watts", "tflops", "gflops_per_watt", "sm_mhz", "runs", "status", "t"]
+REC_KINDS = {"variant": 0, "anchor_default": 1, "anchor_eatss": 2, "confirm": 3}
+
+
+def gather_records(recs, rank, ws, dist, torch, device):
+    """All ranks' sweep records on rank 0 (list of dicts; [] elsewhere): fixed-size float64 rows
+    (kind, tile[3], exact, REC_FIELDS incl. the wall-clock time t) padded to the longest rank and
+    gathered with all_gather_into_tensor -- the per-rank timestamps let harness/report.py normalise
+    each variant by ITS GPU's interpolated EATSS anchor (GPUs differ in clocks, power and drift)."""
+    rows = [[REC_KINDS[r["kind"]], *r["tile"], float(r.get("exact", 1)),
+             *[float(r.get(f, -1) if r.get(f) is not None else -1) for f in REC_FIELDS]] for r in recs]
+    width = 5 + len(REC_FIELDS)
+    cnt = torch.tensor([len(rows)], device=device)
+    dist.all_reduce(cnt, op=dist.ReduceOp.MAX)
+    buf = torch.full((int(cnt.item()), width), float("nan"), dtype=torch.float64, device=device)
+    if rows:
+        buf[: len(rows)] = torch.tensor(rows, dtype=torch.float64, device=device)
+    allb = torch.empty((ws * buf.shape[0], width), dtype=torch.float64, device=device)  # rank blocks, concatenated
+    dist.all_gather_into_tensor(allb, buf)
+    out = []
+    if rank == 0:
+        inv = {v: k for k, v in REC_KINDS.items()}
+        for rr, block in enumerate(allb.reshape(ws, buf.shape[0], width).cpu().numpy()):
+            for x in block:
+                if np.isnan(x[0]):
+                    continue
+                r = {"kind": inv[int(x[0])], "tile": [int(v) for v in x[1:4]], "exact": bool(x[4]), "rank": rr}
+                r.update({f: float(v) for f, v in zip(REC_FIELDS, x[5:])})
+                r["status"] = int(r["status"])
+                out.append(r)
+    return out
 
 
 def nvml_interval_ms(E, device, seconds=1.0):
@@ -93,9 +128,11 @@ def main():
 
     n = a.n
     assert a.kind == "gemm", "the sweep driver covers the gemm nest (config 2)"
-    d = E.desc_builtin("gemm", (n, n, n))
+    d = E.desc_builtin("gemm", (n, n, n), a.dtype)
     d.set_exec(split_pct=a.split)
     gpu = E.gpu_params_query(local)
+    tdt = torch.float64 if a.dtype == "f64" else torch.float32
+    ndt = np.float64 if a.dtype == "f64" else np.float32
     eatss_tile, rep = E.select_tiles(d, gpu, a.split, 16)
     default_tile = (32, 32, 32)
     sizes = [int(x) for x in a.sizes.split(",")]
@@ -112,23 +149,24 @@ def main():
     mine = [v for i, v in enumerate(variants) if i % ws == rank and v not in done]
 
     # inputs: U(0..2) for energy/speed (data-dependent power), I(1..3) for exact parity
-    A = torch.from_numpy(synth.uniform((n, n), 0)).to(dev)
-    B = torch.from_numpy(synth.uniform((n, n), 1)).to(dev)
-    C = torch.from_numpy(synth.uniform((n, n), 2)).to(dev)
-    Ai_h = synth.small_int((n, n), 1); Bi_h = synth.small_int((n, n), 2); Ci_h = synth.small_int((n, n), 3)
+    A = torch.from_numpy(synth.uniform((n, n), 0, dtype=ndt)).to(dev)
+    B = torch.from_numpy(synth.uniform((n, n), 1, dtype=ndt)).to(dev)
+    C = torch.from_numpy(synth.uniform((n, n), 2, dtype=ndt)).to(dev)
+    Ai_h = synth.small_int((n, n), 1, dtype=ndt); Bi_h = synth.small_int((n, n), 2, dtype=ndt)
+    Ci_h = synth.small_int((n, n), 3, dtype=ndt)
     Ai, Bi = torch.from_numpy(Ai_h).to(dev), torch.from_numpy(Bi_h).to(dev)
     g = synth.rng(7)
     ii = g.integers(0, n, 512); jj = g.integers(0, n, 512)
     ref = O.gemm_entries(ii, jj, Ci_h, Ai_h, Bi_h, 1.0, 1.0) if not a.no_parity else None
     iit, jjt = torch.from_numpy(ii).to(dev), torch.from_numpy(jj).to(dev)
-    dpar = E.desc_builtin("gemm", (n, n, n)); dpar.set_scalars(1.0, 1.0); dpar.set_exec(split_pct=a.split)
+    dpar = E.desc_builtin("gemm", (n, n, n), a.dtype); dpar.set_scalars(1.0, 1.0); dpar.set_exec(split_pct=a.split)
 
     os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
     out = open(a.out if ws == 1 else a.out.replace(".jsonl", f".rank{rank}.jsonl"), "a")
     interval = nvml_interval_ms(E, local) if rank == 0 or ws > 1 else None
     meta = {"kind": "meta", "rank": rank, "world": ws, "n": n, "split_pct": a.split, "eatss_tile": list(eatss_tile),
             "default_tile": list(default_tile), "variants_total": len(variants), "variants_mine": len(mine),
-            "window_s": a.window, "nvml_update_ms": interval, "sizes": sizes,
+            "window_s": a.window, "nvml_update_ms": interval, "sizes": sizes, "dtype": a.dtype,
             "gpu": torch.cuda.get_device_name(local), "time": time.time()}
     out.write(json.dumps(meta) + "\n"); out.flush()
 
@@ -179,28 +217,12 @@ def main():
         # gather fixed-size records to rank 0 over NCCL (the only collective of the sweep)
         mine_path = a.out.replace(".jsonl", f".rank{rank}.jsonl")
         recs = [json.loads(l) for l in open(mine_path) if '"kind": "meta"' not in l]
-        F = ["ms", "joules", "watts", "tflops", "gflops_per_watt", "sm_mhz", "runs", "status"]
-        KIND = {"variant": 0, "anchor_default": 1, "anchor_eatss": 2}
-        rows = [[KIND[r["kind"]], *r["tile"], float(r.get("exact", 1)), *[float(r.get(f, -1) or -1) for f in F]]
-                for r in recs]
-        cnt = torch.tensor([len(rows)], device=dev)
-        dist.all_reduce(cnt, op=dist.ReduceOp.MAX)
-        buf = torch.full((int(cnt.item()), 5 + len(F)), float("nan"), dtype=torch.float64, device=dev)
-        if rows:
-            buf[: len(rows)] = torch.tensor(rows, dtype=torch.float64, device=dev)
-        allb = torch.empty((ws,) + tuple(buf.shape), dtype=torch.float64, device=dev)
-        dist.all_gather_into_tensor(allb, buf)
+        allrecs = gather_records(recs, rank, ws, dist, torch, dev)
         if rank == 0:
-            inv = {v: k for k, v in KIND.items()}
             with open(a.out, "a") as fo:
                 fo.write(json.dumps(dict(meta, rank="all", world=ws)) + "\n")
-                for rr, row in enumerate(allb.cpu().numpy()):
-                    for x in row:
-                        if np.isnan(x[0]):
-                            continue
-                        r = {"kind": inv[int(x[0])], "tile": [int(v) for v in x[1:4]], "exact": bool(x[4]), "rank": rr}
-                        r.update({f: float(v) for f, v in zip(F, x[5:])})
-                        fo.write(json.dumps(r) + "\n")
+                for r in allrecs:
+                    fo.write(json.dumps(r) + "\n")
         dist.barrier()
         dist.destroy_process_group()
     if rank == 0:

@@ -133,3 +133,84 @@ def test_gloo_world2_shards_equal_single_process(kind, dims, tiles):
     if kind == "3mm":  # every rank holds the full gathered F after the exchange
         for _, p in res:
             assert np.array_equal(np.asarray(p["F"]), O.three_mm(X["A"], X["B"], X["C"], X["D"])[1])
+
+
+# ------------------------------------------------------------------ the sweep's record gather
+def _fake_records(rank):
+    """Rank r's sweep records: its GPU runs 10% faster per rank (different clocks) and drifts down in
+    time; the EATSS anchors see the same drift -- per-GPU anchor normalisation must undo both."""
+    g = np.random.default_rng(rank)
+    scale = 1.0 + 0.1 * rank
+    recs = []
+    for k in range(12):
+        t = 1000.0 + 10.0 * k + rank
+        drift = 1.0 - 0.01 * k
+        anchor = k % 4 == 0 or k == 11  # anchors bracket every variant (interpolation, not extrapolation)
+        tile = [16, 1024, 16] if anchor else [int(x) for x in g.choice([16, 32, 64], 3)]
+        kind = "anchor_eatss" if anchor else "variant"
+        base = 50.0 if kind == "anchor_eatss" else 40.0 + tile[0] / 8
+        ppw = base * scale * drift
+        recs.append({"kind": kind, "tile": tile, "exact": True, "ms": 1.0, "joules": 1.0 / ppw, "watts": 500.0,
+                     "tflops": ppw * 0.5, "gflops_per_watt": ppw, "sm_mhz": 1800.0, "runs": 10, "status": 0, "t": t})
+    return recs
+
+
+def _gather_worker(rank, world, port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from harness import sweep as SW
+    out = SW.gather_records(_fake_records(rank), rank, world, dist, torch, torch.device("cpu"))
+    if rank == 0:
+        q.put(out)
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_gloo_world2_sweep_gather_keeps_rank_and_time(tmp_path):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_gather_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    got = q.get(timeout=300)
+    for p in ps:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert len(got) == 24
+    for rank in (0, 1):
+        mine = [r for r in got if r["rank"] == rank]
+        want = _fake_records(rank)
+        assert [(r["kind"], r["tile"], r["t"]) for r in mine] == [(w["kind"], w["tile"], w["t"]) for w in want]
+        assert all(abs(r["gflops_per_watt"] - w["gflops_per_watt"]) < 1e-9 for r, w in zip(mine, want))
+    # per-GPU anchor normalisation: after correction a variant's PPW no longer depends on its GPU or time
+    sys.path.insert(0, os.path.join(ROOT, "harness"))
+    import report
+    path = tmp_path / "gathered.jsonl"
+    with open(path, "w") as f:
+        f.write('{"kind": "meta", "eatss_tile": [16, 1024, 16], "nvml_update_ms": 100.0}\n')
+        for r in got:
+            f.write(__import__("json").dumps(r) + "\n")
+    s = report.summarise(str(path))
+    assert s["drift_corrected"]["per_gpu_anchors"] == {"0": 4, "1": 4}
+    meta, var, anc = report.load(str(path))
+    ok = [r for r in var]
+    corr = {}
+    for r in ok:
+        # reproduce the normalisation for the check: variant PPW / its rank's interpolated anchor
+        an = sorted([a for a in anc["anchor_eatss"] if a["rank"] == r["rank"]], key=lambda a: a["t"])
+        v = r["gflops_per_watt"] / np.interp(r["t"], [a["t"] for a in an], [a["gflops_per_watt"] for a in an])
+        corr.setdefault(r["tile"][0], set()).add(round(v, 6))
+    # same tile[0] -> same base PPW on both GPUs -> identical normalised value
+    assert all(len(v) == 1 for v in corr.values()), corr
+
+
+def test_sharded_checksums_compare_row_blocks():
+    from harness import sharded as SH
+    full = torch.arange(6 * 5, dtype=torch.float32).reshape(6, 5) * 0.5
+    a = SH.checksums(torch, full, (2, 4))
+    assert a == SH.checksums(torch, full[2:4].clone())
+    bad = full[2:4].clone()
+    bad[1, 3] = torch.nextafter(bad[1, 3], torch.tensor(1e9))  # one ulp off
+    assert SH.checksums(torch, bad) != a
