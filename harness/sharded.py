@@ -26,14 +26,20 @@ CONFIGS = (("2mm", 4000), ("3mm", 4000), ("syrk", 4000), ("ccsd_t_d1", 48))
 OUT_KEYS = {"2mm": ("tmp", "D"), "3mm": ("E", "G"), "syrk": ("C",), "ccsd_t_d1": ("t3",)}
 
 
-def checksums(torch, t, rows=None):
-    """(sum of the fp32 bit patterns, index-weighted sum) over the rows [r0, r1) of t (int64, wraps)."""
+def checksums(torch, t, rows=None, chunk=1 << 26):
+    """(sum of the fp32 bit patterns, index-weighted sum) over the rows [r0, r1) of t: int64 arithmetic
+    in chunks (the ccsd output is 12G elements), wrapping identically on every rank."""
     x = t.reshape(t.shape[0], -1)
     if rows is not None:
         x = x[rows[0]:rows[1]]
-    b = x.contiguous().view(torch.int32).to(torch.int64).reshape(-1)
-    idx = torch.arange(1, b.numel() + 1, device=b.device, dtype=torch.int64)
-    return int(b.sum().item()), int((b * idx).sum().item())
+    flat = x.reshape(-1)
+    s1 = s2 = 0
+    for c0 in range(0, flat.numel(), chunk):
+        b = flat[c0:c0 + chunk].contiguous().view(torch.int32).to(torch.int64)
+        idx = torch.arange(c0 + 1, c0 + 1 + b.numel(), device=b.device, dtype=torch.int64)
+        s1 += int(b.sum().item())
+        s2 += int((b * idx).sum().item())
+    return s1 & (2 ** 64 - 1), s2 & (2 ** 64 - 1)
 
 
 def _inputs(kind, dims, torch, dev, small_int, seed):

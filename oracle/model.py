@@ -533,7 +533,8 @@ def _evaluate_tensor_6d(prog: Program, gpu: Gpu, opts: Opts, T):
     buffer (N rounded up to a power of two >= 32) next to the 128 columns of the A operand; shared memory:
     three epilogue groups' output tiles (M*N*e rounded to 1 KB) + two stages of the N-side operand (hi, lo;
     k in 32-element atoms) <= max_smem_per_block - 1536.  B (the parallelism term) = M * N, the output
-    tile of one CTA (on the tensor core every parallel loop maps into it; for depth 3 it equals Ti*Tj)."""
+    tile of one CTA (on the tensor core every parallel loop maps into it; for depth 3 it equals Ti*Tj).
+    T4-H: the H weights count only the references streamed per unit (see below)."""
     e = prog.dtype_bytes
     nest = prog.nests[0]
     d = derive(nest, opts.waf)
@@ -552,10 +553,16 @@ def _evaluate_tensor_6d(prog: Program, gpu: Gpu, opts: Opts, T):
     x_stage = -(-(M * N * e) // 1024) * 1024
     v_stage = 2 * (-(-kext // 32)) * N * 128
     feas &= 3 * x_stage + 2 * v_stage <= gpu.max_smem_per_block - 1536
+    # T4-H: the M-side operand is resident in TMEM across every unit of its tile (read from HBM once
+    # per A tile), so only the streamed references -- the output and the N-side operand -- earn the
+    # stride-1 (CMA) weight of Eq. 2: H is derived on the nest without the M-side operand
+    written = {r.array for r in nest.refs if r.write}
+    x_arr = next(r.array for r in d.refs if r.array not in written and set(mset) <= set(r.iters()))
+    Hs = derive(Nest(nest.loops, [r for r in nest.refs if r.array != x_arr]), opts.waf).H
     obj = M * N
     for l in nest.loops:
-        if d.H[l.name]:
-            obj = obj + d.H[l.name] * T[pos[l.name]]
+        if Hs[l.name]:
+            obj = obj + Hs[l.name] * T[pos[l.name]]
     return feas, obj
 
 

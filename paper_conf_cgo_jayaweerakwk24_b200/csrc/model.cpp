@@ -183,8 +183,9 @@ struct Sets6 {
     bool ok = false;
     std::vector<int> m, n;  // loop positions, outermost first
     int k = -1;
+    std::vector<int64_t> H;  // T4-H: Eq. 2 weights without the M-side (TMEM-resident) operand
 };
-Sets6 contraction_sets(const NestEval &ne) {
+Sets6 contraction_sets(const NestEval &ne, int waf) {
     Sets6 r;
     const Nest &n = *ne.nest;
     const int L = (int)n.loops.size();
@@ -202,6 +203,19 @@ Sets6 contraction_sets(const NestEval &ne) {
         if ((y >> p) & 1u) r.n.push_back(p);
     }
     r.ok = r.m.size() == 3 && r.n.size() == 3;
+    // T4-H: the M-side operand stays in TMEM across all units of its tile (read once per A tile), so only
+    // the streamed references (output, N-side operand) earn the stride-1 weight: H of the nest without it
+    int x_array = -1;
+    for (const Ref &rf : n.refs) {
+        uint32_t it = 0;
+        for (const Sub &sb : rf.subs) it |= sb.iters;
+        if (!rf.write && it == x) x_array = rf.array;
+    }
+    Nest reduced;
+    reduced.loops = n.loops;
+    for (const Ref &rf : n.refs)
+        if (rf.array != x_array) reduced.refs.push_back(rf);
+    r.H = derive_nest(reduced, waf).H;
     return r;
 }
 constexpr int64_t kTmemCols = 512;
@@ -293,9 +307,10 @@ struct Search {
                 for (int p : s6.m) M *= T[p];
                 for (int p : s6.n) N *= T[p];
                 obj += M * N;
-            } else {
-                obj += prod(T, ne.m.bset);
+                for (size_t p = 0; p < s6.H.size(); p++) obj += s6.H[p] * T[p];
+                continue;
             }
+            obj += prod(T, ne.m.bset);
             for (size_t p = 0; p < ne.m.H.size(); p++) obj += ne.m.H[p] * T[p];
         }
         return obj;
@@ -386,7 +401,7 @@ extern "C" eatss_status eatss_select_tiles(const eatss_kernel_desc *d, const eat
     s.ext = ext;
     if (o->mode == 2 && s.nests.size() == 1 && s.nests[0].nest->loops.size() >= 4) {
         // tensor-core mode T4: the 6-D contraction pattern of the ccsd executor
-        s.s6 = contraction_sets(s.nests[0]);
+        s.s6 = contraction_sets(s.nests[0], o->warp_align);
         if (!s.s6.ok)
             return fail(EATSS_E_UNSUPPORTED, "eatss_select_tiles: tensor mode needs a depth-3 contraction or the "
                                              "6-D contraction pattern (one reduction loop, 3 + 3 output loops)");
@@ -451,7 +466,8 @@ extern "C" eatss_status eatss_select_tiles(const eatss_kernel_desc *d, const eat
         for (const NestEval &ne : s.nests) {
             if (p >= (int)ne.nest->loops.size()) continue;
             const bool in_b = s.tensor6 ? p != s.s6.k : ((ne.m.bset >> p) & 1u) != 0;
-            if (ne.m.H[p] != 0 || in_b) fr = false;
+            const int64_t h = s.tensor6 ? s.s6.H[p] : ne.m.H[p];
+            if (h != 0 || in_b) fr = false;
         }
         if (fr) s.free_mask |= 1u << p;
     }
