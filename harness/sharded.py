@@ -11,7 +11,9 @@ h3 slabs).  Per config it reports:
   * bit_equal: small-integer inputs (every partial sum exact in fp32 and on the 3xTF32 path: the
     result does not depend on the summation order or the partition), each rank's output rows/slabs
     against rank 0's single-GPU result, compared by 64-bit checksums of the raw fp32 bits per shard;
-  * rel_err: U[-1,1) inputs, the gathered normwise error of the sharded result against the 1-GPU one.
+  * rel_err_vs_1gpu: U[-1,1) inputs (alpha 1.5, beta 1.2), the normwise difference of 4096 sampled
+    entries per rank and output against the 1-GPU result (not 0 even at N = 1: the split-k tail adds its
+    partial sums with atomics, in no fixed order).
 The host logic (partition, exchange, checksum comparison) runs under gloo in tests/test_multigpu_cpu.py.
 """
 from __future__ import annotations
@@ -84,12 +86,34 @@ def run_config(kind, n, E, torch, dist, rank, ws, dev, gpu, steps=3, window_s=1.
             ms = v.item()
         return ms
 
-    # --- U[-1,1): timing, energy, 1-GPU reference timing on rank 0, gathered relative error
+    # --- U[-1,1): timing (sharded and, on rank 0 alone, the whole problem -- interleaved, best of 3 so
+    # both see the same thermal / power state), then energy of the sharded run
     Xd = _inputs(kind, dims, torch, dev, False, 0)
-    X0 = {k: v.clone() for k, v in Xd.items() if k != "t3"}
     shard = lambda: MG.run_shard(kind, dims, tiles, rank, ws, Xd, be)  # noqa: E731
-    out["ms"] = timed(shard, steps)
-    # energy: repeated sharded runs over >= window_s, NVML counter per rank, summed
+    one = lambda: MG.run_shard(kind, dims, tiles, 0, 1, Xd, be1)  # noqa: E731
+
+    def timed_one():
+        ms1 = 0.0
+        if rank == 0:
+            one(); torch.cuda.synchronize()
+            s, e = ev(), ev()
+            s.record()
+            for _ in range(steps):
+                one()
+            e.record(); torch.cuda.synchronize()
+            ms1 = s.elapsed_time(e) / steps
+        if ws > 1:
+            dist.barrier()
+        v = torch.tensor([ms1], dtype=torch.float64, device=dev)
+        if ws > 1:
+            dist.broadcast(v, 0)
+        return v.item()
+
+    t_sh, t_1 = [], []
+    for _ in range(3):
+        t_sh.append(timed(shard, steps))
+        t_1.append(timed_one())
+    out["ms"], out["ms_1gpu"] = min(t_sh), min(t_1)
     torch.cuda.synchronize()
     if ws > 1:
         dist.barrier()
@@ -104,31 +128,17 @@ def run_config(kind, n, E, torch, dist, rank, ws, dev, gpu, steps=3, window_s=1.
     out["joules"] = j.item()
     out["tflops"] = d_full.flops / (out["ms"] * 1e-3) / 1e12
     out["gflops_per_watt"] = d_full.flops / out["joules"] / 1e9 if out["joules"] > 0 else None
-    # 1-GPU reference: rank 0 runs the whole problem (world 1 partition) while the others wait
-    _reset(kind, Xd, X0)
-    ms1 = None
-    if rank == 0:
-        one = lambda: MG.run_shard(kind, dims, tiles, 0, 1, Xd, be1)  # noqa: E731
-        one(); torch.cuda.synchronize()
-        s, e = ev(), ev()
-        s.record()
-        for _ in range(steps):
-            one()
-        e.record(); torch.cuda.synchronize()
-        ms1 = s.elapsed_time(e) / steps
-    if ws > 1:
-        dist.barrier()
-    v = torch.tensor([ms1 or 0.0], dtype=torch.float64, device=dev)
-    if ws > 1:
-        dist.broadcast(v, 0)
-    out["ms_1gpu"] = v.item()
     out["speedup"] = out["ms_1gpu"] / out["ms"]
     out["efficiency"] = out["speedup"] / ws
+    del Xd
     # --- bit-equality on small integers, and the U[-1,1) error, shard vs 1-GPU result
     for small in (True, False):
         Xd = _inputs(kind, dims, torch, dev, small, 11)
         X0 = {k: v.clone() for k, v in Xd.items() if k != "t3"}
-        res, rr = MG.run_shard(kind, dims, tiles, rank, ws, Xd, be)
+        # exact pass: exactly representable scalars (alpha = beta = 1), so every value is an integer
+        # below 2^24 and the result cannot depend on the order of the (split-k atomic) partial sums
+        ab = dict(alpha=1.0, beta=1.0) if small else {}
+        res, rr = MG.run_shard(kind, dims, tiles, rank, ws, Xd, be, **ab)
         torch.cuda.synchronize()
         r0, r1 = rr
         if small:  # checksums of this rank's rows / slabs, taken before the buffers are reused
@@ -143,7 +153,7 @@ def run_config(kind, n, E, torch, dist, rank, ws, dev, gpu, steps=3, window_s=1.
                 samp[k] = (i + r0 * per_row, x[i].double() if x.numel() else torch.zeros(4096, device=dev,
                                                                                             dtype=torch.float64))
         _reset(kind, Xd, X0)
-        ref = MG.run_shard(kind, dims, tiles, 0, 1, Xd, be1)[0] if rank == 0 else None
+        ref = MG.run_shard(kind, dims, tiles, 0, 1, Xd, be1, **ab)[0] if rank == 0 else None
         torch.cuda.synchronize()
         if small:
             gathered = [None] * ws
