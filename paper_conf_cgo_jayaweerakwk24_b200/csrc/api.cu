@@ -28,13 +28,14 @@ static eatss_status cuda_fail(cudaError_t e, const char *where) {
 
 // stencil.cu / ccsd.cu entry points
 cudaError_t launch_jacobi2d_sweep(void *dst, const void *src, const void *bsrc, int64_t n, int64_t Ti,
-                                  int64_t Tj, bool f64, int carveout, int32_t *counts, cudaStream_t s);
+                                  int64_t Tj, bool f64, int carveout, int32_t *counts, cudaStream_t s, int waf);
 cudaError_t launch_interior_copy2d(void *dst, const void *src, int64_t n, bool f64, cudaStream_t s);
 // stencil_untiled.cu: the untiled baseline (engine EATSS_ENGINE_UNTILED; tile vector ignored)
 cudaError_t launch_jacobi2d_untiled(void *dst, const void *src, const void *bsrc, int64_t n, bool f64, cudaStream_t s);
 cudaError_t launch_heat3d_untiled(void *dst, const void *src, int64_t n, bool f64, cudaStream_t s);
 cudaError_t launch_heat3d_sweep(void *dst, const void *src, int64_t n, int64_t Ti, int64_t Tj,
-                                int64_t Tk, bool f64, int carveout, int32_t *counts, cudaStream_t s);
+                                int64_t Tk, bool f64, int carveout, int32_t *counts, cudaStream_t s, int waf);
+int stencil_simt_x(bool heat, int64_t n, const int64_t *t, bool f64, int waf);
 void stencil_plan_dims(bool heat, int64_t n, const int64_t *t, bool f64, int64_t *gx, int64_t *gy,
                        int *bx, int *by, int *vec);
 cudaError_t launch_ccsd_d1(float *t3, const float *t2, const float *v2, const int64_t *dims,
@@ -422,7 +423,7 @@ static cudaError_t stencil_issue(const eatss_kernel_desc *d, const int64_t *t, v
         for (int64_t step = 0; step < d->tsteps && e == cudaSuccess; step++) {
             void *dst = step % 2 == 0 ? B : A, *src = step % 2 == 0 ? A : B;
             e = untiled ? launch_jacobi2d_untiled(dst, src, A, n, f64, s)
-                        : launch_jacobi2d_sweep(dst, src, A, n, t[0], t[1], f64, cv, nullptr, s);
+                        : launch_jacobi2d_sweep(dst, src, A, n, t[0], t[1], f64, cv, nullptr, s, d->exec.warp_align);
         }
         if (e == cudaSuccess && d->tsteps > 0) {
             // the literal copy nest of the last step (both interiors end equal to X_T)
@@ -433,10 +434,10 @@ static cudaError_t stencil_issue(const eatss_kernel_desc *d, const int64_t *t, v
         void *A = b[0], *B = b[1];
         for (int64_t step = 0; step < d->tsteps && e == cudaSuccess; step++) {
             e = untiled ? launch_heat3d_untiled(B, A, n, f64, s)
-                        : launch_heat3d_sweep(B, A, n, t[0], t[1], t[2], f64, cv, nullptr, s);
+                        : launch_heat3d_sweep(B, A, n, t[0], t[1], t[2], f64, cv, nullptr, s, d->exec.warp_align);
             if (e == cudaSuccess)
                 e = untiled ? launch_heat3d_untiled(A, B, n, f64, s)
-                            : launch_heat3d_sweep(A, B, n, t[0], t[1], t[2], f64, cv, nullptr, s);
+                            : launch_heat3d_sweep(A, B, n, t[0], t[1], t[2], f64, cv, nullptr, s, d->exec.warp_align);
         }
     }
     return e;
@@ -454,6 +455,7 @@ static eatss_status stencil_run(eatss_kernel_desc *d, const int64_t *t, void *co
     key.tiles.push_back(d->exec.engine);  // a tiled and an untiled time loop are different graphs
     key.tiles.push_back(d->exec.split_pct);  // the carve-out is captured with each launch
     key.tiles.push_back(d->exec.carveout_exact);
+    key.tiles.push_back(d->exec.warp_align);  // the lane layout is a kernel argument of every captured sweep
     int gdev = 0;
     cudaGetDevice(&gdev);
     key.tiles.push_back(gdev);  // a graph is instantiated for one device
@@ -747,7 +749,7 @@ eatss_status eatss_plan(const eatss_kernel_desc *d, const int64_t *tiles, eatss_
             stencil_plan_dims(d->kind == EATSS_HEAT3D, d->dims[0], t, f64, &o.grid_x, &o.grid_y, &o.block_x,
                               &o.block_y, &o.vec);
             o.grid_z = 1; o.rm = 1; o.rn = o.vec; o.passes = 1; o.carveout_pct = d->exec.split_pct;
-            o.simt_x = std::min(32, o.block_x);
+            o.simt_x = stencil_simt_x(d->kind == EATSS_HEAT3D, d->dims[0], t, f64, d->exec.warp_align);
             for (int p = 0; p < L; p++) o.tile[p] = t[p];
         }
         *n_plans = nn;
@@ -1207,9 +1209,11 @@ eatss_status eatss_coverage(const eatss_kernel_desc *d, int nest, const int64_t 
     const int64_t n = d->dims[0];
     cudaError_t e;
     if (d->kind == EATSS_JACOBI2D)
-        e = launch_jacobi2d_sweep(nullptr, nullptr, nullptr, n, tiles[0], tiles[1], f64, exec_cv(d), counts, s);
+        e = launch_jacobi2d_sweep(nullptr, nullptr, nullptr, n, tiles[0], tiles[1], f64, exec_cv(d), counts, s,
+                                  d->exec.warp_align);
     else if (d->kind == EATSS_HEAT3D)
-        e = launch_heat3d_sweep(nullptr, nullptr, n, tiles[0], tiles[1], tiles[2], f64, exec_cv(d), counts, s);
+        e = launch_heat3d_sweep(nullptr, nullptr, n, tiles[0], tiles[1], tiles[2], f64, exec_cv(d), counts, s,
+                                d->exec.warp_align);
     else
         e = launch_ccsd_d1(nullptr, nullptr, nullptr, d->dims.data(), tiles, 0, d->dims[0], exec_cv(d),
                            counts, s);

@@ -19,6 +19,7 @@
 // heat-3d (PolyBench 4.x) is already a ping-pong (B = f(A); A = f(B)).
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cstdint>
 #include <cstdlib>
 
@@ -247,9 +248,9 @@ __global__ void __launch_bounds__(256) heat3d_sweep(T *__restrict__ dst, const T
 bool jacobi2d_staged_applicable(int64_t n, int64_t Ti, int64_t Tj, bool f64);
 bool heat3d_staged_applicable(int64_t n, int64_t Ti, int64_t Tj, int64_t Tk, bool f64);
 cudaError_t launch_jacobi2d_staged(float *dst, const float *src, const float *bsrc, int64_t n, int64_t Ti, int64_t Tj,
-                                   int split_pct, int32_t *counts, cudaStream_t s);
+                                   int split_pct, int32_t *counts, cudaStream_t s, int waf);
 cudaError_t launch_heat3d_staged(float *dst, const float *src, int64_t n, int64_t Ti, int64_t Tj, int64_t Tk,
-                                 int split_pct, int32_t *counts, cudaStream_t s);
+                                 int split_pct, int32_t *counts, cudaStream_t s, int waf);
 static bool stencil_staged_enabled() {
     static const bool on = !(getenv("EATSS_STENCIL_STAGED") && atoi(getenv("EATSS_STENCIL_STAGED")) == 0);
     return on;
@@ -305,10 +306,10 @@ static void launch_cv(void (*kern)(KArgs...), dim3 grid, dim3 block, int cv, cud
 }
 
 cudaError_t launch_jacobi2d_sweep(void *dst, const void *src, const void *bsrc, int64_t n, int64_t Ti,
-                                  int64_t Tj, bool f64, int carveout, int32_t *counts, cudaStream_t s) {
+                                  int64_t Tj, bool f64, int carveout, int32_t *counts, cudaStream_t s, int waf) {
     if (stencil_staged_enabled() && jacobi2d_staged_applicable(n, Ti, Tj, f64))
         return launch_jacobi2d_staged((float *)dst, (const float *)src, (const float *)bsrc, n, Ti, Tj, carveout,
-                                      counts, s);
+                                      counts, s, waf);
     StencilPlan p = plan_jacobi2d(n, Ti, Tj, f64);
     const int cv = cv_resolve(carveout, 0);
     dim3 grid((unsigned)p.gx, (unsigned)p.gy), block(p.bx, p.by);
@@ -341,9 +342,9 @@ cudaError_t launch_interior_copy2d(void *dst, const void *src, int64_t n, bool f
 }
 
 cudaError_t launch_heat3d_sweep(void *dst, const void *src, int64_t n, int64_t Ti, int64_t Tj,
-                                int64_t Tk, bool f64, int carveout, int32_t *counts, cudaStream_t s) {
+                                int64_t Tk, bool f64, int carveout, int32_t *counts, cudaStream_t s, int waf) {
     if (stencil_staged_enabled() && heat3d_staged_applicable(n, Ti, Tj, Tk, f64))
-        return launch_heat3d_staged((float *)dst, (const float *)src, n, Ti, Tj, Tk, carveout, counts, s);
+        return launch_heat3d_staged((float *)dst, (const float *)src, n, Ti, Tj, Tk, carveout, counts, s, waf);
     StencilPlan p = plan_heat3d(n, Ti, Tj, Tk, f64);
     if (p.gy > 65535) return cudaErrorInvalidConfiguration;
     const int nbj = (int)cdiv(n - 1, Tj);
@@ -371,6 +372,17 @@ void stencil_plan_dims(bool heat, int64_t n, const int64_t *t, bool f64, int64_t
                        int *bx, int *by, int *vec) {
     StencilPlan p = heat ? plan_heat3d(n, t[0], t[1], t[2], f64) : plan_jacobi2d(n, t[0], t[1], f64);
     *gx = p.gx; *gy = p.gy; *bx = p.bx; *by = p.by; *vec = p.vec;
+}
+
+// lanes of a warp along l_s1 for a stencil tile: WAF on the staged paths (they honour exec.warp_align),
+// otherwise the linear layout's run of 16-byte groups (or points) along l_s1
+int stencil_simt_x(bool heat, int64_t n, const int64_t *t, bool f64, int waf) {
+    const bool staged = stencil_staged_enabled() && (heat ? heat3d_staged_applicable(n, t[0], t[1], t[2], f64)
+                                                          : jacobi2d_staged_applicable(n, t[0], t[1], f64));
+    if (staged && waf > 0) return waf;
+    const int64_t along = heat ? t[2] : t[1];
+    const int64_t groups = staged || !f64 ? (along + 3) / 4 : along;
+    return (int)std::min<int64_t>(32, std::max<int64_t>(1, groups));
 }
 
 }  // namespace eatss

@@ -44,6 +44,23 @@ __device__ __forceinline__ void bulk_row_g2s(void *dst, const void *src, unsigne
         : "memory");
 }
 
+// Work items (a, b) of an A x B space, a = the 16-byte column group along the CMA loop l_s1.  waf = 0:
+// linear order (a fastest); waf in {4, 8, 16, 32}: the warp-fraction layout -- lane l of
+// virtual warp w takes a = (w % wa)*waf + l % waf and b = (w / wa)*(32/waf) + l / waf (wa = ceil(A/waf)),
+// i.e. WAF lanes of every warp contiguous along l_s1 and the other 32/WAF lanes on the next rows.
+// Visits every item exactly once; returns false when v is past the space.
+__device__ __forceinline__ bool waf_item(int v, int A, int B, int waf, int &a, int &b) {
+    if (waf <= 0) {
+        a = v % A;
+        b = v / A;
+        return b < B;
+    }
+    const int w = v >> 5, l = v & 31, wa = (A + waf - 1) / waf;
+    a = (w % wa) * waf + l % waf;
+    b = (w / wa) * (32 / waf) + l / waf;
+    return b < B;
+}
+
 // ------------------------------------------------------------------ jacobi-2d
 // Window: rows [ilo-1, ihi+1), columns [cs, ce) = [tj0-4, tj0+Tj+4) clipped to [0, n); n, Tj, tj0
 // multiples of 4, so every window row is a 16-byte-aligned run of (ce-cs)*4 bytes.
@@ -52,7 +69,7 @@ __device__ __forceinline__ void bulk_row_g2s(void *dst, const void *src, unsigne
 template <bool COVER>
 __global__ void __launch_bounds__(256) jacobi2d_staged(float *__restrict__ dst, const float *__restrict__ src,
                                                        const float *__restrict__ bsrc, int64_t n, int Ti, int Tj,
-                                                       int32_t *counts) {
+                                                       int32_t *counts, int waf) {
     extern __shared__ __align__(16) float win[];
     __shared__ uint64_t bar;
     const int64_t ti0 = (int64_t)blockIdx.y * Ti, tj0 = (int64_t)blockIdx.x * Tj;
@@ -102,14 +119,22 @@ __global__ void __launch_bounds__(256) jacobi2d_staged(float *__restrict__ dst, 
     }
     const float c02 = 0.2f;
     const int rows = (int)(ihi - ilo);
-    for (int64_t g = g0 + tid; g < g1; g += blockDim.x) {
+    // items: (column group, row chunk); with a warp alignment the rows are cut into 32/WAF chunks
+    const int ngr = (int)(g1 - g0), nch = waf > 0 ? 32 / waf : 1, per = (rows + nch - 1) / nch;
+    const int span = waf > 0 ? ((ngr + waf - 1) / waf) * waf * nch : ngr;  // virtual items
+    for (int v = tid; v < span; v += blockDim.x) {
+        int ga, ch;
+        if (!waf_item(v, ngr, nch, waf, ga, ch) || ga >= ngr) continue;
+        const int rb = ch * per, re = min(rows, rb + per);
+        if (rb >= re) continue;
+        const int64_t g = g0 + ga;
         const int cl = (int)(4 * g - cs);  // window column of the group's first element
         const bool full = 4 * g >= jlo && 4 * g + 3 < jhi;
         const float *colp = win + cl;
-        float4 u = *reinterpret_cast<const float4 *>(colp);
-        float4 c = *reinterpret_cast<const float4 *>(colp + W);
+        float4 u = *reinterpret_cast<const float4 *>(colp + rb * W);
+        float4 c = *reinterpret_cast<const float4 *>(colp + (rb + 1) * W);
         const int lm = cl > 0 ? -1 : 0, rp = cl + 4 < W ? 4 : 3;  // clamped (unused when clamped)
-        for (int r = 1; r <= rows; r++) {
+        for (int r = rb + 1; r <= re; r++) {
             const float *row = colp + r * W;
             const float4 d = *reinterpret_cast<const float4 *>(row + W);
             const float l = row[lm], rr = row[rp];
@@ -142,7 +167,7 @@ __global__ void __launch_bounds__(256) jacobi2d_staged(float *__restrict__ dst, 
 // barrier untouched) when the tile is empty.  Ends with __syncthreads(): the window may be reused.
 __device__ __forceinline__ bool heat_tile(float *__restrict__ dst, const CUtensorMap *msrc, int64_t n, int Ti,
                                           int Tj, int Tk, int nbj, int64_t bx, int64_t by, float *win,
-                                          uint64_t *bar, unsigned phase) {
+                                          uint64_t *bar, unsigned phase, int waf) {
     const int64_t tk0 = bx * Tk;
     const int64_t ti0 = (by / nbj) * Ti, tj0 = (by % nbj) * Tj;
     const int64_t ilo = ti0 > 1 ? ti0 : 1, ihi = ti0 + Ti < n - 1 ? ti0 + Ti : n - 1;
@@ -164,8 +189,13 @@ __device__ __forceinline__ bool heat_tile(float *__restrict__ dst, const CUtenso
     const int cols = nj * ng;
     const int chunks = max(1, min(ni, (int)blockDim.x / cols));
     const int per = (ni + chunks - 1) / chunks;
-    for (int e = tid; e < cols * chunks; e += blockDim.x) {
-        const int gi = e % ng, jj = (e / ng) % nj, ch = e / cols;
+    // items (k-group, (j, i-chunk)); with a warp alignment WAF lanes of each warp run along k
+    const int nb = nj * chunks, span = waf > 0 ? ((ng + waf - 1) / waf) * waf * (((nb + 32 / waf - 1) / (32 / waf)) * (32 / waf))
+                                              : cols * chunks;
+    for (int e = tid; e < span; e += blockDim.x) {
+        int gi, b;
+        if (!waf_item(e, ng, nb, waf, gi, b) || gi >= ng) continue;
+        const int jj = b % nj, ch = b / nj;
         const int ib = ch * per, ie = min(ni, ib + per);
         if (ib >= ie) continue;
         const int64_t k = 4 * (g0 + gi), j = jlo + jj;
@@ -211,7 +241,8 @@ __device__ __forceinline__ bool heat_tile(float *__restrict__ dst, const CUtenso
 
 template <bool COVER>
 __global__ void __launch_bounds__(256) heat3d_staged(float *__restrict__ dst, const __grid_constant__ CUtensorMap msrc,
-                                                     int64_t n, int Ti, int Tj, int Tk, int nbj, int32_t *counts) {
+                                                     int64_t n, int Ti, int Tj, int Tk, int nbj, int32_t *counts,
+                                                     int waf) {
     extern __shared__ __align__(128) unsigned char win_raw[];
     // TMA destinations must be 128-byte aligned: align the dynamic window by hand
     float *win = reinterpret_cast<float *>(win_raw + ((128u - (su32(win_raw) & 127u)) & 127u));
@@ -241,7 +272,7 @@ __global__ void __launch_bounds__(256) heat3d_staged(float *__restrict__ dst, co
     }
     pdl_wait();
     __syncthreads();
-    heat_tile(dst, &msrc, n, Ti, Tj, Tk, nbj, blockIdx.x, blockIdx.y, win, &bar, 0);
+    heat_tile(dst, &msrc, n, Ti, Tj, Tk, nbj, blockIdx.x, blockIdx.y, win, &bar, 0, waf);
     pdl_trigger();  // after this CTA's stores: the next sweep's launch overlaps this grid's tail
 }
 
@@ -302,28 +333,28 @@ bool heat3d_staged_applicable(int64_t n, int64_t Ti, int64_t Tj, int64_t Tk, boo
 }
 
 cudaError_t launch_jacobi2d_staged(float *dst, const float *src, const float *bsrc, int64_t n, int64_t Ti, int64_t Tj,
-                                   int split_pct, int32_t *counts, cudaStream_t s) {
+                                   int split_pct, int32_t *counts, cudaStream_t s, int waf) {
     const int64_t gx = (n - 1 + Tj - 1) / Tj, gy = (n - 1 + Ti - 1) / Ti;
     if (gy > 65535 || gx > INT32_MAX) return cudaErrorInvalidConfiguration;
     const int smem = counts ? 0 : jacobi_staged_smem(n, Ti, Tj);
     dim3 grid((unsigned)gx, (unsigned)gy), block(256);
     if (counts) {
-        jacobi2d_staged<true><<<grid, block, 0, s>>>(dst, src, bsrc, n, (int)Ti, (int)Tj, counts);
+        jacobi2d_staged<true><<<grid, block, 0, s>>>(dst, src, bsrc, n, (int)Ti, (int)Tj, counts, waf);
         return cudaGetLastError();
     }
     cudaFuncSetAttribute(jacobi2d_staged<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     return launch_pdl(jacobi2d_staged<false>, grid, block, smem, staged_carveout(smem, split_pct), s, dst, src, bsrc,
-                      n, (int)Ti, (int)Tj, (int32_t *)nullptr);
+                      n, (int)Ti, (int)Tj, (int32_t *)nullptr, waf);
 }
 
 cudaError_t launch_heat3d_staged(float *dst, const float *src, int64_t n, int64_t Ti, int64_t Tj, int64_t Tk,
-                                 int split_pct, int32_t *counts, cudaStream_t s) {
+                                 int split_pct, int32_t *counts, cudaStream_t s, int waf) {
     const int64_t nbi = (n - 1 + Ti - 1) / Ti, nbj = (n - 1 + Tj - 1) / Tj, gx = (n - 1 + Tk - 1) / Tk;
     if (nbi * nbj > 65535) return cudaErrorInvalidConfiguration;
     dim3 grid((unsigned)gx, (unsigned)(nbi * nbj)), block(256);
     CUtensorMap m{};
     if (counts) {
-        heat3d_staged<true><<<grid, block, 0, s>>>(dst, m, n, (int)Ti, (int)Tj, (int)Tk, (int)nbj, counts);
+        heat3d_staged<true><<<grid, block, 0, s>>>(dst, m, n, (int)Ti, (int)Tj, (int)Tk, (int)nbj, counts, waf);
         return cudaGetLastError();
     }
     const cuuint64_t dims[3] = {(cuuint64_t)n, (cuuint64_t)n, (cuuint64_t)n};
@@ -337,7 +368,7 @@ cudaError_t launch_heat3d_staged(float *dst, const float *src, int64_t n, int64_
     const int smem = heat_staged_smem(Ti, Tj, Tk);
     cudaFuncSetAttribute(heat3d_staged<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     return launch_pdl(heat3d_staged<false>, grid, block, smem, staged_carveout(smem, split_pct), s, dst,
-                      (const CUtensorMap)m, n, (int)Ti, (int)Tj, (int)Tk, (int)nbj, (int32_t *)nullptr);
+                      (const CUtensorMap)m, n, (int)Ti, (int)Tj, (int)Tk, (int)nbj, (int32_t *)nullptr, waf);
 }
 
 }  // namespace eatss

@@ -85,3 +85,35 @@ def test_carveout_exact_is_reported(cuda_device, split):
     E.run(j, (16, 128), [dev(Aj), dev(Bj)])
     torch.cuda.synchronize()
     assert E.last_carveout(j) == [split, split]
+
+
+@pytest.mark.parametrize("waf", WAFS)
+def test_stencils_waf_bit_identical_to_default_layout(cuda_device, waf):
+    """The warp layout only changes which lane computes which point: every value is bit-identical to the
+    default layout, and within tolerance of the fp64 oracle (heat-3d, jacobi-2d staged paths)."""
+    n, T = 132, 6
+    Aj, Bj = synth.polybench_jacobi2d(n)
+    ref_A, _ = O.jacobi2d(Aj, Bj, T)
+    outs = {}
+    for w in (0, waf):
+        d = E.desc_builtin("jacobi-2d", (n,), tsteps=T)
+        d.set_exec(split_pct=50, engine=1, warp_align=w)
+        Ad, Bd = dev(Aj), dev(Bj)
+        E.run(d, (16, 64), [Ad, Bd])
+        outs[w] = host(Ad)
+    assert np.array_equal(outs[0], outs[waf])
+    assert O.normwise_rel_err(outs[waf], ref_A) <= 1e-5
+    m = 68
+    Ah = synth.uniform((m, m, m), 7); Bh = Ah.copy()
+    ref_h, _ = O.heat3d(Ah, Bh, 3)
+    hs = {}
+    for w in (0, waf):
+        d = E.desc_builtin("heat-3d", (m,), tsteps=3)
+        d.set_exec(split_pct=50, engine=1, warp_align=w)
+        (p,) = E.plan(d, (16, 16, 32))[:1]
+        assert p.simt_x == (w or 8)
+        Ad, Bd = dev(Ah), dev(Bh)
+        E.run(d, (16, 16, 32), [Ad, Bd])
+        hs[w] = host(Ad)
+    assert np.array_equal(hs[0], hs[waf])
+    assert O.normwise_rel_err(hs[waf], ref_h) <= 1e-5

@@ -275,3 +275,13 @@ def test_exec_opts_validation():
         d.set_exec(carveout_exact=2)
     d.set_exec(split_pct=0, warp_align=8, carveout_exact=1)
     assert E.last_carveout(d) == []  # no run yet
+
+
+@pytest.mark.parametrize("waf", [4, 8, 16, 32])
+def test_stencil_plan_reports_warp_alignment(waf):
+    d = E.desc_builtin("jacobi-2d", (4000,), tsteps=10)
+    d.set_exec(split_pct=50, engine=1, warp_align=waf)
+    for p in E.plan(d, (16, 1024)):
+        assert p.simt_x == waf  # staged path: WAF lanes of each warp along j
+    d.set_exec(split_pct=50, engine=1)
+    assert all(p.simt_x == 32 for p in E.plan(d, (16, 1024)))
