@@ -31,14 +31,17 @@ Rules (PAPER.md citation for each):
  13  tie-break: max OBJ, then min sum of T on objective-free positions,
      then max T_{l_s1}, then lexicographically smallest T (reading Q16).
 
-Pin status (tests/test_oracle_model.py; DESIGN.md §2.4):
+Pin status (tests/test_oracle_model.py; DESIGN.md §2.4, §2.6):
   pinned    the worked example (unique optimum), Table II / l_s1 / nrefs,
             heat-3d 9/12 and mttkrp / conv-2d 11/12 feasible configurations (conv-2d's filter
-            size chosen to agree, reading R-N9), Z3 driven as in P:179-181, a hand-solved space, the
-            infeasible spaces.
-  parity unpinned (our readings, held bit-exact against the C++ enumerator only): stencil H weights
-            and footprints (Q6, Q11), the 2-D H rule (Q7), the B-set order beyond three parallel loops
-            (Q12), the split levels (Q17), the sweep sizes (Q19), the tensor-core mode (reading T).
+            size 5 or 6 is the only one reading R agrees with, reading R-N9), Z3 driven as in P:179-181,
+            a hand-solved space, the infeasible spaces, the tensor-mode optima derived by hand; the
+            alternatives Q2 units, Q4 literal sigma, Q7 WARP scale, Q10 array / reference counts and Q11
+            halo-inclusive footprints each break one of P:121 / P:153 / P:282 (Reading switch below).
+  parity unpinned (our readings, held bit-exact against the C++ enumerator; their alternatives keep every
+            printed fact and are measured on B200 instead, harness/readings.py): H weights (Q6), the 2-D
+            H rule (Q7), the B-set order beyond three parallel loops (Q12), the tie-break (Q16); the
+            split levels (Q17), the sweep sizes (Q19); the tensor-core mode (reading T) beyond Eq. 2.
 """
 from __future__ import annotations
 
