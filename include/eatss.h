@@ -169,7 +169,14 @@ typedef struct {
 /* EATSS_ENGINE_UNTILED (jacobi-2d / heat-3d only; others return EATSS_E_UNSUPPORTED): the plain loop
  * nest without tiling -- one thread per interior point, neighbours from global memory, the tile
  * vector ignored -- the "untiled" baseline of BASELINE config 4 (same time loop and arithmetic). */
-typedef enum { EATSS_ENGINE_AUTO = 0, EATSS_ENGINE_SIMT = 1, EATSS_ENGINE_TENSOR = 2, EATSS_ENGINE_UNTILED = 3 } eatss_engine;
+/* EATSS_ENGINE_TENSOR_F16 (fp32 gemm family): the tcgen05 GEMM with 3xFP16 operands -- each row of A and
+ * column of B scaled by a power of two so its largest magnitude lies in [2^14, 2^15), split into fp16
+ * hi + lo (22 significant bits, like 3xTF32), hi*hi + hi*lo + lo*hi accumulated in fp32 and the scales undone
+ * exactly in the epilogue: fp32-level accuracy at fp16 MMA rate.  Same tile vector as EATSS_ENGINE_TENSOR
+ * with Tk counted in fp16 elements: Ti in {128, 256}, Tj in 16..256 step 16, Tk in {16, 32, 64, 128}
+ * (model mode 3).  Other builtins / fp64 descriptors: EATSS_E_UNSUPPORTED. */
+typedef enum { EATSS_ENGINE_AUTO = 0, EATSS_ENGINE_SIMT = 1, EATSS_ENGINE_TENSOR = 2, EATSS_ENGINE_UNTILED = 3,
+               EATSS_ENGINE_TENSOR_F16 = 4 } eatss_engine;
 typedef struct {
     int32_t split_pct;  /* shared-memory carve-out preference, percent of max (sigma) */
     int32_t engine;     /* eatss_engine; AUTO = SIMT unless the tensor-core path applies; UNTILED: stencils */

@@ -499,7 +499,7 @@ def tensor_applicable(prog: Program):
     return False
 
 
-def tensor_domains(prog: Program):
+def tensor_domains(prog: Program, mode: int = 2):
     n0 = prog.nests[0]
     d = derive(n0, 16)
     doms = []
@@ -525,7 +525,7 @@ def tensor_domains(prog: Program):
         elif l.parallel:
             doms.append([128, 256])
         else:
-            doms.append([32, 64])
+            doms.append([32, 64] if mode == 2 else [64, 128])  # whole 128-byte atoms of fp32 / fp16
     return doms
 
 
@@ -570,9 +570,12 @@ def _evaluate_tensor_6d(prog: Program, gpu: Gpu, opts: Opts, T):
 
 
 def evaluate_tensor(prog: Program, gpu: Gpu, opts: Opts, T):
+    """T1-T3 (mode 2: the 3xTF32 engine) or T5 (mode 3: the 3xFP16 engine -- 2-byte operands, B staged
+    K-major by its transposing split, so no 32-column rounding and N per CTA half in multiples of 8)."""
     if tensor_applicable(prog) == "6d":
         return _evaluate_tensor_6d(prog, gpu, opts, T)
-    e = prog.dtype_bytes
+    f16 = opts.mode == 3
+    e = 2 if f16 else prog.dtype_bytes
     feas = np.ones(T[0].shape, dtype=bool)
     obj = np.zeros(T[0].shape, dtype=np.int64)
     for nest in prog.nests:
@@ -581,7 +584,7 @@ def evaluate_tensor(prog: Program, gpu: Gpu, opts: Opts, T):
         rows = [l.name for l in nest.loops if l.parallel and l.name != d.ls1][0]  # UMMA M loop
         cg = T[pos[rows]] // 128
         n_cta = T[pos[d.ls1]] // cg
-        feas &= (T[pos[d.ls1]] % cg == 0) & (n_cta % 16 == 0)                     # T3 legality
+        feas &= (T[pos[d.ls1]] % cg == 0) & (n_cta % (8 if f16 else 16) == 0)     # T3 legality
         feas &= 2 * T[pos[d.ls1]] <= TMEM_COLS                                      # T3 TMEM
         written = {r.array for r in nest.refs if r.write}
         inputs = []
@@ -596,7 +599,7 @@ def evaluate_tensor(prog: Program, gpu: Gpu, opts: Opts, T):
                 if it == rows:
                     v = v * 128
                 elif it == d.ls1:
-                    v = v * (-(-n_cta // 32) * 32 if mn_major else n_cta)
+                    v = v * (-(-n_cta // 32) * 32 if (mn_major and not f16) else n_cta)
                 else:
                     v = v * T[pos[it]]
             vin = vin + v
@@ -611,10 +614,12 @@ def evaluate_tensor(prog: Program, gpu: Gpu, opts: Opts, T):
 def select_tiles(prog: Program, gpu: Gpu, opts: Opts, keep_ties: bool = True, rd: Reading = R) -> Result:
     """Exhaustive maximisation of OBJ over the whole domain (no pruning); `rd` selects the reading."""
     L = prog.L
-    tensor = opts.mode == 2
+    tensor = opts.mode in (2, 3)
     if tensor and not tensor_applicable(prog):
         return Result(None, 0, 0, 0, [])
-    doms = ([np.array(v, dtype=np.int64) for v in tensor_domains(prog)] if tensor else
+    if opts.mode == 3 and tensor_applicable(prog) != "3d":
+        return Result(None, 0, 0, 0, [])  # the 3xFP16 engine runs the depth-3 contractions only
+    doms = ([np.array(v, dtype=np.int64) for v in tensor_domains(prog, opts.mode)] if tensor else
             [np.array(domain(n, gpu, opts.waf), dtype=np.int64) for n in extents(prog)])
     free = objective_free_positions(prog, opts.waf, rd)
     if tensor and tensor_applicable(prog) == "6d":  # T4: objective-free = outside the CTA tile (the reduction)

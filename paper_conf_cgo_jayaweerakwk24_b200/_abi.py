@@ -24,7 +24,7 @@ STATUS_NAMES = {0: "OK", -1: "E_INVALID", -2: "E_INFEASIBLE", -3: "E_CUDA", -4: 
 F32, F64 = 1, 2
 BUILTINS = {"gemm": 0, "2mm": 1, "3mm": 2, "syrk": 3, "jacobi-2d": 4, "heat-3d": 5, "ccsd_t_d1": 6,
             "mvt": 7, "atax": 8, "bicg": 9, "gemver": 10, "mttkrp": 11, "conv-2d": 12}
-ENGINE_AUTO, ENGINE_SIMT, ENGINE_TENSOR, ENGINE_UNTILED = 0, 1, 2, 3
+ENGINE_AUTO, ENGINE_SIMT, ENGINE_TENSOR, ENGINE_UNTILED, ENGINE_TENSOR_F16 = 0, 1, 2, 3, 4
 MAX_LOOPS = 8
 MAX_NESTS = 4
 MAX_BUFFERS = 16

@@ -327,7 +327,8 @@ static bool simt_untranspose(const eatss_kernel_desc *d) {
         const char *e = getenv("EATSS_SYRK_TRANSB");
         return e && atoi(e) != 0;
     }();
-    return d->kind == EATSS_SYRK && d->dtype == EATSS_F32 && d->exec.engine != EATSS_ENGINE_TENSOR && !off;
+    return d->kind == EATSS_SYRK && d->dtype == EATSS_F32 && d->exec.engine != EATSS_ENGINE_TENSOR &&
+           d->exec.engine != EATSS_ENGINE_TENSOR_F16 && !off;
 }
 static void untranspose_nests(const eatss_kernel_desc *d, std::vector<ContractNest> &cn, const void *at) {
     for (auto &n : cn) {
@@ -665,7 +666,7 @@ eatss_status eatss_desc_set_scalars(eatss_kernel_desc *d, double alpha, double b
 eatss_status eatss_desc_set_exec(eatss_kernel_desc *d, const eatss_exec_opts *o) {
     if (!d || !o) return fail(EATSS_E_INVALID, "eatss_desc_set_exec: null argument");
     if (o->split_pct < 0 || o->split_pct > 100) return fail(EATSS_E_INVALID, "split_pct must be 0..100");
-    if (o->engine < 0 || o->engine > 3) return fail(EATSS_E_INVALID, "bad engine");
+    if (o->engine < 0 || o->engine > 4) return fail(EATSS_E_INVALID, "bad engine");
     if (o->warp_align != 0 && o->warp_align != 4 && o->warp_align != 8 && o->warp_align != 16 && o->warp_align != 32)
         return fail(EATSS_E_INVALID, "warp_align must be 0, 4, 8, 16 or 32");
     if (o->carveout_exact != 0 && o->carveout_exact != 1) return fail(EATSS_E_INVALID, "carveout_exact must be 0 or 1");
@@ -878,6 +879,8 @@ static eatss_status run_body(eatss_kernel_desc *d, int only_nest, const int64_t 
     cudaStream_t s = (cudaStream_t)stream;
     if (d->exec.engine == EATSS_ENGINE_UNTILED && d->kind != EATSS_JACOBI2D && d->kind != EATSS_HEAT3D)
         return fail(EATSS_E_UNSUPPORTED, "eatss_run: the untiled engine is the stencils' baseline only");
+    if (d->exec.engine == EATSS_ENGINE_TENSOR_F16 && (!is_contraction(d->kind) || d->dtype != EATSS_F32))
+        return fail(EATSS_E_UNSUPPORTED, "eatss_run: the 3xFP16 tensor engine runs the fp32 gemm family only");
     if (is_contraction(d->kind)) {
         auto cn = contraction_nests(d, buffers);
         const int sl = smem_limit_bytes();
@@ -889,11 +892,13 @@ static eatss_status run_body(eatss_kernel_desc *d, int only_nest, const int64_t 
             untranspose_nests(d, cn, d->ws);
         }
         RunScratch scratch;  // split-operand scratch of the tcgen05 GEMMs (stream-ordered, this run only)
-        if (d->exec.engine == EATSS_ENGINE_TENSOR) {
+        const bool f16 = d->exec.engine == EATSS_ENGINE_TENSOR_F16;
+        if (d->exec.engine == EATSS_ENGINE_TENSOR || f16) {
             size_t need = 0;
             for (int i = 0; i < (int)cn.size(); i++) {
                 ContractPlan p = plan_contraction(cn[i], tiles, sl, d->exec.warp_align);
-                if (tcm_applicable(cn[i], p)) need = std::max(need, tcm_ws_floats(cn[i], p));
+                if (f16 && tcf_applicable(cn[i], p)) need = std::max(need, tcf_ws_floats(cn[i], p));
+                if (!f16 && tcm_applicable(cn[i], p)) need = std::max(need, tcm_ws_floats(cn[i], p));
             }
             if (need) {
                 cudaError_t e = scratch.alloc(need * 4, s);
@@ -905,17 +910,22 @@ static eatss_status run_body(eatss_kernel_desc *d, int only_nest, const int64_t 
             ContractPlan p = plan_contraction(cn[i], tiles, sl, d->exec.warp_align);
             int tsm = 0, tcols = 0;
             const bool want_tc = d->exec.engine == EATSS_ENGINE_TENSOR;
-            // MMA-legal tiles (Ti = 128) take the TMA/SS-UMMA GEMM; narrow tiles the transposed TS kernel
+            // MMA-legal tiles (Ti = 128/256) take the TMA/SS-UMMA GEMM; narrow tiles the transposed TS kernel
             const bool tcm = want_tc && tcm_applicable(cn[i], p);
             const bool tc = want_tc && !tcm && tc_plan(cn[i], p, &tsm, &tcols);
+            const bool tcf = f16 && tcf_applicable(cn[i], p);
             if (want_tc && !tc && !tcm)
                 return fail(EATSS_E_UNSUPPORTED, "eatss_run: tensor engine not applicable to this tile/operand layout");
+            if (f16 && !tcf)
+                return fail(EATSS_E_UNSUPPORTED, "eatss_run: the 3xFP16 tensor engine needs Ti in {128, 256}, Tj in "
+                                                 "16..256 step 16, Tk in {16, 32, 64, 128} fitting two stages");
             cudaEvent_t *ev = kernel_events(d, i);
-            if (ev && !tcm) cudaEventRecord(ev[0], s);
-            cudaError_t e = tcm  ? launch_tcm_contraction(cn[i], p, (float *)scratch.p, scratch.bytes / 4, s, ev)
-                            : tc ? launch_tc_contraction(cn[i], p, exec_cv(d), s)
-                                 : launch_contraction(cn[i], p, exec_cv(d), nullptr, s);
-            if (ev && !tcm) cudaEventRecord(ev[1], s);
+            if (ev && !tcm && !tcf) cudaEventRecord(ev[0], s);
+            cudaError_t e = tcf   ? launch_tcf_contraction(cn[i], p, (float *)scratch.p, scratch.bytes / 4, s, ev)
+                            : tcm ? launch_tcm_contraction(cn[i], p, (float *)scratch.p, scratch.bytes / 4, s, ev)
+                            : tc  ? launch_tc_contraction(cn[i], p, exec_cv(d), s)
+                                  : launch_contraction(cn[i], p, exec_cv(d), nullptr, s);
+            if (ev && !tcm && !tcf) cudaEventRecord(ev[1], s);
             d->last_cv[i] = take_carveout();
             if (e != cudaSuccess) return cuda_fail(e, "eatss_run(contraction)");
         }
@@ -1098,7 +1108,8 @@ eatss_status eatss_run_host(const eatss_kernel_desc *cd, const int64_t *tiles, v
         auto cn = contraction_nests(d, dev_bufs);
         ContractNest full = cn[0];
         const int64_t M = full.M, Ti = std::max<int64_t>(1, std::min(tiles[0], M));
-        const int64_t unit = d->exec.engine == EATSS_ENGINE_TENSOR ? std::max<int64_t>(Ti, 256) : Ti;
+        const bool f16 = d->exec.engine == EATSS_ENGINE_TENSOR_F16;
+        const int64_t unit = d->exec.engine == EATSS_ENGINE_TENSOR || f16 ? std::max<int64_t>(Ti, 256) : Ti;
         int64_t rb = (M + row_blocks - 1) / row_blocks;
         rb = (rb + unit - 1) / unit * unit;
         const int nblk = (int)((M + rb - 1) / rb);
@@ -1108,12 +1119,14 @@ eatss_status eatss_run_host(const eatss_kernel_desc *cd, const int64_t *tiles, v
         cudaMemcpyAsync(dev_bufs[2], hB, d->hbuf_bytes[2], cudaMemcpyHostToDevice, sin);
         const int sl = smem_limit_bytes();
         RunScratch scratch;  // tensor engine: split operands of the largest block (blocks run in order on s)
-        if (d->exec.engine == EATSS_ENGINE_TENSOR) {
+        if (d->exec.engine == EATSS_ENGINE_TENSOR || f16) {
             ContractNest b0 = full;
             b0.M = std::min(rb, M);
             ContractPlan p0 = plan_contraction(b0, tiles, sl, d->exec.warp_align);
-            if (tcm_applicable(b0, p0)) {
-                const cudaError_t ea = scratch.alloc(tcm_ws_floats(b0, p0) * 4, s);
+            const size_t need = f16 ? (tcf_applicable(b0, p0) ? tcf_ws_floats(b0, p0) : 0)
+                                    : (tcm_applicable(b0, p0) ? tcm_ws_floats(b0, p0) : 0);
+            if (need) {
+                const cudaError_t ea = scratch.alloc(need * 4, s);
                 if (ea != cudaSuccess) return cuda_fail(ea, "eatss_run_host(tensor scratch)");
             }
         }
@@ -1134,11 +1147,13 @@ eatss_status eatss_run_host(const eatss_kernel_desc *cd, const int64_t *tiles, v
             int tsm = 0, tcols = 0;
             const bool tcm = want_tc && tcm_applicable(blk, p);
             const bool tc = want_tc && !tcm && tc_plan(blk, p, &tsm, &tcols);
-            if (want_tc && !tc && !tcm)
+            const bool tcf = f16 && tcf_applicable(blk, p);
+            if ((want_tc && !tc && !tcm) || (f16 && !tcf))
                 return fail(EATSS_E_UNSUPPORTED, "eatss_run_host: tensor engine not applicable to this tile");
-            e = tcm  ? launch_tcm_contraction(blk, p, (float *)scratch.p, scratch.bytes / 4, s, nullptr)
-                : tc ? launch_tc_contraction(blk, p, exec_cv(d), s)
-                     : launch_contraction(blk, p, exec_cv(d), nullptr, s);
+            e = tcf   ? launch_tcf_contraction(blk, p, (float *)scratch.p, scratch.bytes / 4, s, nullptr)
+                : tcm ? launch_tcm_contraction(blk, p, (float *)scratch.p, scratch.bytes / 4, s, nullptr)
+                : tc  ? launch_tc_contraction(blk, p, exec_cv(d), s)
+                      : launch_contraction(blk, p, exec_cv(d), nullptr, s);
             if (e != cudaSuccess) return cuda_fail(e, "eatss_run_host(gemm block)");
             cudaEventRecord(ecomp, s);
             cudaStreamWaitEvent(sout, ecomp, 0);
@@ -1222,6 +1237,18 @@ eatss_status eatss_coverage(const eatss_kernel_desc *d, int nest, const int64_t 
 
 int64_t eatss_launches_per_run(const eatss_kernel_desc *d, const int64_t *tiles) {
     if (!d) return -1;
+    if (is_contraction(d->kind) && d->exec.engine == EATSS_ENGINE_TENSOR_F16) {  // fused split + GEMM per nest
+        if (!tiles || check_tiles(d, tiles) != EATSS_OK) return -1;
+        void *b[EATSS_MAX_BUFFERS];
+        for (int i = 0; i < EATSS_MAX_BUFFERS; i++) b[i] = (void *)((uintptr_t)(1 << 20) * (uintptr_t)(i + 1));
+        int64_t total = 0;
+        for (auto &n : contraction_nests(d, b)) {
+            ContractPlan p = plan_contraction(n, tiles, smem_limit_bytes(), d->exec.warp_align);
+            if (!tcf_applicable(n, p)) return -1;
+            total += 2;
+        }
+        return total;
+    }
     if (is_contraction(d->kind) && d->exec.engine == EATSS_ENGINE_TENSOR) {
         if (!tiles || check_tiles(d, tiles) != EATSS_OK) return -1;
         void *b[EATSS_MAX_BUFFERS];  // layout only: aligned dummies, never dereferenced

@@ -61,7 +61,7 @@ bool tc_plan(const ContractNest &n, const ContractPlan &p, int *smem_bytes, int 
 cudaError_t launch_tc_contraction(const ContractNest &n, const ContractPlan &p, int carveout, cudaStream_t s);
 // tcgen05 3xTF32 GEMM for MMA-legal tiles (tc_mma.cu): Ti in {128, 256} (one CTA / a CTA pair),
 // Tj in 16..256 step 16, Tk in {8, 16, 32, 64}
-bool tcm_applicable(const ContractNest &n, const ContractPlan &p);
+bool tcm_applicable(const ContractNest &n, const ContractPlan &p, bool f16 = false);
 // Split-operand workspace (floats) one launch needs: owned by the caller's descriptor, so
 // concurrent descriptors (streams, devices, host threads) never share it.
 size_t tcm_ws_floats(const ContractNest &n, const ContractPlan &p);
@@ -70,6 +70,13 @@ size_t tcm_ws_floats(const ContractNest &n, const ContractPlan &p);
 cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p, float *ws, size_t ws_floats,
                                    cudaStream_t s, cudaEvent_t *ev = nullptr);
 int tcm_launches(const ContractNest &n, const ContractPlan &p);  // kernels one launch_tcm_contraction issues
+// 3xFP16 variant of the same GEMM (engine TENSOR_F16): operands split into fp16 hi / lo after a per-row (A)
+// / per-column (B) power-of-two scaling that keeps them inside fp16's range; same tiles, Tk in fp16 elements
+// (16, 32, 64, 128: 32..256 bytes per stage row); B always K-major (the split transposes a row-major B)
+bool tcf_applicable(const ContractNest &n, const ContractPlan &p);
+size_t tcf_ws_floats(const ContractNest &n, const ContractPlan &p);
+cudaError_t launch_tcf_contraction(const ContractNest &n, const ContractPlan &p, float *ws, size_t ws_floats,
+                                   cudaStream_t s, cudaEvent_t *ev = nullptr);
 cudaError_t launch_contraction(const ContractNest &n, const ContractPlan &p, int carveout_pct,
                                int32_t *coverage_counts, cudaStream_t s);
 // kernels one launch_contraction issues (the SIMT staged path adds a pre-pass when it splits the

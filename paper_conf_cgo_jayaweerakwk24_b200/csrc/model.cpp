@@ -241,7 +241,7 @@ struct Search {
         return v;
     }
 
-    bool tensor = false, tensor6 = false;
+    bool tensor = false, tensor6 = false, f16 = false;  // f16: mode 3 (the 3xFP16 engine)
     Sets6 s6;                        // tensor6: M-side / N-side / reduction positions
     std::vector<int64_t> ext;        // loop extents
     int64_t smem_cap = 0;
@@ -266,7 +266,7 @@ struct Search {
         if (tensor) {  // reading T3
             for (const NestEval &ne : nests) {
                 const int64_t tn = T[ne.m.ls1], cg = T[ne.rows_pos] / 128;
-                if (cg < 1 || tn % cg || (tn / cg) % 16) return false;  // UMMA N per CTA half
+                if (cg < 1 || tn % cg || (tn / cg) % (f16 ? 8 : 16)) return false;  // UMMA N per CTA half
                 if (2 * tn > kTmemCols) return false;                   // two fp32 accumulator buffers
                 const int64_t n_cta = tn / cg;
                 int64_t vin = 0;
@@ -275,7 +275,7 @@ struct Search {
                     for (int p = 0; p < L; p++) {
                         if (!((ne.in_fp[f] >> p) & 1u)) continue;
                         if (p == ne.rows_pos) v *= 128;  // per-CTA rows
-                        else if (p == ne.m.ls1) v *= ne.in_mn[f] ? (n_cta + 31) / 32 * 32 : n_cta;
+                        else if (p == ne.m.ls1) v *= (ne.in_mn[f] && !f16) ? (n_cta + 31) / 32 * 32 : n_cta;
                         else v *= T[p];
                     }
                     vin += v;
@@ -399,6 +399,8 @@ extern "C" eatss_status eatss_select_tiles(const eatss_kernel_desc *d, const eat
         s.nests.push_back(ne);
     }
     s.ext = ext;
+    if (o->mode == 3 && !(s.nests.size() >= 1 && s.nests[0].nest->loops.size() == 3))
+        return fail(EATSS_E_UNSUPPORTED, "eatss_select_tiles: mode 3 (3xFP16 engine) needs depth-3 contraction nests");
     if (o->mode == 2 && s.nests.size() == 1 && s.nests[0].nest->loops.size() >= 4) {
         // tensor-core mode T4: the 6-D contraction pattern of the ccsd executor
         s.s6 = contraction_sets(s.nests[0], o->warp_align);
@@ -425,7 +427,7 @@ extern "C" eatss_status eatss_select_tiles(const eatss_kernel_desc *d, const eat
             if (dm.empty()) dm.push_back(16);
             s.dom.push_back(dm);
         }
-    } else if (o->mode == 2) {
+    } else if (o->mode == 2 || o->mode == 3) {
         // tensor-core mode: depth-3 nests with one serial loop and a parallel l_s1 only
         for (const NestEval &ne : s.nests) {
             int serial = 0;
@@ -434,7 +436,8 @@ extern "C" eatss_status eatss_select_tiles(const eatss_kernel_desc *d, const eat
                 return fail(EATSS_E_UNSUPPORTED, "eatss_select_tiles: tensor mode needs depth-3 contraction nests");
         }
         s.tensor = true;
-        s.esz = e;
+        s.f16 = o->mode == 3;
+        s.esz = s.f16 ? 2 : e;
         s.smem_cap = g->max_smem_per_block;
         const Nest &n0 = d->nests[0];
         for (int p = 0; p < s.L; p++) {
@@ -445,7 +448,7 @@ extern "C" eatss_status eatss_select_tiles(const eatss_kernel_desc *d, const eat
             } else if (n0.loops[p].parallel) {
                 dm = {128, 256};  // UMMA M rows: one CTA (cta_group::1) or a CTA pair (cta_group::2)
             } else {
-                dm = {32, 64};  // k per stage: whole 128-byte swizzle atoms of fp32
+                dm = s.f16 ? std::vector<int64_t>{64, 128} : std::vector<int64_t>{32, 64};  // whole 128-byte atoms
             }
             s.dom.push_back(dm);
         }

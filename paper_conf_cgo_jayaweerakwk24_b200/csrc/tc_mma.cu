@@ -32,6 +32,7 @@
 //   warps 4..19 epilogue: tcgen05.ld of each finished chunk into fp32 registers, then C (16 warps:
 //           a drain of Tj/4 columns per warp keeps short chunks cheap).
 #include <cuda.h>
+#include <cuda_fp16.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -77,6 +78,8 @@ struct Args {
     int nunits;   // nfull + (T - nfull) * sp
     int nkb;      // k-blocks of Tk
     int group_rows;  // tile-order grouping (row groups per group) for L2 reuse
+    const int *__restrict__ rexp;  // 3xFP16 engine: power-of-two exponent of each row of A (scale 2^rexp)
+    const int *__restrict__ cexp;  // ... of each column of B
     unsigned long long *prof;  // development (EATSS_TCM_PROF): per-site cycle counters, else nullptr
     int dbg;  // -DEATSS_DEVTOOLS builds only (EATSS_TCM_DBG; results then wrong): 1 no TMEM drain,
               // 4 no accumulator reset at chunk starts
@@ -112,30 +115,37 @@ __device__ __forceinline__ Unit unit_of(const Args &p, int u) {
     return w;
 }
 
-// K-major operand (rows x Tk of fp32, TMA box inner = min(Tk, 32) elements): swizzle span in bytes,
-// UMMA layout type, and the descriptor of 8-k step ks (atoms of 32 k are rows*128 bytes apart)
-template <int BK>
+// K-major operand rows of BKB bytes per stage (fp32: 4*Tk, fp16: 2*Tk; TMA box inner = min(BKB, 128) bytes):
+// swizzle span, UMMA layout type, and the descriptor of the 32-byte k step ks (one MMA: 8 tf32 / 16 fp16 k);
+// 128-byte atoms along k are rows*128 bytes apart
+template <int BKB>
 struct KMajor {
-    static constexpr int SW = BK >= 32 ? 128 : BK * 4;                    // bytes per swizzled row
+    static constexpr int SW = BKB >= 128 ? 128 : BKB;                     // bytes per swizzled row
     static constexpr uint32_t LAYOUT = SW == 128 ? 2u : SW == 64 ? 4u : 6u;  // SW128 / SW64 / SW32
-    static constexpr int NA = BK > 32 ? BK / 32 : 1;                      // 128-byte atoms along k
+    static constexpr int NA = BKB > 128 ? BKB / 128 : 1;                  // 128-byte atoms along k
     __device__ static uint64_t desc(const unsigned char *base, int rows, int ks) {
         const unsigned char *p = base + (ks / 4) * rows * 128 + (ks % 4) * 32;
         return desc_sw128(p, 16u, (uint32_t)(8 * SW), LAYOUT);
     }
 };
 
-template <int BK, bool TB, int CG>
+// BKB: bytes of k per operand row and stage; F16: 3xFP16 operands (K-major A and B, per-row / per-column
+// power-of-two scales undone in the epilogue), else 3xTF32
+template <int BKB, bool TB, int CG, bool F16>
 __global__ void __launch_bounds__(NTHREADS, 1)
     tc_mma_kernel(const __grid_constant__ CUtensorMap mAhi, const __grid_constant__ CUtensorMap mAlo,
                   const __grid_constant__ CUtensorMap mBhi, const __grid_constant__ CUtensorMap mBlo, const Args p) {
     extern __shared__ __align__(1024) unsigned char smem_raw[];
     unsigned char *smem = smem_raw + ((1024u - (su32(smem_raw) & 1023u)) & 1023u);  // stays a shared pointer
-    using KA = KMajor<BK>;
+    using KA = KMajor<BKB>;
+    constexpr int ESZ = F16 ? 2 : 4;      // operand element bytes
+    constexpr int BK = BKB / ESZ;         // k per stage (elements)
+    constexpr int KA_E = 128 / ESZ;       // k per 128-byte atom (elements)
+    static_assert(!F16 || TB, "the 3xFP16 engine stages B K-major (transposed by its prep pass)");
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const uint32_t rank = CG == 2 ? cta_rank() : 0u;
     const int cid = (int)blockIdx.x / CG, ncl = (int)gridDim.x / CG;
-    constexpr int A_BYTES = BM * BK * 4;  // one A half (hi or lo) per stage
+    constexpr int A_BYTES = BM * BKB;  // one A half (hi or lo) per stage
     const int BNH = p.BNH, B_BYTES = p.b_bytes, STAGE = p.stage;
     const int R = p.R;
     uint64_t *full = reinterpret_cast<uint64_t *>(smem + (size_t)p.S * STAGE);
@@ -192,15 +202,15 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                     const int k0 = kb * BK;
 #pragma unroll
                     for (int a = 0; a < KA::NA; a++) {
-                        tma_2d<CG>(st + a * BM * 128, &mAhi, k0 + 32 * a, i0, fb);
-                        tma_2d<CG>(st + A_BYTES + a * BM * 128, &mAlo, k0 + 32 * a, i0, fb);
+                        tma_2d<CG>(st + a * BM * 128, &mAhi, k0 + KA_E * a, i0, fb);
+                        tma_2d<CG>(st + A_BYTES + a * BM * 128, &mAlo, k0 + KA_E * a, i0, fb);
                     }
                     unsigned char *sb = st + 2 * A_BYTES;
                     if constexpr (TB) {
 #pragma unroll
                         for (int a = 0; a < KA::NA; a++) {
-                            tma_2d<CG>(sb + a * BNH * 128, &mBhi, k0 + 32 * a, jb, fb);
-                            tma_2d<CG>(sb + B_BYTES + a * BNH * 128, &mBlo, k0 + 32 * a, jb, fb);
+                            tma_2d<CG>(sb + a * BNH * 128, &mBhi, k0 + KA_E * a, jb, fb);
+                            tma_2d<CG>(sb + B_BYTES + a * BNH * 128, &mBlo, k0 + KA_E * a, jb, fb);
                         }
                     } else {
                         for (int g = 0; g < p.bgroups; g++) {
@@ -236,7 +246,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                     const unsigned char *sb = st + 2 * A_BYTES;
                     const uint32_t d = tmem + (uint32_t)(bd * 256);
 #pragma unroll
-                    for (int ks = 0; ks < BK / 8; ks++) {
+                    for (int ks = 0; ks < BKB / 32; ks++) {
                         const uint64_t ahi = KA::desc(st, BM, ks);
                         const uint64_t alo = KA::desc(st + A_BYTES, BM, ks);
                         uint64_t bhi, blo;
@@ -247,9 +257,15 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                             bhi = desc_sw128(sb + ks * 1024, (uint32_t)(BK * 128), 512u, 1);
                             blo = desc_sw128(sb + B_BYTES + ks * 1024, (uint32_t)(BK * 128), 512u, 1);
                         }
-                        mma_ss<CG>(d, ahi, bhi, ID, (first && ks == 0) ? 0u : 1u);
-                        mma_ss<CG>(d, ahi, blo, ID, 1u);
-                        mma_ss<CG>(d, alo, bhi, ID, 1u);
+                        if constexpr (F16) {
+                            mma_ss_f16<CG>(d, ahi, bhi, ID, (first && ks == 0) ? 0u : 1u);
+                            mma_ss_f16<CG>(d, ahi, blo, ID, 1u);
+                            mma_ss_f16<CG>(d, alo, bhi, ID, 1u);
+                        } else {
+                            mma_ss<CG>(d, ahi, bhi, ID, (first && ks == 0) ? 0u : 1u);
+                            mma_ss<CG>(d, ahi, blo, ID, 1u);
+                            mma_ss<CG>(d, alo, bhi, ID, 1u);
+                        }
                     }
                     mma_commit<CG>(empty + s);
                     if ((x % R) == R - 1 || x == nk - 1) {
@@ -311,6 +327,14 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             // C(i, j) for row i = i0 + 32q + lane, columns jb .. jb + CW - 1
             const int64_t i = (int64_t)(w.pi * CG + (int)rank) * BM + q * 32 + lane;
             const int64_t jb = (int64_t)w.tj * p.BNT + cq * CW;
+            if constexpr (F16) {  // undo the power-of-two row / column scales: acc * 2^-(rexp_i + cexp_j), exact
+                if (i < p.M && jb < p.N) {
+                    const float fr = __int_as_float((127 - p.rexp[i]) << 23);
+#pragma unroll
+                    for (int c = 0; c < MAXCW; c++)
+                        if (c < CW && jb + c < p.N) acc[c] = (acc[c] * fr) * __int_as_float((127 - __ldg(p.cexp + jb + c)) << 23);
+                }
+            }
             if (i < p.M && jb < p.N) {
                 float *crow = p.C + i * p.ldc + jb;
                 const bool vec = ((p.ldc & 3) == 0) && (jb + CW <= p.N);
@@ -487,6 +511,134 @@ __global__ void __launch_bounds__(256) prep_kernel(const SplitJob j0, const Spli
     }
 }
 
+
+// ------------------------------------------------------------------ 3xFP16 operand split
+// x = a * 2^-s with a = x * 2^s, s chosen per row (A) / per column (B) so that max|a| lies in [2^14, 2^15):
+// hi = rn_f16(a), lo = rn_f16(a - hi) -- a - hi is exact in fp32 -- so hi + lo carries 22 significant
+// bits of a (the same as tf32 hi + lo) and fp16's range is never exceeded; the GEMM accumulates
+// hi*hi + hi*lo + lo*hi in fp32 and its epilogue multiplies by 2^-(s_i + u_j) (exact).
+__device__ __forceinline__ int f16_scale_exp(float m) {
+    if (!(m > 0.f)) return 0;
+    int e;
+    frexpf(m, &e);  // m = f * 2^e, f in [0.5, 1)  ->  m * 2^(15 - e) in [2^14, 2^15)
+    return max(-100, min(100, 15 - e));
+}
+__device__ __forceinline__ void f16_split(float x, float sc, __half &h, __half &l) {
+    const float a = x * sc;
+    h = __float2half_rn(a);
+    l = __float2half_rn(a - __half2float(h));
+}
+struct F16Rows {  // rows x cols fp32 (pitch ldx) -> hi / lo fp16 [rows][ldp], exps[rows]
+    const float *x;
+    int64_t rows, cols, ldx, ldp;
+    __half *hi, *lo;
+    int *exps;
+};
+struct F16Cols {  // K x N fp32 (pitch ldx) -> transposed hi / lo fp16 [N][ldp] (K-major), exps[N]
+    const float *x;
+    int64_t K, N, ldx, ldp;
+    __half *hi, *lo;
+    int *exps;
+};
+// one warp per row: the row's max, then the scaled split (second read from L1 / L2)
+__device__ void f16_rows_body(const F16Rows &j, int64_t w0, int64_t wstride) {
+    const int lane = threadIdx.x & 31;
+    for (int64_t r = w0; r < j.rows; r += wstride) {
+        const float *xr = j.x + r * j.ldx;
+        float m = 0.f;
+        for (int64_t c = lane; c < j.cols; c += 32) m = fmaxf(m, fabsf(xr[c]));
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+        const int s = f16_scale_exp(m);
+        if (lane == 0) j.exps[r] = s;
+        const float sc = __int_as_float((127 + s) << 23);
+        __half *hr = j.hi + r * j.ldp, *lr = j.lo + r * j.ldp;
+        for (int64_t c = 2 * lane; c < j.ldp; c += 64) {
+            __half h0, l0, h1, l1;
+            f16_split(c < j.cols ? xr[c] : 0.f, sc, h0, l0);
+            f16_split(c + 1 < j.cols ? xr[c + 1] : 0.f, sc, h1, l1);
+            *reinterpret_cast<__half2 *>(hr + c) = __halves2half2(h0, h1);
+            *reinterpret_cast<__half2 *>(lr + c) = __halves2half2(l0, l1);
+        }
+    }
+}
+// one CTA (256 threads) per 32-column strip: column maxima, then 64 x 32 tiles transposed through shared
+// memory so both the reads (along j) and the fp16 writes (along k) are coalesced
+__device__ void f16_cols_body(const F16Cols &j, int64_t strip) {
+    __shared__ float t[64][33];
+    __shared__ float red[8][32];
+    __shared__ float sc[32];
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    const int64_t j0 = strip * 32, col = j0 + lane;
+    float m = 0.f;
+    if (col < j.N)
+        for (int64_t k = w; k < j.K; k += 8) m = fmaxf(m, fabsf(j.x[k * j.ldx + col]));
+    red[w][lane] = m;
+    __syncthreads();
+    if (w == 0) {
+        for (int q = 1; q < 8; q++) m = fmaxf(m, red[q][lane]);
+        const int s = f16_scale_exp(m);
+        if (col < j.N) j.exps[col] = s;
+        sc[lane] = __int_as_float((127 + s) << 23);
+    }
+    __syncthreads();
+    for (int64_t k0 = 0; k0 < j.K; k0 += 64) {
+        for (int e = tid; e < 64 * 32; e += 256) {
+            const int kk = e >> 5, jj = e & 31;
+            t[kk][jj] = (k0 + kk < j.K && j0 + jj < j.N) ? j.x[(k0 + kk) * j.ldx + j0 + jj] : 0.f;
+        }
+        __syncthreads();
+        for (int e = tid; e < 32 * 32; e += 256) {  // (column jj, k pair kp)
+            const int jj = e >> 5, kp = e & 31;
+            if (j0 + jj < j.N && k0 + 2 * kp < j.ldp) {
+                __half h0, l0, h1, l1;
+                f16_split(t[2 * kp][jj], sc[jj], h0, l0);
+                f16_split(t[2 * kp + 1][jj], sc[jj], h1, l1);
+                const int64_t o = (j0 + jj) * j.ldp + k0 + 2 * kp;
+                *reinterpret_cast<__half2 *>(j.hi + o) = __halves2half2(h0, h1);
+                *reinterpret_cast<__half2 *>(j.lo + o) = __halves2half2(l0, l1);
+            }
+        }
+        __syncthreads();
+    }
+}
+// One launch before the 3xFP16 GEMM: blocks [0, nbr) split the row operands (A, and B when it is K-major
+// -- syrk), [nbr, nbr + nbc) the column strips of a row-major B, the rest the split-k tail pre-pass.
+__global__ void __launch_bounds__(256) prep_f16_kernel(const F16Rows r0, const F16Rows r1, const F16Cols cj, int nbr,
+                                                       int nbc, const Args p, int rows_per_tile, int bn, int vecC) {
+    const int b = (int)blockIdx.x;
+    if (b < nbr) {
+        const int64_t wstride = (int64_t)nbr * 8, w0 = (int64_t)b * 8 + (threadIdx.x >> 5);
+        if (r0.x) f16_rows_body(r0, w0, wstride);
+        if (r1.x) f16_rows_body(r1, w0, wstride);
+        return;
+    }
+    if (b < nbr + nbc) {
+        for (int64_t st = b - nbr; st < (cj.N + 31) / 32; st += nbc) f16_cols_body(cj, st);
+        return;
+    }
+    const int npb = (int)gridDim.x - nbr - nbc, g4 = (bn + 3) / 4;
+    const int64_t total = (int64_t)(p.T - p.nfull) * rows_per_tile * g4;
+    for (int64_t e = (int64_t)(b - nbr - nbc) * blockDim.x + threadIdx.x; e < total; e += (int64_t)npb * blockDim.x) {
+        const int64_t rowid = e / g4;
+        const int x = (int)(e % g4);
+        const int t = p.nfull + (int)(rowid / rows_per_tile), r = (int)(rowid % rows_per_tile);
+        int pi, tj;
+        tile_coords(t, p.PI, p.TJ, p.group_rows, pi, tj);
+        const int64_t i = (int64_t)pi * rows_per_tile + r, j = (int64_t)tj * bn + 4 * x;
+        if (i >= p.M || j >= p.N) continue;
+        float *c = p.C + i * p.ldc + j;
+        if (vecC && j + 3 < p.N) {
+            float4 v = *reinterpret_cast<float4 *>(c);
+            v = p.init_zero ? make_float4(0.f, 0.f, 0.f, 0.f)
+                            : make_float4(p.beta * v.x, p.beta * v.y, p.beta * v.z, p.beta * v.w);
+            *reinterpret_cast<float4 *>(c) = v;
+        } else {
+            for (int q = 0; q < 4 && j + q < p.N; q++) c[q] = p.init_zero ? 0.f : p.beta * c[q];
+        }
+    }
+}
+
 // ------------------------------------------------------------------ host side
 }  // namespace tcm
 
@@ -495,6 +647,10 @@ __global__ void __launch_bounds__(256) prep_kernel(const SplitJob j0, const Spli
 struct Prep {
     tcm::SplitJob j0{}, j1{};
     int nb0 = 0, nb1 = 0, mode = 1;
+    // 3xFP16: row splits (A; B when K-major) and the column strips of a row-major B
+    tcm::F16Rows r0{}, r1{};
+    tcm::F16Cols cj{};
+    int nbr = 0, nbc = 0;
 };
 
 // Geometry of one tile vector on this engine (shared by applicability, workspace and launch).
@@ -502,21 +658,24 @@ struct TcmGeom {
     bool ok = false;
     int bk = 0, bn = 0, cg = 1, bnh = 0, bgroups = 0, a_bytes = 0, b_bytes = 0, stage = 0, S = 0, smem = 0;
 };
-static TcmGeom tcm_geom(const ContractNest &n, const ContractPlan &p) {
+// f16: the 3xFP16 engine (operands 2 bytes, B always K-major after its transposing split)
+static TcmGeom tcm_geom(const ContractNest &n, const ContractPlan &p, bool f16 = false) {
     TcmGeom g;
     const int64_t Ti = p.rTi, Tj = p.rTj, Tk = p.rTk;
     if (n.f64 || (Ti != 128 && Ti != 256)) return g;
     if (Tj < 16 || Tj > tcm::MAXBN || Tj % 16) return g;
-    if (Tk != 8 && Tk != 16 && Tk != 32 && Tk != 64) return g;
+    const int esz = f16 ? 2 : 4;
+    if (Tk * esz != 32 && Tk * esz != 64 && Tk * esz != 128 && Tk * esz != 256) return g;  // bytes per stage row
     if (n.M > INT32_MAX / 2 || n.N > INT32_MAX / 2 || n.K > INT32_MAX / 2) return g;
+    const bool kmaj_b = n.transB || f16;
     g.bk = (int)Tk;
     g.bn = (int)Tj;
     g.cg = Ti == 256 ? 2 : 1;           // Ti = 256: a CTA pair (cta_group::2) per tile
     g.bnh = g.bn / g.cg;
-    if (g.bnh % (n.transB ? 8 : 16)) return g;  // UMMA N per CTA half: K-major rows in 8s, MN-major in 16s
+    if (g.bnh % (kmaj_b ? 8 : 16)) return g;  // UMMA N per CTA half: K-major rows in 8s, MN-major in 16s
     g.bgroups = (g.bnh + 31) / 32;
-    g.a_bytes = tcm::BM * g.bk * 4;
-    g.b_bytes = n.transB ? g.bnh * g.bk * 4 : g.bgroups * 32 * g.bk * 4;
+    g.a_bytes = tcm::BM * g.bk * esz;
+    g.b_bytes = kmaj_b ? g.bnh * g.bk * esz : g.bgroups * 32 * g.bk * esz;
     g.stage = 2 * g.a_bytes + 2 * g.b_bytes;
     static const int env_s = devsw("EATSS_TCM_STAGES", 0);  // development
     g.S = std::min(8, (232448 - 2048) / g.stage);
@@ -527,7 +686,7 @@ static TcmGeom tcm_geom(const ContractNest &n, const ContractPlan &p) {
     return g;
 }
 
-bool tcm_applicable(const ContractNest &n, const ContractPlan &p) { return tcm_geom(n, p).ok; }
+bool tcm_applicable(const ContractNest &n, const ContractPlan &p, bool f16) { return tcm_geom(n, p, f16).ok; }
 
 // Persistent schedule: full tiles in waves of ncl clusters, the last partial wave split along k
 // into sp parts (so idle clusters take k-slices instead of waiting).  nsm / CG clusters of one
@@ -561,10 +720,10 @@ std::mutex g_ks_mu;
 std::map<std::pair<const void *, int>, KernelState> g_ks;
 }  // namespace
 
-template <int BK, bool TB, int CG>
+template <int BKB, bool TB, int CG, bool F16>
 static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int nsm, const Prep &pr, cudaStream_t s,
                               cudaEvent_t *ev) {
-    auto k = tcm::tc_mma_kernel<BK, TB, CG>;
+    auto k = tcm::tc_mma_kernel<BKB, TB, CG, F16>;
     int dev = 0;
     cudaGetDevice(&dev);
     int ncl = nsm / CG;
@@ -604,8 +763,12 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
         const int64_t tail4 = needs_prepass(a) ? (int64_t)(a.T - a.nfull) * rows * ((a.BNT + 3) / 4) : 0;
         const int npb = (int)std::min<int64_t>((tail4 + 255) / 256, (int64_t)nsm * 4);
         const int vecC = (a.ldc % 4 == 0 && (reinterpret_cast<uintptr_t>(a.C) & 15) == 0) ? 1 : 0;
-        tcm::prep_kernel<<<pr.nb0 + pr.nb1 + npb, 256, 0, s>>>(pr.j0, pr.j1, pr.nb0, pr.nb1, pr.mode, a, rows, a.BNT,
-                                                               vecC);
+        if constexpr (F16)
+            tcm::prep_f16_kernel<<<pr.nbr + pr.nbc + npb, 256, 0, s>>>(pr.r0, pr.r1, pr.cj, pr.nbr, pr.nbc, a, rows,
+                                                                       a.BNT, vecC);
+        else
+            tcm::prep_kernel<<<pr.nb0 + pr.nb1 + npb, 256, 0, s>>>(pr.j0, pr.j1, pr.nb0, pr.nb1, pr.mode, a, rows,
+                                                                   a.BNT, vecC);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
     }
     cfg.gridDim = dim3((unsigned)(CG * ncl));
@@ -615,14 +778,14 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
     return e;
 }
 
-template <bool TB, int CG>
-static cudaError_t launch_bk(int bk, const CUtensorMap *m, const tcm::Args &a, int smem, int nsm, const Prep &pr,
+template <bool TB, int CG, bool F16>
+static cudaError_t launch_bk(int bkb, const CUtensorMap *m, const tcm::Args &a, int smem, int nsm, const Prep &pr,
                              cudaStream_t s, cudaEvent_t *ev) {
-    switch (bk) {
-        case 8: return launch_one<8, TB, CG>(m, a, smem, nsm, pr, s, ev);
-        case 16: return launch_one<16, TB, CG>(m, a, smem, nsm, pr, s, ev);
-        case 32: return launch_one<32, TB, CG>(m, a, smem, nsm, pr, s, ev);
-        case 64: return launch_one<64, TB, CG>(m, a, smem, nsm, pr, s, ev);
+    switch (bkb) {  // bytes of k per operand row and stage
+        case 32: return launch_one<32, TB, CG, F16>(m, a, smem, nsm, pr, s, ev);
+        case 64: return launch_one<64, TB, CG, F16>(m, a, smem, nsm, pr, s, ev);
+        case 128: return launch_one<128, TB, CG, F16>(m, a, smem, nsm, pr, s, ev);
+        case 256: return launch_one<256, TB, CG, F16>(m, a, smem, nsm, pr, s, ev);
         default: return cudaErrorNotSupported;
     }
 }
@@ -750,11 +913,15 @@ cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p,
         cudaMemsetAsync(prof, 0, 16 * sizeof(unsigned long long), s);
         a.prof = prof;
     }
+    a.rexp = a.cexp = nullptr;
     cudaError_t r;
+    const int bkb = 4 * bk;
     if (n.transB)
-        r = cg == 2 ? launch_bk<true, 2>(bk, m, a, g.smem, nsm, pr, s, ev) : launch_bk<true, 1>(bk, m, a, g.smem, nsm, pr, s, ev);
+        r = cg == 2 ? launch_bk<true, 2, false>(bkb, m, a, g.smem, nsm, pr, s, ev)
+                    : launch_bk<true, 1, false>(bkb, m, a, g.smem, nsm, pr, s, ev);
     else
-        r = cg == 2 ? launch_bk<false, 2>(bk, m, a, g.smem, nsm, pr, s, ev) : launch_bk<false, 1>(bk, m, a, g.smem, nsm, pr, s, ev);
+        r = cg == 2 ? launch_bk<false, 2, false>(bkb, m, a, g.smem, nsm, pr, s, ev)
+                    : launch_bk<false, 1, false>(bkb, m, a, g.smem, nsm, pr, s, ev);
     if (a.prof) {
         unsigned long long h[16];
         cudaMemcpyAsync(h, a.prof, sizeof(h), cudaMemcpyDeviceToHost, s);
@@ -766,6 +933,106 @@ cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p,
                 h[0] / nmma, h[1] / nmma, h[2] / (double)h[4], h[3] / (double)h[4], h[4], h[5] / (double)h[6], h[6]);
     }
     return r;
+}
+
+// ------------------------------------------------------------------ 3xFP16 engine (engine = TENSOR_F16)
+namespace {
+struct F16Layout {  // workspace offsets (bytes, 256-aligned): hi/lo fp16 operands and their exponents
+    int64_t Kp = 0;
+    size_t a_hi = 0, a_lo = 0, a_exp = 0, b_hi = 0, b_lo = 0, b_exp = 0, total = 0;
+    bool share = false;  // syrk: A is a row block of the K-major B
+};
+F16Layout f16_layout(const ContractNest &n) {
+    F16Layout L;
+    const float *A = static_cast<const float *>(n.A), *B = static_cast<const float *>(n.B);
+    L.Kp = (n.K + 7) / 8 * 8;  // 16-byte fp16 rows (TMA strides)
+    L.share = n.transB && n.lda == n.ldb && A >= B && (A - B) % n.ldb == 0 && (A - B) / n.ldb + n.M <= n.N;
+    auto al = [](size_t v) { return (v + 255) / 256 * 256; };
+    size_t o = 0;
+    L.b_hi = o; o = al(o + (size_t)n.N * L.Kp * 2);
+    L.b_lo = o; o = al(o + (size_t)n.N * L.Kp * 2);
+    L.b_exp = o; o = al(o + (size_t)n.N * 4);
+    if (!L.share) {
+        L.a_hi = o; o = al(o + (size_t)n.M * L.Kp * 2);
+        L.a_lo = o; o = al(o + (size_t)n.M * L.Kp * 2);
+        L.a_exp = o; o = al(o + (size_t)n.M * 4);
+    }
+    L.total = o;
+    return L;
+}
+}  // namespace
+
+bool tcf_applicable(const ContractNest &n, const ContractPlan &p) { return tcm_geom(n, p, true).ok; }
+size_t tcf_ws_floats(const ContractNest &n, const ContractPlan &) { return f16_layout(n).total / 4 + 64; }
+
+cudaError_t launch_tcf_contraction(const ContractNest &n, const ContractPlan &p, float *ws, size_t ws_floats,
+                                   cudaStream_t s, cudaEvent_t *ev) {
+    const TcmGeom g = tcm_geom(n, p, true);
+    if (!g.ok) return cudaErrorNotSupported;
+    const F16Layout L = f16_layout(n);
+    if (!ws || ws_floats * 4 < L.total) return cudaErrorInvalidValue;
+    char *w = reinterpret_cast<char *>(ws);
+    const float *A = static_cast<const float *>(n.A), *B = static_cast<const float *>(n.B);
+    __half *bhi = reinterpret_cast<__half *>(w + L.b_hi), *blo = reinterpret_cast<__half *>(w + L.b_lo);
+    int *bexp = reinterpret_cast<int *>(w + L.b_exp);
+    const __half *ahi, *alo;
+    const int *aexp;
+    Prep pr;
+    int dev = 0, nsm = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    if (n.transB) {  // B(k, j) = B[j*ldb + k]: rows j are already K-major -> row split, row scale = column scale
+        pr.r0 = tcm::F16Rows{B, n.N, n.K, n.ldb, L.Kp, bhi, blo, bexp};
+    } else {  // row-major B[k][j]: column strips, transposed to K-major
+        pr.cj = tcm::F16Cols{B, n.K, n.N, n.ldb, L.Kp, bhi, blo, bexp};
+        pr.nbc = (int)std::min<int64_t>((n.N + 31) / 32, (int64_t)nsm * 2);
+    }
+    if (L.share) {
+        const int64_t r = (A - B) / n.ldb;
+        ahi = bhi + r * L.Kp;
+        alo = blo + r * L.Kp;
+        aexp = bexp + r;
+    } else {
+        __half *h = reinterpret_cast<__half *>(w + L.a_hi), *l = reinterpret_cast<__half *>(w + L.a_lo);
+        int *e = reinterpret_cast<int *>(w + L.a_exp);
+        (n.transB ? pr.r1 : pr.r0) = tcm::F16Rows{A, n.M, n.K, n.lda, L.Kp, h, l, e};
+        ahi = h;
+        alo = l;
+        aexp = e;
+    }
+    pr.nbr = nsm * 4;
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return e;
+    CUtensorMap m[4];
+    const int bkb = g.bk * 2, kbytes = std::min(bkb, 128), kbox = kbytes / 2;
+    const CUtensorMapSwizzle sw = kbytes == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
+                                  : kbytes == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
+                                                 : CU_TENSOR_MAP_SWIZZLE_32B;
+    const bool ok = tcm::make_map(&m[0], ahi, n.M, n.K, L.Kp, kbox, tcm::BM, sw, true) &&
+                    tcm::make_map(&m[1], alo, n.M, n.K, L.Kp, kbox, tcm::BM, sw, true) &&
+                    tcm::make_map(&m[2], bhi, n.N, n.K, L.Kp, kbox, g.bnh, sw, true) &&
+                    tcm::make_map(&m[3], blo, n.N, n.K, L.Kp, kbox, g.bnh, sw, true);
+    if (!ok) return cudaErrorInvalidValue;
+    tcm::Args a;
+    a.M = n.M; a.N = n.N; a.K = n.K;
+    a.C = static_cast<float *>(n.C); a.ldc = n.ldc;
+    a.alpha = (float)n.alpha; a.beta = (float)n.beta; a.init_zero = n.init_zero ? 1 : 0;
+    a.S = g.S;
+    static const int chunk_env = devsw("EATSS_TCM_CHUNK_K", 0);  // development: k per accumulator chunk
+    a.R = std::max(1, (chunk_env > 0 ? chunk_env : tcm::CHUNK_K) / g.bk);
+    a.BNT = g.bn; a.BNH = g.bnh; a.bgroups = g.bgroups; a.b_bytes = g.b_bytes; a.stage = g.stage;
+    a.idesc = tcm::idesc_f16(g.bn, g.cg);
+    a.nkb = (int)((n.K + g.bk - 1) / g.bk);
+    a.PI = (int)((n.M + g.cg * tcm::BM - 1) / (g.cg * tcm::BM));
+    a.TJ = (int)((n.N + g.bn - 1) / g.bn);
+    static const int group_env = devsw("EATSS_TCM_GROUP", 8);
+    a.group_rows = std::max(1, group_env);
+    a.prof = nullptr;
+    a.dbg = 0;
+    a.rexp = aexp;
+    a.cexp = bexp;
+    return g.cg == 2 ? launch_bk<true, 2, true>(bkb, m, a, g.smem, nsm, pr, s, ev)
+                     : launch_bk<true, 1, true>(bkb, m, a, g.smem, nsm, pr, s, ev);
 }
 
 int tcm_launches(const ContractNest &, const ContractPlan &) {

@@ -139,6 +139,22 @@ __device__ __forceinline__ void mma_ss(uint32_t d, uint64_t a, uint64_t b, uint3
             "l"(a), "l"(b), "r"(idesc), "r"(acc)
             : "memory");
 }
+// D[tmem] (+)= A[smem desc] * B[smem desc], kind::f16 (fp16 operands, fp32 accumulation)
+template <int CG>
+__device__ __forceinline__ void mma_ss_f16(uint32_t d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
+    if constexpr (CG == 1)
+        asm volatile(
+            "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
+            "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(d),
+            "l"(a), "l"(b), "r"(idesc), "r"(acc)
+            : "memory");
+    else
+        asm volatile(
+            "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
+            "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(d),
+            "l"(a), "l"(b), "r"(idesc), "r"(acc)
+            : "memory");
+}
 // arrive on `bar` (same smem offset in every CTA of the pair for CG = 2) when all prior MMAs finish
 template <int CG>
 __device__ __forceinline__ void mma_commit(uint64_t *bar) {
@@ -170,6 +186,11 @@ __device__ __forceinline__ uint64_t desc_sw128(const void *p, uint32_t lbo, uint
 __host__ __device__ constexpr uint32_t idesc(int n, int cg, bool kmajor_b) {
     return (1u << 4) | (2u << 7) | (2u << 10) | (kmajor_b ? 0u : (1u << 16)) | ((uint32_t)(n >> 3) << 17) |
            ((uint32_t)((128 * cg) >> 4) << 24);
+}
+
+// kind::f16 instruction descriptor: D f32, A and B fp16, both K-major, M = 128 * CG, N = n
+__host__ __device__ constexpr uint32_t idesc_f16(int n, int cg) {
+    return (1u << 4) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)((128 * cg) >> 4) << 24);
 }
 
 // ---- TMA with more dimensions, TMA stores, async-proxy fences, named barriers
@@ -258,17 +279,18 @@ inline EncodeTiled encode_fn() {
     return fn;
 }
 
-// 2-D fp32 row-major [rows][cols] (row pitch `ld` elements), box {bc cols (inner), br rows}
-inline bool make_map(CUtensorMap *m, const float *base, int64_t rows, int64_t cols, int64_t ld, int bc, int br,
-                     CUtensorMapSwizzle sw) {
+// 2-D row-major [rows][cols] of fp32 (or fp16 with f16 = true; row pitch `ld` elements), box {bc cols
+// (inner), br rows}
+inline bool make_map(CUtensorMap *m, const void *base, int64_t rows, int64_t cols, int64_t ld, int bc, int br,
+                     CUtensorMapSwizzle sw, bool f16 = false) {
     EncodeTiled enc = encode_fn();
     if (!enc) return false;
     cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
-    cuuint64_t strides[1] = {(cuuint64_t)(ld * 4)};
+    cuuint64_t strides[1] = {(cuuint64_t)(ld * (f16 ? 2 : 4))};
     cuuint32_t box[2] = {(cuuint32_t)bc, (cuuint32_t)br};
     cuuint32_t es[2] = {1, 1};
-    return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float *>(base), dims, strides, box, es,
-               CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+    return enc(m, f16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<void *>(base),
+               dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 

@@ -51,6 +51,11 @@ add("syrk", (4000, 4000), 4, "B200", 50, 16, 2)
 add("gemm", (100, 40, 20), 4, "B200", 50, 16, 2)
 add("gemm", (300, 1100, 204), 4, "B200", 50, 16, 2)
 add("gemm", (4000, 4000, 4000), 4, "GA100", 50, 16, 2)
+# tensor-core mode of the 3xFP16 engine (mode 3: 2-byte operands, K-major B, Tk in {64, 128})
+add("gemm", (4000, 4000, 4000), 4, "B200", 50, 16, 3)
+add("syrk", (4000, 4000), 4, "B200", 50, 16, 3)
+add("3mm", (4000, 4000, 4000, 4000, 4000), 4, "B200", 50, 16, 3)
+add("gemm", (100, 40, 20), 4, "B200", 50, 16, 3)
 add("ccsd_t_d1", (48,), 4, "B200", 50, 4, 2)   # reading T4
 add("ccsd_t_d1", (16,), 4, "B200", 50, 16, 2)
 add("ccsd_t_d1", (24,), 4, "B200", 50, 4, 2)

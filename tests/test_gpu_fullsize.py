@@ -19,8 +19,8 @@ pytestmark = pytest.mark.gpu
 E = pytest.importorskip("paper_conf_cgo_jayaweerakwk24_b200")
 
 N = 4000
-ENGINES = [(1, (16, 1024, 16)), (2, (256, 256, 32))]
-IDS = ["simt", "tensor"]
+ENGINES = [(1, (16, 1024, 16)), (2, (256, 256, 32)), (4, (256, 256, 64))]
+IDS = ["simt", "tensor", "tensor_f16"]
 
 
 def dev(x):

@@ -292,3 +292,15 @@ def test_tensor_mode_6d_hand_checked():
     assert r.tiles == (1, 2, 1, 48, 2, 48, 48) and r.obj == 9408 and r.n_ties == 2
     assert set(r.ties) == {(1, 2, 1, 48, 2, 48, 48), (1, 2, 2, 48, 1, 48, 48)}
     assert M.select_tiles(M.mttkrp(), M.B200, M.Opts(50, 16, 2)).tiles is None  # two reduction loops: no T4
+
+
+def test_tensor_mode_f16_hand_checked():
+    """Reading T, mode 3 (the 3xFP16 engine): 2-byte operands, B K-major (no 32-column rounding), Tk in
+    {64, 128}.  Per-CTA stage bytes x 2 stages = 2*2*2*(128*Tk + Tk*Tj/CG) <= 230400, i.e.
+    Tk*(128 + Tj/CG) <= 28800:  Tk = 64: Tj/CG <= 322 -> every Tj (16 for Ti = 128, 16 for Ti = 256
+    since Tj/2 is a multiple of 8); Tk = 128: Tj/CG <= 97 -> Ti = 128: Tj <= 96 (6), Ti = 256: Tj <= 192
+    (12).  n_feasible = 16 + 16 + 6 + 12 = 50.  OBJ = (Ti + 32)*Tj -> (256, 256, *); (256, 256, 128) needs
+    128*(128 + 128) = 32768 > 28800, so (256, 256, 64) is the unique optimum."""
+    r = M.select_tiles(M.gemm(), M.B200, M.Opts(50, 16, 3))
+    assert r.n_feasible == 50 and r.n_ties == 1 and r.tiles == (256, 256, 64) and r.obj == 288 * 256
+    assert M.select_tiles(M.ccsd_t_d1(48), M.B200, M.Opts(50, 4, 3)).tiles is None
