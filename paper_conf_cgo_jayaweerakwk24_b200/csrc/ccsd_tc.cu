@@ -67,6 +67,8 @@ struct Args {
     int x_bytes;      // t3 tile of a unit: Th2*Th1*Tp6*Tp5*Tp4*4
     int x_stage;      // x_bytes rounded up to 1 KB
     int XB;           // t3 tile buffers per epilogue group (2: the next owned unit is prefetched)
+    int XS;           // XB = 1 with Th2 = 2: the tile moves as two h2 slices (one TMA box and barrier each), so
+                      // the next owned unit's slice s is requested as soon as slice s has been processed
     int order;        // 1: A tiles round-robin over CTAs (concurrent CTAs sweep whole t3 blocks)
     int dbg;          // development only (EATSS_CCSD_TC_DBG): 1 no MMA, 2 no t3 traffic, 4 no v2 loads
     unsigned long long *prof;  // development only (EATSS_CCSD_TC_PROF): cycles per wait site
@@ -344,8 +346,24 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             int h1_0, p5_0, p4_0, c[5];
             a_coords(p, wn.a, h1_0, p5_0, p4_0);
             x_coords(p, wn.hh, wn.p6t, h1_0, p5_0, p4_0, c);
+            if (p.XS) {  // two h2 slices, barriers xb[0], xb[1]
+                const int sb = p.x_bytes / 2;
+                for (int q = 0; q < 2; q++) {
+                    mbar_expect_tx(xb + q, sb);
+                    tma_5d_hint(xbuf + (size_t)q * sb, &mX, c[0], c[1], c[2], c[3] + q, c[4], xb + q, pol);
+                }
+                return;
+            }
             mbar_expect_tx(xb + buf, p.x_bytes);
             tma_5d_hint(xbuf + (size_t)buf * p.x_stage, &mX, c[0], c[1], c[2], c[3], c[4], xb + buf, pol);
+        };
+        auto fetch_slice = [&](const UnitIter &wn, int q) {  // h2 slice q of unit wn -> its half of xbuf
+            int h1_0, p5_0, p4_0, c[5];
+            a_coords(p, wn.a, h1_0, p5_0, p4_0);
+            x_coords(p, wn.hh, wn.p6t, h1_0, p5_0, p4_0, c);
+            const int sb = p.x_bytes / 2;
+            mbar_expect_tx(xb + q, sb);
+            tma_5d_hint(xbuf + (size_t)q * sb, &mX, c[0], c[1], c[2], c[3] + q, c[4], xb + q, pol);
         };
         UnitIter w = iter_begin(p, sc), wn = w;  // wn: this group's next unit to prefetch
         for (int i = 0; i < g && i < sc.n; i++) iter_next(p, sc, wn);
@@ -353,7 +371,8 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         int a_prev = -1, na = 0, own = g, k = 0;  // own: units until this group's next unit; k: owned count
         bool rin = false;
         int64_t rowoff = 0;  // t3 offset of row m for hh = 0, p6 = 0
-        if (p.XB == 2 && leader && !(p.dbg & 2) && un < sc.n) fetch(wn, 0);  // XB = 1 fetches at unit start
+        // XB = 2: the first owned tile now; XS: its two slices now; XB = 1: at unit start
+        if ((p.XB == 2 || p.XS) && leader && !(p.dbg & 2) && un < sc.n) fetch(wn, 0);
         Ring rd;
         for (int64_t u = 0; u < sc.n; u++, iter_next(p, sc, w), rd.next(p.NB), own--) {
             const bool mine = own == 0;
@@ -394,11 +413,13 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             // next owned unit: its buffer was last read for unit k - 1 (XB = 2) -- the group barrier
             // orders those reads before the TMA overwrites it; XB = 1 fetches the current unit here
             for (int i = 0; i < NGRP && un < sc.n; i++, un++) iter_next(p, sc, wn);
-            named_bar(1 + g, 128);
-            if (p.XB == 2) {
-                if (leader && !(p.dbg & 2) && un < sc.n) fetch(wn, buf ^ 1);
-            } else if (leader && !(p.dbg & 2)) {
-                fetch(w, 0);
+            if (!p.XS) {
+                named_bar(1 + g, 128);
+                if (p.XB == 2) {
+                    if (leader && !(p.dbg & 2) && un < sc.n) fetch(wn, buf ^ 1);
+                } else if (leader && !(p.dbg & 2)) {
+                    fetch(w, 0);
+                }
             }
             // columns of this unit: hh = hhb + h2l (h2l < nh valid), p6 = p6b + c6 (c6 < np6 valid)
             int hhb, nh;
@@ -414,7 +435,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             float *const rowp = t3 + rowoff + (int64_t)hhb * s_hh + (int64_t)p6b * sp6;
             const float *xs = reinterpret_cast<const float *>(xbuf + (size_t)buf * p.x_stage) + xrow0;
             const bool io = rin && !(p.dbg & 2);
-            if (!(p.dbg & 2)) TWAIT(7, xb + buf, xph);
+            if (!(p.dbg & 2) && !p.XS) TWAIT(7, xb + buf, xph);
             if (p.prof && leader) atomicAdd(p.prof + 5, 1ull);
             TWAIT(3, dfull + rd.s, rd.ph);
             const long long tproc = p.prof ? clock64() : 0;
@@ -423,6 +444,13 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             constexpr int CH = 16;
             int h2l = 0, c6 = 0;
             for (int c0 = 0; c0 < p.NV; c0 += CH) {
+                if (p.XS && c6 == 0) {  // a new h2 slice: its t3 rows have landed (slice h2l, phase of unit k)
+                    if (h2l == 1) {  // slice 0 fully read by the group: request the next owned unit's slice 0
+                        named_bar(1 + g, 128);
+                        if (leader && !(p.dbg & 2) && un < sc.n) fetch_slice(wn, 0);
+                    }
+                    if (!(p.dbg & 2)) TWAIT(7, xb + h2l, (unsigned)(k & 1));
+                }
                 uint32_t v[CH];
                 tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0), *reinterpret_cast<uint32_t(*)[8]>(v));
                 tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0 + 8), *reinterpret_cast<uint32_t(*)[8]>(v + 8));
@@ -443,6 +471,10 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                 }
                 c6 += CH;
                 if (c6 == p.Tp6) { c6 = 0; h2l++; }
+            }
+            if (p.XS) {  // slice 1 read: request the next owned unit's slice 1
+                named_bar(1 + g, 128);
+                if (leader && !(p.dbg & 2) && un < sc.n) fetch_slice(wn, 1);
             }
             fence_before();
             __syncwarp();
@@ -535,6 +567,8 @@ CcsdTcPlan plan_ccsd_tc(const int64_t *dims, const int64_t *tiles) {
     static const int xb_env = getenv("EATSS_CCSD_TC_XB") ? atoi(getenv("EATSS_CCSD_TC_XB")) : 0;  // development
     if (xb_env > 0) a.XB = std::min(2, xb_env);
     a.SV = std::min(6, (budget - ccsdtc::NGRP * a.XB * a.x_stage) / a.v_stage);
+    static const int xs_env = getenv("EATSS_CCSD_TC_SLICES") ? atoi(getenv("EATSS_CCSD_TC_SLICES")) : 1;
+    a.XS = (a.XB == 1 && a.Th2 == 2 && xs_env != 0) ? 1 : 0;  // development: EATSS_CCSD_TC_SLICES=0 disables
     static const int sv_env = getenv("EATSS_CCSD_TC_VSTAGES") ? atoi(getenv("EATSS_CCSD_TC_VSTAGES")) : 0;
     if (sv_env > 0) a.SV = std::min(a.SV, sv_env);
     if (a.SV < 2) return pl;
@@ -586,7 +620,8 @@ cudaError_t launch_ccsd_tc(float *t3, const float *t2, const float *v2, const in
         const uint64_t d2[5] = {(uint64_t)(P5 * P4), (uint64_t)P6, (uint64_t)H1, (uint64_t)H2, (uint64_t)a.H3};
         const uint64_t s2[4] = {(uint64_t)(P5 * P4) * 4, (uint64_t)(P6 * P5 * P4) * 4, (uint64_t)(H1 * P6 * P5 * P4) * 4,
                                 (uint64_t)(H2 * H1 * P6 * P5 * P4) * 4};
-        const uint32_t b2[5] = {(uint32_t)(a.Tp5 * a.Tp4), (uint32_t)a.Tp6, (uint32_t)a.Th1, (uint32_t)a.Th2, 1};
+        const uint32_t b2[5] = {(uint32_t)(a.Tp5 * a.Tp4), (uint32_t)a.Tp6, (uint32_t)a.Th1,
+                                (uint32_t)(a.XS ? 1 : a.Th2), 1};  // XS: one h2 slice per box
         for (int i = 0; i < 5; i++) { xdims[i] = d2[i]; xbox[i] = b2[i]; }
         for (int i = 0; i < 4; i++) xstr[i] = s2[i];
     }
