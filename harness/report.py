@@ -19,17 +19,18 @@ import numpy as np
 
 
 def load(path):
-    meta, var, anc = None, [], {"anchor_default": [], "anchor_eatss": []}
+    """Records of a sweep JSONL; a tile measured again later (sweep.py --only) keeps its LAST record."""
+    meta, var, anc = None, {}, {"anchor_default": [], "anchor_eatss": []}
     for line in open(path):
         r = json.loads(line)
         k = r.get("kind")
         if k == "meta":
             meta = meta or r
         elif k == "variant":
-            var.append(r)
+            var[(tuple(r["tile"]), r.get("rank", 0))] = r
         elif k in anc:
             anc[k].append(r)
-    return meta, var, anc
+    return meta, list(var.values()), anc
 
 
 def summarise(path):

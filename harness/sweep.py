@@ -53,6 +53,8 @@ def parse():
     ap.add_argument("--no-parity", action="store_true")
     ap.add_argument("--tiles", default="", help="confirmation mode: 'a,b,c;d,e,f' measured --repeats times, interleaved")
     ap.add_argument("--repeats", type=int, default=5)
+    ap.add_argument("--only", default="", help="re-measure just these variants ('a,b,c;d,e,f') as variant records "
+                                               "(harness/report.py keeps the last record of a tile)")
     ap.add_argument("--dtype", choices=["f32", "f64"], default="f32",
                     help="f64: the paper's precision (P:117 FP_factor 2, P:202): model and executor in fp64")
     return ap.parse_args()
@@ -140,6 +142,8 @@ def main():
     random.Random(a.seed).shuffle(variants)
     if a.limit:
         variants = variants[: a.limit]
+    if a.only:
+        variants = [tuple(int(x) for x in t.split(",")) for t in a.only.split(";") if t]
     done = set()
     if a.resume and os.path.exists(a.resume):
         for line in open(a.resume):

@@ -202,14 +202,16 @@ extern "C" eatss_status eatss_sweep(const eatss_kernel_desc *d, const int64_t *v
         while (st == EATSS_OK) {
             pump();
             const double el = std::chrono::duration<double>(clk::now() - ta).count();
-            if (el >= min_window_s) {
+            // the window must contain at least one run launched after ta (a variant slower than the window
+            // would otherwise close it with only the runs queued before ta in flight: zero timed runs)
+            if (el >= min_window_s && launched > runs_a) {
                 if (!have_nvml) break;
                 nvml().energy(h, &cur);
                 if (cur != ea && cur != eb) {
                     if (eb == 0) eb = cur;  // first update after the minimum window closes it
                 }
                 if (eb != 0) break;
-                if (el > min_window_s + 2.0) break;  // counter stalled: give up on energy
+                if (el > min_window_s + 2.0 + 4.0 * ms1 * 1e-3) break;  // counter stalled: give up on energy
             }
             std::this_thread::sleep_for(std::chrono::microseconds(200));
         }
