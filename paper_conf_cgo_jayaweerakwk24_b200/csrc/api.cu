@@ -1237,7 +1237,7 @@ eatss_status eatss_coverage(const eatss_kernel_desc *d, int nest, const int64_t 
 
 int64_t eatss_launches_per_run(const eatss_kernel_desc *d, const int64_t *tiles) {
     if (!d) return -1;
-    if (is_contraction(d->kind) && d->exec.engine == EATSS_ENGINE_TENSOR_F16) {  // fused split + GEMM per nest
+    if (is_contraction(d->kind) && d->exec.engine == EATSS_ENGINE_TENSOR_F16) {
         if (!tiles || check_tiles(d, tiles) != EATSS_OK) return -1;
         void *b[EATSS_MAX_BUFFERS];
         for (int i = 0; i < EATSS_MAX_BUFFERS; i++) b[i] = (void *)((uintptr_t)(1 << 20) * (uintptr_t)(i + 1));
@@ -1245,7 +1245,7 @@ int64_t eatss_launches_per_run(const eatss_kernel_desc *d, const int64_t *tiles)
         for (auto &n : contraction_nests(d, b)) {
             ContractPlan p = plan_contraction(n, tiles, smem_limit_bytes(), d->exec.warp_align);
             if (!tcf_applicable(n, p)) return -1;
-            total += 2;
+            total += n.transB ? 2 : 3;  // (column maxima of a row-major B,) split + tail pre-pass, GEMM
         }
         return total;
     }

@@ -540,72 +540,112 @@ struct F16Cols {  // K x N fp32 (pitch ldx) -> transposed hi / lo fp16 [N][ldp] 
     __half *hi, *lo;
     int *exps;
 };
-// one warp per row: the row's max, then the scaled split (second read from L1 / L2)
+// one warp per row: the row's max, then the scaled split (second read from L1 / L2); 16-byte loads, four
+// in flight per lane (a row is 16 KB at K = 4000: the warp keeps 2 KB in flight)
 __device__ void f16_rows_body(const F16Rows &j, int64_t w0, int64_t wstride) {
     const int lane = threadIdx.x & 31;
     for (int64_t r = w0; r < j.rows; r += wstride) {
         const float *xr = j.x + r * j.ldx;
+        const bool v4 = ((j.ldx & 3) == 0) && ((reinterpret_cast<uintptr_t>(j.x) & 15) == 0);
+        const int64_t n4 = v4 ? j.cols / 4 : 0;
         float m = 0.f;
-        for (int64_t c = lane; c < j.cols; c += 32) m = fmaxf(m, fabsf(xr[c]));
+        for (int64_t c4 = lane; c4 < n4; c4 += 128) {
+            float4 v[4];
+#pragma unroll
+            for (int u = 0; u < 4; u++)
+                v[u] = c4 + 32 * u < n4 ? *reinterpret_cast<const float4 *>(xr + 4 * (c4 + 32 * u))
+                                        : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+            for (int u = 0; u < 4; u++)
+                m = fmaxf(m, fmaxf(fmaxf(fabsf(v[u].x), fabsf(v[u].y)), fmaxf(fabsf(v[u].z), fabsf(v[u].w))));
+        }
+        for (int64_t c = 4 * n4 + lane; c < j.cols; c += 32) m = fmaxf(m, fabsf(xr[c]));
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
         const int s = f16_scale_exp(m);
         if (lane == 0) j.exps[r] = s;
         const float sc = __int_as_float((127 + s) << 23);
         __half *hr = j.hi + r * j.ldp, *lr = j.lo + r * j.ldp;
-        for (int64_t c = 2 * lane; c < j.ldp; c += 64) {
-            __half h0, l0, h1, l1;
-            f16_split(c < j.cols ? xr[c] : 0.f, sc, h0, l0);
-            f16_split(c + 1 < j.cols ? xr[c + 1] : 0.f, sc, h1, l1);
-            *reinterpret_cast<__half2 *>(hr + c) = __halves2half2(h0, h1);
-            *reinterpret_cast<__half2 *>(lr + c) = __halves2half2(l0, l1);
+        // groups of 4 columns (ldp is a multiple of 8): 8-byte fp16 stores
+        for (int64_t c = 4 * lane; c < j.ldp; c += 128) {
+            float x[4];
+            if (v4 && c + 3 < j.cols) {
+                const float4 t = *reinterpret_cast<const float4 *>(xr + c);
+                x[0] = t.x; x[1] = t.y; x[2] = t.z; x[3] = t.w;
+            } else {
+#pragma unroll
+                for (int q = 0; q < 4; q++) x[q] = c + q < j.cols ? xr[c + q] : 0.f;
+            }
+            __half h[4], l[4];
+#pragma unroll
+            for (int q = 0; q < 4; q++) f16_split(x[q], sc, h[q], l[q]);
+            *reinterpret_cast<uint2 *>(hr + c) =
+                make_uint2(*reinterpret_cast<uint32_t *>(&h[0]) | 0u, *reinterpret_cast<uint32_t *>(&h[2]));
+            *reinterpret_cast<uint2 *>(lr + c) =
+                make_uint2(*reinterpret_cast<uint32_t *>(&l[0]) | 0u, *reinterpret_cast<uint32_t *>(&l[2]));
         }
     }
 }
-// one CTA (256 threads) per 32-column strip: column maxima, then 64 x 32 tiles transposed through shared
-// memory so both the reads (along j) and the fp16 writes (along k) are coalesced
-__device__ void f16_cols_body(const F16Cols &j, int64_t strip) {
-    __shared__ float t[64][33];
+// column maxima of a row-major B (K x N): CTA (32-column strip, 256-row chunk), 256 threads -- a thread
+// owns one column, the warps split the chunk; partial maxima meet in colmax via atomicMax on the bit
+// pattern (non-negative floats order like their bits)
+__global__ void __launch_bounds__(256) f16_colmax_kernel(const float *__restrict__ x, int64_t K, int64_t N,
+                                                         int64_t ldx, unsigned *__restrict__ colmax) {
     __shared__ float red[8][32];
-    __shared__ float sc[32];
-    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
-    const int64_t j0 = strip * 32, col = j0 + lane;
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int64_t col = (int64_t)blockIdx.x * 32 + lane, k0 = (int64_t)blockIdx.y * 256;
     float m = 0.f;
-    if (col < j.N)
-        for (int64_t k = w; k < j.K; k += 8) m = fmaxf(m, fabsf(j.x[k * j.ldx + col]));
+    if (col < N) {
+#pragma unroll 8
+        for (int i = w; i < 256; i += 8)
+            if (k0 + i < K) m = fmaxf(m, fabsf(x[(k0 + i) * ldx + col]));
+    }
     red[w][lane] = m;
     __syncthreads();
-    if (w == 0) {
+    if (w == 0 && col < N) {
         for (int q = 1; q < 8; q++) m = fmaxf(m, red[q][lane]);
-        const int s = f16_scale_exp(m);
-        if (col < j.N) j.exps[col] = s;
-        sc[lane] = __int_as_float((127 + s) << 23);
-    }
-    __syncthreads();
-    for (int64_t k0 = 0; k0 < j.K; k0 += 64) {
-        for (int e = tid; e < 64 * 32; e += 256) {
-            const int kk = e >> 5, jj = e & 31;
-            t[kk][jj] = (k0 + kk < j.K && j0 + jj < j.N) ? j.x[(k0 + kk) * j.ldx + j0 + jj] : 0.f;
-        }
-        __syncthreads();
-        for (int e = tid; e < 32 * 32; e += 256) {  // (column jj, k pair kp)
-            const int jj = e >> 5, kp = e & 31;
-            if (j0 + jj < j.N && k0 + 2 * kp < j.ldp) {
-                __half h0, l0, h1, l1;
-                f16_split(t[2 * kp][jj], sc[jj], h0, l0);
-                f16_split(t[2 * kp + 1][jj], sc[jj], h1, l1);
-                const int64_t o = (j0 + jj) * j.ldp + k0 + 2 * kp;
-                *reinterpret_cast<__half2 *>(j.hi + o) = __halves2half2(h0, h1);
-                *reinterpret_cast<__half2 *>(j.lo + o) = __halves2half2(l0, l1);
-            }
-        }
-        __syncthreads();
+        atomicMax(colmax + col, __float_as_uint(m));
     }
 }
-// One launch before the 3xFP16 GEMM: blocks [0, nbr) split the row operands (A, and B when it is K-major
-// -- syrk), [nbr, nbr + nbc) the column strips of a row-major B, the rest the split-k tail pre-pass.
-__global__ void __launch_bounds__(256) prep_f16_kernel(const F16Rows r0, const F16Rows r1, const F16Cols cj, int nbr,
-                                                       int nbc, const Args p, int rows_per_tile, int bn, int vecC) {
+// one 64 x 32 tile (k-chunk, column strip) of a row-major B: scaled, split and transposed through shared
+// memory so both the reads (along j) and the fp16 writes (along k) are coalesced; the column exponents
+// come from colmax (the k-chunk 0 tile records them)
+__device__ void f16_cols_tile(const F16Cols &j, const unsigned *colmax, int64_t tile) {
+    __shared__ float t[64][33];
+    __shared__ float sc[32];
+    const int tid = threadIdx.x;
+    const int64_t nstrip = (j.N + 31) / 32;
+    const int64_t strip = tile % nstrip, k0 = (tile / nstrip) * 64, j0 = strip * 32;
+    if (tid < 32) {
+        const int64_t col = j0 + tid;
+        const int s = col < j.N ? f16_scale_exp(__uint_as_float(colmax[col])) : 0;
+        if (k0 == 0 && col < j.N) j.exps[col] = s;
+        sc[tid] = __int_as_float((127 + s) << 23);
+    }
+    for (int e = tid; e < 64 * 32; e += 256) {
+        const int kk = e >> 5, jj = e & 31;
+        t[kk][jj] = (k0 + kk < j.K && j0 + jj < j.N) ? j.x[(k0 + kk) * j.ldx + j0 + jj] : 0.f;
+    }
+    __syncthreads();
+    for (int e = tid; e < 32 * 32; e += 256) {  // (column jj, k pair kp)
+        const int jj = e >> 5, kp = e & 31;
+        if (j0 + jj < j.N && k0 + 2 * kp < j.ldp) {
+            __half h0, l0, h1, l1;
+            f16_split(t[2 * kp][jj], sc[jj], h0, l0);
+            f16_split(t[2 * kp + 1][jj], sc[jj], h1, l1);
+            const int64_t o = (j0 + jj) * j.ldp + k0 + 2 * kp;
+            *reinterpret_cast<__half2 *>(j.hi + o) = __halves2half2(h0, h1);
+            *reinterpret_cast<__half2 *>(j.lo + o) = __halves2half2(l0, l1);
+        }
+    }
+    __syncthreads();
+}
+// The launch before the 3xFP16 GEMM: blocks [0, nbr) split the row operands (A, and B when it is K-major
+// -- syrk), [nbr, nbr + nbc) the 64 x 32 tiles of a row-major B (its column maxima from f16_colmax_kernel),
+// the rest the split-k tail pre-pass.
+__global__ void __launch_bounds__(256) prep_f16_kernel(const F16Rows r0, const F16Rows r1, const F16Cols cj,
+                                                       const unsigned *colmax, int nbr, int nbc, const Args p,
+                                                       int rows_per_tile, int bn, int vecC) {
     const int b = (int)blockIdx.x;
     if (b < nbr) {
         const int64_t wstride = (int64_t)nbr * 8, w0 = (int64_t)b * 8 + (threadIdx.x >> 5);
@@ -614,7 +654,8 @@ __global__ void __launch_bounds__(256) prep_f16_kernel(const F16Rows r0, const F
         return;
     }
     if (b < nbr + nbc) {
-        for (int64_t st = b - nbr; st < (cj.N + 31) / 32; st += nbc) f16_cols_body(cj, st);
+        const int64_t ntiles = ((cj.N + 31) / 32) * ((cj.ldp + 63) / 64);
+        for (int64_t tile = b - nbr; tile < ntiles; tile += nbc) f16_cols_tile(cj, colmax, tile);
         return;
     }
     const int npb = (int)gridDim.x - nbr - nbc, g4 = (bn + 3) / 4;
@@ -650,6 +691,7 @@ struct Prep {
     // 3xFP16: row splits (A; B when K-major) and the column strips of a row-major B
     tcm::F16Rows r0{}, r1{};
     tcm::F16Cols cj{};
+    unsigned *colmax = nullptr;  // row-major B: per-column max bits (f16_colmax_kernel before the prep launch)
     int nbr = 0, nbc = 0;
 };
 
@@ -763,12 +805,19 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
         const int64_t tail4 = needs_prepass(a) ? (int64_t)(a.T - a.nfull) * rows * ((a.BNT + 3) / 4) : 0;
         const int npb = (int)std::min<int64_t>((tail4 + 255) / 256, (int64_t)nsm * 4);
         const int vecC = (a.ldc % 4 == 0 && (reinterpret_cast<uintptr_t>(a.C) & 15) == 0) ? 1 : 0;
-        if constexpr (F16)
-            tcm::prep_f16_kernel<<<pr.nbr + pr.nbc + npb, 256, 0, s>>>(pr.r0, pr.r1, pr.cj, pr.nbr, pr.nbc, a, rows,
-                                                                       a.BNT, vecC);
-        else
+        if constexpr (F16) {
+            if (pr.colmax) {  // column maxima of a row-major B first (its split needs them)
+                if ((e = cudaMemsetAsync(pr.colmax, 0, (size_t)pr.cj.N * 4, s)) != cudaSuccess) return e;
+                const dim3 g((unsigned)((pr.cj.N + 31) / 32), (unsigned)((pr.cj.K + 255) / 256));
+                tcm::f16_colmax_kernel<<<g, 256, 0, s>>>(pr.cj.x, pr.cj.K, pr.cj.N, pr.cj.ldx, pr.colmax);
+                if ((e = cudaGetLastError()) != cudaSuccess) return e;
+            }
+            tcm::prep_f16_kernel<<<pr.nbr + pr.nbc + npb, 256, 0, s>>>(pr.r0, pr.r1, pr.cj, pr.colmax, pr.nbr,
+                                                                       pr.nbc, a, rows, a.BNT, vecC);
+        } else {
             tcm::prep_kernel<<<pr.nb0 + pr.nb1 + npb, 256, 0, s>>>(pr.j0, pr.j1, pr.nb0, pr.nb1, pr.mode, a, rows,
                                                                    a.BNT, vecC);
+        }
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
     }
     cfg.gridDim = dim3((unsigned)(CG * ncl));
@@ -939,7 +988,7 @@ cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p,
 namespace {
 struct F16Layout {  // workspace offsets (bytes, 256-aligned): hi/lo fp16 operands and their exponents
     int64_t Kp = 0;
-    size_t a_hi = 0, a_lo = 0, a_exp = 0, b_hi = 0, b_lo = 0, b_exp = 0, total = 0;
+    size_t a_hi = 0, a_lo = 0, a_exp = 0, b_hi = 0, b_lo = 0, b_exp = 0, b_max = 0, total = 0;
     bool share = false;  // syrk: A is a row block of the K-major B
 };
 F16Layout f16_layout(const ContractNest &n) {
@@ -952,6 +1001,7 @@ F16Layout f16_layout(const ContractNest &n) {
     L.b_hi = o; o = al(o + (size_t)n.N * L.Kp * 2);
     L.b_lo = o; o = al(o + (size_t)n.N * L.Kp * 2);
     L.b_exp = o; o = al(o + (size_t)n.N * 4);
+    L.b_max = o; o = al(o + (size_t)n.N * 4);
     if (!L.share) {
         L.a_hi = o; o = al(o + (size_t)n.M * L.Kp * 2);
         L.a_lo = o; o = al(o + (size_t)n.M * L.Kp * 2);
@@ -985,7 +1035,8 @@ cudaError_t launch_tcf_contraction(const ContractNest &n, const ContractPlan &p,
         pr.r0 = tcm::F16Rows{B, n.N, n.K, n.ldb, L.Kp, bhi, blo, bexp};
     } else {  // row-major B[k][j]: column strips, transposed to K-major
         pr.cj = tcm::F16Cols{B, n.K, n.N, n.ldb, L.Kp, bhi, blo, bexp};
-        pr.nbc = (int)std::min<int64_t>((n.N + 31) / 32, (int64_t)nsm * 2);
+        pr.colmax = reinterpret_cast<unsigned *>(w + L.b_max);
+        pr.nbc = (int)std::min<int64_t>(((n.N + 31) / 32) * ((L.Kp + 63) / 64), (int64_t)nsm * 8);
     }
     if (L.share) {
         const int64_t r = (A - B) / n.ldb;
