@@ -54,7 +54,8 @@ constexpr int BM = 128;      // rows of i per CTA (UMMA M per SM)
 constexpr int NEPI = 16;     // epilogue warps (4..19): four per TMEM lane quarter, a column quarter each
 constexpr int NTHREADS = (4 + NEPI) * 32;
 constexpr int MAXBN = 256;   // UMMA N limit
-constexpr int CHUNK_K = 128; // k per accumulator chunk (fp32 drain of the truncating accumulation)
+constexpr int CHUNK_K = 128; // k per accumulator chunk (fp32 drain of the truncating accumulation), 3xTF32
+constexpr int CHUNK_K_F16 = 256;  // 3xFP16: K = 16 per MMA, half the truncating accumulations per k
 
 struct Args {
     int64_t M, N, K;
@@ -586,25 +587,44 @@ __device__ void f16_rows_body(const F16Rows &j, int64_t w0, int64_t wstride) {
         }
     }
 }
-// column maxima of a row-major B (K x N): CTA (32-column strip, 256-row chunk), 256 threads -- a thread
-// owns one column, the warps split the chunk; partial maxima meet in colmax via atomicMax on the bit
-// pattern (non-negative floats order like their bits)
+// column maxima of a row-major B (K x N): CTA (128-column strip, 256-row chunk), 256 threads -- a thread
+// owns four adjacent columns (16-byte loads when aligned), the warps split the chunk, eight loads in
+// flight per thread; partial maxima meet in colmax via atomicMax on the bit pattern (non-negative floats
+// order like their bits)
 __global__ void __launch_bounds__(256) f16_colmax_kernel(const float *__restrict__ x, int64_t K, int64_t N,
                                                          int64_t ldx, unsigned *__restrict__ colmax) {
-    __shared__ float red[8][32];
+    __shared__ float4 red[8][32];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    const int64_t col = (int64_t)blockIdx.x * 32 + lane, k0 = (int64_t)blockIdx.y * 256;
-    float m = 0.f;
-    if (col < N) {
+    const int64_t c0 = (int64_t)blockIdx.x * 128 + 4 * lane, k0 = (int64_t)blockIdx.y * 256;
+    const bool v4 = ((ldx & 3) == 0) && ((reinterpret_cast<uintptr_t>(x) & 15) == 0) && c0 + 3 < N;
+    float4 m = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (c0 < N) {
 #pragma unroll 8
-        for (int i = w; i < 256; i += 8)
-            if (k0 + i < K) m = fmaxf(m, fabsf(x[(k0 + i) * ldx + col]));
+        for (int i = w; i < 256; i += 8) {
+            if (k0 + i >= K) break;
+            const float *row = x + (k0 + i) * ldx + c0;
+            float4 v;
+            if (v4) {
+                v = __ldg(reinterpret_cast<const float4 *>(row));
+            } else {
+                v.x = row[0];
+                v.y = c0 + 1 < N ? row[1] : 0.f;
+                v.z = c0 + 2 < N ? row[2] : 0.f;
+                v.w = c0 + 3 < N ? row[3] : 0.f;
+            }
+            m.x = fmaxf(m.x, fabsf(v.x)); m.y = fmaxf(m.y, fabsf(v.y));
+            m.z = fmaxf(m.z, fabsf(v.z)); m.w = fmaxf(m.w, fabsf(v.w));
+        }
     }
     red[w][lane] = m;
     __syncthreads();
-    if (w == 0 && col < N) {
-        for (int q = 1; q < 8; q++) m = fmaxf(m, red[q][lane]);
-        atomicMax(colmax + col, __float_as_uint(m));
+    if (w == 0 && c0 < N) {
+        for (int q = 1; q < 8; q++) {
+            const float4 o = red[q][lane];
+            m.x = fmaxf(m.x, o.x); m.y = fmaxf(m.y, o.y); m.z = fmaxf(m.z, o.z); m.w = fmaxf(m.w, o.w);
+        }
+        const float mm[4] = {m.x, m.y, m.z, m.w};
+        for (int q = 0; q < 4 && c0 + q < N; q++) atomicMax(colmax + c0 + q, __float_as_uint(mm[q]));
     }
 }
 // one 64 x 32 tile (k-chunk, column strip) of a row-major B: scaled, split and transposed through shared
@@ -808,7 +828,7 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
         if constexpr (F16) {
             if (pr.colmax) {  // column maxima of a row-major B first (its split needs them)
                 if ((e = cudaMemsetAsync(pr.colmax, 0, (size_t)pr.cj.N * 4, s)) != cudaSuccess) return e;
-                const dim3 g((unsigned)((pr.cj.N + 31) / 32), (unsigned)((pr.cj.K + 255) / 256));
+                const dim3 g((unsigned)((pr.cj.N + 127) / 128), (unsigned)((pr.cj.K + 255) / 256));
                 tcm::f16_colmax_kernel<<<g, 256, 0, s>>>(pr.cj.x, pr.cj.K, pr.cj.N, pr.cj.ldx, pr.colmax);
                 if ((e = cudaGetLastError()) != cudaSuccess) return e;
             }
@@ -1070,7 +1090,7 @@ cudaError_t launch_tcf_contraction(const ContractNest &n, const ContractPlan &p,
     a.alpha = (float)n.alpha; a.beta = (float)n.beta; a.init_zero = n.init_zero ? 1 : 0;
     a.S = g.S;
     static const int chunk_env = devsw("EATSS_TCM_CHUNK_K", 0);  // development: k per accumulator chunk
-    a.R = std::max(1, (chunk_env > 0 ? chunk_env : tcm::CHUNK_K) / g.bk);
+    a.R = std::max(1, (chunk_env > 0 ? chunk_env : tcm::CHUNK_K_F16) / g.bk);
     a.BNT = g.bn; a.BNH = g.bnh; a.bgroups = g.bgroups; a.b_bytes = g.b_bytes; a.stage = g.stage;
     a.idesc = tcm::idesc_f16(g.bn, g.cg);
     a.nkb = (int)((n.K + g.bk - 1) / g.bk);

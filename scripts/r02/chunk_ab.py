@@ -29,7 +29,7 @@ def one():
     else:
         ref = O.gemm(1.5, 1.2, C, A, B)
         np.save(ref_path, ref)
-    d = E.desc_builtin("gemm", (n, n, n)); d.set_scalars(1.5, 1.2); d.set_exec(50, 2)
+    d = E.desc_builtin("gemm", (n, n, n)); d.set_scalars(1.5, 1.2); d.set_exec(50, int(os.environ.get("ENGINE", "2")))
     Ad, Bd = torch.from_numpy(A).cuda(), torch.from_numpy(B).cuda()
     Cd = torch.from_numpy(C).cuda()
     t = tuple(int(x) for x in os.environ.get("TILE", "256,256,32").split(","))
@@ -46,7 +46,7 @@ def one():
         E.run(d, t, [Cw, Ad, Bd])
     e.record(); torch.cuda.synchronize()
     ms = s.elapsed_time(e) / 50
-    print(json.dumps({"tiles": t, "chunk_k": os.environ.get("EATSS_TCM_CHUNK_K", "128"), "ms": ms, "tflops": 2 * n ** 3 / ms / 1e9,
+    print(json.dumps({"engine": os.environ.get("ENGINE", "2"), "tiles": t, "chunk_k": os.environ.get("EATSS_TCM_CHUNK_K", "128"), "ms": ms, "tflops": 2 * n ** 3 / ms / 1e9,
                       "normwise_rel_err": err, "max_abs_err_over_rms": mx}), flush=True)
 
 
