@@ -534,6 +534,7 @@ struct F16Rows {  // rows x cols fp32 (pitch ldx) -> hi / lo fp16 [rows][ldp], e
     int64_t rows, cols, ldx, ldp;
     __half *hi, *lo;
     int *exps;
+    const unsigned *maxbits;  // row maxima (bit patterns) from f16_max_kernel
 };
 struct F16Cols {  // K x N fp32 (pitch ldx) -> transposed hi / lo fp16 [N][ldp] (K-major), exps[N]
     const float *x;
@@ -541,61 +542,86 @@ struct F16Cols {  // K x N fp32 (pitch ldx) -> transposed hi / lo fp16 [N][ldp] 
     __half *hi, *lo;
     int *exps;
 };
-// one warp per row: the row's max, then the scaled split (second read from L1 / L2); 16-byte loads, four
-// in flight per lane (a row is 16 KB at K = 4000: the warp keeps 2 KB in flight)
+// one warp per row: the scaled split with the row's exponent from its maximum (f16_max_kernel); 16-byte
+// loads, 8-byte fp16 stores, four column groups in flight per lane
 __device__ void f16_rows_body(const F16Rows &j, int64_t w0, int64_t wstride) {
     const int lane = threadIdx.x & 31;
+    const bool v4 = ((j.ldx & 3) == 0) && ((reinterpret_cast<uintptr_t>(j.x) & 15) == 0);
     for (int64_t r = w0; r < j.rows; r += wstride) {
         const float *xr = j.x + r * j.ldx;
-        const bool v4 = ((j.ldx & 3) == 0) && ((reinterpret_cast<uintptr_t>(j.x) & 15) == 0);
-        const int64_t n4 = v4 ? j.cols / 4 : 0;
-        float m = 0.f;
-        for (int64_t c4 = lane; c4 < n4; c4 += 128) {
-            float4 v[4];
-#pragma unroll
-            for (int u = 0; u < 4; u++)
-                v[u] = c4 + 32 * u < n4 ? *reinterpret_cast<const float4 *>(xr + 4 * (c4 + 32 * u))
-                                        : make_float4(0.f, 0.f, 0.f, 0.f);
-#pragma unroll
-            for (int u = 0; u < 4; u++)
-                m = fmaxf(m, fmaxf(fmaxf(fabsf(v[u].x), fabsf(v[u].y)), fmaxf(fabsf(v[u].z), fabsf(v[u].w))));
-        }
-        for (int64_t c = 4 * n4 + lane; c < j.cols; c += 32) m = fmaxf(m, fabsf(xr[c]));
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
-        const int s = f16_scale_exp(m);
+        const int s = f16_scale_exp(__uint_as_float(j.maxbits[r]));
         if (lane == 0) j.exps[r] = s;
         const float sc = __int_as_float((127 + s) << 23);
         __half *hr = j.hi + r * j.ldp, *lr = j.lo + r * j.ldp;
-        // groups of 4 columns (ldp is a multiple of 8): 8-byte fp16 stores
-        for (int64_t c = 4 * lane; c < j.ldp; c += 128) {
-            float x[4];
-            if (v4 && c + 3 < j.cols) {
-                const float4 t = *reinterpret_cast<const float4 *>(xr + c);
-                x[0] = t.x; x[1] = t.y; x[2] = t.z; x[3] = t.w;
-            } else {
+        for (int64_t c0 = 4 * lane; c0 < j.ldp; c0 += 4 * 128) {  // groups of 4 columns (ldp % 8 == 0)
+            float x[4][4];
 #pragma unroll
-                for (int q = 0; q < 4; q++) x[q] = c + q < j.cols ? xr[c + q] : 0.f;
+            for (int u = 0; u < 4; u++) {
+                const int64_t c = c0 + 128 * u;
+                if (v4 && c + 3 < j.cols) {
+                    const float4 t = *reinterpret_cast<const float4 *>(xr + c);
+                    x[u][0] = t.x; x[u][1] = t.y; x[u][2] = t.z; x[u][3] = t.w;
+                } else {
+#pragma unroll
+                    for (int q = 0; q < 4; q++) x[u][q] = c + q < j.cols ? xr[c + q] : 0.f;
+                }
             }
-            __half h[4], l[4];
 #pragma unroll
-            for (int q = 0; q < 4; q++) f16_split(x[q], sc, h[q], l[q]);
-            *reinterpret_cast<uint2 *>(hr + c) =
-                make_uint2(*reinterpret_cast<uint32_t *>(&h[0]) | 0u, *reinterpret_cast<uint32_t *>(&h[2]));
-            *reinterpret_cast<uint2 *>(lr + c) =
-                make_uint2(*reinterpret_cast<uint32_t *>(&l[0]) | 0u, *reinterpret_cast<uint32_t *>(&l[2]));
+            for (int u = 0; u < 4; u++) {
+                const int64_t c = c0 + 128 * u;
+                if (c >= j.ldp) break;
+                __half h[4], l[4];
+#pragma unroll
+                for (int q = 0; q < 4; q++) f16_split(x[u][q], sc, h[q], l[q]);
+                *reinterpret_cast<uint2 *>(hr + c) =
+                    make_uint2(*reinterpret_cast<uint32_t *>(&h[0]), *reinterpret_cast<uint32_t *>(&h[2]));
+                *reinterpret_cast<uint2 *>(lr + c) =
+                    make_uint2(*reinterpret_cast<uint32_t *>(&l[0]), *reinterpret_cast<uint32_t *>(&l[2]));
+            }
         }
+    }
+}
+// row maxima of up to two row operands: CTA (32 rows, 1024-column chunk), a warp per row and chunk, 16-byte
+// loads (eight per lane in flight); partial maxima meet via atomicMax on the bit pattern
+__device__ void f16_rowmax_block(const F16Rows &j, unsigned *maxbits, int64_t blk) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int64_t nch = (j.cols + 1023) / 1024;
+    const int64_t r0 = (blk / nch) * 32, c0 = (blk % nch) * 1024;
+    const bool v4 = ((j.ldx & 3) == 0) && ((reinterpret_cast<uintptr_t>(j.x) & 15) == 0);
+    for (int q = 0; q < 4; q++) {
+        const int64_t r = r0 + 4 * w + q;
+        if (r >= j.rows) break;
+        const float *xr = j.x + r * j.ldx;
+        float m = 0.f;
+        if (v4) {
+            float4 v[8];
+#pragma unroll
+            for (int u = 0; u < 8; u++) {
+                const int64_t c = c0 + 4 * (lane + 32 * u);
+                v[u] = c + 3 < j.cols ? __ldg(reinterpret_cast<const float4 *>(xr + c)) : make_float4(0.f, 0.f, 0.f, 0.f);
+                if (c < j.cols && c + 3 >= j.cols)
+                    for (int e = 0; c + e < j.cols; e++) m = fmaxf(m, fabsf(xr[c + e]));
+            }
+#pragma unroll
+            for (int u = 0; u < 8; u++)
+                m = fmaxf(m, fmaxf(fmaxf(fabsf(v[u].x), fabsf(v[u].y)), fmaxf(fabsf(v[u].z), fabsf(v[u].w))));
+        } else {
+            for (int64_t c = c0 + lane; c < c0 + 1024 && c < j.cols; c += 32) m = fmaxf(m, fabsf(xr[c]));
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+        if (lane == 0) atomicMax(maxbits + r, __float_as_uint(m));
     }
 }
 // column maxima of a row-major B (K x N): CTA (128-column strip, 256-row chunk), 256 threads -- a thread
 // owns four adjacent columns (16-byte loads when aligned), the warps split the chunk, eight loads in
 // flight per thread; partial maxima meet in colmax via atomicMax on the bit pattern (non-negative floats
 // order like their bits)
-__global__ void __launch_bounds__(256) f16_colmax_kernel(const float *__restrict__ x, int64_t K, int64_t N,
-                                                         int64_t ldx, unsigned *__restrict__ colmax) {
+__device__ void f16_colmax_block(const float *__restrict__ x, int64_t K, int64_t N, int64_t ldx,
+                                 unsigned *__restrict__ colmax, int64_t bx, int64_t by) {
     __shared__ float4 red[8][32];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    const int64_t c0 = (int64_t)blockIdx.x * 128 + 4 * lane, k0 = (int64_t)blockIdx.y * 256;
+    const int64_t c0 = bx * 128 + 4 * lane, k0 = by * 256;
     const bool v4 = ((ldx & 3) == 0) && ((reinterpret_cast<uintptr_t>(x) & 15) == 0) && c0 + 3 < N;
     float4 m = make_float4(0.f, 0.f, 0.f, 0.f);
     if (c0 < N) {
@@ -626,6 +652,22 @@ __global__ void __launch_bounds__(256) f16_colmax_kernel(const float *__restrict
         const float mm[4] = {m.x, m.y, m.z, m.w};
         for (int q = 0; q < 4 && c0 + q < N; q++) atomicMax(colmax + c0 + q, __float_as_uint(mm[q]));
     }
+}
+// The maxima pass before the 3xFP16 split (one launch): blocks [0, nr0) row maxima of r0, [nr0, nr0 + nr1)
+// of r1, the rest the column maxima of a row-major B (cj; colmax) -- every block independent
+__global__ void __launch_bounds__(256) f16_max_kernel(const F16Rows r0, unsigned *m0, const F16Rows r1, unsigned *m1,
+                                                      const F16Cols cj, unsigned *colmax, int nr0, int nr1) {
+    const int64_t b = blockIdx.x;
+    if (b < nr0) {
+        f16_rowmax_block(r0, m0, b);
+        return;
+    }
+    if (b < nr0 + nr1) {
+        f16_rowmax_block(r1, m1, b - nr0);
+        return;
+    }
+    const int64_t c = b - nr0 - nr1, nsx = (cj.N + 127) / 128;
+    f16_colmax_block(cj.x, cj.K, cj.N, cj.ldx, colmax, c % nsx, c / nsx);
 }
 // one 64 x 32 tile (k-chunk, column strip) of a row-major B: scaled, split and transposed through shared
 // memory so both the reads (along j) and the fp16 writes (along k) are coalesced; the column exponents
@@ -661,7 +703,7 @@ __device__ void f16_cols_tile(const F16Cols &j, const unsigned *colmax, int64_t 
     __syncthreads();
 }
 // The launch before the 3xFP16 GEMM: blocks [0, nbr) split the row operands (A, and B when it is K-major
-// -- syrk), [nbr, nbr + nbc) the 64 x 32 tiles of a row-major B (its column maxima from f16_colmax_kernel),
+// -- syrk), [nbr, nbr + nbc) the 64 x 32 tiles of a row-major B (its column maxima from f16_max_kernel),
 // the rest the split-k tail pre-pass.
 __global__ void __launch_bounds__(256) prep_f16_kernel(const F16Rows r0, const F16Rows r1, const F16Cols cj,
                                                        const unsigned *colmax, int nbr, int nbc, const Args p,
@@ -711,7 +753,10 @@ struct Prep {
     // 3xFP16: row splits (A; B when K-major) and the column strips of a row-major B
     tcm::F16Rows r0{}, r1{};
     tcm::F16Cols cj{};
-    unsigned *colmax = nullptr;  // row-major B: per-column max bits (f16_colmax_kernel before the prep launch)
+    unsigned *colmax = nullptr;  // row-major B: per-column max bits (f16_max_kernel before the prep launch)
+    unsigned *maxes = nullptr;   // the zero-initialised region holding every max array of this GEMM
+    size_t maxes_bytes = 0;
+    unsigned *m0 = nullptr, *m1 = nullptr;  // row maxima of r0 / r1
     int nbr = 0, nbc = 0;
 };
 
@@ -826,10 +871,15 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
         const int npb = (int)std::min<int64_t>((tail4 + 255) / 256, (int64_t)nsm * 4);
         const int vecC = (a.ldc % 4 == 0 && (reinterpret_cast<uintptr_t>(a.C) & 15) == 0) ? 1 : 0;
         if constexpr (F16) {
-            if (pr.colmax) {  // column maxima of a row-major B first (its split needs them)
-                if ((e = cudaMemsetAsync(pr.colmax, 0, (size_t)pr.cj.N * 4, s)) != cudaSuccess) return e;
-                const dim3 g((unsigned)((pr.cj.N + 127) / 128), (unsigned)((pr.cj.K + 255) / 256));
-                tcm::f16_colmax_kernel<<<g, 256, 0, s>>>(pr.cj.x, pr.cj.K, pr.cj.N, pr.cj.ldx, pr.colmax);
+            {  // maxima of every row of the row operands and column of a row-major B (the split needs them)
+                if ((e = cudaMemsetAsync(pr.maxes, 0, pr.maxes_bytes, s)) != cudaSuccess) return e;
+                auto nrb = [](const tcm::F16Rows &r) {
+                    return r.x ? (int)(((r.rows + 31) / 32) * ((r.cols + 1023) / 1024)) : 0;
+                };
+                const int nr0 = nrb(pr.r0), nr1 = nrb(pr.r1);
+                const int ncb = pr.colmax ? (int)(((pr.cj.N + 127) / 128) * ((pr.cj.K + 255) / 256)) : 0;
+                tcm::f16_max_kernel<<<nr0 + nr1 + ncb, 256, 0, s>>>(pr.r0, pr.m0, pr.r1, pr.m1, pr.cj, pr.colmax, nr0,
+                                                                    nr1);
                 if ((e = cudaGetLastError()) != cudaSuccess) return e;
             }
             tcm::prep_f16_kernel<<<pr.nbr + pr.nbc + npb, 256, 0, s>>>(pr.r0, pr.r1, pr.cj, pr.colmax, pr.nbr,
@@ -1008,7 +1058,7 @@ cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p,
 namespace {
 struct F16Layout {  // workspace offsets (bytes, 256-aligned): hi/lo fp16 operands and their exponents
     int64_t Kp = 0;
-    size_t a_hi = 0, a_lo = 0, a_exp = 0, b_hi = 0, b_lo = 0, b_exp = 0, b_max = 0, total = 0;
+    size_t a_hi = 0, a_lo = 0, a_exp = 0, b_hi = 0, b_lo = 0, b_exp = 0, b_max = 0, a_max = 0, max_end = 0, total = 0;
     bool share = false;  // syrk: A is a row block of the K-major B
 };
 F16Layout f16_layout(const ContractNest &n) {
@@ -1021,7 +1071,9 @@ F16Layout f16_layout(const ContractNest &n) {
     L.b_hi = o; o = al(o + (size_t)n.N * L.Kp * 2);
     L.b_lo = o; o = al(o + (size_t)n.N * L.Kp * 2);
     L.b_exp = o; o = al(o + (size_t)n.N * 4);
-    L.b_max = o; o = al(o + (size_t)n.N * 4);
+    L.b_max = o; o = o + (size_t)n.N * 4;   // maxima: b_max then a_max, contiguous (one memset)
+    L.a_max = o; o = o + (L.share ? 0 : (size_t)n.M * 4);
+    L.max_end = o; o = al(o);
     if (!L.share) {
         L.a_hi = o; o = al(o + (size_t)n.M * L.Kp * 2);
         L.a_lo = o; o = al(o + (size_t)n.M * L.Kp * 2);
@@ -1051,11 +1103,15 @@ cudaError_t launch_tcf_contraction(const ContractNest &n, const ContractPlan &p,
     int dev = 0, nsm = 148;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    unsigned *bmax = reinterpret_cast<unsigned *>(w + L.b_max), *amax = reinterpret_cast<unsigned *>(w + L.a_max);
+    pr.maxes = bmax;
+    pr.maxes_bytes = L.max_end - L.b_max;
     if (n.transB) {  // B(k, j) = B[j*ldb + k]: rows j are already K-major -> row split, row scale = column scale
-        pr.r0 = tcm::F16Rows{B, n.N, n.K, n.ldb, L.Kp, bhi, blo, bexp};
+        pr.r0 = tcm::F16Rows{B, n.N, n.K, n.ldb, L.Kp, bhi, blo, bexp, bmax};
+        pr.m0 = bmax;
     } else {  // row-major B[k][j]: column strips, transposed to K-major
         pr.cj = tcm::F16Cols{B, n.K, n.N, n.ldb, L.Kp, bhi, blo, bexp};
-        pr.colmax = reinterpret_cast<unsigned *>(w + L.b_max);
+        pr.colmax = bmax;
         pr.nbc = (int)std::min<int64_t>(((n.N + 31) / 32) * ((L.Kp + 63) / 64), (int64_t)nsm * 8);
     }
     if (L.share) {
@@ -1066,7 +1122,8 @@ cudaError_t launch_tcf_contraction(const ContractNest &n, const ContractPlan &p,
     } else {
         __half *h = reinterpret_cast<__half *>(w + L.a_hi), *l = reinterpret_cast<__half *>(w + L.a_lo);
         int *e = reinterpret_cast<int *>(w + L.a_exp);
-        (n.transB ? pr.r1 : pr.r0) = tcm::F16Rows{A, n.M, n.K, n.lda, L.Kp, h, l, e};
+        (n.transB ? pr.r1 : pr.r0) = tcm::F16Rows{A, n.M, n.K, n.lda, L.Kp, h, l, e, amax};
+        (n.transB ? pr.m1 : pr.m0) = amax;
         ahi = h;
         alo = l;
         aexp = e;
