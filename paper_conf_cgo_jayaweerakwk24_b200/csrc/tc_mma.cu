@@ -594,17 +594,17 @@ __device__ void f16_rowmax_block(const F16Rows &j, unsigned *maxbits, int64_t bl
         const float *xr = j.x + r * j.ldx;
         float m = 0.f;
         if (v4) {
-            float4 v[8];
+            float4 v[8];  // all eight loads issued before the first use
 #pragma unroll
             for (int u = 0; u < 8; u++) {
                 const int64_t c = c0 + 4 * (lane + 32 * u);
                 v[u] = c + 3 < j.cols ? __ldg(reinterpret_cast<const float4 *>(xr + c)) : make_float4(0.f, 0.f, 0.f, 0.f);
-                if (c < j.cols && c + 3 >= j.cols)
-                    for (int e = 0; c + e < j.cols; e++) m = fmaxf(m, fabsf(xr[c + e]));
             }
 #pragma unroll
             for (int u = 0; u < 8; u++)
                 m = fmaxf(m, fmaxf(fmaxf(fabsf(v[u].x), fabsf(v[u].y)), fmaxf(fabsf(v[u].z), fabsf(v[u].w))));
+            const int64_t ce = c0 + 1024 < j.cols ? c0 + 1024 : j.cols;  // a ragged last group of < 4 columns
+            for (int64_t c = (ce & ~3LL) + lane; c < ce && (ce & 3); c += 32) m = fmaxf(m, fabsf(xr[c]));
         } else {
             for (int64_t c = c0 + lane; c < c0 + 1024 && c < j.cols; c += 32) m = fmaxf(m, fabsf(xr[c]));
         }
@@ -625,21 +625,28 @@ __device__ void f16_colmax_block(const float *__restrict__ x, int64_t K, int64_t
     const bool v4 = ((ldx & 3) == 0) && ((reinterpret_cast<uintptr_t>(x) & 15) == 0) && c0 + 3 < N;
     float4 m = make_float4(0.f, 0.f, 0.f, 0.f);
     if (c0 < N) {
-#pragma unroll 8
-        for (int i = w; i < 256; i += 8) {
-            if (k0 + i >= K) break;
-            const float *row = x + (k0 + i) * ldx + c0;
-            float4 v;
-            if (v4) {
-                v = __ldg(reinterpret_cast<const float4 *>(row));
-            } else {
-                v.x = row[0];
-                v.y = c0 + 1 < N ? row[1] : 0.f;
-                v.z = c0 + 2 < N ? row[2] : 0.f;
-                v.w = c0 + 3 < N ? row[3] : 0.f;
+        for (int i0 = w; i0 < 256; i0 += 64) {  // eight rows per pass, all loads issued before their use
+            float4 v[8];
+#pragma unroll
+            for (int u = 0; u < 8; u++) {
+                const int64_t k = k0 + i0 + 8 * u;
+                const float *row = x + k * ldx + c0;
+                if (k >= K) {
+                    v[u] = make_float4(0.f, 0.f, 0.f, 0.f);
+                } else if (v4) {
+                    v[u] = __ldg(reinterpret_cast<const float4 *>(row));
+                } else {
+                    v[u].x = row[0];
+                    v[u].y = c0 + 1 < N ? row[1] : 0.f;
+                    v[u].z = c0 + 2 < N ? row[2] : 0.f;
+                    v[u].w = c0 + 3 < N ? row[3] : 0.f;
+                }
             }
-            m.x = fmaxf(m.x, fabsf(v.x)); m.y = fmaxf(m.y, fabsf(v.y));
-            m.z = fmaxf(m.z, fabsf(v.z)); m.w = fmaxf(m.w, fabsf(v.w));
+#pragma unroll
+            for (int u = 0; u < 8; u++) {
+                m.x = fmaxf(m.x, fabsf(v[u].x)); m.y = fmaxf(m.y, fabsf(v[u].y));
+                m.z = fmaxf(m.z, fabsf(v[u].z)); m.w = fmaxf(m.w, fabsf(v[u].w));
+            }
         }
     }
     red[w][lane] = m;
@@ -684,9 +691,16 @@ __device__ void f16_cols_tile(const F16Cols &j, const unsigned *colmax, int64_t 
         if (k0 == 0 && col < j.N) j.exps[col] = s;
         sc[tid] = __int_as_float((127 + s) << 23);
     }
-    for (int e = tid; e < 64 * 32; e += 256) {
-        const int kk = e >> 5, jj = e & 31;
-        t[kk][jj] = (k0 + kk < j.K && j0 + jj < j.N) ? j.x[(k0 + kk) * j.ldx + j0 + jj] : 0.f;
+    float v[8];  // the tile's eight loads per thread issued before the shared-memory stores
+#pragma unroll
+    for (int u = 0; u < 8; u++) {
+        const int e = tid + 256 * u, kk = e >> 5, jj = e & 31;
+        v[u] = (k0 + kk < j.K && j0 + jj < j.N) ? __ldg(j.x + (k0 + kk) * j.ldx + j0 + jj) : 0.f;
+    }
+#pragma unroll
+    for (int u = 0; u < 8; u++) {
+        const int e = tid + 256 * u;
+        t[e >> 5][e & 31] = v[u];
     }
     __syncthreads();
     for (int e = tid; e < 32 * 32; e += 256) {  // (column jj, k pair kp)
