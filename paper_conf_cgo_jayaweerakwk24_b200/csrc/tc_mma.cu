@@ -543,7 +543,7 @@ struct F16Cols {  // K x N fp32 (pitch ldx) -> transposed hi / lo fp16 [N][ldp] 
     int *exps;
 };
 // one warp per row: the scaled split with the row's exponent from its maximum (f16_max_kernel); 16-byte
-// loads, 8-byte fp16 stores, four column groups in flight per lane
+// loads, 8-byte fp16 stores, eight column groups in flight per lane
 __device__ void f16_rows_body(const F16Rows &j, int64_t w0, int64_t wstride) {
     const int lane = threadIdx.x & 31;
     const bool v4 = ((j.ldx & 3) == 0) && ((reinterpret_cast<uintptr_t>(j.x) & 15) == 0);
@@ -553,10 +553,10 @@ __device__ void f16_rows_body(const F16Rows &j, int64_t w0, int64_t wstride) {
         if (lane == 0) j.exps[r] = s;
         const float sc = __int_as_float((127 + s) << 23);
         __half *hr = j.hi + r * j.ldp, *lr = j.lo + r * j.ldp;
-        for (int64_t c0 = 4 * lane; c0 < j.ldp; c0 += 4 * 128) {  // groups of 4 columns (ldp % 8 == 0)
-            float x[4][4];
+        for (int64_t c0 = 4 * lane; c0 < j.ldp; c0 += 4 * 256) {  // groups of 4 columns (ldp % 8 == 0)
+            float x[8][4];
 #pragma unroll
-            for (int u = 0; u < 4; u++) {
+            for (int u = 0; u < 8; u++) {
                 const int64_t c = c0 + 128 * u;
                 if (v4 && c + 3 < j.cols) {
                     const float4 t = *reinterpret_cast<const float4 *>(xr + c);
@@ -567,7 +567,7 @@ __device__ void f16_rows_body(const F16Rows &j, int64_t w0, int64_t wstride) {
                 }
             }
 #pragma unroll
-            for (int u = 0; u < 4; u++) {
+            for (int u = 0; u < 8; u++) {
                 const int64_t c = c0 + 128 * u;
                 if (c >= j.ldp) break;
                 __half h[4], l[4];
@@ -676,48 +676,35 @@ __global__ void __launch_bounds__(256) f16_max_kernel(const F16Rows r0, unsigned
     const int64_t c = b - nr0 - nr1, nsx = (cj.N + 127) / 128;
     f16_colmax_block(cj.x, cj.K, cj.N, cj.ldx, colmax, c % nsx, c / nsx);
 }
-// one 64 x 32 tile (k-chunk, column strip) of a row-major B: scaled, split and transposed through shared
-// memory so both the reads (along j) and the fp16 writes (along k) are coalesced; the column exponents
-// come from colmax (the k-chunk 0 tile records them)
+// one 32-column x 128-k tile of a row-major B, no shared memory: lane = column, warp w = k rows
+// [16w, 16w + 16) of the tile.  Each of the 16 loads is one coalesced 128-byte row segment across the warp
+// (all issued before the first use); the thread then owns 16 consecutive k of its column and writes them
+// K-major as two 16-byte stores per half (32 bytes = one sector).  The column exponents come from colmax
+// (the k-chunk 0 tile records them).
 __device__ void f16_cols_tile(const F16Cols &j, const unsigned *colmax, int64_t tile) {
-    __shared__ float t[64][33];
-    __shared__ float sc[32];
-    const int tid = threadIdx.x;
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int64_t nstrip = (j.N + 31) / 32;
-    const int64_t strip = tile % nstrip, k0 = (tile / nstrip) * 64, j0 = strip * 32;
-    if (tid < 32) {
-        const int64_t col = j0 + tid;
-        const int s = col < j.N ? f16_scale_exp(__uint_as_float(colmax[col])) : 0;
-        if (k0 == 0 && col < j.N) j.exps[col] = s;
-        sc[tid] = __int_as_float((127 + s) << 23);
-    }
-    float v[8];  // the tile's eight loads per thread issued before the shared-memory stores
+    const int64_t col = (tile % nstrip) * 32 + lane, k0 = (tile / nstrip) * 128 + 16 * w;
+    if (col >= j.N || k0 >= j.ldp) return;
+    const int s = f16_scale_exp(__uint_as_float(colmax[col]));
+    if (k0 == 0) j.exps[col] = s;
+    const float sc = __int_as_float((127 + s) << 23);
+    float v[16];
 #pragma unroll
-    for (int u = 0; u < 8; u++) {
-        const int e = tid + 256 * u, kk = e >> 5, jj = e & 31;
-        v[u] = (k0 + kk < j.K && j0 + jj < j.N) ? __ldg(j.x + (k0 + kk) * j.ldx + j0 + jj) : 0.f;
-    }
+    for (int u = 0; u < 16; u++) v[u] = k0 + u < j.K ? __ldg(j.x + (k0 + u) * j.ldx + col) : 0.f;
+    __half h[16], l[16];
 #pragma unroll
-    for (int u = 0; u < 8; u++) {
-        const int e = tid + 256 * u;
-        t[e >> 5][e & 31] = v[u];
+    for (int u = 0; u < 16; u++) f16_split(v[u], sc, h[u], l[u]);
+    uint4 *hp = reinterpret_cast<uint4 *>(j.hi + col * j.ldp + k0), *lp = reinterpret_cast<uint4 *>(j.lo + col * j.ldp + k0);
+    hp[0] = *reinterpret_cast<const uint4 *>(&h[0]);
+    lp[0] = *reinterpret_cast<const uint4 *>(&l[0]);
+    if (k0 + 8 < j.ldp) {  // ldp % 8 == 0: the second half exists unless the padded k ends here
+        hp[1] = *reinterpret_cast<const uint4 *>(&h[8]);
+        lp[1] = *reinterpret_cast<const uint4 *>(&l[8]);
     }
-    __syncthreads();
-    for (int e = tid; e < 32 * 32; e += 256) {  // (column jj, k pair kp)
-        const int jj = e >> 5, kp = e & 31;
-        if (j0 + jj < j.N && k0 + 2 * kp < j.ldp) {
-            __half h0, l0, h1, l1;
-            f16_split(t[2 * kp][jj], sc[jj], h0, l0);
-            f16_split(t[2 * kp + 1][jj], sc[jj], h1, l1);
-            const int64_t o = (j0 + jj) * j.ldp + k0 + 2 * kp;
-            *reinterpret_cast<__half2 *>(j.hi + o) = __halves2half2(h0, h1);
-            *reinterpret_cast<__half2 *>(j.lo + o) = __halves2half2(l0, l1);
-        }
-    }
-    __syncthreads();
 }
 // The launch before the 3xFP16 GEMM: blocks [0, nbr) split the row operands (A, and B when it is K-major
-// -- syrk), [nbr, nbr + nbc) the 64 x 32 tiles of a row-major B (its column maxima from f16_max_kernel),
+// -- syrk), [nbr, nbr + nbc) the 32 x 128 tiles of a row-major B (its column maxima from f16_max_kernel),
 // the rest the split-k tail pre-pass.
 __global__ void __launch_bounds__(256) prep_f16_kernel(const F16Rows r0, const F16Rows r1, const F16Cols cj,
                                                        const unsigned *colmax, int nbr, int nbc, const Args p,
@@ -730,7 +717,7 @@ __global__ void __launch_bounds__(256) prep_f16_kernel(const F16Rows r0, const F
         return;
     }
     if (b < nbr + nbc) {
-        const int64_t ntiles = ((cj.N + 31) / 32) * ((cj.ldp + 63) / 64);
+        const int64_t ntiles = ((cj.N + 31) / 32) * ((cj.ldp + 127) / 128);
         for (int64_t tile = b - nbr; tile < ntiles; tile += nbc) f16_cols_tile(cj, colmax, tile);
         return;
     }
@@ -1126,7 +1113,7 @@ cudaError_t launch_tcf_contraction(const ContractNest &n, const ContractPlan &p,
     } else {  // row-major B[k][j]: column strips, transposed to K-major
         pr.cj = tcm::F16Cols{B, n.K, n.N, n.ldb, L.Kp, bhi, blo, bexp};
         pr.colmax = bmax;
-        pr.nbc = (int)std::min<int64_t>(((n.N + 31) / 32) * ((L.Kp + 63) / 64), (int64_t)nsm * 8);
+        pr.nbc = (int)std::min<int64_t>(((n.N + 31) / 32) * ((L.Kp + 127) / 128), (int64_t)nsm * 8);
     }
     if (L.share) {
         const int64_t r = (A - B) / n.ldb;
