@@ -1245,7 +1245,7 @@ int64_t eatss_launches_per_run(const eatss_kernel_desc *d, const int64_t *tiles)
         for (auto &n : contraction_nests(d, b)) {
             ContractPlan p = plan_contraction(n, tiles, smem_limit_bytes(), d->exec.warp_align);
             if (!tcf_applicable(n, p)) return -1;
-            total += 2;  // chunk-scaled split + tail pre-pass, GEMM
+            total += 3;  // row / column maxima, split + tail pre-pass, GEMM
         }
         return total;
     }

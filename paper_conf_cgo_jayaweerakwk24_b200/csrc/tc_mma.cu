@@ -79,9 +79,8 @@ struct Args {
     int nunits;   // nfull + (T - nfull) * sp
     int nkb;      // k-blocks of Tk
     int group_rows;  // tile-order grouping (row groups per group) for L2 reuse
-    const int *__restrict__ rexp;  // 3xFP16 engine: power-of-two exponent of each row of A and chunk (scale 2^rexp)
+    const int *__restrict__ rexp;  // 3xFP16 engine: power-of-two exponent of each row of A (scale 2^rexp)
     const int *__restrict__ cexp;  // ... of each column of B
-    int64_t rexp_ld, cexp_ld;      // exps are chunk-major: rexp[chunk * rexp_ld + i], cexp[chunk * cexp_ld + j]
     unsigned long long *prof;  // development (EATSS_TCM_PROF): per-site cycle counters, else nullptr
     int dbg;  // -DEATSS_DEVTOOLS builds only (EATSS_TCM_DBG; results then wrong): 1 no TMEM drain,
               // 4 no accumulator reset at chunk starts
@@ -109,9 +108,8 @@ __device__ __forceinline__ Unit unit_of(const Args &p, int u) {
     } else {
         const int v = u - p.nfull, part = v % p.sp;
         t = p.nfull + v / p.sp;
-        const int nch = (p.nkb + p.R - 1) / p.R;  // split along whole accumulator chunks
-        w.kb0 = min(p.nkb, p.R * (int)((int64_t)part * nch / p.sp));
-        w.kb1 = min(p.nkb, p.R * (int)((int64_t)(part + 1) * nch / p.sp));
+        w.kb0 = (int)((int64_t)part * p.nkb / p.sp);
+        w.kb1 = (int)((int64_t)(part + 1) * p.nkb / p.sp);
         w.split = p.sp > 1;
     }
     tile_coords(t, p.PI, p.TJ, p.group_rows, w.pi, w.tj);
@@ -235,7 +233,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                 const int nk = w.kb1 - w.kb0;
                 for (int x = 0; x < nk; x++, it++) {
                     const int s = it % p.S, bd = gc & 1;
-                    const bool first = (!F16 && (p.dbg & 4)) ? x == 0 : (x % R) == 0;
+                    const bool first = (p.dbg & 4) ? x == 0 : (x % R) == 0;
                     const long long t0 = p.prof ? clock64() : 0;
                     if (first && gc >= 2) mbar_wait_cluster(dempty + bd, (unsigned)(((gc - 2) >> 1) & 1));
                     const long long t1 = p.prof ? clock64() : 0;
@@ -287,9 +285,6 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         for (int u = cid; u < p.nunits; u += ncl) {
             const Unit w = unit_of(p, u);
             const int nch = (w.kb1 - w.kb0 + R - 1) / R;
-            // C(i, j) for row i = i0 + 32q + lane, columns jb .. jb + CW - 1
-            const int64_t i = (int64_t)(w.pi * CG + (int)rank) * BM + q * 32 + lane;
-            const int64_t jb = (int64_t)w.tj * p.BNT + cq * CW;
             float acc[MAXCW];
 #pragma unroll
             for (int c = 0; c < MAXCW; c++) acc[c] = 0.f;
@@ -300,14 +295,6 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                 const long long t1 = p.prof ? clock64() : 0;
                 fence_after();
                 const uint32_t ta = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(bd * 256 + cq * CW);
-                // 3xFP16: this chunk's scales 2^-(s_i,c + u_j,c), applied as two exact power-of-two products
-                float fr = 1.f;
-                const int *ce = nullptr;
-                if constexpr (F16) {
-                    const int64_t gch = w.kb0 / R + ch;
-                    fr = __int_as_float((127 - (i < p.M ? __ldg(p.rexp + gch * p.rexp_ld + i) : 0)) << 23);
-                    ce = p.cexp + gch * p.cexp_ld + jb;
-                }
                 // drain: four 4-column loads in flight per wait
 #pragma unroll
                 for (int c0 = 0; c0 < MAXCW; c0 += 16) {
@@ -320,18 +307,8 @@ __global__ void __launch_bounds__(NTHREADS, 1)
 #pragma unroll
                         for (int g = 0; g < 4; g++)
                             if (c0 + 4 * g < CW) {
-                                if constexpr (F16) {  // lde % 4 == 0: the 16 bytes holding column jb + c exist if it does
-                                    const int4 ex = jb + c0 + 4 * g < p.N ? __ldg(reinterpret_cast<const int4 *>(ce + c0 + 4 * g))
-                                                                          : make_int4(0, 0, 0, 0);
-                                    const int eu[4] = {ex.x, ex.y, ex.z, ex.w};
 #pragma unroll
-                                    for (int c = 0; c < 4; c++)
-                                        acc[c0 + 4 * g + c] = fmaf(__uint_as_float(v[g][c]) * fr,
-                                                                   __int_as_float((127 - eu[c]) << 23), acc[c0 + 4 * g + c]);
-                                } else {
-#pragma unroll
-                                    for (int c = 0; c < 4; c++) acc[c0 + 4 * g + c] += __uint_as_float(v[g][c]);
-                                }
+                                for (int c = 0; c < 4; c++) acc[c0 + 4 * g + c] += __uint_as_float(v[g][c]);
                             }
                     }
                 }
@@ -348,6 +325,17 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                 }
             }
             const long long te = p.prof ? clock64() : 0;
+            // C(i, j) for row i = i0 + 32q + lane, columns jb .. jb + CW - 1
+            const int64_t i = (int64_t)(w.pi * CG + (int)rank) * BM + q * 32 + lane;
+            const int64_t jb = (int64_t)w.tj * p.BNT + cq * CW;
+            if constexpr (F16) {  // undo the power-of-two row / column scales: acc * 2^-(rexp_i + cexp_j), exact
+                if (i < p.M && jb < p.N) {
+                    const float fr = __int_as_float((127 - p.rexp[i]) << 23);
+#pragma unroll
+                    for (int c = 0; c < MAXCW; c++)
+                        if (c < CW && jb + c < p.N) acc[c] = (acc[c] * fr) * __int_as_float((127 - __ldg(p.cexp + jb + c)) << 23);
+                }
+            }
             if (i < p.M && jb < p.N) {
                 float *crow = p.C + i * p.ldc + jb;
                 const bool vec = ((p.ldc & 3) == 0) && (jb + CW <= p.N);
@@ -526,13 +514,10 @@ __global__ void __launch_bounds__(256) prep_kernel(const SplitJob j0, const Spli
 
 
 // ------------------------------------------------------------------ 3xFP16 operand split
-// x = a * 2^-s with a = x * 2^s, s chosen per row (A) / per column (B) and per accumulator chunk of ck k
-// (Args.R k-blocks: the GEMM drains its fp32 accumulator once per chunk anyway) so that max|a| over the
-// chunk lies in [2^14, 2^15): hi = rn_f16(a), lo = rn_f16(a - hi) -- a - hi is exact in fp32 -- so hi + lo
-// carries 22 significant bits of a (the same as tf32 hi + lo) and fp16's range is never exceeded; the GEMM
-// accumulates hi*hi + hi*lo + lo*hi of one chunk in fp32 and its epilogue adds the chunk times
-// 2^-(s_i,c + u_j,c) (exact) to the running sum.  Chunk-local scales need only the chunk's own values, so
-// the split reads each operand element exactly once (no separate maxima pass).
+// x = a * 2^-s with a = x * 2^s, s chosen per row (A) / per column (B) so that max|a| lies in [2^14, 2^15):
+// hi = rn_f16(a), lo = rn_f16(a - hi) -- a - hi is exact in fp32 -- so hi + lo carries 22 significant
+// bits of a (the same as tf32 hi + lo) and fp16's range is never exceeded; the GEMM accumulates
+// hi*hi + hi*lo + lo*hi in fp32 and its epilogue multiplies by 2^-(s_i + u_j) (exact).
 __device__ __forceinline__ int f16_scale_exp(float m) {
     if (!(m > 0.f)) return 0;
     int e;
@@ -544,80 +529,50 @@ __device__ __forceinline__ void f16_split(float x, float sc, __half &h, __half &
     h = __float2half_rn(a);
     l = __float2half_rn(a - __half2float(h));
 }
-__device__ __forceinline__ float warp_max(float m) {
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
-    return m;
-}
-struct F16Rows {  // rows x cols fp32 (pitch ldx) -> hi / lo fp16 [rows][ldp], exps[chunk][lde] (chunk-major)
+struct F16Rows {  // rows x cols fp32 (pitch ldx) -> hi / lo fp16 [rows][ldp], exps[rows]
     const float *x;
     int64_t rows, cols, ldx, ldp;
     __half *hi, *lo;
     int *exps;
-    int64_t lde;
-    int ck;  // k per chunk (Args.R * Tk)
+    const unsigned *maxbits;  // row maxima (bit patterns) from f16_max_kernel
 };
-struct F16Cols {  // K x N fp32 (pitch ldx) -> transposed hi / lo fp16 [N][ldp] (K-major), exps[chunk][lde]
+struct F16Cols {  // K x N fp32 (pitch ldx) -> transposed hi / lo fp16 [N][ldp] (K-major), exps[N]
     const float *x;
     int64_t K, N, ldx, ldp;
     __half *hi, *lo;
     int *exps;
-    int64_t lde;
-    int ck;
 };
-// Row operand, ck % 128 == 0 and ck <= 1024 (the default ck = 256): a warp item is one row's segment of
-// whole chunks (<= 1024 columns); eight 16-byte loads per lane in flight, the chunk maxima by warp
-// shuffles, then the split from registers with 8-byte fp16 stores.
-__device__ void f16_rows_fast(const F16Rows &j, int64_t w0, int64_t wstride) {
+// one warp per row: the scaled split with the row's exponent from its maximum (f16_max_kernel); 16-byte
+// loads, 8-byte fp16 stores, eight column groups in flight per lane
+__device__ void f16_rows_body(const F16Rows &j, int64_t w0, int64_t wstride) {
     const int lane = threadIdx.x & 31;
     const bool v4 = ((j.ldx & 3) == 0) && ((reinterpret_cast<uintptr_t>(j.x) & 15) == 0);
-    const int ck = j.ck, seg = ck * (1024 / ck), nq = seg / ck, upc = ck / 128;
-    const int64_t nseg = (j.ldp + seg - 1) / seg;
-    for (int64_t item = w0; item < j.rows * nseg; item += wstride) {
-        const int64_t r = item / nseg, c0 = (item % nseg) * seg;
+    for (int64_t r = w0; r < j.rows; r += wstride) {
         const float *xr = j.x + r * j.ldx;
-        float4 v[8];
-#pragma unroll
-        for (int u = 0; u < 8; u++) {
-            const int64_t c = c0 + 128 * u + 4 * lane;
-            if (128 * u < seg && v4 && c + 3 < j.cols) {
-                v[u] = __ldg(reinterpret_cast<const float4 *>(xr + c));
-            } else {
-                const bool in = 128 * u < seg;
-                v[u].x = in && c < j.cols ? xr[c] : 0.f;
-                v[u].y = in && c + 1 < j.cols ? xr[c + 1] : 0.f;
-                v[u].z = in && c + 2 < j.cols ? xr[c + 2] : 0.f;
-                v[u].w = in && c + 3 < j.cols ? xr[c + 3] : 0.f;
-            }
-        }
-        float sc[8];
-#pragma unroll
-        for (int q = 0; q < 8; q++) {
-            if (q < nq) {
-                float m = 0.f;
-#pragma unroll
-                for (int u = 0; u < 8; u++)
-                    if (u >= q * upc && u < (q + 1) * upc)
-                        m = fmaxf(m, fmaxf(fmaxf(fabsf(v[u].x), fabsf(v[u].y)), fmaxf(fabsf(v[u].z), fabsf(v[u].w))));
-                m = warp_max(m);
-                const int e = f16_scale_exp(m);
-                if (lane == 0 && c0 + (int64_t)q * ck < j.cols) j.exps[(c0 / ck + q) * j.lde + r] = e;
-                const float f = __int_as_float((127 + e) << 23);
-#pragma unroll
-                for (int u = 0; u < 8; u++)
-                    if (u >= q * upc && u < (q + 1) * upc) sc[u] = f;
-            }
-        }
+        const int s = f16_scale_exp(__uint_as_float(j.maxbits[r]));
+        if (lane == 0) j.exps[r] = s;
+        const float sc = __int_as_float((127 + s) << 23);
         __half *hr = j.hi + r * j.ldp, *lr = j.lo + r * j.ldp;
+        for (int64_t c0 = 4 * lane; c0 < j.ldp; c0 += 4 * 256) {  // groups of 4 columns (ldp % 8 == 0)
+            float x[8][4];
 #pragma unroll
-        for (int u = 0; u < 8; u++) {
-            const int64_t c = c0 + 128 * u + 4 * lane;
-            if (128 * u < seg && c < j.ldp) {  // ldp % 8 == 0: c < ldp -> c + 3 < ldp
+            for (int u = 0; u < 8; u++) {
+                const int64_t c = c0 + 128 * u;
+                if (v4 && c + 3 < j.cols) {
+                    const float4 t = *reinterpret_cast<const float4 *>(xr + c);
+                    x[u][0] = t.x; x[u][1] = t.y; x[u][2] = t.z; x[u][3] = t.w;
+                } else {
+#pragma unroll
+                    for (int q = 0; q < 4; q++) x[u][q] = c + q < j.cols ? xr[c + q] : 0.f;
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < 8; u++) {
+                const int64_t c = c0 + 128 * u;
+                if (c >= j.ldp) break;
                 __half h[4], l[4];
-                f16_split(v[u].x, sc[u], h[0], l[0]);
-                f16_split(v[u].y, sc[u], h[1], l[1]);
-                f16_split(v[u].z, sc[u], h[2], l[2]);
-                f16_split(v[u].w, sc[u], h[3], l[3]);
+#pragma unroll
+                for (int q = 0; q < 4; q++) f16_split(x[u][q], sc, h[q], l[q]);
                 *reinterpret_cast<uint2 *>(hr + c) =
                     make_uint2(*reinterpret_cast<uint32_t *>(&h[0]), *reinterpret_cast<uint32_t *>(&h[2]));
                 *reinterpret_cast<uint2 *>(lr + c) =
@@ -626,88 +581,144 @@ __device__ void f16_rows_fast(const F16Rows &j, int64_t w0, int64_t wstride) {
         }
     }
 }
-// Row operand, any other ck (development chunk lengths): a warp per (row, chunk), maximum pass then split pass
-__device__ void f16_rows_generic(const F16Rows &j, int64_t w0, int64_t wstride) {
-    const int lane = threadIdx.x & 31;
-    const int64_t nchk = (j.cols + j.ck - 1) / j.ck;
-    for (int64_t item = w0; item < j.rows * nchk; item += wstride) {
-        const int64_t r = item / nchk, q = item % nchk, c0 = q * j.ck;
-        const int64_t c1 = c0 + j.ck < j.ldp ? c0 + j.ck : j.ldp;
+// row maxima of up to two row operands: CTA (32 rows, 1024-column chunk), a warp per row and chunk, 16-byte
+// loads (eight per lane in flight); partial maxima meet via atomicMax on the bit pattern
+__device__ void f16_rowmax_block(const F16Rows &j, unsigned *maxbits, int64_t blk) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int64_t nch = (j.cols + 1023) / 1024;
+    const int64_t r0 = (blk / nch) * 32, c0 = (blk % nch) * 1024;
+    const bool v4 = ((j.ldx & 3) == 0) && ((reinterpret_cast<uintptr_t>(j.x) & 15) == 0);
+    for (int q = 0; q < 4; q++) {
+        const int64_t r = r0 + 4 * w + q;
+        if (r >= j.rows) break;
         const float *xr = j.x + r * j.ldx;
         float m = 0.f;
-        for (int64_t c = c0 + lane; c < c1 && c < j.cols; c += 32) m = fmaxf(m, fabsf(xr[c]));
-        const int e = f16_scale_exp(warp_max(m));
-        if (lane == 0) j.exps[q * j.lde + r] = e;
-        const float f = __int_as_float((127 + e) << 23);
-        for (int64_t c = c0 + lane; c < c1; c += 32) f16_split(c < j.cols ? xr[c] : 0.f, f, j.hi[r * j.ldp + c], j.lo[r * j.ldp + c]);
+        if (v4) {
+            float4 v[8];  // all eight loads issued before the first use
+#pragma unroll
+            for (int u = 0; u < 8; u++) {
+                const int64_t c = c0 + 4 * (lane + 32 * u);
+                v[u] = c + 3 < j.cols ? __ldg(reinterpret_cast<const float4 *>(xr + c)) : make_float4(0.f, 0.f, 0.f, 0.f);
+            }
+#pragma unroll
+            for (int u = 0; u < 8; u++)
+                m = fmaxf(m, fmaxf(fmaxf(fabsf(v[u].x), fabsf(v[u].y)), fmaxf(fabsf(v[u].z), fabsf(v[u].w))));
+            const int64_t ce = c0 + 1024 < j.cols ? c0 + 1024 : j.cols;  // a ragged last group of < 4 columns
+            for (int64_t c = (ce & ~3LL) + lane; c < ce && (ce & 3); c += 32) m = fmaxf(m, fabsf(xr[c]));
+        } else {
+            for (int64_t c = c0 + lane; c < c0 + 1024 && c < j.cols; c += 32) m = fmaxf(m, fabsf(xr[c]));
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+        if (lane == 0) atomicMax(maxbits + r, __float_as_uint(m));
     }
 }
-// Column operand (row-major B): a block per (32-column strip, chunk) -- lane = column, warp w = k rows
-// [32w, 32w + 32) of each 256-k segment of the chunk.  Each load is one coalesced 128-byte row segment across
-// the warp (32 in flight per thread); the column maxima meet in shared memory; the split is written K-major
-// as 16-byte stores (64 bytes = two sectors per thread and half).  A chunk longer than one segment
-// (development chunk lengths) is re-read for the split.
-__device__ void f16_cols_chunk(const F16Cols &j, int64_t tile) {
-    __shared__ float red[8][32];
+// column maxima of a row-major B (K x N): CTA (128-column strip, 256-row chunk), 256 threads -- a thread
+// owns four adjacent columns (16-byte loads when aligned), the warps split the chunk, eight loads in
+// flight per thread; partial maxima meet in colmax via atomicMax on the bit pattern (non-negative floats
+// order like their bits)
+__device__ void f16_colmax_block(const float *__restrict__ x, int64_t K, int64_t N, int64_t ldx,
+                                 unsigned *__restrict__ colmax, int64_t bx, int64_t by) {
+    __shared__ float4 red[8][32];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    const int64_t nstrip = (j.N + 31) / 32;
-    const int64_t col = (tile % nstrip) * 32 + lane, q = tile / nstrip;
-    const int64_t kq0 = q * j.ck, kq1 = kq0 + j.ck < j.ldp ? kq0 + j.ck : j.ldp;
-    const int nseg = (int)((kq1 - kq0 + 255) / 256);
-    float v[32];
-    float m = 0.f;
-    for (int sg = 0; sg < nseg; sg++) {
-        const int64_t k0 = kq0 + 256 * sg + 32 * w;
+    const int64_t c0 = bx * 128 + 4 * lane, k0 = by * 256;
+    const bool v4 = ((ldx & 3) == 0) && ((reinterpret_cast<uintptr_t>(x) & 15) == 0) && c0 + 3 < N;
+    float4 m = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (c0 < N) {
+        for (int i0 = w; i0 < 256; i0 += 64) {  // eight rows per pass, all loads issued before their use
+            float4 v[8];
 #pragma unroll
-        for (int u = 0; u < 32; u++)
-            v[u] = (col < j.N && k0 + u < kq1 && k0 + u < j.K) ? __ldg(j.x + (k0 + u) * j.ldx + col) : 0.f;
+            for (int u = 0; u < 8; u++) {
+                const int64_t k = k0 + i0 + 8 * u;
+                const float *row = x + k * ldx + c0;
+                if (k >= K) {
+                    v[u] = make_float4(0.f, 0.f, 0.f, 0.f);
+                } else if (v4) {
+                    v[u] = __ldg(reinterpret_cast<const float4 *>(row));
+                } else {
+                    v[u].x = row[0];
+                    v[u].y = c0 + 1 < N ? row[1] : 0.f;
+                    v[u].z = c0 + 2 < N ? row[2] : 0.f;
+                    v[u].w = c0 + 3 < N ? row[3] : 0.f;
+                }
+            }
 #pragma unroll
-        for (int u = 0; u < 32; u++) m = fmaxf(m, fabsf(v[u]));
+            for (int u = 0; u < 8; u++) {
+                m.x = fmaxf(m.x, fabsf(v[u].x)); m.y = fmaxf(m.y, fabsf(v[u].y));
+                m.z = fmaxf(m.z, fabsf(v[u].z)); m.w = fmaxf(m.w, fabsf(v[u].w));
+            }
+        }
     }
     red[w][lane] = m;
     __syncthreads();
-#pragma unroll
-    for (int t = 0; t < 8; t++) m = fmaxf(m, red[t][lane]);
-    const int e = f16_scale_exp(m);
-    if (w == 0 && col < j.N) j.exps[q * j.lde + col] = e;
-    const float f = __int_as_float((127 + e) << 23);
-    for (int sg = 0; sg < nseg; sg++) {
-        const int64_t k0 = kq0 + 256 * sg + 32 * w;
-        if (nseg > 1) {
-#pragma unroll
-            for (int u = 0; u < 32; u++)
-                v[u] = (col < j.N && k0 + u < kq1 && k0 + u < j.K) ? __ldg(j.x + (k0 + u) * j.ldx + col) : 0.f;
+    if (w == 0 && c0 < N) {
+        for (int q = 1; q < 8; q++) {
+            const float4 o = red[q][lane];
+            m.x = fmaxf(m.x, o.x); m.y = fmaxf(m.y, o.y); m.z = fmaxf(m.z, o.z); m.w = fmaxf(m.w, o.w);
         }
-        if (col < j.N) {
-            uint4 *hp = reinterpret_cast<uint4 *>(j.hi + col * j.ldp + k0), *lp = reinterpret_cast<uint4 *>(j.lo + col * j.ldp + k0);
-#pragma unroll
-            for (int g = 0; g < 4; g++)
-                if (k0 + 8 * g < kq1) {  // kq1 % 8 == 0
-                    __half h[8], l[8];
-#pragma unroll
-                    for (int u = 0; u < 8; u++) f16_split(v[8 * g + u], f, h[u], l[u]);
-                    hp[g] = *reinterpret_cast<const uint4 *>(h);
-                    lp[g] = *reinterpret_cast<const uint4 *>(l);
-                }
-        }
+        const float mm[4] = {m.x, m.y, m.z, m.w};
+        for (int q = 0; q < 4 && c0 + q < N; q++) atomicMax(colmax + c0 + q, __float_as_uint(mm[q]));
     }
-    __syncthreads();  // red is reused by the block's next tile
+}
+// The maxima pass before the 3xFP16 split (one launch): blocks [0, nr0) row maxima of r0, [nr0, nr0 + nr1)
+// of r1, the rest the column maxima of a row-major B (cj; colmax) -- every block independent
+__global__ void __launch_bounds__(256) f16_max_kernel(const F16Rows r0, unsigned *m0, const F16Rows r1, unsigned *m1,
+                                                      const F16Cols cj, unsigned *colmax, int nr0, int nr1) {
+    const int64_t b = blockIdx.x;
+    if (b < nr0) {
+        f16_rowmax_block(r0, m0, b);
+        return;
+    }
+    if (b < nr0 + nr1) {
+        f16_rowmax_block(r1, m1, b - nr0);
+        return;
+    }
+    const int64_t c = b - nr0 - nr1, nsx = (cj.N + 127) / 128;
+    f16_colmax_block(cj.x, cj.K, cj.N, cj.ldx, colmax, c % nsx, c / nsx);
+}
+// one 32-column x 128-k tile of a row-major B, no shared memory: lane = column, warp w = k rows
+// [16w, 16w + 16) of the tile.  Each of the 16 loads is one coalesced 128-byte row segment across the warp
+// (all issued before the first use); the thread then owns 16 consecutive k of its column and writes them
+// K-major as two 16-byte stores per half (32 bytes = one sector).  The column exponents come from colmax
+// (the k-chunk 0 tile records them).
+__device__ void f16_cols_tile(const F16Cols &j, const unsigned *colmax, int64_t tile) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int64_t nstrip = (j.N + 31) / 32;
+    const int64_t col = (tile % nstrip) * 32 + lane, k0 = (tile / nstrip) * 128 + 16 * w;
+    if (col >= j.N || k0 >= j.ldp) return;
+    const int s = f16_scale_exp(__uint_as_float(colmax[col]));
+    if (k0 == 0) j.exps[col] = s;
+    const float sc = __int_as_float((127 + s) << 23);
+    float v[16];
+#pragma unroll
+    for (int u = 0; u < 16; u++) v[u] = k0 + u < j.K ? __ldg(j.x + (k0 + u) * j.ldx + col) : 0.f;
+    __half h[16], l[16];
+#pragma unroll
+    for (int u = 0; u < 16; u++) f16_split(v[u], sc, h[u], l[u]);
+    uint4 *hp = reinterpret_cast<uint4 *>(j.hi + col * j.ldp + k0), *lp = reinterpret_cast<uint4 *>(j.lo + col * j.ldp + k0);
+    hp[0] = *reinterpret_cast<const uint4 *>(&h[0]);
+    lp[0] = *reinterpret_cast<const uint4 *>(&l[0]);
+    if (k0 + 8 < j.ldp) {  // ldp % 8 == 0: the second half exists unless the padded k ends here
+        hp[1] = *reinterpret_cast<const uint4 *>(&h[8]);
+        lp[1] = *reinterpret_cast<const uint4 *>(&l[8]);
+    }
 }
 // The launch before the 3xFP16 GEMM: blocks [0, nbr) split the row operands (A, and B when it is K-major
-// -- syrk), [nbr, nbr + nbc) the (strip, chunk) tiles of a row-major B, the rest the split-k tail pre-pass.
-__global__ void __launch_bounds__(256, 3) prep_f16_kernel(const F16Rows r0, const F16Rows r1, const F16Cols cj, int nbr,
-                                                       int nbc, const Args p, int rows_per_tile, int bn, int vecC) {
+// -- syrk), [nbr, nbr + nbc) the 32 x 128 tiles of a row-major B (its column maxima from f16_max_kernel),
+// the rest the split-k tail pre-pass.
+__global__ void __launch_bounds__(256) prep_f16_kernel(const F16Rows r0, const F16Rows r1, const F16Cols cj,
+                                                       const unsigned *colmax, int nbr, int nbc, const Args p,
+                                                       int rows_per_tile, int bn, int vecC) {
     const int b = (int)blockIdx.x;
     if (b < nbr) {
         const int64_t wstride = (int64_t)nbr * 8, w0 = (int64_t)b * 8 + (threadIdx.x >> 5);
-        const bool fast = r0.ck % 128 == 0 && r0.ck <= 1024;
-        if (r0.x) fast ? f16_rows_fast(r0, w0, wstride) : f16_rows_generic(r0, w0, wstride);
-        if (r1.x) fast ? f16_rows_fast(r1, w0, wstride) : f16_rows_generic(r1, w0, wstride);
+        if (r0.x) f16_rows_body(r0, w0, wstride);
+        if (r1.x) f16_rows_body(r1, w0, wstride);
         return;
     }
     if (b < nbr + nbc) {
-        const int64_t ntiles = ((cj.N + 31) / 32) * ((cj.K + cj.ck - 1) / cj.ck);
-        for (int64_t tile = b - nbr; tile < ntiles; tile += nbc) f16_cols_chunk(cj, tile);
+        const int64_t ntiles = ((cj.N + 31) / 32) * ((cj.ldp + 127) / 128);
+        for (int64_t tile = b - nbr; tile < ntiles; tile += nbc) f16_cols_tile(cj, colmax, tile);
         return;
     }
     const int npb = (int)gridDim.x - nbr - nbc, g4 = (bn + 3) / 4;
@@ -743,6 +754,10 @@ struct Prep {
     // 3xFP16: row splits (A; B when K-major) and the column strips of a row-major B
     tcm::F16Rows r0{}, r1{};
     tcm::F16Cols cj{};
+    unsigned *colmax = nullptr;  // row-major B: per-column max bits (f16_max_kernel before the prep launch)
+    unsigned *maxes = nullptr;   // the zero-initialised region holding every max array of this GEMM
+    size_t maxes_bytes = 0;
+    unsigned *m0 = nullptr, *m1 = nullptr;  // row maxima of r0 / r1
     int nbr = 0, nbc = 0;
 };
 
@@ -792,7 +807,7 @@ static void schedule(tcm::Args &a, int ncl) {
     a.nfull = a.T;
     static const bool splitk = devsw("EATSS_TCM_SPLITK", 1) != 0;
     if (rem > 0 && splitk) {
-        const int sp = std::min(std::min(4, ncl / rem), (a.nkb + a.R - 1) / a.R);
+        const int sp = std::min(std::min(4, ncl / rem), a.nkb);
         if (sp >= 2) {
             a.sp = sp;
             a.nfull = a.T - rem;
@@ -857,7 +872,18 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
         const int npb = (int)std::min<int64_t>((tail4 + 255) / 256, (int64_t)nsm * 4);
         const int vecC = (a.ldc % 4 == 0 && (reinterpret_cast<uintptr_t>(a.C) & 15) == 0) ? 1 : 0;
         if constexpr (F16) {
-            tcm::prep_f16_kernel<<<pr.nbr + pr.nbc + npb, 256, 0, s>>>(pr.r0, pr.r1, pr.cj, pr.nbr,
+            {  // maxima of every row of the row operands and column of a row-major B (the split needs them)
+                if ((e = cudaMemsetAsync(pr.maxes, 0, pr.maxes_bytes, s)) != cudaSuccess) return e;
+                auto nrb = [](const tcm::F16Rows &r) {
+                    return r.x ? (int)(((r.rows + 31) / 32) * ((r.cols + 1023) / 1024)) : 0;
+                };
+                const int nr0 = nrb(pr.r0), nr1 = nrb(pr.r1);
+                const int ncb = pr.colmax ? (int)(((pr.cj.N + 127) / 128) * ((pr.cj.K + 255) / 256)) : 0;
+                tcm::f16_max_kernel<<<nr0 + nr1 + ncb, 256, 0, s>>>(pr.r0, pr.m0, pr.r1, pr.m1, pr.cj, pr.colmax, nr0,
+                                                                    nr1);
+                if ((e = cudaGetLastError()) != cudaSuccess) return e;
+            }
+            tcm::prep_f16_kernel<<<pr.nbr + pr.nbc + npb, 256, 0, s>>>(pr.r0, pr.r1, pr.cj, pr.colmax, pr.nbr,
                                                                        pr.nbc, a, rows, a.BNT, vecC);
         } else {
             tcm::prep_kernel<<<pr.nb0 + pr.nb1 + npb, 256, 0, s>>>(pr.j0, pr.j1, pr.nb0, pr.nb1, pr.mode, a, rows,
@@ -1008,7 +1034,6 @@ cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p,
         a.prof = prof;
     }
     a.rexp = a.cexp = nullptr;
-    a.rexp_ld = a.cexp_ld = 0;
     cudaError_t r;
     const int bkb = 4 * bk;
     if (n.transB)
@@ -1032,52 +1057,42 @@ cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p,
 
 // ------------------------------------------------------------------ 3xFP16 engine (engine = TENSOR_F16)
 namespace {
-struct F16Layout {  // workspace offsets (bytes, 256-aligned): hi/lo fp16 operands and their chunk exponents
-    int64_t Kp = 0, nchk = 0, lde_a = 0, lde_b = 0;
-    size_t a_hi = 0, a_lo = 0, a_exp = 0, b_hi = 0, b_lo = 0, b_exp = 0, total = 0;
+struct F16Layout {  // workspace offsets (bytes, 256-aligned): hi/lo fp16 operands and their exponents
+    int64_t Kp = 0;
+    size_t a_hi = 0, a_lo = 0, a_exp = 0, b_hi = 0, b_lo = 0, b_exp = 0, b_max = 0, a_max = 0, max_end = 0, total = 0;
     bool share = false;  // syrk: A is a row block of the K-major B
 };
-// ck: k per accumulator chunk (the scale granularity along k)
-F16Layout f16_layout(const ContractNest &n, int64_t ck) {
+F16Layout f16_layout(const ContractNest &n) {
     F16Layout L;
     const float *A = static_cast<const float *>(n.A), *B = static_cast<const float *>(n.B);
     L.Kp = (n.K + 7) / 8 * 8;  // 16-byte fp16 rows (TMA strides)
-    L.nchk = (n.K + ck - 1) / ck;
     L.share = n.transB && n.lda == n.ldb && A >= B && (A - B) % n.ldb == 0 && (A - B) / n.ldb + n.M <= n.N;
-    L.lde_b = (n.N + 3) / 4 * 4;  // exps[chunk][lde]: 16-byte rows (the epilogue reads four columns at once)
-    L.lde_a = L.share ? L.lde_b : (n.M + 3) / 4 * 4;
     auto al = [](size_t v) { return (v + 255) / 256 * 256; };
     size_t o = 0;
     L.b_hi = o; o = al(o + (size_t)n.N * L.Kp * 2);
     L.b_lo = o; o = al(o + (size_t)n.N * L.Kp * 2);
-    L.b_exp = o; o = al(o + (size_t)L.nchk * L.lde_b * 4);
+    L.b_exp = o; o = al(o + (size_t)n.N * 4);
+    L.b_max = o; o = o + (size_t)n.N * 4;   // maxima: b_max then a_max, contiguous (one memset)
+    L.a_max = o; o = o + (L.share ? 0 : (size_t)n.M * 4);
+    L.max_end = o; o = al(o);
     if (!L.share) {
         L.a_hi = o; o = al(o + (size_t)n.M * L.Kp * 2);
         L.a_lo = o; o = al(o + (size_t)n.M * L.Kp * 2);
-        L.a_exp = o; o = al(o + (size_t)L.nchk * L.lde_a * 4);
+        L.a_exp = o; o = al(o + (size_t)n.M * 4);
     }
     L.total = o;
     return L;
 }
-// k per accumulator chunk of this tile (Args.R k-blocks)
-int f16_chunk_k(const TcmGeom &g) {
-    static const int chunk_env = devsw("EATSS_TCM_CHUNK_K", 0);  // development: k per accumulator chunk
-    const int bk = std::max(1, g.bk);
-    return std::max(1, (chunk_env > 0 ? chunk_env : tcm::CHUNK_K_F16) / bk) * bk;
-}
 }  // namespace
 
 bool tcf_applicable(const ContractNest &n, const ContractPlan &p) { return tcm_geom(n, p, true).ok; }
-size_t tcf_ws_floats(const ContractNest &n, const ContractPlan &p) {
-    return f16_layout(n, f16_chunk_k(tcm_geom(n, p, true))).total / 4 + 64;
-}
+size_t tcf_ws_floats(const ContractNest &n, const ContractPlan &) { return f16_layout(n).total / 4 + 64; }
 
 cudaError_t launch_tcf_contraction(const ContractNest &n, const ContractPlan &p, float *ws, size_t ws_floats,
                                    cudaStream_t s, cudaEvent_t *ev) {
     const TcmGeom g = tcm_geom(n, p, true);
     if (!g.ok) return cudaErrorNotSupported;
-    const int ck = f16_chunk_k(g);
-    const F16Layout L = f16_layout(n, ck);
+    const F16Layout L = f16_layout(n);
     if (!ws || ws_floats * 4 < L.total) return cudaErrorInvalidValue;
     char *w = reinterpret_cast<char *>(ws);
     const float *A = static_cast<const float *>(n.A), *B = static_cast<const float *>(n.B);
@@ -1089,11 +1104,16 @@ cudaError_t launch_tcf_contraction(const ContractNest &n, const ContractPlan &p,
     int dev = 0, nsm = 148;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    unsigned *bmax = reinterpret_cast<unsigned *>(w + L.b_max), *amax = reinterpret_cast<unsigned *>(w + L.a_max);
+    pr.maxes = bmax;
+    pr.maxes_bytes = L.max_end - L.b_max;
     if (n.transB) {  // B(k, j) = B[j*ldb + k]: rows j are already K-major -> row split, row scale = column scale
-        pr.r0 = tcm::F16Rows{B, n.N, n.K, n.ldb, L.Kp, bhi, blo, bexp, L.lde_b, ck};
+        pr.r0 = tcm::F16Rows{B, n.N, n.K, n.ldb, L.Kp, bhi, blo, bexp, bmax};
+        pr.m0 = bmax;
     } else {  // row-major B[k][j]: column strips, transposed to K-major
-        pr.cj = tcm::F16Cols{B, n.K, n.N, n.ldb, L.Kp, bhi, blo, bexp, L.lde_b, ck};
-        pr.nbc = (int)std::min<int64_t>(((n.N + 31) / 32) * L.nchk, (int64_t)nsm * 8);
+        pr.cj = tcm::F16Cols{B, n.K, n.N, n.ldb, L.Kp, bhi, blo, bexp};
+        pr.colmax = bmax;
+        pr.nbc = (int)std::min<int64_t>(((n.N + 31) / 32) * ((L.Kp + 127) / 128), (int64_t)nsm * 8);
     }
     if (L.share) {
         const int64_t r = (A - B) / n.ldb;
@@ -1103,7 +1123,8 @@ cudaError_t launch_tcf_contraction(const ContractNest &n, const ContractPlan &p,
     } else {
         __half *h = reinterpret_cast<__half *>(w + L.a_hi), *l = reinterpret_cast<__half *>(w + L.a_lo);
         int *e = reinterpret_cast<int *>(w + L.a_exp);
-        (n.transB ? pr.r1 : pr.r0) = tcm::F16Rows{A, n.M, n.K, n.lda, L.Kp, h, l, e, L.lde_a, ck};
+        (n.transB ? pr.r1 : pr.r0) = tcm::F16Rows{A, n.M, n.K, n.lda, L.Kp, h, l, e, amax};
+        (n.transB ? pr.m1 : pr.m0) = amax;
         ahi = h;
         alo = l;
         aexp = e;
@@ -1126,7 +1147,8 @@ cudaError_t launch_tcf_contraction(const ContractNest &n, const ContractPlan &p,
     a.C = static_cast<float *>(n.C); a.ldc = n.ldc;
     a.alpha = (float)n.alpha; a.beta = (float)n.beta; a.init_zero = n.init_zero ? 1 : 0;
     a.S = g.S;
-    a.R = ck / g.bk;
+    static const int chunk_env = devsw("EATSS_TCM_CHUNK_K", 0);  // development: k per accumulator chunk
+    a.R = std::max(1, (chunk_env > 0 ? chunk_env : tcm::CHUNK_K_F16) / g.bk);
     a.BNT = g.bn; a.BNH = g.bnh; a.bgroups = g.bgroups; a.b_bytes = g.b_bytes; a.stage = g.stage;
     a.idesc = tcm::idesc_f16(g.bn, g.cg);
     a.nkb = (int)((n.K + g.bk - 1) / g.bk);
@@ -1138,8 +1160,6 @@ cudaError_t launch_tcf_contraction(const ContractNest &n, const ContractPlan &p,
     a.dbg = 0;
     a.rexp = aexp;
     a.cexp = bexp;
-    a.rexp_ld = L.lde_a;
-    a.cexp_ld = L.lde_b;
     return g.cg == 2 ? launch_bk<true, 2, true>(bkb, m, a, g.smem, nsm, pr, s, ev)
                      : launch_bk<true, 1, true>(bkb, m, a, g.smem, nsm, pr, s, ev);
 }
