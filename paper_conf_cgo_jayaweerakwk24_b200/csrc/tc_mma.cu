@@ -961,6 +961,35 @@ size_t tcm_ws_floats(const ContractNest &n, const ContractPlan &) {
     return (size_t)(o.ob.need + (o.share ? 0 : o.oa.need) + 64);
 }
 
+// development switches of one GEMM launch: EATSS_TCM_DBG (-DEATSS_DEVTOOLS builds only; results then
+// wrong) and EATSS_TCM_PROF (wait / drain / epilogue cycle profile, printed after the launch)
+static void dev_setup(tcm::Args &a, cudaStream_t s) {
+    a.prof = nullptr;
+#ifdef EATSS_DEVTOOLS
+    a.dbg = devsw("EATSS_TCM_DBG", 0);
+#else
+    a.dbg = 0;
+#endif
+    static unsigned long long *prof = nullptr;
+    if (devsw("EATSS_TCM_PROF", 0)) {
+        if (!prof) cudaMalloc(&prof, 16 * sizeof(unsigned long long));
+        cudaMemsetAsync(prof, 0, 16 * sizeof(unsigned long long), s);
+        a.prof = prof;
+    }
+}
+static void dev_report(const tcm::Args &a, cudaStream_t s) {
+    if (a.prof) {
+        unsigned long long h[16];
+        cudaMemcpyAsync(h, a.prof, sizeof(h), cudaMemcpyDeviceToHost, s);
+        cudaStreamSynchronize(s);
+        const double nmma = (double)a.PI * a.TJ * a.nkb;  // k-blocks issued
+        fprintf(stderr,
+                "tc_mma prof: MMA wait dempty %.0f / wait full %.0f cycles per k-block | EPI wait dfull %.0f / "
+                "drain %.0f per chunk-warp (%llu) | C epilogue %.0f per tile-warp (%llu)\n",
+                h[0] / nmma, h[1] / nmma, h[2] / (double)h[4], h[3] / (double)h[4], h[4], h[5] / (double)h[6], h[6]);
+    }
+}
+
 cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p, float *ws, size_t ws_floats,
                                    cudaStream_t s, cudaEvent_t *ev) {
     const TcmGeom g = tcm_geom(n, p);
@@ -1021,18 +1050,7 @@ cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p,
     a.TJ = (int)((n.N + bn - 1) / bn);
     static const int group_env = devsw("EATSS_TCM_GROUP", 8);  // development: row groups per raster group
     a.group_rows = std::max(1, group_env);
-    a.prof = nullptr;
-#ifdef EATSS_DEVTOOLS
-    a.dbg = devsw("EATSS_TCM_DBG", 0);
-#else
-    a.dbg = 0;
-#endif
-    static unsigned long long *prof = nullptr;
-    if (devsw("EATSS_TCM_PROF", 0)) {  // development: wait / drain / epilogue cycle profile (printed)
-        if (!prof) cudaMalloc(&prof, 16 * sizeof(unsigned long long));
-        cudaMemsetAsync(prof, 0, 16 * sizeof(unsigned long long), s);
-        a.prof = prof;
-    }
+    dev_setup(a, s);
     a.rexp = a.cexp = nullptr;
     cudaError_t r;
     const int bkb = 4 * bk;
@@ -1042,16 +1060,7 @@ cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p,
     else
         r = cg == 2 ? launch_bk<false, 2, false>(bkb, m, a, g.smem, nsm, pr, s, ev)
                     : launch_bk<false, 1, false>(bkb, m, a, g.smem, nsm, pr, s, ev);
-    if (a.prof) {
-        unsigned long long h[16];
-        cudaMemcpyAsync(h, a.prof, sizeof(h), cudaMemcpyDeviceToHost, s);
-        cudaStreamSynchronize(s);
-        const double nmma = (double)a.nunits * a.nkb;  // k-blocks issued (approx.)
-        fprintf(stderr,
-                "tc_mma prof: MMA wait dempty %.0f / wait full %.0f cycles per k-block | EPI wait dfull %.0f / "
-                "drain %.0f per chunk-warp (%llu) | C epilogue %.0f per tile-warp (%llu)\n",
-                h[0] / nmma, h[1] / nmma, h[2] / (double)h[4], h[3] / (double)h[4], h[4], h[5] / (double)h[6], h[6]);
-    }
+    dev_report(a, s);
     return r;
 }
 
@@ -1156,12 +1165,13 @@ cudaError_t launch_tcf_contraction(const ContractNest &n, const ContractPlan &p,
     a.TJ = (int)((n.N + g.bn - 1) / g.bn);
     static const int group_env = devsw("EATSS_TCM_GROUP", 8);
     a.group_rows = std::max(1, group_env);
-    a.prof = nullptr;
-    a.dbg = 0;
+    dev_setup(a, s);
     a.rexp = aexp;
     a.cexp = bexp;
-    return g.cg == 2 ? launch_bk<true, 2, true>(bkb, m, a, g.smem, nsm, pr, s, ev)
-                     : launch_bk<true, 1, true>(bkb, m, a, g.smem, nsm, pr, s, ev);
+    const cudaError_t r = g.cg == 2 ? launch_bk<true, 2, true>(bkb, m, a, g.smem, nsm, pr, s, ev)
+                                    : launch_bk<true, 1, true>(bkb, m, a, g.smem, nsm, pr, s, ev);
+    dev_report(a, s);
+    return r;
 }
 
 int tcm_launches(const ContractNest &, const ContractPlan &) {
