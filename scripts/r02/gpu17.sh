@@ -1,6 +1,6 @@
 # accumulator-chunk cost study (development build with -DEATSS_DEVTOOLS; numbers are not bench values)
 cd $GRAFT_REPO_ROOT; mkdir -p gpurun_out/r02
-EATSS_DEV_NVCC_FLAGS=-DEATSS_DEVTOOLS python paper_conf_cgo_jayaweerakwk24_b200/build.py -j 32 > /dev/null 2>&1 || echo BUILD FAILED
+EATSS_DEV_NVCC_FLAGS=-DEATSS_DEVTOOLS python paper_conf_cgo_jayaweerakwk24_b200/build.py --force -j 32 > /dev/null 2>&1 || echo BUILD FAILED
 T=scripts/time_kernel.py
 for spec in "4 256,256,64 256" "4 256,256,64 4000" "2 256,256,32 128" "2 256,256,32 4000"; do
   set -- $spec
