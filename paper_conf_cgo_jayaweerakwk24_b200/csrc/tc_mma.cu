@@ -83,7 +83,8 @@ struct Args {
     const int *__restrict__ cexp;  // ... of each column of B
     unsigned long long *prof;  // development (EATSS_TCM_PROF): per-site cycle counters, else nullptr
     int dbg;  // -DEATSS_DEVTOOLS builds only (EATSS_TCM_DBG; results then wrong): 1 no TMEM drain,
-              // 4 no accumulator reset at chunk starts
+              // 4 no accumulator reset at chunk starts, 8 no
+              // wait for the drained buffer at chunk starts inside a tile (only at tile starts)
 };
 
 __host__ __device__ inline void tile_coords(int t, int PI, int TJ, int G, int &pi, int &tj) {
@@ -235,7 +236,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                     const int s = it % p.S, bd = gc & 1;
                     const bool first = (p.dbg & 4) ? x == 0 : (x % R) == 0;
                     const long long t0 = p.prof ? clock64() : 0;
-                    if (first && gc >= 2) mbar_wait_cluster(dempty + bd, (unsigned)(((gc - 2) >> 1) & 1));
+                    if (first && gc >= 2 && !((p.dbg & 8) && x > 0)) mbar_wait_cluster(dempty + bd, (unsigned)(((gc - 2) >> 1) & 1));
                     const long long t1 = p.prof ? clock64() : 0;
                     mbar_wait(full + s, (unsigned)((it / p.S) & 1));
                     if (p.prof) {
