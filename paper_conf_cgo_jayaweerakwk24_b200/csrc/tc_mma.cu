@@ -707,7 +707,7 @@ __device__ void f16_cols_tile(const F16Cols &j, const unsigned *colmax, int64_t 
 // The launch before the 3xFP16 GEMM: blocks [0, nbr) split the row operands (A, and B when it is K-major
 // -- syrk), [nbr, nbr + nbc) the 32 x 128 tiles of a row-major B (its column maxima from f16_max_kernel),
 // the rest the split-k tail pre-pass.
-__global__ void __launch_bounds__(256) prep_f16_kernel(const F16Rows r0, const F16Rows r1, const F16Cols cj,
+__global__ void __launch_bounds__(256, 4) prep_f16_kernel(const F16Rows r0, const F16Rows r1, const F16Cols cj,
                                                        const unsigned *colmax, int nbr, int nbc, const Args p,
                                                        int rows_per_tile, int bn, int vecC) {
     const int b = (int)blockIdx.x;
