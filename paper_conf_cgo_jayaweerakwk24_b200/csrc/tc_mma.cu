@@ -544,7 +544,7 @@ struct F16Cols {  // K x N fp32 (pitch ldx) -> transposed hi / lo fp16 [N][ldp] 
     int *exps;
 };
 // one warp per row: the scaled split with the row's exponent from its maximum (f16_max_kernel); 16-byte
-// loads, 8-byte fp16 stores, sixteen column groups in flight per lane
+// loads, 8-byte fp16 stores, eight column groups in flight per lane
 __device__ void f16_rows_body(const F16Rows &j, int64_t w0, int64_t wstride) {
     const int lane = threadIdx.x & 31;
     const bool v4 = ((j.ldx & 3) == 0) && ((reinterpret_cast<uintptr_t>(j.x) & 15) == 0);
@@ -554,10 +554,10 @@ __device__ void f16_rows_body(const F16Rows &j, int64_t w0, int64_t wstride) {
         if (lane == 0) j.exps[r] = s;
         const float sc = __int_as_float((127 + s) << 23);
         __half *hr = j.hi + r * j.ldp, *lr = j.lo + r * j.ldp;
-        for (int64_t c0 = 4 * lane; c0 < j.ldp; c0 += 4 * 512) {  // groups of 4 columns (ldp % 8 == 0)
-            float x[16][4];
+        for (int64_t c0 = 4 * lane; c0 < j.ldp; c0 += 4 * 256) {  // groups of 4 columns (ldp % 8 == 0)
+            float x[8][4];
 #pragma unroll
-            for (int u = 0; u < 16; u++) {
+            for (int u = 0; u < 8; u++) {
                 const int64_t c = c0 + 128 * u;
                 if (v4 && c + 3 < j.cols) {
                     const float4 t = *reinterpret_cast<const float4 *>(xr + c);
@@ -568,7 +568,7 @@ __device__ void f16_rows_body(const F16Rows &j, int64_t w0, int64_t wstride) {
                 }
             }
 #pragma unroll
-            for (int u = 0; u < 16; u++) {
+            for (int u = 0; u < 8; u++) {
                 const int64_t c = c0 + 128 * u;
                 if (c >= j.ldp) break;
                 __half h[4], l[4];
@@ -677,37 +677,37 @@ __global__ void __launch_bounds__(256) f16_max_kernel(const F16Rows r0, unsigned
     const int64_t c = b - nr0 - nr1, nsx = (cj.N + 127) / 128;
     f16_colmax_block(cj.x, cj.K, cj.N, cj.ldx, colmax, c % nsx, c / nsx);
 }
-// one 32-column x 256-k tile of a row-major B, no shared memory: lane = column, warp w = k rows
-// [32w, 32w + 32) of the tile.  Each of the 32 loads is one coalesced 128-byte row segment across the warp
-// (all issued before the first use); the thread then owns 32 consecutive k of its column and writes them
-// K-major as four 16-byte stores per half (two sectors).  The column exponents come from colmax
+// one 32-column x 128-k tile of a row-major B, no shared memory: lane = column, warp w = k rows
+// [16w, 16w + 16) of the tile.  Each of the 16 loads is one coalesced 128-byte row segment across the warp
+// (all issued before the first use); the thread then owns 16 consecutive k of its column and writes them
+// K-major as two 16-byte stores per half (32 bytes = one sector).  The column exponents come from colmax
 // (the k-chunk 0 tile records them).
 __device__ void f16_cols_tile(const F16Cols &j, const unsigned *colmax, int64_t tile) {
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int64_t nstrip = (j.N + 31) / 32;
-    const int64_t col = (tile % nstrip) * 32 + lane, k0 = (tile / nstrip) * 256 + 32 * w;
+    const int64_t col = (tile % nstrip) * 32 + lane, k0 = (tile / nstrip) * 128 + 16 * w;
     if (col >= j.N || k0 >= j.ldp) return;
     const int s = f16_scale_exp(__uint_as_float(colmax[col]));
     if (k0 == 0) j.exps[col] = s;
     const float sc = __int_as_float((127 + s) << 23);
-    float v[32];
+    float v[16];
 #pragma unroll
-    for (int u = 0; u < 32; u++) v[u] = k0 + u < j.K ? __ldg(j.x + (k0 + u) * j.ldx + col) : 0.f;
+    for (int u = 0; u < 16; u++) v[u] = k0 + u < j.K ? __ldg(j.x + (k0 + u) * j.ldx + col) : 0.f;
+    __half h[16], l[16];
+#pragma unroll
+    for (int u = 0; u < 16; u++) f16_split(v[u], sc, h[u], l[u]);
     uint4 *hp = reinterpret_cast<uint4 *>(j.hi + col * j.ldp + k0), *lp = reinterpret_cast<uint4 *>(j.lo + col * j.ldp + k0);
-#pragma unroll
-    for (int g = 0; g < 4; g++)
-        if (k0 + 8 * g < j.ldp) {  // ldp % 8 == 0: each 8-k group is whole or absent
-            __half h[8], l[8];
-#pragma unroll
-            for (int u = 0; u < 8; u++) f16_split(v[8 * g + u], sc, h[u], l[u]);
-            hp[g] = *reinterpret_cast<const uint4 *>(h);
-            lp[g] = *reinterpret_cast<const uint4 *>(l);
-        }
+    hp[0] = *reinterpret_cast<const uint4 *>(&h[0]);
+    lp[0] = *reinterpret_cast<const uint4 *>(&l[0]);
+    if (k0 + 8 < j.ldp) {  // ldp % 8 == 0: the second half exists unless the padded k ends here
+        hp[1] = *reinterpret_cast<const uint4 *>(&h[8]);
+        lp[1] = *reinterpret_cast<const uint4 *>(&l[8]);
+    }
 }
 // The launch before the 3xFP16 GEMM: blocks [0, nbr) split the row operands (A, and B when it is K-major
-// -- syrk), [nbr, nbr + nbc) the 32 x 256 tiles of a row-major B (its column maxima from f16_max_kernel),
+// -- syrk), [nbr, nbr + nbc) the 32 x 128 tiles of a row-major B (its column maxima from f16_max_kernel),
 // the rest the split-k tail pre-pass.
-__global__ void __launch_bounds__(256, 3) prep_f16_kernel(const F16Rows r0, const F16Rows r1, const F16Cols cj,
+__global__ void __launch_bounds__(256, 4) prep_f16_kernel(const F16Rows r0, const F16Rows r1, const F16Cols cj,
                                                        const unsigned *colmax, int nbr, int nbc, const Args p,
                                                        int rows_per_tile, int bn, int vecC) {
     const int b = (int)blockIdx.x;
@@ -718,7 +718,7 @@ __global__ void __launch_bounds__(256, 3) prep_f16_kernel(const F16Rows r0, cons
         return;
     }
     if (b < nbr + nbc) {
-        const int64_t ntiles = ((cj.N + 31) / 32) * ((cj.ldp + 255) / 256);
+        const int64_t ntiles = ((cj.N + 31) / 32) * ((cj.ldp + 127) / 128);
         for (int64_t tile = b - nbr; tile < ntiles; tile += nbc) f16_cols_tile(cj, colmax, tile);
         return;
     }
@@ -1123,7 +1123,7 @@ cudaError_t launch_tcf_contraction(const ContractNest &n, const ContractPlan &p,
     } else {  // row-major B[k][j]: column strips, transposed to K-major
         pr.cj = tcm::F16Cols{B, n.K, n.N, n.ldb, L.Kp, bhi, blo, bexp};
         pr.colmax = bmax;
-        pr.nbc = (int)std::min<int64_t>(((n.N + 31) / 32) * ((L.Kp + 255) / 256), (int64_t)nsm * 8);
+        pr.nbc = (int)std::min<int64_t>(((n.N + 31) / 32) * ((L.Kp + 127) / 128), (int64_t)nsm * 8);
     }
     if (L.share) {
         const int64_t r = (A - B) / n.ldb;
