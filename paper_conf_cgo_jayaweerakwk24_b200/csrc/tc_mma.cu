@@ -81,6 +81,8 @@ struct Args {
     int group_rows;  // tile-order grouping (row groups per group) for L2 reuse
     const int *__restrict__ rexp;  // 3xFP16 engine: power-of-two exponent of each row of A (scale 2^rexp)
     const int *__restrict__ cexp;  // ... of each column of B
+    int fuse;  // 3xTF32: lo halves formed in shared memory by the converter warps (2, 3) from the landed hi
+               // tiles (TMA loads hi only); 0: both halves loaded (lo materialised by the prep launch)
     unsigned long long *prof;  // development (EATSS_TCM_PROF): per-site cycle counters, else nullptr
     int dbg;  // -DEATSS_DEVTOOLS builds only (EATSS_TCM_DBG; results then wrong): 1 no TMEM drain,
               // 4 no accumulator reset at chunk starts, 8 no
@@ -133,6 +135,14 @@ struct KMajor {
 
 // BKB: bytes of k per operand row and stage; F16: 3xFP16 operands (K-major A and B, per-row / per-column
 // power-of-two scales undone in the epilogue), else 3xTF32
+// lo half of four fp32 values for the raw-hi 3xTF32 split (the tensor core reads hi = rz_tf32(x) from x)
+__device__ __forceinline__ float lo1(float x) {
+    uint32_t l;
+    asm("cvt.rna.tf32.f32 %0, %1;\n" : "=r"(l) : "f"(x - __uint_as_float(__float_as_uint(x) & 0xFFFFE000u)));
+    return __uint_as_float(l);
+}
+__device__ __forceinline__ float4 lo4(float4 x) { return make_float4(lo1(x.x), lo1(x.y), lo1(x.z), lo1(x.w)); }
+
 template <int BKB, bool TB, int CG, bool F16>
 __global__ void __launch_bounds__(NTHREADS, 1)
     tc_mma_kernel(const __grid_constant__ CUtensorMap mAhi, const __grid_constant__ CUtensorMap mAlo,
@@ -154,12 +164,16 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     uint64_t *empty = full + p.S;
     uint64_t *dfull = empty + p.S;
     uint64_t *dempty = dfull + 2;
-    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(dempty + 2);
+    uint64_t *lfull = dempty + 2;  // fuse: this CTA's hi tiles of the stage landed (local TMA bytes)
+    uint64_t *conv = lfull + p.S;  // fuse (leader): both CTAs' lo halves of the stage written
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(conv + p.S);
 
     if (tid == 0) {
         for (int s = 0; s < p.S; s++) {
             mbar_init(full + s, 1);
             mbar_init(empty + s, 1);
+            mbar_init(lfull + s, 1);
+            mbar_init(conv + s, 2 * CG);  // converter warps 2 and 3 of each CTA
         }
         for (int b = 0; b < 2; b++) {
             mbar_init(dfull + b, 1);
@@ -199,9 +213,23 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                     const int s = it % p.S;
                     if (it >= p.S) mbar_wait(empty + s, (unsigned)(((it / p.S) - 1) & 1));
                     unsigned char *st = smem + (size_t)s * STAGE;
+                    const int k0 = kb * BK;
+                    if (!F16 && p.fuse) {  // hi tiles only, signalled on this CTA's own barrier
+                        mbar_expect_tx(lfull + s, STAGE / 2);
+                        const uint32_t lb = su32(lfull + s);
+#pragma unroll
+                        for (int a = 0; a < KA::NA; a++) tma_2d<1>(st + a * BM * 128, &mAhi, k0 + KA_E * a, i0, lb);
+                        unsigned char *sb = st + 2 * A_BYTES;
+                        if constexpr (TB) {
+#pragma unroll
+                            for (int a = 0; a < KA::NA; a++) tma_2d<1>(sb + a * BNH * 128, &mBhi, k0 + KA_E * a, jb, lb);
+                        } else {
+                            for (int g = 0; g < p.bgroups; g++) tma_2d<1>(sb + g * (BK * 128), &mBhi, jb + 32 * g, k0, lb);
+                        }
+                        continue;
+                    }
                     if (rank == 0) mbar_expect_tx(full + s, CG * STAGE);
                     const uint32_t fb = fbar0 + 8u * (uint32_t)s;
-                    const int k0 = kb * BK;
 #pragma unroll
                     for (int a = 0; a < KA::NA; a++) {
                         tma_2d<CG>(st + a * BM * 128, &mAhi, k0 + KA_E * a, i0, fb);
@@ -238,7 +266,8 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                     const long long t0 = p.prof ? clock64() : 0;
                     if (first && gc >= 2 && !((p.dbg & 8) && x > 0)) mbar_wait_cluster(dempty + bd, (unsigned)(((gc - 2) >> 1) & 1));
                     const long long t1 = p.prof ? clock64() : 0;
-                    mbar_wait(full + s, (unsigned)((it / p.S) & 1));
+                    if (!F16 && p.fuse) mbar_wait_acq_cluster(conv + s, (unsigned)((it / p.S) & 1));
+                    else mbar_wait(full + s, (unsigned)((it / p.S) & 1));
                     if (p.prof) {
                         atomicAdd(p.prof + 0, (unsigned long long)(t1 - t0));
                         atomicAdd(p.prof + 1, (unsigned long long)(clock64() - t1));
@@ -275,6 +304,48 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                         gc++;
                     }
                 }
+            }
+        }
+    } else if (!F16 && p.fuse && (warp == 2 || warp == 3)) {  // ------------- lo converters
+        // lo = rna_tf32(x - rz_tf32(x)) of every hi element of the stage, written at the same offset of the
+        // lo slot (same box, same swizzle: an element-wise map), 16 bytes per thread and step
+        const int ct = (warp - 2) * 32 + lane;
+        const uint32_t conv0 = CG == 2 ? mapa(su32(conv), 0) : su32(conv);
+        int it = 0;
+        for (int u = cid; u < p.nunits; u += ncl) {
+            const Unit w = unit_of(p, u);
+            for (int kb = w.kb0; kb < w.kb1; kb++, it++) {
+                const int s = it % p.S;
+                mbar_wait(lfull + s, (unsigned)((it / p.S) & 1));
+                unsigned char *st = smem + (size_t)s * STAGE;
+                const float4 *ah = reinterpret_cast<const float4 *>(st);
+                float4 *al = reinterpret_cast<float4 *>(st + A_BYTES);
+                const float4 *bh = reinterpret_cast<const float4 *>(st + 2 * A_BYTES);
+                float4 *bl = reinterpret_cast<float4 *>(st + 2 * A_BYTES + B_BYTES);
+                constexpr int NA4 = A_BYTES / 16 / 64;
+#pragma unroll
+                for (int v0 = 0; v0 < NA4; v0 += 8) {
+                    float4 x[8];
+#pragma unroll
+                    for (int v = 0; v < 8; v++)
+                        if (v0 + v < NA4) x[v] = ah[ct + 64 * (v0 + v)];
+#pragma unroll
+                    for (int v = 0; v < 8; v++)
+                        if (v0 + v < NA4) al[ct + 64 * (v0 + v)] = lo4(x[v]);
+                }
+                const int nb4 = B_BYTES / 16;
+                for (int v0 = ct; v0 < nb4; v0 += 64 * 8) {
+                    float4 x[8];
+#pragma unroll
+                    for (int v = 0; v < 8; v++)
+                        if (v0 + 64 * v < nb4) x[v] = bh[v0 + 64 * v];
+#pragma unroll
+                    for (int v = 0; v < 8; v++)
+                        if (v0 + 64 * v < nb4) bl[v0 + 64 * v] = lo4(x[v]);
+                }
+                fence_proxy_async_smem();  // generic-proxy writes -> tensor-core (async proxy) reads
+                __syncwarp();
+                if (lane == 0) mbar_arrive_release_cluster(conv0 + 8u * (uint32_t)s);
             }
         }
     } else if (warp >= 4) {  // ---------------------------------------- epilogue warps
@@ -790,7 +861,7 @@ static TcmGeom tcm_geom(const ContractNest &n, const ContractPlan &p, bool f16 =
     g.S = std::min(8, (232448 - 2048) / g.stage);
     if (env_s > 0) g.S = std::min(g.S, env_s);
     if (g.S < 2) return g;
-    g.smem = g.S * g.stage + 1024 /*align*/ + 8 * (2 * g.S + 4) + 16;
+    g.smem = g.S * g.stage + 1024 /*align*/ + 8 * (4 * g.S + 4) + 16;
     g.ok = tcm::encode_fn() != nullptr;
     return g;
 }
@@ -887,7 +958,7 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
             tcm::prep_f16_kernel<<<pr.nbr + pr.nbc + npb, 256, 0, s>>>(pr.r0, pr.r1, pr.cj, pr.colmax, pr.nbr,
                                                                        pr.nbc, a, rows, a.BNT, vecC);
         } else {
-            tcm::prep_kernel<<<pr.nb0 + pr.nb1 + npb, 256, 0, s>>>(pr.j0, pr.j1, pr.nb0, pr.nb1, pr.mode, a, rows,
+            tcm::prep_kernel<<<std::max(1, pr.nb0 + pr.nb1 + npb), 256, 0, s>>>(pr.j0, pr.j1, pr.nb0, pr.nb1, pr.mode, a, rows,
                                                                    a.BNT, vecC);
         }
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
@@ -947,13 +1018,20 @@ tcm::SplitJob split_job(Operand &o, float *ws) {  // the split is run by the fus
 struct Operands {
     Operand oa, ob;
     bool share = false;  // syrk: A is a row block of B (both row-major over k): B's split serves A
+    bool fuse = false;   // both operands TMA-legal as they are: lo formed in shared memory, nothing in HBM
 };
+static bool fuse_enabled() {
+    static const bool f = devsw("EATSS_TCM_FUSE", 1) != 0;  // development: 0 = lo materialised by the prep launch
+    return f;
+}
 static Operands operands(const ContractNest &n, int mode) {
     const float *A = static_cast<const float *>(n.A), *B = static_cast<const float *>(n.B);
     Operands o{Operand{A, n.M, n.K, n.lda}, Operand{B, n.transB ? n.N : n.K, n.transB ? n.K : n.N, n.ldb}};
     size_operand(o.oa, mode);
     size_operand(o.ob, mode);
     o.share = n.transB && n.lda == n.ldb && A >= B && (A - B) % n.ldb == 0 && (A - B) / n.ldb + n.M <= o.ob.rows;
+    o.fuse = fuse_enabled() && o.oa.raw_hi && o.ob.raw_hi;
+    if (o.fuse) o.oa.need = o.ob.need = 0;
     return o;
 }
 
@@ -1003,18 +1081,24 @@ cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p,
     if (!ws || ws_floats < (size_t)(ob.need + (share ? 0 : oa.need) + 64)) return cudaErrorInvalidValue;
     Prep pr;
     pr.mode = mode;
-    pr.j0 = split_job(ob, ws);
     int dev = 0, nsm = 148;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     const int kSplitBlocks = nsm * 8;  // grid-stride split blocks over both operands
-    if (share) {
+    if (ops.fuse) {  // TMA reads the operands themselves; the converter warps form lo on chip
+        oa.hi = oa.lo = oa.x;
+        ob.hi = ob.lo = ob.x;
+        oa.ldp = oa.ld;
+        ob.ldp = ob.ld;
+    } else if (share) {
+        pr.j0 = split_job(ob, ws);
         const int64_t r = (A - B) / n.ldb;
         oa.hi = ob.hi + r * ob.ldp;
         oa.lo = ob.lo + r * ob.ldp;
         oa.ldp = ob.ldp;
         pr.nb0 = kSplitBlocks;
     } else {
+        pr.j0 = split_job(ob, ws);
         pr.j1 = split_job(oa, ws + ob.need);
         pr.nb0 = std::max(1, std::min(kSplitBlocks - 1, (int)((double)kSplitBlocks * ob.need / (ob.need + oa.need))));
         pr.nb1 = kSplitBlocks - pr.nb0;
@@ -1052,6 +1136,7 @@ cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p,
     static const int group_env = devsw("EATSS_TCM_GROUP", 8);  // development: row groups per raster group
     a.group_rows = std::max(1, group_env);
     dev_setup(a, s);
+    a.fuse = ops.fuse ? 1 : 0;
     a.rexp = a.cexp = nullptr;
     cudaError_t r;
     const int bkb = 4 * bk;
@@ -1167,6 +1252,7 @@ cudaError_t launch_tcf_contraction(const ContractNest &n, const ContractPlan &p,
     static const int group_env = devsw("EATSS_TCM_GROUP", 8);
     a.group_rows = std::max(1, group_env);
     dev_setup(a, s);
+    a.fuse = 0;
     a.rexp = aexp;
     a.cexp = bexp;
     const cudaError_t r = g.cg == 2 ? launch_bk<true, 2, true>(bkb, m, a, g.smem, nsm, pr, s, ev)
