@@ -88,7 +88,7 @@ struct Args {
     int dbg;  // -DEATSS_DEVTOOLS builds only (EATSS_TCM_DBG; results then wrong): 1 no TMEM drain,
               // 4 no accumulator reset at chunk starts, 8 no
               // wait for the drained buffer at chunk starts inside a tile (only at tile starts), 16 no lo
-              // conversion (fused 3xTF32)
+              // conversion (fused 3xTF32), 32 spin-wait for the accumulator
 };
 
 __host__ __device__ inline void tile_coords(int t, int PI, int TJ, int G, int &pi, int &tj) {
@@ -366,7 +366,10 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             for (int ch = 0; ch < nch; ch++, gc++) {
                 const int bd = gc & 1;
                 const long long t0 = p.prof ? clock64() : 0;
-                mbar_wait(dfull + bd, (unsigned)((gc >> 1) & 1));
+                // suspended (not spinning) while the chunk accumulates: four epilogue warps share each SM
+                // sub-partition with the producer, the MMA issuer and the lo converters
+                if (p.dbg & 32) mbar_wait(dfull + bd, (unsigned)((gc >> 1) & 1));
+                else mbar_wait_sleep(dfull + bd, (unsigned)((gc >> 1) & 1));
                 const long long t1 = p.prof ? clock64() : 0;
                 fence_after();
                 const uint32_t ta = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(bd * 256 + cq * CW);
