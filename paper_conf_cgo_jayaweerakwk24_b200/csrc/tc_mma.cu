@@ -81,14 +81,10 @@ struct Args {
     int group_rows;  // tile-order grouping (row groups per group) for L2 reuse
     const int *__restrict__ rexp;  // 3xFP16 engine: power-of-two exponent of each row of A (scale 2^rexp)
     const int *__restrict__ cexp;  // ... of each column of B
-    int fuse;  // 3xTF32: lo halves formed in shared memory by the converter warps (2, 3) from the landed hi
-               // tiles (TMA loads hi only); 0: both halves loaded (lo materialised by the prep launch)
-    int SL;    // fuse: lo slots (a ring of its own; the S hi stages are then A hi | B hi only)
     unsigned long long *prof;  // development (EATSS_TCM_PROF): per-site cycle counters, else nullptr
     int dbg;  // -DEATSS_DEVTOOLS builds only (EATSS_TCM_DBG; results then wrong): 1 no TMEM drain,
               // 4 no accumulator reset at chunk starts, 8 no
-              // wait for the drained buffer at chunk starts inside a tile (only at tile starts), 16 no lo
-              // conversion (fused 3xTF32), 32 spin-wait for the accumulator
+              // wait for the drained buffer at chunk starts inside a tile (only at tile starts)
 };
 
 __host__ __device__ inline void tile_coords(int t, int PI, int TJ, int G, int &pi, int &tj) {
@@ -137,14 +133,6 @@ struct KMajor {
 
 // BKB: bytes of k per operand row and stage; F16: 3xFP16 operands (K-major A and B, per-row / per-column
 // power-of-two scales undone in the epilogue), else 3xTF32
-// lo half of four fp32 values for the raw-hi 3xTF32 split (the tensor core reads hi = rz_tf32(x) from x)
-__device__ __forceinline__ float lo1(float x) {
-    uint32_t l;
-    asm("cvt.rna.tf32.f32 %0, %1;\n" : "=r"(l) : "f"(x - __uint_as_float(__float_as_uint(x) & 0xFFFFE000u)));
-    return __uint_as_float(l);
-}
-__device__ __forceinline__ float4 lo4(float4 x) { return make_float4(lo1(x.x), lo1(x.y), lo1(x.z), lo1(x.w)); }
-
 template <int BKB, bool TB, int CG, bool F16>
 __global__ void __launch_bounds__(NTHREADS, 1)
     tc_mma_kernel(const __grid_constant__ CUtensorMap mAhi, const __grid_constant__ CUtensorMap mAlo,
@@ -162,26 +150,17 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     constexpr int A_BYTES = BM * BKB;  // one A half (hi or lo) per stage
     const int BNH = p.BNH, B_BYTES = p.b_bytes, STAGE = p.stage;
     const int R = p.R;
-    const bool FU = !F16 && p.fuse;
-    const int HALF = A_BYTES + B_BYTES;  // fuse: one hi slot (A hi | B hi) or lo slot (A lo | B lo)
-    unsigned char *lo_ring = smem + (size_t)p.S * HALF;
-    uint64_t *full = reinterpret_cast<uint64_t *>(smem + (FU ? (size_t)(p.S + p.SL) * HALF : (size_t)p.S * STAGE));
+    uint64_t *full = reinterpret_cast<uint64_t *>(smem + (size_t)p.S * STAGE);
     uint64_t *empty = full + p.S;
     uint64_t *dfull = empty + p.S;
     uint64_t *dempty = dfull + 2;
-    uint64_t *lfull = dempty + 2;  // fuse: this CTA's hi tiles of the stage landed (local TMA bytes)
-    uint64_t *conv = lfull + p.S;  // fuse (leader): both CTAs' lo halves of the stage written
-    uint64_t *lofree = conv + p.S;  // fuse: the MMAs reading a lo slot finished (tcgen05.commit)
-    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(lofree + p.SL);
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(dempty + 2);
 
     if (tid == 0) {
         for (int s = 0; s < p.S; s++) {
             mbar_init(full + s, 1);
             mbar_init(empty + s, 1);
-            mbar_init(lfull + s, 1);
-            mbar_init(conv + s, 2 * CG);  // converter warps 2 and 3 of each CTA
         }
-        for (int s = 0; s < p.SL; s++) mbar_init(lofree + s, 1);
         for (int b = 0; b < 2; b++) {
             mbar_init(dfull + b, 1);
             mbar_init(dempty + b, NEPI * CG);
@@ -219,25 +198,10 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                 for (int kb = w.kb0; kb < w.kb1; kb++, it++) {
                     const int s = it % p.S;
                     if (it >= p.S) mbar_wait(empty + s, (unsigned)(((it / p.S) - 1) & 1));
-                    const int k0 = kb * BK;
-                    if (FU) {  // hi tiles only (slot: A hi | B hi), signalled on this CTA's own barrier
-                        unsigned char *st = smem + (size_t)s * HALF;
-                        mbar_expect_tx(lfull + s, HALF);
-                        const uint32_t lb = su32(lfull + s);
-#pragma unroll
-                        for (int a = 0; a < KA::NA; a++) tma_2d<1>(st + a * BM * 128, &mAhi, k0 + KA_E * a, i0, lb);
-                        unsigned char *sb = st + A_BYTES;
-                        if constexpr (TB) {
-#pragma unroll
-                            for (int a = 0; a < KA::NA; a++) tma_2d<1>(sb + a * BNH * 128, &mBhi, k0 + KA_E * a, jb, lb);
-                        } else {
-                            for (int g = 0; g < p.bgroups; g++) tma_2d<1>(sb + g * (BK * 128), &mBhi, jb + 32 * g, k0, lb);
-                        }
-                        continue;
-                    }
                     unsigned char *st = smem + (size_t)s * STAGE;
                     if (rank == 0) mbar_expect_tx(full + s, CG * STAGE);
                     const uint32_t fb = fbar0 + 8u * (uint32_t)s;
+                    const int k0 = kb * BK;
 #pragma unroll
                     for (int a = 0; a < KA::NA; a++) {
                         tma_2d<CG>(st + a * BM * 128, &mAhi, k0 + KA_E * a, i0, fb);
@@ -274,31 +238,26 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                     const long long t0 = p.prof ? clock64() : 0;
                     if (first && gc >= 2 && !((p.dbg & 8) && x > 0)) mbar_wait_cluster(dempty + bd, (unsigned)(((gc - 2) >> 1) & 1));
                     const long long t1 = p.prof ? clock64() : 0;
-                    if (FU) mbar_wait_acq_cluster(conv + s, (unsigned)((it / p.S) & 1));
-                    else mbar_wait(full + s, (unsigned)((it / p.S) & 1));
+                    mbar_wait(full + s, (unsigned)((it / p.S) & 1));
                     if (p.prof) {
                         atomicAdd(p.prof + 0, (unsigned long long)(t1 - t0));
                         atomicAdd(p.prof + 1, (unsigned long long)(clock64() - t1));
                     }
                     fence_after();
-                    // operand halves: [A hi | A lo | B hi | B lo] per stage, or (fuse) hi slot [A hi | B hi] and
-                    // lo slot [A lo | B lo]
-                    const unsigned char *st = smem + (size_t)s * (FU ? HALF : STAGE);
-                    const unsigned char *lo = FU ? lo_ring + (size_t)(it % p.SL) * HALF : st + A_BYTES;
-                    const unsigned char *pbh = FU ? st + A_BYTES : st + 2 * A_BYTES;
-                    const unsigned char *pbl = FU ? lo + A_BYTES : pbh + B_BYTES;
+                    const unsigned char *st = smem + (size_t)s * STAGE;
+                    const unsigned char *sb = st + 2 * A_BYTES;
                     const uint32_t d = tmem + (uint32_t)(bd * 256);
 #pragma unroll
                     for (int ks = 0; ks < BKB / 32; ks++) {
                         const uint64_t ahi = KA::desc(st, BM, ks);
-                        const uint64_t alo = KA::desc(lo, BM, ks);
+                        const uint64_t alo = KA::desc(st + A_BYTES, BM, ks);
                         uint64_t bhi, blo;
                         if constexpr (TB) {
-                            bhi = KA::desc(pbh, BNH, ks);
-                            blo = KA::desc(pbl, BNH, ks);
+                            bhi = KA::desc(sb, BNH, ks);
+                            blo = KA::desc(sb + B_BYTES, BNH, ks);
                         } else {
-                            bhi = desc_sw128(pbh + ks * 1024, (uint32_t)(BK * 128), 512u, 1);
-                            blo = desc_sw128(pbl + ks * 1024, (uint32_t)(BK * 128), 512u, 1);
+                            bhi = desc_sw128(sb + ks * 1024, (uint32_t)(BK * 128), 512u, 1);
+                            blo = desc_sw128(sb + B_BYTES + ks * 1024, (uint32_t)(BK * 128), 512u, 1);
                         }
                         if constexpr (F16) {
                             mma_ss_f16<CG>(d, ahi, bhi, ID, (first && ks == 0) ? 0u : 1u);
@@ -311,43 +270,10 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                         }
                     }
                     mma_commit<CG>(empty + s);
-                    if (FU) mma_commit<CG>(lofree + it % p.SL);
                     if ((x % R) == R - 1 || x == nk - 1) {
                         mma_commit<CG>(dfull + bd);
                         gc++;
                     }
-                }
-            }
-        }
-    } else if (FU && (warp == 2 || warp == 3)) {  // ------------------------------- lo converters
-        // lo = rna_tf32(x - rz_tf32(x)) of every hi element of the stage, written at the same offset of a lo
-        // slot (same boxes, same swizzle: an element-wise map), 16 bytes per thread and step
-        const int ct = (warp - 2) * 32 + lane;
-        const uint32_t conv0 = CG == 2 ? mapa(su32(conv), 0) : su32(conv);
-        const int n4 = (p.dbg & 16) ? 0 : HALF / 16;
-        int it = 0;
-        for (int u = cid; u < p.nunits; u += ncl) {
-            const Unit w = unit_of(p, u);
-            for (int kb = w.kb0; kb < w.kb1; kb++, it++) {
-                const int s = it % p.S, sl = it % p.SL;
-                mbar_wait(lfull + s, (unsigned)((it / p.S) & 1));
-                if (it >= p.SL) mbar_wait(lofree + sl, (unsigned)(((it / p.SL) - 1) & 1));
-                const float4 *src = reinterpret_cast<const float4 *>(smem + (size_t)s * HALF);
-                float4 *dst = reinterpret_cast<float4 *>(lo_ring + (size_t)sl * HALF);
-                for (int v0 = ct; v0 < n4; v0 += 64 * 8) {
-                    float4 x[8];
-#pragma unroll
-                    for (int v = 0; v < 8; v++)
-                        if (v0 + 64 * v < n4) x[v] = src[v0 + 64 * v];
-#pragma unroll
-                    for (int v = 0; v < 8; v++)
-                        if (v0 + 64 * v < n4) dst[v0 + 64 * v] = lo4(x[v]);
-                }
-                fence_proxy_async_smem();  // generic-proxy writes -> tensor-core (async proxy) reads
-                __syncwarp();
-                if (lane == 0) {  // the leader's own converters: CTA-scope release; the peer's: cluster scope
-                    if (CG == 2 && rank != 0) mbar_arrive_release_cluster(conv0 + 8u * (uint32_t)s);
-                    else mbar_arrive(conv + s);
                 }
             }
         }
@@ -366,10 +292,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             for (int ch = 0; ch < nch; ch++, gc++) {
                 const int bd = gc & 1;
                 const long long t0 = p.prof ? clock64() : 0;
-                // suspended (not spinning) while the chunk accumulates: four epilogue warps share each SM
-                // sub-partition with the producer, the MMA issuer and the lo converters
-                if (p.dbg & 32) mbar_wait(dfull + bd, (unsigned)((gc >> 1) & 1));
-                else mbar_wait_sleep(dfull + bd, (unsigned)((gc >> 1) & 1));
+                mbar_wait(dfull + bd, (unsigned)((gc >> 1) & 1));
                 const long long t1 = p.prof ? clock64() : 0;
                 fence_after();
                 const uint32_t ta = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(bd * 256 + cq * CW);
@@ -843,7 +766,6 @@ struct Prep {
 struct TcmGeom {
     bool ok = false;
     int bk = 0, bn = 0, cg = 1, bnh = 0, bgroups = 0, a_bytes = 0, b_bytes = 0, stage = 0, S = 0, smem = 0;
-    int fS = 0, fSL = 0, fsmem = 0;  // 3xTF32 with on-chip lo: hi stages, lo slots, shared memory
 };
 // f16: the 3xFP16 engine (operands 2 bytes, B always K-major after its transposing split)
 static TcmGeom tcm_geom(const ContractNest &n, const ContractPlan &p, bool f16 = false) {
@@ -868,14 +790,7 @@ static TcmGeom tcm_geom(const ContractNest &n, const ContractPlan &p, bool f16 =
     g.S = std::min(8, (232448 - 2048) / g.stage);
     if (env_s > 0) g.S = std::min(g.S, env_s);
     if (g.S < 2) return g;
-    g.smem = g.S * g.stage + 1024 /*align*/ + 8 * (4 * g.S + 4) + 16;
-    if (!f16) {
-        const int half = g.a_bytes + g.b_bytes;
-        g.fSL = 2;
-        g.fS = std::min(8, (232448 - 2048 - g.fSL * half) / half);
-        if (env_s > 0) g.fS = std::min(g.fS, env_s);
-        g.fsmem = (g.fS + g.fSL) * half + 1024 + 8 * (4 * g.fS + 4 + g.fSL) + 16;
-    }
+    g.smem = g.S * g.stage + 1024 /*align*/ + 8 * (2 * g.S + 4) + 16;
     g.ok = tcm::encode_fn() != nullptr;
     return g;
 }
@@ -972,7 +887,7 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
             tcm::prep_f16_kernel<<<pr.nbr + pr.nbc + npb, 256, 0, s>>>(pr.r0, pr.r1, pr.cj, pr.colmax, pr.nbr,
                                                                        pr.nbc, a, rows, a.BNT, vecC);
         } else {
-            tcm::prep_kernel<<<std::max(1, pr.nb0 + pr.nb1 + npb), 256, 0, s>>>(pr.j0, pr.j1, pr.nb0, pr.nb1, pr.mode, a, rows,
+            tcm::prep_kernel<<<pr.nb0 + pr.nb1 + npb, 256, 0, s>>>(pr.j0, pr.j1, pr.nb0, pr.nb1, pr.mode, a, rows,
                                                                    a.BNT, vecC);
         }
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
@@ -1032,25 +947,18 @@ tcm::SplitJob split_job(Operand &o, float *ws) {  // the split is run by the fus
 struct Operands {
     Operand oa, ob;
     bool share = false;  // syrk: A is a row block of B (both row-major over k): B's split serves A
-    bool fuse = false;   // both operands TMA-legal as they are: lo formed in shared memory, nothing in HBM
 };
-static bool fuse_enabled() {
-    static const bool f = devsw("EATSS_TCM_FUSE", 1) != 0;  // development: 0 = lo materialised by the prep launch
-    return f;
-}
-static Operands operands(const ContractNest &n, int mode, const TcmGeom &g) {
+static Operands operands(const ContractNest &n, int mode) {
     const float *A = static_cast<const float *>(n.A), *B = static_cast<const float *>(n.B);
     Operands o{Operand{A, n.M, n.K, n.lda}, Operand{B, n.transB ? n.N : n.K, n.transB ? n.K : n.N, n.ldb}};
     size_operand(o.oa, mode);
     size_operand(o.ob, mode);
     o.share = n.transB && n.lda == n.ldb && A >= B && (A - B) % n.ldb == 0 && (A - B) / n.ldb + n.M <= o.ob.rows;
-    o.fuse = fuse_enabled() && o.oa.raw_hi && o.ob.raw_hi && g.fS >= 2;
-    if (o.fuse) o.oa.need = o.ob.need = 0;
     return o;
 }
 
-size_t tcm_ws_floats(const ContractNest &n, const ContractPlan &p) {
-    const Operands o = operands(n, split_mode(), tcm_geom(n, p));
+size_t tcm_ws_floats(const ContractNest &n, const ContractPlan &) {
+    const Operands o = operands(n, split_mode());
     return (size_t)(o.ob.need + (o.share ? 0 : o.oa.need) + 64);
 }
 
@@ -1089,30 +997,24 @@ cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p,
     if (!g.ok) return cudaErrorNotSupported;
     const int bn = g.bn, cg = g.cg, bk = g.bk, mode = split_mode();
     const float *A = static_cast<const float *>(n.A), *B = static_cast<const float *>(n.B);
-    Operands ops = operands(n, mode, g);
+    Operands ops = operands(n, mode);
     Operand &oa = ops.oa, &ob = ops.ob;
     const bool share = ops.share;
     if (!ws || ws_floats < (size_t)(ob.need + (share ? 0 : oa.need) + 64)) return cudaErrorInvalidValue;
     Prep pr;
     pr.mode = mode;
+    pr.j0 = split_job(ob, ws);
     int dev = 0, nsm = 148;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     const int kSplitBlocks = nsm * 8;  // grid-stride split blocks over both operands
-    if (ops.fuse) {  // TMA reads the operands themselves; the converter warps form lo on chip
-        oa.hi = oa.lo = oa.x;
-        ob.hi = ob.lo = ob.x;
-        oa.ldp = oa.ld;
-        ob.ldp = ob.ld;
-    } else if (share) {
-        pr.j0 = split_job(ob, ws);
+    if (share) {
         const int64_t r = (A - B) / n.ldb;
         oa.hi = ob.hi + r * ob.ldp;
         oa.lo = ob.lo + r * ob.ldp;
         oa.ldp = ob.ldp;
         pr.nb0 = kSplitBlocks;
     } else {
-        pr.j0 = split_job(ob, ws);
         pr.j1 = split_job(oa, ws + ob.need);
         pr.nb0 = std::max(1, std::min(kSplitBlocks - 1, (int)((double)kSplitBlocks * ob.need / (ob.need + oa.need))));
         pr.nb1 = kSplitBlocks - pr.nb0;
@@ -1139,10 +1041,7 @@ cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p,
     a.M = n.M; a.N = n.N; a.K = n.K;
     a.C = static_cast<float *>(n.C); a.ldc = n.ldc;
     a.alpha = (float)n.alpha; a.beta = (float)n.beta; a.init_zero = n.init_zero ? 1 : 0;
-    a.fuse = ops.fuse ? 1 : 0;
-    a.S = a.fuse ? g.fS : g.S;
-    a.SL = a.fuse ? g.fSL : 0;
-    const int smem = a.fuse ? g.fsmem : g.smem;
+    a.S = g.S;
     static const int chunk_env = devsw("EATSS_TCM_CHUNK_K", 0);  // development: k per accumulator chunk
     a.R = std::max(1, (chunk_env > 0 ? chunk_env : tcm::CHUNK_K) / bk);
     a.BNT = bn; a.BNH = g.bnh; a.bgroups = g.bgroups; a.b_bytes = g.b_bytes; a.stage = g.stage;
@@ -1157,11 +1056,11 @@ cudaError_t launch_tcm_contraction(const ContractNest &n, const ContractPlan &p,
     cudaError_t r;
     const int bkb = 4 * bk;
     if (n.transB)
-        r = cg == 2 ? launch_bk<true, 2, false>(bkb, m, a, smem, nsm, pr, s, ev)
-                    : launch_bk<true, 1, false>(bkb, m, a, smem, nsm, pr, s, ev);
+        r = cg == 2 ? launch_bk<true, 2, false>(bkb, m, a, g.smem, nsm, pr, s, ev)
+                    : launch_bk<true, 1, false>(bkb, m, a, g.smem, nsm, pr, s, ev);
     else
-        r = cg == 2 ? launch_bk<false, 2, false>(bkb, m, a, smem, nsm, pr, s, ev)
-                    : launch_bk<false, 1, false>(bkb, m, a, smem, nsm, pr, s, ev);
+        r = cg == 2 ? launch_bk<false, 2, false>(bkb, m, a, g.smem, nsm, pr, s, ev)
+                    : launch_bk<false, 1, false>(bkb, m, a, g.smem, nsm, pr, s, ev);
     dev_report(a, s);
     return r;
 }
@@ -1268,8 +1167,6 @@ cudaError_t launch_tcf_contraction(const ContractNest &n, const ContractPlan &p,
     static const int group_env = devsw("EATSS_TCM_GROUP", 8);
     a.group_rows = std::max(1, group_env);
     dev_setup(a, s);
-    a.fuse = 0;
-    a.SL = 0;
     a.rexp = aexp;
     a.cexp = bexp;
     const cudaError_t r = g.cg == 2 ? launch_bk<true, 2, true>(bkb, m, a, g.smem, nsm, pr, s, ev)

@@ -43,19 +43,6 @@ __device__ __forceinline__ void mbar_arrive(uint64_t *b) {
 __device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_addr) {
     asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];\n" ::"r"(cluster_addr) : "memory");
 }
-// Arrive with cluster-scope release: publishes this warp's prior shared-memory writes (made visible to the
-// async proxy by fence.proxy.async first) to a waiter of another CTA of the cluster (mbar_wait_acq_cluster).
-__device__ __forceinline__ void mbar_arrive_release_cluster(uint32_t cluster_addr) {
-    asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];\n" ::"r"(cluster_addr) : "memory");
-}
-__device__ __forceinline__ void mbar_wait_acq_cluster(uint64_t *b, unsigned parity) {
-    asm volatile(
-        "{\n.reg .pred p;\nW_%=:\n"
-        "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%0], %1;\n"
-        "@!p bra W_%=;\n}\n" ::"r"(su32(b)),
-        "r"(parity)
-        : "memory");
-}
 __device__ __forceinline__ void mbar_wait(uint64_t *b, unsigned parity) {
     asm volatile(
         "{\n.reg .pred p;\nW_%=:\n"
