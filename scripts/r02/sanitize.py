@@ -29,6 +29,8 @@ def go(kind, dims, tiles, engine, tsteps=0):
 
 go("gemm", (300, 520, 200), (256, 256, 32), 2)      # tc_mma, CTA pair, split tail, ragged
 go("gemm", (260, 300, 136), (128, 48, 16), 2)       # tc_mma single CTA, SW64
+go("gemm", (300, 520, 200), (256, 256, 64), 4)      # tc_mma 3xFP16 (maxima + split launches), CTA pair
+go("syrk", (300, 200), (128, 64, 32), 4)            # tc_mma 3xFP16, shared K-major split
 go("syrk", (300, 200), (256, 96, 64), 2)            # tc_mma K-major B
 go("gemm", (100, 300, 64), (16, 256, 32), 2)        # tc_gemm (narrow-tile TS engine)
 go("gemm", (300, 520, 200), (16, 1024, 16), 1)      # SIMT staged (bulk copies)
