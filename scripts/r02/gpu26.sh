@@ -18,5 +18,5 @@ cap max_f16_r02 "f16_max_kernel" gemm 4000,4000,4000 256,256,64 --engine 4 --ite
 cap tcm_tf32_r02 "tc_mma_kernel" gemm 4000,4000,4000 256,256,32 --engine 2 --iters 2
 cap prep_tf32_r02 "prep_kernel" gemm 4000,4000,4000 256,256,32 --engine 2 --iters 2
 cap simt_gemm_r02 "contract_staged" gemm 4000,4000,4000 16,1024,16 --engine 1 --iters 2
-cap ccsdtc_r02 "ccsd_tc_kernel" ccsd_t_d1 48,48,48,48,48,48,48 1,2,1,48,2,48,48 --engine 2 --iters 1
+cap ccsdtc_r02 "ccsd_tc_kernel" ccsd_t_d1 8,48,48,48,48,48,48 1,2,1,48,2,48,48 --engine 2 --iters 1
 ls $O
