@@ -582,12 +582,12 @@ __device__ void f16_rows_body(const F16Rows &j, int64_t w0, int64_t wstride) {
         }
     }
 }
-// row maxima of up to two row operands: CTA (32 rows, 1024-column chunk), a warp per row and chunk, 16-byte
+// row maxima of up to two row operands: CTA (4 rows per warp, 1024-column chunk), a warp per row and chunk, 16-byte
 // loads (eight per lane in flight); partial maxima meet via atomicMax on the bit pattern
 __device__ void f16_rowmax_block(const F16Rows &j, unsigned *maxbits, int64_t blk) {
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
     const int64_t nch = (j.cols + 1023) / 1024;
-    const int64_t r0 = (blk / nch) * 32, c0 = (blk % nch) * 1024;
+    const int64_t r0 = (blk / nch) * (4 * nw), c0 = (blk % nch) * 1024;
     const bool v4 = ((j.ldx & 3) == 0) && ((reinterpret_cast<uintptr_t>(j.x) & 15) == 0);
     for (int q = 0; q < 4; q++) {
         const int64_t r = r0 + 4 * w + q;
@@ -614,23 +614,23 @@ __device__ void f16_rowmax_block(const F16Rows &j, unsigned *maxbits, int64_t bl
         if (lane == 0) atomicMax(maxbits + r, __float_as_uint(m));
     }
 }
-// column maxima of a row-major B (K x N): CTA (128-column strip, 256-row chunk), 256 threads -- a thread
+// column maxima of a row-major B (K x N): CTA (128-column strip, 256-row chunk), <= 8 warps -- a thread
 // owns four adjacent columns (16-byte loads when aligned), the warps split the chunk, eight loads in
 // flight per thread; partial maxima meet in colmax via atomicMax on the bit pattern (non-negative floats
 // order like their bits)
 __device__ void f16_colmax_block(const float *__restrict__ x, int64_t K, int64_t N, int64_t ldx,
                                  unsigned *__restrict__ colmax, int64_t bx, int64_t by) {
     __shared__ float4 red[8][32];
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
     const int64_t c0 = bx * 128 + 4 * lane, k0 = by * 256;
     const bool v4 = ((ldx & 3) == 0) && ((reinterpret_cast<uintptr_t>(x) & 15) == 0) && c0 + 3 < N;
     float4 m = make_float4(0.f, 0.f, 0.f, 0.f);
     if (c0 < N) {
-        for (int i0 = w; i0 < 256; i0 += 64) {  // eight rows per pass, all loads issued before their use
+        for (int i0 = w; i0 < 256; i0 += 8 * nw) {  // eight rows per pass, all loads issued before their use
             float4 v[8];
 #pragma unroll
             for (int u = 0; u < 8; u++) {
-                const int64_t k = k0 + i0 + 8 * u;
+                const int64_t k = k0 + i0 + nw * u;
                 const float *row = x + k * ldx + c0;
                 if (k >= K) {
                     v[u] = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -653,7 +653,7 @@ __device__ void f16_colmax_block(const float *__restrict__ x, int64_t K, int64_t
     red[w][lane] = m;
     __syncthreads();
     if (w == 0 && c0 < N) {
-        for (int q = 1; q < 8; q++) {
+        for (int q = 1; q < nw; q++) {
             const float4 o = red[q][lane];
             m.x = fmaxf(m.x, o.x); m.y = fmaxf(m.y, o.y); m.z = fmaxf(m.z, o.z); m.w = fmaxf(m.w, o.w);
         }
@@ -661,11 +661,79 @@ __device__ void f16_colmax_block(const float *__restrict__ x, int64_t K, int64_t
         for (int q = 0; q < 4 && c0 + q < N; q++) atomicMax(colmax + c0 + q, __float_as_uint(mm[q]));
     }
 }
-// The maxima pass before the 3xFP16 split (one launch): blocks [0, nr0) row maxima of r0, [nr0, nr0 + nr1)
-// of r1, the rest the column maxima of a row-major B (cj; colmax) -- every block independent
-__global__ void __launch_bounds__(256) f16_max_kernel(const F16Rows r0, unsigned *m0, const F16Rows r1, unsigned *m1,
-                                                      const F16Cols cj, unsigned *colmax, int nr0, int nr1) {
+// Row operand read ONCE: each warp brings a whole row into its shared buffer with one bulk copy (no thread
+// holds the loads: a 16 KB row per warp in flight), takes the maximum from shared memory, then writes the
+// scaled split from it -- max and split fused, so the row operand costs one HBM read instead of two.
+// Needs 16-byte aligned rows of a multiple of 4 columns (the host checks); `buf` = this warp's row buffer.
+__device__ void f16_rows_staged(const F16Rows &j, float *buf, uint64_t *bar, int64_t w0, int64_t wstride) {
+    const int lane = threadIdx.x & 31;
+    const int c4n = (int)(j.cols >> 2), p4n = (int)(j.ldp >> 2);
+    const float4 *b4 = reinterpret_cast<const float4 *>(buf);
+    unsigned phase = 0;
+    for (int64_t r = w0; r < j.rows; r += wstride) {
+        if (lane == 0) {
+            fence_proxy_async_smem();  // the previous row's generic reads before the async-proxy overwrite
+            mbar_expect_tx(bar, (unsigned)(j.cols * 4));
+            bulk_g2s(buf, j.x + r * j.ldx, (unsigned)(j.cols * 4), bar);
+        }
+        mbar_wait(bar, phase);
+        phase ^= 1u;
+        float m = 0.f;
+        for (int c = lane; c < c4n; c += 32) {
+            const float4 v = b4[c];
+            m = fmaxf(m, fmaxf(fmaxf(fabsf(v.x), fabsf(v.y)), fmaxf(fabsf(v.z), fabsf(v.w))));
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+        const int s = f16_scale_exp(m);
+        if (lane == 0) j.exps[r] = s;
+        const float sc = __int_as_float((127 + s) << 23);
+        __half *hr = j.hi + r * j.ldp, *lr = j.lo + r * j.ldp;
+        for (int c = lane; c < p4n; c += 32) {  // 4 columns per lane and step: 8-byte fp16 stores
+            const float4 v = c < c4n ? b4[c] : make_float4(0.f, 0.f, 0.f, 0.f);
+            __half h[4], l[4];
+            f16_split(v.x, sc, h[0], l[0]);
+            f16_split(v.y, sc, h[1], l[1]);
+            f16_split(v.z, sc, h[2], l[2]);
+            f16_split(v.w, sc, h[3], l[3]);
+            *reinterpret_cast<uint2 *>(hr + 4 * c) =
+                make_uint2(*reinterpret_cast<uint32_t *>(&h[0]), *reinterpret_cast<uint32_t *>(&h[2]));
+            *reinterpret_cast<uint2 *>(lr + 4 * c) =
+                make_uint2(*reinterpret_cast<uint32_t *>(&l[0]), *reinterpret_cast<uint32_t *>(&l[2]));
+        }
+        __syncwarp();
+    }
+}
+// The first launch of the 3xFP16 engine (F16_PASS1_THREADS per block, every block independent):
+//   fused = 1: blocks [0, nr0) split the row operands r0 then r1 read once (f16_rows_staged; dynamic shared
+//              memory = one row buffer per warp);
+//   fused = 0: blocks [0, nr0) row maxima of r0, [nr0, nr0 + nr1) of r1 (the split follows in prep_f16_kernel);
+// the rest: the column maxima of a row-major B (cj; colmax).
+constexpr int F16_PASS1_THREADS = 128;
+__global__ void __launch_bounds__(F16_PASS1_THREADS) f16_max_kernel(const F16Rows r0, unsigned *m0, const F16Rows r1,
+                                                                   unsigned *m1, const F16Cols cj, unsigned *colmax,
+                                                                   int nr0, int nr1, int fused, int rowbuf_floats) {
     const int64_t b = blockIdx.x;
+    if (fused && b < nr0) {
+        extern __shared__ __align__(16) float f16_rowbuf[];
+        __shared__ __align__(8) uint64_t bars[F16_PASS1_THREADS / 32];
+        const int w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+        if ((threadIdx.x & 31) == 0) {
+            mbar_init(bars + w, 1);
+            asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+        }
+        __syncwarp();
+        const int64_t w0 = b * nw + w, ws = (int64_t)nr0 * nw;
+        float *buf = f16_rowbuf + (size_t)w * rowbuf_floats;
+        if (r0.x) f16_rows_staged(r0, buf, bars + w, w0, ws);
+        if (r1.x) f16_rows_staged(r1, buf, bars + w, w0, ws);
+        return;
+    }
+    if (fused) {
+        const int64_t c = b - nr0, nsx = (cj.N + 127) / 128;
+        f16_colmax_block(cj.x, cj.K, cj.N, cj.ldx, colmax, c % nsx, c / nsx);
+        return;
+    }
     if (b < nr0) {
         f16_rowmax_block(r0, m0, b);
         return;
@@ -759,6 +827,7 @@ struct Prep {
     unsigned *maxes = nullptr;   // the zero-initialised region holding every max array of this GEMM
     size_t maxes_bytes = 0;
     unsigned *m0 = nullptr, *m1 = nullptr;  // row maxima of r0 / r1
+    bool fused_rows = false;  // row operands split in the first launch, each row read once (f16_rows_staged)
     int nbr = 0, nbc = 0;
 };
 
@@ -873,19 +942,42 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
         const int npb = (int)std::min<int64_t>((tail4 + 255) / 256, (int64_t)nsm * 4);
         const int vecC = (a.ldc % 4 == 0 && (reinterpret_cast<uintptr_t>(a.C) & 15) == 0) ? 1 : 0;
         if constexpr (F16) {
-            {  // maxima of every row of the row operands and column of a row-major B (the split needs them)
+            {  // first launch: the row operands (fused: split, each row read once; else their maxima) and the
+               // column maxima of a row-major B
                 if ((e = cudaMemsetAsync(pr.maxes, 0, pr.maxes_bytes, s)) != cudaSuccess) return e;
-                auto nrb = [](const tcm::F16Rows &r) {
-                    return r.x ? (int)(((r.rows + 31) / 32) * ((r.cols + 1023) / 1024)) : 0;
-                };
-                const int nr0 = nrb(pr.r0), nr1 = nrb(pr.r1);
+                constexpr int TPB = tcm::F16_PASS1_THREADS, NW = TPB / 32;
                 const int ncb = pr.colmax ? (int)(((pr.cj.N + 127) / 128) * ((pr.cj.K + 255) / 256)) : 0;
-                tcm::f16_max_kernel<<<nr0 + nr1 + ncb, 256, 0, s>>>(pr.r0, pr.m0, pr.r1, pr.m1, pr.cj, pr.colmax, nr0,
-                                                                    nr1);
+                int nr0 = 0, nr1 = 0, rowbuf = 0;
+                size_t dsm = 0;
+                if (pr.fused_rows) {
+                    const tcm::F16Rows &rr = pr.r0.x ? pr.r0 : pr.r1;
+                    rowbuf = (int)((rr.cols + 3) / 4 * 4);
+                    dsm = (size_t)NW * rowbuf * sizeof(float);
+                    const int64_t nrows = std::max(pr.r0.x ? pr.r0.rows : 0, pr.r1.x ? pr.r1.rows : 0);
+                    nr0 = (int)std::min<int64_t>((nrows + NW - 1) / NW, (int64_t)nsm * 3);
+                    auto kf = tcm::f16_max_kernel;
+                    std::lock_guard<std::mutex> lk(g_ks_mu);
+                    KernelState &ks = g_ks[{reinterpret_cast<const void *>(kf), dev}];
+                    if (ks.smem < (int)dsm) {
+                        if ((e = cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsm)) !=
+                            cudaSuccess)
+                            return e;
+                        ks.smem = (int)dsm;
+                    }
+                } else {
+                    auto nrb = [](const tcm::F16Rows &r) {
+                        return r.x ? (int)(((r.rows + 4 * NW - 1) / (4 * NW)) * ((r.cols + 1023) / 1024)) : 0;
+                    };
+                    nr0 = nrb(pr.r0);
+                    nr1 = nrb(pr.r1);
+                }
+                tcm::f16_max_kernel<<<nr0 + nr1 + ncb, TPB, dsm, s>>>(pr.r0, pr.m0, pr.r1, pr.m1, pr.cj, pr.colmax,
+                                                                      nr0, nr1, pr.fused_rows ? 1 : 0, rowbuf);
                 if ((e = cudaGetLastError()) != cudaSuccess) return e;
             }
-            tcm::prep_f16_kernel<<<pr.nbr + pr.nbc + npb, 256, 0, s>>>(pr.r0, pr.r1, pr.cj, pr.colmax, pr.nbr,
-                                                                       pr.nbc, a, rows, a.BNT, vecC);
+            const int nbr = pr.fused_rows ? 0 : pr.nbr;  // fused: the rows are already split
+            tcm::prep_f16_kernel<<<std::max(1, nbr + pr.nbc + npb), 256, 0, s>>>(pr.r0, pr.r1, pr.cj, pr.colmax, nbr,
+                                                                               pr.nbc, a, rows, a.BNT, vecC);
         } else {
             tcm::prep_kernel<<<pr.nb0 + pr.nb1 + npb, 256, 0, s>>>(pr.j0, pr.j1, pr.nb0, pr.nb1, pr.mode, a, rows,
                                                                    a.BNT, vecC);
@@ -1140,6 +1232,14 @@ cudaError_t launch_tcf_contraction(const ContractNest &n, const ContractPlan &p,
         aexp = e;
     }
     pr.nbr = nsm * 4;
+    {  // the row operands can be read once (bulk-copied rows) when 16-byte aligned, whole float4s, <= 48 KB
+        auto ok = [](const tcm::F16Rows &r) {
+            return !r.x || ((r.ldx & 3) == 0 && (reinterpret_cast<uintptr_t>(r.x) & 15) == 0 && (r.cols & 3) == 0 &&
+                            r.cols * 4 <= 48 * 1024);
+        };
+        static const bool staged_rows = devsw("EATSS_TCF_STAGED_ROWS", 1) != 0;  // development: 0 = two reads
+        pr.fused_rows = staged_rows && ok(pr.r0) && ok(pr.r1) && (pr.r0.x || pr.r1.x);
+    }
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
     CUtensorMap m[4];
