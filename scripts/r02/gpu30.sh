@@ -23,3 +23,10 @@ run EATSS_TCM_DBG=16
 T="scripts/time_kernel.py gemm 4000,4000,4000 256,128,64 --engine 4 --iters 50 --kernel-ms"
 run EATSS_TCM_DBG=0
 run EATSS_TCM_DBG=16
+# heat-3d resident time loop: parity, then timing vs one launch per sweep (EATSS_HEAT_RESIDENT=0)
+timeout 600 python -m pytest tests/test_gpu_heat_resident.py tests/test_gpu_parity.py -k "heat" -q -x -p no:cacheprovider 2>&1 | tail -3
+for rep in 1 2; do
+for r in 1 0; do
+  echo "== heat resident=$r"; EATSS_HEAT_RESIDENT=$r timeout 120 python scripts/time_kernel.py heat-3d 120 16,16,32 --tsteps 500 --iters 5 2>&1 | tail -1
+  EATSS_HEAT_RESIDENT=$r timeout 120 python scripts/time_kernel.py heat-3d 512 16,16,32 --tsteps 5 --iters 5 2>&1 | tail -1
+done; done
