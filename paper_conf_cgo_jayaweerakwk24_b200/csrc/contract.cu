@@ -49,6 +49,7 @@ struct CArgs {
     int sp;          // staged: 1 = 2-D grid, no split
     int passes_i, passes_j;
     int waf;          // lanes of each warp along j (0: linear layout, tx fastest)
+    int bulk_spread;  // staged bulk path: the per-row B copies are issued by lane 0 of every warp (else thread 0)
     int32_t *counts;  // coverage mode
 };
 
@@ -791,6 +792,8 @@ static cudaError_t launch_typed(const ContractNest &n, const ContractPlan &p, in
     a.gx = p.grid_x; a.nfull = 0; a.sp = 1;
     a.passes_i = p.passes_i; a.passes_j = p.passes_j;
     a.waf = p.waf;
+    static const int spread = devsw("EATSS_SIMT_BULK_SPREAD", 1);  // development A/B
+    a.bulk_spread = spread;
     a.counts = counts;
     if (counts) return by_variant<T, MODE_COVER>(a, p, n.transB, carveout, s);
     if (p.staged) {

@@ -120,9 +120,17 @@ __global__ void __launch_bounds__((16384 / (RM * RN)) < 1024 ? (16384 / (RM * RN
             const int64_t k0 = (int64_t)(ks0 + t) * p.Tk;
             const int kt = (int)imin64(p.Tk, p.K - k0);
             if constexpr (BULK) {
-                if (tid == 0) {
-                    mbar_arrive_expect_tx(bars + s, (unsigned)(kt * cols * 4));
-                    const T *src = p.B + k0 * p.ldb + j0;
+                // one bulk copy per B row; spread over lane 0 of every warp, so no warp falls a whole
+                // k-tile of copy issue behind the others (the trailing barrier would wait for it).  A copy
+                // may complete before thread 0's expect_tx: the transaction count goes transiently
+                // negative, and the phase cannot complete before thread 0's arrival.
+                const T *src = p.B + k0 * p.ldb + j0;
+                if (tid == 0) mbar_arrive_expect_tx(bars + s, (unsigned)(kt * cols * 4));
+                if (p.bulk_spread) {
+                    if ((tid & 31) == 0)
+                        for (int kk = tid >> 5; kk < kt; kk += (nthr + 31) >> 5)
+                            bulk_g2s(Bs + kk * bjp, src + kk * p.ldb, cols * 4, bars + s);
+                } else if (tid == 0) {
                     for (int kk = 0; kk < kt; kk++) bulk_g2s(Bs + kk * bjp, src + kk * p.ldb, cols * 4, bars + s);
                 }
             }

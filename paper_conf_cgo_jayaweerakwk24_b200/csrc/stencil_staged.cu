@@ -363,8 +363,10 @@ __global__ void __launch_bounds__(256) heat3d_resident(float *__restrict__ A, fl
         float *dst = (s & 1) ? A : B;
         const float *src = (s & 1) ? B : A;
         if (s > 0) {
-            if (tid < 6 && nbr[tid] >= 0)
+            if (tid < 6 && nbr[tid] >= 0) {
                 while (ld_acquire_gpu(flags + nbr[tid]) < (unsigned)s) __nanosleep(20);
+                __threadfence();  // as cooperative groups' grid sync: the barrier then orders every thread's loads
+            }
             __syncthreads();
             for (int e = tid; e < nfi + nfj + nfk; e += blockDim.x) {
                 if (e < nfi) {  // i faces: planes ilo-1 and ihi, rows [jlo, jhi), k-groups

@@ -30,3 +30,10 @@ for r in 1 0; do
   echo "== heat resident=$r"; EATSS_HEAT_RESIDENT=$r timeout 120 python scripts/time_kernel.py heat-3d 120 16,16,32 --tsteps 500 --iters 5 2>&1 | tail -1
   EATSS_HEAT_RESIDENT=$r timeout 120 python scripts/time_kernel.py heat-3d 512 16,16,32 --tsteps 5 --iters 5 2>&1 | tail -1
 done; done
+# SIMT staged executor: B row copies issued by every warp's lane 0 (1) vs thread 0 alone (0)
+timeout 900 python -m pytest tests/test_gpu_parity.py tests/test_gpu_waf.py -q -x -p no:cacheprovider -k "gemm or 2mm or syrk" 2>&1 | tail -2
+for rep in 1 2 3; do for v in 1 0; do
+  echo "== simt spread=$v"; EATSS_SIMT_BULK_SPREAD=$v timeout 120 python scripts/time_kernel.py gemm 4000,4000,4000 16,1024,16 --engine 1 --iters 20 2>&1 | tail -1
+  EATSS_SIMT_BULK_SPREAD=$v timeout 120 python scripts/time_kernel.py gemm 4000,4000,4000 32,512,48 --engine 1 --iters 20 2>&1 | tail -1
+done; done
+for t in 512 128; do echo "== simt threads=$t"; EATSS_THREADS=$t timeout 120 python scripts/time_kernel.py gemm 4000,4000,4000 16,1024,16 --engine 1 --iters 20 2>&1 | tail -1; done
