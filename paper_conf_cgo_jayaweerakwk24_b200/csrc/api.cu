@@ -33,11 +33,6 @@ cudaError_t launch_interior_copy2d(void *dst, const void *src, int64_t n, bool f
 // stencil_untiled.cu: the untiled baseline (engine EATSS_ENGINE_UNTILED; tile vector ignored)
 cudaError_t launch_jacobi2d_untiled(void *dst, const void *src, const void *bsrc, int64_t n, bool f64, cudaStream_t s);
 cudaError_t launch_heat3d_untiled(void *dst, const void *src, int64_t n, bool f64, cudaStream_t s);
-bool heat3d_staged_applicable(int64_t n, int64_t Ti, int64_t Tj, int64_t Tk, bool f64);
-int heat_resident_tiles(int64_t n, int64_t Ti, int64_t Tj, int64_t Tk);
-bool heat3d_resident_applicable(int64_t n, int64_t Ti, int64_t Tj, int64_t Tk);
-cudaError_t launch_heat3d_resident(float *A, float *B, int64_t n, int64_t Ti, int64_t Tj, int64_t Tk, int nsweeps,
-                                   int split_pct, unsigned *flags, cudaStream_t s, int waf);
 cudaError_t launch_heat3d_sweep(void *dst, const void *src, int64_t n, int64_t Ti, int64_t Tj,
                                 int64_t Tk, bool f64, int carveout, int32_t *counts, cudaStream_t s, int waf);
 int stencil_simt_x(bool heat, int64_t n, const int64_t *t, bool f64, int waf);
@@ -450,26 +445,6 @@ static cudaError_t stencil_issue(const eatss_kernel_desc *d, const int64_t *t, v
 }
 
 static eatss_status stencil_run(eatss_kernel_desc *d, const int64_t *t, void *const *b, cudaStream_t s) {
-    if (d->kind == EATSS_HEAT3D && d->dtype == EATSS_F32 && d->exec.engine != EATSS_ENGINE_UNTILED &&
-        d->tsteps >= 2 && d->dims[0] >= 3) {
-        // the whole time loop in one launch when every tile can stay resident (stencil_staged.cu); else
-        // one launch per sweep below
-        const int64_t n = d->dims[0];
-        if (heat3d_staged_applicable(n, t[0], t[1], t[2], false)) {
-            eatss_status st = ensure_ws(d, (size_t)heat_resident_tiles(n, t[0], t[1], t[2]) * sizeof(unsigned));
-            if (st != EATSS_OK) return st;
-            take_carveout();
-            cudaError_t e = launch_heat3d_resident((float *)b[0], (float *)b[1], n, t[0], t[1], t[2],
-                                                   (int)(2 * d->tsteps), exec_cv(d), (unsigned *)d->ws, s,
-                                                   d->exec.warp_align);
-            if (e == cudaSuccess) {
-                d->graph_cv = take_carveout();
-                return EATSS_OK;
-            }
-            if (e != cudaErrorNotSupported) return cuda_fail(e, "eatss_run(heat-3d resident)");
-            cudaGetLastError();
-        }
-    }
     if (!d->exec.use_graph || d->tsteps <= 1) {
         take_carveout();
         cudaError_t e = stencil_issue(d, t, b, s);
@@ -1306,12 +1281,7 @@ int64_t eatss_launches_per_run(const eatss_kernel_desc *d, const int64_t *tiles)
     switch (d->kind) {
         case EATSS_CCSD_T_D1: return 1;
         case EATSS_JACOBI2D: return d->tsteps + (d->tsteps > 0 ? 1 : 0);
-        case EATSS_HEAT3D:  // one resident launch for the whole time loop when every tile fits at once
-            if (tiles && d->dtype == EATSS_F32 && d->exec.engine != EATSS_ENGINE_UNTILED && d->tsteps >= 2 &&
-                d->dims[0] >= 3 && check_tiles(d, tiles) == EATSS_OK &&
-                heat3d_resident_applicable(d->dims[0], tiles[0], tiles[1], tiles[2]))
-                return 1;
-            return 2 * d->tsteps;
+        case EATSS_HEAT3D: return 2 * d->tsteps;
         case EATSS_MVT: case EATSS_BICG: return 1;  // one fused pass over the matrix
         case EATSS_ATAX: return 2;
         case EATSS_GEMVER: return 3;

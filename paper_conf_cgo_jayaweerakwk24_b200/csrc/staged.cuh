@@ -44,7 +44,7 @@ __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, unsigned by
 
 template <typename T, int RM, int RN, int V, bool TRANSB>
 __global__ void __launch_bounds__((16384 / (RM * RN)) < 1024 ? (16384 / (RM * RN)) : 1024,
-                                  (TRANSB && RM * RN == 64 && sizeof(T) == 4) ? 2 : 1)
+                                  (RM * RN == 64 && sizeof(T) == 4) ? 2 : 1)  // 8x8 fp32: two CTAs per SM (<= 128 registers)
     contract_staged_kernel(const CArgs<T> p) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     constexpr int VN = RN / V;

@@ -276,169 +276,6 @@ __global__ void __launch_bounds__(256) heat3d_staged(float *__restrict__ dst, co
     pdl_trigger();  // after this CTA's stores: the next sweep's launch overlaps this grid's tail
 }
 
-// ------------------------------------------------------------------ heat-3d, resident time loop
-// The whole time loop in ONE launch when every EATSS tile can be resident at once (the paper's
-// heat-3d size N = 120 is 13.8 MB for both arrays: it fits in the 148 SMs' shared memory).  One
-// CTA per tile for all sweeps; its window stays in shared memory (two windows: X_s and X_{s+1}), so a
-// sweep reloads only the cells its 7-point stencil takes from the six face neighbours (and the
-// non-output cells of its 16-byte k-groups), after those neighbours' progress flags say they have
-// finished the previous sweep.  Same tiles, same per-point arithmetic and association as
-// heat_tile (bit-identical results); every sweep still writes its outputs to the global array it
-// would write in the launched loop, so A and B end exactly as after 2*tsteps launched sweeps.
-// Hazards: sweep s of tile t reads X_s from its face neighbours' cells of array src_s after their
-// flags reach s (they wrote those cells in sweep s-1), and overwrites its own cells of the array
-// holding X_{s-1} only after the same flags say every neighbour has finished sweep s-1 -- including
-// that sweep's reads of those cells.
-__device__ __forceinline__ unsigned ld_acquire_gpu(const unsigned *p) {
-    unsigned v;
-    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];\n" : "=r"(v) : "l"(p) : "memory");
-    return v;
-}
-__device__ __forceinline__ void st_release_gpu(unsigned *p, unsigned v) {
-    asm volatile("st.release.gpu.global.u32 [%0], %1;\n" ::"l"(p), "r"(v) : "memory");
-}
-
-struct HeatTile {
-    int64_t ti0, tj0, tk0, ilo, ihi, jlo, jhi, klo, khi, g0, g1;
-};
-__device__ __forceinline__ HeatTile heat_tile_of(int64_t n, int Ti, int Tj, int Tk, int bi, int bj, int bk) {
-    HeatTile t;
-    t.ti0 = (int64_t)bi * Ti; t.tj0 = (int64_t)bj * Tj; t.tk0 = (int64_t)bk * Tk;
-    t.ilo = t.ti0 > 1 ? t.ti0 : 1; t.ihi = t.ti0 + Ti < n - 1 ? t.ti0 + Ti : n - 1;
-    t.jlo = t.tj0 > 1 ? t.tj0 : 1; t.jhi = t.tj0 + Tj < n - 1 ? t.tj0 + Tj : n - 1;
-    t.klo = t.tk0 > 1 ? t.tk0 : 1; t.khi = t.tk0 + Tk < n - 1 ? t.tk0 + Tk : n - 1;
-    t.g0 = t.klo >> 2; t.g1 = ((t.khi - 1) >> 2) + 1;
-    return t;
-}
-
-__global__ void __launch_bounds__(256) heat3d_resident(float *__restrict__ A, float *__restrict__ B,
-                                                       const __grid_constant__ CUtensorMap mA, int64_t n, int Ti,
-                                                       int Tj, int Tk, int nbj, int nbk, int nsweeps,
-                                                       unsigned *__restrict__ flags, int waf, int wfloats) {
-    extern __shared__ __align__(128) unsigned char rwin_raw[];
-    float *w0 = reinterpret_cast<float *>(rwin_raw + ((128u - (su32(rwin_raw) & 127u)) & 127u));
-    float *w1 = w0 + wfloats;
-    __shared__ uint64_t bar;
-    __shared__ int nbr[6];
-    const int tid = threadIdx.x;
-    const int bk = (int)(blockIdx.x % nbk), bij = (int)(blockIdx.x / nbk), bi = bij / nbj, bj = bij % nbj;
-    const int nbi = (int)(gridDim.x / nbk) / nbj;
-    const HeatTile T = heat_tile_of(n, Ti, Tj, Tk, bi, bj, bk);
-    if (T.ilo >= T.ihi || T.jlo >= T.jhi || T.klo >= T.khi) {  // empty tile: never a neighbour to wait for
-        if (tid == 0) st_release_gpu(flags + blockIdx.x, (unsigned)nsweeps);
-        return;
-    }
-    if (tid < 6) {  // face neighbours (tile index or -1): i-1, i+1, j-1, j+1, k-1, k+1
-        const int d = tid >> 1, sgn = (tid & 1) ? 1 : -1;
-        const int ni = bi + (d == 0 ? sgn : 0), nj = bj + (d == 1 ? sgn : 0), nk = bk + (d == 2 ? sgn : 0);
-        nbr[tid] = (ni < 0 || ni >= nbi || nj < 0 || nj >= nbj || nk < 0 || nk >= nbk) ? -1 : (ni * nbj + nj) * nbk + nk;
-    }
-    if (tid == 0) {
-        mbar_init(&bar, 1);
-        asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
-        mbar_expect_tx(&bar, (unsigned)((Ti + 2) * (Tj + 2) * (Tk + 8) * 4));
-        tcm::tma_3d(w0, &mA, (int)(T.tk0 - 4), (int)(T.tj0 - 1), (int)(T.ti0 - 1), &bar);  // X_0's window
-    }
-    __syncthreads();
-    mbar_wait(&bar, 0);
-    const int KW = Tk + 8, JW = Tj + 2, plane = JW * KW;
-    const int ng = (int)(T.g1 - T.g0), nj = (int)(T.jhi - T.jlo), ni = (int)(T.ihi - T.ilo);
-    const int64_t nn = n * n;
-    // window offset of global cell (i, j, k)
-    auto woff = [&](int64_t i, int64_t j, int64_t k) {
-        return (int)(i - (T.ti0 - 1)) * plane + (int)(j - (T.tj0 - 1)) * KW + (int)(k - (T.tk0 - 4));
-    };
-    // refill counts: i faces and j faces as float4 k-groups, then the k cells of every (i, j) column
-    const int nfi = 2 * nj * ng, nfj = 2 * ni * ng;
-    const int kbefore = (int)(T.klo - 4 * T.g0) + 1, kafter = (int)(4 * T.g1 - T.khi) + 1;  // incl. 4g0-1, 4g1
-    const int kcells = kbefore + kafter, nfk = ni * nj * kcells;
-    const int cols = nj * ng;
-    const int chunks = max(1, min(ni, (int)blockDim.x / cols));
-    const int per = (ni + chunks - 1) / chunks;
-    const int nb = nj * chunks, span = waf > 0 ? ((ng + waf - 1) / waf) * waf * (((nb + 32 / waf - 1) / (32 / waf)) * (32 / waf))
-                                              : cols * chunks;
-    const float c = 0.125f, two = 2.0f;
-    for (int s = 0; s < nsweeps; s++) {
-        float *cur = (s & 1) ? w1 : w0, *nxt = (s & 1) ? w0 : w1;
-        float *dst = (s & 1) ? A : B;
-        const float *src = (s & 1) ? B : A;
-        if (s > 0) {
-            if (tid < 6 && nbr[tid] >= 0) {
-                while (ld_acquire_gpu(flags + nbr[tid]) < (unsigned)s) __nanosleep(20);
-                __threadfence();  // as cooperative groups' grid sync: the barrier then orders every thread's loads
-            }
-            __syncthreads();
-            for (int e = tid; e < nfi + nfj + nfk; e += blockDim.x) {
-                if (e < nfi) {  // i faces: planes ilo-1 and ihi, rows [jlo, jhi), k-groups
-                    const int g = e % ng, r = e / ng, jj = r % nj, f = r / nj;
-                    const int64_t i = f ? T.ihi : T.ilo - 1, j = T.jlo + jj, k = 4 * (T.g0 + g);
-                    *reinterpret_cast<float4 *>(cur + woff(i, j, k)) =
-                        __ldcg(reinterpret_cast<const float4 *>(src + i * nn + j * n + k));
-                } else if (e < nfi + nfj) {  // j faces: rows jlo-1 and jhi of planes [ilo, ihi)
-                    const int x = e - nfi, g = x % ng, r = x / ng, ii = r % ni, f = r / ni;
-                    const int64_t i = T.ilo + ii, j = f ? T.jhi : T.jlo - 1, k = 4 * (T.g0 + g);
-                    *reinterpret_cast<float4 *>(cur + woff(i, j, k)) =
-                        __ldcg(reinterpret_cast<const float4 *>(src + i * nn + j * n + k));
-                } else {  // k cells of each (i, j) column: 4g0-1 .. klo-1 and khi .. 4g1
-                    const int x = e - nfi - nfj, q = x % kcells, col = x / kcells, jj = col % nj, ii = col / nj;
-                    const int64_t i = T.ilo + ii, j = T.jlo + jj;
-                    const int64_t k = q < kbefore ? 4 * T.g0 - 1 + q : T.khi + (q - kbefore);
-                    if (k >= 0 && k < n) cur[woff(i, j, k)] = __ldcg(src + i * nn + j * n + k);
-                }
-            }
-            __syncthreads();
-        }
-        for (int e = tid; e < span; e += blockDim.x) {
-            int gi, b;
-            if (!waf_item(e, ng, nb, waf, gi, b) || gi >= ng) continue;
-            const int jj = b % nj, ch = b / nj;
-            const int ib = ch * per, ie = min(ni, ib + per);
-            if (ib >= ie) continue;
-            const int64_t k = 4 * (T.g0 + gi), j = T.jlo + jj;
-            const int wk = (int)(k - (T.tk0 - 4)), wj = (int)(j - (T.tj0 - 1));
-            const float *colp = cur + wj * KW + wk;
-            float *ncol = nxt + wj * KW + wk;
-            const bool full = k >= T.klo && k + 3 < T.khi;
-            const int wi0 = (int)(T.ilo + ib - (T.ti0 - 1));
-            float4 u = *reinterpret_cast<const float4 *>(colp + (wi0 - 1) * plane);
-            float4 x = *reinterpret_cast<const float4 *>(colp + wi0 * plane);
-            for (int wi = wi0; wi < wi0 + (ie - ib); wi++) {
-                const float *p = colp + wi * plane;
-                const float4 ip = *reinterpret_cast<const float4 *>(p + plane);
-                const float4 jp = *reinterpret_cast<const float4 *>(p + KW);
-                const float4 jm = *reinterpret_cast<const float4 *>(p - KW);
-                const float km1 = p[-1], kp4 = p[4];
-                float4 o;
-#define HEAT_PT3(X, IP, IM, JP, JM, KP, KM) \
-    (c * (IP - two * X + IM) + c * (JP - two * X + JM) + c * (KP - two * X + KM) + X)
-                o.x = HEAT_PT3(x.x, ip.x, u.x, jp.x, jm.x, x.y, km1);
-                o.y = HEAT_PT3(x.y, ip.y, u.y, jp.y, jm.y, x.z, x.x);
-                o.z = HEAT_PT3(x.z, ip.z, u.z, jp.z, jm.z, x.w, x.y);
-                o.w = HEAT_PT3(x.w, ip.w, u.w, jp.w, jm.w, kp4, x.z);
-#undef HEAT_PT3
-                *reinterpret_cast<float4 *>(ncol + wi * plane) = o;  // non-output lanes are refilled next sweep
-                const int64_t i = T.ti0 - 1 + wi;
-                float *out = dst + i * nn + j * n + k;
-                if (full) {
-                    *reinterpret_cast<float4 *>(out) = o;
-                } else {
-                    const float ov[4] = {o.x, o.y, o.z, o.w};
-#pragma unroll
-                    for (int q = 0; q < 4; q++)
-                        if (k + q >= T.klo && k + q < T.khi) out[q] = ov[q];
-                }
-                u = x;
-                x = ip;
-            }
-        }
-        __syncthreads();  // every output of sweep s stored (CTA scope) ...
-        if (tid == 0) {
-            __threadfence();  // ... and ordered before the flag at GPU scope (cumulative through the barrier)
-            st_release_gpu(flags + blockIdx.x, (unsigned)(s + 1));
-        }
-    }
-}
-
 constexpr int kSmemTarget = 113 * 1024;  // at least two resident CTAs per SM
 
 // launch with programmatic stream serialization allowed (the kernel calls pdl_trigger / pdl_wait);
@@ -532,75 +369,6 @@ cudaError_t launch_heat3d_staged(float *dst, const float *src, int64_t n, int64_
     cudaFuncSetAttribute(heat3d_staged<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     return launch_pdl(heat3d_staged<false>, grid, block, smem, staged_carveout(smem, split_pct), s, dst,
                       (const CUtensorMap)m, n, (int)Ti, (int)Tj, (int)Tk, (int)nbj, (int32_t *)nullptr, waf);
-}
-
-
-// The resident time loop (heat3d_resident): nsweeps sweeps in one cooperative launch; flags = one
-// unsigned per tile, zeroed here.  cudaErrorNotSupported when the tiles cannot all be resident (the
-// caller then launches one grid per sweep).
-int heat_resident_tiles(int64_t n, int64_t Ti, int64_t Tj, int64_t Tk) {
-    return (int)(((n - 1 + Ti - 1) / Ti) * ((n - 1 + Tj - 1) / Tj) * ((n - 1 + Tk - 1) / Tk));
-}
-static int heat_resident_wfloats(int64_t Ti, int64_t Tj, int64_t Tk) {
-    return (int)(((Ti + 2) * (Tj + 2) * (Tk + 8) + 31) / 32 * 32);
-}
-// every tile resident at once on the current device (two windows per CTA), with the resident path enabled
-bool heat3d_resident_applicable(int64_t n, int64_t Ti, int64_t Tj, int64_t Tk) {
-    static const bool on = [] {  // development: EATSS_HEAT_RESIDENT=0 keeps one launch per sweep
-        const char *e = getenv("EATSS_HEAT_RESIDENT");
-        return !(e && atoi(e) == 0);
-    }();
-    if (!on || !heat3d_staged_applicable(n, Ti, Tj, Tk, false)) return false;
-    const int smem = 2 * heat_resident_wfloats(Ti, Tj, Tk) * 4 + 128;
-    int dev = 0, nsm = 0, per_sm = 0;
-    if (cudaGetDevice(&dev) != cudaSuccess ||
-        cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess ||
-        cudaFuncSetAttribute(heat3d_resident, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess ||
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, heat3d_resident, 256, smem) != cudaSuccess) {
-        cudaGetLastError();
-        return false;
-    }
-    return (int64_t)per_sm * nsm >= heat_resident_tiles(n, Ti, Tj, Tk);
-}
-cudaError_t launch_heat3d_resident(float *A, float *B, int64_t n, int64_t Ti, int64_t Tj, int64_t Tk, int nsweeps,
-                                   int split_pct, unsigned *flags, cudaStream_t s, int waf) {
-    if (!flags || nsweeps < 4 || !heat3d_resident_applicable(n, Ti, Tj, Tk)) return cudaErrorNotSupported;
-    const int64_t nbj = (n - 1 + Tj - 1) / Tj, nbk = (n - 1 + Tk - 1) / Tk;
-    const int64_t ntiles = heat_resident_tiles(n, Ti, Tj, Tk);
-    const int wfloats = heat_resident_wfloats(Ti, Tj, Tk);
-    const int smem = 2 * wfloats * 4 + 128;
-    cudaError_t e;
-    const int cv = staged_carveout(smem, split_pct);
-    CUtensorMap m{};
-    const cuuint64_t dims[3] = {(cuuint64_t)n, (cuuint64_t)n, (cuuint64_t)n};
-    const cuuint64_t strides[2] = {(cuuint64_t)n * 4, (cuuint64_t)n * n * 4};
-    const cuuint32_t box[3] = {(cuuint32_t)(Tk + 8), (cuuint32_t)(Tj + 2), (cuuint32_t)(Ti + 2)};
-    const cuuint32_t es[3] = {1, 1, 1};
-    if (tcm::encode_fn()(&m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, A, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                         CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                         CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
-        return cudaErrorInvalidValue;
-    if ((e = cudaMemsetAsync(flags, 0, (size_t)ntiles * sizeof(unsigned), s)) != cudaSuccess) return e;
-    cudaLaunchConfig_t cfg{};
-    cfg.gridDim = dim3((unsigned)ntiles);
-    cfg.blockDim = dim3(256);
-    cfg.dynamicSmemBytes = (size_t)smem;
-    cfg.stream = s;
-    cudaLaunchAttribute at[2];
-    at[0].id = cudaLaunchAttributeCooperative;  // every CTA resident: the flag waits cannot deadlock
-    at[0].val.cooperative = 1;
-    at[1].id = cudaLaunchAttributePreferredSharedMemoryCarveout;
-    at[1].val.sharedMemCarveout = (unsigned)cv;
-    cfg.attrs = at;
-    cfg.numAttrs = 2;
-    note_carveout(cv);
-    e = cudaLaunchKernelEx(&cfg, heat3d_resident, A, B, (const CUtensorMap)m, n, (int)Ti, (int)Tj, (int)Tk, (int)nbj,
-                           (int)nbk, nsweeps, flags, waf, wfloats);
-    if (e == cudaErrorCooperativeLaunchTooLarge) {  // e.g. an exact carve-out below two CTAs per SM
-        cudaGetLastError();
-        return cudaErrorNotSupported;
-    }
-    return e;
 }
 
 }  // namespace eatss

@@ -822,38 +822,6 @@ __device__ void tail_prepass_block(const Args &p, int blk, int npb, int rows_per
     }
 }
 
-// Second launch of the 3xFP16 engine when B's column maxima ran alone in the first (split order 1):
-// blocks [0, nbc) split B into K-major tiles while B is still L2-resident from the maxima pass (four warps
-// cover a 32 x 128 tile in two passes), blocks [nbc, nbc + nr0) split the row operands read once
-// (f16_rows_staged, one row buffer per warp in dynamic shared memory), the rest the split-k tail pre-pass.
-__global__ void __launch_bounds__(F16_PASS1_THREADS) f16_split_kernel(const F16Cols cj, const unsigned *colmax,
-                                                                     int nbc, const F16Rows r0, const F16Rows r1,
-                                                                     int nr0, int rowbuf_floats, const Args p,
-                                                                     int rows_per_tile, int bn, int vecC) {
-    const int b = (int)blockIdx.x, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
-    if (b < nbc) {
-        const int64_t ntiles = ((cj.N + 31) / 32) * ((cj.ldp + 127) / 128);
-        for (int64_t tile = b; tile < ntiles; tile += nbc)
-            for (int v = w; v < 8; v += nw) f16_cols_tile(cj, colmax, tile, v);
-        return;
-    }
-    if (b < nbc + nr0) {
-        extern __shared__ __align__(16) float f16_rowbuf2[];
-        __shared__ __align__(8) uint64_t bars[F16_PASS1_THREADS / 32];
-        if ((threadIdx.x & 31) == 0) {
-            mbar_init(bars + w, 1);
-            asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
-        }
-        __syncwarp();
-        const int64_t w0 = (int64_t)(b - nbc) * nw + w, ws = (int64_t)nr0 * nw;
-        float *buf = f16_rowbuf2 + (size_t)w * rowbuf_floats;
-        if (r0.x) f16_rows_staged(r0, buf, bars + w, w0, ws);
-        if (r1.x) f16_rows_staged(r1, buf, bars + w, w0, ws);
-        return;
-    }
-    tail_prepass_block(p, b - nbc - nr0, (int)gridDim.x - nbc - nr0, rows_per_tile, bn, vecC);
-}
-
 // ------------------------------------------------------------------ host side
 }  // namespace tcm
 
@@ -984,36 +952,6 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
         const int npb = (int)std::min<int64_t>((tail4 + 255) / 256, (int64_t)nsm * 4);
         const int vecC = (a.ldc % 4 == 0 && (reinterpret_cast<uintptr_t>(a.C) & 15) == 0) ? 1 : 0;
         if constexpr (F16) {
-            static const int split_order = devsw("EATSS_TCF_SPLIT_ORDER", 0);  // development A/B
-            if (split_order == 1 && pr.fused_rows && pr.colmax) {
-                // launch 1: B's column maxima alone; launch 2: B's split first (B still in L2), then the
-                // row operands read once, then the tail pre-pass
-                if ((e = cudaMemsetAsync(pr.maxes, 0, pr.maxes_bytes, s)) != cudaSuccess) return e;
-                constexpr int TPB = tcm::F16_PASS1_THREADS, NW = TPB / 32;
-                const int ncb = (int)(((pr.cj.N + 127) / 128) * ((pr.cj.K + 255) / 256));
-                tcm::f16_max_kernel<<<ncb, TPB, 0, s>>>(pr.r0, pr.m0, pr.r1, pr.m1, pr.cj, pr.colmax, 0, 0, 1, 0);
-                if ((e = cudaGetLastError()) != cudaSuccess) return e;
-                const tcm::F16Rows &rr = pr.r0.x ? pr.r0 : pr.r1;
-                const int rowbuf = (int)((rr.cols + 3) / 4 * 4);
-                const size_t dsm = (size_t)NW * rowbuf * sizeof(float);
-                const int64_t nrows = std::max(pr.r0.x ? pr.r0.rows : 0, pr.r1.x ? pr.r1.rows : 0);
-                const int nr0 = (int)std::min<int64_t>((nrows + NW - 1) / NW, (int64_t)nsm * 3);
-                const int nbc = (int)std::min<int64_t>(((pr.cj.N + 31) / 32) * ((pr.cj.ldp + 127) / 128), (int64_t)nsm * 12);
-                auto kf = tcm::f16_split_kernel;
-                {
-                    std::lock_guard<std::mutex> lk(g_ks_mu);
-                    KernelState &ks = g_ks[{reinterpret_cast<const void *>(kf), dev}];
-                    if (ks.smem < (int)dsm) {
-                        if ((e = cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsm)) !=
-                            cudaSuccess)
-                            return e;
-                        ks.smem = (int)dsm;
-                    }
-                }
-                const int npb2 = (int)std::min<int64_t>((tail4 + TPB - 1) / TPB, (int64_t)nsm * 8);
-                tcm::f16_split_kernel<<<nbc + nr0 + npb2, TPB, dsm, s>>>(pr.cj, pr.colmax, nbc, pr.r0, pr.r1, nr0,
-                                                                         rowbuf, a, rows, a.BNT, vecC);
-            } else {
             {  // first launch: the row operands (fused: split, each row read once; else their maxima) and the
                // column maxima of a row-major B
                 if ((e = cudaMemsetAsync(pr.maxes, 0, pr.maxes_bytes, s)) != cudaSuccess) return e;
@@ -1050,7 +988,6 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
             const int nbr = pr.fused_rows ? 0 : pr.nbr;  // fused: the rows are already split
             tcm::prep_f16_kernel<<<std::max(1, nbr + pr.nbc + npb), 256, 0, s>>>(pr.r0, pr.r1, pr.cj, pr.colmax, nbr,
                                                                                pr.nbc, a, rows, a.BNT, vecC);
-            }
         } else {
             tcm::prep_kernel<<<pr.nb0 + pr.nb1 + npb, 256, 0, s>>>(pr.j0, pr.j1, pr.nb0, pr.nb1, pr.mode, a, rows,
                                                                    a.BNT, vecC);

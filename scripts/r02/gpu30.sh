@@ -2,10 +2,10 @@
 # split order A/B (0: rows+colmax then B split; 1: colmax, then B split + rows), dbg 16 = no MMAs (operand delivery only), 32 = no operand TMA (MMA only), raster group and chunk
 cd $GRAFT_REPO_ROOT; mkdir -p gpurun_out/r02
 EATSS_DEV_NVCC_FLAGS=-DEATSS_DEVTOOLS python paper_conf_cgo_jayaweerakwk24_b200/build.py --force -j 32 > /dev/null 2>&1 || echo BUILD FAILED
-EATSS_TCF_SPLIT_ORDER=1 timeout 600 python -m pytest tests/test_gpu_f16.py tests/test_gpu_fullsize.py -k "f16 or tensor16" -q -x -p no:cacheprovider 2>&1 | tail -2
+
 T="scripts/time_kernel.py gemm 4000,4000,4000 256,256,64 --engine 4 --iters 50 --kernel-ms"
 run() { echo "== $*"; env "$@" timeout 120 python $T 2>&1 | tail -2; }
-for rep in 1 2 3; do run EATSS_TCF_SPLIT_ORDER=0; run EATSS_TCF_SPLIT_ORDER=1; done
+
 for rep in 1 2; do
 run EATSS_TCM_DBG=0
 run EATSS_TCM_DBG=16
@@ -23,13 +23,6 @@ run EATSS_TCM_DBG=16
 T="scripts/time_kernel.py gemm 4000,4000,4000 256,128,64 --engine 4 --iters 50 --kernel-ms"
 run EATSS_TCM_DBG=0
 run EATSS_TCM_DBG=16
-# heat-3d resident time loop: parity, then timing vs one launch per sweep (EATSS_HEAT_RESIDENT=0)
-timeout 600 python -m pytest tests/test_gpu_heat_resident.py tests/test_gpu_parity.py -k "heat" -q -x -p no:cacheprovider 2>&1 | tail -3
-for rep in 1 2; do
-for r in 1 0; do
-  echo "== heat resident=$r"; EATSS_HEAT_RESIDENT=$r timeout 120 python scripts/time_kernel.py heat-3d 120 16,16,32 --tsteps 500 --iters 5 2>&1 | tail -1
-  EATSS_HEAT_RESIDENT=$r timeout 120 python scripts/time_kernel.py heat-3d 512 16,16,32 --tsteps 5 --iters 5 2>&1 | tail -1
-done; done
 # SIMT staged executor: B row copies issued by every warp's lane 0 (1) vs thread 0 alone (0)
 timeout 900 python -m pytest tests/test_gpu_parity.py tests/test_gpu_waf.py -q -x -p no:cacheprovider -k "gemm or 2mm or syrk" 2>&1 | tail -2
 for rep in 1 2 3; do for v in 1 0; do
