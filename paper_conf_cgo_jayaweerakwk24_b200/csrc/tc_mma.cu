@@ -777,13 +777,54 @@ __device__ void f16_cols_tile(const F16Cols &j, const unsigned *colmax, int64_t 
         lp[1] = *reinterpret_cast<const uint4 *>(&l[8]);
     }
 }
+// The same 32-column x 128-k tile through shared memory (256 threads): the loads are the coalesced row
+// segments of f16_cols_tile, the split halves of each column are parked in shared memory, and every
+// column's K-major run (128 k = 256 bytes per half) then leaves as ONE contiguous warp store -- instead of
+// 16-byte pieces of 32 different columns per store instruction.
+constexpr int F16T_LD = 128 + 8;  // halves per parked column (16-byte pad: 16-byte lane stores stay 4 wavefronts)
+__device__ void f16_cols_tile_smem(const F16Cols &j, const unsigned *colmax, int64_t tile, __half *sh, __half *sl) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int64_t nstrip = (j.N + 31) / 32;
+    const int64_t c0 = (tile % nstrip) * 32, kt0 = (tile / nstrip) * 128;
+    const int64_t col = c0 + lane, k0 = kt0 + 16 * w;
+    if (col < j.N && k0 < j.ldp) {
+        const int s = f16_scale_exp(__uint_as_float(colmax[col]));
+        if (kt0 == 0 && w == 0) j.exps[col] = s;
+        const float sc = __int_as_float((127 + s) << 23);
+        float v[16];
+#pragma unroll
+        for (int u = 0; u < 16; u++) v[u] = k0 + u < j.K ? __ldg(j.x + (k0 + u) * j.ldx + col) : 0.f;
+        __half h[16], l[16];
+#pragma unroll
+        for (int u = 0; u < 16; u++) f16_split(v[u], sc, h[u], l[u]);
+        uint4 *hp = reinterpret_cast<uint4 *>(sh + lane * F16T_LD + 16 * w);
+        uint4 *lp = reinterpret_cast<uint4 *>(sl + lane * F16T_LD + 16 * w);
+        hp[0] = *reinterpret_cast<const uint4 *>(&h[0]);
+        hp[1] = *reinterpret_cast<const uint4 *>(&h[8]);
+        lp[0] = *reinterpret_cast<const uint4 *>(&l[0]);
+        lp[1] = *reinterpret_cast<const uint4 *>(&l[8]);
+    }
+    __syncthreads();
+    // warp w writes columns 4w .. 4w+3: lane l the 4 halves at k = kt0 + 4l (ldp % 8 == 0: whole or none)
+    const int64_t k = kt0 + 4 * lane;
+#pragma unroll
+    for (int q = 0; q < 4; q++) {
+        const int cl = 4 * w + q;
+        const int64_t c = c0 + cl;
+        if (c < j.N && k < j.ldp) {
+            *reinterpret_cast<uint2 *>(j.hi + c * j.ldp + k) = *reinterpret_cast<const uint2 *>(sh + cl * F16T_LD + 4 * lane);
+            *reinterpret_cast<uint2 *>(j.lo + c * j.ldp + k) = *reinterpret_cast<const uint2 *>(sl + cl * F16T_LD + 4 * lane);
+        }
+    }
+    __syncthreads();  // the parked tile may be overwritten by the block's next tile
+}
 __device__ void tail_prepass_block(const Args &p, int blk, int npb, int rows_per_tile, int bn, int vecC);
 // The launch before the 3xFP16 GEMM: blocks [0, nbr) split the row operands (A, and B when it is K-major
 // -- syrk), [nbr, nbr + nbc) the 32 x 128 tiles of a row-major B (its column maxima from f16_max_kernel),
 // the rest the split-k tail pre-pass.
 __global__ void __launch_bounds__(256, 4) prep_f16_kernel(const F16Rows r0, const F16Rows r1, const F16Cols cj,
                                                        const unsigned *colmax, int nbr, int nbc, const Args p,
-                                                       int rows_per_tile, int bn, int vecC) {
+                                                       int rows_per_tile, int bn, int vecC, int parked) {
     const int b = (int)blockIdx.x;
     if (b < nbr) {
         const int64_t wstride = (int64_t)nbr * 8, w0 = (int64_t)b * 8 + (threadIdx.x >> 5);
@@ -793,7 +834,11 @@ __global__ void __launch_bounds__(256, 4) prep_f16_kernel(const F16Rows r0, cons
     }
     if (b < nbr + nbc) {
         const int64_t ntiles = ((cj.N + 31) / 32) * ((cj.ldp + 127) / 128);
-        for (int64_t tile = b - nbr; tile < ntiles; tile += nbc) f16_cols_tile(cj, colmax, tile, threadIdx.x >> 5);
+        __shared__ __align__(16) __half park[2][32 * F16T_LD];
+        for (int64_t tile = b - nbr; tile < ntiles; tile += nbc) {
+            if (parked) f16_cols_tile_smem(cj, colmax, tile, park[0], park[1]);
+            else f16_cols_tile(cj, colmax, tile, threadIdx.x >> 5);
+        }
         return;
     }
     tail_prepass_block(p, b - nbr - nbc, (int)gridDim.x - nbr - nbc, rows_per_tile, bn, vecC);
@@ -987,7 +1032,8 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
             }
             const int nbr = pr.fused_rows ? 0 : pr.nbr;  // fused: the rows are already split
             tcm::prep_f16_kernel<<<std::max(1, nbr + pr.nbc + npb), 256, 0, s>>>(pr.r0, pr.r1, pr.cj, pr.colmax, nbr,
-                                                                               pr.nbc, a, rows, a.BNT, vecC);
+                                                                               pr.nbc, a, rows, a.BNT, vecC,
+                                                                               devsw("EATSS_TCF_PARKED", 1));
         } else {
             tcm::prep_kernel<<<pr.nb0 + pr.nb1 + npb, 256, 0, s>>>(pr.j0, pr.j1, pr.nb0, pr.nb1, pr.mode, a, rows,
                                                                    a.BNT, vecC);
