@@ -131,6 +131,9 @@ struct KMajor {
     }
 };
 
+// programmatic dependent launch (the launches of one GEMM are chained with it)
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;\n" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;\n" ::: "memory"); }
 // BKB: bytes of k per operand row and stage; F16: 3xFP16 operands (K-major A and B, per-row / per-column
 // power-of-two scales undone in the epilogue), else 3xTF32
 template <int BKB, bool TB, int CG, bool F16>
@@ -186,6 +189,9 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     if constexpr (CG == 2) cluster_sync(); else __syncthreads();
     fence_after();
     const uint32_t tmem = *tmem_slot;
+    // programmatic dependent launch: the prologue above overlapped the split launch's tail; operands,
+    // exponents and the pre-scaled C are read only after it has completed (a no-op without the attribute)
+    pdl_wait();
 
     if (warp == 0) {
         if (lane == 0) {  // ---------------------------------------------- TMA producer
@@ -715,9 +721,9 @@ __device__ void f16_rows_staged(const F16Rows &j, float *buf, uint64_t *bar, int
 //   fused = 0: blocks [0, nr0) row maxima of r0, [nr0, nr0 + nr1) of r1 (the split follows in prep_f16_kernel);
 // the rest: the column maxima of a row-major B (cj; colmax).
 constexpr int F16_PASS1_THREADS = 128;
-__global__ void __launch_bounds__(F16_PASS1_THREADS) f16_max_kernel(const F16Rows r0, unsigned *m0, const F16Rows r1,
-                                                                   unsigned *m1, const F16Cols cj, unsigned *colmax,
-                                                                   int nr0, int nr1, int fused, int rowbuf_floats) {
+__device__ __forceinline__ void f16_max_body(const F16Rows &r0, unsigned *m0, const F16Rows &r1, unsigned *m1,
+                                             const F16Cols &cj, unsigned *colmax, int nr0, int nr1, int fused,
+                                             int rowbuf_floats) {
     const int64_t b = blockIdx.x;
     if (fused && b < nr0) {
         extern __shared__ __align__(16) float f16_rowbuf[];
@@ -749,6 +755,14 @@ __global__ void __launch_bounds__(F16_PASS1_THREADS) f16_max_kernel(const F16Row
     }
     const int64_t c = b - nr0 - nr1, nsx = (cj.N + 127) / 128;
     f16_colmax_block(cj.x, cj.K, cj.N, cj.ldx, colmax, c % nsx, c / nsx);
+}
+// Launch 1 of the 3xFP16 chain.  Each block lets the split launch be scheduled once its own stores are
+// issued (programmatic dependent launch); the split launch still waits for this whole grid.
+__global__ void __launch_bounds__(F16_PASS1_THREADS) f16_max_kernel(const F16Rows r0, unsigned *m0, const F16Rows r1,
+                                                                   unsigned *m1, const F16Cols cj, unsigned *colmax,
+                                                                   int nr0, int nr1, int fused, int rowbuf_floats) {
+    f16_max_body(r0, m0, r1, m1, cj, colmax, nr0, nr1, fused, rowbuf_floats);
+    pdl_trigger();
 }
 // one 32-column x 128-k tile of a row-major B, no shared memory: lane = column, warp w = k rows
 // [16w, 16w + 16) of the tile.  Each of the 16 loads is one coalesced 128-byte row segment across the warp
@@ -822,9 +836,9 @@ __device__ void tail_prepass_block(const Args &p, int blk, int npb, int rows_per
 // The launch before the 3xFP16 GEMM: blocks [0, nbr) split the row operands (A, and B when it is K-major
 // -- syrk), [nbr, nbr + nbc) the 32 x 128 tiles of a row-major B (its column maxima from f16_max_kernel),
 // the rest the split-k tail pre-pass.
-__global__ void __launch_bounds__(256, 4) prep_f16_kernel(const F16Rows r0, const F16Rows r1, const F16Cols cj,
-                                                       const unsigned *colmax, int nbr, int nbc, const Args p,
-                                                       int rows_per_tile, int bn, int vecC, int parked) {
+__device__ __forceinline__ void prep_f16_body(const F16Rows &r0, const F16Rows &r1, const F16Cols &cj,
+                                              const unsigned *colmax, int nbr, int nbc, const Args &p,
+                                              int rows_per_tile, int bn, int vecC, int parked) {
     const int b = (int)blockIdx.x;
     if (b < nbr) {
         const int64_t wstride = (int64_t)nbr * 8, w0 = (int64_t)b * 8 + (threadIdx.x >> 5);
@@ -842,6 +856,13 @@ __global__ void __launch_bounds__(256, 4) prep_f16_kernel(const F16Rows r0, cons
         return;
     }
     tail_prepass_block(p, b - nbr - nbc, (int)gridDim.x - nbr - nbc, rows_per_tile, bn, vecC);
+}
+__global__ void __launch_bounds__(256, 4) prep_f16_kernel(const F16Rows r0, const F16Rows r1, const F16Cols cj,
+                                                       const unsigned *colmax, int nbr, int nbc, const Args p,
+                                                       int rows_per_tile, int bn, int vecC, int parked) {
+    pdl_wait();  // launch 1 complete and visible (column maxima, row splits)
+    prep_f16_body(r0, r1, cj, colmax, nbr, nbc, p, rows_per_tile, bn, vecC, parked);
+    pdl_trigger();
 }
 // split-k tail pre-pass: C := init_zero ? 0 : beta*C on the tiles t >= nfull, block `blk` of `npb`
 __device__ void tail_prepass_block(const Args &p, int blk, int npb, int rows_per_tile, int bn, int vecC) {
@@ -960,12 +981,16 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
     int dev = 0;
     cudaGetDevice(&dev);
     int ncl = nsm / CG;
+    // programmatic dependent launch of the split launch(es) and the GEMM (EATSS_TCM_PDL=0: plain launches)
+    static const bool pdl = devsw("EATSS_TCM_PDL", 1) != 0;
     cudaLaunchConfig_t cfg = {};
-    cudaLaunchAttribute attr[1];
+    cudaLaunchAttribute attr[2];
     attr[0].id = cudaLaunchAttributeClusterDimension;
     attr[0].val.clusterDim.x = CG;
     attr[0].val.clusterDim.y = 1;
     attr[0].val.clusterDim.z = 1;
+    attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[1].val.programmaticStreamSerializationAllowed = pdl ? 1 : 0;
     cfg.blockDim = dim3(tcm::NTHREADS);
     cfg.dynamicSmemBytes = (size_t)smem;
     cfg.stream = s;
@@ -1031,9 +1056,18 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
                 if ((e = cudaGetLastError()) != cudaSuccess) return e;
             }
             const int nbr = pr.fused_rows ? 0 : pr.nbr;  // fused: the rows are already split
-            tcm::prep_f16_kernel<<<std::max(1, nbr + pr.nbc + npb), 256, 0, s>>>(pr.r0, pr.r1, pr.cj, pr.colmax, nbr,
-                                                                               pr.nbc, a, rows, a.BNT, vecC,
-                                                                               devsw("EATSS_TCF_PARKED", 1));
+            cudaLaunchConfig_t pc = {};
+            cudaLaunchAttribute pa[1];
+            pa[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+            pa[0].val.programmaticStreamSerializationAllowed = pdl ? 1 : 0;
+            pc.gridDim = dim3((unsigned)std::max(1, nbr + pr.nbc + npb));
+            pc.blockDim = dim3(256);
+            pc.stream = s;
+            pc.attrs = pa;
+            pc.numAttrs = 1;
+            e = cudaLaunchKernelEx(&pc, tcm::prep_f16_kernel, pr.r0, pr.r1, pr.cj, (const unsigned *)pr.colmax, nbr,
+                                   pr.nbc, (const tcm::Args)a, rows, (int)a.BNT, vecC, devsw("EATSS_TCF_PARKED", 1));
+            if (e != cudaSuccess) return e;
         } else {
             tcm::prep_kernel<<<pr.nb0 + pr.nb1 + npb, 256, 0, s>>>(pr.j0, pr.j1, pr.nb0, pr.nb1, pr.mode, a, rows,
                                                                    a.BNT, vecC);
@@ -1041,6 +1075,7 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
     }
     cfg.gridDim = dim3((unsigned)(CG * ncl));
+    cfg.numAttrs = 2;  // + programmatic serialization (the occupancy query above used the cluster attribute only)
     if (ev) cudaEventRecord(ev[0], s);
     e = cudaLaunchKernelEx(&cfg, k, m[0], m[1], m[2], m[3], a);
     if (ev) cudaEventRecord(ev[1], s);
