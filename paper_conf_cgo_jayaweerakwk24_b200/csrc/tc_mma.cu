@@ -981,8 +981,11 @@ static cudaError_t launch_one(const CUtensorMap *m, tcm::Args a, int smem, int n
     int dev = 0;
     cudaGetDevice(&dev);
     int ncl = nsm / CG;
-    // programmatic dependent launch of the split launch(es) and the GEMM (EATSS_TCM_PDL=0: plain launches)
-    static const bool pdl = devsw("EATSS_TCM_PDL", 1) != 0;
+    // programmatic dependent launch of the split launch(es) and the GEMM (EATSS_TCM_PDL=0: plain launches);
+    // not when the GEMM is bracketed by timing events (exec.time_kernels): the event record between the
+    // launches would put the early-launched GEMM's wait inside its own timed window
+    static const bool pdl_env = devsw("EATSS_TCM_PDL", 1) != 0;
+    const bool pdl = pdl_env && ev == nullptr;
     cudaLaunchConfig_t cfg = {};
     cudaLaunchAttribute attr[2];
     attr[0].id = cudaLaunchAttributeClusterDimension;
