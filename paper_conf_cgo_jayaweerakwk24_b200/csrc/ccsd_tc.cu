@@ -45,6 +45,7 @@ namespace ccsdtc {
 using namespace tcm;
 
 constexpr int NGRP = 3;          // epilogue groups; group g owns the units u with u % NGRP == g
+constexpr int XSMAX = 8;         // t3 tile slices per unit (barriers per group)
 constexpr int NEPI = 4 * NGRP;   // epilogue warps (a group = one warp per TMEM lane quarter)
 constexpr int NTHREADS = (4 + NEPI) * 32;
 constexpr int MROWS = 128;  // UMMA M
@@ -67,8 +68,9 @@ struct Args {
     int x_bytes;      // t3 tile of a unit: Th2*Th1*Tp6*Tp5*Tp4*4
     int x_stage;      // x_bytes rounded up to 1 KB
     int XB;           // t3 tile buffers per epilogue group (2: the next owned unit is prefetched)
-    int XS;           // XB = 1 with Th2 = 2: the tile moves as two h2 slices (one TMA box and barrier each), so
+    int XS;           // XB = 1: the tile moves as XS slices (one TMA box and barrier each; 0 = whole tiles), so
                       // the next owned unit's slice s is requested as soon as slice s has been processed
+    int sph, p6s;     // slices per h2 plane and p6 columns per slice (XS = Th2 * sph, p6s = Tp6 / sph)
     int order;        // 1: A tiles round-robin over CTAs (concurrent CTAs sweep whole t3 blocks)
     int dbg;          // development only (EATSS_CCSD_TC_DBG): 1 no MMA, 2 no t3 traffic, 4 no v2 loads
     unsigned long long *prof;  // development only (EATSS_CCSD_TC_PROF): cycles per wait site
@@ -233,8 +235,8 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     // layout: V ring [SV] {hi [nkb], lo [nkb]}, t3 tiles [NGRP][XB], barriers
     unsigned char *vring = smem;
     unsigned char *xring = vring + (size_t)p.SV * p.v_stage;
-    uint64_t *xbar = reinterpret_cast<uint64_t *>(xring + (size_t)NGRP * p.XB * p.x_stage);  // [NGRP][2]
-    uint64_t *vfull = xbar + 2 * NGRP;
+    uint64_t *xbar = reinterpret_cast<uint64_t *>(xring + (size_t)NGRP * p.XB * p.x_stage);  // [NGRP][XSMAX]
+    uint64_t *vfull = xbar + XSMAX * NGRP;
     uint64_t *vempty = vfull + p.SV;
     uint64_t *dfull = vempty + p.SV;
     uint64_t *dempty = dfull + 4;
@@ -252,7 +254,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             mbar_init(dfull + b, 1);
             mbar_init(dempty + b, 4);
         }
-        for (int b = 0; b < 2 * NGRP; b++) mbar_init(xbar + b, 1);
+        for (int b = 0; b < XSMAX * NGRP; b++) mbar_init(xbar + b, 1);
         mbar_init(afull, 4);  // the owning epilogue group writes A into TMEM
         mbar_init(aempty, 1);
         asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
@@ -338,32 +340,36 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         const int xstep = p.Tp5 * p.Tp4;                                 // smem column (p6) stride
         const int xrow0 = h1l * p.Tp6 * xstep + p5l * p.Tp4 + p4l;       // smem offset of row m
         const int xh2 = p.Th1 * p.Tp6 * xstep;                           // smem stride of h2l
+        const int xslice = p.Th1 * p.p6s * xstep;                        // smem floats per slice
+        const int xrow0s = h1l * p.p6s * xstep + p5l * p.Tp4 + p4l;      // row m inside a slice
         unsigned char *xbuf = xring + (size_t)g * p.XB * p.x_stage;
-        uint64_t *xb = xbar + 2 * g;
+        uint64_t *xb = xbar + XSMAX * g;
         const bool leader = q == 0 && lane == 0;
         const uint64_t pol = policy_evict_first();  // t3 is touched once: keep v2 / t2 in L2
         auto fetch = [&](const UnitIter &wn, int buf) {  // t3 tile of unit wn -> xbuf[buf]
             int h1_0, p5_0, p4_0, c[5];
             a_coords(p, wn.a, h1_0, p5_0, p4_0);
             x_coords(p, wn.hh, wn.p6t, h1_0, p5_0, p4_0, c);
-            if (p.XS) {  // two h2 slices, barriers xb[0], xb[1]
-                const int sb = p.x_bytes / 2;
-                for (int q = 0; q < 2; q++) {
+            if (p.XS) {  // XS slices (h2 plane q / sph, p6 part q % sph), barriers xb[0 .. XS-1]
+                const int sb = p.x_bytes / p.XS;
+                for (int q = 0; q < p.XS; q++) {
                     mbar_expect_tx(xb + q, sb);
-                    tma_5d_hint(xbuf + (size_t)q * sb, &mX, c[0], c[1], c[2], c[3] + q, c[4], xb + q, pol);
+                    tma_5d_hint(xbuf + (size_t)q * sb, &mX, c[0], c[1] + (q % p.sph) * p.p6s, c[2], c[3] + q / p.sph,
+                                c[4], xb + q, pol);
                 }
                 return;
             }
             mbar_expect_tx(xb + buf, p.x_bytes);
             tma_5d_hint(xbuf + (size_t)buf * p.x_stage, &mX, c[0], c[1], c[2], c[3], c[4], xb + buf, pol);
         };
-        auto fetch_slice = [&](const UnitIter &wn, int q) {  // h2 slice q of unit wn -> its half of xbuf
+        auto fetch_slice = [&](const UnitIter &wn, int q) {  // slice q of unit wn -> its part of xbuf
             int h1_0, p5_0, p4_0, c[5];
             a_coords(p, wn.a, h1_0, p5_0, p4_0);
             x_coords(p, wn.hh, wn.p6t, h1_0, p5_0, p4_0, c);
-            const int sb = p.x_bytes / 2;
+            const int sb = p.x_bytes / p.XS;
             mbar_expect_tx(xb + q, sb);
-            tma_5d_hint(xbuf + (size_t)q * sb, &mX, c[0], c[1], c[2], c[3] + q, c[4], xb + q, pol);
+            tma_5d_hint(xbuf + (size_t)q * sb, &mX, c[0], c[1] + (q % p.sph) * p.p6s, c[2], c[3] + q / p.sph, c[4],
+                        xb + q, pol);
         };
         UnitIter w = iter_begin(p, sc), wn = w;  // wn: this group's next unit to prefetch
         for (int i = 0; i < g && i < sc.n; i++) iter_next(p, sc, wn);
@@ -434,6 +440,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             const int p6b = w.p6t * p.Tp6, np6 = min(p.Tp6, p.P6 - p6b);
             float *const rowp = t3 + rowoff + (int64_t)hhb * s_hh + (int64_t)p6b * sp6;
             const float *xs = reinterpret_cast<const float *>(xbuf + (size_t)buf * p.x_stage) + xrow0;
+            const float *xsl = reinterpret_cast<const float *>(xbuf) + xrow0s;  // slices (XB = 1)
             const bool io = rin && !(p.dbg & 2);
             if (!(p.dbg & 2) && !p.XS) TWAIT(7, xb + buf, xph);
             if (p.prof && leader) atomicAdd(p.prof + 5, 1ull);
@@ -442,19 +449,20 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             fence_after();
             // chunks of 16 columns (Tp6 % 16 == 0: never two h2 in a chunk), walked without divisions
             constexpr int CH = 16;
-            int h2l = 0, c6 = 0;
+            int h2l = 0, c6 = 0, q = 0, cq = 0;  // q: slice of this chunk, cq: column within the slice
             for (int c0 = 0; c0 < p.NV; c0 += CH) {
-                if (p.XS && c6 == 0) {  // a new h2 slice: its t3 rows have landed (slice h2l, phase of unit k)
-                    if (h2l == 1) {  // slice 0 fully read by the group: request the next owned unit's slice 0
+                if (p.XS && cq == 0) {  // a new slice: its t3 rows have landed (slice q, phase of unit k)
+                    if (q >= 1) {  // slice q-1 fully read by the group: request the next owned unit's slice q-1
                         named_bar(1 + g, 128);
-                        if (leader && !(p.dbg & 2) && un < sc.n) fetch_slice(wn, 0);
+                        if (leader && !(p.dbg & 2) && un < sc.n) fetch_slice(wn, q - 1);
                     }
-                    if (!(p.dbg & 2)) TWAIT(7, xb + h2l, (unsigned)(k & 1));
+                    if (!(p.dbg & 2)) TWAIT(7, xb + q, (unsigned)(k & 1));
                 }
                 uint32_t v[CH];
                 tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0), *reinterpret_cast<uint32_t(*)[8]>(v));
                 tmem_ld8(trow + (uint32_t)(rd.s * p.bstride + c0 + 8), *reinterpret_cast<uint32_t(*)[8]>(v + 8));
-                const float *xc = xs + h2l * xh2 + c6 * xstep;
+                // slice layout [q][h1l][p6 within the slice][(p5, p4)]; without slices q = h2l, p6s = Tp6
+                const float *xc = p.XS ? xsl + q * xslice + cq * xstep : xs + h2l * xh2 + c6 * xstep;
                 float x[CH];  // rows m >= Th1*Tp5*Tp4 lie outside the tile (and possibly the window)
 #pragma unroll
                 for (int c = 0; c < CH; c++) x[c] = live ? xc[c * xstep] : 0.f;
@@ -471,10 +479,12 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                 }
                 c6 += CH;
                 if (c6 == p.Tp6) { c6 = 0; h2l++; }
+                cq += CH;
+                if (cq == p.p6s) { cq = 0; q++; }
             }
-            if (p.XS) {  // slice 1 read: request the next owned unit's slice 1
+            if (p.XS) {  // the last slice read: request the next owned unit's last slice
                 named_bar(1 + g, 128);
-                if (leader && !(p.dbg & 2) && un < sc.n) fetch_slice(wn, 1);
+                if (leader && !(p.dbg & 2) && un < sc.n) fetch_slice(wn, p.XS - 1);
             }
             fence_before();
             __syncwarp();
@@ -567,8 +577,20 @@ CcsdTcPlan plan_ccsd_tc(const int64_t *dims, const int64_t *tiles) {
     static const int xb_env = getenv("EATSS_CCSD_TC_XB") ? atoi(getenv("EATSS_CCSD_TC_XB")) : 0;  // development
     if (xb_env > 0) a.XB = std::min(2, xb_env);
     a.SV = std::min(6, (budget - ccsdtc::NGRP * a.XB * a.x_stage) / a.v_stage);
-    static const int xs_env = getenv("EATSS_CCSD_TC_SLICES") ? atoi(getenv("EATSS_CCSD_TC_SLICES")) : 1;
-    a.XS = (a.XB == 1 && a.Th2 == 2 && xs_env != 0) ? 1 : 0;  // development: EATSS_CCSD_TC_SLICES=0 disables
+    // t3 slices (XB = 1, Th2 > 1 layout): one per h2 plane by default; finer (h2 plane, p6 part of >= 16 columns)
+    // slices measured slower at dims 48 (6 slices 24.2 ms, 2 slices 19.0-20.1 ms, none 22.0 ms:
+    // profiles/r02/experiments/gpu41_ccsd_slices.log); EATSS_CCSD_TC_SLICES = 0 / XS overrides (development)
+    static const int xs_env = getenv("EATSS_CCSD_TC_SLICES") ? atoi(getenv("EATSS_CCSD_TC_SLICES")) : -1;
+    a.XS = 0; a.sph = 1; a.p6s = a.Tp6;
+    if (a.XB == 1 && a.Th2 > 1 && xs_env != 0) {
+        for (int sph = xs_env > 0 ? a.Tp6 / 16 : 1; sph >= 1; sph--) {
+            const int xs = a.Th2 * sph;
+            if (a.Tp6 % sph || (a.Tp6 / sph) % 16 || xs > ccsdtc::XSMAX) continue;
+            if (xs_env > 0 && xs != xs_env) continue;
+            a.XS = xs; a.sph = sph; a.p6s = a.Tp6 / sph;
+            break;
+        }
+    }
     static const int sv_env = getenv("EATSS_CCSD_TC_VSTAGES") ? atoi(getenv("EATSS_CCSD_TC_VSTAGES")) : 0;
     if (sv_env > 0) a.SV = std::min(a.SV, sv_env);
     if (a.SV < 2) return pl;
@@ -620,8 +642,8 @@ cudaError_t launch_ccsd_tc(float *t3, const float *t2, const float *v2, const in
         const uint64_t d2[5] = {(uint64_t)(P5 * P4), (uint64_t)P6, (uint64_t)H1, (uint64_t)H2, (uint64_t)a.H3};
         const uint64_t s2[4] = {(uint64_t)(P5 * P4) * 4, (uint64_t)(P6 * P5 * P4) * 4, (uint64_t)(H1 * P6 * P5 * P4) * 4,
                                 (uint64_t)(H2 * H1 * P6 * P5 * P4) * 4};
-        const uint32_t b2[5] = {(uint32_t)(a.Tp5 * a.Tp4), (uint32_t)a.Tp6, (uint32_t)a.Th1,
-                                (uint32_t)(a.XS ? 1 : a.Th2), 1};  // XS: one h2 slice per box
+        const uint32_t b2[5] = {(uint32_t)(a.Tp5 * a.Tp4), (uint32_t)(a.XS ? a.p6s : a.Tp6), (uint32_t)a.Th1,
+                                (uint32_t)(a.XS ? 1 : a.Th2), 1};  // XS: one (h2, p6 part) slice per box
         for (int i = 0; i < 5; i++) { xdims[i] = d2[i]; xbox[i] = b2[i]; }
         for (int i = 0; i < 4; i++) xstr[i] = s2[i];
     }
