@@ -51,7 +51,14 @@ namespace eatss {
 namespace tcm {
 
 constexpr int BM = 128;      // rows of i per CTA (UMMA M per SM)
-constexpr int NEPI = 16;     // epilogue warps (4..19): four per TMEM lane quarter, a column quarter each
+#ifndef EATSS_TCM_NEPI
+#define EATSS_TCM_NEPI 12
+#endif
+// epilogue warps (4 .. 3+NEPI): NEPI/4 per TMEM lane quarter, each a contiguous column range of the tile.
+// 12 (16 warps in all, four per SM sub-partition) leaves 128 registers per thread for up to 88 fp32
+// accumulators; 16 (20 warps) caps every thread at 96 and spills accumulators around the drains.
+constexpr int NEPI = EATSS_TCM_NEPI;
+constexpr int NEPQ = NEPI / 4;   // epilogue warps per lane quarter
 constexpr int NTHREADS = (4 + NEPI) * 32;
 constexpr int MAXBN = 256;   // UMMA N limit
 constexpr int CHUNK_K = 128; // k per accumulator chunk (fp32 drain of the truncating accumulation), 3xTF32
@@ -290,8 +297,11 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         }
     } else if (warp >= 4) {  // ---------------------------------------- epilogue warps
         const int e = warp - 4, q = warp & 3, cq = e >> 2;  // TMEM lane quarter, column quarter
-        const int CW = p.BNT / 4;  // columns per epilogue warp (multiple of 4)
-        constexpr int MAXCW = MAXBN / 4;
+        // columns per epilogue warp: ceil(Tj / NEPQ) rounded up to 8 (16-byte fp32 runs), the last warp of a
+        // quarter takes the rest
+        const int CW0 = ((p.BNT + NEPQ - 1) / NEPQ + 7) / 8 * 8;
+        const int CW = max(0, min(CW0, p.BNT - cq * CW0));
+        constexpr int MAXCW = ((MAXBN + NEPQ - 1) / NEPQ + 7) / 8 * 8;
         const uint32_t demp0 = CG == 2 ? mapa(su32(dempty), 0) : su32(dempty);
         int gc = 0;
         for (int u = cid; u < p.nunits; u += ncl) {
@@ -306,7 +316,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
                 mbar_wait(dfull + bd, (unsigned)((gc >> 1) & 1));
                 const long long t1 = p.prof ? clock64() : 0;
                 fence_after();
-                const uint32_t ta = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(bd * 256 + cq * CW);
+                const uint32_t ta = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(bd * 256 + cq * CW0);
                 // drain: four 4-column loads in flight per wait
 #pragma unroll
                 for (int c0 = 0; c0 < MAXCW; c0 += 16) {
@@ -339,7 +349,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             const long long te = p.prof ? clock64() : 0;
             // C(i, j) for row i = i0 + 32q + lane, columns jb .. jb + CW - 1
             const int64_t i = (int64_t)(w.pi * CG + (int)rank) * BM + q * 32 + lane;
-            const int64_t jb = (int64_t)w.tj * p.BNT + cq * CW;
+            const int64_t jb = (int64_t)w.tj * p.BNT + cq * CW0;
             if constexpr (F16) {  // undo the power-of-two row / column scales: acc * 2^-(rexp_i + cexp_j), exact
                 if (i < p.M && jb < p.N) {
                     const float fr = __int_as_float((127 - p.rexp[i]) << 23);
