@@ -38,11 +38,13 @@ def parse():
     ap.add_argument("--repeats", type=int, default=5)
     ap.add_argument("--window", type=float, default=1.0)
     ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--engine", type=int, choices=[2, 4], default=2,
+                    help="2 = 3xTF32 (reading T mode 2), 4 = 3xFP16 (mode 3; Tk counts fp16 elements)")
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "tensor_sweep.jsonl"))
     return ap.parse_args()
 
 
-def exact_gemm(E, torch, tiles):
+def exact_gemm(E, torch, tiles, engine=2):
     """Small-integer gemm through the tensor engine: 512 sampled entries equal the fp64 oracle."""
     import synth
     from oracle import numeric as O
@@ -50,7 +52,7 @@ def exact_gemm(E, torch, tiles):
     n = N
     d = E.desc_builtin("gemm", (n, n, n))
     d.set_scalars(1.0, 1.0)
-    d.set_exec(split_pct=50, engine=2)
+    d.set_exec(split_pct=50, engine=engine)
     Ah, Bh, Ch = synth.small_int((n, n), 1), synth.small_int((n, n), 2), synth.small_int((n, n), 3)
     C = torch.from_numpy(Ch).cuda()
     E.run(d, tiles, [C, torch.from_numpy(Ah).cuda(), torch.from_numpy(Bh).cuda()])
@@ -73,15 +75,19 @@ def main():
         for kind in a.kinds.split(","):
             dims = KINDS[kind]
             d = E.desc_builtin(kind, dims)
-            d.set_exec(split_pct=50, engine=2)
-            pick, _ = E.select_tiles(d, gpu, split_pct=50, waf=16, mode=2)
-            space = [(ti, tj, tk) for ti in (128, 256) for tj in range(16, 257, 16) for tk in (8, 16, 32, 64)]
+            d.set_exec(split_pct=50, engine=a.engine)
+            mode = 2 if a.engine == 2 else 3
+            pick, _ = E.select_tiles(d, gpu, split_pct=50, waf=16, mode=mode)
+            tks = (8, 16, 32, 64) if a.engine == 2 else (16, 32, 64, 128)  # 32 .. 256 bytes of k per stage row
+            tk_t = 32 if a.engine == 2 else 64                               # reading T: whole 128-byte atoms
+            space = [(ti, tj, tk) for ti in (128, 256) for tj in range(16, 257, 16) for tk in tks]
             if kind != "gemm":
-                space = [v for v in space if v[2] >= 32]
-            variants = [v for v in space if E.launches_per_run(d, v) == 2]  # executable on tcgen05
+                space = [v for v in space if v[2] >= tk_t]
+            nl = 2 if a.engine == 2 else 3  # launches per nest on the engine: executable there
+            variants = [v for v in space if E.launches_per_run(d, v) == nl]
             gen = torch.Generator(device="cuda").manual_seed(0)
             bufs = [torch.rand(d.buffer_elems(i), device="cuda", generator=gen) * 2 - 1 for i in range(d.num_buffers)]
-            exact = {v: exact_gemm(E, torch, v) for v in variants} if kind == "gemm" else {}
+            exact = {v: exact_gemm(E, torch, v, a.engine) for v in variants} if kind == "gemm" else {}
             ppw = {v: [] for v in variants}
             tf = {v: [] for v in variants}
             watts = {v: [] for v in variants}
@@ -92,7 +98,7 @@ def main():
                     rec = dict(kind=kind, tiles=list(v), rep=rep, ms=m.ms_per_run, tflops=m.tflops,
                                watts=m.avg_watts, ppw=m.gflops_per_watt, joules=m.joules_per_run,
                                sm_mhz=m.sm_mhz_median, status=m.status, eatss_pick=tuple(v) == tuple(pick),
-                               reading_t=v[2] >= 32, exact=exact.get(v))
+                               reading_t=v[2] >= tk_t, exact=exact.get(v), engine=a.engine)
                     f.write(json.dumps(rec) + "\n"); f.flush()
                     if m.status == 0 and m.gflops_per_watt > 0:
                         ppw[v].append(m.gflops_per_watt); tf[v].append(m.tflops); watts[v].append(m.avg_watts)
@@ -106,7 +112,7 @@ def main():
                     if ppw[v]}
             perf = max(rows, key=lambda v: rows[v]["tflops"][0])
             eff = max(rows, key=lambda v: rows[v]["ppw"][0])
-            s = dict(eatss_pick=list(pick), n_variants=len(rows), perf_optimal=dict(tiles=list(perf), **rows[perf]),
+            s = dict(engine=a.engine, eatss_pick=list(pick), n_variants=len(rows), perf_optimal=dict(tiles=list(perf), **rows[perf]),
                      ppw_optimal=dict(tiles=list(eff), **rows[eff]),
                      distinct=perf != eff,
                      separated=perf != eff and rows[eff]["ppw"][1][0] > rows[perf]["ppw"][1][1],
