@@ -182,7 +182,9 @@ typedef struct {
     int32_t engine;     /* eatss_engine; AUTO = SIMT unless the tensor-core path applies; UNTILED: stencils */
     int32_t use_graph;  /* stencils: replay the time loop as one CUDA graph (default 1) */
     int32_t time_kernels; /* 1: record CUDA events around each nest's main compute kernel on the
-                             run's stream (read back with eatss_last_kernel_ms); default 0 */
+                             run's stream (read back with eatss_last_kernel_ms); default 0.  The tensor
+                             engines chain their split launch(es) and GEMM with programmatic dependent
+                             launch, except under time_kernels = 1 (the events bracket the GEMM alone) */
     int32_t warp_align; /* SIMT contraction executor: lanes of every warp laid contiguously along the
                            CMA loop l_s1 -- the "SIMT length as a fraction of the warp size" (P:25,
                            P:125): WAF in {4, 8, 16, 32}, the remaining 32/WAF lanes of the warp
