@@ -19,6 +19,7 @@
 #include <cstdlib>
 
 #include "contract.cuh"
+#include "devsw.hpp"
 
 #include "tc_ptx.cuh"
 
@@ -42,6 +43,32 @@ __device__ __forceinline__ void bulk_row_g2s(void *dst, const void *src, unsigne
         "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n" ::"r"(su32(dst)),
         "l"(src), "r"(bytes), "r"(su32(bar))
         : "memory");
+}
+
+// L2 residency hints for the jacobi-2d ping-pong at L2-sized grids (N = 4000: 2 x 64 MB against 126 MB of
+// L2): the source window is read evict-first (a line, once read, is the preferred victim) and the
+// destination is written evict-last, so the array the next sweep reads stays in L2 while the one just read
+// makes room.
+__device__ __forceinline__ uint64_t policy_evict_last() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;\n" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ void bulk_row_g2s_hint(void *dst, const void *src, unsigned bytes, uint64_t *bar,
+                                                  uint64_t pol) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;\n" ::"r"(
+            su32(dst)),
+        "l"(src), "r"(bytes), "r"(su32(bar)), "l"(pol)
+        : "memory");
+}
+__device__ __forceinline__ void st_hint_v4(float *p, float4 v, uint64_t pol) {
+    asm volatile("st.global.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;\n" ::"l"(p), "f"(v.x), "f"(v.y), "f"(v.z),
+                 "f"(v.w), "l"(pol)
+                 : "memory");
+}
+__device__ __forceinline__ void st_hint(float *p, float v, uint64_t pol) {
+    asm volatile("st.global.L2::cache_hint.f32 [%0], %1, %2;\n" ::"l"(p), "f"(v), "l"(pol) : "memory");
 }
 
 // Work items (a, b) of an A x B space, a = the 16-byte column group along the CMA loop l_s1.  waf = 0:
@@ -69,7 +96,7 @@ __device__ __forceinline__ bool waf_item(int v, int A, int B, int waf, int &a, i
 template <bool COVER>
 __global__ void __launch_bounds__(256) jacobi2d_staged(float *__restrict__ dst, const float *__restrict__ src,
                                                        const float *__restrict__ bsrc, int64_t n, int Ti, int Tj,
-                                                       int32_t *counts, int waf) {
+                                                       int32_t *counts, int waf, int l2hint) {
     extern __shared__ __align__(16) float win[];
     __shared__ uint64_t bar;
     const int64_t ti0 = (int64_t)blockIdx.y * Ti, tj0 = (int64_t)blockIdx.x * Tj;
@@ -100,7 +127,13 @@ __global__ void __launch_bounds__(256) jacobi2d_staged(float *__restrict__ dst, 
     if (tid < 32) {
         if (tid == 0) mbar_expect_tx(&bar, (unsigned)(nr * W * 4));
         __syncwarp();
-        for (int r = tid; r < nr; r += 32) bulk_row_g2s(win + r * W, src + (r0 + r) * n + cs, (unsigned)W * 4, &bar);
+        if (l2hint) {
+            const uint64_t pf = tcm::policy_evict_first();
+            for (int r = tid; r < nr; r += 32)
+                bulk_row_g2s_hint(win + r * W, src + (r0 + r) * n + cs, (unsigned)W * 4, &bar, pf);
+        } else {
+            for (int r = tid; r < nr; r += 32) bulk_row_g2s(win + r * W, src + (r0 + r) * n + cs, (unsigned)W * 4, &bar);
+        }
     }
     mbar_wait(&bar, 0);
     if (bsrc != src) {  // boundary cells of the window: from bsrc
@@ -118,6 +151,7 @@ __global__ void __launch_bounds__(256) jacobi2d_staged(float *__restrict__ dst, 
         }
     }
     const float c02 = 0.2f;
+    const uint64_t pl = l2hint ? policy_evict_last() : 0;
     const int rows = (int)(ihi - ilo);
     // items: (column group, row chunk); with a warp alignment the rows are cut into 32/WAF chunks
     const int ngr = (int)(g1 - g0), nch = waf > 0 ? 32 / waf : 1, per = (rows + nch - 1) / nch;
@@ -145,12 +179,16 @@ __global__ void __launch_bounds__(256) jacobi2d_staged(float *__restrict__ dst, 
             o.w = c02 * ((((c.w + c.z) + rr) + d.w) + u.w);
             float *out = dst + (r0 + r) * n + 4 * g;
             if (full) {
-                *reinterpret_cast<float4 *>(out) = o;
+                if (l2hint) st_hint_v4(out, o, pl);
+                else *reinterpret_cast<float4 *>(out) = o;
             } else {
                 const float ov[4] = {o.x, o.y, o.z, o.w};
 #pragma unroll
                 for (int q = 0; q < 4; q++)
-                    if (4 * g + q >= jlo && 4 * g + q < jhi) out[q] = ov[q];
+                    if (4 * g + q >= jlo && 4 * g + q < jhi) {
+                        if (l2hint) st_hint(out + q, ov[q], pl);
+                        else out[q] = ov[q];
+                    }
             }
             u = c;
             c = d;
@@ -339,12 +377,20 @@ cudaError_t launch_jacobi2d_staged(float *dst, const float *src, const float *bs
     const int smem = counts ? 0 : jacobi_staged_smem(n, Ti, Tj);
     dim3 grid((unsigned)gx, (unsigned)gy), block(256);
     if (counts) {
-        jacobi2d_staged<true><<<grid, block, 0, s>>>(dst, src, bsrc, n, (int)Ti, (int)Tj, counts, waf);
+        jacobi2d_staged<true><<<grid, block, 0, s>>>(dst, src, bsrc, n, (int)Ti, (int)Tj, counts, waf, 0);
         return cudaGetLastError();
     }
+    // L2 hints when the two arrays are about L2-sized (between half and twice the L2): smaller grids stay
+    // resident anyway, larger ones stream from HBM whatever the hints
+    int dev = 0, l2 = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev);
+    static const int hint_env = devsw("EATSS_JACOBI_L2HINT", 1);  // development A/B
+    const double both = 2.0 * (double)n * (double)n * 4.0;
+    const int l2hint = (hint_env && l2 > 0 && both >= 0.5 * l2 && both <= 2.0 * l2) ? 1 : 0;
     cudaFuncSetAttribute(jacobi2d_staged<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     return launch_pdl(jacobi2d_staged<false>, grid, block, smem, staged_carveout(smem, split_pct), s, dst, src, bsrc,
-                      n, (int)Ti, (int)Tj, (int32_t *)nullptr, waf);
+                      n, (int)Ti, (int)Tj, (int32_t *)nullptr, waf, l2hint);
 }
 
 cudaError_t launch_heat3d_staged(float *dst, const float *src, int64_t n, int64_t Ti, int64_t Tj, int64_t Tk,
