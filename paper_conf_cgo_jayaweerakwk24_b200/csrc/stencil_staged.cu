@@ -49,11 +49,7 @@ __device__ __forceinline__ void bulk_row_g2s(void *dst, const void *src, unsigne
 // L2): the source window is read evict-first (a line, once read, is the preferred victim) and the
 // destination is written evict-last, so the array the next sweep reads stays in L2 while the one just read
 // makes room.
-__device__ __forceinline__ uint64_t policy_evict_last() {
-    uint64_t pol;
-    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;\n" : "=l"(pol));
-    return pol;
-}
+using tcm::policy_evict_last;
 __device__ __forceinline__ void bulk_row_g2s_hint(void *dst, const void *src, unsigned bytes, uint64_t *bar,
                                                   uint64_t pol) {
     asm volatile(
