@@ -50,3 +50,16 @@ t = timed(two_streams)
 print(f"H2D two streams: {t:.3f} ms = {192e6 / t / 1e6:.1f} GB/s")
 t = timed(lambda: ho.copy_(do, non_blocking=True))
 print(f"D2H 64 MB: {t:.3f} ms = {64e6 / t / 1e6:.1f} GB/s")
+
+
+def both():
+    with torch.cuda.stream(s1):
+        d.copy_(h, non_blocking=True)
+    with torch.cuda.stream(s2):
+        ho.copy_(do, non_blocking=True)
+    torch.cuda.current_stream().wait_stream(s1)
+    torch.cuda.current_stream().wait_stream(s2)
+
+
+t = timed(both)
+print(f"H2D 192 MB + concurrent D2H 64 MB: {t:.3f} ms (H2D alone 3.46 ms at 55.5 GB/s)")
